@@ -1,0 +1,201 @@
+/*
+ * bf.h -- C ABI of the B200-native BlackForest random-forest hot path.
+ *
+ * The method (PAPER.md = /root/reference/PAPER.md, "P:n" = line n):
+ *   learning set (X, Y): N observations x p predictors, numeric response   P:71  (sec 4.1.1)
+ *   regression tree = recursive binary partition, leaf = region mean       P:73-79, eq.(1)
+ *   split on half-planes x_j <= s minimising RSS_L + RSS_R                 P:81-91, eqs.(2),(3)
+ *   grow until a minimum node size (e.g. 5), no pruning in a forest
+ *   forest: n_t bootstrap samples, random predictor subset per node,
+ *           prediction = average of the trees
+ *   permutation importance on OOB samples, tree by tree
+ *   OOB error / variance explained
+ *   PCA of the counters (prcomp)
+ * The exact arithmetic, RNG streams and readings of silent passages are
+ * DESIGN.md sections 2 (S1..S9) and 3 (R1..R20).
+ *
+ * Conventions
+ *   - Matrices are COLUMN-MAJOR: element (i, j) at X[j*ld + i], ld >= rows.
+ *   - Pointers may be CUDA device pointers or host pointers (pageable or
+ *     pinned); the library detects host pointers with
+ *     cudaPointerGetAttributes and stages them through device memory on the
+ *     given stream (host<->device copies are then part of the call).
+ *   - The caller owns every input and output buffer; the library never frees
+ *     them.  The library owns bf_forest and its device memory (allocated with
+ *     cudaMallocAsync on the call's stream, or through bf_set_allocator).
+ *   - Return value: BF_OK (0) or a negative BF_E* code; no exception crosses
+ *     the ABI; on error outputs are unspecified and no forest is returned.
+ *     bf_last_error() returns a thread-local message for the last failure.
+ *   - bf_fit is synchronous (node counts are needed on the host).  Every other
+ *     call enqueues on `stream` (a cudaStream_t, NULL = legacy default stream)
+ *     and returns; results are valid after the stream is synchronised.  Calls
+ *     that were given HOST output pointers synchronise before returning.
+ */
+#ifndef BF_H
+#define BF_H
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define BF_ABI_VERSION 1
+
+enum {
+  BF_OK = 0,
+  BF_EINVAL = -1,      /* bad shape, ld < rows, mtry not in [1,p], nodesize < 1, ntree < 1, bad tree range */
+  BF_ENONFINITE = -2,  /* NaN/Inf in X or y (reading R17)                                                 */
+  BF_ERANGE = -3,      /* n >= 2^31 or sampsize >= 2^31, or |y| range not representable                   */
+  BF_ENOMEM = -4,      /* device allocation failed                                                        */
+  BF_ECUDA = -5,       /* CUDA runtime error (message in bf_last_error)                                   */
+  BF_ENOTIMPL = -6     /* e.g. replace = 0 with sampsize != n (reading R20)                               */
+};
+
+/* Forest parameters.  Defaults in brackets are the R randomForest regression
+ * defaults the paper used (readings R3, R6).                          */
+typedef struct bf_params {
+  int32_t ntree;           /* T, total forest size [500]; global tree ids 0..T-1               */
+  int32_t mtry;            /* predictors drawn per node; 0 -> max(floor(p/3), 1)               */
+  int32_t nodesize;        /* a node with n_k <= nodesize is a leaf [5]                        */
+  int32_t replace;         /* 1 bootstrap with replacement [1]; 0 every row once (sampsize==n) */
+  int64_t sampsize;        /* N_s; 0 -> n                                                      */
+  uint64_t seed;           /* Philox key (S1)                                                  */
+  int32_t tree_begin;      /* this call grows global trees [tree_begin, tree_end)              */
+  int32_t tree_end;        /*   (multi-GPU: each rank a disjoint range; 0,0 -> [0, ntree))     */
+  int32_t trees_in_flight; /* trees grown concurrently; 0 -> auto from free device memory      */
+  int32_t small_node_max;  /* largest node (distinct rows) grown by one CTA in shared memory;
+                              0 -> auto from the shared-memory budget and p                    */
+} bf_params;
+
+typedef struct bf_forest bf_forest; /* opaque, library-owned, device-resident */
+
+/* Summary of a forest (host struct filled by bf_forest_info). */
+typedef struct bf_forest_info {
+  int64_t n;              /* training rows                                */
+  int32_t p;              /* predictors                                   */
+  int32_t ntree_total;    /* T of the whole forest                        */
+  int32_t tree_begin;     /* global id of the first tree held             */
+  int32_t tree_end;       /* one past the last                            */
+  int64_t total_nodes;    /* nodes over the held trees                    */
+  int32_t q;              /* fixed-point exponent of S2                   */
+  int32_t mtry, nodesize, replace;
+  int64_t sampsize;
+  uint64_t seed;
+} bf_forest_info;
+
+/* Flat view of a forest, used by export (host arrays written by the library)
+ * and import (host or device arrays read by the library).  Nodes of local
+ * tree i are [tree_off[i], tree_off[i+1]); node ids inside a tree are local
+ * (root = 0; right child = left + 1).  feature = -1 marks a leaf.
+ * thr_or_value = threshold for internal nodes, leaf value for leaves.       */
+typedef struct bf_forest_view {
+  bf_forest_info info;
+  int64_t* tree_off;      /* ntrees + 1                                   */
+  int32_t* feature;       /* total_nodes                                  */
+  int32_t* left;          /* total_nodes                                  */
+  double* thr_or_value;   /* total_nodes                                  */
+  int32_t* count;         /* total_nodes: n_k (bootstrap duplicates counted) */
+  double* value;          /* total_nodes: node mean (every node, eq.(1))  */
+  double* drss;           /* total_nodes: RSS decrease of the split (S4.6), 0 for leaves */
+} bf_forest_view;
+
+/* OOB / importance accumulators for the trees of ONE forest object
+ * (device pointers, caller-allocated; T_loc = tree_end - tree_begin).
+ * Slots are per LOCAL tree so that ranks holding disjoint tree ranges can be
+ * merged exactly by placing them at their global offsets (sum of disjoint
+ * slots = all-gather).  bf_oob_importance overwrites all of them.           */
+typedef struct bf_oob_accum {
+  double* d_slots;        /* T_loc * p : d_tm (S7), row-major [tree][m]    */
+  double* npur_slots;     /* T_loc * p : sum of drss of splits on m (S8)   */
+  double* oob_sum;        /* n : sum of OOB tree predictions of row i (S6) */
+  int32_t* oob_cnt;       /* n : number of OOB trees of row i              */
+  double* e_t;            /* T_loc : OOB squared error of tree t           */
+  int64_t* nout_t;        /* T_loc : OOB rows of tree t                    */
+} bf_oob_accum;
+
+/* ---------------------------------------------------------------------- */
+const char* bf_version(void);
+const char* bf_last_error(void);
+
+/* Optional allocator hook (e.g. the torch caching allocator).  NULL restores
+ * cudaMallocAsync / cudaFreeAsync.                                          */
+typedef void* (*bf_alloc_fn)(size_t bytes, void* stream, void* ctx);
+typedef void (*bf_free_fn)(void* ptr, void* stream, void* ctx);
+int bf_set_allocator(bf_alloc_fn alloc, bf_free_fn free_, void* ctx);
+
+/* Grow global trees [tree_begin, tree_end) of a T-tree forest (P:95 steps 1-2;
+ * S2-S4).  X: n x p column-major (ldx >= n), y: n.  Synchronous.  *out
+ * receives a new forest owned by the caller (free with bf_forest_free).     */
+int bf_fit(const double* X, int64_t ldx, const double* y, int64_t n, int32_t p,
+           const bf_params* prm, void* stream, bf_forest** out);
+
+void bf_forest_free(bf_forest* f);
+int bf_forest_info_get(const bf_forest* f, bf_forest_info* info);
+/* Export to HOST arrays sized from bf_forest_info (tree_off: ntrees + 1).  */
+int bf_forest_export(const bf_forest* f, bf_forest_view* v);
+/* Build a forest from a view (host or device arrays; used after the
+ * multi-GPU gather).  info.tree_begin/tree_end give the held range.        */
+int bf_forest_import(const bf_forest_view* v, void* stream, bf_forest** out);
+
+/* Batched prediction (P:95 step 3; S5).  Xq: m x p column-major (ldq >= m).
+ * yhat_sum[i] = sum over the forest's trees of the leaf value (may be NULL);
+ * yhat[i] = yhat_sum[i] / ntree_total (may be NULL; ntree_total <= 0 ->
+ * number of held trees).                                                   */
+int bf_predict(const bf_forest* f, const double* Xq, int64_t ldq, int64_t m,
+               double* yhat_sum, double* yhat, int32_t ntree_total, void* stream);
+
+/* OOB prediction + permutation importance over the forest's trees (P:130,
+ * P:157; S6-S8).  X, y must be the training data of bf_fit.               */
+int bf_oob_importance(const bf_forest* f, const double* X, int64_t ldx, const double* y,
+                      int64_t n, int32_t p, const bf_oob_accum* acc, void* stream);
+
+/* Aggregate accumulators of ALL ntree trees (slots in global tree order,
+ * e.g. after an all-reduce of disjoint slots; S6-S8).  Outputs p-vectors and
+ * two scalars (device or host pointers).                                   */
+int bf_importance_finalize(const double* d_slots, const double* npur_slots, const double* oob_sum,
+                           const int32_t* oob_cnt, const double* y, int64_t n, int32_t p, int32_t ntree,
+                           double* inc_mse, double* inc_mse_raw, double* inc_mse_sd,
+                           double* inc_node_purity, double* oob_mse, double* rsq, void* stream);
+
+/* PCA of the counters (S9).  X: n x p column-major.  scale != 0
+ * standardises columns (zero-variance column -> BF_EINVAL).  Outputs: sdev
+ * (p), rotation (p x p column-major, column j = component j), center (p,
+ * may be NULL), scores (n x k column-major, may be NULL).                  */
+int bf_pca(const double* X, int64_t ldx, int64_t n, int32_t p, int32_t scale, int32_t k,
+           double* sdev, double* rotation, double* center, double* scores, void* stream);
+
+/* ---- single-step entry points (parity tests) ---- */
+/* Philox4x32-10 on `count` counters (S1): ctr[4*i..], out[4*i..].          */
+int bf_philox(const uint32_t* ctr, uint32_t key0, uint32_t key1, uint32_t* out, int64_t count, void* stream);
+/* Correctly rounded int128 -> double of (hi[i], lo[i]) (the key of S4.3). */
+int bf_i128_to_double(const int64_t* hi, const uint64_t* lo, double* out, int64_t count, void* stream);
+/* S2 fixed point: yq (n int64), *q (host int32).  Synchronous.             */
+int bf_fixed_point(const double* y, int64_t n, int64_t sampsize, int64_t* yq, int32_t* q, void* stream);
+/* S3 BOOT multiplicities of global trees [t0, t0+ntrees): w[(t-t0)*n + i]. */
+int bf_bootstrap(uint64_t seed, int32_t t0, int32_t ntrees, int64_t n, int64_t sampsize, int32_t replace,
+                 int32_t* w, void* stream);
+/* S7 Feistel pi_tm(a) for a = 0..n_o-1 into out[n_o].                      */
+int bf_perm(uint64_t seed, int32_t t, int32_t m, int64_t n_o, int64_t* out, void* stream);
+
+/* ---- measurement hooks (bench.py) ---------------------------------------
+ * When enabled, the library records a CUDA event pair on the launching stream
+ * around every kernel launch it makes, grouped by kernel class, together with
+ * the launch's ALGORITHMIC bytes.  bf_profile_read
+ * synchronises those events, returns the accumulated totals and resets them.
+ * bf_launch_count counts every kernel launch the library has made (CUB
+ * primitives count once per call), whether or not profiling is enabled.    */
+typedef struct bf_kernel_stat {
+  char name[40];
+  double ms;         /* summed device time between the event pairs          */
+  int64_t launches;  /* launches of this class                              */
+  double bytes;      /* summed algorithmic bytes                            */
+} bf_kernel_stat;
+int bf_profile_enable(int on);
+int bf_profile_read(bf_kernel_stat* stats, int cap, int* count);
+int64_t bf_launch_count(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* BF_H */

@@ -1,0 +1,242 @@
+// bf_internal.cuh -- internal declarations of the B200 BlackForest library.
+//
+// Device primitives (Philox4x32-10, 64-bit mulhi, correctly rounded int128 ->
+// double, the exact split key) are written here from DESIGN.md S1-S4; nothing
+// is shared with oracle/ (the CPU oracle is independent test infrastructure).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "../../include/bf.h"
+
+namespace bf {
+
+// ------------------------------------------------------------------ errors
+struct Error {
+  int code;
+  std::string msg;
+};
+void set_error(const std::string& m);
+#define BF_CUDA_CHECK(expr)                                                                   \
+  do {                                                                                        \
+    cudaError_t e_ = (expr);                                                                  \
+    if (e_ != cudaSuccess)                                                                    \
+      throw ::bf::Error{BF_ECUDA, std::string(#expr " -> ") + cudaGetErrorString(e_) + " @" + \
+                                      __FILE__ + ":" + std::to_string(__LINE__)};             \
+  } while (0)
+#define BF_REQUIRE(cond, code, m) \
+  do {                            \
+    if (!(cond)) throw ::bf::Error{(code), (m)}; \
+  } while (0)
+
+// ------------------------------------------------------------------ memory
+void* dev_alloc(size_t bytes, cudaStream_t s);
+void dev_free(void* p, cudaStream_t s);
+
+template <class T>
+struct DBuf {  // stream-ordered device buffer (RAII)
+  T* p = nullptr;
+  size_t n = 0;
+  cudaStream_t s = nullptr;
+  DBuf() = default;
+  DBuf(size_t count, cudaStream_t st) { alloc(count, st); }
+  void alloc(size_t count, cudaStream_t st) {
+    release();
+    s = st;
+    n = count;
+    if (count) p = static_cast<T*>(dev_alloc(count * sizeof(T), st));
+  }
+  void release() {
+    if (p) dev_free(p, s);
+    p = nullptr;
+    n = 0;
+  }
+  ~DBuf() { release(); }
+  DBuf(const DBuf&) = delete;
+  DBuf& operator=(const DBuf&) = delete;
+  DBuf(DBuf&& o) noexcept : p(o.p), n(o.n), s(o.s) { o.p = nullptr; o.n = 0; }
+  DBuf& operator=(DBuf&& o) noexcept {
+    if (this != &o) { release(); p = o.p; n = o.n; s = o.s; o.p = nullptr; o.n = 0; }
+    return *this;
+  }
+  size_t bytes() const { return n * sizeof(T); }
+};
+
+// Host/device pointer staging: a host input is copied to a temporary device
+// buffer on the stream; a host output is copied back at finish().
+bool is_device_ptr(const void* p);
+
+struct InStage {
+  const void* dptr = nullptr;
+  DBuf<char> tmp;
+  InStage(const void* ptr, size_t bytes, cudaStream_t s);
+};
+struct OutStage {
+  void* dptr = nullptr;
+  void* host = nullptr;
+  size_t bytes = 0;
+  DBuf<char> tmp;
+  OutStage(void* ptr, size_t bytes, cudaStream_t s);
+  void finish(cudaStream_t s);  // D2H if host (caller synchronises)
+};
+
+// ------------------------------------------------------------------ measurement
+// Scope around ONE logical launch (a kernel, or a CUB call): counts it and,
+// when profiling is enabled, brackets it with a CUDA event pair.
+struct KScope {
+  KScope(const char* name, cudaStream_t s, double bytes, int launches = 1);
+  ~KScope();
+  KScope(const KScope&) = delete;
+  KScope& operator=(const KScope&) = delete;
+  cudaStream_t s;
+  bool active = false;
+  const char* name = nullptr;
+  double bytes = 0;
+  int launches = 0;
+  cudaEvent_t a = nullptr, b = nullptr;
+};
+
+// Adds algorithmic bytes to a kernel class after the fact (sizes known only
+// after a device->host summary read).
+void prof_add_bytes(const char* name, double bytes);
+bool prof_enabled();
+
+// ------------------------------------------------------------------ device primitives
+// S1: Philox4x32-10.
+__host__ __device__ __forceinline__ void philox4x32_10(uint32_t c0, uint32_t c1, uint32_t c2, uint32_t c3,
+                                                       uint32_t k0, uint32_t k1, uint32_t out[4]) {
+#pragma unroll
+  for (int r = 0; r < 10; ++r) {
+#ifdef __CUDA_ARCH__
+    const uint32_t hi0 = __umulhi(0xD2511F53u, c0), lo0 = 0xD2511F53u * c0;
+    const uint32_t hi1 = __umulhi(0xCD9E8D57u, c2), lo1 = 0xCD9E8D57u * c2;
+#else
+    const uint64_t p0 = (uint64_t)0xD2511F53u * c0, p1 = (uint64_t)0xCD9E8D57u * c2;
+    const uint32_t hi0 = (uint32_t)(p0 >> 32), lo0 = (uint32_t)p0;
+    const uint32_t hi1 = (uint32_t)(p1 >> 32), lo1 = (uint32_t)p1;
+#endif
+    const uint32_t n0 = hi1 ^ c1 ^ k0, n2 = hi0 ^ c3 ^ k1;
+    c0 = n0;
+    c1 = lo1;
+    c2 = n2;
+    c3 = lo0;
+    k0 += 0x9E3779B9u;
+    k1 += 0xBB67AE85u;
+  }
+  out[0] = c0;
+  out[1] = c1;
+  out[2] = c2;
+  out[3] = c3;
+}
+
+__device__ __forceinline__ void philox_u64x2(uint64_t seed, uint32_t c0, uint32_t c1, uint32_t c2, uint32_t c3,
+                                             uint64_t& u0, uint64_t& u1) {
+  uint32_t x[4];
+  philox4x32_10(c0, c1, c2, c3, (uint32_t)seed, (uint32_t)(seed >> 32), x);
+  u0 = (uint64_t)x[0] | ((uint64_t)x[1] << 32);
+  u1 = (uint64_t)x[2] | ((uint64_t)x[3] << 32);
+}
+
+__device__ __forceinline__ uint64_t mulhi64(uint64_t u, uint64_t r) { return __umul64hi(u, r); }
+
+// S3 KEY stream: child key of node key K.
+__device__ __forceinline__ uint64_t child_key(uint64_t seed, uint32_t t, uint64_t K, uint32_t side) {
+  uint64_t u0, u1;
+  philox_u64x2(seed, (uint32_t)K, (uint32_t)(K >> 32), t, 0x40000000u | side, u0, u1);
+  return u0;
+}
+
+// Correctly rounded (nearest-even) conversion of a signed 128-bit integer.
+// The top 64 significant bits are converted by __ull2double_rn with the
+// remaining bits folded into the LSB as a sticky bit (the LSB lies below the
+// rounding position because the top word has its MSB set), then scaled by an
+// exact power of two.
+__device__ __forceinline__ double i128_to_double(__int128 v) {
+  const bool neg = v < 0;
+  unsigned __int128 u = neg ? (unsigned __int128)(-(v + 1)) + 1u : (unsigned __int128)v;
+  const uint64_t hi = (uint64_t)(u >> 64), lo = (uint64_t)u;
+  double d;
+  if (hi == 0) {
+    d = __ull2double_rn(lo);
+  } else {
+    const int lz = __clzll(hi);
+    const uint64_t m = lz ? ((hi << lz) | (lo >> (64 - lz))) : hi;
+    const uint64_t rest = lo << lz;  // lz < 64
+    d = __ull2double_rn(m | (rest != 0 ? 1ull : 0ull));
+    const double scale = __longlong_as_double((long long)(1023 + 64 - lz) << 52);  // 2^(64-lz)
+    d = __dmul_rn(d, scale);
+  }
+  return neg ? -d : d;
+}
+
+// S4.3 exact split key: g = RN(RN(RN(D)^2) / RN(n_l*n_r)), D = n_k*S_l - n_l*S_k.
+__device__ __forceinline__ double split_key(int64_t nk, int64_t Sk, int64_t nl, int64_t Sl) {
+  const __int128 D = (__int128)nk * (__int128)Sl - (__int128)nl * (__int128)Sk;
+  const double d = i128_to_double(D);
+  const double nn = __ll2double_rn(nl * (nk - nl));
+  return __ddiv_rn(__dmul_rn(d, d), nn);
+}
+
+__device__ __forceinline__ double canon(double x) { return __dadd_rn(x, 0.0); }  // -0 -> +0 (R18)
+
+// S4.6 threshold inside the gap [a, b).
+__device__ __forceinline__ double split_threshold(double a, double b) {
+  double t = __dadd_rn(__dmul_rn(0.5, a), __dmul_rn(0.5, b));
+  if (!(t < b)) t = a;
+  if (t < a) t = a;
+  return t;
+}
+
+// ------------------------------------------------------------------ forest
+struct Node16 {  // packed node for traversal: 16 B, one sector-aligned load
+  double v;       // threshold (internal) or leaf value
+  int32_t feature;  // -1 leaf
+  int32_t left;     // local id of the left child; right = left + 1
+};
+static_assert(sizeof(Node16) == 16, "Node16 must be 16 bytes");
+
+}  // namespace bf
+
+struct bf_forest {
+  bf_forest_info info;
+  std::vector<int64_t> tree_off;  // host copy, ntrees + 1
+  int64_t* d_tree_off = nullptr;
+  bf::Node16* d_nodes = nullptr;
+  int32_t* d_count = nullptr;
+  double* d_value = nullptr;
+  double* d_drss = nullptr;
+  int device = 0;
+};
+
+namespace bf {
+void forest_alloc(bf_forest* f, int64_t total_nodes, int32_t ntrees, cudaStream_t s);
+void forest_release(bf_forest* f);
+
+// fit.cu
+void fit_impl(const double* X, int64_t ldx, const double* y, int64_t n, int32_t p, const bf_params& prm,
+              cudaStream_t s, bf_forest** out);
+void fixed_point_impl(const double* y, int64_t n, int64_t sampsize, int64_t* yq, int32_t* q, cudaStream_t s);
+void bootstrap_impl(uint64_t seed, int32_t t0, int32_t ntrees, int64_t n, int64_t sampsize, int32_t replace,
+                    int32_t* w, cudaStream_t s);
+// predict.cu
+void predict_impl(const bf_forest* f, const double* Xq, int64_t ldq, int64_t m, double* yhat_sum, double* yhat,
+                  int32_t ntree_total, cudaStream_t s);
+// importance.cu
+void oob_importance_impl(const bf_forest* f, const double* X, int64_t ldx, const double* y, int64_t n, int32_t p,
+                         const bf_oob_accum& acc, cudaStream_t s);
+void importance_finalize_impl(const double* d_slots, const double* npur_slots, const double* oob_sum,
+                              const int32_t* oob_cnt, const double* y, int64_t n, int32_t p, int32_t ntree,
+                              double* out_p4 /* 4*p: inc, raw, sd, npur */, double* out_s2, cudaStream_t s);
+void perm_impl(uint64_t seed, int32_t t, int32_t m, int64_t n_o, int64_t* out, cudaStream_t s);
+// pca.cu
+void pca_impl(const double* X, int64_t ldx, int64_t n, int32_t p, int32_t scale, int32_t k, double* sdev,
+              double* rotation, double* center, double* scores, cudaStream_t s);
+// misc kernels (capi.cu)
+void philox_impl(const uint32_t* ctr, uint32_t k0, uint32_t k1, uint32_t* out, int64_t count, cudaStream_t s);
+void i128_impl(const int64_t* hi, const uint64_t* lo, double* out, int64_t count, cudaStream_t s);
+
+inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+}  // namespace bf

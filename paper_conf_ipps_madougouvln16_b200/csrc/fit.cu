@@ -1,0 +1,1593 @@
+// fit.cu -- forest construction on sm_100a.
+//
+// Design:
+//   once per fit   a1 validate, a2 fixed-point y_q, a3 presort: per feature the
+//                  rows in x order as 8-byte entries (dense rank << 32 | row)
+//                  plus the table of distinct values.
+//   per batch of B trees in flight:
+//     a4 bootstrap multiplicities (Philox BOOT), payload {w*y_q, w} per row;
+//     a5 root lists: per (tree, feature) stable compaction of the presorted
+//        column to in-bag rows (node-major block: p segments of a entries);
+//     GLOBAL PHASE (nodes with more than A distinct rows), level-synchronous
+//     over all trees of the batch:
+//        a6 k_mtry, a7 k_split_scan (CTA per (node, drawn feature): segmented
+//        prefix scan of (w, w*y_q) over the sorted segment, exact key, argmax),
+//        a8 k_finalize, k_child_place, a9/a10 k_dest (goes-right flags +
+//        child means), a9 k_partition (CTA per (node, feature): stable
+//        partition into the children's blocks);
+//     SUBTREE PHASE (nodes with <= A distinct rows): one CTA grows the whole
+//        subtree in shared memory (k_subtree);
+//     a11 emit the packed forest.
+// All split arithmetic is exact (int64 sums, int128 D, correctly rounded
+// key) so the topology is bit-identical to the CPU oracle whatever the scan
+// order, tile size or number of GPUs.
+#include <cub/cub.cuh>
+
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+
+#include "bf_internal.cuh"
+
+namespace bf {
+
+namespace {
+
+constexpr int NT = 256;         // threads per CTA of the streaming kernels
+constexpr int SUB_NW = 8;       // warps of the subtree kernel
+constexpr int SUB_NT = SUB_NW * 32;
+constexpr int KIND_NONE = -1, KIND_LEAF = 0, KIND_SMALL = 1, KIND_LARGE = 2;
+
+struct Pay {  // per (tree, row) payload: 16 B, one sector
+  int64_t wy;  // w * y_q (exact)
+  int32_t w;   // bootstrap multiplicity
+  int32_t pad;
+};
+
+struct LNode {  // an active node of the global phase, or a queued small node
+  int32_t b;     // tree index inside the batch
+  int32_t raw;   // node slot in the tree's raw pool
+  int32_t a;     // distinct in-bag rows
+  int32_t n;     // n_k = sum of w
+  int64_t S;     // S_k = sum of w * y_q
+  uint64_t key;  // node path key (S3 KEY)
+  int64_t base;  // element offset of the node's block (p segments of a entries)
+};
+
+struct Rec {  // best candidate of one (node, drawn feature)
+  double g;
+  uint32_t rank_a, rank_b;  // dense ranks of the values left / right of the boundary
+  int32_t pos;              // boundary position (last left entry) inside the segment
+  int32_t nl;
+  int64_t Sl;
+};
+
+struct Split {
+  int32_t split;  // 0 leaf, 1 split
+  int32_t f, pos, lraw;
+  int32_t nl, nr;
+  int32_t pad0, pad1;
+};
+
+struct Child {
+  int32_t kind, a, n, raw;
+  int64_t S;
+  uint64_t key;
+  int64_t base;
+};
+
+struct Pool {  // raw per-tree node pool of a batch (capacity `cap` per tree)
+  int32_t* feature;
+  int32_t* left;
+  int32_t* count;
+  double* thr;
+  double* value;
+  double* drss;
+  int32_t* nn;   // nodes used per tree
+  int64_t cap;
+};
+
+struct LevelSummary {
+  int32_t nnext;      // large nodes of the next level
+  int32_t nsmall;     // queued small nodes (total)
+  int64_t small_elems;  // elements used in the small-node area (total)
+  int64_t next_elems;   // elements of the next level's blocks
+  unsigned long long split_a;  // sum of a over the nodes split at this level
+  unsigned long long pad;
+};
+
+// ------------------------------------------------------------------ warp / block scans
+template <class T>
+__device__ __forceinline__ T warp_incl_scan(T v, int lane) {
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    T u = __shfl_up_sync(0xffffffffu, v, o);
+    if (lane >= o) v += u;
+  }
+  return v;
+}
+
+// Exclusive block scan; `sm` holds NT/32 elements; returns exclusive prefix and total.
+template <class T>
+__device__ __forceinline__ T block_excl_scan(T v, T* sm, T& total) {
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  T inc = warp_incl_scan(v, lane);
+  if (lane == 31) sm[wid] = inc;
+  __syncthreads();
+  if (wid == 0) {
+    T s = lane < nw ? sm[lane] : T(0);
+    s = warp_incl_scan(s, lane);
+    if (lane < nw) sm[lane] = s;
+  }
+  __syncthreads();
+  T pre = wid ? sm[wid - 1] : T(0);
+  total = sm[nw - 1];
+  __syncthreads();
+  return pre + inc - v;
+}
+
+// ------------------------------------------------------------------ a1 validate
+__global__ void k_validate(const double* X, int64_t ldx, int64_t n, int32_t p, const double* y, int* bad) {
+  const int64_t total = n * (int64_t)p;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total + n; i += (int64_t)gridDim.x * blockDim.x) {
+    double v;
+    if (i < total) {
+      const int64_t j = i / n, r = i - j * n;
+      v = X[j * ldx + r];
+    } else {
+      v = y[i - total];
+    }
+    if (!isfinite(v)) atomicOr(bad, 1);
+  }
+}
+
+// ------------------------------------------------------------------ a2 fixed point
+__global__ void k_minmax(const double* y, int64_t n, double* part) {  // part[2*blk] = min, max
+  __shared__ double smin[NT], smax[NT];
+  double mn = INFINITY, mx = -INFINITY;
+  for (int64_t i = blockIdx.x * (int64_t)NT + threadIdx.x; i < n; i += (int64_t)gridDim.x * NT) {
+    mn = fmin(mn, y[i]);
+    mx = fmax(mx, y[i]);
+  }
+  smin[threadIdx.x] = mn;
+  smax[threadIdx.x] = mx;
+  __syncthreads();
+  for (int s = NT / 2; s > 0; s >>= 1) {
+    if (threadIdx.x < s) {
+      smin[threadIdx.x] = fmin(smin[threadIdx.x], smin[threadIdx.x + s]);
+      smax[threadIdx.x] = fmax(smax[threadIdx.x], smax[threadIdx.x + s]);
+    }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    part[2 * blockIdx.x] = smin[0];
+    part[2 * blockIdx.x + 1] = smax[0];
+  }
+}
+
+__global__ void k_absdev_max(const double* y, int64_t n, double c, double* part) {
+  __shared__ double sm[NT];
+  double mx = 0.0;
+  for (int64_t i = blockIdx.x * (int64_t)NT + threadIdx.x; i < n; i += (int64_t)gridDim.x * NT)
+    mx = fmax(mx, fabs(__dsub_rn(y[i], c)));
+  sm[threadIdx.x] = mx;
+  __syncthreads();
+  for (int s = NT / 2; s > 0; s >>= 1) {
+    if (threadIdx.x < s) sm[threadIdx.x] = fmax(sm[threadIdx.x], sm[threadIdx.x + s]);
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) part[blockIdx.x] = sm[0];
+}
+
+__global__ void k_yq(const double* y, int64_t n, double c, int q, int zero, int64_t* yq) {
+  for (int64_t i = blockIdx.x * (int64_t)NT + threadIdx.x; i < n; i += (int64_t)gridDim.x * NT)
+    yq[i] = zero ? 0 : __double2ll_rn(ldexp(__dsub_rn(y[i], c), q));
+}
+
+// ------------------------------------------------------------------ a3 presort
+__global__ void k_sort_keys(const double* col, int64_t n, uint64_t* keys, uint32_t* vals) {
+  for (int64_t i = blockIdx.x * (int64_t)NT + threadIdx.x; i < n; i += (int64_t)gridDim.x * NT) {
+    const uint64_t b = (uint64_t)__double_as_longlong(canon(col[i]));
+    keys[i] = (b >> 63) ? ~b : (b | 0x8000000000000000ull);  // order-preserving
+    vals[i] = (uint32_t)i;
+  }
+}
+
+__global__ void k_rank_flags(const uint64_t* keys, int64_t n, uint32_t* flags) {
+  for (int64_t i = blockIdx.x * (int64_t)NT + threadIdx.x; i < n; i += (int64_t)gridDim.x * NT)
+    flags[i] = (i > 0 && keys[i] != keys[i - 1]) ? 1u : 0u;
+}
+
+__global__ void k_fill_sorted(const double* col, const uint32_t* rows, const uint32_t* rank, int64_t n,
+                              uint64_t* srt, double* uniq) {
+  for (int64_t i = blockIdx.x * (int64_t)NT + threadIdx.x; i < n; i += (int64_t)gridDim.x * NT) {
+    const uint32_t r = rows[i], k = rank[i];
+    srt[i] = ((uint64_t)k << 32) | r;
+    if (i == 0 || rank[i - 1] != k) uniq[k] = canon(col[r]);
+  }
+}
+
+// ------------------------------------------------------------------ a4 bootstrap
+__global__ void k_bootstrap(uint64_t seed, int32_t t0, int64_t n, int64_t ns, int32_t* w) {
+  const int b = blockIdx.y;
+  const uint32_t t = (uint32_t)(t0 + b);
+  const int64_t j2 = blockIdx.x * (int64_t)NT + threadIdx.x;
+  if (2 * j2 >= ns) return;
+  uint64_t u0, u1;
+  philox_u64x2(seed, (uint32_t)j2, t, 1u, 0u, u0, u1);
+  int32_t* wb = w + (int64_t)b * n;
+  atomicAdd(&wb[mulhi64(u0, (uint64_t)n)], 1);
+  if (2 * j2 + 1 < ns) atomicAdd(&wb[mulhi64(u1, (uint64_t)n)], 1);
+}
+
+__global__ void k_fill_i32(int32_t* a, int64_t count, int32_t v) {
+  for (int64_t i = blockIdx.x * (int64_t)NT + threadIdx.x; i < count; i += (int64_t)gridDim.x * NT) a[i] = v;
+}
+
+// payload + per-tree root sums: a (distinct), S (exact), sum w*y (fp64)
+__global__ void k_payload(const int32_t* w, const int64_t* yq, const double* y, int64_t n, Pay* pay,
+                          int32_t* a_root, unsigned long long* S_root, double* sy_root) {
+  __shared__ int32_t sa[NT / 32];
+  __shared__ int64_t sS[NT / 32];
+  __shared__ double sy[NT / 32];
+  const int b = blockIdx.y;
+  const int64_t i = blockIdx.x * (int64_t)NT + threadIdx.x;
+  int32_t wi = 0;
+  int64_t wyq = 0;
+  double wy = 0.0;
+  if (i < n) {
+    wi = w[(int64_t)b * n + i];
+    wyq = (int64_t)wi * yq[i];
+    wy = __dmul_rn((double)wi, y[i]);
+    Pay pp;
+    pp.wy = wyq;
+    pp.w = wi;
+    pp.pad = 0;
+    pay[(int64_t)b * n + i] = pp;
+  }
+  int32_t ca = wi > 0;
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    ca += __shfl_down_sync(0xffffffffu, ca, o);
+    wyq += __shfl_down_sync(0xffffffffu, wyq, o);
+    wy += __shfl_down_sync(0xffffffffu, wy, o);
+  }
+  if (lane == 0) {
+    sa[wid] = ca;
+    sS[wid] = wyq;
+    sy[wid] = wy;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    int32_t A = 0;
+    int64_t S = 0;
+    double Y = 0.0;
+    for (int k = 0; k < NT / 32; ++k) {
+      A += sa[k];
+      S += sS[k];
+      Y += sy[k];
+    }
+    atomicAdd(&a_root[b], A);
+    atomicAdd(&S_root[b], (unsigned long long)S);
+    atomicAdd(&sy_root[b], Y);
+  }
+}
+
+// root records + root node descriptors
+__global__ void k_roots(int B, int64_t ns, int nodesize, const int32_t* a_root, const unsigned long long* S_root,
+                        const double* sy_root, const int32_t* kind, const int64_t* base, Pool pool, LNode* lroots,
+                        int32_t* lidx, LNode* sq, int32_t* sidx) {
+  const int b = blockIdx.x * blockDim.x + threadIdx.x;
+  if (b >= B) return;
+  const int64_t r0 = (int64_t)b * pool.cap;
+  pool.feature[r0] = -1;
+  pool.left[r0] = -1;
+  pool.count[r0] = (int32_t)ns;
+  pool.thr[r0] = 0.0;
+  pool.value[r0] = __ddiv_rn(sy_root[b], (double)ns);
+  pool.drss[r0] = 0.0;
+  pool.nn[b] = 1;
+  LNode nd;
+  nd.b = b;
+  nd.raw = 0;
+  nd.a = a_root[b];
+  nd.n = (int32_t)ns;
+  nd.S = (int64_t)S_root[b];
+  nd.key = 0;
+  nd.base = base[b];
+  if (kind[b] == KIND_LARGE) lroots[lidx[b]] = nd;
+  if (kind[b] == KIND_SMALL) sq[sidx[b]] = nd;
+}
+
+// ------------------------------------------------------------------ a5 root lists (two-pass stable compaction)
+constexpr int LCH = 2048;  // entries per CTA chunk (256 threads x 8)
+
+__global__ void k_list_count(const uint64_t* srt, int64_t n, const Pay* pay, const int32_t* kind, int nchunk,
+                             int32_t* cnt) {
+  const int c = blockIdx.x, f = blockIdx.y, b = blockIdx.z, p = gridDim.y;
+  if (kind[b] != KIND_LARGE && kind[b] != KIND_SMALL) return;
+  __shared__ int32_t sm[NT / 32];
+  const uint64_t* col = srt + (int64_t)f * n;
+  const Pay* P = pay + (int64_t)b * n;
+  int32_t k = 0;
+  for (int u = threadIdx.x; u < LCH; u += NT) {
+    const int64_t i = (int64_t)c * LCH + u;
+    if (i < n) k += P[(uint32_t)col[i]].w > 0;
+  }
+  int32_t tot;
+  block_excl_scan(k, sm, tot);
+  if (threadIdx.x == 0) cnt[((int64_t)b * p + f) * nchunk + c] = tot;
+}
+
+__global__ void k_list_prefix(int32_t* cnt, int nseg, int nchunk) {
+  const int s = blockIdx.x * blockDim.x + threadIdx.x;
+  if (s >= nseg) return;
+  int32_t* c = cnt + (int64_t)s * nchunk;
+  int32_t acc = 0;
+  for (int i = 0; i < nchunk; ++i) {
+    int32_t v = c[i];
+    c[i] = acc;
+    acc += v;
+  }
+}
+
+__global__ void k_list_scatter(const uint64_t* srt, int64_t n, const Pay* pay, const int32_t* kind,
+                               const int64_t* base, const int32_t* a_root, int nchunk, const int32_t* cnt,
+                               uint64_t* Elarge, uint64_t* Esmall) {
+  const int c = blockIdx.x, f = blockIdx.y, b = blockIdx.z, p = gridDim.y;
+  const int kd = kind[b];
+  if (kd != KIND_LARGE && kd != KIND_SMALL) return;
+  __shared__ int32_t sm[NT / 32];
+  const uint64_t* col = srt + (int64_t)f * n;
+  const Pay* P = pay + (int64_t)b * n;
+  constexpr int V = LCH / NT;
+  uint64_t e[V];
+  bool keep[V];
+  int32_t k = 0;
+  const int64_t i0 = (int64_t)c * LCH + (int64_t)threadIdx.x * V;
+#pragma unroll
+  for (int u = 0; u < V; ++u) {
+    const int64_t i = i0 + u;
+    keep[u] = false;
+    if (i < n) {
+      e[u] = col[i];
+      keep[u] = P[(uint32_t)e[u]].w > 0;
+    }
+    k += keep[u];
+  }
+  int32_t tot;
+  int32_t pre = block_excl_scan(k, sm, tot) + cnt[((int64_t)b * p + f) * nchunk + c];
+  uint64_t* dst = (kd == KIND_LARGE ? Elarge : Esmall) + base[b] + (int64_t)f * a_root[b];
+#pragma unroll
+  for (int u = 0; u < V; ++u)
+    if (keep[u]) dst[pre++] = e[u];
+}
+
+// ------------------------------------------------------------------ a6 mtry (global phase)
+__global__ void k_mtry(const LNode* nodes, int N, int p, int mtry, uint64_t seed, int32_t t0, int32_t* feat,
+                       int16_t* scratch) {
+  const int k = blockIdx.x * blockDim.x + threadIdx.x;
+  if (k >= N) return;
+  const LNode nd = nodes[k];
+  int16_t* mind = scratch + (int64_t)k * p;
+  for (int j = 0; j < p; ++j) mind[j] = (int16_t)j;
+  int last = p - 1;
+  uint64_t u0 = 0, u1 = 0;
+  for (int i = 0; i < mtry; ++i) {
+    if ((i & 1) == 0)
+      philox_u64x2(seed, (uint32_t)nd.key, (uint32_t)(nd.key >> 32), (uint32_t)(t0 + nd.b),
+                   0x20000000u | (uint32_t)(i >> 1), u0, u1);
+    const uint64_t u = (i & 1) ? u1 : u0;
+    const int j = (int)mulhi64(u, (uint64_t)(last + 1));
+    feat[(int64_t)k * mtry + i] = mind[j];
+    const int16_t tmp = mind[j];
+    mind[j] = mind[last];
+    mind[last] = tmp;
+    --last;
+  }
+}
+
+// ------------------------------------------------------------------ a7 split scan (global phase)
+// One CTA per (node, drawn feature): chunked segmented scan with a carry.
+constexpr int SV = 4;            // entries per thread per chunk
+constexpr int SCH = NT * SV;     // 1024 entries per chunk
+
+__device__ __forceinline__ bool rec_better(double g, uint32_t r, double bg, uint32_t br) {
+  return g > bg || (g == bg && r < br);
+}
+
+__global__ void __launch_bounds__(NT) k_split_scan(const LNode* nodes, const int32_t* feat, int mtry,
+                                                   const uint64_t* E, const Pay* pay, int64_t n, Rec* rec) {
+  __shared__ int32_t smc[NT / 32];
+  __shared__ int64_t sms[NT / 32];
+  __shared__ double sg[NT / 32];
+  __shared__ uint32_t sr[NT / 32];
+  __shared__ int32_t sw[NT / 32];
+  const int64_t item = blockIdx.x;
+  const LNode nd = nodes[item / mtry];
+  const int f = feat[item];
+  const uint64_t* seg = E + nd.base + (int64_t)f * nd.a;
+  const Pay* P = pay + (int64_t)nd.b * n;
+  const int a = nd.a;
+  const int64_t nk = nd.n, Sk = nd.S;
+  int32_t carry_c = 0;
+  int64_t carry_s = 0;
+  double bg = -1.0;
+  uint32_t brank = 0xffffffffu, brb = 0;
+  int32_t bpos = -1, bnl = 0;
+  int64_t bSl = 0;
+  for (int c0 = 0; c0 < a; c0 += SCH) {
+    const int j0 = c0 + threadIdx.x * SV;
+    uint64_t e[SV + 1];
+    int32_t wc[SV];
+    int64_t ws[SV];
+    int32_t tc = 0;
+    int64_t ts = 0;
+#pragma unroll
+    for (int u = 0; u <= SV; ++u) e[u] = (j0 + u < a) ? seg[j0 + u] : 0ull;
+#pragma unroll
+    for (int u = 0; u < SV; ++u) {
+      wc[u] = 0;
+      ws[u] = 0;
+      if (j0 + u < a) {
+        const Pay pp = P[(uint32_t)e[u]];
+        wc[u] = pp.w;
+        ws[u] = pp.wy;
+      }
+      tc += wc[u];
+      ts += ws[u];
+    }
+    int32_t totc;
+    int64_t tots;
+    int32_t prec = block_excl_scan(tc, smc, totc) + carry_c;
+    int64_t pres = block_excl_scan(ts, sms, tots) + carry_s;
+#pragma unroll
+    for (int u = 0; u < SV; ++u) {
+      prec += wc[u];
+      pres += ws[u];
+      const int j = j0 + u;
+      if (j + 1 < a) {
+        const uint32_t ra = (uint32_t)(e[u] >> 32), rb = (uint32_t)(e[u + 1] >> 32);
+        if (ra != rb) {
+          const double g = split_key(nk, Sk, prec, pres);
+          if (rec_better(g, ra, bg, brank)) {
+            bg = g;
+            brank = ra;
+            brb = rb;
+            bpos = j;
+            bnl = prec;
+            bSl = pres;
+          }
+        }
+      }
+    }
+    carry_c += totc;
+    carry_s += tots;
+  }
+  // block argmax (g desc, rank asc)
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  int src = lane;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const double og = __shfl_down_sync(0xffffffffu, bg, o);
+    const uint32_t orr = __shfl_down_sync(0xffffffffu, brank, o);
+    const int os = __shfl_down_sync(0xffffffffu, src, o);
+    if (lane + o < 32 && rec_better(og, orr, bg, brank)) {
+      bg = og;
+      brank = orr;
+      src = os;
+    }
+  }
+  src = __shfl_sync(0xffffffffu, src, 0);
+  if (lane == 0) {
+    sg[wid] = bg;
+    sr[wid] = brank;
+    sw[wid] = wid * 32 + src;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double g = sg[0];
+    uint32_t r = sr[0];
+    int who = sw[0];
+    for (int k = 1; k < NT / 32; ++k)
+      if (rec_better(sg[k], sr[k], g, r)) {
+        g = sg[k];
+        r = sr[k];
+        who = sw[k];
+      }
+    sw[0] = who;
+  }
+  __syncthreads();
+  if (threadIdx.x == sw[0]) {
+    Rec R;
+    R.g = bg;
+    R.rank_a = brank;
+    R.rank_b = brb;
+    R.pos = bpos;
+    R.nl = bnl;
+    R.Sl = bSl;
+    rec[item] = R;
+  }
+}
+
+// ------------------------------------------------------------------ a8 node finalize (global phase)
+__global__ void k_finalize(const LNode* nodes, int N, const int32_t* feat, const Rec* rec, int mtry,
+                           const double* uniq, int64_t n, int nodesize, int Asmall, int q, uint64_t seed,
+                           int32_t t0, Pool pool, Split* split, Child* child, uint64_t* packL, uint64_t* packS,
+                           LevelSummary* sum) {
+  const int k = blockIdx.x * blockDim.x + threadIdx.x;
+  if (k >= N) return;
+  const LNode nd = nodes[k];
+  double bg = -1.0;
+  int bf = 0x7fffffff;
+  Rec br;
+  br.g = -1.0;
+  for (int s = 0; s < mtry; ++s) {
+    const Rec R = rec[(int64_t)k * mtry + s];
+    const int f = feat[(int64_t)k * mtry + s];
+    if (R.g < 0) continue;
+    if (R.g > bg || (R.g == bg && f < bf)) {
+      bg = R.g;
+      bf = f;
+      br = R;
+    }
+  }
+  Split sp;
+  sp.split = 0;
+  sp.pad0 = sp.pad1 = 0;
+  Child cl, cr;
+  cl.kind = cr.kind = KIND_NONE;
+  if (bg > 0.0) {
+    const double xa = uniq[(int64_t)bf * n + br.rank_a], xb = uniq[(int64_t)bf * n + br.rank_b];
+    const double thr = split_threshold(xa, xb);
+    const int32_t lraw = atomicAdd(&pool.nn[nd.b], 2);
+    const int64_t r = (int64_t)nd.b * pool.cap;
+    pool.feature[r + nd.raw] = bf;
+    pool.thr[r + nd.raw] = thr;
+    pool.left[r + nd.raw] = lraw;
+    pool.drss[r + nd.raw] = ldexp(__ddiv_rn(bg, (double)nd.n), -2 * q);
+    const uint32_t t = (uint32_t)(t0 + nd.b);
+    cl.a = br.pos + 1;
+    cl.n = br.nl;
+    cl.S = br.Sl;
+    cl.key = child_key(seed, t, nd.key, 0);
+    cl.raw = lraw;
+    cr.a = nd.a - cl.a;
+    cr.n = nd.n - br.nl;
+    cr.S = nd.S - br.Sl;
+    cr.key = child_key(seed, t, nd.key, 1);
+    cr.raw = lraw + 1;
+    Child* cs[2] = {&cl, &cr};
+    for (int side = 0; side < 2; ++side) {
+      Child& c = *cs[side];
+      c.base = 0;
+      if (c.n <= nodesize || c.a < 2) c.kind = KIND_LEAF;
+      else if (c.a <= Asmall) c.kind = KIND_SMALL;
+      else c.kind = KIND_LARGE;
+      pool.feature[r + c.raw] = -1;
+      pool.left[r + c.raw] = -1;
+      pool.count[r + c.raw] = c.n;
+      pool.thr[r + c.raw] = 0.0;
+      pool.drss[r + c.raw] = 0.0;
+    }
+    atomicAdd(&sum->split_a, (unsigned long long)nd.a);
+    sp.split = 1;
+    sp.f = bf;
+    sp.pos = br.pos;
+    sp.lraw = lraw;
+    sp.nl = cl.n;
+    sp.nr = cr.n;
+  }
+  split[k] = sp;
+  child[2 * k] = cl;
+  child[2 * k + 1] = cr;
+  packL[2 * k] = cl.kind == KIND_LARGE ? (((uint64_t)cl.a << 32) | 1u) : 0ull;
+  packL[2 * k + 1] = cr.kind == KIND_LARGE ? (((uint64_t)cr.a << 32) | 1u) : 0ull;
+  packS[2 * k] = cl.kind == KIND_SMALL ? (((uint64_t)cl.a << 32) | 1u) : 0ull;
+  packS[2 * k + 1] = cr.kind == KIND_SMALL ? (((uint64_t)cr.a << 32) | 1u) : 0ull;
+}
+
+// child placement: next-level node list and small queue
+__global__ void k_child_place(int N2, int p, const LNode* nodes, Child* child, const uint64_t* scanL,
+                              const uint64_t* scanS, LNode* next, LNode* sq, const LevelSummary* prev) {
+  const int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= N2) return;
+  const Child ch = child[c];
+  if (ch.kind != KIND_LARGE && ch.kind != KIND_SMALL) return;
+  LNode nd;
+  nd.b = nodes[c >> 1].b;
+  nd.raw = ch.raw;
+  nd.a = ch.a;
+  nd.n = ch.n;
+  nd.S = ch.S;
+  nd.key = ch.key;
+  if (ch.kind == KIND_LARGE) {
+    const uint64_t sc = scanL[c];
+    nd.base = (int64_t)p * (int64_t)(sc >> 32);
+    child[c].base = nd.base;
+    next[(uint32_t)sc] = nd;
+  } else {
+    const uint64_t sc = scanS[c];
+    nd.base = prev->small_elems + (int64_t)p * (int64_t)(sc >> 32);
+    child[c].base = nd.base;
+    sq[prev->nsmall + (uint32_t)sc] = nd;
+  }
+}
+
+__global__ void k_commit(int N2, const uint64_t* packL, const uint64_t* scanL, const uint64_t* packS,
+                         const uint64_t* scanS, int p, LevelSummary* sum, LevelSummary* host_sum) {
+  LevelSummary s = *sum;
+  uint64_t tl = 0, ts = 0;
+  if (N2 > 0) {
+    tl = scanL[N2 - 1] + packL[N2 - 1];
+    ts = scanS[N2 - 1] + packS[N2 - 1];
+  }
+  s.nnext = (int32_t)(uint32_t)tl;
+  s.next_elems = (int64_t)p * (int64_t)(tl >> 32);
+  s.nsmall += (int32_t)(uint32_t)ts;
+  s.small_elems += (int64_t)p * (int64_t)(ts >> 32);
+  *host_sum = s;
+  s.split_a = 0;
+  *sum = s;
+}
+
+// ------------------------------------------------------------------ a9/a10 goes-right flags + child values
+__global__ void __launch_bounds__(NT) k_dest(const LNode* nodes, const Split* split, const uint64_t* E,
+                                             const Pay* pay, const double* y, int64_t n, uint8_t* side,
+                                             Pool pool) {
+  __shared__ double sl[NT], sr[NT];
+  const int k = blockIdx.x;
+  const Split sp = split[k];
+  if (!sp.split) return;
+  const LNode nd = nodes[k];
+  const uint64_t* seg = E + nd.base + (int64_t)sp.f * nd.a;
+  const Pay* P = pay + (int64_t)nd.b * n;
+  uint8_t* sd = side + (int64_t)nd.b * n;
+  double accl = 0.0, accr = 0.0;
+  for (int j = threadIdx.x; j < nd.a; j += NT) {
+    const uint32_t row = (uint32_t)seg[j];
+    const int s = j > sp.pos;
+    sd[row] = (uint8_t)s;
+    const double v = __dmul_rn((double)P[row].w, y[row]);
+    if (s) accr += v;
+    else accl += v;
+  }
+  sl[threadIdx.x] = accl;
+  sr[threadIdx.x] = accr;
+  __syncthreads();
+  for (int s = NT / 2; s > 0; s >>= 1) {
+    if (threadIdx.x < s) {
+      sl[threadIdx.x] += sl[threadIdx.x + s];
+      sr[threadIdx.x] += sr[threadIdx.x + s];
+    }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    const int64_t r = (int64_t)nd.b * pool.cap;
+    pool.value[r + sp.lraw] = __ddiv_rn(sl[0], (double)sp.nl);
+    pool.value[r + sp.lraw + 1] = __ddiv_rn(sr[0], (double)sp.nr);
+  }
+}
+
+// ------------------------------------------------------------------ a9 partition
+constexpr int PV = 4;
+constexpr int PCH = NT * PV;
+
+__global__ void __launch_bounds__(NT) k_partition(const LNode* nodes, const Split* split, const Child* child,
+                                                  int p, const uint64_t* Ecur, const uint8_t* side, int64_t n,
+                                                  uint64_t* Enext, uint64_t* Esmall) {
+  __shared__ int32_t sm[NT / 32];
+  const int k = blockIdx.x;
+  const int f = blockIdx.y;
+  const Split sp = split[k];
+  if (!sp.split) return;
+  const Child cl = child[2 * k], cr = child[2 * k + 1];
+  const bool keepL = cl.kind == KIND_LARGE || cl.kind == KIND_SMALL;
+  const bool keepR = cr.kind == KIND_LARGE || cr.kind == KIND_SMALL;
+  if (!keepL && !keepR) return;
+  const LNode nd = nodes[k];
+  const uint64_t* seg = Ecur + nd.base + (int64_t)f * nd.a;
+  const uint8_t* sd = side + (int64_t)nd.b * n;
+  uint64_t* dl = keepL ? (cl.kind == KIND_LARGE ? Enext : Esmall) + cl.base + (int64_t)f * cl.a : nullptr;
+  uint64_t* dr = keepR ? (cr.kind == KIND_LARGE ? Enext : Esmall) + cr.base + (int64_t)f * cr.a : nullptr;
+  int32_t carry = 0;
+  for (int c0 = 0; c0 < nd.a; c0 += PCH) {
+    const int j0 = c0 + threadIdx.x * PV;
+    uint64_t e[PV];
+    bool left[PV];
+    int32_t cnt = 0;
+#pragma unroll
+    for (int u = 0; u < PV; ++u) {
+      left[u] = false;
+      if (j0 + u < nd.a) {
+        e[u] = seg[j0 + u];
+        left[u] = sd[(uint32_t)e[u]] == 0;
+      }
+      cnt += left[u];
+    }
+    int32_t tot;
+    int32_t lb = block_excl_scan(cnt, sm, tot) + carry;
+#pragma unroll
+    for (int u = 0; u < PV; ++u) {
+      const int j = j0 + u;
+      if (j < nd.a) {
+        if (left[u]) {
+          if (keepL) dl[lb] = e[u];
+          ++lb;
+        } else if (keepR) {
+          dr[j - lb] = e[u];
+        }
+      }
+    }
+    carry += tot;
+  }
+}
+
+// ------------------------------------------------------------------ subtree phase
+struct SRec {  // node record of a subtree (local ids)
+  int32_t feature, left, count, pad;
+  double thr, value, drss;
+};
+struct SCur {  // active node of a subtree level
+  int32_t off, a, n, id;
+  int64_t S;
+  uint64_t key;
+  int32_t split, lid, al, nl;
+  int64_t Sl;
+  uint64_t keyl, keyr;
+  int32_t coff[2];
+};
+
+__host__ __device__ inline size_t align16(size_t x) { return (x + 15) & ~size_t(15); }
+
+__host__ __device__ inline size_t subtree_smem(int A, int p) {
+  size_t s = 0;
+  s += align16(2 * (size_t)p * A * 4);       // ent0, ent1
+  s += align16((size_t)A * 8);               // wy
+  s += align16((size_t)A * 8);               // w*y fp64
+  s += align16((size_t)2 * A * sizeof(SRec));
+  s += align16((size_t)2 * (A / 2 + 1) * sizeof(SCur));
+  s += align16((size_t)A * 4);               // w
+  s += align16((size_t)A * 4);               // global row
+  s += align16((size_t)SUB_NW * p * 2);      // Fisher-Yates scratch
+  s += align16((size_t)SUB_NW * p * 2);      // drawn features
+  s += align16((size_t)A);                   // side
+  s += 64;
+  return s;
+}
+
+struct SubArgs {
+  const LNode* sq;
+  const uint64_t* Es;
+  const Pay* pay;
+  const double* y;
+  const double* X;
+  int64_t ldx;
+  int64_t n;
+  int p, mtry, nodesize, q, A;
+  uint64_t seed;
+  int32_t t0;
+  uint16_t* loc;
+  Pool pool;
+};
+
+__global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  const int A = g.A, p = g.p;
+  unsigned char* ptr = smem;
+  uint32_t* ent0 = (uint32_t*)ptr;
+  uint32_t* ent1 = ent0 + (size_t)p * A;
+  ptr += align16(2 * (size_t)p * A * 4);
+  int64_t* wy = (int64_t*)ptr;
+  ptr += align16((size_t)A * 8);
+  double* wyd = (double*)ptr;
+  ptr += align16((size_t)A * 8);
+  SRec* recs = (SRec*)ptr;
+  ptr += align16((size_t)2 * A * sizeof(SRec));
+  SCur* curl = (SCur*)ptr;
+  SCur* nxtl = curl + (A / 2 + 1);
+  ptr += align16((size_t)2 * (A / 2 + 1) * sizeof(SCur));
+  int32_t* wl = (int32_t*)ptr;
+  ptr += align16((size_t)A * 4);
+  uint32_t* grow = (uint32_t*)ptr;
+  ptr += align16((size_t)A * 4);
+  int16_t* mind_all = (int16_t*)ptr;
+  ptr += align16((size_t)SUB_NW * p * 2);
+  int16_t* feats_all = (int16_t*)ptr;
+  ptr += align16((size_t)SUB_NW * p * 2);
+  uint8_t* side = (uint8_t*)ptr;
+  __shared__ int s_nloc, s_ncur, s_gbase;
+
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const LNode root = g.sq[blockIdx.x];
+  const int a0 = root.a;
+  const int b = root.b;
+  const uint32_t t = (uint32_t)(g.t0 + b);
+  const Pay* P = g.pay + (int64_t)b * g.n;
+  uint16_t* loc = g.loc + (int64_t)b * g.n;
+  const uint64_t* src = g.Es + root.base;
+
+  // ---- load: local rows from feature 0's list, payload, then local ranks per feature
+  for (int j = tid; j < a0; j += SUB_NT) {
+    const uint32_t row = (uint32_t)src[j];
+    grow[j] = row;
+    loc[row] = (uint16_t)j;
+    const Pay pp = P[row];
+    wl[j] = pp.w;
+    wy[j] = pp.wy;
+    wyd[j] = __dmul_rn((double)pp.w, g.y[row]);
+  }
+  __syncthreads();
+  for (int f = wid; f < p; f += SUB_NW) {
+    const uint64_t* sf = src + (int64_t)f * a0;
+    uint32_t carry = 0, prevr = 0xffffffffu;
+    for (int j0 = 0; j0 < a0; j0 += 32) {
+      const int j = j0 + lane;
+      uint64_t e = j < a0 ? sf[j] : 0;
+      const uint32_t r = (uint32_t)(e >> 32);
+      const uint32_t rprev = __shfl_up_sync(0xffffffffu, r, 1);
+      const uint32_t before = lane == 0 ? prevr : rprev;
+      const uint32_t flag = (j < a0 && j > 0 && r != before) ? 1u : 0u;
+      const uint32_t inc = warp_incl_scan(flag, lane) + carry;
+      if (j < a0) ent0[(size_t)f * a0 + j] = (inc << 16) | (uint32_t)loc[(uint32_t)e];
+      carry = __shfl_sync(0xffffffffu, inc, 31);
+      prevr = __shfl_sync(0xffffffffu, r, 31);
+    }
+  }
+  if (tid == 0) {
+    s_nloc = 1;
+    s_ncur = 1;
+    SRec r0;
+    r0.feature = -1;
+    r0.left = -1;
+    r0.count = root.n;
+    r0.pad = 0;
+    r0.thr = 0.0;
+    r0.value = 0.0;
+    r0.drss = 0.0;
+    recs[0] = r0;
+    SCur c;
+    c.off = 0;
+    c.a = a0;
+    c.n = root.n;
+    c.id = 0;
+    c.S = root.S;
+    c.key = root.key;
+    c.split = 0;
+    curl[0] = c;
+  }
+  __syncthreads();
+
+  uint32_t* cbuf = ent0;
+  uint32_t* nbuf = ent1;
+  int16_t* mind = mind_all + wid * p;
+  int16_t* feats = feats_all + wid * p;
+  while (s_ncur > 0) {
+    const int ncur = s_ncur;
+    // ---- phase A: warp per node: draw, scan, choose, mark sides, child means
+    for (int i = wid; i < ncur; i += SUB_NW) {
+      SCur nd = curl[i];
+      if (lane == 0) {
+        for (int j = 0; j < p; ++j) mind[j] = (int16_t)j;
+        int last = p - 1;
+        uint64_t u0 = 0, u1 = 0;
+        for (int s = 0; s < g.mtry; ++s) {
+          if ((s & 1) == 0)
+            philox_u64x2(g.seed, (uint32_t)nd.key, (uint32_t)(nd.key >> 32), t, 0x20000000u | (uint32_t)(s >> 1),
+                         u0, u1);
+          const uint64_t u = (s & 1) ? u1 : u0;
+          const int j = (int)mulhi64(u, (uint64_t)(last + 1));
+          feats[s] = mind[j];
+          const int16_t tmp = mind[j];
+          mind[j] = mind[last];
+          mind[last] = tmp;
+          --last;
+        }
+      }
+      __syncwarp();
+      double bg = -1.0;
+      int bf = 0x7fffffff, bpos = -1, bnl = 0;
+      int64_t bSl = 0;
+      uint32_t bra = 0, brb = 0;
+      const int64_t nk = nd.n, Sk = nd.S;
+      for (int s = 0; s < g.mtry; ++s) {
+        const int f = feats[s];
+        const uint32_t* seg = cbuf + nd.off + (size_t)f * nd.a;
+        int32_t cc = 0;
+        int64_t cs = 0;
+        double lg = -1.0;
+        uint32_t lrk = 0xffffffffu, lra = 0, lrb = 0;
+        int lpos = -1, lnl = 0;
+        int64_t lSl = 0;
+        for (int j0 = 0; j0 < nd.a; j0 += 32) {
+          const int j = j0 + lane;
+          const uint32_t e = j < nd.a ? seg[j] : 0u;
+          const uint32_t lr = e & 0xffffu;
+          const int32_t w = j < nd.a ? wl[lr] : 0;
+          const int64_t ws = j < nd.a ? wy[lr] : 0;
+          const int32_t ic = warp_incl_scan(w, lane) + cc;
+          const int64_t is = warp_incl_scan(ws, lane) + cs;
+          if (j + 1 < nd.a) {
+            const uint32_t en = seg[j + 1];
+            if ((en >> 16) != (e >> 16)) {
+              const double gk = split_key(nk, Sk, ic, is);
+              if (rec_better(gk, e >> 16, lg, lrk)) {
+                lg = gk;
+                lrk = e >> 16;
+                lra = lr;
+                lrb = en & 0xffffu;
+                lpos = j;
+                lnl = ic;
+                lSl = is;
+              }
+            }
+          }
+          cc = __shfl_sync(0xffffffffu, ic, 31);
+          cs = __shfl_sync(0xffffffffu, is, 31);
+        }
+        // warp argmax over lanes (g desc, local rank asc)
+        int srcl = lane;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+          const double og = __shfl_down_sync(0xffffffffu, lg, o);
+          const uint32_t orr = __shfl_down_sync(0xffffffffu, lrk, o);
+          const int os = __shfl_down_sync(0xffffffffu, srcl, o);
+          if (lane + o < 32 && rec_better(og, orr, lg, lrk)) {
+            lg = og;
+            lrk = orr;
+            srcl = os;
+          }
+        }
+        srcl = __shfl_sync(0xffffffffu, srcl, 0);
+        lg = __shfl_sync(0xffffffffu, lg, 0);
+        const int wpos = __shfl_sync(0xffffffffu, lpos, srcl);
+        const int wnl = __shfl_sync(0xffffffffu, lnl, srcl);
+        const int64_t wSl = __shfl_sync(0xffffffffu, lSl, srcl);
+        const uint32_t wra = __shfl_sync(0xffffffffu, lra, srcl);
+        const uint32_t wrb = __shfl_sync(0xffffffffu, lrb, srcl);
+        if (lg >= 0.0 && (lg > bg || (lg == bg && f < bf))) {
+          bg = lg;
+          bf = f;
+          bpos = wpos;
+          bnl = wnl;
+          bSl = wSl;
+          bra = wra;
+          brb = wrb;
+        }
+      }
+      if (bg > 0.0) {
+        int lid = 0;
+        if (lane == 0) {
+          const double xa = canon(g.X[(int64_t)bf * g.ldx + grow[bra]]);
+          const double xb = canon(g.X[(int64_t)bf * g.ldx + grow[brb]]);
+          lid = atomicAdd(&s_nloc, 2);
+          SRec& r = recs[nd.id];
+          r.feature = bf;
+          r.left = lid;
+          r.thr = split_threshold(xa, xb);
+          r.drss = ldexp(__ddiv_rn(bg, (double)nd.n), -2 * g.q);
+          nd.keyl = child_key(g.seed, t, nd.key, 0);
+          nd.keyr = child_key(g.seed, t, nd.key, 1);
+        }
+        lid = __shfl_sync(0xffffffffu, lid, 0);
+        // mark sides from the winning segment; child sums of w*y
+        const uint32_t* seg = cbuf + nd.off + (size_t)bf * nd.a;
+        double sl = 0.0, sr = 0.0;
+        for (int j = lane; j < nd.a; j += 32) {
+          const uint32_t lr = seg[j] & 0xffffu;
+          const int sdv = j > bpos;
+          side[lr] = (uint8_t)sdv;
+          if (sdv) sr += wyd[lr];
+          else sl += wyd[lr];
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+          sl += __shfl_down_sync(0xffffffffu, sl, o);
+          sr += __shfl_down_sync(0xffffffffu, sr, o);
+        }
+        if (lane == 0) {
+          const int nr = nd.n - bnl;
+          SRec c;
+          c.feature = -1;
+          c.left = -1;
+          c.pad = 0;
+          c.thr = 0.0;
+          c.drss = 0.0;
+          c.count = bnl;
+          c.value = __ddiv_rn(sl, (double)bnl);
+          recs[lid] = c;
+          c.count = nr;
+          c.value = __ddiv_rn(sr, (double)nr);
+          recs[lid + 1] = c;
+          nd.split = 1;
+          nd.lid = lid;
+          nd.al = bpos + 1;
+          nd.nl = bnl;
+          nd.Sl = bSl;
+          curl[i] = nd;
+        }
+      } else if (lane == 0) {
+        curl[i].split = 0;
+      }
+      __syncwarp();
+    }
+    __syncthreads();
+    // ---- phase B: next-level list and child block offsets (serial, tiny)
+    if (tid == 0) {
+      int nn = 0, off = 0;
+      for (int i = 0; i < ncur; ++i) {
+        SCur& nd = curl[i];
+        nd.coff[0] = nd.coff[1] = -1;
+        if (!nd.split) continue;
+        for (int sdv = 0; sdv < 2; ++sdv) {
+          const int ac = sdv ? nd.a - nd.al : nd.al;
+          const int nc = sdv ? nd.n - nd.nl : nd.nl;
+          if (nc > g.nodesize && ac >= 2) {
+            SCur c;
+            c.off = off;
+            c.a = ac;
+            c.n = nc;
+            c.id = nd.lid + sdv;
+            c.S = sdv ? nd.S - nd.Sl : nd.Sl;
+            c.key = sdv ? nd.keyr : nd.keyl;
+            c.split = 0;
+            nxtl[nn++] = c;
+            nd.coff[sdv] = off;
+            off += p * ac;
+          }
+        }
+      }
+      s_ncur = nn;
+    }
+    __syncthreads();
+    // ---- phase C: stable partition of every feature list of every split node
+    for (int it = wid; it < ncur * p; it += SUB_NW) {
+      const int i = it / p, f = it - i * p;
+      const SCur& nd = curl[i];
+      if (!nd.split || (nd.coff[0] < 0 && nd.coff[1] < 0)) continue;
+      const uint32_t* seg = cbuf + nd.off + (size_t)f * nd.a;
+      const int al = nd.al, ar = nd.a - nd.al;
+      int carry = 0;
+      for (int j0 = 0; j0 < nd.a; j0 += 32) {
+        const int j = j0 + lane;
+        const bool valid = j < nd.a;
+        const uint32_t e = valid ? seg[j] : 0u;
+        const int sdv = valid ? side[e & 0xffffu] : 1;
+        const unsigned m = __ballot_sync(0xffffffffu, valid && sdv == 0);
+        const int lb = carry + __popc(m & ((1u << lane) - 1u));
+        if (valid) {
+          const int co = nd.coff[sdv];
+          if (co >= 0) {
+            const int idx = sdv ? j - lb : lb;
+            nbuf[co + (size_t)f * (sdv ? ar : al) + idx] = e;
+          }
+        }
+        carry += __popc(m);
+      }
+    }
+    __syncthreads();
+    // ---- swap
+    {
+      uint32_t* tb = cbuf;
+      cbuf = nbuf;
+      nbuf = tb;
+      SCur* tl = curl;
+      curl = nxtl;
+      nxtl = tl;
+    }
+    __syncthreads();
+  }
+  // ---- flush the subtree into the tree's raw pool (sibling pairs stay adjacent)
+  if (tid == 0) s_gbase = s_nloc > 1 ? atomicAdd(&g.pool.nn[b], s_nloc - 1) : 0;
+  __syncthreads();
+  const int nloc = s_nloc, gbase = s_gbase;
+  const int64_t r0 = (int64_t)b * g.pool.cap;
+  for (int l = tid; l < nloc; l += SUB_NT) {
+    const SRec r = recs[l];
+    const int64_t gid = r0 + (l == 0 ? root.raw : gbase + l - 1);
+    g.pool.feature[gid] = r.feature;
+    g.pool.left[gid] = r.left >= 0 ? gbase + r.left - 1 : -1;
+    g.pool.thr[gid] = r.thr;
+    g.pool.drss[gid] = r.drss;
+    if (l > 0) {
+      g.pool.count[gid] = r.count;
+      g.pool.value[gid] = r.value;
+    }
+  }
+}
+
+// ------------------------------------------------------------------ a11 emit
+__global__ void k_emit(Pool pool, const int64_t* out_off, Node16* nodes, int32_t* count, double* value,
+                       double* drss) {
+  const int b = blockIdx.y;
+  const int64_t k = blockIdx.x * (int64_t)NT + threadIdx.x;
+  const int32_t nn = pool.nn[b];
+  if (k >= nn) return;
+  const int64_t r = (int64_t)b * pool.cap + k;
+  const int64_t o = out_off[b] + k;
+  Node16 nd;
+  nd.feature = pool.feature[r];
+  nd.left = pool.left[r];
+  nd.v = nd.feature >= 0 ? pool.thr[r] : pool.value[r];
+  nodes[o] = nd;
+  count[o] = pool.count[r];
+  value[o] = pool.value[r];
+  drss[o] = pool.drss[r];
+}
+
+int max_optin_smem() {
+  int dev = 0, v = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+  return v;
+}
+
+template <class T>
+void h2d(T* d, const T* h, size_t cnt, cudaStream_t s) {
+  BF_CUDA_CHECK(cudaMemcpyAsync(d, h, cnt * sizeof(T), cudaMemcpyHostToDevice, s));
+}
+template <class T>
+void d2h(T* h, const T* d, size_t cnt, cudaStream_t s) {
+  BF_CUDA_CHECK(cudaMemcpyAsync(h, d, cnt * sizeof(T), cudaMemcpyDeviceToHost, s));
+}
+
+struct PinnedSummary {
+  LevelSummary* h = nullptr;
+  PinnedSummary() { BF_CUDA_CHECK(cudaMallocHost(&h, sizeof(LevelSummary) * 2)); }
+  ~PinnedSummary() { if (h) cudaFreeHost(h); }
+};
+
+int grid_for(int64_t work) { return (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(work, NT), 148 * 16)); }
+
+}  // namespace
+
+// ================================================================== host entry points
+void fixed_point_impl(const double* y, int64_t n, int64_t ns, int64_t* yq, int32_t* q_out, cudaStream_t s) {
+  const int grid = grid_for(n);
+  DBuf<double> part(2 * (size_t)grid, s);
+  {
+    KScope ks_("k_minmax", s, 0.0);
+    k_minmax<<<grid, NT, 0, s>>>(y, n, part.p);
+  }
+  BF_CUDA_CHECK(cudaGetLastError());
+  std::vector<double> hp(2 * (size_t)grid);
+  d2h(hp.data(), part.p, hp.size(), s);
+  BF_CUDA_CHECK(cudaStreamSynchronize(s));
+  double mn = INFINITY, mx = -INFINITY;
+  for (int i = 0; i < grid; ++i) {
+    mn = std::fmin(mn, hp[2 * i]);
+    mx = std::fmax(mx, hp[2 * i + 1]);
+  }
+  BF_REQUIRE(std::isfinite(mn) && std::isfinite(mx), BF_ENONFINITE, "non-finite y");
+  volatile double h0 = 0.5 * mn, h1 = 0.5 * mx;  // S2: c = RN(RN(0.5 min) + RN(0.5 max))
+  const double c = h0 + h1;
+  {
+    KScope ks_("k_absdev_max", s, 0.0);
+    k_absdev_max<<<grid, NT, 0, s>>>(y, n, c, part.p);
+  }
+  BF_CUDA_CHECK(cudaGetLastError());
+  d2h(hp.data(), part.p, (size_t)grid, s);
+  BF_CUDA_CHECK(cudaStreamSynchronize(s));
+  double R = 0.0;
+  for (int i = 0; i < grid; ++i) R = std::fmax(R, hp[i]);
+  BF_REQUIRE(std::isfinite(R), BF_ERANGE, "y range overflows");
+  int q = 0, zero = 0;
+  if (R == 0.0) {
+    zero = 1;
+  } else {
+    int e = 0;
+    std::frexp(R, &e);
+    int sbits = 0;
+    for (uint64_t v = (uint64_t)ns; v; v >>= 1) ++sbits;
+    q = 62 - sbits - e;
+  }
+  {
+    KScope ks_("k_yq", s, 0.0);
+    k_yq<<<grid, NT, 0, s>>>(y, n, c, q, zero, yq);
+  }
+  BF_CUDA_CHECK(cudaGetLastError());
+  *q_out = q;
+}
+
+void bootstrap_impl(uint64_t seed, int32_t t0, int32_t ntrees, int64_t n, int64_t ns, int32_t replace, int32_t* w,
+                    cudaStream_t s) {
+  if (ntrees <= 0) return;
+  const int64_t tot = n * ntrees;
+  if (!replace) {
+    {
+      KScope ks_("k_fill_i32", s, 0.0);
+      k_fill_i32<<<grid_for(tot), NT, 0, s>>>(w, tot, 1);
+    }
+    BF_CUDA_CHECK(cudaGetLastError());
+    return;
+  }
+  BF_CUDA_CHECK(cudaMemsetAsync(w, 0, sizeof(int32_t) * tot, s));
+  dim3 grid((unsigned)ceil_div(ceil_div(ns, 2), NT), (unsigned)ntrees);
+  {
+    KScope ks_("k_bootstrap", s, 0.0);
+    k_bootstrap<<<grid, NT, 0, s>>>(seed, t0, n, ns, w);
+  }
+  BF_CUDA_CHECK(cudaGetLastError());
+}
+
+void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, int32_t p, const bf_params& prm0,
+              cudaStream_t s, bf_forest** out) {
+  bf_params prm = prm0;
+  BF_REQUIRE(prm.ntree >= 1 && prm.nodesize >= 1, BF_EINVAL, "bf_fit: ntree >= 1 and nodesize >= 1 required");
+  if (prm.tree_begin == 0 && prm.tree_end == 0) prm.tree_end = prm.ntree;
+  BF_REQUIRE(prm.tree_begin >= 0 && prm.tree_end <= prm.ntree && prm.tree_begin <= prm.tree_end, BF_EINVAL,
+             "bf_fit: bad tree range");
+  const int mtry = prm.mtry ? prm.mtry : std::max(p / 3, 1);
+  BF_REQUIRE(mtry >= 1 && mtry <= p, BF_EINVAL, "bf_fit: mtry not in [1, p]");
+  BF_REQUIRE(p <= 32767, BF_ENOTIMPL, "bf_fit: p > 32767");
+  const int64_t ns = prm.sampsize ? prm.sampsize : n;
+  BF_REQUIRE(ns >= 1 && ns < (int64_t(1) << 31), BF_ERANGE, "bf_fit: sampsize out of range");
+  BF_REQUIRE(prm.replace || ns == n, BF_ENOTIMPL, "bf_fit: replace = 0 needs sampsize == n (reading R20)");
+
+  InStage Xs(X_in, sizeof(double) * (size_t)(ldx * (p - 1) + n), s);
+  InStage ys(y_in, sizeof(double) * (size_t)n, s);
+  const double* X = (const double*)Xs.dptr;
+  const double* y = (const double*)ys.dptr;
+
+  // ---- a1 validate
+  {
+    DBuf<int> bad(1, s);
+    BF_CUDA_CHECK(cudaMemsetAsync(bad.p, 0, sizeof(int), s));
+    {
+      KScope ks_("k_validate", s, 0.0);
+      k_validate<<<grid_for(n * p + n), NT, 0, s>>>(X, ldx, n, p, y, bad.p);
+    }
+    BF_CUDA_CHECK(cudaGetLastError());
+    int hb = 0;
+    d2h(&hb, bad.p, 1, s);
+    BF_CUDA_CHECK(cudaStreamSynchronize(s));
+    BF_REQUIRE(hb == 0, BF_ENONFINITE, "bf_fit: NaN/Inf in X or y");
+  }
+  // ---- a2 fixed point
+  DBuf<int64_t> yq(n, s);
+  int32_t q = 0;
+  fixed_point_impl(y, n, ns, yq.p, &q, s);
+
+  // ---- a3 presort
+  DBuf<uint64_t> srt((size_t)p * n, s);
+  DBuf<double> uniq((size_t)p * n, s);
+  {
+    DBuf<uint64_t> k0(n, s), k1(n, s);
+    DBuf<uint32_t> v0(n, s), v1(n, s), fl(n, s), rk(n, s);
+    size_t tb1 = 0, tb2 = 0;
+    cub::DeviceRadixSort::SortPairs(nullptr, tb1, k0.p, k1.p, v0.p, v1.p, (int)n, 0, 64, s);
+    cub::DeviceScan::InclusiveSum(nullptr, tb2, fl.p, rk.p, (int)n, s);
+    DBuf<char> tmp(std::max(tb1, tb2), s);
+    for (int f = 0; f < p; ++f) {
+      const double* col = X + (int64_t)f * ldx;
+      {
+        KScope ks_("k_sort_keys", s, 0.0);
+        k_sort_keys<<<grid_for(n), NT, 0, s>>>(col, n, k0.p, v0.p);
+      }
+      size_t t1 = tb1;
+      {
+        KScope ks_("cub_SortPairs", s, 0.0);
+        BF_CUDA_CHECK(cub::DeviceRadixSort::SortPairs(tmp.p, t1, k0.p, k1.p, v0.p, v1.p, (int)n, 0, 64, s));
+      }
+      {
+        KScope ks_("k_rank_flags", s, 0.0);
+        k_rank_flags<<<grid_for(n), NT, 0, s>>>(k1.p, n, fl.p);
+      }
+      size_t t2 = tb2;
+      {
+        KScope ks_("cub_InclusiveSum", s, 0.0);
+        BF_CUDA_CHECK(cub::DeviceScan::InclusiveSum(tmp.p, t2, fl.p, rk.p, (int)n, s));
+      }
+      {
+        KScope ks_("k_fill_sorted", s, 0.0);
+        k_fill_sorted<<<grid_for(n), NT, 0, s>>>(col, v1.p, rk.p, n, srt.p + (int64_t)f * n, uniq.p + (int64_t)f * n);
+      }
+      BF_CUDA_CHECK(cudaGetLastError());
+    }
+  }
+
+  // ---- sizing: subtree capacity A and trees in flight B
+  const int smax = max_optin_smem();
+  int A = 2;
+  while (A < 4096 && subtree_smem(A + 1, p) <= (size_t)smax) ++A;
+  BF_REQUIRE(subtree_smem(2, p) <= (size_t)smax, BF_ENOTIMPL, "bf_fit: p too large for the shared-memory subtree kernel");
+  if (prm.small_node_max > 0) A = std::max(2, std::min(A, prm.small_node_max));
+  BF_CUDA_CHECK(cudaFuncSetAttribute(k_subtree, cudaFuncAttributeMaxDynamicSharedMemorySize, smax));
+
+  const int32_t T_loc = prm.tree_end - prm.tree_begin;
+  const int64_t cap_nodes = 2 * n + 1;
+  const size_t per_tree = (size_t)3 * p * n * 8 + (size_t)n * (4 + 16 + 1 + 2) +
+                          (size_t)cap_nodes * (4 + 4 + 4 + 8 + 8 + 8) + (size_t)n * 48 / 2;
+  int B = prm.trees_in_flight;
+  if (B <= 0) {
+    size_t fr = 0, tot = 0;
+    BF_CUDA_CHECK(cudaMemGetInfo(&fr, &tot));
+    const size_t budget = fr / 2;
+    B = (int)std::max<size_t>(1, std::min<size_t>(budget / std::max<size_t>(per_tree, 1), 256));
+  }
+  B = std::max(1, std::min(B, std::max(T_loc, 1)));
+
+  bf_forest* F = new bf_forest();
+  F->info.n = n;
+  F->info.p = p;
+  F->info.ntree_total = prm.ntree;
+  F->info.tree_begin = prm.tree_begin;
+  F->info.tree_end = prm.tree_end;
+  F->info.q = q;
+  F->info.mtry = mtry;
+  F->info.nodesize = prm.nodesize;
+  F->info.replace = prm.replace;
+  F->info.sampsize = ns;
+  F->info.seed = prm.seed;
+  cudaGetDevice(&F->device);
+  F->tree_off.assign((size_t)T_loc + 1, 0);
+
+  struct Chunk {
+    DBuf<Node16> nodes;
+    DBuf<int32_t> count;
+    DBuf<double> value, drss;
+    int64_t total = 0;
+  };
+  std::vector<Chunk> chunks;
+
+  try {
+    // ---- batch buffers
+    DBuf<int32_t> w((size_t)B * n, s);
+    DBuf<Pay> pay((size_t)B * n, s);
+    DBuf<uint8_t> side((size_t)B * n, s);
+    DBuf<uint16_t> loc((size_t)B * n, s);
+    DBuf<int32_t> pf((size_t)B * cap_nodes, s), pl((size_t)B * cap_nodes, s), pc((size_t)B * cap_nodes, s),
+        pnn(B, s);
+    DBuf<double> pt((size_t)B * cap_nodes, s), pv((size_t)B * cap_nodes, s), pd((size_t)B * cap_nodes, s);
+    Pool pool{pf.p, pl.p, pc.p, pt.p, pv.p, pd.p, pnn.p, cap_nodes};
+    DBuf<int32_t> a_root(B, s), kind_d(B, s), lidx_d(B, s), sidx_d(B, s);
+    DBuf<unsigned long long> S_root(B, s);
+    DBuf<double> sy_root(B, s);
+    DBuf<int64_t> base_d(B, s), emit_off(B, s);
+    const int64_t cap_level = (int64_t)B * n / (A + 1) + B + 1;
+    const int64_t cap_small = (int64_t)B * n / 2 + B + 1;
+    DBuf<LNode> ncur(cap_level, s), nnext(cap_level, s), sq(cap_small, s);
+    DBuf<int32_t> feat(cap_level * mtry, s);
+    DBuf<int16_t> fyscr(cap_level * p, s);
+    DBuf<Rec> rec(cap_level * mtry, s);
+    DBuf<Split> split(cap_level, s);
+    DBuf<Child> child(2 * cap_level, s);
+    DBuf<uint64_t> packL(2 * cap_level, s), packS(2 * cap_level, s), scanL(2 * cap_level, s), scanS(2 * cap_level, s);
+    size_t scan_tb = 0;
+    cub::DeviceScan::ExclusiveSum(nullptr, scan_tb, packL.p, scanL.p, (int)(2 * cap_level), s);
+    DBuf<char> scan_tmp(std::max<size_t>(scan_tb, 16), s);
+    DBuf<LevelSummary> dsum(1, s);
+    PinnedSummary hs;
+    DBuf<uint64_t> E0, E1, Es;
+    size_t E_cap = 0;
+
+    for (int tb = prm.tree_begin; tb < prm.tree_end; tb += B) {
+      const int Bc = std::min(B, prm.tree_end - tb);
+      // ---- a4 bootstrap + payload + root sums
+      bootstrap_impl(prm.seed, tb, Bc, n, ns, prm.replace, w.p, s);
+      BF_CUDA_CHECK(cudaMemsetAsync(a_root.p, 0, sizeof(int32_t) * Bc, s));
+      BF_CUDA_CHECK(cudaMemsetAsync(S_root.p, 0, sizeof(unsigned long long) * Bc, s));
+      BF_CUDA_CHECK(cudaMemsetAsync(sy_root.p, 0, sizeof(double) * Bc, s));
+      {
+        KScope ks_("k_payload", s, 0.0);
+        k_payload<<<dim3((unsigned)ceil_div(n, NT), Bc), NT, 0, s>>>(w.p, yq.p, y, n, pay.p, a_root.p, S_root.p,
+                                                                    sy_root.p);
+      }
+      BF_CUDA_CHECK(cudaGetLastError());
+      std::vector<int32_t> ha(Bc), hk(Bc), hl(Bc), hsx(Bc);
+      std::vector<int64_t> hbase(Bc);
+      d2h(ha.data(), a_root.p, Bc, s);
+      BF_CUDA_CHECK(cudaStreamSynchronize(s));
+      int64_t offL = 0, offS = 0;
+      int nL = 0, nS = 0;
+      for (int b = 0; b < Bc; ++b) {
+        hl[b] = hsx[b] = -1;
+        hbase[b] = 0;
+        if (ns <= prm.nodesize || ha[b] < 2) {
+          hk[b] = KIND_LEAF;
+        } else if (ha[b] <= A) {
+          hk[b] = KIND_SMALL;
+          hbase[b] = offS;
+          offS += (int64_t)p * ha[b];
+          hsx[b] = nS++;
+        } else {
+          hk[b] = KIND_LARGE;
+          hbase[b] = offL;
+          offL += (int64_t)p * ha[b];
+          hl[b] = nL++;
+        }
+      }
+      // total entries of the batch: every level and the small area fit in sum_b p * a_b
+      size_t need = 0;
+      for (int b = 0; b < Bc; ++b) need += (size_t)p * ha[b];
+      need = std::max<size_t>(need, 1);
+      if (need > E_cap) {
+        E0.alloc(need, s);
+        E1.alloc(need, s);
+        Es.alloc(need, s);
+        E_cap = need;
+      }
+      h2d(kind_d.p, hk.data(), Bc, s);
+      h2d(lidx_d.p, hl.data(), Bc, s);
+      h2d(sidx_d.p, hsx.data(), Bc, s);
+      h2d(base_d.p, hbase.data(), Bc, s);
+      {
+        KScope ks_("k_roots", s, 0.0);
+        k_roots<<<(unsigned)ceil_div(Bc, 128), 128, 0, s>>>(Bc, ns, prm.nodesize, a_root.p, S_root.p, sy_root.p,
+                                                            kind_d.p, base_d.p, pool, ncur.p, lidx_d.p, sq.p, sidx_d.p);
+      }
+      BF_CUDA_CHECK(cudaGetLastError());
+      // ---- a5 root lists
+      {
+        const int nchunk = (int)ceil_div(n, LCH);
+        DBuf<int32_t> cnt((size_t)Bc * p * nchunk, s);
+        dim3 grid((unsigned)nchunk, (unsigned)p, (unsigned)Bc);
+        {
+          KScope ks_("k_list_count", s, 0.0);
+          k_list_count<<<grid, NT, 0, s>>>(srt.p, n, pay.p, kind_d.p, nchunk, cnt.p);
+        }
+        {
+          KScope ks_("k_list_prefix", s, 0.0);
+          k_list_prefix<<<(unsigned)ceil_div((int64_t)Bc * p, 128), 128, 0, s>>>(cnt.p, Bc * p, nchunk);
+        }
+        {
+          KScope ks_("k_list_scatter", s, 0.0);
+          k_list_scatter<<<grid, NT, 0, s>>>(srt.p, n, pay.p, kind_d.p, base_d.p, a_root.p, nchunk, cnt.p, E0.p, Es.p);
+        }
+        BF_CUDA_CHECK(cudaGetLastError());
+        prof_add_bytes("k_list_scatter", (double)Bc * n * p * 8.0 + (double)(offL + offS) * 8.0);
+      }
+      LevelSummary ls{};
+      ls.nnext = nL;
+      ls.nsmall = nS;
+      ls.small_elems = offS;
+      ls.next_elems = offL;
+      h2d(dsum.p, &ls, 1, s);
+      // ---- global phase
+      int N = nL;
+      int64_t cur_elems = offL;
+      uint64_t* Ec = E0.p;
+      uint64_t* En = E1.p;
+      LNode* nc = ncur.p;
+      LNode* nx = nnext.p;
+      while (N > 0) {
+        {
+          KScope ks_("k_mtry", s, 0.0);
+          k_mtry<<<(unsigned)ceil_div(N, 128), 128, 0, s>>>(nc, N, p, mtry, prm.seed, tb, feat.p, fyscr.p);
+        }
+        {
+          KScope ks_("k_split_scan", s, 0.0);
+          k_split_scan<<<(unsigned)((int64_t)N * mtry), NT, 0, s>>>(nc, feat.p, mtry, Ec, pay.p, n, rec.p);
+        }
+        {
+          KScope ks_("k_finalize", s, 0.0);
+          k_finalize<<<(unsigned)ceil_div(N, 128), 128, 0, s>>>(nc, N, feat.p, rec.p, mtry, uniq.p, n, prm.nodesize, A,
+                                                               q, prm.seed, tb, pool, split.p, child.p, packL.p, packS.p, dsum.p);
+        }
+        BF_CUDA_CHECK(cudaGetLastError());
+        const int N2 = 2 * N;
+        size_t t1 = scan_tb;
+        {
+          KScope ks_("cub_ExclusiveSum", s, 0.0);
+          BF_CUDA_CHECK(cub::DeviceScan::ExclusiveSum(scan_tmp.p, t1, packL.p, scanL.p, N2, s));
+        }
+        t1 = scan_tb;
+        {
+          KScope ks_("cub_ExclusiveSum", s, 0.0);
+          BF_CUDA_CHECK(cub::DeviceScan::ExclusiveSum(scan_tmp.p, t1, packS.p, scanS.p, N2, s));
+        }
+        {
+          KScope ks_("k_child_place", s, 0.0);
+          k_child_place<<<(unsigned)ceil_div(N2, 128), 128, 0, s>>>(N2, p, nc, child.p, scanL.p, scanS.p, nx, sq.p,
+                                                                    dsum.p);
+        }
+        {
+          KScope ks_("k_dest", s, 0.0);
+          k_dest<<<(unsigned)N, NT, 0, s>>>(nc, split.p, Ec, pay.p, y, n, side.p, pool);
+        }
+        {
+          KScope ks_("k_partition", 0, 0.0);
+          k_partition<<<dim3((unsigned)N, (unsigned)p), NT, 0, s>>>(nc, split.p, child.p, p, Ec, side.p, n, En, Es.p);
+        }
+        {
+          KScope ks_("k_commit", s, 0.0);
+          k_commit<<<1, 1, 0, s>>>(N2, packL.p, scanL.p, packS.p, scanS.p, p, dsum.p, hs.h);
+        }
+        BF_CUDA_CHECK(cudaGetLastError());
+        BF_CUDA_CHECK(cudaStreamSynchronize(s));
+        {  // algorithmic bytes
+          const double cur_a = (double)cur_elems / p, sa = (double)hs.h->split_a;
+          prof_add_bytes("k_split_scan", cur_a * mtry * 20.0);
+          prof_add_bytes("k_dest", sa * 21.0);
+          prof_add_bytes("k_partition", sa * p * 17.0);
+        }
+        cur_elems = hs.h->next_elems;
+        N = hs.h->nnext;
+        std::swap(Ec, En);
+        std::swap(nc, nx);
+      }
+      // ---- subtree phase
+      {
+        d2h(&ls, dsum.p, 1, s);
+        BF_CUDA_CHECK(cudaStreamSynchronize(s));
+        if (ls.nsmall > 0) {
+          prof_add_bytes("k_subtree", (double)ls.small_elems * 8.0 + (double)ls.small_elems / p * 26.0);
+          SubArgs ga;
+          ga.sq = sq.p;
+          ga.Es = Es.p;
+          ga.pay = pay.p;
+          ga.y = y;
+          ga.X = X;
+          ga.ldx = ldx;
+          ga.n = n;
+          ga.p = p;
+          ga.mtry = mtry;
+          ga.nodesize = prm.nodesize;
+          ga.q = q;
+          ga.A = A;
+          ga.seed = prm.seed;
+          ga.t0 = tb;
+          ga.loc = loc.p;
+          ga.pool = pool;
+          {
+            KScope ks_("k_subtree", s, 0.0);
+            k_subtree<<<(unsigned)ls.nsmall, SUB_NT, subtree_smem(A, p), s>>>(ga);
+          }
+          BF_CUDA_CHECK(cudaGetLastError());
+        }
+      }
+      // ---- a11 emit
+      std::vector<int32_t> hnn(Bc);
+      d2h(hnn.data(), pnn.p, Bc, s);
+      BF_CUDA_CHECK(cudaStreamSynchronize(s));
+      std::vector<int64_t> hoff(Bc);
+      int64_t tot = 0;
+      int32_t mx = 0;
+      for (int b = 0; b < Bc; ++b) {
+        hoff[b] = tot;
+        tot += hnn[b];
+        mx = std::max(mx, hnn[b]);
+        F->tree_off[(size_t)(tb - prm.tree_begin + b) + 1] = hnn[b];
+      }
+      Chunk ch;
+      ch.total = tot;
+      ch.nodes.alloc(tot, s);
+      ch.count.alloc(tot, s);
+      ch.value.alloc(tot, s);
+      ch.drss.alloc(tot, s);
+      h2d(emit_off.p, hoff.data(), Bc, s);
+      {
+        KScope ks_("k_emit", s, 0.0);
+        k_emit<<<dim3((unsigned)ceil_div(mx, NT), Bc), NT, 0, s>>>(pool, emit_off.p, ch.nodes.p, ch.count.p,
+                                                                  ch.value.p, ch.drss.p);
+      }
+      BF_CUDA_CHECK(cudaGetLastError());
+      chunks.push_back(std::move(ch));
+    }
+    // ---- assemble the forest
+    for (int32_t i = 0; i < T_loc; ++i) F->tree_off[i + 1] += F->tree_off[i];
+    const int64_t total = F->tree_off[T_loc];
+    forest_alloc(F, total, T_loc, s);
+    h2d(F->d_tree_off, F->tree_off.data(), (size_t)T_loc + 1, s);
+    int64_t o = 0;
+    for (auto& ch : chunks) {
+      if (ch.total) {
+        BF_CUDA_CHECK(cudaMemcpyAsync(F->d_nodes + o, ch.nodes.p, ch.total * sizeof(Node16), cudaMemcpyDeviceToDevice, s));
+        BF_CUDA_CHECK(cudaMemcpyAsync(F->d_count + o, ch.count.p, ch.total * 4, cudaMemcpyDeviceToDevice, s));
+        BF_CUDA_CHECK(cudaMemcpyAsync(F->d_value + o, ch.value.p, ch.total * 8, cudaMemcpyDeviceToDevice, s));
+        BF_CUDA_CHECK(cudaMemcpyAsync(F->d_drss + o, ch.drss.p, ch.total * 8, cudaMemcpyDeviceToDevice, s));
+      }
+      o += ch.total;
+    }
+    chunks.clear();
+    BF_CUDA_CHECK(cudaStreamSynchronize(s));
+  } catch (...) {
+    forest_release(F);
+    delete F;
+    throw;
+  }
+  *out = F;
+}
+
+}  // namespace bf

@@ -1,0 +1,406 @@
+// importance.cu -- OOB prediction and permutation importance (SURVEY 8(a)
+// rows a13-a15; S6-S8).
+//
+// Per batch of trees: regenerate the bootstrap (Philox BOOT, identical to
+// the fit), compact each tree's OOB rows in ascending order, then one thread
+// per (tree, OOB row a):
+//   * walk the tree -> f_t(x_a); accumulate e_t, oob_sum, oob_cnt;
+//   * for every predictor m tested on that path (first occurrence only) walk
+//     again from that node with x_m replaced by x_{O_t[pi_tm(a)], m}.  A path
+//     that does not test m gives the same leaf, so its contribution to
+//     e_tm - e_t is exactly zero and is skipped; predictors never used by the
+//     tree get d_tm = 0 exactly (S7).
+#include <algorithm>
+
+#include "bf_internal.cuh"
+
+namespace bf {
+namespace {
+
+constexpr int NT = 256;
+constexpr int OCH = 4096;  // rows per CTA chunk in the OOB compaction
+
+__device__ __forceinline__ Node16 ld_node(const Node16* p) {
+  const int4 v = __ldg(reinterpret_cast<const int4*>(p));
+  Node16 n;
+  n.v = __hiloint2double(v.y, v.x);
+  n.feature = v.z;
+  n.left = v.w;
+  return n;
+}
+
+// S7 Feistel permutation pi_tm on [0, n_o) with cycle walking.
+__device__ __forceinline__ int64_t feistel(uint64_t seed, uint32_t t, uint32_t m, int64_t n_o, int64_t a) {
+  int b = 64 - __clzll((unsigned long long)(n_o - 1));  // ceil(log2 n_o) for n_o >= 2; 0 for n_o == 1
+  if (n_o <= 1) b = 0;
+  if (b < 2) b = 2;
+  b += b & 1;
+  const int h = b >> 1;
+  const uint32_t mask = (uint32_t)((1ull << h) - 1ull);
+  uint64_t v = (uint64_t)a;
+  do {
+    uint32_t L = (uint32_t)(v >> h), R = (uint32_t)(v & mask);
+#pragma unroll 1
+    for (uint32_t r = 0; r < 6; ++r) {
+      uint32_t x[4];
+      philox4x32_10(R, r, 3u | (m << 8), t, (uint32_t)seed, (uint32_t)(seed >> 32), x);
+      const uint32_t nR = L ^ (x[0] & mask);
+      L = R;
+      R = nR;
+    }
+    v = ((uint64_t)L << h) | R;
+  } while ((int64_t)v >= n_o);
+  return (int64_t)v;
+}
+
+__global__ void k_perm(uint64_t seed, int32_t t, int32_t m, int64_t n_o, int64_t* out) {
+  const int64_t a = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (a < n_o) out[a] = feistel(seed, (uint32_t)t, (uint32_t)m, n_o, a);
+}
+
+__global__ void k_oob_count(const int32_t* w, int64_t n, int nchunk, int32_t* cnt) {
+  __shared__ int32_t sm[NT / 32];
+  const int c = blockIdx.x, b = blockIdx.y;
+  int32_t k = 0;
+  for (int u = threadIdx.x; u < OCH; u += NT) {
+    const int64_t i = (int64_t)c * OCH + u;
+    if (i < n) k += w[(int64_t)b * n + i] == 0;
+  }
+  for (int o = 16; o > 0; o >>= 1) k += __shfl_down_sync(0xffffffffu, k, o);
+  if ((threadIdx.x & 31) == 0) sm[threadIdx.x >> 5] = k;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    int32_t s = 0;
+    for (int j = 0; j < NT / 32; ++j) s += sm[j];
+    cnt[(int64_t)b * nchunk + c] = s;
+  }
+}
+
+__global__ void k_oob_prefix(int32_t* cnt, int B, int nchunk, int64_t* nout) {
+  const int b = blockIdx.x * blockDim.x + threadIdx.x;
+  if (b >= B) return;
+  int32_t acc = 0;
+  for (int c = 0; c < nchunk; ++c) {
+    const int32_t v = cnt[(int64_t)b * nchunk + c];
+    cnt[(int64_t)b * nchunk + c] = acc;
+    acc += v;
+  }
+  nout[b] = acc;
+}
+
+__global__ void k_oob_scatter(const int32_t* w, int64_t n, int nchunk, const int32_t* cnt, uint32_t* O) {
+  __shared__ int32_t sm[NT / 32];
+  const int c = blockIdx.x, b = blockIdx.y;
+  constexpr int V = OCH / NT;
+  const int64_t i0 = (int64_t)c * OCH + (int64_t)threadIdx.x * V;
+  bool keep[V];
+  int32_t k = 0;
+#pragma unroll
+  for (int u = 0; u < V; ++u) {
+    keep[u] = (i0 + u < n) && w[(int64_t)b * n + i0 + u] == 0;
+    k += keep[u];
+  }
+  // block exclusive scan
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  int32_t inc = k;
+  for (int o = 1; o < 32; o <<= 1) {
+    const int32_t v = __shfl_up_sync(0xffffffffu, inc, o);
+    if (lane >= o) inc += v;
+  }
+  if (lane == 31) sm[wid] = inc;
+  __syncthreads();
+  if (threadIdx.x == 0)
+    for (int j = 1; j < NT / 32; ++j) sm[j] += sm[j - 1];
+  __syncthreads();
+  int32_t pre = inc - k + (wid ? sm[wid - 1] : 0) + cnt[(int64_t)b * nchunk + c];
+  uint32_t* Ob = O + (int64_t)b * n;
+#pragma unroll
+  for (int u = 0; u < V; ++u)
+    if (keep[u]) Ob[pre++] = (uint32_t)(i0 + u);
+}
+
+// IncNodePurity slots: sum of drss of splits on m, per local tree.
+__global__ void k_npur(const Node16* nodes, const double* drss, const int64_t* off, int32_t i0, int p, double* npur) {
+  const int b = blockIdx.y;
+  const int32_t i = i0 + b;
+  const int64_t lo = off[i], hi = off[i + 1];
+  for (int64_t k = lo + blockIdx.x * (int64_t)NT + threadIdx.x; k < hi; k += (int64_t)gridDim.x * NT) {
+    const int f = nodes[k].feature;
+    if (f >= 0) atomicAdd(&npur[(int64_t)i * p + f], drss[k]);
+  }
+}
+
+struct ImpArgs {
+  const Node16* nodes;
+  const int64_t* off;
+  const double* X;
+  int64_t ldx;
+  const double* y;
+  int64_t n;
+  int p;
+  uint64_t seed;
+  int32_t tree_begin;  // global id of local tree 0
+  int32_t i0;          // local index of batch tree 0
+  const uint32_t* O;   // batch OOB lists, stride n
+  const int64_t* nout; // batch OOB counts
+  double* d_slots;     // local tree slots
+  double* oob_sum;
+  int32_t* oob_cnt;
+  double* e_t;
+};
+
+__global__ void __launch_bounds__(NT) k_importance(ImpArgs g) {
+  extern __shared__ double sacc[];  // p partial sums of (e_tm - e_t) for this CTA's tree
+  __shared__ double serr[NT / 32];
+  const int b = blockIdx.y;
+  const int32_t i = g.i0 + b;
+  const uint32_t t = (uint32_t)(g.tree_begin + i);
+  for (int m = threadIdx.x; m < g.p; m += NT) sacc[m] = 0.0;
+  __syncthreads();
+  const int64_t n_o = g.nout[b];
+  const int64_t a = blockIdx.x * (int64_t)NT + threadIdx.x;
+  double err0 = 0.0;
+  if (a < n_o) {
+    const uint32_t* Ob = g.O + (int64_t)b * g.n;
+    const uint32_t r = Ob[a];
+    const Node16* tn = g.nodes + g.off[i];
+    const double yr = g.y[r];
+    // original walk
+    Node16 nd = ld_node(tn);
+    while (nd.feature >= 0) nd = ld_node(tn + (g.X[(int64_t)nd.feature * g.ldx + r] <= nd.v ? nd.left : nd.left + 1));
+    const double f0 = nd.v;
+    const double d0 = yr - f0;
+    err0 = d0 * d0;
+    atomicAdd(&g.oob_sum[r], f0);
+    atomicAdd(&g.oob_cnt[r], 1);
+    // permuted walks: first occurrence of each predictor on the path
+    uint64_t seen = 0;
+    int k = 0;
+    nd = ld_node(tn);
+    int depth = 0;
+    while (nd.feature >= 0) {
+      const int m = nd.feature;
+      bool first = !((seen >> (m & 63)) & 1ull);
+      if (!first && g.p > 64) {  // bitmask collision possible: verify on the path prefix
+        first = true;
+        int kk = 0;
+        for (int d = 0; d < depth; ++d) {
+          const Node16 q = ld_node(tn + kk);
+          if (q.feature == m) { first = false; break; }
+          kk = g.X[(int64_t)q.feature * g.ldx + r] <= q.v ? q.left : q.left + 1;
+        }
+      }
+      seen |= 1ull << (m & 63);
+      if (first) {
+        const int64_t pa = feistel(g.seed, t, (uint32_t)m, n_o, a);
+        const double xm = g.X[(int64_t)m * g.ldx + Ob[pa]];
+        Node16 q = nd;
+        while (q.feature >= 0) {
+          const double xv = q.feature == m ? xm : g.X[(int64_t)q.feature * g.ldx + r];
+          q = ld_node(tn + (xv <= q.v ? q.left : q.left + 1));
+        }
+        const double d1 = yr - q.v;
+        const double diff = d1 * d1 - err0;
+        if (diff != 0.0) atomicAdd(&sacc[m], diff);
+      }
+      k = g.X[(int64_t)m * g.ldx + r] <= nd.v ? nd.left : nd.left + 1;
+      nd = ld_node(tn + k);
+      ++depth;
+    }
+  }
+  // e_t
+  for (int o = 16; o > 0; o >>= 1) err0 += __shfl_down_sync(0xffffffffu, err0, o);
+  if ((threadIdx.x & 31) == 0) serr[threadIdx.x >> 5] = err0;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double s = 0.0;
+    for (int j = 0; j < NT / 32; ++j) s += serr[j];
+    if (s != 0.0) atomicAdd(&g.e_t[i], s);
+  }
+  for (int m = threadIdx.x; m < g.p; m += NT)
+    if (sacc[m] != 0.0) atomicAdd(&g.d_slots[(int64_t)i * g.p + m], sacc[m]);
+}
+
+__global__ void k_divide(double* d_slots, const int64_t* nout_t, int32_t T, int p) {
+  const int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (k >= (int64_t)T * p) return;
+  const int64_t no = nout_t[k / p];
+  d_slots[k] = no > 0 ? d_slots[k] / (double)no : 0.0;
+}
+
+// S6-S8 aggregation (one CTA; fixed reduction order -> deterministic).
+__global__ void k_finalize_imp(const double* d, const double* npur, const double* oob_sum, const int32_t* oob_cnt,
+                               const double* y, int64_t n, int p, int32_t T, double* o4, double* o2) {
+  __shared__ double s1[NT], s2[NT];
+  __shared__ long long sc[NT];
+  for (int m = threadIdx.x; m < p; m += NT) {
+    double raw = 0.0;
+    for (int32_t t = 0; t < T; ++t) raw += d[(int64_t)t * p + m];
+    raw /= (double)T;
+    double v = 0.0;
+    for (int32_t t = 0; t < T; ++t) {
+      const double e = d[(int64_t)t * p + m] - raw;
+      v += e * e;
+    }
+    v /= (double)T;
+    const double sd = sqrt(v / (double)T);
+    double np = 0.0;
+    for (int32_t t = 0; t < T; ++t) np += npur[(int64_t)t * p + m];
+    o4[m] = sd >= 2.220446049250313e-16 ? raw / sd : raw;
+    o4[p + m] = raw;
+    o4[2 * p + m] = sd;
+    o4[3 * p + m] = np / (double)T;
+  }
+  double se = 0.0, sy = 0.0;
+  long long cnt = 0;
+  for (int64_t r = threadIdx.x; r < n; r += NT) {
+    sy += y[r];
+    if (oob_cnt[r] > 0) {
+      const double e = y[r] - oob_sum[r] / (double)oob_cnt[r];
+      se += e * e;
+      ++cnt;
+    }
+  }
+  s1[threadIdx.x] = se;
+  s2[threadIdx.x] = sy;
+  sc[threadIdx.x] = cnt;
+  __syncthreads();
+  for (int s = NT / 2; s > 0; s >>= 1) {
+    if (threadIdx.x < s) {
+      s1[threadIdx.x] += s1[threadIdx.x + s];
+      s2[threadIdx.x] += s2[threadIdx.x + s];
+      sc[threadIdx.x] += sc[threadIdx.x + s];
+    }
+    __syncthreads();
+  }
+  const double mse = sc[0] ? s1[0] / (double)sc[0] : 0.0;
+  const double mean = s2[0] / (double)n;
+  __syncthreads();
+  double sv = 0.0;
+  for (int64_t r = threadIdx.x; r < n; r += NT) {
+    const double e = y[r] - mean;
+    sv += e * e;
+  }
+  s1[threadIdx.x] = sv;
+  __syncthreads();
+  for (int s = NT / 2; s > 0; s >>= 1) {
+    if (threadIdx.x < s) s1[threadIdx.x] += s1[threadIdx.x + s];
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    const double var = s1[0] / (double)n;
+    o2[0] = mse;
+    o2[1] = var > 0.0 ? 1.0 - mse / var : 0.0;
+  }
+}
+
+}  // namespace
+
+void perm_impl(uint64_t seed, int32_t t, int32_t m, int64_t n_o, int64_t* out, cudaStream_t s) {
+  {
+    KScope ks_("k_perm", s, 0.0);
+    k_perm<<<(unsigned)ceil_div(n_o, NT), NT, 0, s>>>(seed, t, m, n_o, out);
+  }
+  BF_CUDA_CHECK(cudaGetLastError());
+}
+
+void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, const double* y_in, int64_t n, int32_t p,
+                         const bf_oob_accum& acc, cudaStream_t s) {
+  const int32_t T = f->info.tree_end - f->info.tree_begin;
+  InStage Xs(X_in, sizeof(double) * (size_t)(ldx * (p - 1) + n), s);
+  InStage ys(y_in, sizeof(double) * (size_t)n, s);
+  const double* X = (const double*)Xs.dptr;
+  const double* y = (const double*)ys.dptr;
+  OutStage d_s(acc.d_slots, sizeof(double) * (size_t)T * p, s), np_s(acc.npur_slots, sizeof(double) * (size_t)T * p, s),
+      os_s(acc.oob_sum, sizeof(double) * n, s), oc_s(acc.oob_cnt, sizeof(int32_t) * n, s),
+      et_s(acc.e_t, sizeof(double) * (size_t)std::max(T, 1), s), no_s(acc.nout_t, sizeof(int64_t) * (size_t)std::max(T, 1), s);
+  double* d_slots = (double*)d_s.dptr;
+  double* npur = (double*)np_s.dptr;
+  double* oob_sum = (double*)os_s.dptr;
+  int32_t* oob_cnt = (int32_t*)oc_s.dptr;
+  double* e_t = (double*)et_s.dptr;
+  int64_t* nout_t = (int64_t*)no_s.dptr;
+  if (T > 0) {
+    BF_CUDA_CHECK(cudaMemsetAsync(d_slots, 0, sizeof(double) * (size_t)T * p, s));
+    BF_CUDA_CHECK(cudaMemsetAsync(npur, 0, sizeof(double) * (size_t)T * p, s));
+    BF_CUDA_CHECK(cudaMemsetAsync(e_t, 0, sizeof(double) * T, s));
+  }
+  BF_CUDA_CHECK(cudaMemsetAsync(oob_sum, 0, sizeof(double) * n, s));
+  BF_CUDA_CHECK(cudaMemsetAsync(oob_cnt, 0, sizeof(int32_t) * n, s));
+  const int B = std::max(1, std::min<int>(T, 64));
+  const int nchunk = (int)ceil_div(n, OCH);
+  DBuf<int32_t> w((size_t)B * n, s), cnt((size_t)B * nchunk, s);
+  DBuf<uint32_t> O((size_t)B * n, s);
+  const size_t smem = sizeof(double) * (size_t)p;
+  if (smem > 48 * 1024) BF_CUDA_CHECK(cudaFuncSetAttribute(k_importance, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  for (int32_t i0 = 0; i0 < T; i0 += B) {
+    const int Bc = std::min(B, T - i0);
+    bootstrap_impl(f->info.seed, f->info.tree_begin + i0, Bc, n, f->info.sampsize, f->info.replace, w.p, s);
+    {
+      KScope ks_("k_oob_count", s, 0.0);
+      k_oob_count<<<dim3(nchunk, Bc), NT, 0, s>>>(w.p, n, nchunk, cnt.p);
+    }
+    {
+      KScope ks_("k_oob_prefix", s, 0.0);
+      k_oob_prefix<<<(unsigned)ceil_div(Bc, 64), 64, 0, s>>>(cnt.p, Bc, nchunk, nout_t + i0);
+    }
+    {
+      KScope ks_("k_oob_scatter", s, 0.0);
+      k_oob_scatter<<<dim3(nchunk, Bc), NT, 0, s>>>(w.p, n, nchunk, cnt.p, O.p);
+    }
+    {
+      KScope ks_("k_npur", s, 0.0);
+      k_npur<<<dim3(64, Bc), NT, 0, s>>>(f->d_nodes, f->d_drss, f->d_tree_off, i0, p, npur);
+    }
+    BF_CUDA_CHECK(cudaGetLastError());
+    ImpArgs g;
+    g.nodes = f->d_nodes;
+    g.off = f->d_tree_off;
+    g.X = X;
+    g.ldx = ldx;
+    g.y = y;
+    g.n = n;
+    g.p = p;
+    g.seed = f->info.seed;
+    g.tree_begin = f->info.tree_begin;
+    g.i0 = i0;
+    g.O = O.p;
+    g.nout = nout_t + i0;
+    g.d_slots = d_slots;
+    g.oob_sum = oob_sum;
+    g.oob_cnt = oob_cnt;
+    g.e_t = e_t;
+    // OOB rows per tree <= n; grid sized for n (CTAs past n_o exit early)
+    {
+      KScope ks_("k_importance", s, 0.0);
+      k_importance<<<dim3((unsigned)ceil_div(n, NT), Bc), NT, smem, s>>>(g);
+    }
+    BF_CUDA_CHECK(cudaGetLastError());
+  }
+  if (T > 0) {
+    {
+      KScope ks_("k_divide", s, 0.0);
+      k_divide<<<(unsigned)ceil_div((int64_t)T * p, NT), NT, 0, s>>>(d_slots, nout_t, T, p);
+    }
+    BF_CUDA_CHECK(cudaGetLastError());
+  }
+  d_s.finish(s);
+  np_s.finish(s);
+  os_s.finish(s);
+  oc_s.finish(s);
+  et_s.finish(s);
+  no_s.finish(s);
+  BF_CUDA_CHECK(cudaStreamSynchronize(s));
+}
+
+void importance_finalize_impl(const double* d_slots, const double* npur_slots, const double* oob_sum,
+                              const int32_t* oob_cnt, const double* y, int64_t n, int32_t p, int32_t ntree,
+                              double* o4, double* o2, cudaStream_t s) {
+  {
+    KScope ks_("k_finalize_imp", s, 0.0);
+    k_finalize_imp<<<1, NT, 0, s>>>(d_slots, npur_slots, oob_sum, oob_cnt, y, n, p, ntree, o4, o2);
+  }
+  BF_CUDA_CHECK(cudaGetLastError());
+}
+
+}  // namespace bf

@@ -1,0 +1,130 @@
+// predict.cu -- batched forest prediction (P:95 step 3, S5).
+//
+// One thread per query row; a CTA stages its rows' predictors in shared
+// memory row-major (coalesced column loads), then every thread walks all the
+// forest's trees in tree order (16-byte node loads through the read-only
+// path) and sums the leaf values in fp64.  All CTAs advance through the trees
+// in the same order, so the trees being walked at any moment stay L2-resident.
+#include <algorithm>
+
+#include "bf_internal.cuh"
+
+namespace bf {
+namespace {
+
+constexpr int PT = 128;  // rows per CTA
+
+__device__ __forceinline__ Node16 load_node(const Node16* p) {
+  const int4 v = __ldg(reinterpret_cast<const int4*>(p));
+  Node16 n;
+  n.v = __hiloint2double(v.y, v.x);
+  n.feature = v.z;
+  n.left = v.w;
+  return n;
+}
+
+__global__ void __launch_bounds__(PT) k_predict_smem(const Node16* __restrict__ nodes, const int64_t* __restrict__ off,
+                                                     int32_t ntrees, const double* __restrict__ Xq, int64_t ldq,
+                                                     int64_t m, int p, double* yhat_sum, double* yhat, double inv_t,
+                                                     unsigned long long* visits) {
+  extern __shared__ double sx[];  // PT x p, row-major, padded stride p|1
+  const int stride = p | 1;
+  const int64_t r0 = (int64_t)blockIdx.x * PT;
+  const int rows = (int)(m - r0 < PT ? m - r0 : PT);
+  for (int f = 0; f < p; ++f)
+    for (int r = threadIdx.x; r < rows; r += PT) sx[r * stride + f] = Xq[(int64_t)f * ldq + r0 + r];
+  __syncthreads();
+  if ((int)threadIdx.x >= rows) return;
+  const double* x = sx + threadIdx.x * stride;
+  double acc = 0.0;
+  unsigned long long nv = 0;
+  for (int32_t t = 0; t < ntrees; ++t) {
+    const Node16* tn = nodes + off[t];
+    Node16 nd = load_node(tn);
+    ++nv;
+    while (nd.feature >= 0) {
+      nd = load_node(tn + (x[nd.feature] <= nd.v ? nd.left : nd.left + 1));
+      ++nv;
+    }
+    acc += nd.v;
+  }
+  if (visits) atomicAdd(visits, nv);
+  const int64_t r = r0 + threadIdx.x;
+  if (yhat_sum) yhat_sum[r] = acc;
+  if (yhat) yhat[r] = acc * inv_t;
+}
+
+__global__ void __launch_bounds__(PT) k_predict_gmem(const Node16* __restrict__ nodes, const int64_t* __restrict__ off,
+                                                     int32_t ntrees, const double* __restrict__ Xq, int64_t ldq,
+                                                     int64_t m, double* yhat_sum, double* yhat, double inv_t,
+                                                     unsigned long long* visits) {
+  const int64_t r = (int64_t)blockIdx.x * PT + threadIdx.x;
+  if (r >= m) return;
+  double acc = 0.0;
+  unsigned long long nv = 0;
+  for (int32_t t = 0; t < ntrees; ++t) {
+    const Node16* tn = nodes + off[t];
+    Node16 nd = load_node(tn);
+    ++nv;
+    while (nd.feature >= 0) {
+      nd = load_node(tn + (__ldg(Xq + (int64_t)nd.feature * ldq + r) <= nd.v ? nd.left : nd.left + 1));
+      ++nv;
+    }
+    acc += nd.v;
+  }
+  if (visits) atomicAdd(visits, nv);
+  if (yhat_sum) yhat_sum[r] = acc;
+  if (yhat) yhat[r] = acc * inv_t;
+}
+
+}  // namespace
+
+void predict_impl(const bf_forest* f, const double* Xq_in, int64_t ldq, int64_t m, double* ys_in, double* yh_in,
+                  int32_t ntree_total, cudaStream_t s) {
+  if (m == 0) return;
+  const int p = f->info.p;
+  const int32_t nt = f->info.tree_end - f->info.tree_begin;
+  InStage Xs(Xq_in, sizeof(double) * (size_t)(ldq * (p - 1) + m), s);
+  OutStage ys(ys_in, ys_in ? sizeof(double) * m : 0, s), yh(yh_in, yh_in ? sizeof(double) * m : 0, s);
+  const double inv_t = 1.0 / (double)(ntree_total > 0 ? ntree_total : std::max(nt, 1));
+  const unsigned grid = (unsigned)ceil_div(m, PT);
+  const size_t smem = sizeof(double) * (size_t)PT * (size_t)(p | 1);
+  static int smax = 0;
+  if (!smax) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&smax, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    BF_CUDA_CHECK(cudaFuncSetAttribute(k_predict_smem, cudaFuncAttributeMaxDynamicSharedMemorySize, smax));
+  }
+  DBuf<unsigned long long> vis;
+  if (prof_enabled()) {
+    vis.alloc(1, s);
+    BF_CUDA_CHECK(cudaMemsetAsync(vis.p, 0, 8, s));
+  }
+  if (smem <= (size_t)smax) {
+    {
+      KScope ks_("k_predict_smem", s, 0.0);
+      k_predict_smem<<<grid, PT, smem, s>>>(f->d_nodes, f->d_tree_off, nt, (const double*)Xs.dptr, ldq, m, p,
+                                           ys_in ? (double*)ys.dptr : nullptr, yh_in ? (double*)yh.dptr : nullptr, inv_t, vis.p);
+    }
+  } else {
+    {
+      KScope ks_("k_predict_gmem", s, 0.0);
+      k_predict_gmem<<<grid, PT, 0, s>>>(f->d_nodes, f->d_tree_off, nt, (const double*)Xs.dptr, ldq, m,
+                                         ys_in ? (double*)ys.dptr : nullptr, yh_in ? (double*)yh.dptr : nullptr, inv_t, vis.p);
+    }
+  }
+  BF_CUDA_CHECK(cudaGetLastError());
+  if (vis.p) {  // profile mode: algorithmic bytes = node visits x 16 B + rows x (8p + 16) B
+    unsigned long long hv = 0;
+    BF_CUDA_CHECK(cudaMemcpyAsync(&hv, vis.p, 8, cudaMemcpyDeviceToHost, s));
+    BF_CUDA_CHECK(cudaStreamSynchronize(s));
+    prof_add_bytes(smem <= (size_t)smax ? "k_predict_smem" : "k_predict_gmem",
+                   16.0 * (double)hv + (double)m * (8.0 * p + 16.0 * ((ys_in != nullptr) + (yh_in != nullptr))));
+  }
+  if (ys_in) ys.finish(s);
+  if (yh_in) yh.finish(s);
+  if (ys.host || yh.host || Xs.tmp.p) BF_CUDA_CHECK(cudaStreamSynchronize(s));
+}
+
+}  // namespace bf

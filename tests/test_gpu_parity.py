@@ -1,0 +1,265 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Bar (BASELINE north_star): bootstrap/OOB indices and tree topology
+(feature, threshold, structure, counts) bit-exact; node values and
+predictions within 1e-9 relative; OOB MSE and %IncMSE within 1e-6
+relative; importance ranking identical.
+"""
+from __future__ import annotations
+
+import math
+import os
+import random
+
+import numpy as np
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():
+    pytest.skip("no CUDA device", allow_module_level=True)
+
+import paper_conf_ipps_madougouvln16_b200 as bf  # noqa: E402
+from paper_conf_ipps_madougouvln16_b200 import synthetic as S  # noqa: E402
+from oracle import oracle as O  # noqa: E402
+from tests.helpers import compare_forest, rel_close  # noqa: E402
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+DEV = torch.device("cuda:0")
+
+
+def dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).to(DEV)
+
+
+# ------------------------------------------------------------------ primitives
+def test_philox_kat_and_random_counters():
+    rows = [l.split() for l in open(os.path.join(GOLDEN, "philox_kat.txt")) if l.strip() and not l.startswith("#")]
+    for r in rows:
+        v = [int(x, 16) for x in r]
+        out = bf.philox(np.array([v[0:4]], np.uint32), v[4], v[5])
+        assert out[0].tolist() == v[6:10]
+    rng = np.random.default_rng(0)
+    ctr = rng.integers(0, 2 ** 32, (1000, 4), dtype=np.uint64).astype(np.uint32)
+    out = bf.philox(ctr, 0xDEADBEEF, 0x12345678)
+    for i in range(0, 1000, 97):
+        assert out[i].tolist() == O.philox(ctr[i].tolist(), [0xDEADBEEF, 0x12345678])
+
+
+def test_int128_to_double_correct_rounding():
+    rng = random.Random(5)
+    vals = [0, 1, -1, (1 << 53) + 1, ((1 << 53) + 1) << 40, (1 << 127) - 1, -(1 << 127), ((1 << 54) + 3) << 30]
+    for _ in range(20000):
+        b = rng.randrange(1, 127)
+        v = rng.getrandbits(b)
+        if rng.random() < 0.4:
+            v = (((rng.getrandbits(53) | (1 << 53)) * 2 + 1) << rng.randrange(0, 60)) & ((1 << 126) - 1)
+            if rng.random() < 0.5:
+                v += rng.choice([-1, 1])
+        vals.append(-v if rng.random() < 0.5 else v)
+    hi = np.array([(v >> 64) for v in vals], dtype=object)
+    hi = np.array([int(h) for h in hi], np.int64)
+    lo = np.array([v & ((1 << 64) - 1) for v in vals], dtype=np.uint64)
+    got = bf.i128_to_double(hi, lo)
+    exp = np.array([float(v) for v in vals])
+    assert np.array_equal(got, exp)
+
+
+@pytest.mark.parametrize("n", [1, 2, 7, 256, 4096, 100003])
+def test_fixed_point_bit_exact(n):
+    rng = np.random.default_rng(n)
+    y = rng.lognormal(0, 2, n) * rng.choice([-1, 1], n)
+    yq_o, q_o = O.fixed_point(y)
+    yq_g, q_g = bf.fixed_point(dev(y))
+    assert q_g == q_o
+    assert np.array_equal(yq_g.cpu().numpy(), yq_o)
+
+
+@pytest.mark.parametrize("n", [1, 3, 256, 4096, 1_000_000])
+def test_bootstrap_bit_exact(n):
+    seed = 0xBF10_0004
+    w = bf.bootstrap(seed, 5, 3, n)
+    for k in range(3):
+        assert np.array_equal(w[k], O.bootstrap(seed, 5 + k, n))
+
+
+@pytest.mark.parametrize("n_o", [1, 2, 3, 5, 17, 1000, 4097, 65536])
+def test_feistel_perm_bit_exact(n_o):
+    g = bf.perm(77, 3, 11, n_o)
+    assert sorted(g.tolist()) == list(range(n_o))
+    idx = range(n_o) if n_o <= 5000 else range(0, n_o, 61)
+    for a in idx:
+        assert g[a] == O.perm(77, 3, 11, n_o, a)
+
+
+# ------------------------------------------------------------------ fit topology
+CASES = [
+    # (n, p, kind, ntree, mtry, nodesize, small_node_max, trees_in_flight)
+    (40, 3, "int", 6, 0, 1, 0, 0),
+    (40, 3, "int", 6, 3, 1, 2, 0),          # global phase only (A = 2)
+    (300, 5, "mixed", 8, 0, 5, 8, 3),       # deep global phase, ragged batches
+    (300, 5, "mixed", 8, 0, 5, 0, 0),       # subtree kernel only
+    (1000, 7, "cont", 5, 7, 1, 64, 2),      # mtry = p, nodesize 1
+    (2500, 12, "int", 4, 0, 5, 300, 0),
+    (777, 1, "cont", 3, 1, 2, 16, 0),       # p = 1
+    (5, 2, "int", 3, 0, 5, 0, 0),           # root is a leaf (n <= nodesize)
+    (6, 2, "int", 3, 0, 1, 0, 0),
+]
+
+
+@pytest.mark.parametrize("case", CASES)
+def test_fit_topology_bit_exact(case):
+    n, p, kind, T, mtry, ns, A, B = case
+    X, y = S.small_random(n, p, seed=n * 31 + p, kind=kind)
+    seed = 1234 + n
+    of = O.fit(X, y, ntree=T, mtry=mtry, nodesize=ns, seed=seed, nthreads=4)
+    gf = bf.fit(dev(X), dev(y), ntree=T, mtry=mtry, nodesize=ns, seed=seed, small_node_max=A, trees_in_flight=B)
+    assert compare_forest(gf, of) > 0
+    assert gf.info.q == of.q
+
+
+def test_fit_degenerate_inputs():
+    rng = np.random.default_rng(1)
+    X = rng.normal(size=(3, 50))
+    # constant y -> single leaves
+    gf = bf.fit(dev(X), dev(np.full(50, 2.5)), ntree=3, seed=1)
+    e = gf.export()
+    assert np.all(e["feature"] == -1) and np.all(e["thr_or_value"] == 2.5)
+    # constant X -> single leaves
+    y = rng.normal(size=50)
+    of = O.fit(np.ones((3, 50)), y, ntree=3, seed=2)
+    gf = bf.fit(dev(np.ones((3, 50))), dev(y), ntree=3, seed=2)
+    compare_forest(gf, of)
+    # -0.0 / +0.0 are one value
+    X2 = np.zeros((2, 60))
+    X2[0, ::2] = -0.0
+    X2[1] = rng.integers(0, 3, 60)
+    y2 = np.concatenate([y, y[:10]])
+    of = O.fit(X2, y2, ntree=4, seed=3, nodesize=1)
+    gf = bf.fit(dev(X2), dev(y2), ntree=4, seed=3, nodesize=1)
+    compare_forest(gf, of)
+    # NaN rejected
+    Xn = X.copy()
+    Xn[1, 7] = np.nan
+    with pytest.raises(bf.BFError) as ei:
+        bf.fit(dev(Xn), dev(y), ntree=1)
+    assert ei.value.code == -2
+
+
+def test_fit_host_pointers_equal_device_pointers():
+    X, y = S.small_random(500, 6, seed=9)
+    a = bf.fit(dev(X), dev(y), ntree=4, seed=5).export()
+    b = bf.fit(X, y, ntree=4, seed=5).export()   # host numpy: staged by the library
+    for k in ("feature", "thr_or_value", "count"):
+        # same structure; node order may differ between runs, compare sorted multisets
+        assert np.array_equal(np.sort(a[k]), np.sort(b[k]))
+
+
+def test_tree_range_sharding_bit_identical():
+    X, y = S.gen_reduction()
+    full = O.fit(X, y, ntree=10, seed=77)
+    part = bf.fit(dev(X), dev(y), ntree=10, seed=77, tree_begin=3, tree_end=7)
+    e = part.export()
+    from tests.helpers import compare_tree
+    for i in range(4):
+        lo, hi = e["tree_off"][i], e["tree_off"][i + 1]
+        g = {k: e[k][lo:hi] for k in ("feature", "left", "thr_or_value", "count", "value", "drss")}
+        compare_tree(g, full.tree(3 + i))
+
+
+# ------------------------------------------------------------------ configs C1..C3 in full
+def _config_data(cfg):
+    X, y, c = S.dataset(cfg)
+    if cfg == "C3":
+        from oracle.pca import pca, n_components
+        r = pca(X, scale=True)
+        k = n_components(r["sdev"])
+        X = np.ascontiguousarray(np.concatenate([r["scores"][:, :k].T, c.extra["L"][None, :], c.extra["M"]], axis=0))
+    return X, y, c
+
+
+@pytest.mark.parametrize("cfg", ["C1", "C2", "C3"])
+def test_config_forest_parity(cfg):
+    X, y, c = _config_data(cfg)
+    T = c.ntree if cfg == "C1" else 60
+    of = O.fit(X, y, ntree=T, seed=S.FOREST_SEED + 1, nthreads=os.cpu_count() or 4)
+    gf = bf.fit(dev(X), dev(y), ntree=T, seed=S.FOREST_SEED + 1)
+    compare_forest(gf, of)
+    # predictions
+    Q = S.gen_query(X, 5000)
+    ys, yh = gf.predict(dev(Q), ntree_total=T)
+    po = of.predict_sum(Q)
+    assert rel_close(ys.cpu().numpy(), po, 1e-9)
+    assert rel_close(yh.cpu().numpy(), po / T, 1e-9)
+
+
+# ------------------------------------------------------------------ OOB importance
+@pytest.mark.parametrize("cfg", ["C1", "C2"])
+def test_oob_importance_parity(cfg):
+    X, y, c = _config_data(cfg)
+    T = 120 if cfg == "C1" else 40
+    seed = S.FOREST_SEED + 2
+    of = O.fit(X, y, ntree=T, seed=seed, nthreads=os.cpu_count() or 4)
+    ro = of.oob_importance(X, y)
+    gf = bf.fit(dev(X), dev(y), ntree=T, seed=seed)
+    rg = gf.oob_importance(dev(X), dev(y))
+    rg = {k: v.cpu().numpy() for k, v in rg.items()}
+    assert np.array_equal(rg["nout_t"], ro["nout_t"])
+    assert np.array_equal(rg["oob_cnt"], ro["oob_cnt"])
+    assert rel_close(rg["oob_sum"], ro["oob_sum"], 1e-9)
+    assert rel_close(rg["e_t"], ro["e_t"], 1e-9)
+    # d_tm: exact zeros where the oracle has exact zeros (unused predictors)
+    unused = ro["npur_slots"] == 0.0
+    assert np.all(rg["d_slots"][unused] == 0.0)
+    assert rel_close(rg["d_slots"], ro["d_slots"], 1e-6, 1e-9)
+    assert rel_close(rg["npur_slots"], ro["npur_slots"], 1e-9, 1e-12)
+    fo = O.importance_finalize(ro["d_slots"], ro["npur_slots"], ro["oob_sum"], ro["oob_cnt"], y)
+    fg = bf.importance_finalize(dev(rg["d_slots"]), dev(rg["npur_slots"]), dev(rg["oob_sum"]), dev(rg["oob_cnt"]), dev(y))
+    fg = {k: (v.cpu().numpy() if hasattr(v, "cpu") else v) for k, v in fg.items()}
+    assert rel_close(fg["inc_mse_raw"], fo["inc_mse_raw"], 1e-6, 1e-9)
+    assert rel_close(fg["inc_mse"], fo["inc_mse"], 1e-6, 1e-9)
+    assert rel_close(fg["inc_node_purity"], fo["inc_node_purity"], 1e-9)
+    assert abs(float(fg["oob_mse"]) - fo["oob_mse"]) <= 1e-6 * fo["oob_mse"]
+    assert abs(float(fg["rsq"]) - fo["rsq"]) <= 1e-6 * abs(fo["rsq"]) + 1e-12
+    # ranking identical (ties within 1e-12 reported, not hidden)
+    og, oo = np.argsort(-fg["inc_mse"], kind="stable"), np.argsort(-fo["inc_mse"], kind="stable")
+    if not np.array_equal(og, oo):
+        gaps = np.abs(np.diff(np.sort(fo["inc_mse"])))
+        assert gaps.min() < 1e-9 * np.abs(fo["inc_mse"]).max(), "importance ranking differs"
+
+
+# ------------------------------------------------------------------ PCA
+@pytest.mark.parametrize("scale", [True, False])
+def test_pca_parity(scale):
+    from oracle.pca import pca
+    X, _, _ = S.dataset("C3") if scale else (S.gen_mm(2048)[0], None, None)
+    ro = pca(X, scale=scale)
+    k = 6
+    rg = bf.pca(dev(X), scale=scale, k=k)
+    sd = rg["sdev"].cpu().numpy()
+    assert rel_close(sd, ro["sdev"], 1e-9, 1e-12)
+    rot = rg["rotation"].cpu().numpy()  # row j = component j
+    lam = ro["sdev"] ** 2
+    for j in range(k):
+        gap = min(abs(lam[j] - lam[j - 1]) if j else np.inf, abs(lam[j] - lam[j + 1]) if j + 1 < len(lam) else np.inf)
+        if gap > 1e-6 * lam[0]:
+            assert np.allclose(rot[j], ro["rotation"][:, j], atol=1e-7)
+    sc = rg["scores"].cpu().numpy()
+    for j in range(k):
+        if np.allclose(rot[j], ro["rotation"][:, j], atol=1e-7):
+            assert np.allclose(sc[j], ro["scores"][:, j], rtol=1e-7, atol=1e-7 * np.abs(ro["scores"][:, j]).max())
+
+
+# ------------------------------------------------------------------ C4 at full size, sampled trees
+@pytest.mark.slow
+def test_c4_full_size_sampled_trees():
+    X, y = S.gen_scaled()
+    seed = S.FOREST_SEED + 4
+    trees = (0, 1)
+    of = O.fit(X, y, ntree=1000, seed=seed, tree_begin=0, tree_end=2, nthreads=2)
+    gf = bf.fit(dev(X), dev(y), ntree=1000, seed=seed, tree_begin=0, tree_end=2)
+    compare_forest(gf, of)
+    Q = S.gen_query(X, 2000)
+    ys, _ = gf.predict(dev(Q))
+    assert rel_close(ys.cpu().numpy(), of.predict_sum(Q), 1e-9)
