@@ -239,4 +239,18 @@ void philox_impl(const uint32_t* ctr, uint32_t k0, uint32_t k1, uint32_t* out, i
 void i128_impl(const int64_t* hi, const uint64_t* lo, double* out, int64_t count, cudaStream_t s);
 
 inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+// Largest dynamic shared memory a launch of `func` may request (opt-in limit
+// minus the kernel's static shared memory); sets the attribute accordingly.
+template <class F>
+int dyn_smem_limit(F func) {
+  int dev = 0, optin = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+  cudaFuncAttributes fa;
+  cudaFuncGetAttributes(&fa, (const void*)func);
+  const int lim = optin - (int)fa.sharedSizeBytes;
+  cudaFuncSetAttribute((const void*)func, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
+  return lim;
+}
 }  // namespace bf

@@ -24,6 +24,19 @@ void* dev_alloc(size_t bytes, cudaStream_t s) {
     BF_REQUIRE(p != nullptr, BF_ENOMEM, "allocator hook returned NULL for " + std::to_string(bytes) + " bytes");
     return p;
   }
+  static bool pool_cfg = false;
+  if (!pool_cfg) {
+    // keep freed blocks cached in the device pool (no unmap/remap of the GBs of
+    // per-fit work space at every synchronisation point)
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+      uint64_t thr = UINT64_MAX;
+      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+    pool_cfg = true;
+  }
   cudaError_t e = cudaMallocAsync(&p, bytes, s);
   if (e != cudaSuccess) {
     cudaGetLastError();

@@ -34,7 +34,7 @@ namespace bf {
 namespace {
 
 constexpr int NT = 256;         // threads per CTA of the streaming kernels
-constexpr int SUB_NW = 8;       // warps of the subtree kernel
+constexpr int SUB_NW = 16;      // warps of the subtree kernel
 constexpr int SUB_NT = SUB_NW * 32;
 constexpr int KIND_NONE = -1, KIND_LEAF = 0, KIND_SMALL = 1, KIND_LARGE = 2;
 
@@ -397,6 +397,19 @@ __device__ __forceinline__ bool rec_better(double g, uint32_t r, double bg, uint
   return g > bg || (g == bg && r < br);
 }
 
+// fp32 screen of a candidate against the running best key: true unless the
+// candidate's exact key is certainly below `best` (relative error of the
+// screen < 2^-20; candidates that might round to >= best take the exact path).
+__device__ __forceinline__ bool screen_may_win(int64_t nk, int64_t Sk, int64_t nl, int64_t Sl, double best) {
+  if (best <= 0.0) return true;
+  const __int128 D = (__int128)nk * (__int128)Sl - (__int128)nl * (__int128)Sk;
+  const double d = (double)(float)(double)D;  // coarse but monotone-safe within 2^-22 relative
+  const double nn = (double)(nl * (nk - nl));
+  const double gapprox = d * d * (double)__frcp_rn((float)nn);
+  return gapprox >= best * (1.0 - 1.0 / (1 << 18));
+}
+
+
 __global__ void __launch_bounds__(NT) k_split_scan(const LNode* nodes, const int32_t* feat, int mtry,
                                                    const uint64_t* E, const Pay* pay, int64_t n, Rec* rec) {
   __shared__ int32_t smc[NT / 32];
@@ -449,7 +462,7 @@ __global__ void __launch_bounds__(NT) k_split_scan(const LNode* nodes, const int
       const int j = j0 + u;
       if (j + 1 < a) {
         const uint32_t ra = (uint32_t)(e[u] >> 32), rb = (uint32_t)(e[u + 1] >> 32);
-        if (ra != rb) {
+        if (ra != rb && screen_may_win(nk, Sk, prec, pres, bg)) {
           const double g = split_key(nk, Sk, prec, pres);
           if (rec_better(g, ra, bg, brank)) {
             bg = g;
@@ -724,35 +737,65 @@ __global__ void __launch_bounds__(NT) k_partition(const LNode* nodes, const Spli
   }
 }
 
-// ------------------------------------------------------------------ subtree phase
+// ------------------------------------------------------------------ subtree phase (one CTA per small node)
+// Layout: the subtree's rows occupy local ids 0..a0-1.  list[f][0..a0) holds
+// feature f's entries ((local rank << 16) | local row) sorted by value; every
+// node owns the same column range [lo, lo+a) in every feature row, and a split
+// partitions each row's range in place (left part first), so children ranges
+// nest.  R[row][f] = local rank (index of the first entry of the row's value)
+// lets a warp evaluate a tiny node (a <= 32: one lane per row) by sorting the
+// 32 ranks in registers instead of maintaining p partitioned lists.
+constexpr int TINY = 32;
+
 struct SRec {  // node record of a subtree (local ids)
   int32_t feature, left, count, pad;
   double thr, value, drss;
 };
-struct SCur {  // active node of a subtree level
-  int32_t off, a, n, id;
+struct MNode {  // medium node (a > TINY) of a subtree level
+  int32_t lo, a, n, id;
   int64_t S;
   uint64_t key;
   int32_t split, lid, al, nl;
   int64_t Sl;
   uint64_t keyl, keyr;
-  int32_t coff[2];
+  int32_t kind[2];
+};
+struct TNode {  // tiny node (a <= TINY)
+  int32_t lo, a, n, id;
+  int64_t S;
+  uint64_t key;
+};
+struct WRec {  // best candidate found by one warp for its share of a node's features
+  double g;
+  int32_t f;
+  uint32_t lrank;
+  int32_t pos, nl;
+  int64_t Sl;
+  uint32_t ra, rb;
 };
 
 __host__ __device__ inline size_t align16(size_t x) { return (x + 15) & ~size_t(15); }
+__host__ __device__ inline int rank_stride(int p) {  // u16 row stride of R: 2*(odd) -> conflict-free columns
+  int rs = (p + 1) & ~1;
+  if (((rs >> 1) & 1) == 0) rs += 2;
+  return rs;
+}
+__host__ __device__ inline int max_medium(int A) { return A / (TINY + 1) + 2; }
 
 __host__ __device__ inline size_t subtree_smem(int A, int p) {
   size_t s = 0;
-  s += align16(2 * (size_t)p * A * 4);       // ent0, ent1
-  s += align16((size_t)A * 8);               // wy
-  s += align16((size_t)A * 8);               // w*y fp64
-  s += align16((size_t)2 * A * sizeof(SRec));
-  s += align16((size_t)2 * (A / 2 + 1) * sizeof(SCur));
-  s += align16((size_t)A * 4);               // w
-  s += align16((size_t)A * 4);               // global row
-  s += align16((size_t)SUB_NW * p * 2);      // Fisher-Yates scratch
-  s += align16((size_t)SUB_NW * p * 2);      // drawn features
-  s += align16((size_t)A);                   // side
+  s += align16((size_t)p * A * 4);                    // list
+  s += align16((size_t)A * rank_stride(p) * 2);       // R
+  s += align16((size_t)SUB_NW * A * 4);               // per-warp partition temp
+  s += align16((size_t)A * 8) * 2;                    // wy, w*y
+  s += align16((size_t)A * 4) * 2;                    // w, global row
+  s += align16((size_t)A);                            // side
+  s += align16((size_t)2 * A * sizeof(SRec));         // node records
+  s += align16((size_t)2 * max_medium(A) * sizeof(MNode));
+  s += align16((size_t)(A / 2 + 1) * sizeof(TNode));  // tiny queue
+  s += align16((size_t)SUB_NW * (TINY + 2) * sizeof(TNode));  // DFS stacks
+  s += align16((size_t)SUB_NW * p * 2) * 2;           // Fisher-Yates scratch, drawn features
+  s += align16((size_t)SUB_NW * sizeof(WRec));
   s += 64;
   return s;
 }
@@ -772,32 +815,86 @@ struct SubArgs {
   Pool pool;
 };
 
+// S4.2 mtry draw by one warp: Philox words computed by the lanes, the
+// partial Fisher-Yates swaps applied by lane 0 in shared memory.
+__device__ __forceinline__ void warp_draw_mtry(uint64_t seed, uint32_t t, uint64_t key, int p, int mtry, int16_t* mind,
+                                               int16_t* feats, int lane) {
+  for (int j = lane; j < p; j += 32) mind[j] = (int16_t)j;
+  __syncwarp();
+  int last = p - 1;
+  for (int c0 = 0; c0 < mtry; c0 += 64) {
+    uint64_t u0 = 0, u1 = 0;
+    const int call = (c0 >> 1) + lane;
+    if (2 * call < mtry) philox_u64x2(seed, (uint32_t)key, (uint32_t)(key >> 32), t, 0x20000000u | (uint32_t)call, u0, u1);
+    const int cend = min(mtry, c0 + 64);
+    for (int s = c0; s < cend; ++s) {
+      const int sl = (s - c0) >> 1;
+      const uint64_t ua = __shfl_sync(0xffffffffu, u0, sl);
+      const uint64_t ub = __shfl_sync(0xffffffffu, u1, sl);
+      if (lane == 0) {
+        const uint64_t u = (s & 1) ? ub : ua;
+        const int j = (int)mulhi64(u, (uint64_t)(last + 1));
+        feats[s] = mind[j];
+        const int16_t tmp = mind[j];
+        mind[j] = mind[last];
+        mind[last] = tmp;
+      }
+      --last;
+    }
+  }
+  __syncwarp();
+}
+
+__device__ __forceinline__ uint32_t bitonic_sort32(uint32_t key, int lane) {
+#pragma unroll
+  for (int k = 2; k <= 32; k <<= 1) {
+#pragma unroll
+    for (int j = k >> 1; j > 0; j >>= 1) {
+      const uint32_t o = __shfl_xor_sync(0xffffffffu, key, j);
+      const bool up = (lane & k) == 0;
+      const bool lower = (lane & j) == 0;
+      key = (lower == up) ? min(key, o) : max(key, o);
+    }
+  }
+  return key;
+}
+
 __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   extern __shared__ __align__(16) unsigned char smem[];
-  const int A = g.A, p = g.p;
+  const int A = g.A, p = g.p, RS = rank_stride(p), MM = max_medium(A);
   unsigned char* ptr = smem;
-  uint32_t* ent0 = (uint32_t*)ptr;
-  uint32_t* ent1 = ent0 + (size_t)p * A;
-  ptr += align16(2 * (size_t)p * A * 4);
+  uint32_t* list = (uint32_t*)ptr;
+  ptr += align16((size_t)p * A * 4);
+  uint16_t* R = (uint16_t*)ptr;
+  ptr += align16((size_t)A * RS * 2);
+  uint32_t* temp_all = (uint32_t*)ptr;
+  ptr += align16((size_t)SUB_NW * A * 4);
   int64_t* wy = (int64_t*)ptr;
   ptr += align16((size_t)A * 8);
   double* wyd = (double*)ptr;
   ptr += align16((size_t)A * 8);
-  SRec* recs = (SRec*)ptr;
-  ptr += align16((size_t)2 * A * sizeof(SRec));
-  SCur* curl = (SCur*)ptr;
-  SCur* nxtl = curl + (A / 2 + 1);
-  ptr += align16((size_t)2 * (A / 2 + 1) * sizeof(SCur));
   int32_t* wl = (int32_t*)ptr;
   ptr += align16((size_t)A * 4);
   uint32_t* grow = (uint32_t*)ptr;
   ptr += align16((size_t)A * 4);
+  uint8_t* side = (uint8_t*)ptr;
+  ptr += align16((size_t)A);
+  SRec* recs = (SRec*)ptr;
+  ptr += align16((size_t)2 * A * sizeof(SRec));
+  MNode* curl = (MNode*)ptr;
+  MNode* nxtl = curl + MM;
+  ptr += align16((size_t)2 * MM * sizeof(MNode));
+  TNode* tq = (TNode*)ptr;
+  ptr += align16((size_t)(A / 2 + 1) * sizeof(TNode));
+  TNode* stacks = (TNode*)ptr;
+  ptr += align16((size_t)SUB_NW * (TINY + 2) * sizeof(TNode));
   int16_t* mind_all = (int16_t*)ptr;
   ptr += align16((size_t)SUB_NW * p * 2);
   int16_t* feats_all = (int16_t*)ptr;
   ptr += align16((size_t)SUB_NW * p * 2);
-  uint8_t* side = (uint8_t*)ptr;
-  __shared__ int s_nloc, s_ncur, s_gbase;
+  WRec* wrec = (WRec*)ptr;
+  __shared__ int s_nloc, s_ncur, s_gbase, s_qtail, s_qhead;
+  __shared__ int32_t s_scan[SUB_NW];
 
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const LNode root = g.sq[blockIdx.x];
@@ -807,8 +904,11 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   const Pay* P = g.pay + (int64_t)b * g.n;
   uint16_t* loc = g.loc + (int64_t)b * g.n;
   const uint64_t* src = g.Es + root.base;
+  int16_t* mind = mind_all + wid * p;
+  int16_t* feats = feats_all + wid * p;
+  uint32_t* temp = temp_all + (size_t)wid * A;
 
-  // ---- load: local rows from feature 0's list, payload, then local ranks per feature
+  // ---- load 1: local rows = feature 0's order; payload; global row -> local id
   for (int j = tid; j < a0; j += SUB_NT) {
     const uint32_t row = (uint32_t)src[j];
     grow[j] = row;
@@ -819,25 +919,50 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
     wyd[j] = __dmul_rn((double)pp.w, g.y[row]);
   }
   __syncthreads();
-  for (int f = wid; f < p; f += SUB_NW) {
-    const uint64_t* sf = src + (int64_t)f * a0;
-    uint32_t carry = 0, prevr = 0xffffffffu;
-    for (int j0 = 0; j0 < a0; j0 += 32) {
-      const int j = j0 + lane;
-      uint64_t e = j < a0 ? sf[j] : 0;
-      const uint32_t r = (uint32_t)(e >> 32);
-      const uint32_t rprev = __shfl_up_sync(0xffffffffu, r, 1);
-      const uint32_t before = lane == 0 ? prevr : rprev;
-      const uint32_t flag = (j < a0 && j > 0 && r != before) ? 1u : 0u;
-      const uint32_t inc = warp_incl_scan(flag, lane) + carry;
-      if (j < a0) ent0[(size_t)f * a0 + j] = (inc << 16) | (uint32_t)loc[(uint32_t)e];
-      carry = __shfl_sync(0xffffffffu, inc, 31);
-      prevr = __shfl_sync(0xffffffffu, r, 31);
+  // ---- load 2: warp per feature; local rank = index of the first entry of the same value
+  {
+    constexpr int GRP = 8;  // chunks of 32 entries in flight per warp
+    const int nch = (a0 + 31) >> 5;
+    for (int f = wid; f < p; f += SUB_NW) {
+      const uint64_t* sf = src + (int64_t)f * a0;
+      int carry_gs = 0;
+      uint32_t prev_last = 0xffffffffu;
+      for (int c0 = 0; c0 < nch; c0 += GRP) {
+        uint32_t rk[GRP];
+        uint16_t lr[GRP];
+#pragma unroll
+        for (int c = 0; c < GRP; ++c) {
+          const int j = (c0 + c) * 32 + lane;
+          const uint64_t e = j < a0 ? sf[j] : ~0ull;
+          rk[c] = (uint32_t)(e >> 32);
+          lr[c] = j < a0 ? loc[(uint32_t)e] : 0;
+        }
+#pragma unroll
+        for (int c = 0; c < GRP; ++c) {
+          if (c0 + c >= nch) break;
+          const int j = (c0 + c) * 32 + lane;
+          const uint32_t up = __shfl_up_sync(0xffffffffu, rk[c], 1);
+          const uint32_t prv = lane == 0 ? prev_last : up;
+          int gs = (j > 0 && rk[c] != prv) ? j : 0;
+#pragma unroll
+          for (int o = 1; o < 32; o <<= 1) {
+            const int v = __shfl_up_sync(0xffffffffu, gs, o);
+            if (lane >= o) gs = max(gs, v);
+          }
+          gs = max(gs, carry_gs);
+          if (j < a0) {
+            list[(size_t)f * a0 + j] = ((uint32_t)gs << 16) | lr[c];
+            R[(size_t)lr[c] * RS + f] = (uint16_t)gs;
+          }
+          carry_gs = __shfl_sync(0xffffffffu, gs, 31);
+          prev_last = __shfl_sync(0xffffffffu, rk[c], 31);
+        }
+      }
     }
   }
   if (tid == 0) {
     s_nloc = 1;
-    s_ncur = 1;
+    s_qhead = 0;
     SRec r0;
     r0.feature = -1;
     r0.left = -1;
@@ -847,116 +972,345 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
     r0.value = 0.0;
     r0.drss = 0.0;
     recs[0] = r0;
-    SCur c;
-    c.off = 0;
-    c.a = a0;
-    c.n = root.n;
-    c.id = 0;
-    c.S = root.S;
-    c.key = root.key;
-    c.split = 0;
-    curl[0] = c;
+    if (a0 > TINY) {
+      MNode c;
+      c.lo = 0;
+      c.a = a0;
+      c.n = root.n;
+      c.id = 0;
+      c.S = root.S;
+      c.key = root.key;
+      c.split = 0;
+      curl[0] = c;
+      s_ncur = 1;
+      s_qtail = 0;
+    } else {
+      TNode c;
+      c.lo = 0;
+      c.a = a0;
+      c.n = root.n;
+      c.id = 0;
+      c.S = root.S;
+      c.key = root.key;
+      tq[0] = c;
+      s_ncur = 0;
+      s_qtail = 1;
+    }
   }
   __syncthreads();
 
-  uint32_t* cbuf = ent0;
-  uint32_t* nbuf = ent1;
-  int16_t* mind = mind_all + wid * p;
-  int16_t* feats = feats_all + wid * p;
+  // ================= medium levels (a > TINY): level-synchronous inside the CTA
   while (s_ncur > 0) {
     const int ncur = s_ncur;
-    // ---- phase A: warp per node: draw, scan, choose, mark sides, child means
-    for (int i = wid; i < ncur; i += SUB_NW) {
-      SCur nd = curl[i];
-      if (lane == 0) {
-        for (int j = 0; j < p; ++j) mind[j] = (int16_t)j;
-        int last = p - 1;
-        uint64_t u0 = 0, u1 = 0;
-        for (int s = 0; s < g.mtry; ++s) {
-          if ((s & 1) == 0)
-            philox_u64x2(g.seed, (uint32_t)nd.key, (uint32_t)(nd.key >> 32), t, 0x20000000u | (uint32_t)(s >> 1),
-                         u0, u1);
-          const uint64_t u = (s & 1) ? u1 : u0;
-          const int j = (int)mulhi64(u, (uint64_t)(last + 1));
-          feats[s] = mind[j];
-          const int16_t tmp = mind[j];
-          mind[j] = mind[last];
-          mind[last] = tmp;
-          --last;
-        }
-      }
-      __syncwarp();
-      double bg = -1.0;
-      int bf = 0x7fffffff, bpos = -1, bnl = 0;
-      int64_t bSl = 0;
-      uint32_t bra = 0, brb = 0;
-      const int64_t nk = nd.n, Sk = nd.S;
-      for (int s = 0; s < g.mtry; ++s) {
-        const int f = feats[s];
-        const uint32_t* seg = cbuf + nd.off + (size_t)f * nd.a;
-        int32_t cc = 0;
-        int64_t cs = 0;
-        double lg = -1.0;
-        uint32_t lrk = 0xffffffffu, lra = 0, lrb = 0;
-        int lpos = -1, lnl = 0;
-        int64_t lSl = 0;
-        for (int j0 = 0; j0 < nd.a; j0 += 32) {
-          const int j = j0 + lane;
-          const uint32_t e = j < nd.a ? seg[j] : 0u;
-          const uint32_t lr = e & 0xffffu;
-          const int32_t w = j < nd.a ? wl[lr] : 0;
-          const int64_t ws = j < nd.a ? wy[lr] : 0;
-          const int32_t ic = warp_incl_scan(w, lane) + cc;
-          const int64_t is = warp_incl_scan(ws, lane) + cs;
-          if (j + 1 < nd.a) {
-            const uint32_t en = seg[j + 1];
-            if ((en >> 16) != (e >> 16)) {
-              const double gk = split_key(nk, Sk, ic, is);
-              if (rec_better(gk, e >> 16, lg, lrk)) {
-                lg = gk;
-                lrk = e >> 16;
-                lra = lr;
-                lrb = en & 0xffffu;
-                lpos = j;
-                lnl = ic;
-                lSl = is;
+    int G = 1;
+    while (G * 2 * ncur <= SUB_NW) G *= 2;
+    const int ngroups = SUB_NW / G, group = wid / G, sub = wid - group * G;
+    const int rounds = (ncur + ngroups - 1) / ngroups;
+    for (int rd = 0; rd < rounds; ++rd) {
+      const int i = rd * ngroups + group;
+      const bool active = i < ncur;
+      MNode nd;
+      if (active) {
+        nd = curl[i];
+        warp_draw_mtry(g.seed, t, nd.key, p, g.mtry, mind, feats, lane);
+        double bg = -1.0;
+        int bf = 0x7fffffff, bpos = -1, bnl = 0;
+        int64_t bSl = 0;
+        uint32_t bra = 0, brb = 0, brk = 0xffffffffu;
+        const int64_t nk = nd.n, Sk = nd.S;
+        for (int s = sub; s < g.mtry; s += G) {
+          const int f = feats[s];
+          const uint32_t* seg = list + (size_t)f * a0 + nd.lo;
+          int32_t cc = 0;
+          int64_t cs = 0;
+          double lg = -1.0;
+          uint32_t lrk = 0xffffffffu, lra = 0, lrb = 0;
+          int lpos = -1, lnl = 0;
+          int64_t lSl = 0;
+          for (int j0 = 0; j0 < nd.a; j0 += 32) {
+            const int j = j0 + lane;
+            const uint32_t e = j < nd.a ? seg[j] : 0u;
+            const uint32_t lr = e & 0xffffu;
+            const int32_t w = j < nd.a ? wl[lr] : 0;
+            const int64_t ws = j < nd.a ? wy[lr] : 0;
+            const int32_t ic = warp_incl_scan(w, lane) + cc;
+            const int64_t is = warp_incl_scan(ws, lane) + cs;
+            if (j + 1 < nd.a) {
+              const uint32_t en = seg[j + 1];
+              if ((en >> 16) != (e >> 16) && screen_may_win(nk, Sk, ic, is, lg)) {
+                const double gk = split_key(nk, Sk, ic, is);
+                if (rec_better(gk, e >> 16, lg, lrk)) {
+                  lg = gk;
+                  lrk = e >> 16;
+                  lra = lr;
+                  lrb = en & 0xffffu;
+                  lpos = j;
+                  lnl = ic;
+                  lSl = is;
+                }
               }
             }
+            cc = __shfl_sync(0xffffffffu, ic, 31);
+            cs = __shfl_sync(0xffffffffu, is, 31);
           }
-          cc = __shfl_sync(0xffffffffu, ic, 31);
-          cs = __shfl_sync(0xffffffffu, is, 31);
-        }
-        // warp argmax over lanes (g desc, local rank asc)
-        int srcl = lane;
+          int srcl = lane;
 #pragma unroll
-        for (int o = 16; o > 0; o >>= 1) {
-          const double og = __shfl_down_sync(0xffffffffu, lg, o);
-          const uint32_t orr = __shfl_down_sync(0xffffffffu, lrk, o);
-          const int os = __shfl_down_sync(0xffffffffu, srcl, o);
-          if (lane + o < 32 && rec_better(og, orr, lg, lrk)) {
-            lg = og;
-            lrk = orr;
-            srcl = os;
+          for (int o = 16; o > 0; o >>= 1) {
+            const double og = __shfl_down_sync(0xffffffffu, lg, o);
+            const uint32_t orr = __shfl_down_sync(0xffffffffu, lrk, o);
+            const int os = __shfl_down_sync(0xffffffffu, srcl, o);
+            if (lane + o < 32 && rec_better(og, orr, lg, lrk)) {
+              lg = og;
+              lrk = orr;
+              srcl = os;
+            }
+          }
+          srcl = __shfl_sync(0xffffffffu, srcl, 0);
+          lg = __shfl_sync(0xffffffffu, lg, 0);
+          lrk = __shfl_sync(0xffffffffu, lrk, 0);
+          const int wpos = __shfl_sync(0xffffffffu, lpos, srcl);
+          const int wnl = __shfl_sync(0xffffffffu, lnl, srcl);
+          const int64_t wSl = __shfl_sync(0xffffffffu, lSl, srcl);
+          const uint32_t wra = __shfl_sync(0xffffffffu, lra, srcl);
+          const uint32_t wrb = __shfl_sync(0xffffffffu, lrb, srcl);
+          if (lg >= 0.0 && (lg > bg || (lg == bg && f < bf))) {
+            bg = lg;
+            bf = f;
+            brk = lrk;
+            bpos = wpos;
+            bnl = wnl;
+            bSl = wSl;
+            bra = wra;
+            brb = wrb;
           }
         }
-        srcl = __shfl_sync(0xffffffffu, srcl, 0);
-        lg = __shfl_sync(0xffffffffu, lg, 0);
-        const int wpos = __shfl_sync(0xffffffffu, lpos, srcl);
-        const int wnl = __shfl_sync(0xffffffffu, lnl, srcl);
-        const int64_t wSl = __shfl_sync(0xffffffffu, lSl, srcl);
-        const uint32_t wra = __shfl_sync(0xffffffffu, lra, srcl);
-        const uint32_t wrb = __shfl_sync(0xffffffffu, lrb, srcl);
-        if (lg >= 0.0 && (lg > bg || (lg == bg && f < bf))) {
-          bg = lg;
-          bf = f;
-          bpos = wpos;
-          bnl = wnl;
-          bSl = wSl;
-          bra = wra;
-          brb = wrb;
+        if (lane == 0) {
+          WRec r;
+          r.g = bg;
+          r.f = bf;
+          r.lrank = brk;
+          r.pos = bpos;
+          r.nl = bnl;
+          r.Sl = bSl;
+          r.ra = bra;
+          r.rb = brb;
+          wrec[wid] = r;
         }
       }
-      if (bg > 0.0) {
+      __syncthreads();
+      if (active && sub == 0) {
+        WRec best = wrec[wid];
+        for (int k = 1; k < G; ++k) {
+          const WRec r = wrec[wid + k];
+          if (r.g >= 0.0 && (r.g > best.g || (r.g == best.g && r.f < best.f))) best = r;
+        }
+        if (best.g > 0.0) {
+          int lid = 0;
+          if (lane == 0) {
+            const double xa = canon(g.X[(int64_t)best.f * g.ldx + grow[best.ra]]);
+            const double xb = canon(g.X[(int64_t)best.f * g.ldx + grow[best.rb]]);
+            lid = atomicAdd(&s_nloc, 2);
+            SRec& r = recs[nd.id];
+            r.feature = best.f;
+            r.left = lid;
+            r.thr = split_threshold(xa, xb);
+            r.drss = ldexp(__ddiv_rn(best.g, (double)nd.n), -2 * g.q);
+            nd.keyl = child_key(g.seed, t, nd.key, 0);
+            nd.keyr = child_key(g.seed, t, nd.key, 1);
+          }
+          lid = __shfl_sync(0xffffffffu, lid, 0);
+          const uint32_t* seg = list + (size_t)best.f * a0 + nd.lo;
+          double sl = 0.0, sr = 0.0;
+          for (int j = lane; j < nd.a; j += 32) {
+            const uint32_t lr = seg[j] & 0xffffu;
+            const int sdv = j > best.pos;
+            side[lr] = (uint8_t)sdv;
+            if (sdv) sr += wyd[lr];
+            else sl += wyd[lr];
+          }
+#pragma unroll
+          for (int o = 16; o > 0; o >>= 1) {
+            sl += __shfl_down_sync(0xffffffffu, sl, o);
+            sr += __shfl_down_sync(0xffffffffu, sr, o);
+          }
+          if (lane == 0) {
+            const int nr = nd.n - best.nl, al = best.pos + 1, ar = nd.a - al;
+            SRec c;
+            c.feature = -1;
+            c.left = -1;
+            c.pad = 0;
+            c.thr = 0.0;
+            c.drss = 0.0;
+            c.count = best.nl;
+            c.value = __ddiv_rn(sl, (double)best.nl);
+            recs[lid] = c;
+            c.count = nr;
+            c.value = __ddiv_rn(sr, (double)nr);
+            recs[lid + 1] = c;
+            nd.split = 1;
+            nd.lid = lid;
+            nd.al = al;
+            nd.nl = best.nl;
+            nd.Sl = best.Sl;
+            nd.kind[0] = (best.nl <= g.nodesize || al < 2) ? KIND_LEAF : (al <= TINY ? KIND_SMALL : KIND_LARGE);
+            nd.kind[1] = (nr <= g.nodesize || ar < 2) ? KIND_LEAF : (ar <= TINY ? KIND_SMALL : KIND_LARGE);
+            curl[i] = nd;
+          }
+        } else if (lane == 0) {
+          curl[i].split = 0;
+        }
+      }
+      __syncthreads();
+    }
+    // ---- next medium level (block scan) and tiny queue (atomic append)
+    {
+      int kc = 0;
+      MNode nd;
+      if (tid < ncur) {
+        nd = curl[tid];
+        if (nd.split) kc = (nd.kind[0] == KIND_LARGE) + (nd.kind[1] == KIND_LARGE);
+      }
+      int totc;
+      int idx = block_excl_scan(kc, s_scan, totc);
+      if (tid < ncur && nd.split) {
+        for (int sdv = 0; sdv < 2; ++sdv) {
+          const int kd = nd.kind[sdv];
+          if (kd == KIND_LEAF) continue;
+          const int lo = sdv ? nd.lo + nd.al : nd.lo;
+          const int a = sdv ? nd.a - nd.al : nd.al;
+          const int nn = sdv ? nd.n - nd.nl : nd.nl;
+          const int64_t S = sdv ? nd.S - nd.Sl : nd.Sl;
+          const uint64_t key = sdv ? nd.keyr : nd.keyl;
+          if (kd == KIND_LARGE) {
+            MNode c;
+            c.lo = lo;
+            c.a = a;
+            c.n = nn;
+            c.id = nd.lid + sdv;
+            c.S = S;
+            c.key = key;
+            c.split = 0;
+            nxtl[idx++] = c;
+          } else {
+            TNode c;
+            c.lo = lo;
+            c.a = a;
+            c.n = nn;
+            c.id = nd.lid + sdv;
+            c.S = S;
+            c.key = key;
+            tq[atomicAdd(&s_qtail, 1)] = c;
+          }
+        }
+      }
+      if (tid == 0) s_ncur = totc;
+    }
+    // ---- in-place stable partition of the node ranges: every feature row if a child stays
+    //      medium, feature 0's row (the row list) if a child is tiny
+    for (int it = wid; it < ncur * p; it += SUB_NW) {
+      const int i = it / p, f = it - i * p;
+      const MNode& nd = curl[i];
+      if (!nd.split) continue;
+      const bool med = nd.kind[0] == KIND_LARGE || nd.kind[1] == KIND_LARGE;
+      const bool tiny = nd.kind[0] == KIND_SMALL || nd.kind[1] == KIND_SMALL;
+      if (!(med || (tiny && f == 0))) continue;
+      uint32_t* seg = list + (size_t)f * a0 + nd.lo;
+      const int al = nd.al;
+      int carry = 0;
+      for (int j0 = 0; j0 < nd.a; j0 += 32) {
+        const int j = j0 + lane;
+        const bool valid = j < nd.a;
+        const uint32_t e = valid ? seg[j] : 0u;
+        const int sdv = valid ? side[e & 0xffffu] : 1;
+        const unsigned m = __ballot_sync(0xffffffffu, valid && sdv == 0);
+        const int lb = carry + __popc(m & ((1u << lane) - 1u));
+        if (valid) temp[sdv ? al + (j - lb) : lb] = e;
+        carry += __popc(m);
+      }
+      __syncwarp();
+      for (int j = lane; j < nd.a; j += 32) seg[j] = temp[j];
+      __syncwarp();
+    }
+    __syncthreads();
+    {
+      MNode* tl = curl;
+      curl = nxtl;
+      nxtl = tl;
+    }
+  }
+
+  // ================= tiny nodes: one warp per node, depth-first, lanes = rows
+  {
+    TNode* stk = stacks + (size_t)wid * (TINY + 2);
+    const int qtail = s_qtail;
+    for (;;) {
+      int qi = 0;
+      if (lane == 0) qi = atomicAdd(&s_qhead, 1);
+      qi = __shfl_sync(0xffffffffu, qi, 0);
+      if (qi >= qtail) break;
+      if (lane == 0) stk[0] = tq[qi];
+      __syncwarp();
+      int sp = 1;
+      while (sp > 0) {
+        const TNode nd = stk[--sp];
+        __syncwarp();
+        const bool valid = lane < nd.a;
+        const uint32_t ent = valid ? list[nd.lo + lane] : 0u;  // feature 0's row = the row list
+        const uint32_t lrow = ent & 0xffffu;
+        const int32_t w = valid ? wl[lrow] : 0;
+        const int64_t wv = valid ? wy[lrow] : 0;
+        warp_draw_mtry(g.seed, t, nd.key, p, g.mtry, mind, feats, lane);
+        const int64_t nk = nd.n, Sk = nd.S;
+        double bg = -1.0;
+        int bf = 0x7fffffff;
+        uint32_t brk = 0;
+        int bnl = 0, bpos = 0;
+        int64_t bSl = 0;
+        uint32_t bra = 0, brb = 0;
+        for (int s = 0; s < g.mtry; ++s) {
+          const int f = feats[s];
+          const uint32_t rk0 = valid ? (uint32_t)R[(size_t)lrow * RS + f] : 0xffffu;
+          const uint32_t sk = bitonic_sort32((rk0 << 5) | (uint32_t)lane, lane);
+          const int srcl = (int)(sk & 31u);
+          const uint32_t rk = sk >> 5;
+          const int32_t ws = __shfl_sync(0xffffffffu, w, srcl);
+          const int64_t wys = __shfl_sync(0xffffffffu, wv, srcl);
+          const int32_t ic = warp_incl_scan(ws, lane);
+          const int64_t is = warp_incl_scan(wys, lane);
+          const uint32_t rkn = __shfl_down_sync(0xffffffffu, rk, 1);
+          double lg = -1.0;
+          if (lane + 1 < nd.a && rk != rkn && screen_may_win(nk, Sk, ic, is, bg)) lg = split_key(nk, Sk, ic, is);
+          // warp argmax (g desc, rank asc == lane asc)
+          double mg = lg;
+          int ml = lane;
+#pragma unroll
+          for (int o = 16; o > 0; o >>= 1) {
+            const double og = __shfl_down_sync(0xffffffffu, mg, o);
+            const int ol = __shfl_down_sync(0xffffffffu, ml, o);
+            if (lane + o < 32 && (og > mg || (og == mg && ol < ml))) {
+              mg = og;
+              ml = ol;
+            }
+          }
+          mg = __shfl_sync(0xffffffffu, mg, 0);
+          ml = __shfl_sync(0xffffffffu, ml, 0);
+          if (mg >= 0.0 && (mg > bg || (mg == bg && f < bf))) {
+            bg = mg;
+            bf = f;
+            bpos = ml;
+            brk = __shfl_sync(0xffffffffu, rk, ml);
+            bnl = __shfl_sync(0xffffffffu, ic, ml);
+            bSl = __shfl_sync(0xffffffffu, is, ml);
+            const int sa = __shfl_sync(0xffffffffu, srcl, ml);
+            const int sb = __shfl_sync(0xffffffffu, srcl, min(ml + 1, 31));
+            bra = __shfl_sync(0xffffffffu, lrow, sa);
+            brb = __shfl_sync(0xffffffffu, lrow, sb);
+          } else {
+            // keep every lane's copies uniform (the shuffles above are warp-uniform branches)
+          }
+        }
+        if (!(bg > 0.0)) continue;  // leaf: the record already holds count and value
+        // split
         int lid = 0;
         if (lane == 0) {
           const double xa = canon(g.X[(int64_t)bf * g.ldx + grow[bra]]);
@@ -967,24 +1321,19 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
           r.left = lid;
           r.thr = split_threshold(xa, xb);
           r.drss = ldexp(__ddiv_rn(bg, (double)nd.n), -2 * g.q);
-          nd.keyl = child_key(g.seed, t, nd.key, 0);
-          nd.keyr = child_key(g.seed, t, nd.key, 1);
         }
         lid = __shfl_sync(0xffffffffu, lid, 0);
-        // mark sides from the winning segment; child sums of w*y
-        const uint32_t* seg = cbuf + nd.off + (size_t)bf * nd.a;
-        double sl = 0.0, sr = 0.0;
-        for (int j = lane; j < nd.a; j += 32) {
-          const uint32_t lr = seg[j] & 0xffffu;
-          const int sdv = j > bpos;
-          side[lr] = (uint8_t)sdv;
-          if (sdv) sr += wyd[lr];
-          else sl += wyd[lr];
-        }
+        const bool right = valid && (uint32_t)R[(size_t)lrow * RS + bf] > brk;
+        const bool left = valid && !right;
+        const unsigned ml_ = __ballot_sync(0xffffffffu, left), mr_ = __ballot_sync(0xffffffffu, right);
+        const int al = __popc(ml_), ar = __popc(mr_);
+        const unsigned lt = (1u << lane) - 1u;
+        if (valid) list[nd.lo + (left ? __popc(ml_ & lt) : al + __popc(mr_ & lt))] = ent;
+        double vl = left ? wyd[lrow] : 0.0, vr = right ? wyd[lrow] : 0.0;
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) {
-          sl += __shfl_down_sync(0xffffffffu, sl, o);
-          sr += __shfl_down_sync(0xffffffffu, sr, o);
+          vl += __shfl_down_sync(0xffffffffu, vl, o);
+          vr += __shfl_down_sync(0xffffffffu, vr, o);
         }
         if (lane == 0) {
           const int nr = nd.n - bnl;
@@ -995,89 +1344,40 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
           c.thr = 0.0;
           c.drss = 0.0;
           c.count = bnl;
-          c.value = __ddiv_rn(sl, (double)bnl);
+          c.value = __ddiv_rn(vl, (double)bnl);
           recs[lid] = c;
           c.count = nr;
-          c.value = __ddiv_rn(sr, (double)nr);
+          c.value = __ddiv_rn(vr, (double)nr);
           recs[lid + 1] = c;
-          nd.split = 1;
-          nd.lid = lid;
-          nd.al = bpos + 1;
-          nd.nl = bnl;
-          nd.Sl = bSl;
-          curl[i] = nd;
-        }
-      } else if (lane == 0) {
-        curl[i].split = 0;
-      }
-      __syncwarp();
-    }
-    __syncthreads();
-    // ---- phase B: next-level list and child block offsets (serial, tiny)
-    if (tid == 0) {
-      int nn = 0, off = 0;
-      for (int i = 0; i < ncur; ++i) {
-        SCur& nd = curl[i];
-        nd.coff[0] = nd.coff[1] = -1;
-        if (!nd.split) continue;
-        for (int sdv = 0; sdv < 2; ++sdv) {
-          const int ac = sdv ? nd.a - nd.al : nd.al;
-          const int nc = sdv ? nd.n - nd.nl : nd.nl;
-          if (nc > g.nodesize && ac >= 2) {
-            SCur c;
-            c.off = off;
-            c.a = ac;
-            c.n = nc;
-            c.id = nd.lid + sdv;
-            c.S = sdv ? nd.S - nd.Sl : nd.Sl;
-            c.key = sdv ? nd.keyr : nd.keyl;
-            c.split = 0;
-            nxtl[nn++] = c;
-            nd.coff[sdv] = off;
-            off += p * ac;
+          const uint64_t kl = child_key(g.seed, t, nd.key, 0), kr = child_key(g.seed, t, nd.key, 1);
+          // push right first so the left subtree is processed next (any order is valid)
+          if (nr > g.nodesize && ar >= 2) {
+            TNode c2;
+            c2.lo = nd.lo + al;
+            c2.a = ar;
+            c2.n = nr;
+            c2.id = lid + 1;
+            c2.S = nd.S - bSl;
+            c2.key = kr;
+            stk[sp] = c2;
+          }
+          if (bnl > g.nodesize && al >= 2) {
+            TNode c2;
+            c2.lo = nd.lo;
+            c2.a = al;
+            c2.n = bnl;
+            c2.id = lid;
+            c2.S = bSl;
+            c2.key = kl;
+            stk[sp + ((nr > g.nodesize && ar >= 2) ? 1 : 0)] = c2;
           }
         }
-      }
-      s_ncur = nn;
-    }
-    __syncthreads();
-    // ---- phase C: stable partition of every feature list of every split node
-    for (int it = wid; it < ncur * p; it += SUB_NW) {
-      const int i = it / p, f = it - i * p;
-      const SCur& nd = curl[i];
-      if (!nd.split || (nd.coff[0] < 0 && nd.coff[1] < 0)) continue;
-      const uint32_t* seg = cbuf + nd.off + (size_t)f * nd.a;
-      const int al = nd.al, ar = nd.a - nd.al;
-      int carry = 0;
-      for (int j0 = 0; j0 < nd.a; j0 += 32) {
-        const int j = j0 + lane;
-        const bool valid = j < nd.a;
-        const uint32_t e = valid ? seg[j] : 0u;
-        const int sdv = valid ? side[e & 0xffffu] : 1;
-        const unsigned m = __ballot_sync(0xffffffffu, valid && sdv == 0);
-        const int lb = carry + __popc(m & ((1u << lane) - 1u));
-        if (valid) {
-          const int co = nd.coff[sdv];
-          if (co >= 0) {
-            const int idx = sdv ? j - lb : lb;
-            nbuf[co + (size_t)f * (sdv ? ar : al) + idx] = e;
-          }
-        }
-        carry += __popc(m);
+        sp += ((nd.n - bnl) > g.nodesize && ar >= 2) + (bnl > g.nodesize && al >= 2);
+        __syncwarp();
       }
     }
-    __syncthreads();
-    // ---- swap
-    {
-      uint32_t* tb = cbuf;
-      cbuf = nbuf;
-      nbuf = tb;
-      SCur* tl = curl;
-      curl = nxtl;
-      nxtl = tl;
-    }
-    __syncthreads();
   }
+  __syncthreads();
   // ---- flush the subtree into the tree's raw pool (sibling pairs stay adjacent)
   if (tid == 0) s_gbase = s_nloc > 1 ? atomicAdd(&g.pool.nn[b], s_nloc - 1) : 0;
   __syncthreads();
@@ -1288,12 +1588,11 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
   }
 
   // ---- sizing: subtree capacity A and trees in flight B
-  const int smax = max_optin_smem();
+  const int smax = dyn_smem_limit(k_subtree);
   int A = 2;
-  while (A < 4096 && subtree_smem(A + 1, p) <= (size_t)smax) ++A;
+  while (A < 1024 && subtree_smem(A + 1, p) <= (size_t)smax) ++A;  // load 2 holds <= 32 chunks of 32
   BF_REQUIRE(subtree_smem(2, p) <= (size_t)smax, BF_ENOTIMPL, "bf_fit: p too large for the shared-memory subtree kernel");
   if (prm.small_node_max > 0) A = std::max(2, std::min(A, prm.small_node_max));
-  BF_CUDA_CHECK(cudaFuncSetAttribute(k_subtree, cudaFuncAttributeMaxDynamicSharedMemorySize, smax));
 
   const int32_t T_loc = prm.tree_end - prm.tree_begin;
   const int64_t cap_nodes = 2 * n + 1;

@@ -332,7 +332,7 @@ void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, co
   DBuf<int32_t> w((size_t)B * n, s), cnt((size_t)B * nchunk, s);
   DBuf<uint32_t> O((size_t)B * n, s);
   const size_t smem = sizeof(double) * (size_t)p;
-  if (smem > 48 * 1024) BF_CUDA_CHECK(cudaFuncSetAttribute(k_importance, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  if (smem > 48 * 1024) BF_REQUIRE(smem <= (size_t)dyn_smem_limit(k_importance), BF_ENOTIMPL, "p too large");
   for (int32_t i0 = 0; i0 < T; i0 += B) {
     const int Bc = std::min(B, T - i0);
     bootstrap_impl(f->info.seed, f->info.tree_begin + i0, Bc, n, f->info.sampsize, f->info.replace, w.p, s);

@@ -273,11 +273,8 @@ void pca_impl(const double* X_in, int64_t ldx, int64_t n, int32_t p, int32_t sca
   }
   const int np = p * (p + 1) / 2;
   const size_t gsm = sizeof(double) * ((size_t)GR * p + np);
-  int dev = 0, smax = 0;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&smax, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+  const int smax = dyn_smem_limit(k_gram);
   BF_REQUIRE(gsm <= (size_t)smax, BF_ENOTIMPL, "bf_pca: p too large for the shared-memory Gram");
-  BF_CUDA_CHECK(cudaFuncSetAttribute(k_gram, cudaFuncAttributeMaxDynamicSharedMemorySize, smax));
   const int nparts = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, GR), 296));
   DBuf<double> part((size_t)nparts * np, s);
   {
@@ -291,8 +288,7 @@ void pca_impl(const double* X_in, int64_t ldx, int64_t n, int32_t p, int32_t sca
   BF_CUDA_CHECK(cudaGetLastError());
   const int P = p + (p & 1);
   const size_t jsm = sizeof(double) * (2 * (size_t)p * p + P) + sizeof(int) * P + 16;
-  BF_REQUIRE(jsm <= (size_t)smax, BF_ENOTIMPL, "bf_pca: p too large for the shared-memory Jacobi");
-  BF_CUDA_CHECK(cudaFuncSetAttribute(k_jacobi, cudaFuncAttributeMaxDynamicSharedMemorySize, smax));
+  BF_REQUIRE(jsm <= (size_t)dyn_smem_limit(k_jacobi), BF_ENOTIMPL, "bf_pca: p too large for the shared-memory Jacobi");
   {
     KScope ks_("k_jacobi", s, 0.0);
     k_jacobi<<<1, NT, jsm, s>>>(C.p, p, (double*)sdv.dptr, (double*)rot.dptr);

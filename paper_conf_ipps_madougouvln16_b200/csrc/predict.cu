@@ -90,12 +90,7 @@ void predict_impl(const bf_forest* f, const double* Xq_in, int64_t ldq, int64_t 
   const unsigned grid = (unsigned)ceil_div(m, PT);
   const size_t smem = sizeof(double) * (size_t)PT * (size_t)(p | 1);
   static int smax = 0;
-  if (!smax) {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&smax, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-    BF_CUDA_CHECK(cudaFuncSetAttribute(k_predict_smem, cudaFuncAttributeMaxDynamicSharedMemorySize, smax));
-  }
+  if (!smax) smax = dyn_smem_limit(k_predict_smem);
   DBuf<unsigned long long> vis;
   if (prof_enabled()) {
     vis.alloc(1, s);
