@@ -24,6 +24,9 @@
 #include <cub/cub.cuh>
 
 #include <algorithm>
+#include <cstdio>
+#include <ctime>
+#include <cstdlib>
 #include <cmath>
 #include <cstring>
 
@@ -38,11 +41,14 @@ constexpr int SUB_NW = 16;      // warps of the subtree kernel
 constexpr int SUB_NT = SUB_NW * 32;
 constexpr int KIND_NONE = -1, KIND_LEAF = 0, KIND_SMALL = 1, KIND_LARGE = 2;
 
-struct Pay {  // per (tree, row) payload: 16 B, one sector
-  int64_t wy;  // w * y_q (exact)
-  int32_t w;   // bootstrap multiplicity
-  int32_t pad;
-};
+// List entry (8 B): dense rank of the value (24 bits) | row (24 bits) | bootstrap
+// multiplicity w (16 bits).  Entries of a segment are kept in value order, so the
+// scan reads w from the entry and gathers only y_q[row] (one 8 MB array shared
+// by every tree: L2-resident) instead of a per-tree payload.
+__host__ __device__ __forceinline__ uint32_t e_rank(uint64_t e) { return (uint32_t)(e >> 40); }
+__host__ __device__ __forceinline__ uint32_t e_row(uint64_t e) { return (uint32_t)(e >> 16) & 0xffffffu; }
+__host__ __device__ __forceinline__ int32_t e_w(uint64_t e) { return (int32_t)(e & 0xffffu); }
+constexpr int64_t MAX_ROWS = int64_t(1) << 24;
 
 struct LNode {  // an active node of the global phase, or a queued small node
   int32_t b;     // tree index inside the batch
@@ -202,7 +208,7 @@ __global__ void k_fill_sorted(const double* col, const uint32_t* rows, const uin
                               uint64_t* srt, double* uniq) {
   for (int64_t i = blockIdx.x * (int64_t)NT + threadIdx.x; i < n; i += (int64_t)gridDim.x * NT) {
     const uint32_t r = rows[i], k = rank[i];
-    srt[i] = ((uint64_t)k << 32) | r;
+    srt[i] = ((uint64_t)k << 40) | ((uint64_t)r << 16);
     if (i == 0 || rank[i - 1] != k) uniq[k] = canon(col[r]);
   }
 }
@@ -225,7 +231,7 @@ __global__ void k_fill_i32(int32_t* a, int64_t count, int32_t v) {
 }
 
 // payload + per-tree root sums: a (distinct), S (exact), sum w*y (fp64)
-__global__ void k_payload(const int32_t* w, const int64_t* yq, const double* y, int64_t n, Pay* pay,
+__global__ void k_payload(const int32_t* w, const int64_t* yq, const double* y, int64_t n, int32_t* wmax,
                           int32_t* a_root, unsigned long long* S_root, double* sy_root) {
   __shared__ int32_t sa[NT / 32];
   __shared__ int64_t sS[NT / 32];
@@ -239,11 +245,7 @@ __global__ void k_payload(const int32_t* w, const int64_t* yq, const double* y, 
     wi = w[(int64_t)b * n + i];
     wyq = (int64_t)wi * yq[i];
     wy = __dmul_rn((double)wi, y[i]);
-    Pay pp;
-    pp.wy = wyq;
-    pp.w = wi;
-    pp.pad = 0;
-    pay[(int64_t)b * n + i] = pp;
+    if (wi > 0xffff) atomicMax(wmax, wi);
   }
   int32_t ca = wi > 0;
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -303,17 +305,17 @@ __global__ void k_roots(int B, int64_t ns, int nodesize, const int32_t* a_root, 
 // ------------------------------------------------------------------ a5 root lists (two-pass stable compaction)
 constexpr int LCH = 2048;  // entries per CTA chunk (256 threads x 8)
 
-__global__ void k_list_count(const uint64_t* srt, int64_t n, const Pay* pay, const int32_t* kind, int nchunk,
+__global__ void k_list_count(const uint64_t* srt, int64_t n, const int32_t* wts, const int32_t* kind, int nchunk,
                              int32_t* cnt) {
   const int c = blockIdx.x, f = blockIdx.y, b = blockIdx.z, p = gridDim.y;
   if (kind[b] != KIND_LARGE && kind[b] != KIND_SMALL) return;
   __shared__ int32_t sm[NT / 32];
   const uint64_t* col = srt + (int64_t)f * n;
-  const Pay* P = pay + (int64_t)b * n;
+  const int32_t* W = wts + (int64_t)b * n;
   int32_t k = 0;
   for (int u = threadIdx.x; u < LCH; u += NT) {
     const int64_t i = (int64_t)c * LCH + u;
-    if (i < n) k += P[(uint32_t)col[i]].w > 0;
+    if (i < n) k += W[e_row(col[i])] > 0;
   }
   int32_t tot;
   block_excl_scan(k, sm, tot);
@@ -332,7 +334,7 @@ __global__ void k_list_prefix(int32_t* cnt, int nseg, int nchunk) {
   }
 }
 
-__global__ void k_list_scatter(const uint64_t* srt, int64_t n, const Pay* pay, const int32_t* kind,
+__global__ void k_list_scatter(const uint64_t* srt, int64_t n, const int32_t* wts, const int32_t* kind,
                                const int64_t* base, const int32_t* a_root, int nchunk, const int32_t* cnt,
                                uint64_t* Elarge, uint64_t* Esmall) {
   const int c = blockIdx.x, f = blockIdx.y, b = blockIdx.z, p = gridDim.y;
@@ -340,7 +342,7 @@ __global__ void k_list_scatter(const uint64_t* srt, int64_t n, const Pay* pay, c
   if (kd != KIND_LARGE && kd != KIND_SMALL) return;
   __shared__ int32_t sm[NT / 32];
   const uint64_t* col = srt + (int64_t)f * n;
-  const Pay* P = pay + (int64_t)b * n;
+  const int32_t* W = wts + (int64_t)b * n;
   constexpr int V = LCH / NT;
   uint64_t e[V];
   bool keep[V];
@@ -352,7 +354,9 @@ __global__ void k_list_scatter(const uint64_t* srt, int64_t n, const Pay* pay, c
     keep[u] = false;
     if (i < n) {
       e[u] = col[i];
-      keep[u] = P[(uint32_t)e[u]].w > 0;
+      const int32_t wv = W[e_row(e[u])];
+      keep[u] = wv > 0;
+      e[u] |= (uint64_t)(uint32_t)wv;
     }
     k += keep[u];
   }
@@ -397,21 +401,39 @@ __device__ __forceinline__ bool rec_better(double g, uint32_t r, double bg, uint
   return g > bg || (g == bg && r < br);
 }
 
-// fp32 screen of a candidate against the running best key: true unless the
-// candidate's exact key is certainly below `best` (relative error of the
-// screen < 2^-20; candidates that might round to >= best take the exact path).
+// Screen of a candidate against the running best key, in fp64 with a
+// rigorous bound (no int128): d = RN(RN(nk*Sl) - RN(nl*Sk)) satisfies
+// |d - D| <= 2^-50 (|nk*Sl| + |nl*Sk|), so gU = (|d| + E)^2 * rcp(nn) * (1 + 2^-20)
+// bounds the exact D^2/(nl*nr) from above.  Returns false only if the
+// correctly rounded key of S4.3 is certainly below `best`.
 __device__ __forceinline__ bool screen_may_win(int64_t nk, int64_t Sk, int64_t nl, int64_t Sl, double best) {
   if (best <= 0.0) return true;
-  const __int128 D = (__int128)nk * (__int128)Sl - (__int128)nl * (__int128)Sk;
-  const double d = (double)(float)(double)D;  // coarse but monotone-safe within 2^-22 relative
+  const double a = (double)nk * (double)Sl, bb = (double)nl * (double)Sk;
+  const double d = fabs(a - bb);
+  const double E = (fabs(a) + fabs(bb)) * 8.881784197001252e-16;  // 2^-50
+  const double u = (d + E) * (1.0 + 8.881784197001252e-16);
   const double nn = (double)(nl * (nk - nl));
-  const double gapprox = d * d * (double)__frcp_rn((float)nn);
-  return gapprox >= best * (1.0 - 1.0 / (1 << 18));
+  const double gU = u * u * (double)__frcp_rn((float)nn) * (1.0 + 9.5367431640625e-07);  // (1 + 2^-20)
+  return gU >= best;
 }
+
+// Warp argmax of (key desc, tie asc) with 64-bit keys (0 = no candidate):
+// returns the winning lane (or -1).  key = bits(g) + 1 for a candidate with
+// key g >= 0, which preserves the order of non-negative doubles.
+__device__ __forceinline__ int warp_argmax_key(uint64_t key, uint32_t tie) {
+  const uint32_t hi = (uint32_t)(key >> 32), lo = (uint32_t)key;
+  const uint32_t mh = __reduce_max_sync(0xffffffffu, hi);
+  const uint32_t ml = __reduce_max_sync(0xffffffffu, hi == mh ? lo : 0u);
+  if (mh == 0 && ml == 0) return -1;
+  const bool top = hi == mh && lo == ml;
+  const uint32_t mt = __reduce_min_sync(0xffffffffu, top ? tie : 0xffffffffu);
+  return __ffs(__ballot_sync(0xffffffffu, top && tie == mt)) - 1;
+}
+__device__ __forceinline__ uint64_t gkey(double g) { return g >= 0.0 ? (uint64_t)__double_as_longlong(g) + 1ull : 0ull; }
 
 
 __global__ void __launch_bounds__(NT) k_split_scan(const LNode* nodes, const int32_t* feat, int mtry,
-                                                   const uint64_t* E, const Pay* pay, int64_t n, Rec* rec) {
+                                                   const uint64_t* E, const int64_t* yq, Rec* rec) {
   __shared__ int32_t smc[NT / 32];
   __shared__ int64_t sms[NT / 32];
   __shared__ double sg[NT / 32];
@@ -421,7 +443,6 @@ __global__ void __launch_bounds__(NT) k_split_scan(const LNode* nodes, const int
   const LNode nd = nodes[item / mtry];
   const int f = feat[item];
   const uint64_t* seg = E + nd.base + (int64_t)f * nd.a;
-  const Pay* P = pay + (int64_t)nd.b * n;
   const int a = nd.a;
   const int64_t nk = nd.n, Sk = nd.S;
   int32_t carry_c = 0;
@@ -444,9 +465,8 @@ __global__ void __launch_bounds__(NT) k_split_scan(const LNode* nodes, const int
       wc[u] = 0;
       ws[u] = 0;
       if (j0 + u < a) {
-        const Pay pp = P[(uint32_t)e[u]];
-        wc[u] = pp.w;
-        ws[u] = pp.wy;
+        wc[u] = e_w(e[u]);
+        ws[u] = (int64_t)wc[u] * __ldg(yq + e_row(e[u]));
       }
       tc += wc[u];
       ts += ws[u];
@@ -461,7 +481,7 @@ __global__ void __launch_bounds__(NT) k_split_scan(const LNode* nodes, const int
       pres += ws[u];
       const int j = j0 + u;
       if (j + 1 < a) {
-        const uint32_t ra = (uint32_t)(e[u] >> 32), rb = (uint32_t)(e[u + 1] >> 32);
+        const uint32_t ra = e_rank(e[u]), rb = e_rank(e[u + 1]);
         if (ra != rb && screen_may_win(nk, Sk, prec, pres, bg)) {
           const double g = split_key(nk, Sk, prec, pres);
           if (rec_better(g, ra, bg, brank)) {
@@ -647,7 +667,7 @@ __global__ void k_commit(int N2, const uint64_t* packL, const uint64_t* scanL, c
 
 // ------------------------------------------------------------------ a9/a10 goes-right flags + child values
 __global__ void __launch_bounds__(NT) k_dest(const LNode* nodes, const Split* split, const uint64_t* E,
-                                             const Pay* pay, const double* y, int64_t n, uint8_t* side,
+                                             const double* y, int64_t n, uint8_t* side,
                                              Pool pool) {
   __shared__ double sl[NT], sr[NT];
   const int k = blockIdx.x;
@@ -655,14 +675,14 @@ __global__ void __launch_bounds__(NT) k_dest(const LNode* nodes, const Split* sp
   if (!sp.split) return;
   const LNode nd = nodes[k];
   const uint64_t* seg = E + nd.base + (int64_t)sp.f * nd.a;
-  const Pay* P = pay + (int64_t)nd.b * n;
   uint8_t* sd = side + (int64_t)nd.b * n;
   double accl = 0.0, accr = 0.0;
   for (int j = threadIdx.x; j < nd.a; j += NT) {
-    const uint32_t row = (uint32_t)seg[j];
+    const uint64_t ej = seg[j];
+    const uint32_t row = e_row(ej);
     const int s = j > sp.pos;
     sd[row] = (uint8_t)s;
-    const double v = __dmul_rn((double)P[row].w, y[row]);
+    const double v = __dmul_rn((double)e_w(ej), y[row]);
     if (s) accr += v;
     else accl += v;
   }
@@ -684,7 +704,7 @@ __global__ void __launch_bounds__(NT) k_dest(const LNode* nodes, const Split* sp
 }
 
 // ------------------------------------------------------------------ a9 partition
-constexpr int PV = 4;
+constexpr int PV = 8;
 constexpr int PCH = NT * PV;
 
 __global__ void __launch_bounds__(NT) k_partition(const LNode* nodes, const Split* split, const Child* child,
@@ -715,7 +735,7 @@ __global__ void __launch_bounds__(NT) k_partition(const LNode* nodes, const Spli
       left[u] = false;
       if (j0 + u < nd.a) {
         e[u] = seg[j0 + u];
-        left[u] = sd[(uint32_t)e[u]] == 0;
+        left[u] = sd[e_row(e[u])] == 0;
       }
       cnt += left[u];
     }
@@ -739,17 +759,23 @@ __global__ void __launch_bounds__(NT) k_partition(const LNode* nodes, const Spli
 
 // ------------------------------------------------------------------ subtree phase (one CTA per small node)
 // Layout: the subtree's rows occupy local ids 0..a0-1.  list[f][0..a0) holds
-// feature f's entries ((local rank << 16) | local row) sorted by value; every
-// node owns the same column range [lo, lo+a) in every feature row, and a split
-// partitions each row's range in place (left part first), so children ranges
-// nest.  R[row][f] = local rank (index of the first entry of the row's value)
-// lets a warp evaluate a tiny node (a <= 32: one lane per row) by sorting the
-// 32 ranks in registers instead of maintaining p partitioned lists.
-constexpr int TINY = 32;
+// feature f's entries ((local rank << 16) | local row) sorted by value.  A
+// MEDIUM node (a > TINY) owns the same column range [lo, lo+a) in every
+// feature row; its split partitions each row's range in place (left part
+// first), so children ranges nest.  A TINY root (a <= TINY) keeps its range
+// [rlo, rlo+ra); its descendants are bit masks over the root's rows (bit =
+// index of the row inside the root), evaluated by one warp with lane k
+// holding the k-th entry of the root's sorted segment -- the node's rows in
+// feature order are the lanes whose row bit is set, so no per-node sort or
+// list partition is needed.  Tiny nodes go through a CTA-wide work queue so
+// every warp stays busy until the whole subtree is grown.
+constexpr int TINY = 64;
+constexpr int TGRP = 4;   // drawn predictors staged per group in the tiny path
 
-struct SRec {  // node record of a subtree (local ids)
-  int32_t feature, left, count, pad;
-  double thr, value, drss;
+struct SRec {  // node record of a subtree (local ids); thr is computed at flush from rows (ra, rb)
+  int32_t feature, left, count;
+  uint16_t ra, rb;
+  double value, drss;
 };
 struct MNode {  // medium node (a > TINY) of a subtree level
   int32_t lo, a, n, id;
@@ -760,8 +786,11 @@ struct MNode {  // medium node (a > TINY) of a subtree level
   uint64_t keyl, keyr;
   int32_t kind[2];
 };
-struct TNode {  // tiny node (a <= TINY)
-  int32_t lo, a, n, id;
+struct TNode {  // tiny node: mask over the rows of its tiny root [rlo, rlo+ra)
+  int32_t rlo, ra;
+  uint64_t mask;
+  int32_t id;
+  int32_t n;           // written last: n > 0 marks the entry as ready
   int64_t S;
   uint64_t key;
 };
@@ -775,27 +804,21 @@ struct WRec {  // best candidate found by one warp for its share of a node's fea
 };
 
 __host__ __device__ inline size_t align16(size_t x) { return (x + 15) & ~size_t(15); }
-__host__ __device__ inline int rank_stride(int p) {  // u16 row stride of R: 2*(odd) -> conflict-free columns
-  int rs = (p + 1) & ~1;
-  if (((rs >> 1) & 1) == 0) rs += 2;
-  return rs;
-}
 __host__ __device__ inline int max_medium(int A) { return A / (TINY + 1) + 2; }
 
 __host__ __device__ inline size_t subtree_smem(int A, int p) {
   size_t s = 0;
   s += align16((size_t)p * A * 4);                    // list
-  s += align16((size_t)A * rank_stride(p) * 2);       // R
   s += align16((size_t)SUB_NW * A * 4);               // per-warp partition temp
   s += align16((size_t)A * 8) * 2;                    // wy, w*y
   s += align16((size_t)A * 4) * 2;                    // w, global row
-  s += align16((size_t)A);                            // side
+  s += align16((size_t)A) * 2;                        // side, row index inside its tiny root
   s += align16((size_t)2 * A * sizeof(SRec));         // node records
   s += align16((size_t)2 * max_medium(A) * sizeof(MNode));
-  s += align16((size_t)(A / 2 + 1) * sizeof(TNode));  // tiny queue
-  s += align16((size_t)SUB_NW * (TINY + 2) * sizeof(TNode));  // DFS stacks
+  s += align16((size_t)(A + 1) * sizeof(TNode));      // tiny work queue
   s += align16((size_t)SUB_NW * p * 2) * 2;           // Fisher-Yates scratch, drawn features
   s += align16((size_t)SUB_NW * sizeof(WRec));
+  s += align16((size_t)SUB_NW * TGRP * TINY * 4);     // tiny staging
   s += 64;
   return s;
 }
@@ -803,7 +826,7 @@ __host__ __device__ inline size_t subtree_smem(int A, int p) {
 struct SubArgs {
   const LNode* sq;
   const uint64_t* Es;
-  const Pay* pay;
+  const int64_t* yq;
   const double* y;
   const double* X;
   int64_t ldx;
@@ -813,60 +836,57 @@ struct SubArgs {
   int32_t t0;
   uint16_t* loc;
   Pool pool;
+  unsigned long long* stats;  // optional phase counters (BF_SUBTREE_STATS=1), else NULL
 };
 
-// S4.2 mtry draw by one warp: Philox words computed by the lanes, the
-// partial Fisher-Yates swaps applied by lane 0 in shared memory.
-__device__ __forceinline__ void warp_draw_mtry(uint64_t seed, uint32_t t, uint64_t key, int p, int mtry, int16_t* mind,
+// S4.2 mtry draw by one warp, in parallel.  Draw i picks position
+// j_i = mulhi64(U_i, p - i) of the current array, then swaps positions j_i
+// and p-1-i.  The content of position x after draws 0..i-1 is found by
+// tracing the swaps backwards (x <- p-1-k if x == j_k, x <- j_k if
+// x == p-1-k, for k = i-1 .. 0), so lane i computes feature i on its own
+// from the j values of the earlier draws (kept in shared memory).
+__device__ __forceinline__ void warp_draw_mtry(uint64_t seed, uint32_t t, uint64_t key, int p, int mtry, int16_t* jbuf,
                                                int16_t* feats, int lane) {
-  for (int j = lane; j < p; j += 32) mind[j] = (int16_t)j;
+  for (int i0 = 0; i0 < mtry; i0 += 32) {
+    const int i = i0 + lane;
+    if (i < mtry) {
+      uint64_t u0, u1;
+      philox_u64x2(seed, (uint32_t)key, (uint32_t)(key >> 32), t, 0x20000000u | (uint32_t)(i >> 1), u0, u1);
+      jbuf[i] = (int16_t)mulhi64((i & 1) ? u1 : u0, (uint64_t)(p - i));
+    }
+  }
   __syncwarp();
-  int last = p - 1;
-  for (int c0 = 0; c0 < mtry; c0 += 64) {
-    uint64_t u0 = 0, u1 = 0;
-    const int call = (c0 >> 1) + lane;
-    if (2 * call < mtry) philox_u64x2(seed, (uint32_t)key, (uint32_t)(key >> 32), t, 0x20000000u | (uint32_t)call, u0, u1);
-    const int cend = min(mtry, c0 + 64);
-    for (int s = c0; s < cend; ++s) {
-      const int sl = (s - c0) >> 1;
-      const uint64_t ua = __shfl_sync(0xffffffffu, u0, sl);
-      const uint64_t ub = __shfl_sync(0xffffffffu, u1, sl);
-      if (lane == 0) {
-        const uint64_t u = (s & 1) ? ub : ua;
-        const int j = (int)mulhi64(u, (uint64_t)(last + 1));
-        feats[s] = mind[j];
-        const int16_t tmp = mind[j];
-        mind[j] = mind[last];
-        mind[last] = tmp;
+  for (int i0 = 0; i0 < mtry; i0 += 32) {
+    const int i = i0 + lane;
+    if (i < mtry) {
+      int x = jbuf[i];
+      for (int k = i - 1; k >= 0; --k) {
+        const int jk = jbuf[k], lk = p - 1 - k;
+        x = (x == jk) ? lk : ((x == lk) ? jk : x);
       }
-      --last;
+      feats[i] = (int16_t)x;
     }
   }
   __syncwarp();
 }
 
-__device__ __forceinline__ uint32_t bitonic_sort32(uint32_t key, int lane) {
-#pragma unroll
-  for (int k = 2; k <= 32; k <<= 1) {
-#pragma unroll
-    for (int j = k >> 1; j > 0; j >>= 1) {
-      const uint32_t o = __shfl_xor_sync(0xffffffffu, key, j);
-      const bool up = (lane & k) == 0;
-      const bool lower = (lane & j) == 0;
-      key = (lower == up) ? min(key, o) : max(key, o);
-    }
-  }
-  return key;
+__device__ __forceinline__ void tq_push(TNode* q, int* alloc, int* pending, const TNode& nd) {
+  atomicAdd(pending, 1);
+  const int idx = atomicAdd(alloc, 1);
+  TNode c = nd;
+  const int32_t n = c.n;
+  c.n = 0;
+  q[idx] = c;
+  __threadfence_block();
+  *(volatile int32_t*)&q[idx].n = n;
 }
 
 __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   extern __shared__ __align__(16) unsigned char smem[];
-  const int A = g.A, p = g.p, RS = rank_stride(p), MM = max_medium(A);
+  const int A = g.A, p = g.p, MM = max_medium(A);
   unsigned char* ptr = smem;
   uint32_t* list = (uint32_t*)ptr;
   ptr += align16((size_t)p * A * 4);
-  uint16_t* R = (uint16_t*)ptr;
-  ptr += align16((size_t)A * RS * 2);
   uint32_t* temp_all = (uint32_t*)ptr;
   ptr += align16((size_t)SUB_NW * A * 4);
   int64_t* wy = (int64_t*)ptr;
@@ -879,21 +899,23 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   ptr += align16((size_t)A * 4);
   uint8_t* side = (uint8_t*)ptr;
   ptr += align16((size_t)A);
+  uint8_t* rmap = (uint8_t*)ptr;
+  ptr += align16((size_t)A);
   SRec* recs = (SRec*)ptr;
   ptr += align16((size_t)2 * A * sizeof(SRec));
   MNode* curl = (MNode*)ptr;
   MNode* nxtl = curl + MM;
   ptr += align16((size_t)2 * MM * sizeof(MNode));
   TNode* tq = (TNode*)ptr;
-  ptr += align16((size_t)(A / 2 + 1) * sizeof(TNode));
-  TNode* stacks = (TNode*)ptr;
-  ptr += align16((size_t)SUB_NW * (TINY + 2) * sizeof(TNode));
+  ptr += align16((size_t)(A + 1) * sizeof(TNode));
   int16_t* mind_all = (int16_t*)ptr;
   ptr += align16((size_t)SUB_NW * p * 2);
   int16_t* feats_all = (int16_t*)ptr;
   ptr += align16((size_t)SUB_NW * p * 2);
   WRec* wrec = (WRec*)ptr;
-  __shared__ int s_nloc, s_ncur, s_gbase, s_qtail, s_qhead;
+  ptr += align16((size_t)SUB_NW * sizeof(WRec));
+  uint32_t* stg_all = (uint32_t*)ptr;
+  __shared__ int s_nloc, s_ncur, s_gbase, s_alloc, s_head, s_pending;
   __shared__ int32_t s_scan[SUB_NW];
 
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
@@ -901,23 +923,28 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   const int a0 = root.a;
   const int b = root.b;
   const uint32_t t = (uint32_t)(g.t0 + b);
-  const Pay* P = g.pay + (int64_t)b * g.n;
   uint16_t* loc = g.loc + (int64_t)b * g.n;
   const uint64_t* src = g.Es + root.base;
   int16_t* mind = mind_all + wid * p;
   int16_t* feats = feats_all + wid * p;
   uint32_t* temp = temp_all + (size_t)wid * A;
+  long long tclk[5];
+  tclk[0] = clock64();
+  int n_med = 0, n_tiny = 0;
+  long long busy = 0;
 
   // ---- load 1: local rows = feature 0's order; payload; global row -> local id
   for (int j = tid; j < a0; j += SUB_NT) {
-    const uint32_t row = (uint32_t)src[j];
+    const uint64_t ej = src[j];
+    const uint32_t row = e_row(ej);
+    const int32_t wv = e_w(ej);
     grow[j] = row;
     loc[row] = (uint16_t)j;
-    const Pay pp = P[row];
-    wl[j] = pp.w;
-    wy[j] = pp.wy;
-    wyd[j] = __dmul_rn((double)pp.w, g.y[row]);
+    wl[j] = wv;
+    wy[j] = (int64_t)wv * g.yq[row];
+    wyd[j] = __dmul_rn((double)wv, g.y[row]);
   }
+  for (int j = tid; j <= a0; j += SUB_NT) tq[j].n = 0;
   __syncthreads();
   // ---- load 2: warp per feature; local rank = index of the first entry of the same value
   {
@@ -934,8 +961,8 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         for (int c = 0; c < GRP; ++c) {
           const int j = (c0 + c) * 32 + lane;
           const uint64_t e = j < a0 ? sf[j] : ~0ull;
-          rk[c] = (uint32_t)(e >> 32);
-          lr[c] = j < a0 ? loc[(uint32_t)e] : 0;
+          rk[c] = j < a0 ? e_rank(e) : 0xffffffffu;
+          lr[c] = j < a0 ? loc[e_row(e)] : 0;
         }
 #pragma unroll
         for (int c = 0; c < GRP; ++c) {
@@ -950,10 +977,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
             if (lane >= o) gs = max(gs, v);
           }
           gs = max(gs, carry_gs);
-          if (j < a0) {
-            list[(size_t)f * a0 + j] = ((uint32_t)gs << 16) | lr[c];
-            R[(size_t)lr[c] * RS + f] = (uint16_t)gs;
-          }
+          if (j < a0) list[(size_t)f * a0 + j] = ((uint32_t)gs << 16) | lr[c];
           carry_gs = __shfl_sync(0xffffffffu, gs, 31);
           prev_last = __shfl_sync(0xffffffffu, rk[c], 31);
         }
@@ -962,13 +986,14 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   }
   if (tid == 0) {
     s_nloc = 1;
-    s_qhead = 0;
+    s_head = 0;
+    s_alloc = 0;
+    s_pending = 0;
     SRec r0;
     r0.feature = -1;
     r0.left = -1;
     r0.count = root.n;
-    r0.pad = 0;
-    r0.thr = 0.0;
+    r0.ra = r0.rb = 0;
     r0.value = 0.0;
     r0.drss = 0.0;
     recs[0] = r0;
@@ -983,25 +1008,29 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       c.split = 0;
       curl[0] = c;
       s_ncur = 1;
-      s_qtail = 0;
     } else {
-      TNode c;
-      c.lo = 0;
-      c.a = a0;
-      c.n = root.n;
-      c.id = 0;
-      c.S = root.S;
-      c.key = root.key;
-      tq[0] = c;
       s_ncur = 0;
-      s_qtail = 1;
     }
   }
   __syncthreads();
+  if (a0 <= TINY && tid == 0) {
+    TNode c;
+    c.rlo = 0;
+    c.ra = a0;
+    c.mask = a0 == 64 ? ~0ull : ((1ull << a0) - 1ull);
+    c.id = 0;
+    c.n = root.n;
+    c.S = root.S;
+    c.key = root.key;
+    tq_push(tq, &s_alloc, &s_pending, c);
+  }
+  __syncthreads();
+  tclk[1] = clock64();
 
   // ================= medium levels (a > TINY): level-synchronous inside the CTA
   while (s_ncur > 0) {
     const int ncur = s_ncur;
+    n_med += ncur;
     int G = 1;
     while (G * 2 * ncur <= SUB_NW) G *= 2;
     const int ngroups = SUB_NW / G, group = wid / G, sub = wid - group * G;
@@ -1053,21 +1082,9 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
             cc = __shfl_sync(0xffffffffu, ic, 31);
             cs = __shfl_sync(0xffffffffu, is, 31);
           }
-          int srcl = lane;
-#pragma unroll
-          for (int o = 16; o > 0; o >>= 1) {
-            const double og = __shfl_down_sync(0xffffffffu, lg, o);
-            const uint32_t orr = __shfl_down_sync(0xffffffffu, lrk, o);
-            const int os = __shfl_down_sync(0xffffffffu, srcl, o);
-            if (lane + o < 32 && rec_better(og, orr, lg, lrk)) {
-              lg = og;
-              lrk = orr;
-              srcl = os;
-            }
-          }
-          srcl = __shfl_sync(0xffffffffu, srcl, 0);
-          lg = __shfl_sync(0xffffffffu, lg, 0);
-          lrk = __shfl_sync(0xffffffffu, lrk, 0);
+          const int srcl = max(warp_argmax_key(gkey(lg), lrk), 0);
+          lg = __shfl_sync(0xffffffffu, lg, srcl);
+          lrk = __shfl_sync(0xffffffffu, lrk, srcl);
           const int wpos = __shfl_sync(0xffffffffu, lpos, srcl);
           const int wnl = __shfl_sync(0xffffffffu, lnl, srcl);
           const int64_t wSl = __shfl_sync(0xffffffffu, lSl, srcl);
@@ -1107,13 +1124,12 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         if (best.g > 0.0) {
           int lid = 0;
           if (lane == 0) {
-            const double xa = canon(g.X[(int64_t)best.f * g.ldx + grow[best.ra]]);
-            const double xb = canon(g.X[(int64_t)best.f * g.ldx + grow[best.rb]]);
             lid = atomicAdd(&s_nloc, 2);
             SRec& r = recs[nd.id];
             r.feature = best.f;
             r.left = lid;
-            r.thr = split_threshold(xa, xb);
+            r.ra = (uint16_t)best.ra;
+            r.rb = (uint16_t)best.rb;
             r.drss = ldexp(__ddiv_rn(best.g, (double)nd.n), -2 * g.q);
             nd.keyl = child_key(g.seed, t, nd.key, 0);
             nd.keyr = child_key(g.seed, t, nd.key, 1);
@@ -1138,8 +1154,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
             SRec c;
             c.feature = -1;
             c.left = -1;
-            c.pad = 0;
-            c.thr = 0.0;
+            c.ra = c.rb = 0;
             c.drss = 0.0;
             c.count = best.nl;
             c.value = __ddiv_rn(sl, (double)best.nl);
@@ -1162,7 +1177,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       }
       __syncthreads();
     }
-    // ---- next medium level (block scan) and tiny queue (atomic append)
+    // ---- next medium level (block scan) and tiny roots (work queue; processed after the medium levels)
     {
       int kc = 0;
       MNode nd;
@@ -1193,27 +1208,24 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
             nxtl[idx++] = c;
           } else {
             TNode c;
-            c.lo = lo;
-            c.a = a;
-            c.n = nn;
+            c.rlo = lo;
+            c.ra = a;
+            c.mask = a == 64 ? ~0ull : ((1ull << a) - 1ull);
             c.id = nd.lid + sdv;
+            c.n = nn;
             c.S = S;
             c.key = key;
-            tq[atomicAdd(&s_qtail, 1)] = c;
+            tq_push(tq, &s_alloc, &s_pending, c);
           }
         }
       }
       if (tid == 0) s_ncur = totc;
     }
-    // ---- in-place stable partition of the node ranges: every feature row if a child stays
-    //      medium, feature 0's row (the row list) if a child is tiny
+    // ---- in-place stable partition of every feature row of every split node with a non-leaf child
     for (int it = wid; it < ncur * p; it += SUB_NW) {
       const int i = it / p, f = it - i * p;
       const MNode& nd = curl[i];
-      if (!nd.split) continue;
-      const bool med = nd.kind[0] == KIND_LARGE || nd.kind[1] == KIND_LARGE;
-      const bool tiny = nd.kind[0] == KIND_SMALL || nd.kind[1] == KIND_SMALL;
-      if (!(med || (tiny && f == 0))) continue;
+      if (!nd.split || (nd.kind[0] == KIND_LEAF && nd.kind[1] == KIND_LEAF)) continue;
       uint32_t* seg = list + (size_t)f * a0 + nd.lo;
       const int al = nd.al;
       int carry = 0;
@@ -1239,109 +1251,173 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
     }
   }
 
-  // ================= tiny nodes: one warp per node, depth-first, lanes = rows
+  // ================= tiny nodes: row index inside each tiny root, then the work queue
+  tclk[2] = clock64();
   {
-    TNode* stk = stacks + (size_t)wid * (TINY + 2);
-    const int qtail = s_qtail;
-    for (;;) {
-      int qi = 0;
-      if (lane == 0) qi = atomicAdd(&s_qhead, 1);
-      qi = __shfl_sync(0xffffffffu, qi, 0);
-      if (qi >= qtail) break;
-      if (lane == 0) stk[0] = tq[qi];
-      __syncwarp();
-      int sp = 1;
-      while (sp > 0) {
-        const TNode nd = stk[--sp];
+    const int nroots = s_alloc;
+    for (int qi = wid; qi < nroots; qi += SUB_NW) {
+      const TNode& r = tq[qi];
+      for (int k = lane; k < r.ra; k += 32) rmap[list[r.rlo + k] & 0xffffu] = (uint8_t)k;
+    }
+  }
+  __syncthreads();
+  for (;;) {
+    int h = -1;
+    if (lane == 0) {
+      unsigned ns = 32;
+      for (;;) {
+        const int hd = *(volatile int*)&s_head;
+        if (hd < *(volatile int*)&s_alloc) {
+          if (atomicCAS(&s_head, hd, hd + 1) == hd) {
+            h = hd;
+            break;
+          }
+        } else if (*(volatile int*)&s_pending == 0) {
+          break;
+        } else {
+          __nanosleep(ns);
+          ns = min(ns * 2, 256);
+        }
+      }
+      if (h >= 0)
+        while (*(volatile int32_t*)&tq[h].n == 0) __nanosleep(32);
+      __threadfence_block();
+    }
+    h = __shfl_sync(0xffffffffu, h, 0);
+    if (h < 0) break;
+    TNode nd = tq[h];
+    bool have = true;
+    const long long tb0 = clock64();
+    while (have) {
+      have = false;
+      ++n_tiny;
+      const int rlo = nd.rlo, ra = nd.ra;
+      const int an = __popcll(nd.mask);  // distinct rows of the node
+      warp_draw_mtry(g.seed, t, nd.key, p, g.mtry, mind, feats, lane);
+      const int64_t nk = nd.n, Sk = nd.S;
+      uint32_t* stg = stg_all + (size_t)wid * TGRP * TINY;
+      const unsigned lt = (1u << lane) - 1u;
+      // lane-local best over all (feature, boundary) items: key g, tie = (feature << 16 | rank)
+      double lg = -1.0;
+      uint32_t ltie = 0xffffffffu, lra = 0, lrb = 0;
+      int32_t lnl = 0;
+      int64_t lSl = 0;
+      for (int s0 = 0; s0 < g.mtry; s0 += TGRP) {
+        const int ng = min(TGRP, g.mtry - s0);
+        // stage: the node's entries of each drawn feature, in value order, packed [slot][0..an)
+  #pragma unroll
+        for (int u = 0; u < TGRP; ++u) {
+          if (u >= ng) break;
+          const int f = feats[s0 + u];
+          const uint32_t* seg = list + (size_t)f * a0 + rlo;
+          const uint32_t e0 = lane < ra ? seg[lane] : 0u, e1 = lane + 32 < ra ? seg[lane + 32] : 0u;
+          const bool v0 = lane < ra && ((nd.mask >> rmap[e0 & 0xffffu]) & 1ull);
+          const bool v1 = lane + 32 < ra && ((nd.mask >> rmap[e1 & 0xffffu]) & 1ull);
+          const unsigned m0 = __ballot_sync(0xffffffffu, v0), m1 = __ballot_sync(0xffffffffu, v1);
+          if (v0) stg[u * an + __popc(m0 & lt)] = e0;
+          if (v1) stg[u * an + __popc(m0) + __popc(m1 & lt)] = e1;
+        }
         __syncwarp();
-        const bool valid = lane < nd.a;
-        const uint32_t ent = valid ? list[nd.lo + lane] : 0u;  // feature 0's row = the row list
-        const uint32_t lrow = ent & 0xffffu;
-        const int32_t w = valid ? wl[lrow] : 0;
-        const int64_t wv = valid ? wy[lrow] : 0;
-        warp_draw_mtry(g.seed, t, nd.key, p, g.mtry, mind, feats, lane);
-        const int64_t nk = nd.n, Sk = nd.S;
-        double bg = -1.0;
-        int bf = 0x7fffffff;
-        uint32_t brk = 0;
-        int bnl = 0, bpos = 0;
-        int64_t bSl = 0;
-        uint32_t bra = 0, brb = 0;
-        for (int s = 0; s < g.mtry; ++s) {
-          const int f = feats[s];
-          const uint32_t rk0 = valid ? (uint32_t)R[(size_t)lrow * RS + f] : 0xffffu;
-          const uint32_t sk = bitonic_sort32((rk0 << 5) | (uint32_t)lane, lane);
-          const int srcl = (int)(sk & 31u);
-          const uint32_t rk = sk >> 5;
-          const int32_t ws = __shfl_sync(0xffffffffu, w, srcl);
-          const int64_t wys = __shfl_sync(0xffffffffu, wv, srcl);
-          const int32_t ic = warp_incl_scan(ws, lane);
-          const int64_t is = warp_incl_scan(wys, lane);
-          const uint32_t rkn = __shfl_down_sync(0xffffffffu, rk, 1);
-          double lg = -1.0;
-          if (lane + 1 < nd.a && rk != rkn && screen_may_win(nk, Sk, ic, is, bg)) lg = split_key(nk, Sk, ic, is);
-          // warp argmax (g desc, rank asc == lane asc)
-          double mg = lg;
-          int ml = lane;
-#pragma unroll
-          for (int o = 16; o > 0; o >>= 1) {
-            const double og = __shfl_down_sync(0xffffffffu, mg, o);
-            const int ol = __shfl_down_sync(0xffffffffu, ml, o);
-            if (lane + o < 32 && (og > mg || (og == mg && ol < ml))) {
-              mg = og;
-              ml = ol;
+        // dense passes over the ng*an (slot, position) items: segmented scans by slot
+        const int total = ng * an;
+        int32_t cw = 0;
+        int64_t cs = 0;
+        for (int i0 = 0; i0 < total; i0 += 32) {
+          const int i = i0 + lane;
+          const bool act = i < total;
+          const int sl = act ? i / an : ng;
+          const int j = act ? i - sl * an : 0;
+          const uint32_t e = act ? stg[i] : 0u;
+          const uint32_t lr = e & 0xffffu;
+          int32_t w = act ? wl[lr] : 0;
+          int64_t wv = act ? wy[lr] : 0;
+          // inclusive segmented scan (segments are slot runs; lane-o is in my slot iff o <= j)
+  #pragma unroll
+          for (int o = 1; o < 32; o <<= 1) {
+            const int32_t uw = __shfl_up_sync(0xffffffffu, w, o);
+            const int64_t uv = __shfl_up_sync(0xffffffffu, wv, o);
+            if (lane >= o && o <= j) {
+              w += uw;
+              wv += uv;
             }
           }
-          mg = __shfl_sync(0xffffffffu, mg, 0);
-          ml = __shfl_sync(0xffffffffu, ml, 0);
-          if (mg >= 0.0 && (mg > bg || (mg == bg && f < bf))) {
-            bg = mg;
-            bf = f;
-            bpos = ml;
-            brk = __shfl_sync(0xffffffffu, rk, ml);
-            bnl = __shfl_sync(0xffffffffu, ic, ml);
-            bSl = __shfl_sync(0xffffffffu, is, ml);
-            const int sa = __shfl_sync(0xffffffffu, srcl, ml);
-            const int sb = __shfl_sync(0xffffffffu, srcl, min(ml + 1, 31));
-            bra = __shfl_sync(0xffffffffu, lrow, sa);
-            brb = __shfl_sync(0xffffffffu, lrow, sb);
-          } else {
-            // keep every lane's copies uniform (the shuffles above are warp-uniform branches)
+          // my slot started before this pass (j > lane): add the previous pass's carry
+          if (j > lane) {
+            w += cw;
+            wv += cs;
           }
+          const int32_t lw = __shfl_sync(0xffffffffu, w, 31);
+          const int64_t lv = __shfl_sync(0xffffffffu, wv, 31);
+          const int lj = __shfl_sync(0xffffffffu, j, 31);
+          const bool cont = lj + 1 < an;  // last item's slot continues into the next pass
+          if (act && j + 1 < an) {
+            const uint32_t en = stg[i + 1];
+            if ((en >> 16) != (e >> 16) && screen_may_win(nk, Sk, w, wv, lg)) {
+              const double gk = split_key(nk, Sk, w, wv);
+              const uint32_t tie = ((uint32_t)feats[s0 + sl] << 16) | (e >> 16);
+              if (gk > lg || (gk == lg && tie < ltie)) {
+                lg = gk;
+                ltie = tie;
+                lnl = w;
+                lSl = wv;
+                lra = lr;
+                lrb = en & 0xffffu;
+              }
+            }
+          }
+          cw = cont ? lw : 0;
+          cs = cont ? lv : 0;
         }
-        if (!(bg > 0.0)) continue;  // leaf: the record already holds count and value
-        // split
-        int lid = 0;
-        if (lane == 0) {
-          const double xa = canon(g.X[(int64_t)bf * g.ldx + grow[bra]]);
-          const double xb = canon(g.X[(int64_t)bf * g.ldx + grow[brb]]);
-          lid = atomicAdd(&s_nloc, 2);
-          SRec& r = recs[nd.id];
-          r.feature = bf;
-          r.left = lid;
-          r.thr = split_threshold(xa, xb);
-          r.drss = ldexp(__ddiv_rn(bg, (double)nd.n), -2 * g.q);
+        __syncwarp();
+      }
+      const int wlane = warp_argmax_key(gkey(lg), ltie);
+      const double bg = wlane >= 0 ? __shfl_sync(0xffffffffu, lg, wlane) : -1.0;
+      if (bg > 0.0) {
+        const uint32_t tie = __shfl_sync(0xffffffffu, ltie, wlane);
+        const int bf = (int)(tie >> 16);
+        const uint32_t brk = tie & 0xffffu;
+        const int32_t bnl = __shfl_sync(0xffffffffu, lnl, wlane);
+        const int64_t bSl = __shfl_sync(0xffffffffu, lSl, wlane);
+        const uint32_t bra = __shfl_sync(0xffffffffu, lra, wlane);
+        const uint32_t brb = __shfl_sync(0xffffffffu, lrb, wlane);
+        // child masks from the winning feature's order: left = rank <= brk
+        const uint32_t* seg = list + (size_t)bf * a0 + rlo;
+        uint64_t mL = 0;
+        double vl = 0.0, vr = 0.0;
+  #pragma unroll
+        for (int hh = 0; hh < 2; ++hh) {
+          const int k = lane + 32 * hh;
+          const uint32_t e = k < ra ? seg[k] : 0u;
+          const uint32_t lrow = e & 0xffffu;
+          const int ri = k < ra ? rmap[lrow] : 0;
+          const bool valid = k < ra && ((nd.mask >> ri) & 1ull);
+          const bool left = valid && (e >> 16) <= brk;
+          const uint32_t lo = __reduce_or_sync(0xffffffffu, (left && ri < 32) ? (1u << ri) : 0u);
+          const uint32_t hi = __reduce_or_sync(0xffffffffu, (left && ri >= 32) ? (1u << (ri - 32)) : 0u);
+          mL |= ((uint64_t)hi << 32) | lo;
+          if (left) vl += wyd[lrow];
+          else if (valid) vr += wyd[lrow];
         }
-        lid = __shfl_sync(0xffffffffu, lid, 0);
-        const bool right = valid && (uint32_t)R[(size_t)lrow * RS + bf] > brk;
-        const bool left = valid && !right;
-        const unsigned ml_ = __ballot_sync(0xffffffffu, left), mr_ = __ballot_sync(0xffffffffu, right);
-        const int al = __popc(ml_), ar = __popc(mr_);
-        const unsigned lt = (1u << lane) - 1u;
-        if (valid) list[nd.lo + (left ? __popc(ml_ & lt) : al + __popc(mr_ & lt))] = ent;
-        double vl = left ? wyd[lrow] : 0.0, vr = right ? wyd[lrow] : 0.0;
-#pragma unroll
+        const uint64_t mR = nd.mask & ~mL;
+  #pragma unroll
         for (int o = 16; o > 0; o >>= 1) {
           vl += __shfl_down_sync(0xffffffffu, vl, o);
           vr += __shfl_down_sync(0xffffffffu, vr, o);
         }
+        int lid = 0;
         if (lane == 0) {
+          lid = atomicAdd(&s_nloc, 2);
+          SRec& r = recs[nd.id];
+          r.feature = bf;
+          r.left = lid;
+          r.ra = (uint16_t)bra;
+          r.rb = (uint16_t)brb;
+          r.drss = ldexp(__ddiv_rn(bg, (double)nd.n), -2 * g.q);
           const int nr = nd.n - bnl;
           SRec c;
           c.feature = -1;
           c.left = -1;
-          c.pad = 0;
-          c.thr = 0.0;
+          c.ra = c.rb = 0;
           c.drss = 0.0;
           c.count = bnl;
           c.value = __ddiv_rn(vl, (double)bnl);
@@ -1349,35 +1425,50 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
           c.count = nr;
           c.value = __ddiv_rn(vr, (double)nr);
           recs[lid + 1] = c;
-          const uint64_t kl = child_key(g.seed, t, nd.key, 0), kr = child_key(g.seed, t, nd.key, 1);
-          // push right first so the left subtree is processed next (any order is valid)
-          if (nr > g.nodesize && ar >= 2) {
-            TNode c2;
-            c2.lo = nd.lo + al;
-            c2.a = ar;
-            c2.n = nr;
-            c2.id = lid + 1;
-            c2.S = nd.S - bSl;
-            c2.key = kr;
-            stk[sp] = c2;
-          }
-          if (bnl > g.nodesize && al >= 2) {
-            TNode c2;
-            c2.lo = nd.lo;
-            c2.a = al;
-            c2.n = bnl;
-            c2.id = lid;
-            c2.S = bSl;
-            c2.key = kl;
-            stk[sp + ((nr > g.nodesize && ar >= 2) ? 1 : 0)] = c2;
-          }
         }
-        sp += ((nd.n - bnl) > g.nodesize && ar >= 2) + (bnl > g.nodesize && al >= 2);
-        __syncwarp();
+        lid = __shfl_sync(0xffffffffu, lid, 0);
+        // child keys on lanes 0 and 1
+        const uint64_t ck = child_key(g.seed, t, nd.key, lane & 1);
+        const uint64_t kl = __shfl_sync(0xffffffffu, ck, 0), kr = __shfl_sync(0xffffffffu, ck, 1);
+        const int nr = nd.n - bnl;
+        const bool gl = bnl > g.nodesize && __popcll(mL) >= 2;
+        const bool gr = nr > g.nodesize && __popcll(mR) >= 2;
+        TNode cl, cr;
+        cl.rlo = cr.rlo = nd.rlo;
+        cl.ra = cr.ra = nd.ra;
+        cl.mask = mL;
+        cl.id = lid;
+        cl.n = bnl;
+        cl.S = bSl;
+        cl.key = kl;
+        cr.mask = mR;
+        cr.id = lid + 1;
+        cr.n = nr;
+        cr.S = nd.S - bSl;
+        cr.key = kr;
+        // continue with one child in this warp, hand the sibling to the queue
+        if (gl && gr) {
+          if (lane == 0) tq_push(tq, &s_alloc, &s_pending, cr);
+          nd = cl;
+          have = true;
+        } else if (gl) {
+          nd = cl;
+          have = true;
+        } else if (gr) {
+          nd = cr;
+          have = true;
+        }
       }
+
     }
+    busy += clock64() - tb0;
+    if (lane == 0) atomicSub(&s_pending, 1);
+    __syncwarp();
   }
   __syncthreads();
+  const long long t_tiny_end = clock64();
+  __syncthreads();
+  tclk[3] = clock64();
   // ---- flush the subtree into the tree's raw pool (sibling pairs stay adjacent)
   if (tid == 0) s_gbase = s_nloc > 1 ? atomicAdd(&g.pool.nn[b], s_nloc - 1) : 0;
   __syncthreads();
@@ -1388,11 +1479,33 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
     const int64_t gid = r0 + (l == 0 ? root.raw : gbase + l - 1);
     g.pool.feature[gid] = r.feature;
     g.pool.left[gid] = r.left >= 0 ? gbase + r.left - 1 : -1;
-    g.pool.thr[gid] = r.thr;
+    double thr = 0.0;
+    if (r.feature >= 0)
+      thr = split_threshold(canon(g.X[(int64_t)r.feature * g.ldx + grow[r.ra]]),
+                            canon(g.X[(int64_t)r.feature * g.ldx + grow[r.rb]]));
+    g.pool.thr[gid] = thr;
     g.pool.drss[gid] = r.drss;
     if (l > 0) {
       g.pool.count[gid] = r.count;
       g.pool.value[gid] = r.value;
+    }
+  }
+  if (g.stats) {
+    tclk[4] = clock64();
+    if (tid == 0) {
+      atomicAdd(&g.stats[0], (unsigned long long)(tclk[1] - tclk[0]));
+      atomicAdd(&g.stats[1], (unsigned long long)(tclk[2] - tclk[1]));
+      atomicAdd(&g.stats[2], (unsigned long long)(tclk[3] - tclk[2]));
+      atomicAdd(&g.stats[3], (unsigned long long)(tclk[4] - tclk[3]));
+      atomicAdd(&g.stats[4], (unsigned long long)n_med);
+      atomicAdd(&g.stats[5], 1ull);
+      atomicAdd(&g.stats[6], (unsigned long long)a0);
+      atomicAdd(&g.stats[9], (unsigned long long)s_nloc);
+    }
+    if (lane == 0) {
+      atomicAdd(&g.stats[7], (unsigned long long)n_tiny);
+      atomicAdd(&g.stats[8], (unsigned long long)(t_tiny_end - tclk[2]));  // busy+idle per warp in tiny phase
+      atomicAdd(&g.stats[10], (unsigned long long)busy);
     }
   }
 }
@@ -1511,8 +1624,41 @@ void bootstrap_impl(uint64_t seed, int32_t t0, int32_t ntrees, int64_t n, int64_
   BF_CUDA_CHECK(cudaGetLastError());
 }
 
+struct PhaseTimer {  // BF_FIT_TIMING=1: host wall time per fit phase (stream-synchronised)
+  bool on;
+  cudaStream_t s;
+  double t0, last;
+  std::vector<std::pair<std::string, double>> acc;
+  static double now() {
+    timespec ts;
+    clock_gettime(CLOCK_MONOTONIC, &ts);
+    return ts.tv_sec + ts.tv_nsec * 1e-9;
+  }
+  explicit PhaseTimer(cudaStream_t st) : on(getenv("BF_FIT_TIMING") != nullptr), s(st) { t0 = last = now(); }
+  void mark(const char* name) {
+    if (!on) return;
+    cudaStreamSynchronize(s);
+    const double t = now();
+    for (auto& kv : acc)
+      if (kv.first == name) {
+        kv.second += t - last;
+        last = t;
+        return;
+      }
+    acc.emplace_back(name, t - last);
+    last = t;
+  }
+  ~PhaseTimer() {
+    if (!on) return;
+    fprintf(stderr, "[fit timing] total %.1f ms:", (now() - t0) * 1e3);
+    for (auto& kv : acc) fprintf(stderr, " %s=%.1f", kv.first.c_str(), kv.second * 1e3);
+    fprintf(stderr, "\n");
+  }
+};
+
 void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, int32_t p, const bf_params& prm0,
               cudaStream_t s, bf_forest** out) {
+  PhaseTimer ptm(s);
   bf_params prm = prm0;
   BF_REQUIRE(prm.ntree >= 1 && prm.nodesize >= 1, BF_EINVAL, "bf_fit: ntree >= 1 and nodesize >= 1 required");
   if (prm.tree_begin == 0 && prm.tree_end == 0) prm.tree_end = prm.ntree;
@@ -1521,6 +1667,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
   const int mtry = prm.mtry ? prm.mtry : std::max(p / 3, 1);
   BF_REQUIRE(mtry >= 1 && mtry <= p, BF_EINVAL, "bf_fit: mtry not in [1, p]");
   BF_REQUIRE(p <= 32767, BF_ENOTIMPL, "bf_fit: p > 32767");
+  BF_REQUIRE(n < MAX_ROWS, BF_ENOTIMPL, "bf_fit: n >= 2^24 rows (24-bit row/rank fields of the list entries)");
   const int64_t ns = prm.sampsize ? prm.sampsize : n;
   BF_REQUIRE(ns >= 1 && ns < (int64_t(1) << 31), BF_ERANGE, "bf_fit: sampsize out of range");
   BF_REQUIRE(prm.replace || ns == n, BF_ENOTIMPL, "bf_fit: replace = 0 needs sampsize == n (reading R20)");
@@ -1544,6 +1691,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
     BF_CUDA_CHECK(cudaStreamSynchronize(s));
     BF_REQUIRE(hb == 0, BF_ENONFINITE, "bf_fit: NaN/Inf in X or y");
   }
+  ptm.mark("validate");
   // ---- a2 fixed point
   DBuf<int64_t> yq(n, s);
   int32_t q = 0;
@@ -1587,6 +1735,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
     }
   }
 
+  ptm.mark("presort");
   // ---- sizing: subtree capacity A and trees in flight B
   const int smax = dyn_smem_limit(k_subtree);
   int A = 2;
@@ -1631,9 +1780,11 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
   std::vector<Chunk> chunks;
 
   try {
+    ptm.mark("setup");
     // ---- batch buffers
     DBuf<int32_t> w((size_t)B * n, s);
-    DBuf<Pay> pay((size_t)B * n, s);
+    DBuf<int32_t> wmax(1, s);
+    BF_CUDA_CHECK(cudaMemsetAsync(wmax.p, 0, sizeof(int32_t), s));
     DBuf<uint8_t> side((size_t)B * n, s);
     DBuf<uint16_t> loc((size_t)B * n, s);
     DBuf<int32_t> pf((size_t)B * cap_nodes, s), pl((size_t)B * cap_nodes, s), pc((size_t)B * cap_nodes, s),
@@ -1661,6 +1812,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
     DBuf<uint64_t> E0, E1, Es;
     size_t E_cap = 0;
 
+    ptm.mark("alloc");
     for (int tb = prm.tree_begin; tb < prm.tree_end; tb += B) {
       const int Bc = std::min(B, prm.tree_end - tb);
       // ---- a4 bootstrap + payload + root sums
@@ -1670,14 +1822,17 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
       BF_CUDA_CHECK(cudaMemsetAsync(sy_root.p, 0, sizeof(double) * Bc, s));
       {
         KScope ks_("k_payload", s, 0.0);
-        k_payload<<<dim3((unsigned)ceil_div(n, NT), Bc), NT, 0, s>>>(w.p, yq.p, y, n, pay.p, a_root.p, S_root.p,
+        k_payload<<<dim3((unsigned)ceil_div(n, NT), Bc), NT, 0, s>>>(w.p, yq.p, y, n, wmax.p, a_root.p, S_root.p,
                                                                     sy_root.p);
       }
       BF_CUDA_CHECK(cudaGetLastError());
       std::vector<int32_t> ha(Bc), hk(Bc), hl(Bc), hsx(Bc);
       std::vector<int64_t> hbase(Bc);
+      int32_t hwmax = 0;
       d2h(ha.data(), a_root.p, Bc, s);
+      d2h(&hwmax, wmax.p, 1, s);
       BF_CUDA_CHECK(cudaStreamSynchronize(s));
+      BF_REQUIRE(hwmax <= 0xffff, BF_ERANGE, "bf_fit: a bootstrap multiplicity exceeds 65535");
       int64_t offL = 0, offS = 0;
       int nL = 0, nS = 0;
       for (int b = 0; b < Bc; ++b) {
@@ -1724,7 +1879,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
         dim3 grid((unsigned)nchunk, (unsigned)p, (unsigned)Bc);
         {
           KScope ks_("k_list_count", s, 0.0);
-          k_list_count<<<grid, NT, 0, s>>>(srt.p, n, pay.p, kind_d.p, nchunk, cnt.p);
+          k_list_count<<<grid, NT, 0, s>>>(srt.p, n, w.p, kind_d.p, nchunk, cnt.p);
         }
         {
           KScope ks_("k_list_prefix", s, 0.0);
@@ -1732,11 +1887,12 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
         }
         {
           KScope ks_("k_list_scatter", s, 0.0);
-          k_list_scatter<<<grid, NT, 0, s>>>(srt.p, n, pay.p, kind_d.p, base_d.p, a_root.p, nchunk, cnt.p, E0.p, Es.p);
+          k_list_scatter<<<grid, NT, 0, s>>>(srt.p, n, w.p, kind_d.p, base_d.p, a_root.p, nchunk, cnt.p, E0.p, Es.p);
         }
         BF_CUDA_CHECK(cudaGetLastError());
         prof_add_bytes("k_list_scatter", (double)Bc * n * p * 8.0 + (double)(offL + offS) * 8.0);
       }
+      ptm.mark("boot+lists");
       LevelSummary ls{};
       ls.nnext = nL;
       ls.nsmall = nS;
@@ -1757,7 +1913,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
         }
         {
           KScope ks_("k_split_scan", s, 0.0);
-          k_split_scan<<<(unsigned)((int64_t)N * mtry), NT, 0, s>>>(nc, feat.p, mtry, Ec, pay.p, n, rec.p);
+          k_split_scan<<<(unsigned)((int64_t)N * mtry), NT, 0, s>>>(nc, feat.p, mtry, Ec, yq.p, rec.p);
         }
         {
           KScope ks_("k_finalize", s, 0.0);
@@ -1783,7 +1939,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
         }
         {
           KScope ks_("k_dest", s, 0.0);
-          k_dest<<<(unsigned)N, NT, 0, s>>>(nc, split.p, Ec, pay.p, y, n, side.p, pool);
+          k_dest<<<(unsigned)N, NT, 0, s>>>(nc, split.p, Ec, y, n, side.p, pool);
         }
         {
           KScope ks_("k_partition", 0, 0.0);
@@ -1806,6 +1962,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
         std::swap(Ec, En);
         std::swap(nc, nx);
       }
+      ptm.mark("global_levels");
       // ---- subtree phase
       {
         d2h(&ls, dsum.p, 1, s);
@@ -1815,7 +1972,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
           SubArgs ga;
           ga.sq = sq.p;
           ga.Es = Es.p;
-          ga.pay = pay.p;
+          ga.yq = yq.p;
           ga.y = y;
           ga.X = X;
           ga.ldx = ldx;
@@ -1829,13 +1986,31 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
           ga.t0 = tb;
           ga.loc = loc.p;
           ga.pool = pool;
+          ga.stats = nullptr;
+          static const bool want_stats = getenv("BF_SUBTREE_STATS") != nullptr;
+          DBuf<unsigned long long> st;
+          if (want_stats) {
+            st.alloc(16, s);
+            BF_CUDA_CHECK(cudaMemsetAsync(st.p, 0, 16 * 8, s));
+            ga.stats = st.p;
+          }
           {
             KScope ks_("k_subtree", s, 0.0);
             k_subtree<<<(unsigned)ls.nsmall, SUB_NT, subtree_smem(A, p), s>>>(ga);
           }
+          if (want_stats) {
+            unsigned long long h[16];
+            d2h(h, st.p, 16, s);
+            BF_CUDA_CHECK(cudaStreamSynchronize(s));
+            const double c = (double)h[5];
+            fprintf(stderr, "[subtree] A=%d ctas=%llu mean_a0=%.1f cyc/cta: load=%.0f medium=%.0f tiny=%.0f flush=%.0f | medium nodes/cta=%.1f tiny nodes/cta=%.1f nodes/cta=%.1f warp-cyc in tiny/cta=%.0f busy=%.0f (%.0f per tiny node)\n",
+                    A, h[5], h[6] / c, h[0] / c, h[1] / c, h[2] / c, h[3] / c, h[4] / c, h[7] / c, h[9] / c, h[8] / c,
+                    h[10] / c, h[10] / (double)(h[7] ? h[7] : 1));
+          }
           BF_CUDA_CHECK(cudaGetLastError());
         }
       }
+      ptm.mark("subtree");
       // ---- a11 emit
       std::vector<int32_t> hnn(Bc);
       d2h(hnn.data(), pnn.p, Bc, s);
@@ -1881,6 +2056,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
     }
     chunks.clear();
     BF_CUDA_CHECK(cudaStreamSynchronize(s));
+    ptm.mark("emit+assemble");
   } catch (...) {
     forest_release(F);
     delete F;
