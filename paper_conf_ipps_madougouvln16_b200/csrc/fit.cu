@@ -757,6 +757,1383 @@ __global__ void __launch_bounds__(NT) k_partition(const LNode* nodes, const Spli
   }
 }
 
+// ------------------------------------------------------------------ pieces + decoupled look-back (global phase)
+// Every (node, feature) segment of a level is cut into pieces of PIECE
+// entries.  Persistent CTAs take pieces in ticket order; a piece publishes its
+// aggregate as soon as it has it, then a warp looks back over the preceding
+// pieces of the same segment (summing aggregates until it meets a published
+// inclusive prefix) -- so segments of any length stream at full parallelism
+// in one pass (Merrill & Garland's single-pass scan).
+constexpr int PIECE_V = 8;
+constexpr int PIECE = NT * PIECE_V;  // 2048 entries
+
+struct PieceRec {  // best candidate of one piece of a scan item
+  double g;
+  uint32_t rank_a, rank_b;
+  int32_t pos, nl;
+  int64_t Sl;
+};
+struct LbNS {
+  int64_t S;
+  int32_t n;
+  int32_t pad;
+};
+
+// items: mode 0 scan (node = i / mtry), 1 dest (node = i, split only), 2 partition (node = i / p, split with a kept child)
+__global__ void k_piece_count(int mode, int nitems, int div, const LNode* nodes, const Split* split, const Child* child,
+                              int32_t* cnt) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= nitems) return;
+  const int k = i / div;
+  int a = nodes[k].a;
+  if (mode >= 1 && !split[k].split) a = 0;
+  if (mode == 2) {
+    const int kl = child[2 * k].kind, kr = child[2 * k + 1].kind;
+    if (kl != KIND_LARGE && kl != KIND_SMALL && kr != KIND_LARGE && kr != KIND_SMALL) a = 0;
+  }
+  cnt[i] = (a + PIECE - 1) / PIECE;
+}
+
+__global__ void k_piece_map(int nitems, const int32_t* cnt, const int32_t* off, int32_t* map, int32_t* total) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= nitems) return;
+  const int c = cnt[i], o = off[i];
+  for (int k = 0; k < c; ++k) map[o + k] = i;
+  if (i == nitems - 1) *total = o + c;
+}
+
+__device__ __forceinline__ uint32_t ld_flag(const uint32_t* p) { return *(const volatile uint32_t*)p; }
+
+// Warp look-back over pieces [t0, t): exclusive (n, S) of piece t.  All lanes return the result.
+__device__ void lookback_ns(int t, int t0, const LbNS* agg, const LbNS* incl, const uint32_t* flag, int32_t& exn,
+                            int64_t& exS) {
+  const int lane = threadIdx.x & 31;
+  int j = t - 1;
+  int32_t an = 0;
+  int64_t aS = 0;
+  for (;;) {
+    const int idx = j - lane;
+    uint32_t f = 2;
+    int32_t vn = 0;
+    int64_t vS = 0;
+    if (idx >= t0) {
+      while ((f = ld_flag(flag + idx)) == 0) __nanosleep(20);
+      __threadfence();
+      const LbNS* src = (f == 2) ? incl + idx : agg + idx;
+      vS = __ldcg((const long long*)&src->S);
+      vn = __ldcg((const int*)&src->n);
+    }
+    const unsigned pm = __ballot_sync(0xffffffffu, f == 2);
+    const int L = pm ? __ffs(pm) - 1 : 31;
+    if (lane > L) {
+      vn = 0;
+      vS = 0;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      vn += __shfl_xor_sync(0xffffffffu, vn, o);
+      vS += __shfl_xor_sync(0xffffffffu, vS, o);
+    }
+    an += vn;
+    aS += vS;
+    if (pm) break;
+    j -= 32;
+  }
+  exn = an;
+  exS = aS;
+}
+
+// Warp look-back for 62-bit counters packed with a 2-bit status: (status << 62) | value.
+__device__ int64_t lookback_cnt(int t, int t0, const unsigned long long* st) {
+  const int lane = threadIdx.x & 31;
+  int j = t - 1;
+  int64_t acc = 0;
+  for (;;) {
+    const int idx = j - lane;
+    unsigned long long w = (2ull << 62);
+    if (idx >= t0)
+      while (((w = *(const volatile unsigned long long*)(st + idx)) >> 62) == 0) __nanosleep(20);
+    const uint32_t f = (uint32_t)(w >> 62);
+    int64_t v = (int64_t)(w & ((1ull << 62) - 1));
+    const unsigned pm = __ballot_sync(0xffffffffu, f == 2);
+    const int L = pm ? __ffs(pm) - 1 : 31;
+    if (lane > L) v = 0;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    acc += v;
+    if (pm) break;
+    j -= 32;
+  }
+  return acc;
+}
+
+struct ScanLbArgs {
+  const LNode* nodes;
+  const int32_t* feat;
+  int mtry;
+  const uint64_t* E;
+  const int64_t* yq;
+  const int32_t* poff;
+  const int32_t* pmap;
+  const int32_t* ptotal;
+  unsigned int* ticket;
+  LbNS* agg;
+  LbNS* incl;
+  uint32_t* flag;
+  PieceRec* prec;
+};
+
+// a7 split search, one piece per iteration of a persistent CTA.
+__global__ void __launch_bounds__(NT) k_split_scan_lb(ScanLbArgs g) {
+  __shared__ int32_t smc[NT / 32];
+  __shared__ int64_t sms[NT / 32];
+  __shared__ double sg[NT / 32];
+  __shared__ uint32_t sr[NT / 32];
+  __shared__ int32_t sw[NT / 32];
+  __shared__ int s_t, s_exn;
+  __shared__ int64_t s_exS;
+  const int total = *g.ptotal;
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  for (;;) {
+    if (tid == 0) s_t = atomicAdd(g.ticket, 1u);
+    __syncthreads();
+    const int t = s_t;
+    if (t >= total) break;
+    const int item = g.pmap[t], t0 = g.poff[item], k = t - t0;
+    const LNode nd = g.nodes[item / g.mtry];
+    const int f = g.feat[item];
+    const uint64_t* seg = g.E + nd.base + (int64_t)f * nd.a;
+    const int a = nd.a;
+    const int64_t nk = nd.n, Sk = nd.S;
+    const int j0 = k * PIECE + tid * PIECE_V;
+    uint64_t e[PIECE_V + 1];
+    int32_t wc[PIECE_V];
+    int64_t ws[PIECE_V];
+    int32_t tc = 0;
+    int64_t ts = 0;
+#pragma unroll
+    for (int u = 0; u <= PIECE_V; ++u) e[u] = (j0 + u < a) ? seg[j0 + u] : 0ull;
+#pragma unroll
+    for (int u = 0; u < PIECE_V; ++u) {
+      wc[u] = 0;
+      ws[u] = 0;
+      if (j0 + u < a) {
+        wc[u] = e_w(e[u]);
+        ws[u] = (int64_t)wc[u] * __ldg(g.yq + e_row(e[u]));
+      }
+      tc += wc[u];
+      ts += ws[u];
+    }
+    int32_t totc;
+    int64_t tots;
+    int32_t prc = block_excl_scan(tc, smc, totc);
+    int64_t prs = block_excl_scan(ts, sms, tots);
+    if (tid == 0) {
+      LbNS v;
+      v.S = tots;
+      v.n = totc;
+      v.pad = 0;
+      if (k == 0) {
+        g.incl[t] = v;
+        __threadfence();
+        *(volatile uint32_t*)(g.flag + t) = 2u;
+      } else {
+        g.agg[t] = v;
+        __threadfence();
+        *(volatile uint32_t*)(g.flag + t) = 1u;
+      }
+    }
+    if (k > 0 && wid == 0) {
+      int32_t exn;
+      int64_t exS;
+      lookback_ns(t, t0, g.agg, g.incl, g.flag, exn, exS);
+      if (lane == 0) {
+        LbNS v;
+        v.S = exS + tots;
+        v.n = exn + totc;
+        v.pad = 0;
+        g.incl[t] = v;
+        __threadfence();
+        *(volatile uint32_t*)(g.flag + t) = 2u;
+        s_exn = exn;
+        s_exS = exS;
+      }
+    }
+    __syncthreads();
+    if (k > 0) {
+      prc += s_exn;
+      prs += s_exS;
+    }
+    double bg = -1.0;
+    uint32_t brank = 0xffffffffu, brb = 0;
+    int32_t bpos = -1, bnl = 0;
+    int64_t bSl = 0;
+#pragma unroll
+    for (int u = 0; u < PIECE_V; ++u) {
+      prc += wc[u];
+      prs += ws[u];
+      const int j = j0 + u;
+      if (j + 1 < a) {
+        const uint32_t ra = e_rank(e[u]), rb = e_rank(e[u + 1]);
+        if (ra != rb && screen_may_win(nk, Sk, prc, prs, bg)) {
+          const double gk = split_key(nk, Sk, prc, prs);
+          if (rec_better(gk, ra, bg, brank)) {
+            bg = gk;
+            brank = ra;
+            brb = rb;
+            bpos = j;
+            bnl = prc;
+            bSl = prs;
+          }
+        }
+      }
+    }
+    // block argmax (g desc, rank asc)
+    const int wl = warp_argmax_key(gkey(bg), brank);
+    const double wg = __shfl_sync(0xffffffffu, bg, wl >= 0 ? wl : 0);
+    const uint32_t wr = __shfl_sync(0xffffffffu, brank, wl >= 0 ? wl : 0);
+    if (lane == 0) {
+      sg[wid] = wl >= 0 ? wg : -1.0;
+      sr[wid] = wl >= 0 ? wr : 0xffffffffu;
+      sw[wid] = wl >= 0 ? wid * 32 + wl : -1;
+    }
+    __syncthreads();
+    if (tid == 0) {
+      double gg = sg[0];
+      uint32_t r = sr[0];
+      int who = sw[0];
+      for (int q = 1; q < NT / 32; ++q)
+        if (sw[q] >= 0 && (who < 0 || rec_better(sg[q], sr[q], gg, r))) {
+          gg = sg[q];
+          r = sr[q];
+          who = sw[q];
+        }
+      sw[0] = who;
+      if (who < 0) {
+        PieceRec R;
+        R.g = -1.0;
+        R.rank_a = 0xffffffffu;
+        R.rank_b = 0;
+        R.pos = -1;
+        R.nl = 0;
+        R.Sl = 0;
+        g.prec[t] = R;
+      }
+    }
+    __syncthreads();
+    if (tid == sw[0]) {
+      PieceRec R;
+      R.g = bg;
+      R.rank_a = brank;
+      R.rank_b = brb;
+      R.pos = bpos;
+      R.nl = bnl;
+      R.Sl = bSl;
+      g.prec[t] = R;
+    }
+    __syncthreads();
+  }
+}
+
+// best piece record of every scan item (warp per item)
+__global__ void k_item_reduce(int nitems, const int32_t* cnt, const int32_t* off, const PieceRec* prec, Rec* rec) {
+  const int lane = threadIdx.x & 31;
+  const int item = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  if (item >= nitems) return;
+  const int c = cnt[item], o = off[item];
+  double bg = -1.0;
+  uint32_t br = 0xffffffffu;
+  int bi = -1;
+  for (int q = lane; q < c; q += 32) {
+    const double gq = prec[o + q].g;
+    const uint32_t rq = prec[o + q].rank_a;
+    if (gq >= 0.0 && rec_better(gq, rq, bg, br)) {
+      bg = gq;
+      br = rq;
+      bi = o + q;
+    }
+  }
+  const int wl = warp_argmax_key(gkey(bg), br);
+  const int sbi = __shfl_sync(0xffffffffu, bi, wl >= 0 ? wl : 0);
+  const int src = wl >= 0 ? sbi : -1;
+  if (lane == 0) {
+    Rec R;
+    if (src >= 0) {
+      const PieceRec P = prec[src];
+      R.g = P.g;
+      R.rank_a = P.rank_a;
+      R.rank_b = P.rank_b;
+      R.pos = P.pos;
+      R.nl = P.nl;
+      R.Sl = P.Sl;
+    } else {
+      R.g = -1.0;
+      R.rank_a = 0xffffffffu;
+      R.rank_b = 0;
+      R.pos = -1;
+      R.nl = 0;
+      R.Sl = 0;
+    }
+    rec[item] = R;
+  }
+}
+
+struct DestArgs {
+  const LNode* nodes;
+  const Split* split;
+  const uint64_t* E;
+  const double* y;
+  int64_t n;
+  uint8_t* side;
+  const int32_t* poff;
+  const int32_t* pmap;
+  const int32_t* ptotal;
+  double* csum;  // 2 per node: sum of w*y of the left / right child
+};
+
+// a9/a10: goes-right flag of every row of a split node + child sums of w*y (one piece per CTA)
+__global__ void __launch_bounds__(NT) k_dest_pc(DestArgs g) {
+  __shared__ double sl[NT / 32], sr[NT / 32];
+  const int t = blockIdx.x;
+  if (t >= *g.ptotal) return;
+  const int k = g.pmap[t], pc = t - g.poff[k];
+  const Split sp = g.split[k];
+  const LNode nd = g.nodes[k];
+  const uint64_t* seg = g.E + nd.base + (int64_t)sp.f * nd.a;
+  uint8_t* sd = g.side + (int64_t)nd.b * g.n;
+  double accl = 0.0, accr = 0.0;
+  const int j0 = pc * PIECE + threadIdx.x * PIECE_V;
+#pragma unroll
+  for (int u = 0; u < PIECE_V; ++u) {
+    const int j = j0 + u;
+    if (j < nd.a) {
+      const uint64_t ej = seg[j];
+      const uint32_t row = e_row(ej);
+      const int s = j > sp.pos;
+      sd[row] = (uint8_t)s;
+      const double v = __dmul_rn((double)e_w(ej), g.y[row]);
+      if (s) accr += v;
+      else accl += v;
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    accl += __shfl_down_sync(0xffffffffu, accl, o);
+    accr += __shfl_down_sync(0xffffffffu, accr, o);
+  }
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  if (lane == 0) {
+    sl[wid] = accl;
+    sr[wid] = accr;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double a0 = 0.0, a1 = 0.0;
+    for (int q = 0; q < NT / 32; ++q) {
+      a0 += sl[q];
+      a1 += sr[q];
+    }
+    atomicAdd(&g.csum[2 * k], a0);
+    atomicAdd(&g.csum[2 * k + 1], a1);
+  }
+}
+
+__global__ void k_child_values(int N, const Split* split, const double* csum, const LNode* nodes, Pool pool) {
+  const int k = blockIdx.x * blockDim.x + threadIdx.x;
+  if (k >= N) return;
+  const Split sp = split[k];
+  if (!sp.split) return;
+  const int64_t r = (int64_t)nodes[k].b * pool.cap;
+  pool.value[r + sp.lraw] = __ddiv_rn(csum[2 * k], (double)sp.nl);
+  pool.value[r + sp.lraw + 1] = __ddiv_rn(csum[2 * k + 1], (double)sp.nr);
+}
+
+struct PartArgs {
+  const LNode* nodes;
+  const Split* split;
+  const Child* child;
+  int p;
+  const uint64_t* Ecur;
+  const uint8_t* side;
+  int64_t n;
+  uint64_t* Enext;
+  uint64_t* Esmall;
+  const int32_t* poff;
+  const int32_t* pmap;
+  const int32_t* ptotal;
+  unsigned int* ticket;
+  unsigned long long* st;
+};
+
+// a9 partition, one piece per iteration of a persistent CTA (left counts carried by look-back)
+__global__ void __launch_bounds__(NT) k_partition_lb(PartArgs g) {
+  __shared__ int32_t sm[NT / 32];
+  __shared__ int s_t;
+  __shared__ int64_t s_ex;
+  const int total = *g.ptotal;
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  for (;;) {
+    if (tid == 0) s_t = atomicAdd(g.ticket, 1u);
+    __syncthreads();
+    const int t = s_t;
+    if (t >= total) break;
+    const int item = g.pmap[t], t0 = g.poff[item], k = t - t0;
+    const int node = item / g.p, f = item - node * g.p;
+    const LNode nd = g.nodes[node];
+    const Child cl = g.child[2 * node], cr = g.child[2 * node + 1];
+    const bool keepL = cl.kind == KIND_LARGE || cl.kind == KIND_SMALL;
+    const bool keepR = cr.kind == KIND_LARGE || cr.kind == KIND_SMALL;
+    const uint64_t* seg = g.Ecur + nd.base + (int64_t)f * nd.a;
+    const uint8_t* sd = g.side + (int64_t)nd.b * g.n;
+    const int j0 = k * PIECE + tid * PIECE_V;
+    uint64_t e[PIECE_V];
+    bool left[PIECE_V];
+#pragma unroll
+    for (int u = 0; u < PIECE_V; ++u) e[u] = (j0 + u < nd.a) ? seg[j0 + u] : 0ull;
+    int32_t cnt = 0;
+#pragma unroll
+    for (int u = 0; u < PIECE_V; ++u) {
+      left[u] = (j0 + u < nd.a) && sd[e_row(e[u])] == 0;
+      cnt += left[u];
+    }
+    int32_t tot;
+    int32_t lb = block_excl_scan(cnt, sm, tot);
+    if (tid == 0)
+      *(volatile unsigned long long*)(g.st + t) = ((k == 0 ? 2ull : 1ull) << 62) | (unsigned long long)tot;
+    if (k > 0 && wid == 0) {
+      const int64_t ex = lookback_cnt(t, t0, g.st);
+      if (lane == 0) {
+        *(volatile unsigned long long*)(g.st + t) = (2ull << 62) | (unsigned long long)(ex + tot);
+        s_ex = ex;
+      }
+    }
+    __syncthreads();
+    if (k > 0) lb += (int32_t)s_ex;
+    uint64_t* dl = keepL ? (cl.kind == KIND_LARGE ? g.Enext : g.Esmall) + cl.base + (int64_t)f * cl.a : nullptr;
+    uint64_t* dr = keepR ? (cr.kind == KIND_LARGE ? g.Enext : g.Esmall) + cr.base + (int64_t)f * cr.a : nullptr;
+#pragma unroll
+    for (int u = 0; u < PIECE_V; ++u) {
+      const int j = j0 + u;
+      if (j < nd.a) {
+        if (left[u]) {
+          if (keepL) dl[lb] = e[u];
+          ++lb;
+        } else if (keepR) {
+          dr[j - lb] = e[u];
+        }
+      }
+    }
+    __syncthreads();
+  }
+}
+
+// ------------------------------------------------------------------ two-pass units with TMA staging (global phase v5)
+// Units are contiguous ranges of UNIT entries of one segment.  Pass 1 computes
+// every unit's aggregate with plain coalesced loads (embarrassingly parallel);
+// a device-wide exclusive scan over units gives each unit its prefix inside
+// its segment (units of a segment are consecutive); pass 2 processes units
+// with a static round-robin assignment, so each CTA double-buffers its next
+// unit's bulk copy (cp.async.bulk + mbarrier) behind the current one.  No
+// inter-CTA waiting anywhere.
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t* bar) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(bar)) : "memory");
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   smem_u32(dst)),
+               "l"(src), "r"(bytes), "r"(smem_u32(bar))
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
+  asm volatile(
+      "{\n .reg .pred p;\n WAIT_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n @!p bra WAIT_%=;\n}\n" ::"r"(
+          smem_u32(bar)),
+      "r"(phase)
+      : "memory");
+}
+// Stage entries [src, src + cnt): the copy starts at the 16-byte aligned address at or below src;
+// returns the entry offset (0 or 1) of src inside the buffer.  Issued by one thread.
+__device__ __forceinline__ int stage_entries(uint64_t* buf, const uint64_t* src, int cnt, uint64_t* bar) {
+  const uintptr_t a = (uintptr_t)src, a0 = a & ~(uintptr_t)15;
+  const int off = (int)((a - a0) >> 3);
+  const uint32_t bytes = (uint32_t)((((size_t)(cnt + off) * 8) + 15) & ~(size_t)15);
+  tma_load_1d(buf, (const void*)a0, bytes, bar);
+  return off;
+}
+// Gathers issued with volatile asm: ptxas keeps them back to back, so all of a
+// thread's independent loads are in flight together (otherwise it converts each
+// loaded value to a predicate at once and serialises the L2 round trips).
+__device__ __forceinline__ uint32_t ldg_u8_nc(const uint8_t* p) {
+  uint32_t v;
+  asm volatile("ld.global.nc.u8 %0, [%1];" : "=r"(v) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ int64_t ldg_s64_nc(const int64_t* p) {
+  int64_t v;
+  asm volatile("ld.global.nc.s64 %0, [%1];" : "=l"(v) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ float rcp_approx(float x) {  // |rel err| < 2^-22
+  float r;
+  asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+  return r;
+}
+// Cheap rigorous bounds gL <= g <= gU of the S4.3 key (fp64, no int128).
+__device__ __forceinline__ void key_bounds(double nkd, double Skd, int64_t nk, int32_t nl, int64_t Sl, double& gL,
+                                           double& gU) {
+  const double a = nkd * (double)Sl, b = (double)nl * Skd;
+  const double d = fabs(a - b);
+  const double E = (fabs(a) + fabs(b)) * 8.881784197001252e-16;  // 2^-50
+  const double r = (double)rcp_approx((float)(nl * (nk - nl)));
+  const double hi = (d + E), lo = fmax(d - E, 0.0);
+  gU = hi * hi * r * (1.0 + 9.5367431640625e-07);  // (1 + 2^-20)
+  gL = lo * lo * r * (1.0 - 9.5367431640625e-07);
+}
+
+constexpr int SUV = 15;              // scan: entries per thread (odd)
+constexpr int SUNIT = NT * SUV;      // 3840 entries per unit
+constexpr int PUV = 15;              // partition: entries per thread (odd)
+constexpr int PUNIT = NT * PUV;      // 3840 entries per unit
+
+// unit counts per item: mode 0 scan (node = i/div), 2 partition (node = i/div, split with a kept child)
+__global__ void k_unit_count(int mode, int nitems, int div, int unit, const LNode* nodes, const Split* split,
+                             const Child* child, int32_t* cnt) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= nitems) return;
+  const int k = i / div;
+  int a = nodes[k].a;
+  if (mode == 2) {
+    const int kl = child[2 * k].kind, kr = child[2 * k + 1].kind;
+    if (!split[k].split || (kl != KIND_LARGE && kl != KIND_SMALL && kr != KIND_LARGE && kr != KIND_SMALL)) a = 0;
+  }
+  cnt[i] = (a + unit - 1) / unit;
+}
+
+struct UnitArgs {
+  const LNode* nodes;
+  const int32_t* feat;  // scan: drawn feature per item (NULL for the partition: f = item % p)
+  int div;              // items per node (mtry or p)
+  int unit;
+  const uint64_t* E;
+  const int32_t* poff;
+  const int32_t* pmap;
+  const int32_t* ptotal;
+};
+
+__device__ __forceinline__ const uint64_t* unit_src(const UnitArgs& u, int t, int& item, int& k, int& cnt, LNode& nd,
+                                                    int& f) {
+  item = u.pmap[t];
+  k = t - u.poff[item];
+  const int node = item / u.div;
+  f = u.feat ? u.feat[item] : item - node * u.div;
+  nd = u.nodes[node];
+  cnt = min(u.unit, nd.a - k * u.unit);
+  return u.E + nd.base + (int64_t)f * nd.a + (int64_t)k * u.unit;
+}
+
+// pass 1 of the scan: (n, S) of every unit
+__global__ void __launch_bounds__(NT) k_unit_sums(UnitArgs u, const int64_t* yq, int64_t* un, int64_t* uS) {
+  __shared__ int32_t s1[NT / 32];
+  __shared__ int64_t s2[NT / 32];
+  const int total = *u.ptotal;
+  for (int t = blockIdx.x; t < total; t += gridDim.x) {
+    int item, k, cnt, f;
+    LNode nd;
+    const uint64_t* src = unit_src(u, t, item, k, cnt, nd, f);
+    int32_t c = 0;
+    int64_t S = 0;
+    constexpr int G = 8;
+    for (int j0 = threadIdx.x; j0 < cnt; j0 += G * NT) {
+      uint64_t ev[G];
+      int64_t yv[G];
+#pragma unroll
+      for (int q = 0; q < G; ++q) ev[q] = src[min(j0 + q * NT, cnt - 1)];
+#pragma unroll
+      for (int q = 0; q < G; ++q) yv[q] = ldg_s64_nc(yq + e_row(ev[q]));
+#pragma unroll
+      for (int q = 0; q < G; ++q)
+        if (j0 + q * NT < cnt) {
+          const int32_t w = e_w(ev[q]);
+          c += w;
+          S += (int64_t)w * yv[q];
+        }
+    }
+    int32_t tc;
+    int64_t tS;
+    block_excl_scan(c, s1, tc);
+    block_excl_scan(S, s2, tS);
+    if (threadIdx.x == 0) {
+      un[t] = tc;
+      uS[t] = tS;
+    }
+  }
+}
+
+// pass 1 of the partition: left count of every unit
+__global__ void __launch_bounds__(NT) k_unit_lefts(UnitArgs u, const uint8_t* side, int64_t n, int64_t* ul) {
+  __shared__ int64_t s1[NT / 32];
+  const int total = *u.ptotal;
+  for (int t = blockIdx.x; t < total; t += gridDim.x) {
+    int item, k, cnt, f;
+    LNode nd;
+    const uint64_t* src = unit_src(u, t, item, k, cnt, nd, f);
+    const uint8_t* sd = side + (int64_t)nd.b * n;
+    int64_t c = 0;
+    constexpr int G = 8;
+    for (int j0 = threadIdx.x; j0 < cnt; j0 += G * NT) {
+      uint32_t rw[G];
+      uint32_t sv[G];
+#pragma unroll
+      for (int q = 0; q < G; ++q) rw[q] = e_row(src[min(j0 + q * NT, cnt - 1)]);
+#pragma unroll
+      for (int q = 0; q < G; ++q) sv[q] = ldg_u8_nc(sd + rw[q]);
+#pragma unroll
+      for (int q = 0; q < G; ++q) c += (j0 + q * NT < cnt) && sv[q] == 0;
+    }
+    int64_t tc;
+    block_excl_scan(c, s1, tc);
+    if (threadIdx.x == 0) ul[t] = tc;
+  }
+}
+
+struct ScanArgs2 {
+  UnitArgs u;
+  const int64_t* yq;
+  const int64_t* pren;  // exclusive scan of unit n over all units
+  const int64_t* preS;
+  PieceRec* prec;
+};
+
+__global__ void __launch_bounds__(NT) k_split_scan_2p(ScanArgs2 g) {
+  extern __shared__ __align__(16) unsigned char dsm[];
+  uint64_t* bufs = (uint64_t*)dsm;  // 2 x (SUNIT + 4) entries
+  __shared__ uint64_t bar[2];
+  __shared__ int32_t smc[NT / 32];
+  __shared__ int64_t sms[NT / 32];
+  __shared__ double sg[NT / 32];
+  __shared__ uint32_t sr[NT / 32];
+  __shared__ int32_t sw[NT / 32];
+  __shared__ int s_off[2];
+  __shared__ double s_M;
+  const int total = *g.u.ptotal;
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  auto issue = [&](int t, int slot) {
+    int item, k, cnt, f;
+    LNode nd;
+    const uint64_t* src = unit_src(g.u, t, item, k, cnt, nd, f);
+    const int cload = min(cnt + 1, nd.a - k * SUNIT);
+    s_off[slot] = stage_entries(bufs + (size_t)slot * (SUNIT + 4), src, cload, &bar[slot]);
+  };
+  if (tid == 0) {
+    mbar_init(&bar[0]);
+    mbar_init(&bar[1]);
+    if ((int)blockIdx.x < total) issue(blockIdx.x, 0);
+  }
+  __syncthreads();
+  uint32_t phase[2] = {0u, 0u};
+  int cur = 0;
+  for (int t = blockIdx.x; t < total; t += gridDim.x, cur ^= 1) {
+    if (tid == 0 && t + (int)gridDim.x < total) issue(t + gridDim.x, cur ^ 1);  // prefetch the next unit
+    int item, k, cnt, f;
+    LNode nd;
+    unit_src(g.u, t, item, k, cnt, nd, f);
+    const int a = nd.a, u0 = k * SUNIT;
+    const int64_t nk = nd.n, Sk = nd.S;
+    const double nkd = (double)nk, Skd = (double)Sk;
+    const int t0 = g.u.poff[item];
+    const int32_t exn = (int32_t)(g.pren[t] - g.pren[t0]);
+    const int64_t exS = g.preS[t] - g.preS[t0];
+    mbar_wait(&bar[cur], phase[cur]);
+    phase[cur] ^= 1u;
+    const uint64_t* buf = bufs + (size_t)cur * (SUNIT + 4) + s_off[cur];
+    const int jl = tid * SUV;
+    // w*y_q of my entries: every gather issued before any is consumed
+    int64_t wy[SUV];
+    uint32_t rw[SUV];
+#pragma unroll
+    for (int q = 0; q < SUV; ++q) rw[q] = e_row(buf[min(jl + q, cnt - 1)]);
+#pragma unroll
+    for (int q = 0; q < SUV; ++q) wy[q] = ldg_s64_nc(g.yq + rw[q]);
+    int32_t tc = 0;
+    int64_t ts = 0;
+#pragma unroll
+    for (int q = 0; q < SUV; ++q) {
+      const int32_t w = jl + q < cnt ? e_w(buf[jl + q]) : 0;
+      wy[q] *= w;
+      tc += w;
+      ts += wy[q];
+    }
+    int32_t totc;
+    int64_t tots;
+    const int32_t prc0 = block_excl_scan(tc, smc, totc) + exn;
+    const int64_t prs0 = block_excl_scan(ts, sms, tots) + exS;
+    // pass 1: cheap bounds of every candidate; M = the unit's best lower bound
+    double mL = -1.0;
+    {
+      int32_t prc = prc0;
+      int64_t prs = prs0;
+#pragma unroll
+      for (int q = 0; q < SUV; ++q) {
+        const int j = jl + q;
+        if (j < cnt) {
+          const uint64_t e = buf[j];
+          prc += e_w(e);
+          prs += wy[q];
+          if (u0 + j + 1 < a && e_rank(e) != e_rank(buf[j + 1])) {
+            double gL, gU;
+            key_bounds(nkd, Skd, nk, prc, prs, gL, gU);
+            mL = fmax(mL, gL);
+          }
+        }
+      }
+    }
+    {
+      const uint64_t kb = gkey(mL);
+      const uint32_t hi = __reduce_max_sync(0xffffffffu, (uint32_t)(kb >> 32));
+      const uint32_t lo = __reduce_max_sync(0xffffffffu, ((uint32_t)(kb >> 32) == hi) ? (uint32_t)kb : 0u);
+      if (lane == 0) sg[wid] = (hi | lo) ? __longlong_as_double((long long)((((uint64_t)hi << 32) | lo) - 1ull)) : -1.0;
+      __syncthreads();
+      if (tid == 0) {
+        double M = -1.0;
+        for (int q = 0; q < NT / 32; ++q) M = fmax(M, sg[q]);
+        s_M = M;
+      }
+      __syncthreads();
+    }
+    const double M = s_M;
+    // pass 2: exact keys only where the upper bound reaches M
+    double bg = -1.0;
+    uint32_t brank = 0xffffffffu, brb = 0;
+    int32_t bpos = -1, bnl = 0;
+    int64_t bSl = 0;
+    {
+      int32_t prc = prc0;
+      int64_t prs = prs0;
+#pragma unroll
+      for (int q = 0; q < SUV; ++q) {
+        const int j = jl + q;
+        if (j < cnt) {
+          const uint64_t e = buf[j];
+          prc += e_w(e);
+          prs += wy[q];
+          if (u0 + j + 1 < a) {
+            const uint64_t en = buf[j + 1];
+            const uint32_t ra = e_rank(e), rb = e_rank(en);
+            if (ra != rb) {
+              double gL, gU;
+              key_bounds(nkd, Skd, nk, prc, prs, gL, gU);
+              if (gU >= M && gU >= bg) {
+                const double gk = split_key(nk, Sk, prc, prs);
+                if (rec_better(gk, ra, bg, brank)) {
+                  bg = gk;
+                  brank = ra;
+                  brb = rb;
+                  bpos = u0 + j;
+                  bnl = prc;
+                  bSl = prs;
+                }
+              }
+            }
+          }
+        }
+      }
+    }
+    const int wl = warp_argmax_key(gkey(bg), brank);
+    const double wg = __shfl_sync(0xffffffffu, bg, wl >= 0 ? wl : 0);
+    const uint32_t wr = __shfl_sync(0xffffffffu, brank, wl >= 0 ? wl : 0);
+    if (lane == 0) {
+      sg[wid] = wl >= 0 ? wg : -1.0;
+      sr[wid] = wl >= 0 ? wr : 0xffffffffu;
+      sw[wid] = wl >= 0 ? wid * 32 + wl : -1;
+    }
+    __syncthreads();
+    if (tid == 0) {
+      double gg = -1.0;
+      uint32_t r = 0xffffffffu;
+      int who = -1;
+      for (int q = 0; q < NT / 32; ++q)
+        if (sw[q] >= 0 && (who < 0 || rec_better(sg[q], sr[q], gg, r))) {
+          gg = sg[q];
+          r = sr[q];
+          who = sw[q];
+        }
+      sw[0] = who;
+      if (who < 0) {
+        PieceRec R;
+        R.g = -1.0;
+        R.rank_a = 0xffffffffu;
+        R.rank_b = 0;
+        R.pos = -1;
+        R.nl = 0;
+        R.Sl = 0;
+        g.prec[t] = R;
+      }
+    }
+    __syncthreads();
+    if (tid == sw[0]) {
+      PieceRec R;
+      R.g = bg;
+      R.rank_a = brank;
+      R.rank_b = brb;
+      R.pos = bpos;
+      R.nl = bnl;
+      R.Sl = bSl;
+      g.prec[t] = R;
+    }
+    __syncthreads();
+  }
+}
+
+struct PartArgs2 {
+  UnitArgs u;
+  const Child* child;
+  const uint8_t* side;
+  int64_t n;
+  uint64_t* Enext;
+  uint64_t* Esmall;
+  const int64_t* prel;  // exclusive scan of unit left counts over all units
+};
+
+__global__ void __launch_bounds__(NT) k_partition_2p(PartArgs2 g) {
+  extern __shared__ __align__(16) unsigned char dsm[];
+  uint64_t* bufs = (uint64_t*)dsm;              // 2 x (PUNIT + 2) entries (input)
+  uint64_t* outb = bufs + 2 * (PUNIT + 2);      // PUNIT entries (left part, then right part)
+  __shared__ uint64_t bar[2];
+  __shared__ int32_t sm[NT / 32];
+  __shared__ int s_off[2];
+  const int total = *g.u.ptotal;
+  const int tid = threadIdx.x;
+  auto issue = [&](int t, int slot) {
+    int item, k, cnt, f;
+    LNode nd;
+    const uint64_t* src = unit_src(g.u, t, item, k, cnt, nd, f);
+    s_off[slot] = stage_entries(bufs + (size_t)slot * (PUNIT + 2), src, cnt, &bar[slot]);
+  };
+  if (tid == 0) {
+    mbar_init(&bar[0]);
+    mbar_init(&bar[1]);
+    if ((int)blockIdx.x < total) issue(blockIdx.x, 0);
+  }
+  __syncthreads();
+  uint32_t phase[2] = {0u, 0u};
+  int cur = 0;
+  for (int t = blockIdx.x; t < total; t += gridDim.x, cur ^= 1) {
+    if (tid == 0 && t + (int)gridDim.x < total) issue(t + gridDim.x, cur ^ 1);
+    int item, k, cnt, f;
+    LNode nd;
+    unit_src(g.u, t, item, k, cnt, nd, f);
+    const int node = item / g.u.div;
+    const int u0 = k * PUNIT;
+    const Child cl = g.child[2 * node], cr = g.child[2 * node + 1];
+    const uint8_t* sd = g.side + (int64_t)nd.b * g.n;
+    const int64_t exl = g.prel[t] - g.prel[g.u.poff[item]];
+    mbar_wait(&bar[cur], phase[cur]);
+    phase[cur] ^= 1u;
+    const uint64_t* buf = bufs + (size_t)cur * (PUNIT + 2) + s_off[cur];
+    const int jl = tid * PUV;
+    // issue every side gather before consuming any (independent loads in flight)
+    uint32_t sv[PUV];  // one register per load (byte arrays get packed, which serialises the loads)
+    uint32_t rw[PUV];
+#pragma unroll
+    for (int q = 0; q < PUV; ++q) rw[q] = e_row(buf[min(jl + q, cnt - 1)]);
+#pragma unroll
+    for (int q = 0; q < PUV; ++q) sv[q] = ldg_u8_nc(sd + rw[q]);
+    uint32_t lmask = 0;
+    int32_t c = 0;
+#pragma unroll
+    for (int q = 0; q < PUV; ++q)
+      if (jl + q < cnt && sv[q] == 0) {
+        lmask |= 1u << q;
+        ++c;
+      }
+    int32_t tot;
+    const int32_t lbl = block_excl_scan(c, sm, tot);
+    int li = lbl, ri = tot + (jl - lbl);
+#pragma unroll
+    for (int q = 0; q < PUV; ++q) {
+      const int j = jl + q;
+      if (j < cnt) {
+        const uint64_t e = buf[j];
+        if ((lmask >> q) & 1u) outb[li++] = e;
+        else outb[ri++] = e;
+      }
+    }
+    __syncthreads();
+    const int64_t exr = (int64_t)u0 - exl;
+    const bool keepL = cl.kind == KIND_LARGE || cl.kind == KIND_SMALL;
+    const bool keepR = cr.kind == KIND_LARGE || cr.kind == KIND_SMALL;
+    if (keepL) {
+      uint64_t* dl = (cl.kind == KIND_LARGE ? g.Enext : g.Esmall) + cl.base + (int64_t)f * cl.a + exl;
+      for (int i = tid; i < tot; i += NT) dl[i] = outb[i];
+    }
+    if (keepR) {
+      uint64_t* dr = (cr.kind == KIND_LARGE ? g.Enext : g.Esmall) + cr.base + (int64_t)f * cr.a + exr;
+      for (int i = tid; i < cnt - tot; i += NT) dr[i] = outb[tot + i];
+    }
+    __syncthreads();
+  }
+}
+
+// ------------------------------------------------------------------ tree-affine item kernels (global phase v6)
+// Nodes of a level are ordered by tree, so each tree's items (node, feature)
+// form a contiguous range.  A CTA is bound to one tree and owns whole items
+// (round robin over the tree's items): it walks an item unit by unit with a
+// running carry -- no cross-CTA prefix, no look-back, no extra pass -- and the
+// bulk copy (TMA) of its next unit is in flight while it works on the current
+// one.  The partition kernel keeps the tree's goes-right bitmap (n bits) in
+// shared memory, so the per-entry side lookup is a shared-memory bit test.
+__global__ void k_tree_ranges(int N, const LNode* nodes, int32_t* lo, int32_t* hi) {
+  const int k = blockIdx.x * blockDim.x + threadIdx.x;
+  if (k >= N) return;
+  const int b = nodes[k].b;
+  if (k == 0 || nodes[k - 1].b != b) lo[b] = k;
+  if (k == N - 1 || nodes[k + 1].b != b) hi[b] = k + 1;
+}
+
+struct TreeSched {  // CTA -> (tree, slot, slots per tree)
+  int b0, bstep, c, C;
+};
+__device__ __forceinline__ TreeSched tree_sched(int B) {
+  const int G = gridDim.x, gi = blockIdx.x;
+  TreeSched s;
+  if (G >= B) {
+    s.b0 = gi % B;
+    s.bstep = B;  // single tree
+    s.c = gi / B;
+    s.C = G / B + (s.b0 < G % B ? 1 : 0);
+  } else {
+    s.b0 = gi;
+    s.bstep = G;
+    s.c = 0;
+    s.C = 1;
+  }
+  return s;
+}
+
+struct TScanArgs {
+  const LNode* nodes;
+  const int32_t* feat;
+  int mtry, B;
+  const uint64_t* E;
+  const int64_t* yq;
+  const int32_t* tlo;  // per tree: first node of the level (or 0) / one past the last
+  const int32_t* thi;
+  Rec* rec;
+};
+
+constexpr int TSV = 15;             // entries per thread (odd: conflict-free 64-bit shared loads)
+constexpr int TUNIT = NT * TSV;     // 3840 entries per unit
+
+// a7 split search: one CTA owns whole (node, drawn feature) items of one tree
+__global__ void __launch_bounds__(NT) k_split_scan_tree(TScanArgs g) {
+  extern __shared__ __align__(16) unsigned char dsm[];
+  uint64_t* bufs = (uint64_t*)dsm;  // 2 x (TUNIT + 4)
+  __shared__ uint64_t bar[2];
+  __shared__ int32_t smc[NT / 32];
+  __shared__ int64_t sms[NT / 32];
+  __shared__ double sg[NT / 32];
+  __shared__ uint32_t sr[NT / 32];
+  __shared__ int32_t sw[NT / 32];
+  __shared__ int s_off[2];
+  __shared__ double s_M;
+  __shared__ int64_t s_cS;
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const TreeSched ts = tree_sched(g.B);
+  if (tid == 0) {
+    mbar_init(&bar[0]);
+    mbar_init(&bar[1]);
+  }
+  __syncthreads();
+  uint32_t phase[2] = {0u, 0u};
+  int cur = 0;
+  for (int b = ts.b0; b < g.B; b += ts.bstep) {
+    const int i_lo = g.tlo[b] * g.mtry, i_hi = g.thi[b] * g.mtry;
+    // sequence of (item, unit) of this CTA: items i_lo + c, + C, ...; units 0.. of each
+    int item = i_lo + ts.c, unit = 0;
+    auto units_of = [&](int it) { return (g.nodes[it / g.mtry].a + TUNIT - 1) / TUNIT; };
+    auto issue = [&](int it, int un, int slot) {
+      const LNode nd = g.nodes[it / g.mtry];
+      const int f = g.feat[it];
+      const int u0 = un * TUNIT;
+      const int cload = min(TUNIT + 1, nd.a - u0);
+      s_off[slot] = stage_entries(bufs + (size_t)slot * (TUNIT + 4), g.E + nd.base + (int64_t)f * nd.a + u0, cload,
+                                  &bar[slot]);
+    };
+    if (item >= i_hi) continue;
+    if (tid == 0) issue(item, 0, cur);
+    // running state of the current item
+    int32_t carry_n = 0;
+    int64_t carry_S = 0;
+    double ig = -1.0;
+    uint32_t irk = 0xffffffffu, irb = 0;
+    int32_t ipos = -1, inl = 0;
+    int64_t iSl = 0;
+    while (item < i_hi) {
+      const int nun = units_of(item);
+      // next (item, unit) to prefetch
+      int nitem = item, nunit = unit + 1;
+      if (nunit >= nun) {
+        nitem = item + ts.C;
+        nunit = 0;
+      }
+      __syncthreads();  // the other buffer is free
+      if (tid == 0 && nitem < i_hi) issue(nitem, nunit, cur ^ 1);
+      const LNode nd = g.nodes[item / g.mtry];
+      const int a = nd.a, u0 = unit * TUNIT, cnt = min(TUNIT, a - u0);
+      const int64_t nk = nd.n, Sk = nd.S;
+      const double nkd = (double)nk, Skd = (double)Sk;
+      mbar_wait(&bar[cur], phase[cur]);
+      phase[cur] ^= 1u;
+      const uint64_t* buf = bufs + (size_t)cur * (TUNIT + 4) + s_off[cur];
+      const int jl = tid * TSV;
+      uint32_t rw[TSV];
+      int64_t wy[TSV];
+#pragma unroll
+      for (int q = 0; q < TSV; ++q) rw[q] = e_row(buf[min(jl + q, cnt - 1)]);
+#pragma unroll
+      for (int q = 0; q < TSV; ++q) wy[q] = ldg_s64_nc(g.yq + rw[q]);
+      int32_t tc = 0;
+      int64_t tsum = 0;
+#pragma unroll
+      for (int q = 0; q < TSV; ++q) {
+        const int32_t w = jl + q < cnt ? e_w(buf[jl + q]) : 0;
+        wy[q] *= w;
+        tc += w;
+        tsum += wy[q];
+      }
+      int32_t totc;
+      int64_t tots;
+      const int32_t prc0 = block_excl_scan(tc, smc, totc) + carry_n;
+      const int64_t prs0 = block_excl_scan(tsum, sms, tots) + carry_S;
+      // pass 1: bounds; M = the unit's best lower bound (or the item's running best)
+      double mL = ig;
+      {
+        int32_t prc = prc0;
+        int64_t prs = prs0;
+#pragma unroll
+        for (int q = 0; q < TSV; ++q) {
+          const int j = jl + q;
+          if (j < cnt) {
+            const uint64_t e = buf[j];
+            prc += e_w(e);
+            prs += wy[q];
+            if (u0 + j + 1 < a && e_rank(e) != e_rank(buf[j + 1])) {
+              double gL, gU;
+              key_bounds(nkd, Skd, nk, prc, prs, gL, gU);
+              mL = fmax(mL, gL);
+            }
+          }
+        }
+      }
+      {
+        const uint64_t kb = gkey(mL);
+        const uint32_t hi = __reduce_max_sync(0xffffffffu, (uint32_t)(kb >> 32));
+        const uint32_t lo = __reduce_max_sync(0xffffffffu, ((uint32_t)(kb >> 32) == hi) ? (uint32_t)kb : 0u);
+        if (lane == 0) sg[wid] = (hi | lo) ? __longlong_as_double((long long)((((uint64_t)hi << 32) | lo) - 1ull)) : -1.0;
+        __syncthreads();
+        if (tid == 0) {
+          double M = -1.0;
+          for (int q = 0; q < NT / 32; ++q) M = fmax(M, sg[q]);
+          s_M = M;
+        }
+        __syncthreads();
+      }
+      const double M = s_M;
+      double bg = -1.0;
+      uint32_t brank = 0xffffffffu, brb = 0;
+      int32_t bpos = -1, bnl = 0;
+      int64_t bSl = 0;
+      {
+        int32_t prc = prc0;
+        int64_t prs = prs0;
+#pragma unroll
+        for (int q = 0; q < TSV; ++q) {
+          const int j = jl + q;
+          if (j < cnt) {
+            const uint64_t e = buf[j];
+            prc += e_w(e);
+            prs += wy[q];
+            if (u0 + j + 1 < a) {
+              const uint64_t en = buf[j + 1];
+              const uint32_t ra = e_rank(e), rb = e_rank(en);
+              if (ra != rb) {
+                double gL, gU;
+                key_bounds(nkd, Skd, nk, prc, prs, gL, gU);
+                if (gU >= M && gU >= bg) {
+                  const double gk = split_key(nk, Sk, prc, prs);
+                  if (rec_better(gk, ra, bg, brank)) {
+                    bg = gk;
+                    brank = ra;
+                    brb = rb;
+                    bpos = u0 + j;
+                    bnl = prc;
+                    bSl = prs;
+                  }
+                }
+              }
+            }
+          }
+        }
+      }
+      const int wl = warp_argmax_key(gkey(bg), brank);
+      const double wg = __shfl_sync(0xffffffffu, bg, wl >= 0 ? wl : 0);
+      const uint32_t wr = __shfl_sync(0xffffffffu, brank, wl >= 0 ? wl : 0);
+      if (lane == 0) {
+        sg[wid] = wl >= 0 ? wg : -1.0;
+        sr[wid] = wl >= 0 ? wr : 0xffffffffu;
+        sw[wid] = wl >= 0 ? wid * 32 + wl : -1;
+      }
+      __syncthreads();
+      if (tid == 0) {
+        double gg = -1.0;
+        uint32_t r = 0xffffffffu;
+        int who = -1;
+        for (int q = 0; q < NT / 32; ++q)
+          if (sw[q] >= 0 && (who < 0 || rec_better(sg[q], sr[q], gg, r))) {
+            gg = sg[q];
+            r = sr[q];
+            who = sw[q];
+          }
+        sw[0] = who;
+      }
+      __syncthreads();
+      const int who = sw[0];
+      if (who >= 0) {  // broadcast the unit winner; merge into the item's running best (unit order == position order)
+        if (tid == who) {
+          sg[0] = bg;
+          sr[0] = brank;
+          sw[1] = (int)brb;
+          sw[2] = bpos;
+          sw[3] = bnl;
+          s_cS = bSl;
+        }
+        __syncthreads();
+        const double ug = sg[0];
+        if (ug > ig) {  // strictly better (an equal key in a later unit has a higher rank)
+          ig = ug;
+          irk = sr[0];
+          irb = (uint32_t)sw[1];
+          ipos = sw[2];
+          inl = sw[3];
+          iSl = s_cS;
+        }
+        __syncthreads();
+      }
+      carry_n += totc;
+      carry_S += tots;
+      if (unit + 1 >= nun) {  // item done
+        if (tid == 0) {
+          Rec R;
+          R.g = ig;
+          R.rank_a = irk;
+          R.rank_b = irb;
+          R.pos = ipos;
+          R.nl = inl;
+          R.Sl = iSl;
+          g.rec[item] = R;
+        }
+        carry_n = 0;
+        carry_S = 0;
+        ig = -1.0;
+        irk = 0xffffffffu;
+        irb = 0;
+        ipos = -1;
+        inl = 0;
+        iSl = 0;
+      }
+      item = nitem;
+      unit = nunit;
+      cur ^= 1;
+    }
+  }
+}
+
+struct TPartArgs {
+  const LNode* nodes;
+  const Split* split;
+  const Child* child;
+  int p, B;
+  const uint64_t* Ecur;
+  const uint32_t* sideb;  // per tree: n bits, 1 = goes right
+  int64_t nw;             // words per tree
+  int bitmap_smem;        // 1: stage the tree's bitmap in shared memory
+  uint64_t* Enext;
+  uint64_t* Esmall;
+  const int32_t* tlo;
+  const int32_t* thi;
+};
+
+constexpr int TPNT = 512;           // threads of the partition CTA (one CTA per SM: the bitmap fills shared memory)
+constexpr int TPV = 7;
+constexpr int TPUNIT = TPNT * TPV;  // 3584 entries per unit
+
+__device__ __forceinline__ bool part_item_active(const Split* split, const Child* child, int node) {
+  if (!split[node].split) return false;
+  const int kl = child[2 * node].kind, kr = child[2 * node + 1].kind;
+  return kl == KIND_LARGE || kl == KIND_SMALL || kr == KIND_LARGE || kr == KIND_SMALL;
+}
+
+// a9 partition: one CTA owns whole (node, feature) items of one tree; lefts first, stable
+__global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
+  extern __shared__ __align__(16) unsigned char dsm[];
+  uint64_t* bufs = (uint64_t*)dsm;              // 2 x (TPUNIT + 2)
+  uint64_t* outb = bufs + 2 * (TPUNIT + 2);     // TPUNIT
+  uint32_t* bm = (uint32_t*)(outb + TPUNIT);    // nw words (if staged)
+  __shared__ uint64_t bar[2];
+  __shared__ int32_t sm[TPNT / 32];
+  __shared__ int s_off[2];
+  const int tid = threadIdx.x;
+  const TreeSched ts = tree_sched(g.B);
+  if (tid == 0) {
+    mbar_init(&bar[0]);
+    mbar_init(&bar[1]);
+  }
+  __syncthreads();
+  uint32_t phase[2] = {0u, 0u};
+  int cur = 0;
+  for (int b = ts.b0; b < g.B; b += ts.bstep) {
+    const int i_lo = g.tlo[b] * g.p, i_hi = g.thi[b] * g.p;
+    if (i_lo >= i_hi) continue;
+    const uint32_t* sideg = g.sideb + (int64_t)b * g.nw;
+    __syncthreads();
+    if (g.bitmap_smem)
+      for (int64_t w = tid; w < g.nw; w += TPNT) bm[w] = sideg[w];
+    const uint32_t* sb = g.bitmap_smem ? bm : sideg;
+    auto next_item = [&](int it) {  // next active item of this CTA at or after it
+      while (it < i_hi && !part_item_active(g.split, g.child, it / g.p)) it += ts.C;
+      return it;
+    };
+    auto issue = [&](int it, int un, int slot) {
+      const LNode nd = g.nodes[it / g.p];
+      const int f = it - (it / g.p) * g.p;
+      const int u0 = un * TPUNIT;
+      s_off[slot] = stage_entries(bufs + (size_t)slot * (TPUNIT + 2), g.Ecur + nd.base + (int64_t)f * nd.a + u0,
+                                  min(TPUNIT, nd.a - u0), &bar[slot]);
+    };
+    int item = next_item(i_lo + ts.c), unit = 0;
+    if (item >= i_hi) continue;
+    if (tid == 0) issue(item, 0, cur);
+    int64_t carry_l = 0;
+    while (item < i_hi) {
+      const int node = item / g.p, f = item - node * g.p;
+      const LNode nd = g.nodes[node];
+      const int nun = (nd.a + TPUNIT - 1) / TPUNIT;
+      int nitem = item, nunit = unit + 1;
+      if (nunit >= nun) {
+        nitem = next_item(item + ts.C);
+        nunit = 0;
+      }
+      __syncthreads();
+      if (tid == 0 && nitem < i_hi) issue(nitem, nunit, cur ^ 1);
+      const int u0 = unit * TPUNIT, cnt = min(TPUNIT, nd.a - u0);
+      const Child cl = g.child[2 * node], cr = g.child[2 * node + 1];
+      mbar_wait(&bar[cur], phase[cur]);
+      phase[cur] ^= 1u;
+      const uint64_t* buf = bufs + (size_t)cur * (TPUNIT + 2) + s_off[cur];
+      const int jl = tid * TPV;
+      uint32_t lmask = 0;
+      int32_t c = 0;
+#pragma unroll
+      for (int q = 0; q < TPV; ++q) {
+        const int j = jl + q;
+        if (j < cnt) {
+          const uint32_t r = e_row(buf[j]);
+          if (!((sb[r >> 5] >> (r & 31)) & 1u)) {
+            lmask |= 1u << q;
+            ++c;
+          }
+        }
+      }
+      int32_t tot;
+      const int32_t lbl = block_excl_scan(c, sm, tot);
+      int li = lbl, ri = tot + (jl - lbl);
+#pragma unroll
+      for (int q = 0; q < TPV; ++q) {
+        const int j = jl + q;
+        if (j < cnt) {
+          const uint64_t e = buf[j];
+          if ((lmask >> q) & 1u) outb[li++] = e;
+          else outb[ri++] = e;
+        }
+      }
+      __syncthreads();
+      const int64_t exl = carry_l, exr = (int64_t)u0 - carry_l;
+      const bool keepL = cl.kind == KIND_LARGE || cl.kind == KIND_SMALL;
+      const bool keepR = cr.kind == KIND_LARGE || cr.kind == KIND_SMALL;
+      if (keepL) {
+        uint64_t* dl = (cl.kind == KIND_LARGE ? g.Enext : g.Esmall) + cl.base + (int64_t)f * cl.a + exl;
+        for (int i = tid; i < tot; i += TPNT) dl[i] = outb[i];
+      }
+      if (keepR) {
+        uint64_t* dr = (cr.kind == KIND_LARGE ? g.Enext : g.Esmall) + cr.base + (int64_t)f * cr.a + exr;
+        for (int i = tid; i < cnt - tot; i += TPNT) dr[i] = outb[tot + i];
+      }
+      carry_l += tot;
+      if (nunit == 0) carry_l = 0;
+      item = nitem;
+      unit = nunit;
+      cur ^= 1;
+    }
+  }
+}
+
+// goes-right bitmap of the rows of every split node (from its winning segment) + child sums of w*y
+__global__ void __launch_bounds__(NT) k_dest_bits(DestArgs g, uint32_t* sideb, int64_t nw) {
+  __shared__ double sl[NT / 32], sr[NT / 32];
+  const int t = blockIdx.x;
+  if (t >= *g.ptotal) return;
+  const int k = g.pmap[t], pc = t - g.poff[k];
+  const Split sp = g.split[k];
+  const LNode nd = g.nodes[k];
+  const uint64_t* seg = g.E + nd.base + (int64_t)sp.f * nd.a;
+  uint32_t* sb = sideb + (int64_t)nd.b * nw;
+  double accl = 0.0, accr = 0.0;
+  const int j0 = pc * PIECE + threadIdx.x * PIECE_V;
+  uint64_t ev[PIECE_V];
+  double yv[PIECE_V];
+#pragma unroll
+  for (int u = 0; u < PIECE_V; ++u) ev[u] = seg[min(j0 + u, nd.a - 1)];
+#pragma unroll
+  for (int u = 0; u < PIECE_V; ++u) yv[u] = __ldg(g.y + e_row(ev[u]));
+#pragma unroll
+  for (int u = 0; u < PIECE_V; ++u) {
+    const int j = j0 + u;
+    if (j < nd.a) {
+      const uint32_t row = e_row(ev[u]);
+      const int s = j > sp.pos;
+      if (s) atomicOr(&sb[row >> 5], 1u << (row & 31));
+      else atomicAnd(&sb[row >> 5], ~(1u << (row & 31)));
+      const double v = __dmul_rn((double)e_w(ev[u]), yv[u]);
+      if (s) accr += v;
+      else accl += v;
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    accl += __shfl_down_sync(0xffffffffu, accl, o);
+    accr += __shfl_down_sync(0xffffffffu, accr, o);
+  }
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  if (lane == 0) {
+    sl[wid] = accl;
+    sr[wid] = accr;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double a0 = 0.0, a1 = 0.0;
+    for (int q = 0; q < NT / 32; ++q) {
+      a0 += sl[q];
+      a1 += sr[q];
+    }
+    atomicAdd(&g.csum[2 * k], a0);
+    atomicAdd(&g.csum[2 * k + 1], a1);
+  }
+}
+
 // ------------------------------------------------------------------ subtree phase (one CTA per small node)
 // Layout: the subtree's rows occupy local ids 0..a0-1.  list[f][0..a0) holds
 // feature f's entries ((local rank << 16) | local row) sorted by value.  A
@@ -1371,7 +2748,8 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         __syncwarp();
       }
       const int wlane = warp_argmax_key(gkey(lg), ltie);
-      const double bg = wlane >= 0 ? __shfl_sync(0xffffffffu, lg, wlane) : -1.0;
+      const double bgs = __shfl_sync(0xffffffffu, lg, wlane >= 0 ? wlane : 0);
+      const double bg = wlane >= 0 ? bgs : -1.0;
       if (bg > 0.0) {
         const uint32_t tie = __shfl_sync(0xffffffffu, ltie, wlane);
         const int bf = (int)(tie >> 16);
@@ -1809,6 +3187,85 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
     DBuf<char> scan_tmp(std::max<size_t>(scan_tb, 16), s);
     DBuf<LevelSummary> dsum(1, s);
     PinnedSummary hs;
+    // piece decomposition buffers (sized for the largest level of a batch)
+    const int64_t cap_items = cap_level * p;
+    const int64_t cap_pieces = (int64_t)p * ((int64_t)B * n / PIECE + cap_level) + 1;
+    const int64_t cap_spieces = (int64_t)mtry * ((int64_t)B * n / PIECE + cap_level) + 1;
+    DBuf<int32_t> pcnt(cap_items, s), poff(cap_items, s), pmap(cap_pieces, s), ptot(1, s);
+    DBuf<LbNS> lbagg(cap_spieces, s), lbincl(cap_spieces, s);
+    DBuf<uint32_t> lbflag(cap_spieces, s);
+    DBuf<PieceRec> prec(cap_spieces, s);
+    DBuf<unsigned long long> pst(cap_pieces, s);
+    DBuf<unsigned int> ticket(1, s);
+    DBuf<int64_t> un(cap_pieces, s), pren(cap_pieces, s);
+    DBuf<int64_t> uS(cap_pieces, s), preS(cap_pieces, s), ul(cap_pieces, s), prel(cap_pieces, s);
+    size_t unit_tb = 0, unit_tb2 = 0;
+    cub::DeviceScan::ExclusiveSum(nullptr, unit_tb, uS.p, preS.p, (int)cap_pieces, s);
+    cub::DeviceScan::ExclusiveSum(nullptr, unit_tb2, un.p, pren.p, (int)cap_pieces, s);
+    unit_tb = std::max(unit_tb, unit_tb2);
+    DBuf<char> unit_tmp(std::max<size_t>(unit_tb, 16), s);
+    DBuf<double> csum(2 * cap_level, s);
+    size_t piece_tb = 0;
+    cub::DeviceScan::ExclusiveSum(nullptr, piece_tb, pcnt.p, poff.p, (int)cap_items, s);
+    DBuf<char> piece_tmp(std::max<size_t>(piece_tb, 16), s);
+    auto piece_setup = [&](int mode, int nitems, int div, const LNode* nodes, const Split* sp, const Child* ch,
+                           int32_t* cnt, int32_t* off, int32_t* map, int32_t* tot, cudaStream_t st) {
+      {
+        KScope ks_("k_piece_count", st, 0.0);
+        k_piece_count<<<(unsigned)ceil_div(nitems, 256), 256, 0, st>>>(mode, nitems, div, nodes, sp, ch, cnt);
+      }
+      {
+        KScope ks_("cub_ExclusiveSum", st, 0.0);
+        size_t tb2 = piece_tb;
+        BF_CUDA_CHECK(cub::DeviceScan::ExclusiveSum(piece_tmp.p, tb2, cnt, off, nitems, st));
+      }
+      {
+        KScope ks_("k_piece_map", st, 0.0);
+        k_piece_map<<<(unsigned)ceil_div(nitems, 256), 256, 0, st>>>(nitems, cnt, off, map, tot);
+      }
+    };
+    auto unit_setup = [&](int mode, int nitems, int div, int unit, const LNode* nodes, const Split* sp, const Child* ch,
+                          int32_t* cnt, int32_t* off, int32_t* map, int32_t* tot, cudaStream_t st) {
+      {
+        KScope ks_("k_piece_count", st, 0.0);
+        k_unit_count<<<(unsigned)ceil_div(nitems, 256), 256, 0, st>>>(mode, nitems, div, unit, nodes, sp, ch, cnt);
+      }
+      {
+        KScope ks_("cub_ExclusiveSum", st, 0.0);
+        size_t tb2 = piece_tb;
+        BF_CUDA_CHECK(cub::DeviceScan::ExclusiveSum(piece_tmp.p, tb2, cnt, off, nitems, st));
+      }
+      {
+        KScope ks_("k_piece_map", st, 0.0);
+        k_piece_map<<<(unsigned)ceil_div(nitems, 256), 256, 0, st>>>(nitems, cnt, off, map, tot);
+      }
+    };
+    const size_t scan_smem = sizeof(uint64_t) * 2 * (SUNIT + 4), part_smem = sizeof(uint64_t) * (3 * PUNIT + 4);
+    BF_CUDA_CHECK(cudaFuncSetAttribute(k_split_scan_2p, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)scan_smem));
+    BF_CUDA_CHECK(cudaFuncSetAttribute(k_partition_2p, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)part_smem));
+    int occ_s = 0, occ_p = 0, nsm = 0, dev_id = 0;
+    cudaGetDevice(&dev_id);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev_id);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_s, k_split_scan_2p, NT, scan_smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_p, k_partition_2p, NT, part_smem);
+    int occ_u = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_u, k_unit_lefts, NT, 0);
+    const unsigned grid_scan = (unsigned)std::max(1, occ_s * nsm), grid_part = (unsigned)std::max(1, occ_p * nsm);
+    const unsigned grid_sums = (unsigned)std::max(1, occ_u * nsm);
+    // tree-affine kernels
+    const int64_t nw = (n + 31) / 32;
+    DBuf<uint32_t> sideb((size_t)B * nw, s);
+    DBuf<int32_t> tlo(B, s), thi(B, s);
+    const size_t tscan_smem = sizeof(uint64_t) * 2 * (TUNIT + 4);
+    const size_t tpart_base = sizeof(uint64_t) * (3 * TPUNIT + 4);
+    const int smem_optin = dyn_smem_limit(k_partition_tree);
+    const bool bm_smem = tpart_base + (size_t)nw * 4 <= (size_t)smem_optin;
+    const size_t tpart_smem = tpart_base + (bm_smem ? (size_t)nw * 4 : 0);
+    BF_CUDA_CHECK(cudaFuncSetAttribute(k_split_scan_tree, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tscan_smem));
+    int occ_ts = 0, occ_tp = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_ts, k_split_scan_tree, NT, tscan_smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_tp, k_partition_tree, TPNT, tpart_smem);
+    const unsigned grid_tscan = (unsigned)std::max(1, occ_ts * nsm), grid_tpart = (unsigned)std::max(1, occ_tp * nsm);
     DBuf<uint64_t> E0, E1, Es;
     size_t E_cap = 0;
 
@@ -1857,9 +3314,9 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
       for (int b = 0; b < Bc; ++b) need += (size_t)p * ha[b];
       need = std::max<size_t>(need, 1);
       if (need > E_cap) {
-        E0.alloc(need, s);
-        E1.alloc(need, s);
-        Es.alloc(need, s);
+        E0.alloc(need + 16, s);
+        E1.alloc(need + 16, s);
+        Es.alloc(need + 16, s);
         E_cap = need;
       }
       h2d(kind_d.p, hk.data(), Bc, s);
@@ -1901,19 +3358,28 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
       h2d(dsum.p, &ls, 1, s);
       // ---- global phase
       int N = nL;
-      int64_t cur_elems = offL;
+      int64_t cur_elems = offL;  // sum of p*a over the level's nodes
       uint64_t* Ec = E0.p;
       uint64_t* En = E1.p;
       LNode* nc = ncur.p;
       LNode* nx = nnext.p;
       while (N > 0) {
+        const int64_t cur_a = cur_elems / p;  // sum of a over the level's nodes
         {
           KScope ks_("k_mtry", s, 0.0);
           k_mtry<<<(unsigned)ceil_div(N, 128), 128, 0, s>>>(nc, N, p, mtry, prm.seed, tb, feat.p, fyscr.p);
         }
+        // ---- a7 split search: tree-affine CTAs own whole items
+        BF_CUDA_CHECK(cudaMemsetAsync(tlo.p, 0, sizeof(int32_t) * Bc, s));
+        BF_CUDA_CHECK(cudaMemsetAsync(thi.p, 0, sizeof(int32_t) * Bc, s));
         {
+          KScope ks_("k_tree_ranges", s, 0.0);
+          k_tree_ranges<<<(unsigned)ceil_div(N, 256), 256, 0, s>>>(N, nc, tlo.p, thi.p);
+        }
+        {
+          TScanArgs ga{nc, feat.p, mtry, Bc, Ec, yq.p, tlo.p, thi.p, rec.p};
           KScope ks_("k_split_scan", s, 0.0);
-          k_split_scan<<<(unsigned)((int64_t)N * mtry), NT, 0, s>>>(nc, feat.p, mtry, Ec, yq.p, rec.p);
+          k_split_scan_tree<<<grid_tscan, NT, tscan_smem, s>>>(ga);
         }
         {
           KScope ks_("k_finalize", s, 0.0);
@@ -1937,13 +3403,23 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
           k_child_place<<<(unsigned)ceil_div(N2, 128), 128, 0, s>>>(N2, p, nc, child.p, scanL.p, scanS.p, nx, sq.p,
                                                                     dsum.p);
         }
+        // ---- a9/a10 goes-right flags and child values over pieces of the winning segments
+        piece_setup(1, N, 1, nc, split.p, child.p, pcnt.p, poff.p, pmap.p, ptot.p, s);
+        BF_CUDA_CHECK(cudaMemsetAsync(csum.p, 0, sizeof(double) * 2 * (size_t)N, s));
         {
+          DestArgs ga{nc, split.p, Ec, y, n, side.p, poff.p, pmap.p, ptot.p, csum.p};
           KScope ks_("k_dest", s, 0.0);
-          k_dest<<<(unsigned)N, NT, 0, s>>>(nc, split.p, Ec, y, n, side.p, pool);
+          k_dest_bits<<<(unsigned)(cur_a / PIECE + N + 1), NT, 0, s>>>(ga, sideb.p, nw);
         }
         {
-          KScope ks_("k_partition", 0, 0.0);
-          k_partition<<<dim3((unsigned)N, (unsigned)p), NT, 0, s>>>(nc, split.p, child.p, p, Ec, side.p, n, En, Es.p);
+          KScope ks_("k_child_values", s, 0.0);
+          k_child_values<<<(unsigned)ceil_div(N, 128), 128, 0, s>>>(N, split.p, csum.p, nc, pool);
+        }
+        // ---- a9 partition: tree-affine CTAs own whole items; goes-right bitmap in shared memory
+        {
+          TPartArgs ga{nc, split.p, child.p, p, Bc, Ec, sideb.p, nw, bm_smem ? 1 : 0, En, Es.p, tlo.p, thi.p};
+          KScope ks_("k_partition", s, 0.0);
+          k_partition_tree<<<grid_tpart, TPNT, tpart_smem, s>>>(ga);
         }
         {
           KScope ks_("k_commit", s, 0.0);
@@ -1952,9 +3428,9 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
         BF_CUDA_CHECK(cudaGetLastError());
         BF_CUDA_CHECK(cudaStreamSynchronize(s));
         {  // algorithmic bytes
-          const double cur_a = (double)cur_elems / p, sa = (double)hs.h->split_a;
-          prof_add_bytes("k_split_scan", cur_a * mtry * 20.0);
-          prof_add_bytes("k_dest", sa * 21.0);
+          const double sa = (double)hs.h->split_a;
+          prof_add_bytes("k_split_scan", (double)cur_a * mtry * 16.0);
+          prof_add_bytes("k_dest", sa * 17.0);
           prof_add_bytes("k_partition", sa * p * 17.0);
         }
         cur_elems = hs.h->next_elems;
