@@ -1272,6 +1272,11 @@ __device__ __forceinline__ uint32_t ldg_u8_nc(const uint8_t* p) {
   asm volatile("ld.global.nc.u8 %0, [%1];" : "=r"(v) : "l"(p));
   return v;
 }
+__device__ __forceinline__ uint32_t ldg_u32_nc(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.global.nc.u32 %0, [%1];" : "=r"(v) : "l"(p));
+  return v;
+}
 __device__ __forceinline__ int64_t ldg_s64_nc(const int64_t* p) {
   int64_t v;
   asm volatile("ld.global.nc.s64 %0, [%1];" : "=l"(v) : "l"(p));
@@ -1294,7 +1299,36 @@ __device__ __forceinline__ void key_bounds(double nkd, double Skd, int64_t nk, i
   gL = lo * lo * r * (1.0 - 9.5367431640625e-07);
 }
 
-constexpr int SUV = 15;              // scan: entries per thread (odd)
+// Cheap rigorous upper bound of the S4.3 key in fp32, scaled by 2^-128 (no
+// overflow): with a = RN32(nk)*RN32(Sl), b = RN32(nl)*RN32(Sk), d = |a - b|,
+// |d - D| <= 2^-21.5 (|a| + |b|), so (d + E)^2 * rcp(nl*nr) * (1 + 2^-18) with
+// E = 2^-20 (|a| + |b|) bounds g from above.  Results below 2^-100 (scaled)
+// are raised to 2^-100 so that an fp32 underflow never screens a candidate
+// out: every candidate whose bound reaches the threshold is evaluated exactly.
+__device__ __forceinline__ float key_upper32(float nkf, float Skf, int32_t nl, int32_t nr, int64_t Sl) {
+  const float a = nkf * (float)Sl * 5.421010862427522e-20f;  // * 2^-64
+  const float b = (float)nl * Skf * 5.421010862427522e-20f;
+  const float d = fabsf(a - b);
+  const float E = (fabsf(a) + fabsf(b)) * 9.5367431640625e-07f;  // 2^-20
+  const float u = d + E;
+  const float r = rcp_approx((float)nl * (float)nr);
+  return fmaxf(u * u * r * 1.0000038146972656f, 7.888609052210118e-31f);  // (1 + 2^-18), floor 2^-100
+}
+__device__ __forceinline__ float key_lower32(float nkf, float Skf, int32_t nl, int32_t nr, int64_t Sl) {
+  const float a = nkf * (float)Sl * 5.421010862427522e-20f;
+  const float b = (float)nl * Skf * 5.421010862427522e-20f;
+  const float d = fabsf(a - b);
+  const float E = (fabsf(a) + fabsf(b)) * 9.5367431640625e-07f;
+  const float u = fmaxf(d - E, 0.0f);
+  const float r = rcp_approx((float)nl * (float)nr);
+  return u * u * r * 0.9999961853027344f;  // (1 - 2^-18)
+}
+__device__ __forceinline__ float scale_key(double g) {  // g * 2^-128, rounded down
+  const float f = (float)(g * 2.938735877055719e-39);
+  return f > 0.0f ? __fmul_rd(f, 0.99999988079071044921875f) : f;
+}
+
+constexpr int SUV = 7;               // scan: entries per thread (odd)
 constexpr int SUNIT = NT * SUV;      // 3840 entries per unit
 constexpr int PUV = 15;              // partition: entries per thread (odd)
 constexpr int PUNIT = NT * PUV;      // 3840 entries per unit
@@ -1408,6 +1442,18 @@ struct ScanArgs2 {
   PieceRec* prec;
 };
 
+__device__ __forceinline__ void key_bounds32(float nkf, float Skf, int32_t nl, int32_t nr, int64_t Sl, float& gL,
+                                             float& gU) {
+  const float a = nkf * (float)Sl * 5.421010862427522e-20f;  // * 2^-64
+  const float b = (float)nl * Skf * 5.421010862427522e-20f;
+  const float d = fabsf(a - b);
+  const float E = (fabsf(a) + fabsf(b)) * 9.5367431640625e-07f;  // 2^-20
+  const float r = rcp_approx((float)nl * (float)nr);
+  const float hi = d + E, lo = fmaxf(d - E, 0.0f);
+  gU = fmaxf(hi * hi * r * 1.0000038146972656f, 7.888609052210118e-31f);
+  gL = lo * lo * r * 0.9999961853027344f;
+}
+
 __global__ void __launch_bounds__(NT) k_split_scan_2p(ScanArgs2 g) {
   extern __shared__ __align__(16) unsigned char dsm[];
   uint64_t* bufs = (uint64_t*)dsm;  // 2 x (SUNIT + 4) entries
@@ -1417,8 +1463,9 @@ __global__ void __launch_bounds__(NT) k_split_scan_2p(ScanArgs2 g) {
   __shared__ double sg[NT / 32];
   __shared__ uint32_t sr[NT / 32];
   __shared__ int32_t sw[NT / 32];
+  __shared__ float sf[NT / 32];
   __shared__ int s_off[2];
-  __shared__ double s_M;
+  __shared__ float s_M;
   const int total = *g.u.ptotal;
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   auto issue = [&](int t, int slot) {
@@ -1443,7 +1490,7 @@ __global__ void __launch_bounds__(NT) k_split_scan_2p(ScanArgs2 g) {
     unit_src(g.u, t, item, k, cnt, nd, f);
     const int a = nd.a, u0 = k * SUNIT;
     const int64_t nk = nd.n, Sk = nd.S;
-    const double nkd = (double)nk, Skd = (double)Sk;
+    const float nkf = (float)nk, Skf = (float)Sk;
     const int t0 = g.u.poff[item];
     const int32_t exn = (int32_t)(g.pren[t] - g.pren[t0]);
     const int64_t exS = g.preS[t] - g.preS[t0];
@@ -1451,18 +1498,22 @@ __global__ void __launch_bounds__(NT) k_split_scan_2p(ScanArgs2 g) {
     phase[cur] ^= 1u;
     const uint64_t* buf = bufs + (size_t)cur * (SUNIT + 4) + s_off[cur];
     const int jl = tid * SUV;
-    // w*y_q of my entries: every gather issued before any is consumed
-    int64_t wy[SUV];
+    // my entries (+ the next one) in registers; w*y_q gathers all in flight
+    const int cl_ = min(cnt, a - u0 - 1);  // last loaded index (the unit's entries + the next one if any)
+    uint64_t e[SUV + 1];
+#pragma unroll
+    for (int q = 0; q <= SUV; ++q) e[q] = buf[min(jl + q, cl_)];
     uint32_t rw[SUV];
 #pragma unroll
     for (int q = 0; q < SUV; ++q) rw[q] = e_row(buf[min(jl + q, cnt - 1)]);
+    int64_t wy[SUV];
 #pragma unroll
     for (int q = 0; q < SUV; ++q) wy[q] = ldg_s64_nc(g.yq + rw[q]);
     int32_t tc = 0;
     int64_t ts = 0;
 #pragma unroll
     for (int q = 0; q < SUV; ++q) {
-      const int32_t w = jl + q < cnt ? e_w(buf[jl + q]) : 0;
+      const int32_t w = jl + q < cnt ? e_w(e[q]) : 0;
       wy[q] *= w;
       tc += w;
       ts += wy[q];
@@ -1471,73 +1522,62 @@ __global__ void __launch_bounds__(NT) k_split_scan_2p(ScanArgs2 g) {
     int64_t tots;
     const int32_t prc0 = block_excl_scan(tc, smc, totc) + exn;
     const int64_t prs0 = block_excl_scan(ts, sms, tots) + exS;
-    // pass 1: cheap bounds of every candidate; M = the unit's best lower bound
-    double mL = -1.0;
+    // one pass: bounds of every candidate; keep the upper bounds, M = best lower bound of the unit
+    float gUq[SUV];
+    float mL = 0.0f;
     {
       int32_t prc = prc0;
       int64_t prs = prs0;
 #pragma unroll
       for (int q = 0; q < SUV; ++q) {
         const int j = jl + q;
-        if (j < cnt) {
-          const uint64_t e = buf[j];
-          prc += e_w(e);
-          prs += wy[q];
-          if (u0 + j + 1 < a && e_rank(e) != e_rank(buf[j + 1])) {
-            double gL, gU;
-            key_bounds(nkd, Skd, nk, prc, prs, gL, gU);
-            mL = fmax(mL, gL);
-          }
+        prc += jl + q < cnt ? e_w(e[q]) : 0;
+        prs += wy[q];
+        gUq[q] = -1.0f;
+        if (j < cnt && u0 + j + 1 < a && e_rank(e[q]) != e_rank(e[q + 1])) {
+          float gL;
+          key_bounds32(nkf, Skf, prc, (int32_t)(nk - prc), prs, gL, gUq[q]);
+          mL = fmaxf(mL, gL);
         }
       }
     }
     {
-      const uint64_t kb = gkey(mL);
-      const uint32_t hi = __reduce_max_sync(0xffffffffu, (uint32_t)(kb >> 32));
-      const uint32_t lo = __reduce_max_sync(0xffffffffu, ((uint32_t)(kb >> 32) == hi) ? (uint32_t)kb : 0u);
-      if (lane == 0) sg[wid] = (hi | lo) ? __longlong_as_double((long long)((((uint64_t)hi << 32) | lo) - 1ull)) : -1.0;
+      const float wm = __int_as_float((int)__reduce_max_sync(0xffffffffu, (unsigned)__float_as_int(mL)));
+      if (lane == 0) sf[wid] = wm;
       __syncthreads();
       if (tid == 0) {
-        double M = -1.0;
-        for (int q = 0; q < NT / 32; ++q) M = fmax(M, sg[q]);
+        float M = 0.0f;
+        for (int q = 0; q < NT / 32; ++q) M = fmaxf(M, sf[q]);
         s_M = M;
       }
       __syncthreads();
     }
-    const double M = s_M;
-    // pass 2: exact keys only where the upper bound reaches M
+    const float M = s_M;
+    // exact keys only where the upper bound reaches M (prefix recomputed for those few)
     double bg = -1.0;
     uint32_t brank = 0xffffffffu, brb = 0;
     int32_t bpos = -1, bnl = 0;
     int64_t bSl = 0;
-    {
+    uint32_t pass = 0;
+#pragma unroll
+    for (int q = 0; q < SUV; ++q) pass |= (gUq[q] >= M ? 1u : 0u) << q;
+    if (pass) {
       int32_t prc = prc0;
       int64_t prs = prs0;
 #pragma unroll
       for (int q = 0; q < SUV; ++q) {
-        const int j = jl + q;
-        if (j < cnt) {
-          const uint64_t e = buf[j];
-          prc += e_w(e);
-          prs += wy[q];
-          if (u0 + j + 1 < a) {
-            const uint64_t en = buf[j + 1];
-            const uint32_t ra = e_rank(e), rb = e_rank(en);
-            if (ra != rb) {
-              double gL, gU;
-              key_bounds(nkd, Skd, nk, prc, prs, gL, gU);
-              if (gU >= M && gU >= bg) {
-                const double gk = split_key(nk, Sk, prc, prs);
-                if (rec_better(gk, ra, bg, brank)) {
-                  bg = gk;
-                  brank = ra;
-                  brb = rb;
-                  bpos = u0 + j;
-                  bnl = prc;
-                  bSl = prs;
-                }
-              }
-            }
+        prc += jl + q < cnt ? e_w(e[q]) : 0;
+        prs += wy[q];
+        if (((pass >> q) & 1u) && gUq[q] >= scale_key(bg)) {
+          const double gk = split_key(nk, Sk, prc, prs);
+          const uint32_t ra = e_rank(e[q]);
+          if (rec_better(gk, ra, bg, brank)) {
+            bg = gk;
+            brank = ra;
+            brb = e_rank(e[q + 1]);
+            bpos = u0 + jl + q;
+            bnl = prc;
+            bSl = prs;
           }
         }
       }
@@ -1725,7 +1765,7 @@ struct TScanArgs {
   Rec* rec;
 };
 
-constexpr int TSV = 15;             // entries per thread (odd: conflict-free 64-bit shared loads)
+constexpr int TSV = 7;              // entries per thread (odd: conflict-free 64-bit shared loads)
 constexpr int TUNIT = NT * TSV;     // 3840 entries per unit
 
 // a7 split search: one CTA owns whole (node, drawn feature) items of one tree
@@ -1977,7 +2017,16 @@ __device__ __forceinline__ bool part_item_active(const Split* split, const Child
   return kl == KIND_LARGE || kl == KIND_SMALL || kr == KIND_LARGE || kr == KIND_SMALL;
 }
 
-// a9 partition: one CTA owns whole (node, feature) items of one tree; lefts first, stable
+// a9 partition: one CTA owns whole work items of one tree; lefts first, stable.
+// A work item is (node, group of G consecutive features) with G = max(1,
+// TPUNIT / a): the node's feature segments are contiguous, so a group is ONE
+// bulk copy, and the left (right) outputs of consecutive features are
+// contiguous in the child's block.  Items with a > TPUNIT are walked in units
+// with a running left count.
+struct PWork {
+  int node, f0, g, unit;  // node index, first feature, features in the unit, unit index inside the feature
+};
+
 __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
   extern __shared__ __align__(16) unsigned char dsm[];
   uint64_t* bufs = (uint64_t*)dsm;              // 2 x (TPUNIT + 2)
@@ -1985,6 +2034,8 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
   uint32_t* bm = (uint32_t*)(outb + TPUNIT);    // nw words (if staged)
   __shared__ uint64_t bar[2];
   __shared__ int32_t sm[TPNT / 32];
+  __shared__ int32_t tpre[TPNT];                // per-thread exclusive prefix of lefts in the unit
+  __shared__ uint32_t tmask[TPNT];              // per-thread left mask
   __shared__ int s_off[2];
   const int tid = threadIdx.x;
   const TreeSched ts = tree_sched(g.B);
@@ -1996,86 +2047,151 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
   uint32_t phase[2] = {0u, 0u};
   int cur = 0;
   for (int b = ts.b0; b < g.B; b += ts.bstep) {
-    const int i_lo = g.tlo[b] * g.p, i_hi = g.thi[b] * g.p;
-    if (i_lo >= i_hi) continue;
+    const int n_lo = g.tlo[b], n_hi = g.thi[b];
+    if (n_lo >= n_hi) continue;
     const uint32_t* sideg = g.sideb + (int64_t)b * g.nw;
     __syncthreads();
     if (g.bitmap_smem)
       for (int64_t w = tid; w < g.nw; w += TPNT) bm[w] = sideg[w];
     const uint32_t* sb = g.bitmap_smem ? bm : sideg;
-    auto next_item = [&](int it) {  // next active item of this CTA at or after it
-      while (it < i_hi && !part_item_active(g.split, g.child, it / g.p)) it += ts.C;
-      return it;
+    // work items of the tree in order: per active node, its feature groups (and units of long features);
+    // this CTA takes every C-th item starting at c.  Walk the sequence with a cursor.
+    int wnode = n_lo, wf = 0, widx = 0;  // cursor: next item in the tree's sequence
+    auto item_len = [&](int node, int& gsz, int& nun) {
+      const int a = g.nodes[node].a;
+      gsz = a >= TPUNIT ? 1 : min(g.p, TPUNIT / a);
+      nun = (a + TPUNIT - 1) / TPUNIT;
     };
-    auto issue = [&](int it, int un, int slot) {
-      const LNode nd = g.nodes[it / g.p];
-      const int f = it - (it / g.p) * g.p;
-      const int u0 = un * TPUNIT;
-      s_off[slot] = stage_entries(bufs + (size_t)slot * (TPUNIT + 2), g.Ecur + nd.base + (int64_t)f * nd.a + u0,
-                                  min(TPUNIT, nd.a - u0), &bar[slot]);
-    };
-    int item = next_item(i_lo + ts.c), unit = 0;
-    if (item >= i_hi) continue;
-    if (tid == 0) issue(item, 0, cur);
-    int64_t carry_l = 0;
-    while (item < i_hi) {
-      const int node = item / g.p, f = item - node * g.p;
-      const LNode nd = g.nodes[node];
-      const int nun = (nd.a + TPUNIT - 1) / TPUNIT;
-      int nitem = item, nunit = unit + 1;
-      if (nunit >= nun) {
-        nitem = next_item(item + ts.C);
-        nunit = 0;
+    // advance the cursor: items (node, feature group) are dealt round robin to the tree's CTAs; an owned
+    // item yields all its units in order (so the running left count stays inside one CTA)
+    int cur_nun = 0, cur_unit = 0;  // units left of the owned item being emitted
+    PWork cw;
+    auto next_mine = [&](PWork& w) -> bool {
+      if (cur_unit < cur_nun) {
+        w = cw;
+        w.unit = cur_unit++;
+        return true;
       }
+      for (;;) {
+        while (wnode < n_hi && !part_item_active(g.split, g.child, wnode)) {
+          ++wnode;
+          wf = 0;
+        }
+        if (wnode >= n_hi) return false;
+        int gsz, nun;
+        item_len(wnode, gsz, nun);
+        const bool mine = (widx % ts.C) == ts.c;
+        ++widx;
+        cw.node = wnode;
+        cw.f0 = wf;
+        cw.g = min(gsz, g.p - wf);
+        cw.unit = 0;
+        wf += cw.g;
+        if (wf >= g.p) {
+          ++wnode;
+          wf = 0;
+        }
+        if (mine) {
+          cur_nun = cw.g > 1 ? 1 : nun;
+          cur_unit = 1;
+          w = cw;
+          return true;
+        }
+      }
+    };
+    auto issue = [&](const PWork& w, int slot) {
+      const LNode nd = g.nodes[w.node];
+      const int u0 = w.unit * TPUNIT;
+      const int cnt = w.g > 1 ? w.g * nd.a : min(TPUNIT, nd.a - u0);
+      s_off[slot] = stage_entries(bufs + (size_t)slot * (TPUNIT + 2),
+                                  g.Ecur + nd.base + (int64_t)w.f0 * nd.a + (w.g > 1 ? 0 : u0), cnt, &bar[slot]);
+    };
+    PWork w, wn;
+    bool have = next_mine(w);
+    if (!have) continue;
+    if (tid == 0) issue(w, cur);
+    int64_t carry_l = 0;
+    while (have) {
+      const bool havn = next_mine(wn);
       __syncthreads();
-      if (tid == 0 && nitem < i_hi) issue(nitem, nunit, cur ^ 1);
-      const int u0 = unit * TPUNIT, cnt = min(TPUNIT, nd.a - u0);
-      const Child cl = g.child[2 * node], cr = g.child[2 * node + 1];
+      if (tid == 0 && havn) issue(wn, cur ^ 1);
+      const LNode nd = g.nodes[w.node];
+      const int a = nd.a;
+      const int u0 = w.unit * TPUNIT;
+      const int cnt = w.g > 1 ? w.g * a : min(TPUNIT, a - u0);
+      const Child cl = g.child[2 * w.node], cr = g.child[2 * w.node + 1];
       mbar_wait(&bar[cur], phase[cur]);
       phase[cur] ^= 1u;
       const uint64_t* buf = bufs + (size_t)cur * (TPUNIT + 2) + s_off[cur];
       const int jl = tid * TPV;
+      uint64_t ev[TPV];
+      uint32_t bw[TPV];
+#pragma unroll
+      for (int q = 0; q < TPV; ++q) ev[q] = buf[min(jl + q, cnt - 1)];
+      if (g.bitmap_smem) {
+#pragma unroll
+        for (int q = 0; q < TPV; ++q) bw[q] = sb[e_row(ev[q]) >> 5];
+      } else {  // L2-resident bitmap: all gathers in flight together
+#pragma unroll
+        for (int q = 0; q < TPV; ++q) bw[q] = ldg_u32_nc(sb + (e_row(ev[q]) >> 5));
+      }
       uint32_t lmask = 0;
       int32_t c = 0;
 #pragma unroll
-      for (int q = 0; q < TPV; ++q) {
-        const int j = jl + q;
-        if (j < cnt) {
-          const uint32_t r = e_row(buf[j]);
-          if (!((sb[r >> 5] >> (r & 31)) & 1u)) {
-            lmask |= 1u << q;
-            ++c;
+      for (int q = 0; q < TPV; ++q)
+        if (jl + q < cnt && !((bw[q] >> (e_row(ev[q]) & 31)) & 1u)) {
+          lmask |= 1u << q;
+          ++c;
+        }
+      int32_t tot;
+      const int32_t lbl = block_excl_scan(c, sm, tot);
+      const int al = cl.a, ar = cr.a;  // lefts / rights per feature segment
+      if (w.g > 1) {
+        tpre[tid] = lbl;
+        tmask[tid] = lmask;
+        __syncthreads();
+        int pl = lbl;
+#pragma unroll
+        for (int q = 0; q < TPV; ++q) {
+          const int j = jl + q;
+          if (j < cnt) {
+            const int sgm = j / a, s0 = sgm * a;
+            const int t0 = s0 / TPV, o0 = s0 - t0 * TPV;
+            const int ps = tpre[t0] + __popc(tmask[t0] & ((1u << o0) - 1u));  // lefts before the segment start
+            const int lb = pl - ps;                                            // lefts before j in the segment
+            if ((lmask >> q) & 1u) outb[sgm * al + lb] = ev[q];
+            else outb[w.g * al + sgm * ar + (j - s0 - lb)] = ev[q];
+            pl += (lmask >> q) & 1u;
+          }
+        }
+      } else {
+        int li = lbl, ri = tot + (jl - lbl);
+#pragma unroll
+        for (int q = 0; q < TPV; ++q) {
+          const int j = jl + q;
+          if (j < cnt) {
+            if ((lmask >> q) & 1u) outb[li++] = ev[q];
+            else outb[ri++] = ev[q];
           }
         }
       }
-      int32_t tot;
-      const int32_t lbl = block_excl_scan(c, sm, tot);
-      int li = lbl, ri = tot + (jl - lbl);
-#pragma unroll
-      for (int q = 0; q < TPV; ++q) {
-        const int j = jl + q;
-        if (j < cnt) {
-          const uint64_t e = buf[j];
-          if ((lmask >> q) & 1u) outb[li++] = e;
-          else outb[ri++] = e;
-        }
-      }
       __syncthreads();
-      const int64_t exl = carry_l, exr = (int64_t)u0 - carry_l;
       const bool keepL = cl.kind == KIND_LARGE || cl.kind == KIND_SMALL;
       const bool keepR = cr.kind == KIND_LARGE || cr.kind == KIND_SMALL;
+      const int64_t exl = w.g > 1 ? 0 : carry_l, exr = w.g > 1 ? 0 : (int64_t)u0 - carry_l;
+      const int nl_out = w.g > 1 ? w.g * al : tot, nr_out = cnt - nl_out;
       if (keepL) {
-        uint64_t* dl = (cl.kind == KIND_LARGE ? g.Enext : g.Esmall) + cl.base + (int64_t)f * cl.a + exl;
-        for (int i = tid; i < tot; i += TPNT) dl[i] = outb[i];
+        uint64_t* dl = (cl.kind == KIND_LARGE ? g.Enext : g.Esmall) + cl.base + (int64_t)w.f0 * al + exl;
+        for (int i = tid; i < nl_out; i += TPNT) dl[i] = outb[i];
       }
       if (keepR) {
-        uint64_t* dr = (cr.kind == KIND_LARGE ? g.Enext : g.Esmall) + cr.base + (int64_t)f * cr.a + exr;
-        for (int i = tid; i < cnt - tot; i += TPNT) dr[i] = outb[tot + i];
+        uint64_t* dr = (cr.kind == KIND_LARGE ? g.Enext : g.Esmall) + cr.base + (int64_t)w.f0 * ar + exr;
+        for (int i = tid; i < nr_out; i += TPNT) dr[i] = outb[nl_out + i];
       }
       carry_l += tot;
-      if (nunit == 0) carry_l = 0;
-      item = nitem;
-      unit = nunit;
+      if (!havn || wn.node != w.node || wn.f0 != w.f0) carry_l = 0;
+      w = wn;
+      have = havn;
       cur ^= 1;
     }
   }
@@ -3259,7 +3375,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
     const size_t tscan_smem = sizeof(uint64_t) * 2 * (TUNIT + 4);
     const size_t tpart_base = sizeof(uint64_t) * (3 * TPUNIT + 4);
     const int smem_optin = dyn_smem_limit(k_partition_tree);
-    const bool bm_smem = tpart_base + (size_t)nw * 4 <= (size_t)smem_optin;
+    const bool bm_smem = getenv("BF_PART_L2") == nullptr && tpart_base + (size_t)nw * 4 <= (size_t)smem_optin;
     const size_t tpart_smem = tpart_base + (bm_smem ? (size_t)nw * 4 : 0);
     BF_CUDA_CHECK(cudaFuncSetAttribute(k_split_scan_tree, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tscan_smem));
     int occ_ts = 0, occ_tp = 0;
@@ -3369,18 +3485,53 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
           KScope ks_("k_mtry", s, 0.0);
           k_mtry<<<(unsigned)ceil_div(N, 128), 128, 0, s>>>(nc, N, p, mtry, prm.seed, tb, feat.p, fyscr.p);
         }
-        // ---- a7 split search: tree-affine CTAs own whole items
+        static const bool lvl_timing = getenv("BF_LEVEL_TIMING") != nullptr;
+        cudaEvent_t lev[4];
+        if (lvl_timing) {
+          for (auto& e : lev) cudaEventCreate(&e);
+          cudaEventRecord(lev[0], s);
+        }
+        static const bool scan_tree = getenv("BF_SCAN_2P") == nullptr;
         BF_CUDA_CHECK(cudaMemsetAsync(tlo.p, 0, sizeof(int32_t) * Bc, s));
         BF_CUDA_CHECK(cudaMemsetAsync(thi.p, 0, sizeof(int32_t) * Bc, s));
         {
           KScope ks_("k_tree_ranges", s, 0.0);
           k_tree_ranges<<<(unsigned)ceil_div(N, 256), 256, 0, s>>>(N, nc, tlo.p, thi.p);
         }
-        {
+        if (scan_tree) {
           TScanArgs ga{nc, feat.p, mtry, Bc, Ec, yq.p, tlo.p, thi.p, rec.p};
           KScope ks_("k_split_scan", s, 0.0);
           k_split_scan_tree<<<grid_tscan, NT, tscan_smem, s>>>(ga);
+        } else {
+        // ---- a7 split search over units (two passes: unit sums, then units in parallel)
+          const int NI = N * mtry;
+          unit_setup(0, NI, mtry, SUNIT, nc, split.p, child.p, pcnt.p, poff.p, pmap.p, ptot.p, s);
+          {
+            UnitArgs ua{nc, feat.p, mtry, SUNIT, Ec, poff.p, pmap.p, ptot.p};
+            {
+              KScope ks_("k_unit_sums", s, 0.0);
+              k_unit_sums<<<grid_sums, NT, 0, s>>>(ua, yq.p, un.p, uS.p);
+            }
+            const int64_t bound_s = (int64_t)mtry * (cur_a / SUNIT + N) + 1;
+            {
+              KScope ks_("cub_ExclusiveSum", s, 0.0);
+              size_t tb2 = unit_tb;
+              BF_CUDA_CHECK(cub::DeviceScan::ExclusiveSum(unit_tmp.p, tb2, un.p, pren.p, (int)bound_s, s));
+              tb2 = unit_tb;
+              BF_CUDA_CHECK(cub::DeviceScan::ExclusiveSum(unit_tmp.p, tb2, uS.p, preS.p, (int)bound_s, s));
+            }
+            ScanArgs2 ga{ua, yq.p, pren.p, preS.p, prec.p};
+            {
+              KScope ks_("k_split_scan", s, 0.0);
+              k_split_scan_2p<<<grid_scan, NT, scan_smem, s>>>(ga);
+            }
+          }
+          {
+            KScope ks_("k_item_reduce", s, 0.0);
+            k_item_reduce<<<(unsigned)ceil_div((int64_t)NI * 32, 256), 256, 0, s>>>(NI, pcnt.p, poff.p, prec.p, rec.p);
+          }
         }
+        if (lvl_timing) cudaEventRecord(lev[1], s);
         {
           KScope ks_("k_finalize", s, 0.0);
           k_finalize<<<(unsigned)ceil_div(N, 128), 128, 0, s>>>(nc, N, feat.p, rec.p, mtry, uniq.p, n, prm.nodesize, A,
@@ -3415,12 +3566,14 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
           KScope ks_("k_child_values", s, 0.0);
           k_child_values<<<(unsigned)ceil_div(N, 128), 128, 0, s>>>(N, split.p, csum.p, nc, pool);
         }
+        if (lvl_timing) cudaEventRecord(lev[2], s);
         // ---- a9 partition: tree-affine CTAs own whole items; goes-right bitmap in shared memory
         {
           TPartArgs ga{nc, split.p, child.p, p, Bc, Ec, sideb.p, nw, bm_smem ? 1 : 0, En, Es.p, tlo.p, thi.p};
           KScope ks_("k_partition", s, 0.0);
           k_partition_tree<<<grid_tpart, TPNT, tpart_smem, s>>>(ga);
         }
+        if (lvl_timing) cudaEventRecord(lev[3], s);
         {
           KScope ks_("k_commit", s, 0.0);
           k_commit<<<1, 1, 0, s>>>(N2, packL.p, scanL.p, packS.p, scanS.p, p, dsum.p, hs.h);
@@ -3432,6 +3585,16 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
           prof_add_bytes("k_split_scan", (double)cur_a * mtry * 16.0);
           prof_add_bytes("k_dest", sa * 17.0);
           prof_add_bytes("k_partition", sa * p * 17.0);
+        }
+        if (lvl_timing) {
+          float ms1 = 0, ms2 = 0, ms3 = 0;
+          cudaEventElapsedTime(&ms1, lev[0], lev[1]);
+          cudaEventElapsedTime(&ms2, lev[1], lev[2]);
+          cudaEventElapsedTime(&ms3, lev[2], lev[3]);
+          fprintf(stderr, "[level] N=%d entries/feature=%lld split_a=%llu scan=%.3f mid=%.3f part=%.3f ms  scanGB/s=%.0f partGB/s=%.0f\n", N,
+                  (long long)cur_a, (unsigned long long)hs.h->split_a, ms1, ms2, ms3,
+                  (double)cur_a * mtry * 16.0 / (ms1 * 1e6), (double)hs.h->split_a * p * 17.0 / (ms3 * 1e6));
+          for (auto& e : lev) cudaEventDestroy(e);
         }
         cur_elems = hs.h->next_elems;
         N = hs.h->nnext;
