@@ -12,7 +12,8 @@
 namespace bf {
 namespace {
 
-constexpr int PT = 128;  // rows per CTA
+constexpr int PT = 128;   // rows per CTA
+constexpr int PILP = 8;  // trees walked concurrently by one thread
 
 __device__ __forceinline__ Node16 load_node(const Node16* p) {
   const int4 v = __ldg(reinterpret_cast<const int4*>(p));
@@ -23,35 +24,68 @@ __device__ __forceinline__ Node16 load_node(const Node16* p) {
   return n;
 }
 
+// Trees [t_begin, t_end) of one tree block for every row; partial sums are
+// accumulated into yhat_sum (first block writes), so leaves are still added in
+// tree order.  A block of a few trees stays L2-resident while all rows walk it.
 __global__ void __launch_bounds__(PT) k_predict_smem(const Node16* __restrict__ nodes, const int64_t* __restrict__ off,
-                                                     int32_t ntrees, const double* __restrict__ Xq, int64_t ldq,
+                                                     int32_t t_begin, int32_t t_end, int first, int last,
+                                                     const double* __restrict__ Xq, int64_t ldq,
                                                      int64_t m, int p, double* yhat_sum, double* yhat, double inv_t,
                                                      unsigned long long* visits) {
   extern __shared__ double sx[];  // PT x p, row-major, padded stride p|1
   const int stride = p | 1;
   const int64_t r0 = (int64_t)blockIdx.x * PT;
   const int rows = (int)(m - r0 < PT ? m - r0 : PT);
-  for (int f = 0; f < p; ++f)
-    for (int r = threadIdx.x; r < rows; r += PT) sx[r * stride + f] = Xq[(int64_t)f * ldq + r0 + r];
+  {  // stage the tile: every thread's column loads in flight together (16 at a time)
+    const int r = threadIdx.x;
+    const bool ok = r < rows;
+    const double* src = Xq + r0 + (ok ? r : 0);
+    for (int f0 = 0; f0 < p; f0 += 16) {
+      double v[16];
+#pragma unroll
+      for (int u = 0; u < 16; ++u) v[u] = (f0 + u < p) ? __ldcs(src + (int64_t)(f0 + u) * ldq) : 0.0;
+#pragma unroll
+      for (int u = 0; u < 16; ++u)
+        if (f0 + u < p && ok) sx[r * stride + f0 + u] = v[u];
+    }
+  }
   __syncthreads();
   if ((int)threadIdx.x >= rows) return;
   const double* x = sx + threadIdx.x * stride;
-  double acc = 0.0;
+  const int64_t rr = r0 + threadIdx.x;
+  double acc = first ? 0.0 : yhat_sum[rr];
   unsigned long long nv = 0;
-  for (int32_t t = 0; t < ntrees; ++t) {
-    const Node16* tn = nodes + off[t];
-    Node16 nd = load_node(tn);
-    ++nv;
-    while (nd.feature >= 0) {
-      nd = load_node(tn + (x[nd.feature] <= nd.v ? nd.left : nd.left + 1));
-      ++nv;
+  // ILP trees walked together (independent dependency chains; the last group
+  // of a block is masked); leaf values are added in tree order, as in S5
+  for (int32_t t = t_begin; t < t_end; t += PILP) {
+    const int na = t_end - t < PILP ? t_end - t : PILP;
+    const Node16* tn[PILP];
+    Node16 nd[PILP];
+#pragma unroll
+    for (int u = 0; u < PILP; ++u) {
+      tn[u] = nodes + off[t + (u < na ? u : 0)];
+      nd[u] = load_node(tn[u]);
+      if (u >= na) nd[u].feature = -1;
     }
-    acc += nd.v;
+    nv += na;
+    bool any = true;
+    while (any) {
+      any = false;
+#pragma unroll
+      for (int u = 0; u < PILP; ++u)
+        if (nd[u].feature >= 0) {
+          nd[u] = load_node(tn[u] + (x[nd[u].feature] <= nd[u].v ? nd[u].left : nd[u].left + 1));
+          ++nv;
+          any = true;
+        }
+    }
+#pragma unroll
+    for (int u = 0; u < PILP; ++u)
+      if (u < na) acc += nd[u].v;
   }
   if (visits) atomicAdd(visits, nv);
-  const int64_t r = r0 + threadIdx.x;
-  if (yhat_sum) yhat_sum[r] = acc;
-  if (yhat) yhat[r] = acc * inv_t;
+  yhat_sum[rr] = acc;
+  if (last && yhat) yhat[rr] = acc * inv_t;
 }
 
 __global__ void __launch_bounds__(PT) k_predict_gmem(const Node16* __restrict__ nodes, const int64_t* __restrict__ off,
@@ -97,16 +131,34 @@ void predict_impl(const bf_forest* f, const double* Xq_in, int64_t ldq, int64_t 
     BF_CUDA_CHECK(cudaMemsetAsync(vis.p, 0, 8, s));
   }
   if (smem <= (size_t)smax) {
-    {
-      KScope ks_("k_predict_smem", s, 0.0);
-      k_predict_smem<<<grid, PT, smem, s>>>(f->d_nodes, f->d_tree_off, nt, (const double*)Xs.dptr, ldq, m, p,
-                                           ys_in ? (double*)ys.dptr : nullptr, yh_in ? (double*)yh.dptr : nullptr, inv_t, vis.p);
+    // tree blocks of <= 64 MB of nodes (L2-resident while every row walks them)
+    double* ysum = ys_in ? (double*)ys.dptr : nullptr;
+    DBuf<double> ytmp;
+    if (!ysum) {
+      ytmp.alloc(m, s);
+      ysum = ytmp.p;
+    }
+    const int64_t block_bytes = 64ll << 20;
+    int32_t t0 = 0;
+    while (t0 < nt || (nt == 0 && t0 == 0)) {
+      int32_t t1 = t0 + 1;
+      while (t1 < nt && (f->tree_off[t1 + 1] - f->tree_off[t0]) * (int64_t)sizeof(Node16) <= block_bytes) ++t1;
+      if (t1 < nt && t1 - t0 > PILP) t1 = t0 + (t1 - t0) / PILP * PILP;  // whole ILP groups
+      if (nt == 0) t1 = 0;
+      {
+        KScope ks_("k_predict_smem", s, 0.0);
+        k_predict_smem<<<grid, PT, smem, s>>>(f->d_nodes, f->d_tree_off, t0, t1, t0 == 0, t1 >= nt,
+                                             (const double*)Xs.dptr, ldq, m, p, ysum,
+                                             yh_in ? (double*)yh.dptr : nullptr, inv_t, vis.p);
+      }
+      if (nt == 0) break;
+      t0 = t1;
     }
   } else {
     {
       KScope ks_("k_predict_gmem", s, 0.0);
       k_predict_gmem<<<grid, PT, 0, s>>>(f->d_nodes, f->d_tree_off, nt, (const double*)Xs.dptr, ldq, m,
-                                         ys_in ? (double*)ys.dptr : nullptr, yh_in ? (double*)yh.dptr : nullptr, inv_t, vis.p);
+                                       ys_in ? (double*)ys.dptr : nullptr, yh_in ? (double*)yh.dptr : nullptr, inv_t, vis.p);
     }
   }
   BF_CUDA_CHECK(cudaGetLastError());
