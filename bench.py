@@ -58,6 +58,20 @@ def peaks():
         return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md)"
 
 
+def ncu_traffic(kernel: str):
+    """DRAM bytes (read + write) per launch of `kernel` from the newest committed
+    `ncu --set full` summary under profiles/ (tools/ncu_summary.py), or None."""
+    import glob
+    for d in sorted(glob.glob(os.path.join(ROOT, "profiles", "r[0-9]*")), reverse=True):
+        f = os.path.join(d, f"full_{kernel}.json")
+        if os.path.exists(f):
+            try:
+                return float(json.load(open(f))["dram_bytes"]), os.path.relpath(f, ROOT)
+            except Exception:
+                pass
+    return None, None
+
+
 class Clocks:
     """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
 
@@ -171,12 +185,12 @@ def run_ours(args):
     import torch.distributed as dist
 
     import paper_conf_ipps_madougouvln16_b200 as bf
+    from paper_conf_ipps_madougouvln16_b200 import distributed as D
 
     rank, world, local = dist_setup(args)
     dev = torch.device("cuda", local)
     S, cfg, T, m = workload(args)
-    t0 = ((rank * T) // world)
-    t1 = (((rank + 1) * T) // world)
+    t0, t1 = D.tree_range(rank, world, T)
     X, y, _ = S.dataset(args.config)
     p, n = X.shape
     Xh = torch.from_numpy(X).pin_memory()
@@ -209,21 +223,16 @@ def run_ours(args):
             ps, _ = forest.predict(Qs, ntree_total=T)
             if host:
                 ps = torch.from_numpy(ps).to(dev)
-            if world > 1:
-                dist.all_reduce(ps)
-            pred = ps[:1] / T
+            pred = D.allreduce_predictions(ps, T) if world > 1 else ps / T
         e[2].record(stream)
         acc = forest.oob_importance(Xs, ys_)
         if host:
             acc = {k: torch.from_numpy(v).to(dev) for k, v in acc.items()}
-        dsl = torch.zeros((T, p), dtype=torch.float64, device=dev)
-        npu = torch.zeros((T, p), dtype=torch.float64, device=dev)
-        dsl[t0:t1] = acc["d_slots"]
-        npu[t0:t1] = acc["npur_slots"]
-        osum, ocnt = acc["oob_sum"], acc["oob_cnt"]
-        if world > 1:
-            for tns in (dsl, npu, osum, ocnt):
-                dist.all_reduce(tns)
+        if world > 1:  # disjoint per-tree slots: the all-reduce is an exact all-gather
+            m = D.merge_importance(acc, t0, t1, T)
+            dsl, npu, osum, ocnt = m["d_slots"], m["npur_slots"], m["oob_sum"], m["oob_cnt"]
+        else:
+            dsl, npu, osum, ocnt = acc["d_slots"], acc["npur_slots"], acc["oob_sum"], acc["oob_cnt"]
         fin = bf.importance_finalize(dsl, npu, osum, ocnt, yd)
         e[3].record(stream)
         pc = bf.pca(Xs, scale=True, k=k_pca)
@@ -301,8 +310,10 @@ def run_ours(args):
     if dom:
         d = kern[dom]
         achieved = d["bytes"] / (d["ms"] / 1e3) / 1e9 if d["bytes"] > 0 else 0.0
+        traffic, tsrc = ncu_traffic(dom)
         roof = {"kernel": dom, "bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
-                "frac": achieved / hbm, "traffic": None, "peak_source": hbm_src,
+                "frac": achieved / hbm, "traffic": traffic, "traffic_source": tsrc, "peak_source": hbm_src,
+                "algorithmic_bytes_per_launch": d["bytes"] / max(d["launches"], 1),
                 "share_of_step": d["ms"] / args.steps / ms,
                 "avg_launch_ms": d["ms"] / max(d["launches"], 1)}
     kernels = {k: {"ms_per_step": v["ms"] / args.steps, "launches_per_step": v["launches"] / args.steps,

@@ -432,118 +432,6 @@ __device__ __forceinline__ int warp_argmax_key(uint64_t key, uint32_t tie) {
 __device__ __forceinline__ uint64_t gkey(double g) { return g >= 0.0 ? (uint64_t)__double_as_longlong(g) + 1ull : 0ull; }
 
 
-__global__ void __launch_bounds__(NT) k_split_scan(const LNode* nodes, const int32_t* feat, int mtry,
-                                                   const uint64_t* E, const int64_t* yq, Rec* rec) {
-  __shared__ int32_t smc[NT / 32];
-  __shared__ int64_t sms[NT / 32];
-  __shared__ double sg[NT / 32];
-  __shared__ uint32_t sr[NT / 32];
-  __shared__ int32_t sw[NT / 32];
-  const int64_t item = blockIdx.x;
-  const LNode nd = nodes[item / mtry];
-  const int f = feat[item];
-  const uint64_t* seg = E + nd.base + (int64_t)f * nd.a;
-  const int a = nd.a;
-  const int64_t nk = nd.n, Sk = nd.S;
-  int32_t carry_c = 0;
-  int64_t carry_s = 0;
-  double bg = -1.0;
-  uint32_t brank = 0xffffffffu, brb = 0;
-  int32_t bpos = -1, bnl = 0;
-  int64_t bSl = 0;
-  for (int c0 = 0; c0 < a; c0 += SCH) {
-    const int j0 = c0 + threadIdx.x * SV;
-    uint64_t e[SV + 1];
-    int32_t wc[SV];
-    int64_t ws[SV];
-    int32_t tc = 0;
-    int64_t ts = 0;
-#pragma unroll
-    for (int u = 0; u <= SV; ++u) e[u] = (j0 + u < a) ? seg[j0 + u] : 0ull;
-#pragma unroll
-    for (int u = 0; u < SV; ++u) {
-      wc[u] = 0;
-      ws[u] = 0;
-      if (j0 + u < a) {
-        wc[u] = e_w(e[u]);
-        ws[u] = (int64_t)wc[u] * __ldg(yq + e_row(e[u]));
-      }
-      tc += wc[u];
-      ts += ws[u];
-    }
-    int32_t totc;
-    int64_t tots;
-    int32_t prec = block_excl_scan(tc, smc, totc) + carry_c;
-    int64_t pres = block_excl_scan(ts, sms, tots) + carry_s;
-#pragma unroll
-    for (int u = 0; u < SV; ++u) {
-      prec += wc[u];
-      pres += ws[u];
-      const int j = j0 + u;
-      if (j + 1 < a) {
-        const uint32_t ra = e_rank(e[u]), rb = e_rank(e[u + 1]);
-        if (ra != rb && screen_may_win(nk, Sk, prec, pres, bg)) {
-          const double g = split_key(nk, Sk, prec, pres);
-          if (rec_better(g, ra, bg, brank)) {
-            bg = g;
-            brank = ra;
-            brb = rb;
-            bpos = j;
-            bnl = prec;
-            bSl = pres;
-          }
-        }
-      }
-    }
-    carry_c += totc;
-    carry_s += tots;
-  }
-  // block argmax (g desc, rank asc)
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  int src = lane;
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) {
-    const double og = __shfl_down_sync(0xffffffffu, bg, o);
-    const uint32_t orr = __shfl_down_sync(0xffffffffu, brank, o);
-    const int os = __shfl_down_sync(0xffffffffu, src, o);
-    if (lane + o < 32 && rec_better(og, orr, bg, brank)) {
-      bg = og;
-      brank = orr;
-      src = os;
-    }
-  }
-  src = __shfl_sync(0xffffffffu, src, 0);
-  if (lane == 0) {
-    sg[wid] = bg;
-    sr[wid] = brank;
-    sw[wid] = wid * 32 + src;
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    double g = sg[0];
-    uint32_t r = sr[0];
-    int who = sw[0];
-    for (int k = 1; k < NT / 32; ++k)
-      if (rec_better(sg[k], sr[k], g, r)) {
-        g = sg[k];
-        r = sr[k];
-        who = sw[k];
-      }
-    sw[0] = who;
-  }
-  __syncthreads();
-  if (threadIdx.x == sw[0]) {
-    Rec R;
-    R.g = bg;
-    R.rank_a = brank;
-    R.rank_b = brb;
-    R.pos = bpos;
-    R.nl = bnl;
-    R.Sl = bSl;
-    rec[item] = R;
-  }
-}
-
 // ------------------------------------------------------------------ a8 node finalize (global phase)
 __global__ void k_finalize(const LNode* nodes, int N, const int32_t* feat, const Rec* rec, int mtry,
                            const double* uniq, int64_t n, int nodesize, int Asmall, int q, uint64_t seed,
@@ -665,119 +553,11 @@ __global__ void k_commit(int N2, const uint64_t* packL, const uint64_t* scanL, c
   *sum = s;
 }
 
-// ------------------------------------------------------------------ a9/a10 goes-right flags + child values
-__global__ void __launch_bounds__(NT) k_dest(const LNode* nodes, const Split* split, const uint64_t* E,
-                                             const double* y, int64_t n, uint8_t* side,
-                                             Pool pool) {
-  __shared__ double sl[NT], sr[NT];
-  const int k = blockIdx.x;
-  const Split sp = split[k];
-  if (!sp.split) return;
-  const LNode nd = nodes[k];
-  const uint64_t* seg = E + nd.base + (int64_t)sp.f * nd.a;
-  uint8_t* sd = side + (int64_t)nd.b * n;
-  double accl = 0.0, accr = 0.0;
-  for (int j = threadIdx.x; j < nd.a; j += NT) {
-    const uint64_t ej = seg[j];
-    const uint32_t row = e_row(ej);
-    const int s = j > sp.pos;
-    sd[row] = (uint8_t)s;
-    const double v = __dmul_rn((double)e_w(ej), y[row]);
-    if (s) accr += v;
-    else accl += v;
-  }
-  sl[threadIdx.x] = accl;
-  sr[threadIdx.x] = accr;
-  __syncthreads();
-  for (int s = NT / 2; s > 0; s >>= 1) {
-    if (threadIdx.x < s) {
-      sl[threadIdx.x] += sl[threadIdx.x + s];
-      sr[threadIdx.x] += sr[threadIdx.x + s];
-    }
-    __syncthreads();
-  }
-  if (threadIdx.x == 0) {
-    const int64_t r = (int64_t)nd.b * pool.cap;
-    pool.value[r + sp.lraw] = __ddiv_rn(sl[0], (double)sp.nl);
-    pool.value[r + sp.lraw + 1] = __ddiv_rn(sr[0], (double)sp.nr);
-  }
-}
-
-// ------------------------------------------------------------------ a9 partition
-constexpr int PV = 8;
-constexpr int PCH = NT * PV;
-
-__global__ void __launch_bounds__(NT) k_partition(const LNode* nodes, const Split* split, const Child* child,
-                                                  int p, const uint64_t* Ecur, const uint8_t* side, int64_t n,
-                                                  uint64_t* Enext, uint64_t* Esmall) {
-  __shared__ int32_t sm[NT / 32];
-  const int k = blockIdx.x;
-  const int f = blockIdx.y;
-  const Split sp = split[k];
-  if (!sp.split) return;
-  const Child cl = child[2 * k], cr = child[2 * k + 1];
-  const bool keepL = cl.kind == KIND_LARGE || cl.kind == KIND_SMALL;
-  const bool keepR = cr.kind == KIND_LARGE || cr.kind == KIND_SMALL;
-  if (!keepL && !keepR) return;
-  const LNode nd = nodes[k];
-  const uint64_t* seg = Ecur + nd.base + (int64_t)f * nd.a;
-  const uint8_t* sd = side + (int64_t)nd.b * n;
-  uint64_t* dl = keepL ? (cl.kind == KIND_LARGE ? Enext : Esmall) + cl.base + (int64_t)f * cl.a : nullptr;
-  uint64_t* dr = keepR ? (cr.kind == KIND_LARGE ? Enext : Esmall) + cr.base + (int64_t)f * cr.a : nullptr;
-  int32_t carry = 0;
-  for (int c0 = 0; c0 < nd.a; c0 += PCH) {
-    const int j0 = c0 + threadIdx.x * PV;
-    uint64_t e[PV];
-    bool left[PV];
-    int32_t cnt = 0;
-#pragma unroll
-    for (int u = 0; u < PV; ++u) {
-      left[u] = false;
-      if (j0 + u < nd.a) {
-        e[u] = seg[j0 + u];
-        left[u] = sd[e_row(e[u])] == 0;
-      }
-      cnt += left[u];
-    }
-    int32_t tot;
-    int32_t lb = block_excl_scan(cnt, sm, tot) + carry;
-#pragma unroll
-    for (int u = 0; u < PV; ++u) {
-      const int j = j0 + u;
-      if (j < nd.a) {
-        if (left[u]) {
-          if (keepL) dl[lb] = e[u];
-          ++lb;
-        } else if (keepR) {
-          dr[j - lb] = e[u];
-        }
-      }
-    }
-    carry += tot;
-  }
-}
-
-// ------------------------------------------------------------------ pieces + decoupled look-back (global phase)
-// Every (node, feature) segment of a level is cut into pieces of PIECE
-// entries.  Persistent CTAs take pieces in ticket order; a piece publishes its
-// aggregate as soon as it has it, then a warp looks back over the preceding
-// pieces of the same segment (summing aggregates until it meets a published
-// inclusive prefix) -- so segments of any length stream at full parallelism
-// in one pass (Merrill & Garland's single-pass scan).
+// ------------------------------------------------------------------ pieces (goes-right flags)
+// Every winning segment of a level is cut into pieces of PIECE entries; one
+// CTA per piece (k_dest_bits).
 constexpr int PIECE_V = 8;
 constexpr int PIECE = NT * PIECE_V;  // 2048 entries
-
-struct PieceRec {  // best candidate of one piece of a scan item
-  double g;
-  uint32_t rank_a, rank_b;
-  int32_t pos, nl;
-  int64_t Sl;
-};
-struct LbNS {
-  int64_t S;
-  int32_t n;
-  int32_t pad;
-};
 
 // items: mode 0 scan (node = i / mtry), 1 dest (node = i, split only), 2 partition (node = i / p, split with a kept child)
 __global__ void k_piece_count(int mode, int nitems, int div, const LNode* nodes, const Split* split, const Child* child,
@@ -802,282 +582,6 @@ __global__ void k_piece_map(int nitems, const int32_t* cnt, const int32_t* off, 
   if (i == nitems - 1) *total = o + c;
 }
 
-__device__ __forceinline__ uint32_t ld_flag(const uint32_t* p) { return *(const volatile uint32_t*)p; }
-
-// Warp look-back over pieces [t0, t): exclusive (n, S) of piece t.  All lanes return the result.
-__device__ void lookback_ns(int t, int t0, const LbNS* agg, const LbNS* incl, const uint32_t* flag, int32_t& exn,
-                            int64_t& exS) {
-  const int lane = threadIdx.x & 31;
-  int j = t - 1;
-  int32_t an = 0;
-  int64_t aS = 0;
-  for (;;) {
-    const int idx = j - lane;
-    uint32_t f = 2;
-    int32_t vn = 0;
-    int64_t vS = 0;
-    if (idx >= t0) {
-      while ((f = ld_flag(flag + idx)) == 0) __nanosleep(20);
-      __threadfence();
-      const LbNS* src = (f == 2) ? incl + idx : agg + idx;
-      vS = __ldcg((const long long*)&src->S);
-      vn = __ldcg((const int*)&src->n);
-    }
-    const unsigned pm = __ballot_sync(0xffffffffu, f == 2);
-    const int L = pm ? __ffs(pm) - 1 : 31;
-    if (lane > L) {
-      vn = 0;
-      vS = 0;
-    }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-      vn += __shfl_xor_sync(0xffffffffu, vn, o);
-      vS += __shfl_xor_sync(0xffffffffu, vS, o);
-    }
-    an += vn;
-    aS += vS;
-    if (pm) break;
-    j -= 32;
-  }
-  exn = an;
-  exS = aS;
-}
-
-// Warp look-back for 62-bit counters packed with a 2-bit status: (status << 62) | value.
-__device__ int64_t lookback_cnt(int t, int t0, const unsigned long long* st) {
-  const int lane = threadIdx.x & 31;
-  int j = t - 1;
-  int64_t acc = 0;
-  for (;;) {
-    const int idx = j - lane;
-    unsigned long long w = (2ull << 62);
-    if (idx >= t0)
-      while (((w = *(const volatile unsigned long long*)(st + idx)) >> 62) == 0) __nanosleep(20);
-    const uint32_t f = (uint32_t)(w >> 62);
-    int64_t v = (int64_t)(w & ((1ull << 62) - 1));
-    const unsigned pm = __ballot_sync(0xffffffffu, f == 2);
-    const int L = pm ? __ffs(pm) - 1 : 31;
-    if (lane > L) v = 0;
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-    acc += v;
-    if (pm) break;
-    j -= 32;
-  }
-  return acc;
-}
-
-struct ScanLbArgs {
-  const LNode* nodes;
-  const int32_t* feat;
-  int mtry;
-  const uint64_t* E;
-  const int64_t* yq;
-  const int32_t* poff;
-  const int32_t* pmap;
-  const int32_t* ptotal;
-  unsigned int* ticket;
-  LbNS* agg;
-  LbNS* incl;
-  uint32_t* flag;
-  PieceRec* prec;
-};
-
-// a7 split search, one piece per iteration of a persistent CTA.
-__global__ void __launch_bounds__(NT) k_split_scan_lb(ScanLbArgs g) {
-  __shared__ int32_t smc[NT / 32];
-  __shared__ int64_t sms[NT / 32];
-  __shared__ double sg[NT / 32];
-  __shared__ uint32_t sr[NT / 32];
-  __shared__ int32_t sw[NT / 32];
-  __shared__ int s_t, s_exn;
-  __shared__ int64_t s_exS;
-  const int total = *g.ptotal;
-  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  for (;;) {
-    if (tid == 0) s_t = atomicAdd(g.ticket, 1u);
-    __syncthreads();
-    const int t = s_t;
-    if (t >= total) break;
-    const int item = g.pmap[t], t0 = g.poff[item], k = t - t0;
-    const LNode nd = g.nodes[item / g.mtry];
-    const int f = g.feat[item];
-    const uint64_t* seg = g.E + nd.base + (int64_t)f * nd.a;
-    const int a = nd.a;
-    const int64_t nk = nd.n, Sk = nd.S;
-    const int j0 = k * PIECE + tid * PIECE_V;
-    uint64_t e[PIECE_V + 1];
-    int32_t wc[PIECE_V];
-    int64_t ws[PIECE_V];
-    int32_t tc = 0;
-    int64_t ts = 0;
-#pragma unroll
-    for (int u = 0; u <= PIECE_V; ++u) e[u] = (j0 + u < a) ? seg[j0 + u] : 0ull;
-#pragma unroll
-    for (int u = 0; u < PIECE_V; ++u) {
-      wc[u] = 0;
-      ws[u] = 0;
-      if (j0 + u < a) {
-        wc[u] = e_w(e[u]);
-        ws[u] = (int64_t)wc[u] * __ldg(g.yq + e_row(e[u]));
-      }
-      tc += wc[u];
-      ts += ws[u];
-    }
-    int32_t totc;
-    int64_t tots;
-    int32_t prc = block_excl_scan(tc, smc, totc);
-    int64_t prs = block_excl_scan(ts, sms, tots);
-    if (tid == 0) {
-      LbNS v;
-      v.S = tots;
-      v.n = totc;
-      v.pad = 0;
-      if (k == 0) {
-        g.incl[t] = v;
-        __threadfence();
-        *(volatile uint32_t*)(g.flag + t) = 2u;
-      } else {
-        g.agg[t] = v;
-        __threadfence();
-        *(volatile uint32_t*)(g.flag + t) = 1u;
-      }
-    }
-    if (k > 0 && wid == 0) {
-      int32_t exn;
-      int64_t exS;
-      lookback_ns(t, t0, g.agg, g.incl, g.flag, exn, exS);
-      if (lane == 0) {
-        LbNS v;
-        v.S = exS + tots;
-        v.n = exn + totc;
-        v.pad = 0;
-        g.incl[t] = v;
-        __threadfence();
-        *(volatile uint32_t*)(g.flag + t) = 2u;
-        s_exn = exn;
-        s_exS = exS;
-      }
-    }
-    __syncthreads();
-    if (k > 0) {
-      prc += s_exn;
-      prs += s_exS;
-    }
-    double bg = -1.0;
-    uint32_t brank = 0xffffffffu, brb = 0;
-    int32_t bpos = -1, bnl = 0;
-    int64_t bSl = 0;
-#pragma unroll
-    for (int u = 0; u < PIECE_V; ++u) {
-      prc += wc[u];
-      prs += ws[u];
-      const int j = j0 + u;
-      if (j + 1 < a) {
-        const uint32_t ra = e_rank(e[u]), rb = e_rank(e[u + 1]);
-        if (ra != rb && screen_may_win(nk, Sk, prc, prs, bg)) {
-          const double gk = split_key(nk, Sk, prc, prs);
-          if (rec_better(gk, ra, bg, brank)) {
-            bg = gk;
-            brank = ra;
-            brb = rb;
-            bpos = j;
-            bnl = prc;
-            bSl = prs;
-          }
-        }
-      }
-    }
-    // block argmax (g desc, rank asc)
-    const int wl = warp_argmax_key(gkey(bg), brank);
-    const double wg = __shfl_sync(0xffffffffu, bg, wl >= 0 ? wl : 0);
-    const uint32_t wr = __shfl_sync(0xffffffffu, brank, wl >= 0 ? wl : 0);
-    if (lane == 0) {
-      sg[wid] = wl >= 0 ? wg : -1.0;
-      sr[wid] = wl >= 0 ? wr : 0xffffffffu;
-      sw[wid] = wl >= 0 ? wid * 32 + wl : -1;
-    }
-    __syncthreads();
-    if (tid == 0) {
-      double gg = sg[0];
-      uint32_t r = sr[0];
-      int who = sw[0];
-      for (int q = 1; q < NT / 32; ++q)
-        if (sw[q] >= 0 && (who < 0 || rec_better(sg[q], sr[q], gg, r))) {
-          gg = sg[q];
-          r = sr[q];
-          who = sw[q];
-        }
-      sw[0] = who;
-      if (who < 0) {
-        PieceRec R;
-        R.g = -1.0;
-        R.rank_a = 0xffffffffu;
-        R.rank_b = 0;
-        R.pos = -1;
-        R.nl = 0;
-        R.Sl = 0;
-        g.prec[t] = R;
-      }
-    }
-    __syncthreads();
-    if (tid == sw[0]) {
-      PieceRec R;
-      R.g = bg;
-      R.rank_a = brank;
-      R.rank_b = brb;
-      R.pos = bpos;
-      R.nl = bnl;
-      R.Sl = bSl;
-      g.prec[t] = R;
-    }
-    __syncthreads();
-  }
-}
-
-// best piece record of every scan item (warp per item)
-__global__ void k_item_reduce(int nitems, const int32_t* cnt, const int32_t* off, const PieceRec* prec, Rec* rec) {
-  const int lane = threadIdx.x & 31;
-  const int item = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  if (item >= nitems) return;
-  const int c = cnt[item], o = off[item];
-  double bg = -1.0;
-  uint32_t br = 0xffffffffu;
-  int bi = -1;
-  for (int q = lane; q < c; q += 32) {
-    const double gq = prec[o + q].g;
-    const uint32_t rq = prec[o + q].rank_a;
-    if (gq >= 0.0 && rec_better(gq, rq, bg, br)) {
-      bg = gq;
-      br = rq;
-      bi = o + q;
-    }
-  }
-  const int wl = warp_argmax_key(gkey(bg), br);
-  const int sbi = __shfl_sync(0xffffffffu, bi, wl >= 0 ? wl : 0);
-  const int src = wl >= 0 ? sbi : -1;
-  if (lane == 0) {
-    Rec R;
-    if (src >= 0) {
-      const PieceRec P = prec[src];
-      R.g = P.g;
-      R.rank_a = P.rank_a;
-      R.rank_b = P.rank_b;
-      R.pos = P.pos;
-      R.nl = P.nl;
-      R.Sl = P.Sl;
-    } else {
-      R.g = -1.0;
-      R.rank_a = 0xffffffffu;
-      R.rank_b = 0;
-      R.pos = -1;
-      R.nl = 0;
-      R.Sl = 0;
-    }
-    rec[item] = R;
-  }
-}
-
 struct DestArgs {
   const LNode* nodes;
   const Split* split;
@@ -1091,53 +595,6 @@ struct DestArgs {
   double* csum;  // 2 per node: sum of w*y of the left / right child
 };
 
-// a9/a10: goes-right flag of every row of a split node + child sums of w*y (one piece per CTA)
-__global__ void __launch_bounds__(NT) k_dest_pc(DestArgs g) {
-  __shared__ double sl[NT / 32], sr[NT / 32];
-  const int t = blockIdx.x;
-  if (t >= *g.ptotal) return;
-  const int k = g.pmap[t], pc = t - g.poff[k];
-  const Split sp = g.split[k];
-  const LNode nd = g.nodes[k];
-  const uint64_t* seg = g.E + nd.base + (int64_t)sp.f * nd.a;
-  uint8_t* sd = g.side + (int64_t)nd.b * g.n;
-  double accl = 0.0, accr = 0.0;
-  const int j0 = pc * PIECE + threadIdx.x * PIECE_V;
-#pragma unroll
-  for (int u = 0; u < PIECE_V; ++u) {
-    const int j = j0 + u;
-    if (j < nd.a) {
-      const uint64_t ej = seg[j];
-      const uint32_t row = e_row(ej);
-      const int s = j > sp.pos;
-      sd[row] = (uint8_t)s;
-      const double v = __dmul_rn((double)e_w(ej), g.y[row]);
-      if (s) accr += v;
-      else accl += v;
-    }
-  }
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) {
-    accl += __shfl_down_sync(0xffffffffu, accl, o);
-    accr += __shfl_down_sync(0xffffffffu, accr, o);
-  }
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  if (lane == 0) {
-    sl[wid] = accl;
-    sr[wid] = accr;
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    double a0 = 0.0, a1 = 0.0;
-    for (int q = 0; q < NT / 32; ++q) {
-      a0 += sl[q];
-      a1 += sr[q];
-    }
-    atomicAdd(&g.csum[2 * k], a0);
-    atomicAdd(&g.csum[2 * k + 1], a1);
-  }
-}
-
 __global__ void k_child_values(int N, const Split* split, const double* csum, const LNode* nodes, Pool pool) {
   const int k = blockIdx.x * blockDim.x + threadIdx.x;
   if (k >= N) return;
@@ -1148,93 +605,7 @@ __global__ void k_child_values(int N, const Split* split, const double* csum, co
   pool.value[r + sp.lraw + 1] = __ddiv_rn(csum[2 * k + 1], (double)sp.nr);
 }
 
-struct PartArgs {
-  const LNode* nodes;
-  const Split* split;
-  const Child* child;
-  int p;
-  const uint64_t* Ecur;
-  const uint8_t* side;
-  int64_t n;
-  uint64_t* Enext;
-  uint64_t* Esmall;
-  const int32_t* poff;
-  const int32_t* pmap;
-  const int32_t* ptotal;
-  unsigned int* ticket;
-  unsigned long long* st;
-};
-
-// a9 partition, one piece per iteration of a persistent CTA (left counts carried by look-back)
-__global__ void __launch_bounds__(NT) k_partition_lb(PartArgs g) {
-  __shared__ int32_t sm[NT / 32];
-  __shared__ int s_t;
-  __shared__ int64_t s_ex;
-  const int total = *g.ptotal;
-  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  for (;;) {
-    if (tid == 0) s_t = atomicAdd(g.ticket, 1u);
-    __syncthreads();
-    const int t = s_t;
-    if (t >= total) break;
-    const int item = g.pmap[t], t0 = g.poff[item], k = t - t0;
-    const int node = item / g.p, f = item - node * g.p;
-    const LNode nd = g.nodes[node];
-    const Child cl = g.child[2 * node], cr = g.child[2 * node + 1];
-    const bool keepL = cl.kind == KIND_LARGE || cl.kind == KIND_SMALL;
-    const bool keepR = cr.kind == KIND_LARGE || cr.kind == KIND_SMALL;
-    const uint64_t* seg = g.Ecur + nd.base + (int64_t)f * nd.a;
-    const uint8_t* sd = g.side + (int64_t)nd.b * g.n;
-    const int j0 = k * PIECE + tid * PIECE_V;
-    uint64_t e[PIECE_V];
-    bool left[PIECE_V];
-#pragma unroll
-    for (int u = 0; u < PIECE_V; ++u) e[u] = (j0 + u < nd.a) ? seg[j0 + u] : 0ull;
-    int32_t cnt = 0;
-#pragma unroll
-    for (int u = 0; u < PIECE_V; ++u) {
-      left[u] = (j0 + u < nd.a) && sd[e_row(e[u])] == 0;
-      cnt += left[u];
-    }
-    int32_t tot;
-    int32_t lb = block_excl_scan(cnt, sm, tot);
-    if (tid == 0)
-      *(volatile unsigned long long*)(g.st + t) = ((k == 0 ? 2ull : 1ull) << 62) | (unsigned long long)tot;
-    if (k > 0 && wid == 0) {
-      const int64_t ex = lookback_cnt(t, t0, g.st);
-      if (lane == 0) {
-        *(volatile unsigned long long*)(g.st + t) = (2ull << 62) | (unsigned long long)(ex + tot);
-        s_ex = ex;
-      }
-    }
-    __syncthreads();
-    if (k > 0) lb += (int32_t)s_ex;
-    uint64_t* dl = keepL ? (cl.kind == KIND_LARGE ? g.Enext : g.Esmall) + cl.base + (int64_t)f * cl.a : nullptr;
-    uint64_t* dr = keepR ? (cr.kind == KIND_LARGE ? g.Enext : g.Esmall) + cr.base + (int64_t)f * cr.a : nullptr;
-#pragma unroll
-    for (int u = 0; u < PIECE_V; ++u) {
-      const int j = j0 + u;
-      if (j < nd.a) {
-        if (left[u]) {
-          if (keepL) dl[lb] = e[u];
-          ++lb;
-        } else if (keepR) {
-          dr[j - lb] = e[u];
-        }
-      }
-    }
-    __syncthreads();
-  }
-}
-
-// ------------------------------------------------------------------ two-pass units with TMA staging (global phase v5)
-// Units are contiguous ranges of UNIT entries of one segment.  Pass 1 computes
-// every unit's aggregate with plain coalesced loads (embarrassingly parallel);
-// a device-wide exclusive scan over units gives each unit its prefix inside
-// its segment (units of a segment are consecutive); pass 2 processes units
-// with a static round-robin assignment, so each CTA double-buffers its next
-// unit's bulk copy (cp.async.bulk + mbarrier) behind the current one.  No
-// inter-CTA waiting anywhere.
+// ------------------------------------------------------------------ TMA bulk copies + read-only gathers (global phase)
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void mbar_init(uint64_t* bar) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(bar)) : "memory");
@@ -1297,425 +668,6 @@ __device__ __forceinline__ void key_bounds(double nkd, double Skd, int64_t nk, i
   const double hi = (d + E), lo = fmax(d - E, 0.0);
   gU = hi * hi * r * (1.0 + 9.5367431640625e-07);  // (1 + 2^-20)
   gL = lo * lo * r * (1.0 - 9.5367431640625e-07);
-}
-
-// Cheap rigorous upper bound of the S4.3 key in fp32, scaled by 2^-128 (no
-// overflow): with a = RN32(nk)*RN32(Sl), b = RN32(nl)*RN32(Sk), d = |a - b|,
-// |d - D| <= 2^-21.5 (|a| + |b|), so (d + E)^2 * rcp(nl*nr) * (1 + 2^-18) with
-// E = 2^-20 (|a| + |b|) bounds g from above.  Results below 2^-100 (scaled)
-// are raised to 2^-100 so that an fp32 underflow never screens a candidate
-// out: every candidate whose bound reaches the threshold is evaluated exactly.
-__device__ __forceinline__ float key_upper32(float nkf, float Skf, int32_t nl, int32_t nr, int64_t Sl) {
-  const float a = nkf * (float)Sl * 5.421010862427522e-20f;  // * 2^-64
-  const float b = (float)nl * Skf * 5.421010862427522e-20f;
-  const float d = fabsf(a - b);
-  const float E = (fabsf(a) + fabsf(b)) * 9.5367431640625e-07f;  // 2^-20
-  const float u = d + E;
-  const float r = rcp_approx((float)nl * (float)nr);
-  return fmaxf(u * u * r * 1.0000038146972656f, 7.888609052210118e-31f);  // (1 + 2^-18), floor 2^-100
-}
-__device__ __forceinline__ float key_lower32(float nkf, float Skf, int32_t nl, int32_t nr, int64_t Sl) {
-  const float a = nkf * (float)Sl * 5.421010862427522e-20f;
-  const float b = (float)nl * Skf * 5.421010862427522e-20f;
-  const float d = fabsf(a - b);
-  const float E = (fabsf(a) + fabsf(b)) * 9.5367431640625e-07f;
-  const float u = fmaxf(d - E, 0.0f);
-  const float r = rcp_approx((float)nl * (float)nr);
-  return u * u * r * 0.9999961853027344f;  // (1 - 2^-18)
-}
-__device__ __forceinline__ float scale_key(double g) {  // g * 2^-128, rounded down
-  const float f = (float)(g * 2.938735877055719e-39);
-  return f > 0.0f ? __fmul_rd(f, 0.99999988079071044921875f) : f;
-}
-
-constexpr int SUV = 7;               // scan: entries per thread (odd)
-constexpr int SUNIT = NT * SUV;      // 3840 entries per unit
-constexpr int PUV = 15;              // partition: entries per thread (odd)
-constexpr int PUNIT = NT * PUV;      // 3840 entries per unit
-
-// unit counts per item: mode 0 scan (node = i/div), 2 partition (node = i/div, split with a kept child)
-__global__ void k_unit_count(int mode, int nitems, int div, int unit, const LNode* nodes, const Split* split,
-                             const Child* child, int32_t* cnt) {
-  const int i = blockIdx.x * blockDim.x + threadIdx.x;
-  if (i >= nitems) return;
-  const int k = i / div;
-  int a = nodes[k].a;
-  if (mode == 2) {
-    const int kl = child[2 * k].kind, kr = child[2 * k + 1].kind;
-    if (!split[k].split || (kl != KIND_LARGE && kl != KIND_SMALL && kr != KIND_LARGE && kr != KIND_SMALL)) a = 0;
-  }
-  cnt[i] = (a + unit - 1) / unit;
-}
-
-struct UnitArgs {
-  const LNode* nodes;
-  const int32_t* feat;  // scan: drawn feature per item (NULL for the partition: f = item % p)
-  int div;              // items per node (mtry or p)
-  int unit;
-  const uint64_t* E;
-  const int32_t* poff;
-  const int32_t* pmap;
-  const int32_t* ptotal;
-};
-
-__device__ __forceinline__ const uint64_t* unit_src(const UnitArgs& u, int t, int& item, int& k, int& cnt, LNode& nd,
-                                                    int& f) {
-  item = u.pmap[t];
-  k = t - u.poff[item];
-  const int node = item / u.div;
-  f = u.feat ? u.feat[item] : item - node * u.div;
-  nd = u.nodes[node];
-  cnt = min(u.unit, nd.a - k * u.unit);
-  return u.E + nd.base + (int64_t)f * nd.a + (int64_t)k * u.unit;
-}
-
-// pass 1 of the scan: (n, S) of every unit
-__global__ void __launch_bounds__(NT) k_unit_sums(UnitArgs u, const int64_t* yq, int64_t* un, int64_t* uS) {
-  __shared__ int32_t s1[NT / 32];
-  __shared__ int64_t s2[NT / 32];
-  const int total = *u.ptotal;
-  for (int t = blockIdx.x; t < total; t += gridDim.x) {
-    int item, k, cnt, f;
-    LNode nd;
-    const uint64_t* src = unit_src(u, t, item, k, cnt, nd, f);
-    int32_t c = 0;
-    int64_t S = 0;
-    constexpr int G = 8;
-    for (int j0 = threadIdx.x; j0 < cnt; j0 += G * NT) {
-      uint64_t ev[G];
-      int64_t yv[G];
-#pragma unroll
-      for (int q = 0; q < G; ++q) ev[q] = src[min(j0 + q * NT, cnt - 1)];
-#pragma unroll
-      for (int q = 0; q < G; ++q) yv[q] = ldg_s64_nc(yq + e_row(ev[q]));
-#pragma unroll
-      for (int q = 0; q < G; ++q)
-        if (j0 + q * NT < cnt) {
-          const int32_t w = e_w(ev[q]);
-          c += w;
-          S += (int64_t)w * yv[q];
-        }
-    }
-    int32_t tc;
-    int64_t tS;
-    block_excl_scan(c, s1, tc);
-    block_excl_scan(S, s2, tS);
-    if (threadIdx.x == 0) {
-      un[t] = tc;
-      uS[t] = tS;
-    }
-  }
-}
-
-// pass 1 of the partition: left count of every unit
-__global__ void __launch_bounds__(NT) k_unit_lefts(UnitArgs u, const uint8_t* side, int64_t n, int64_t* ul) {
-  __shared__ int64_t s1[NT / 32];
-  const int total = *u.ptotal;
-  for (int t = blockIdx.x; t < total; t += gridDim.x) {
-    int item, k, cnt, f;
-    LNode nd;
-    const uint64_t* src = unit_src(u, t, item, k, cnt, nd, f);
-    const uint8_t* sd = side + (int64_t)nd.b * n;
-    int64_t c = 0;
-    constexpr int G = 8;
-    for (int j0 = threadIdx.x; j0 < cnt; j0 += G * NT) {
-      uint32_t rw[G];
-      uint32_t sv[G];
-#pragma unroll
-      for (int q = 0; q < G; ++q) rw[q] = e_row(src[min(j0 + q * NT, cnt - 1)]);
-#pragma unroll
-      for (int q = 0; q < G; ++q) sv[q] = ldg_u8_nc(sd + rw[q]);
-#pragma unroll
-      for (int q = 0; q < G; ++q) c += (j0 + q * NT < cnt) && sv[q] == 0;
-    }
-    int64_t tc;
-    block_excl_scan(c, s1, tc);
-    if (threadIdx.x == 0) ul[t] = tc;
-  }
-}
-
-struct ScanArgs2 {
-  UnitArgs u;
-  const int64_t* yq;
-  const int64_t* pren;  // exclusive scan of unit n over all units
-  const int64_t* preS;
-  PieceRec* prec;
-};
-
-__device__ __forceinline__ void key_bounds32(float nkf, float Skf, int32_t nl, int32_t nr, int64_t Sl, float& gL,
-                                             float& gU) {
-  const float a = nkf * (float)Sl * 5.421010862427522e-20f;  // * 2^-64
-  const float b = (float)nl * Skf * 5.421010862427522e-20f;
-  const float d = fabsf(a - b);
-  const float E = (fabsf(a) + fabsf(b)) * 9.5367431640625e-07f;  // 2^-20
-  const float r = rcp_approx((float)nl * (float)nr);
-  const float hi = d + E, lo = fmaxf(d - E, 0.0f);
-  gU = fmaxf(hi * hi * r * 1.0000038146972656f, 7.888609052210118e-31f);
-  gL = lo * lo * r * 0.9999961853027344f;
-}
-
-__global__ void __launch_bounds__(NT) k_split_scan_2p(ScanArgs2 g) {
-  extern __shared__ __align__(16) unsigned char dsm[];
-  uint64_t* bufs = (uint64_t*)dsm;  // 2 x (SUNIT + 4) entries
-  __shared__ uint64_t bar[2];
-  __shared__ int32_t smc[NT / 32];
-  __shared__ int64_t sms[NT / 32];
-  __shared__ double sg[NT / 32];
-  __shared__ uint32_t sr[NT / 32];
-  __shared__ int32_t sw[NT / 32];
-  __shared__ float sf[NT / 32];
-  __shared__ int s_off[2];
-  __shared__ float s_M;
-  const int total = *g.u.ptotal;
-  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  auto issue = [&](int t, int slot) {
-    int item, k, cnt, f;
-    LNode nd;
-    const uint64_t* src = unit_src(g.u, t, item, k, cnt, nd, f);
-    const int cload = min(cnt + 1, nd.a - k * SUNIT);
-    s_off[slot] = stage_entries(bufs + (size_t)slot * (SUNIT + 4), src, cload, &bar[slot]);
-  };
-  if (tid == 0) {
-    mbar_init(&bar[0]);
-    mbar_init(&bar[1]);
-    if ((int)blockIdx.x < total) issue(blockIdx.x, 0);
-  }
-  __syncthreads();
-  uint32_t phase[2] = {0u, 0u};
-  int cur = 0;
-  for (int t = blockIdx.x; t < total; t += gridDim.x, cur ^= 1) {
-    if (tid == 0 && t + (int)gridDim.x < total) issue(t + gridDim.x, cur ^ 1);  // prefetch the next unit
-    int item, k, cnt, f;
-    LNode nd;
-    unit_src(g.u, t, item, k, cnt, nd, f);
-    const int a = nd.a, u0 = k * SUNIT;
-    const int64_t nk = nd.n, Sk = nd.S;
-    const float nkf = (float)nk, Skf = (float)Sk;
-    const int t0 = g.u.poff[item];
-    const int32_t exn = (int32_t)(g.pren[t] - g.pren[t0]);
-    const int64_t exS = g.preS[t] - g.preS[t0];
-    mbar_wait(&bar[cur], phase[cur]);
-    phase[cur] ^= 1u;
-    const uint64_t* buf = bufs + (size_t)cur * (SUNIT + 4) + s_off[cur];
-    const int jl = tid * SUV;
-    // my entries (+ the next one) in registers; w*y_q gathers all in flight
-    const int cl_ = min(cnt, a - u0 - 1);  // last loaded index (the unit's entries + the next one if any)
-    uint64_t e[SUV + 1];
-#pragma unroll
-    for (int q = 0; q <= SUV; ++q) e[q] = buf[min(jl + q, cl_)];
-    uint32_t rw[SUV];
-#pragma unroll
-    for (int q = 0; q < SUV; ++q) rw[q] = e_row(buf[min(jl + q, cnt - 1)]);
-    int64_t wy[SUV];
-#pragma unroll
-    for (int q = 0; q < SUV; ++q) wy[q] = ldg_s64_nc(g.yq + rw[q]);
-    int32_t tc = 0;
-    int64_t ts = 0;
-#pragma unroll
-    for (int q = 0; q < SUV; ++q) {
-      const int32_t w = jl + q < cnt ? e_w(e[q]) : 0;
-      wy[q] *= w;
-      tc += w;
-      ts += wy[q];
-    }
-    int32_t totc;
-    int64_t tots;
-    const int32_t prc0 = block_excl_scan(tc, smc, totc) + exn;
-    const int64_t prs0 = block_excl_scan(ts, sms, tots) + exS;
-    // one pass: bounds of every candidate; keep the upper bounds, M = best lower bound of the unit
-    float gUq[SUV];
-    float mL = 0.0f;
-    {
-      int32_t prc = prc0;
-      int64_t prs = prs0;
-#pragma unroll
-      for (int q = 0; q < SUV; ++q) {
-        const int j = jl + q;
-        prc += jl + q < cnt ? e_w(e[q]) : 0;
-        prs += wy[q];
-        gUq[q] = -1.0f;
-        if (j < cnt && u0 + j + 1 < a && e_rank(e[q]) != e_rank(e[q + 1])) {
-          float gL;
-          key_bounds32(nkf, Skf, prc, (int32_t)(nk - prc), prs, gL, gUq[q]);
-          mL = fmaxf(mL, gL);
-        }
-      }
-    }
-    {
-      const float wm = __int_as_float((int)__reduce_max_sync(0xffffffffu, (unsigned)__float_as_int(mL)));
-      if (lane == 0) sf[wid] = wm;
-      __syncthreads();
-      if (tid == 0) {
-        float M = 0.0f;
-        for (int q = 0; q < NT / 32; ++q) M = fmaxf(M, sf[q]);
-        s_M = M;
-      }
-      __syncthreads();
-    }
-    const float M = s_M;
-    // exact keys only where the upper bound reaches M (prefix recomputed for those few)
-    double bg = -1.0;
-    uint32_t brank = 0xffffffffu, brb = 0;
-    int32_t bpos = -1, bnl = 0;
-    int64_t bSl = 0;
-    uint32_t pass = 0;
-#pragma unroll
-    for (int q = 0; q < SUV; ++q) pass |= (gUq[q] >= M ? 1u : 0u) << q;
-    if (pass) {
-      int32_t prc = prc0;
-      int64_t prs = prs0;
-#pragma unroll
-      for (int q = 0; q < SUV; ++q) {
-        prc += jl + q < cnt ? e_w(e[q]) : 0;
-        prs += wy[q];
-        if (((pass >> q) & 1u) && gUq[q] >= scale_key(bg)) {
-          const double gk = split_key(nk, Sk, prc, prs);
-          const uint32_t ra = e_rank(e[q]);
-          if (rec_better(gk, ra, bg, brank)) {
-            bg = gk;
-            brank = ra;
-            brb = e_rank(e[q + 1]);
-            bpos = u0 + jl + q;
-            bnl = prc;
-            bSl = prs;
-          }
-        }
-      }
-    }
-    const int wl = warp_argmax_key(gkey(bg), brank);
-    const double wg = __shfl_sync(0xffffffffu, bg, wl >= 0 ? wl : 0);
-    const uint32_t wr = __shfl_sync(0xffffffffu, brank, wl >= 0 ? wl : 0);
-    if (lane == 0) {
-      sg[wid] = wl >= 0 ? wg : -1.0;
-      sr[wid] = wl >= 0 ? wr : 0xffffffffu;
-      sw[wid] = wl >= 0 ? wid * 32 + wl : -1;
-    }
-    __syncthreads();
-    if (tid == 0) {
-      double gg = -1.0;
-      uint32_t r = 0xffffffffu;
-      int who = -1;
-      for (int q = 0; q < NT / 32; ++q)
-        if (sw[q] >= 0 && (who < 0 || rec_better(sg[q], sr[q], gg, r))) {
-          gg = sg[q];
-          r = sr[q];
-          who = sw[q];
-        }
-      sw[0] = who;
-      if (who < 0) {
-        PieceRec R;
-        R.g = -1.0;
-        R.rank_a = 0xffffffffu;
-        R.rank_b = 0;
-        R.pos = -1;
-        R.nl = 0;
-        R.Sl = 0;
-        g.prec[t] = R;
-      }
-    }
-    __syncthreads();
-    if (tid == sw[0]) {
-      PieceRec R;
-      R.g = bg;
-      R.rank_a = brank;
-      R.rank_b = brb;
-      R.pos = bpos;
-      R.nl = bnl;
-      R.Sl = bSl;
-      g.prec[t] = R;
-    }
-    __syncthreads();
-  }
-}
-
-struct PartArgs2 {
-  UnitArgs u;
-  const Child* child;
-  const uint8_t* side;
-  int64_t n;
-  uint64_t* Enext;
-  uint64_t* Esmall;
-  const int64_t* prel;  // exclusive scan of unit left counts over all units
-};
-
-__global__ void __launch_bounds__(NT) k_partition_2p(PartArgs2 g) {
-  extern __shared__ __align__(16) unsigned char dsm[];
-  uint64_t* bufs = (uint64_t*)dsm;              // 2 x (PUNIT + 2) entries (input)
-  uint64_t* outb = bufs + 2 * (PUNIT + 2);      // PUNIT entries (left part, then right part)
-  __shared__ uint64_t bar[2];
-  __shared__ int32_t sm[NT / 32];
-  __shared__ int s_off[2];
-  const int total = *g.u.ptotal;
-  const int tid = threadIdx.x;
-  auto issue = [&](int t, int slot) {
-    int item, k, cnt, f;
-    LNode nd;
-    const uint64_t* src = unit_src(g.u, t, item, k, cnt, nd, f);
-    s_off[slot] = stage_entries(bufs + (size_t)slot * (PUNIT + 2), src, cnt, &bar[slot]);
-  };
-  if (tid == 0) {
-    mbar_init(&bar[0]);
-    mbar_init(&bar[1]);
-    if ((int)blockIdx.x < total) issue(blockIdx.x, 0);
-  }
-  __syncthreads();
-  uint32_t phase[2] = {0u, 0u};
-  int cur = 0;
-  for (int t = blockIdx.x; t < total; t += gridDim.x, cur ^= 1) {
-    if (tid == 0 && t + (int)gridDim.x < total) issue(t + gridDim.x, cur ^ 1);
-    int item, k, cnt, f;
-    LNode nd;
-    unit_src(g.u, t, item, k, cnt, nd, f);
-    const int node = item / g.u.div;
-    const int u0 = k * PUNIT;
-    const Child cl = g.child[2 * node], cr = g.child[2 * node + 1];
-    const uint8_t* sd = g.side + (int64_t)nd.b * g.n;
-    const int64_t exl = g.prel[t] - g.prel[g.u.poff[item]];
-    mbar_wait(&bar[cur], phase[cur]);
-    phase[cur] ^= 1u;
-    const uint64_t* buf = bufs + (size_t)cur * (PUNIT + 2) + s_off[cur];
-    const int jl = tid * PUV;
-    // issue every side gather before consuming any (independent loads in flight)
-    uint32_t sv[PUV];  // one register per load (byte arrays get packed, which serialises the loads)
-    uint32_t rw[PUV];
-#pragma unroll
-    for (int q = 0; q < PUV; ++q) rw[q] = e_row(buf[min(jl + q, cnt - 1)]);
-#pragma unroll
-    for (int q = 0; q < PUV; ++q) sv[q] = ldg_u8_nc(sd + rw[q]);
-    uint32_t lmask = 0;
-    int32_t c = 0;
-#pragma unroll
-    for (int q = 0; q < PUV; ++q)
-      if (jl + q < cnt && sv[q] == 0) {
-        lmask |= 1u << q;
-        ++c;
-      }
-    int32_t tot;
-    const int32_t lbl = block_excl_scan(c, sm, tot);
-    int li = lbl, ri = tot + (jl - lbl);
-#pragma unroll
-    for (int q = 0; q < PUV; ++q) {
-      const int j = jl + q;
-      if (j < cnt) {
-        const uint64_t e = buf[j];
-        if ((lmask >> q) & 1u) outb[li++] = e;
-        else outb[ri++] = e;
-      }
-    }
-    __syncthreads();
-    const int64_t exr = (int64_t)u0 - exl;
-    const bool keepL = cl.kind == KIND_LARGE || cl.kind == KIND_SMALL;
-    const bool keepR = cr.kind == KIND_LARGE || cr.kind == KIND_SMALL;
-    if (keepL) {
-      uint64_t* dl = (cl.kind == KIND_LARGE ? g.Enext : g.Esmall) + cl.base + (int64_t)f * cl.a + exl;
-      for (int i = tid; i < tot; i += NT) dl[i] = outb[i];
-    }
-    if (keepR) {
-      uint64_t* dr = (cr.kind == KIND_LARGE ? g.Enext : g.Esmall) + cr.base + (int64_t)f * cr.a + exr;
-      for (int i = tid; i < cnt - tot; i += NT) dr[i] = outb[tot + i];
-    }
-    __syncthreads();
-  }
 }
 
 // ------------------------------------------------------------------ tree-affine item kernels (global phase v6)
@@ -2263,7 +1215,8 @@ __global__ void __launch_bounds__(NT) k_dest_bits(DestArgs g, uint32_t* sideb, i
 // list partition is needed.  Tiny nodes go through a CTA-wide work queue so
 // every warp stays busy until the whole subtree is grown.
 constexpr int TINY = 64;
-constexpr int TGRP = 4;   // drawn predictors staged per group in the tiny path
+constexpr int TGRP = 7;   // drawn predictors staged per group in the tiny path
+constexpr int TPU = 4;    // scan passes interleaved in the tiny path
 
 struct SRec {  // node record of a subtree (local ids); thr is computed at flush from rows (ra, rb)
   int32_t feature, left, count;
@@ -2298,11 +1251,12 @@ struct WRec {  // best candidate found by one warp for its share of a node's fea
 
 __host__ __device__ inline size_t align16(size_t x) { return (x + 15) & ~size_t(15); }
 __host__ __device__ inline int max_medium(int A) { return A / (TINY + 1) + 2; }
+__host__ __device__ inline int sub_temp(int A) { return A > TGRP * TINY ? A : TGRP * TINY; }
 
 __host__ __device__ inline size_t subtree_smem(int A, int p) {
   size_t s = 0;
   s += align16((size_t)p * A * 4);                    // list
-  s += align16((size_t)SUB_NW * A * 4);               // per-warp partition temp
+  s += align16((size_t)SUB_NW * sub_temp(A) * 4);     // per-warp partition temp / tiny staging
   s += align16((size_t)A * 8) * 2;                    // wy, w*y
   s += align16((size_t)A * 4) * 2;                    // w, global row
   s += align16((size_t)A) * 2;                        // side, row index inside its tiny root
@@ -2311,7 +1265,6 @@ __host__ __device__ inline size_t subtree_smem(int A, int p) {
   s += align16((size_t)(A + 1) * sizeof(TNode));      // tiny work queue
   s += align16((size_t)SUB_NW * p * 2) * 2;           // Fisher-Yates scratch, drawn features
   s += align16((size_t)SUB_NW * sizeof(WRec));
-  s += align16((size_t)SUB_NW * TGRP * TINY * 4);     // tiny staging
   s += 64;
   return s;
 }
@@ -2381,7 +1334,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   uint32_t* list = (uint32_t*)ptr;
   ptr += align16((size_t)p * A * 4);
   uint32_t* temp_all = (uint32_t*)ptr;
-  ptr += align16((size_t)SUB_NW * A * 4);
+  ptr += align16((size_t)SUB_NW * sub_temp(A) * 4);
   int64_t* wy = (int64_t*)ptr;
   ptr += align16((size_t)A * 8);
   double* wyd = (double*)ptr;
@@ -2407,7 +1360,6 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   ptr += align16((size_t)SUB_NW * p * 2);
   WRec* wrec = (WRec*)ptr;
   ptr += align16((size_t)SUB_NW * sizeof(WRec));
-  uint32_t* stg_all = (uint32_t*)ptr;
   __shared__ int s_nloc, s_ncur, s_gbase, s_alloc, s_head, s_pending;
   __shared__ int32_t s_scan[SUB_NW];
 
@@ -2420,7 +1372,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   const uint64_t* src = g.Es + root.base;
   int16_t* mind = mind_all + wid * p;
   int16_t* feats = feats_all + wid * p;
-  uint32_t* temp = temp_all + (size_t)wid * A;
+  uint32_t* temp = temp_all + (size_t)wid * sub_temp(A);
   long long tclk[5];
   tclk[0] = clock64();
   int n_med = 0, n_tiny = 0;
@@ -2768,8 +1720,8 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         } else if (*(volatile int*)&s_pending == 0) {
           break;
         } else {
-          __nanosleep(ns);
-          ns = min(ns * 2, 256);
+          __nanosleep(ns);  // idle warp: back off so the busy warps keep the issue slots
+          ns = min(ns * 2, 2048);
         }
       }
       if (h >= 0)
@@ -2786,9 +1738,11 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       ++n_tiny;
       const int rlo = nd.rlo, ra = nd.ra;
       const int an = __popcll(nd.mask);  // distinct rows of the node
+      const long long c0_ = g.stats ? clock64() : 0;
       warp_draw_mtry(g.seed, t, nd.key, p, g.mtry, mind, feats, lane);
+      const long long c1_ = g.stats ? clock64() : 0;
       const int64_t nk = nd.n, Sk = nd.S;
-      uint32_t* stg = stg_all + (size_t)wid * TGRP * TINY;
+      uint32_t* stg = temp;  // the medium levels' partition buffer (>= TGRP * TINY entries)
       const unsigned lt = (1u << lane) - 1u;
       // lane-local best over all (feature, boundary) items: key g, tie = (feature << 16 | rank)
       double lg = -1.0;
@@ -2797,72 +1751,103 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       int64_t lSl = 0;
       for (int s0 = 0; s0 < g.mtry; s0 += TGRP) {
         const int ng = min(TGRP, g.mtry - s0);
-        // stage: the node's entries of each drawn feature, in value order, packed [slot][0..an)
-  #pragma unroll
+        // stage: the node's entries of each drawn feature, in value order, packed [slot][0..an).
+        // All loads of the group are issued before any store (ILP across features).
+        uint32_t ev[2 * TGRP];
+        uint8_t ri[2 * TGRP];
+#pragma unroll
         for (int u = 0; u < TGRP; ++u) {
-          if (u >= ng) break;
-          const int f = feats[s0 + u];
-          const uint32_t* seg = list + (size_t)f * a0 + rlo;
-          const uint32_t e0 = lane < ra ? seg[lane] : 0u, e1 = lane + 32 < ra ? seg[lane + 32] : 0u;
-          const bool v0 = lane < ra && ((nd.mask >> rmap[e0 & 0xffffu]) & 1ull);
-          const bool v1 = lane + 32 < ra && ((nd.mask >> rmap[e1 & 0xffffu]) & 1ull);
+          const uint32_t* seg = list + (size_t)feats[s0 + (u < ng ? u : 0)] * a0 + rlo;
+          ev[2 * u] = (u < ng && lane < ra) ? seg[lane] : 0u;
+          ev[2 * u + 1] = (u < ng && lane + 32 < ra) ? seg[lane + 32] : 0u;
+        }
+#pragma unroll
+        for (int k = 0; k < 2 * TGRP; ++k) ri[k] = rmap[ev[k] & 0xffffu];
+#pragma unroll
+        for (int u = 0; u < TGRP; ++u) {
+          const bool v0 = u < ng && lane < ra && ((nd.mask >> ri[2 * u]) & 1ull);
+          const bool v1 = u < ng && lane + 32 < ra && ((nd.mask >> ri[2 * u + 1]) & 1ull);
           const unsigned m0 = __ballot_sync(0xffffffffu, v0), m1 = __ballot_sync(0xffffffffu, v1);
-          if (v0) stg[u * an + __popc(m0 & lt)] = e0;
-          if (v1) stg[u * an + __popc(m0) + __popc(m1 & lt)] = e1;
+          if (v0) stg[u * an + __popc(m0 & lt)] = ev[2 * u];
+          if (v1) stg[u * an + __popc(m0) + __popc(m1 & lt)] = ev[2 * u + 1];
         }
         __syncwarp();
-        // dense passes over the ng*an (slot, position) items: segmented scans by slot
+        // dense passes over the ng*an (slot, position) items: segmented scans by slot,
+        // TPU passes at a time with their loads and shuffles interleaved
         const int total = ng * an;
         int32_t cw = 0;
         int64_t cs = 0;
-        for (int i0 = 0; i0 < total; i0 += 32) {
-          const int i = i0 + lane;
-          const bool act = i < total;
-          const int sl = act ? i / an : ng;
-          const int j = act ? i - sl * an : 0;
-          const uint32_t e = act ? stg[i] : 0u;
-          const uint32_t lr = e & 0xffffu;
-          int32_t w = act ? wl[lr] : 0;
-          int64_t wv = act ? wy[lr] : 0;
-          // inclusive segmented scan (segments are slot runs; lane-o is in my slot iff o <= j)
-  #pragma unroll
+        for (int i0 = 0; i0 < total; i0 += 32 * TPU) {
+          uint32_t e[TPU], en[TPU];
+          int32_t w[TPU];
+          int64_t wv[TPU];
+          int jj[TPU];
+#pragma unroll
+          for (int k = 0; k < TPU; ++k) {
+            const int i = i0 + 32 * k + lane;
+            const bool act = i < total;
+            const int sl = act ? i / an : ng;
+            jj[k] = act ? i - sl * an : 0;
+            e[k] = act ? stg[i] : 0u;
+            en[k] = (act && jj[k] + 1 < an) ? stg[i + 1] : 0u;
+          }
+#pragma unroll
+          for (int k = 0; k < TPU; ++k) {
+            const bool act = i0 + 32 * k + lane < total;
+            const uint32_t lr = e[k] & 0xffffu;
+            w[k] = act ? wl[lr] : 0;
+            wv[k] = act ? wy[lr] : 0;
+          }
+          // inclusive segmented scans (segments are slot runs; lane-o is in my slot iff o <= j)
+#pragma unroll
           for (int o = 1; o < 32; o <<= 1) {
-            const int32_t uw = __shfl_up_sync(0xffffffffu, w, o);
-            const int64_t uv = __shfl_up_sync(0xffffffffu, wv, o);
-            if (lane >= o && o <= j) {
-              w += uw;
-              wv += uv;
-            }
-          }
-          // my slot started before this pass (j > lane): add the previous pass's carry
-          if (j > lane) {
-            w += cw;
-            wv += cs;
-          }
-          const int32_t lw = __shfl_sync(0xffffffffu, w, 31);
-          const int64_t lv = __shfl_sync(0xffffffffu, wv, 31);
-          const int lj = __shfl_sync(0xffffffffu, j, 31);
-          const bool cont = lj + 1 < an;  // last item's slot continues into the next pass
-          if (act && j + 1 < an) {
-            const uint32_t en = stg[i + 1];
-            if ((en >> 16) != (e >> 16) && screen_may_win(nk, Sk, w, wv, lg)) {
-              const double gk = split_key(nk, Sk, w, wv);
-              const uint32_t tie = ((uint32_t)feats[s0 + sl] << 16) | (e >> 16);
-              if (gk > lg || (gk == lg && tie < ltie)) {
-                lg = gk;
-                ltie = tie;
-                lnl = w;
-                lSl = wv;
-                lra = lr;
-                lrb = en & 0xffffu;
+#pragma unroll
+            for (int k = 0; k < TPU; ++k) {
+              const int32_t uw = __shfl_up_sync(0xffffffffu, w[k], o);
+              const int64_t uv = __shfl_up_sync(0xffffffffu, wv[k], o);
+              if (lane >= o && o <= jj[k]) {
+                w[k] += uw;
+                wv[k] += uv;
               }
             }
           }
-          cw = cont ? lw : 0;
-          cs = cont ? lv : 0;
+#pragma unroll
+          for (int k = 0; k < TPU; ++k) {
+            if (i0 + 32 * k >= total) break;
+            // my slot started before this pass (j > lane): add the previous pass's carry
+            if (jj[k] > lane) {
+              w[k] += cw;
+              wv[k] += cs;
+            }
+            const int32_t lw = __shfl_sync(0xffffffffu, w[k], 31);
+            const int64_t lv = __shfl_sync(0xffffffffu, wv[k], 31);
+            const int lj = __shfl_sync(0xffffffffu, jj[k], 31);
+            const bool cont = lj + 1 < an;  // last item's slot continues into the next pass
+            cw = cont ? lw : 0;
+            cs = cont ? lv : 0;
+          }
+#pragma unroll
+          for (int k = 0; k < TPU; ++k) {
+            const int i = i0 + 32 * k + lane;
+            if (i < total && jj[k] + 1 < an && (en[k] >> 16) != (e[k] >> 16) &&
+                screen_may_win(nk, Sk, w[k], wv[k], lg)) {
+              const double gk = split_key(nk, Sk, w[k], wv[k]);
+              const uint32_t tie = ((uint32_t)feats[s0 + i / an] << 16) | (e[k] >> 16);
+              if (gk > lg || (gk == lg && tie < ltie)) {
+                lg = gk;
+                ltie = tie;
+                lnl = w[k];
+                lSl = wv[k];
+                lra = e[k] & 0xffffu;
+                lrb = en[k] & 0xffffu;
+              }
+            }
+          }
         }
         __syncwarp();
       }
+      const long long c2_ = g.stats ? clock64() : 0;
+      if (g.stats && lane == 0) { atomicAdd(&g.stats[11], (unsigned long long)(c1_ - c0_)); atomicAdd(&g.stats[12], (unsigned long long)(c2_ - c1_)); }
       const int wlane = warp_argmax_key(gkey(lg), ltie);
       const double bgs = __shfl_sync(0xffffffffu, lg, wlane >= 0 ? wlane : 0);
       const double bg = wlane >= 0 ? bgs : -1.0;
@@ -3303,26 +2288,12 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
     DBuf<char> scan_tmp(std::max<size_t>(scan_tb, 16), s);
     DBuf<LevelSummary> dsum(1, s);
     PinnedSummary hs;
-    // piece decomposition buffers (sized for the largest level of a batch)
-    const int64_t cap_items = cap_level * p;
-    const int64_t cap_pieces = (int64_t)p * ((int64_t)B * n / PIECE + cap_level) + 1;
-    const int64_t cap_spieces = (int64_t)mtry * ((int64_t)B * n / PIECE + cap_level) + 1;
-    DBuf<int32_t> pcnt(cap_items, s), poff(cap_items, s), pmap(cap_pieces, s), ptot(1, s);
-    DBuf<LbNS> lbagg(cap_spieces, s), lbincl(cap_spieces, s);
-    DBuf<uint32_t> lbflag(cap_spieces, s);
-    DBuf<PieceRec> prec(cap_spieces, s);
-    DBuf<unsigned long long> pst(cap_pieces, s);
-    DBuf<unsigned int> ticket(1, s);
-    DBuf<int64_t> un(cap_pieces, s), pren(cap_pieces, s);
-    DBuf<int64_t> uS(cap_pieces, s), preS(cap_pieces, s), ul(cap_pieces, s), prel(cap_pieces, s);
-    size_t unit_tb = 0, unit_tb2 = 0;
-    cub::DeviceScan::ExclusiveSum(nullptr, unit_tb, uS.p, preS.p, (int)cap_pieces, s);
-    cub::DeviceScan::ExclusiveSum(nullptr, unit_tb2, un.p, pren.p, (int)cap_pieces, s);
-    unit_tb = std::max(unit_tb, unit_tb2);
-    DBuf<char> unit_tmp(std::max<size_t>(unit_tb, 16), s);
+    // piece decomposition of the winning segments (k_dest_bits), sized for the largest level of a batch
+    const int64_t cap_pieces = (int64_t)B * n / PIECE + cap_level + 1;
+    DBuf<int32_t> pcnt(cap_level, s), poff(cap_level, s), pmap(cap_pieces, s), ptot(1, s);
     DBuf<double> csum(2 * cap_level, s);
     size_t piece_tb = 0;
-    cub::DeviceScan::ExclusiveSum(nullptr, piece_tb, pcnt.p, poff.p, (int)cap_items, s);
+    cub::DeviceScan::ExclusiveSum(nullptr, piece_tb, pcnt.p, poff.p, (int)cap_level, s);
     DBuf<char> piece_tmp(std::max<size_t>(piece_tb, 16), s);
     auto piece_setup = [&](int mode, int nitems, int div, const LNode* nodes, const Split* sp, const Child* ch,
                            int32_t* cnt, int32_t* off, int32_t* map, int32_t* tot, cudaStream_t st) {
@@ -3340,34 +2311,9 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
         k_piece_map<<<(unsigned)ceil_div(nitems, 256), 256, 0, st>>>(nitems, cnt, off, map, tot);
       }
     };
-    auto unit_setup = [&](int mode, int nitems, int div, int unit, const LNode* nodes, const Split* sp, const Child* ch,
-                          int32_t* cnt, int32_t* off, int32_t* map, int32_t* tot, cudaStream_t st) {
-      {
-        KScope ks_("k_piece_count", st, 0.0);
-        k_unit_count<<<(unsigned)ceil_div(nitems, 256), 256, 0, st>>>(mode, nitems, div, unit, nodes, sp, ch, cnt);
-      }
-      {
-        KScope ks_("cub_ExclusiveSum", st, 0.0);
-        size_t tb2 = piece_tb;
-        BF_CUDA_CHECK(cub::DeviceScan::ExclusiveSum(piece_tmp.p, tb2, cnt, off, nitems, st));
-      }
-      {
-        KScope ks_("k_piece_map", st, 0.0);
-        k_piece_map<<<(unsigned)ceil_div(nitems, 256), 256, 0, st>>>(nitems, cnt, off, map, tot);
-      }
-    };
-    const size_t scan_smem = sizeof(uint64_t) * 2 * (SUNIT + 4), part_smem = sizeof(uint64_t) * (3 * PUNIT + 4);
-    BF_CUDA_CHECK(cudaFuncSetAttribute(k_split_scan_2p, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)scan_smem));
-    BF_CUDA_CHECK(cudaFuncSetAttribute(k_partition_2p, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)part_smem));
-    int occ_s = 0, occ_p = 0, nsm = 0, dev_id = 0;
+    int nsm = 0, dev_id = 0;
     cudaGetDevice(&dev_id);
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev_id);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_s, k_split_scan_2p, NT, scan_smem);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_p, k_partition_2p, NT, part_smem);
-    int occ_u = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_u, k_unit_lefts, NT, 0);
-    const unsigned grid_scan = (unsigned)std::max(1, occ_s * nsm), grid_part = (unsigned)std::max(1, occ_p * nsm);
-    const unsigned grid_sums = (unsigned)std::max(1, occ_u * nsm);
     // tree-affine kernels
     const int64_t nw = (n + 31) / 32;
     DBuf<uint32_t> sideb((size_t)B * nw, s);
@@ -3491,45 +2437,16 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
           for (auto& e : lev) cudaEventCreate(&e);
           cudaEventRecord(lev[0], s);
         }
-        static const bool scan_tree = getenv("BF_SCAN_2P") == nullptr;
         BF_CUDA_CHECK(cudaMemsetAsync(tlo.p, 0, sizeof(int32_t) * Bc, s));
         BF_CUDA_CHECK(cudaMemsetAsync(thi.p, 0, sizeof(int32_t) * Bc, s));
         {
           KScope ks_("k_tree_ranges", s, 0.0);
           k_tree_ranges<<<(unsigned)ceil_div(N, 256), 256, 0, s>>>(N, nc, tlo.p, thi.p);
         }
-        if (scan_tree) {
+        {  // ---- a7 split search: tree-affine CTAs own whole (node, drawn feature) items
           TScanArgs ga{nc, feat.p, mtry, Bc, Ec, yq.p, tlo.p, thi.p, rec.p};
-          KScope ks_("k_split_scan", s, 0.0);
+          KScope ks_("k_split_scan_tree", s, 0.0);
           k_split_scan_tree<<<grid_tscan, NT, tscan_smem, s>>>(ga);
-        } else {
-        // ---- a7 split search over units (two passes: unit sums, then units in parallel)
-          const int NI = N * mtry;
-          unit_setup(0, NI, mtry, SUNIT, nc, split.p, child.p, pcnt.p, poff.p, pmap.p, ptot.p, s);
-          {
-            UnitArgs ua{nc, feat.p, mtry, SUNIT, Ec, poff.p, pmap.p, ptot.p};
-            {
-              KScope ks_("k_unit_sums", s, 0.0);
-              k_unit_sums<<<grid_sums, NT, 0, s>>>(ua, yq.p, un.p, uS.p);
-            }
-            const int64_t bound_s = (int64_t)mtry * (cur_a / SUNIT + N) + 1;
-            {
-              KScope ks_("cub_ExclusiveSum", s, 0.0);
-              size_t tb2 = unit_tb;
-              BF_CUDA_CHECK(cub::DeviceScan::ExclusiveSum(unit_tmp.p, tb2, un.p, pren.p, (int)bound_s, s));
-              tb2 = unit_tb;
-              BF_CUDA_CHECK(cub::DeviceScan::ExclusiveSum(unit_tmp.p, tb2, uS.p, preS.p, (int)bound_s, s));
-            }
-            ScanArgs2 ga{ua, yq.p, pren.p, preS.p, prec.p};
-            {
-              KScope ks_("k_split_scan", s, 0.0);
-              k_split_scan_2p<<<grid_scan, NT, scan_smem, s>>>(ga);
-            }
-          }
-          {
-            KScope ks_("k_item_reduce", s, 0.0);
-            k_item_reduce<<<(unsigned)ceil_div((int64_t)NI * 32, 256), 256, 0, s>>>(NI, pcnt.p, poff.p, prec.p, rec.p);
-          }
         }
         if (lvl_timing) cudaEventRecord(lev[1], s);
         {
@@ -3559,7 +2476,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
         BF_CUDA_CHECK(cudaMemsetAsync(csum.p, 0, sizeof(double) * 2 * (size_t)N, s));
         {
           DestArgs ga{nc, split.p, Ec, y, n, side.p, poff.p, pmap.p, ptot.p, csum.p};
-          KScope ks_("k_dest", s, 0.0);
+          KScope ks_("k_dest_bits", s, 0.0);
           k_dest_bits<<<(unsigned)(cur_a / PIECE + N + 1), NT, 0, s>>>(ga, sideb.p, nw);
         }
         {
@@ -3570,7 +2487,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
         // ---- a9 partition: tree-affine CTAs own whole items; goes-right bitmap in shared memory
         {
           TPartArgs ga{nc, split.p, child.p, p, Bc, Ec, sideb.p, nw, bm_smem ? 1 : 0, En, Es.p, tlo.p, thi.p};
-          KScope ks_("k_partition", s, 0.0);
+          KScope ks_("k_partition_tree", s, 0.0);
           k_partition_tree<<<grid_tpart, TPNT, tpart_smem, s>>>(ga);
         }
         if (lvl_timing) cudaEventRecord(lev[3], s);
@@ -3582,9 +2499,9 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
         BF_CUDA_CHECK(cudaStreamSynchronize(s));
         {  // algorithmic bytes
           const double sa = (double)hs.h->split_a;
-          prof_add_bytes("k_split_scan", (double)cur_a * mtry * 16.0);
-          prof_add_bytes("k_dest", sa * 17.0);
-          prof_add_bytes("k_partition", sa * p * 17.0);
+          prof_add_bytes("k_split_scan_tree", (double)cur_a * mtry * 16.0);
+          prof_add_bytes("k_dest_bits", sa * 17.0);
+          prof_add_bytes("k_partition_tree", sa * p * 17.0);
         }
         if (lvl_timing) {
           float ms1 = 0, ms2 = 0, ms3 = 0;
@@ -3642,6 +2559,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
             d2h(h, st.p, 16, s);
             BF_CUDA_CHECK(cudaStreamSynchronize(s));
             const double c = (double)h[5];
+            fprintf(stderr, "[subtree tiny] draw=%.0f groups=%.0f per tiny node\n", h[11] / (double)(h[7] ? h[7] : 1), h[12] / (double)(h[7] ? h[7] : 1));
             fprintf(stderr, "[subtree] A=%d ctas=%llu mean_a0=%.1f cyc/cta: load=%.0f medium=%.0f tiny=%.0f flush=%.0f | medium nodes/cta=%.1f tiny nodes/cta=%.1f nodes/cta=%.1f warp-cyc in tiny/cta=%.0f busy=%.0f (%.0f per tiny node)\n",
                     A, h[5], h[6] / c, h[0] / c, h[1] / c, h[2] / c, h[3] / c, h[4] / c, h[7] / c, h[9] / c, h[8] / c,
                     h[10] / c, h[10] / (double)(h[7] ? h[7] : 1));
