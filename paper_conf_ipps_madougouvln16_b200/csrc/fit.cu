@@ -2,22 +2,29 @@
 //
 // Design:
 //   once per fit   a1 validate, a2 fixed-point y_q, a3 presort: per feature the
-//                  rows in x order as 8-byte entries (dense rank << 32 | row)
-//                  plus the table of distinct values.
+//                  rows in x order (CUB radix sort of order-preserving keys),
+//                  the dense rank of every value and the table of distinct values.
 //   per batch of B trees in flight:
-//     a4 bootstrap multiplicities (Philox BOOT), payload {w*y_q, w} per row;
+//     a4 bootstrap multiplicities (Philox BOOT), root sums;
 //     a5 root lists: per (tree, feature) stable compaction of the presorted
-//        column to in-bag rows (node-major block: p segments of a entries);
+//        column to the in-bag rows, 8-byte entries rank|row|w (node-major
+//        block: p segments of a entries, each in value order);
 //     GLOBAL PHASE (nodes with more than A distinct rows), level-synchronous
 //     over all trees of the batch:
-//        a6 k_mtry, a7 k_split_scan (CTA per (node, drawn feature): segmented
-//        prefix scan of (w, w*y_q) over the sorted segment, exact key, argmax),
-//        a8 k_finalize, k_child_place, a9/a10 k_dest (goes-right flags +
-//        child means), a9 k_partition (CTA per (node, feature): stable
-//        partition into the children's blocks);
+//        a6 k_mtry; a7 k_split_scan_tree (tree-affine CTAs own whole
+//        (node, drawn feature) items: TMA-staged units, segmented prefix scan
+//        of (w, w*y_q) with a carry, rigorous fp64 screen, exact key near the
+//        max); a8 k_finalize + CUB scans + k_child_place; a9/a10 k_dest_bits
+//        (goes-right bitmap of the winning segments + child sums of w*y) and
+//        k_child_values; a9 k_partition_tree (tree-affine CTAs, goes-right
+//        bitmap in shared memory, stable partition of all p segments into the
+//        children's blocks, small children to the subtree queue);
 //     SUBTREE PHASE (nodes with <= A distinct rows): one CTA grows the whole
-//        subtree in shared memory (k_subtree);
-//     a11 emit the packed forest.
+//        subtree in shared memory (k_subtree: medium levels with in-place
+//        nested ranges, then tiny nodes of <= 64 rows as bit masks over their
+//        tiny root's sorted segments, through a CTA work queue);
+//     a11 k_emit: raw per-tree pools -> packed node arrays (root 0, right =
+//        left + 1; slot order is allocation order, not BFS: DESIGN.md R21).
 // All split arithmetic is exact (int64 sums, int128 D, correctly rounded
 // key) so the topology is bit-identical to the CPU oracle whatever the scan
 // order, tile size or number of GPUs.
