@@ -724,22 +724,39 @@ struct TScanArgs {
   Rec* rec;
 };
 
-constexpr int TSV = 7;              // entries per thread (odd: conflict-free 64-bit shared loads)
-constexpr int TUNIT = NT * TSV;     // 3840 entries per unit
+constexpr int TSV = 9;              // entries per thread (odd: conflict-free 64-bit shared loads)
+constexpr int TUNIT = NT * TSV;     // 2304 entries per unit (18 KB bulk copy)
 
-// a7 split search: one CTA owns whole (node, drawn feature) items of one tree
-__global__ void __launch_bounds__(NT) k_split_scan_tree(TScanArgs g) {
+// The exact key off the unrolled scan loops (rarely reached: only where the upper bound passes the screen).
+__device__ __noinline__ double split_key_call(int64_t nk, int64_t Sk, int64_t nl, int64_t Sl) {
+  return split_key(nk, Sk, nl, Sl);
+}
+
+struct WBest {  // best exact candidate of one warp for the current unit
+  double g;
+  uint32_t rank, rb;
+  int32_t pos, nl;
+  int64_t Sl;
+};
+
+// a7 split search: one CTA owns whole (node, drawn feature) items of one tree.
+// Per unit (TMA bulk copy, double-buffered): each thread takes TSV consecutive
+// entries, gathers y_q[row] (all TSV in flight), scans serially in registers on
+// top of ONE block scan of (n, S); every boundary gets cheap rigorous bounds
+// gL <= g <= gU (fp64), the unit's threshold M = max(best gL, item best) is one
+// block max, and only boundaries with gU >= M get the exact S4.3 key.  Four
+// barriers per unit; each thread re-derives the block results from the
+// per-warp values, so there are no broadcast round trips.
+__global__ void __launch_bounds__(NT, 2) k_split_scan_tree(TScanArgs g) {
   extern __shared__ __align__(16) unsigned char dsm[];
   uint64_t* bufs = (uint64_t*)dsm;  // 2 x (TUNIT + 4)
+  constexpr int NW = NT / 32;
   __shared__ uint64_t bar[2];
-  __shared__ int32_t smc[NT / 32];
-  __shared__ int64_t sms[NT / 32];
-  __shared__ double sg[NT / 32];
-  __shared__ uint32_t sr[NT / 32];
-  __shared__ int32_t sw[NT / 32];
+  __shared__ int32_t smc[NW];
+  __shared__ int64_t sms[NW];
+  __shared__ double smL[NW];
+  __shared__ WBest swb[NW];
   __shared__ int s_off[2];
-  __shared__ double s_M;
-  __shared__ int64_t s_cS;
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const TreeSched ts = tree_sched(g.B);
   if (tid == 0) {
@@ -751,9 +768,7 @@ __global__ void __launch_bounds__(NT) k_split_scan_tree(TScanArgs g) {
   int cur = 0;
   for (int b = ts.b0; b < g.B; b += ts.bstep) {
     const int i_lo = g.tlo[b] * g.mtry, i_hi = g.thi[b] * g.mtry;
-    // sequence of (item, unit) of this CTA: items i_lo + c, + C, ...; units 0.. of each
     int item = i_lo + ts.c, unit = 0;
-    auto units_of = [&](int it) { return (g.nodes[it / g.mtry].a + TUNIT - 1) / TUNIT; };
     auto issue = [&](int it, int un, int slot) {
       const LNode nd = g.nodes[it / g.mtry];
       const int f = g.feat[it];
@@ -764,24 +779,26 @@ __global__ void __launch_bounds__(NT) k_split_scan_tree(TScanArgs g) {
     };
     if (item >= i_hi) continue;
     if (tid == 0) issue(item, 0, cur);
-    // running state of the current item
+    // running state of the current item (identical in every thread)
     int32_t carry_n = 0;
     int64_t carry_S = 0;
-    double ig = -1.0;
-    uint32_t irk = 0xffffffffu, irb = 0;
-    int32_t ipos = -1, inl = 0;
-    int64_t iSl = 0;
+    WBest ib;
+    ib.g = -1.0;
+    ib.rank = 0xffffffffu;
+    ib.rb = 0;
+    ib.pos = -1;
+    ib.nl = 0;
+    ib.Sl = 0;
+    LNode nd = g.nodes[item / g.mtry];
     while (item < i_hi) {
-      const int nun = units_of(item);
-      // next (item, unit) to prefetch
+      const int nun = (nd.a + TUNIT - 1) / TUNIT;
       int nitem = item, nunit = unit + 1;
       if (nunit >= nun) {
         nitem = item + ts.C;
         nunit = 0;
       }
-      __syncthreads();  // the other buffer is free
+      __syncthreads();  // S0: the other buffer and the per-warp slots are free
       if (tid == 0 && nitem < i_hi) issue(nitem, nunit, cur ^ 1);
-      const LNode nd = g.nodes[item / g.mtry];
       const int a = nd.a, u0 = unit * TUNIT, cnt = min(TUNIT, a - u0);
       const int64_t nk = nd.n, Sk = nd.S;
       const double nkd = (double)nk, Skd = (double)Sk;
@@ -789,63 +806,98 @@ __global__ void __launch_bounds__(NT) k_split_scan_tree(TScanArgs g) {
       phase[cur] ^= 1u;
       const uint64_t* buf = bufs + (size_t)cur * (TUNIT + 4) + s_off[cur];
       const int jl = tid * TSV;
-      uint32_t rw[TSV];
+      // the thread's entries, read from shared memory once: rank (and the next entry's), w, w * y_q
+      uint32_t rk[TSV + 1];
+      int32_t wq[TSV];
       int64_t wy[TSV];
 #pragma unroll
-      for (int q = 0; q < TSV; ++q) rw[q] = e_row(buf[min(jl + q, cnt - 1)]);
-#pragma unroll
-      for (int q = 0; q < TSV; ++q) wy[q] = ldg_s64_nc(g.yq + rw[q]);
+      for (int q = 0; q < TSV; ++q) {
+        const bool in = jl + q < cnt;
+        const uint64_t e = buf[min(jl + q, cnt)];  // buf[cnt]: the next unit's first entry (if any)
+        rk[q] = e_rank(e);
+        wq[q] = in ? e_w(e) : 0;
+        wy[q] = ldg_s64_nc(g.yq + (in ? e_row(e) : 0u));
+      }
+      rk[TSV] = e_rank(buf[min(jl + TSV, cnt)]);  // the entry after my last (checked against a below)
       int32_t tc = 0;
       int64_t tsum = 0;
 #pragma unroll
       for (int q = 0; q < TSV; ++q) {
-        const int32_t w = jl + q < cnt ? e_w(buf[jl + q]) : 0;
-        wy[q] *= w;
-        tc += w;
+        wy[q] *= wq[q];
+        tc += wq[q];
         tsum += wy[q];
       }
-      int32_t totc;
-      int64_t tots;
-      const int32_t prc0 = block_excl_scan(tc, smc, totc) + carry_n;
-      const int64_t prs0 = block_excl_scan(tsum, sms, tots) + carry_S;
-      // pass 1: bounds; M = the unit's best lower bound (or the item's running best)
-      double mL = ig;
+      // S1: one block scan of (n, S): warp inclusive scans, per-warp totals, every thread adds the earlier warps'
+      int32_t ic = tc;
+      int64_t is = tsum;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int32_t uc = __shfl_up_sync(0xffffffffu, ic, o);
+        const int64_t us = __shfl_up_sync(0xffffffffu, is, o);
+        if (lane >= o) {
+          ic += uc;
+          is += us;
+        }
+      }
+      if (lane == 31) {
+        smc[wid] = ic;
+        sms[wid] = is;
+      }
+      __syncthreads();
+      int32_t prc0 = carry_n + ic - tc, totc = 0;
+      int64_t prs0 = carry_S + is - tsum, tots = 0;
+#pragma unroll
+      for (int k = 0; k < NW; ++k) {
+        const int32_t c = smc[k];
+        const int64_t v = sms[k];
+        if (k < wid) {
+          prc0 += c;
+          prs0 += v;
+        }
+        totc += c;
+        tots += v;
+      }
+      // bounds of every boundary; the thread's best lower bound
+      float gUf[TSV];
+      double mL = ib.g;
       {
         int32_t prc = prc0;
         int64_t prs = prs0;
 #pragma unroll
         for (int q = 0; q < TSV; ++q) {
+          gUf[q] = -1.0f;
           const int j = jl + q;
           if (j < cnt) {
-            const uint64_t e = buf[j];
-            prc += e_w(e);
+            prc += wq[q];
             prs += wy[q];
-            if (u0 + j + 1 < a && e_rank(e) != e_rank(buf[j + 1])) {
+            if (u0 + j + 1 < a && rk[q] != rk[q + 1]) {
               double gL, gU;
               key_bounds(nkd, Skd, nk, prc, prs, gL, gU);
               mL = fmax(mL, gL);
+              gUf[q] = __double2float_ru(gU);
             }
           }
         }
       }
+      // S2: block max of the lower bounds -> M
       {
         const uint64_t kb = gkey(mL);
         const uint32_t hi = __reduce_max_sync(0xffffffffu, (uint32_t)(kb >> 32));
         const uint32_t lo = __reduce_max_sync(0xffffffffu, ((uint32_t)(kb >> 32) == hi) ? (uint32_t)kb : 0u);
-        if (lane == 0) sg[wid] = (hi | lo) ? __longlong_as_double((long long)((((uint64_t)hi << 32) | lo) - 1ull)) : -1.0;
-        __syncthreads();
-        if (tid == 0) {
-          double M = -1.0;
-          for (int q = 0; q < NT / 32; ++q) M = fmax(M, sg[q]);
-          s_M = M;
-        }
-        __syncthreads();
+        if (lane == 0) smL[wid] = (hi | lo) ? __longlong_as_double((long long)((((uint64_t)hi << 32) | lo) - 1ull)) : -1.0;
       }
-      const double M = s_M;
-      double bg = -1.0;
-      uint32_t brank = 0xffffffffu, brb = 0;
-      int32_t bpos = -1, bnl = 0;
-      int64_t bSl = 0;
+      __syncthreads();
+      double M = -1.0;
+#pragma unroll
+      for (int k = 0; k < NW; ++k) M = fmax(M, smL[k]);
+      // exact keys where the upper bound reaches M
+      WBest tb;
+      tb.g = -1.0;
+      tb.rank = 0xffffffffu;
+      tb.rb = 0;
+      tb.pos = -1;
+      tb.nl = 0;
+      tb.Sl = 0;
       {
         int32_t prc = prc0;
         int64_t prs = prs0;
@@ -853,96 +905,57 @@ __global__ void __launch_bounds__(NT) k_split_scan_tree(TScanArgs g) {
         for (int q = 0; q < TSV; ++q) {
           const int j = jl + q;
           if (j < cnt) {
-            const uint64_t e = buf[j];
-            prc += e_w(e);
+            prc += wq[q];
             prs += wy[q];
-            if (u0 + j + 1 < a) {
-              const uint64_t en = buf[j + 1];
-              const uint32_t ra = e_rank(e), rb = e_rank(en);
-              if (ra != rb) {
-                double gL, gU;
-                key_bounds(nkd, Skd, nk, prc, prs, gL, gU);
-                if (gU >= M && gU >= bg) {
-                  const double gk = split_key(nk, Sk, prc, prs);
-                  if (rec_better(gk, ra, bg, brank)) {
-                    bg = gk;
-                    brank = ra;
-                    brb = rb;
-                    bpos = u0 + j;
-                    bnl = prc;
-                    bSl = prs;
-                  }
-                }
+            if ((double)gUf[q] >= M && gUf[q] >= 0.0f) {
+              const double gk = split_key_call(nk, Sk, prc, prs);
+              const uint32_t ra = rk[q];
+              if (rec_better(gk, ra, tb.g, tb.rank)) {
+                tb.g = gk;
+                tb.rank = ra;
+                tb.rb = rk[q + 1];
+                tb.pos = u0 + j;
+                tb.nl = prc;
+                tb.Sl = prs;
               }
             }
           }
         }
       }
-      const int wl = warp_argmax_key(gkey(bg), brank);
-      const double wg = __shfl_sync(0xffffffffu, bg, wl >= 0 ? wl : 0);
-      const uint32_t wr = __shfl_sync(0xffffffffu, brank, wl >= 0 ? wl : 0);
-      if (lane == 0) {
-        sg[wid] = wl >= 0 ? wg : -1.0;
-        sr[wid] = wl >= 0 ? wr : 0xffffffffu;
-        sw[wid] = wl >= 0 ? wid * 32 + wl : -1;
+      // S3: per-warp winners; every thread merges them (unit order == position order)
+      {
+        const int wl = warp_argmax_key(gkey(tb.g), tb.rank);
+        if (wl >= 0 && lane == wl) swb[wid] = tb;
+        if (wl < 0 && lane == 0) swb[wid].g = -1.0;
       }
       __syncthreads();
-      if (tid == 0) {
-        double gg = -1.0;
-        uint32_t r = 0xffffffffu;
-        int who = -1;
-        for (int q = 0; q < NT / 32; ++q)
-          if (sw[q] >= 0 && (who < 0 || rec_better(sg[q], sr[q], gg, r))) {
-            gg = sg[q];
-            r = sr[q];
-            who = sw[q];
-          }
-        sw[0] = who;
-      }
-      __syncthreads();
-      const int who = sw[0];
-      if (who >= 0) {  // broadcast the unit winner; merge into the item's running best (unit order == position order)
-        if (tid == who) {
-          sg[0] = bg;
-          sr[0] = brank;
-          sw[1] = (int)brb;
-          sw[2] = bpos;
-          sw[3] = bnl;
-          s_cS = bSl;
-        }
-        __syncthreads();
-        const double ug = sg[0];
-        if (ug > ig) {  // strictly better (an equal key in a later unit has a higher rank)
-          ig = ug;
-          irk = sr[0];
-          irb = (uint32_t)sw[1];
-          ipos = sw[2];
-          inl = sw[3];
-          iSl = s_cS;
-        }
-        __syncthreads();
+#pragma unroll
+      for (int k = 0; k < NW; ++k) {
+        const double kg = swb[k].g;
+        if (kg >= 0.0 && (kg > ib.g || (kg == ib.g && swb[k].rank < ib.rank))) ib = swb[k];
       }
       carry_n += totc;
       carry_S += tots;
       if (unit + 1 >= nun) {  // item done
         if (tid == 0) {
           Rec R;
-          R.g = ig;
-          R.rank_a = irk;
-          R.rank_b = irb;
-          R.pos = ipos;
-          R.nl = inl;
-          R.Sl = iSl;
+          R.g = ib.g;
+          R.rank_a = ib.rank;
+          R.rank_b = ib.rb;
+          R.pos = ib.pos;
+          R.nl = ib.nl;
+          R.Sl = ib.Sl;
           g.rec[item] = R;
         }
         carry_n = 0;
         carry_S = 0;
-        ig = -1.0;
-        irk = 0xffffffffu;
-        irb = 0;
-        ipos = -1;
-        inl = 0;
-        iSl = 0;
+        ib.g = -1.0;
+        ib.rank = 0xffffffffu;
+        ib.rb = 0;
+        ib.pos = -1;
+        ib.nl = 0;
+        ib.Sl = 0;
+        if (nitem < i_hi) nd = g.nodes[nitem / g.mtry];
       }
       item = nitem;
       unit = nunit;
@@ -964,6 +977,8 @@ struct TPartArgs {
   uint64_t* Esmall;
   const int32_t* tlo;
   const int32_t* thi;
+  const int32_t* ioff;  // per node: first work item (N + 1 entries; items of a tree are contiguous)
+  const int2* imap;     // per work item: (node, first feature)
 };
 
 constexpr int TPNT = 512;           // threads of the partition CTA (one CTA per SM: the bitmap fills shared memory)
@@ -974,6 +989,25 @@ __device__ __forceinline__ bool part_item_active(const Split* split, const Child
   if (!split[node].split) return false;
   const int kl = child[2 * node].kind, kr = child[2 * node + 1].kind;
   return kl == KIND_LARGE || kl == KIND_SMALL || kr == KIND_LARGE || kr == KIND_SMALL;
+}
+
+__host__ __device__ __forceinline__ int part_group(int a, int p) { return a >= TPUNIT ? 1 : min(p, TPUNIT / a); }
+
+// Work items of the partition (node, group of consecutive features), listed per level so that a
+// partition CTA finds its next item with one load instead of walking the tree's item sequence.
+__global__ void k_part_items_count(int N, int p, const LNode* nodes, const Split* split, const Child* child,
+                                   int32_t* cnt) {
+  const int k = blockIdx.x * blockDim.x + threadIdx.x;
+  if (k > N) return;
+  int c = 0;
+  if (k < N && part_item_active(split, child, k)) c = (p + part_group(nodes[k].a, p) - 1) / part_group(nodes[k].a, p);
+  cnt[k] = c;
+}
+__global__ void k_part_items_map(int N, int p, const LNode* nodes, const int32_t* cnt, const int32_t* off, int2* map) {
+  const int k = blockIdx.x * blockDim.x + threadIdx.x;
+  if (k >= N) return;
+  const int c = cnt[k], o = off[k], gsz = part_group(nodes[k].a, p);
+  for (int i = 0; i < c; ++i) map[o + i] = make_int2(k, i * gsz);
 }
 
 // a9 partition: one CTA owns whole work items of one tree; lefts first, stable.
@@ -1013,16 +1047,10 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
     if (g.bitmap_smem)
       for (int64_t w = tid; w < g.nw; w += TPNT) bm[w] = sideg[w];
     const uint32_t* sb = g.bitmap_smem ? bm : sideg;
-    // work items of the tree in order: per active node, its feature groups (and units of long features);
-    // this CTA takes every C-th item starting at c.  Walk the sequence with a cursor.
-    int wnode = n_lo, wf = 0, widx = 0;  // cursor: next item in the tree's sequence
-    auto item_len = [&](int node, int& gsz, int& nun) {
-      const int a = g.nodes[node].a;
-      gsz = a >= TPUNIT ? 1 : min(g.p, TPUNIT / a);
-      nun = (a + TPUNIT - 1) / TPUNIT;
-    };
-    // advance the cursor: items (node, feature group) are dealt round robin to the tree's CTAs; an owned
-    // item yields all its units in order (so the running left count stays inside one CTA)
+    // this CTA's work items of the tree: every C-th item of the tree's contiguous item range (k_part_items_*);
+    // an owned item yields all its units in order (so the running left count stays inside one CTA)
+    int jcur = g.ioff[n_lo] + ts.c;
+    const int jend = g.ioff[n_hi];
     int cur_nun = 0, cur_unit = 0;  // units left of the owned item being emitted
     PWork cw;
     auto next_mine = [&](PWork& w) -> bool {
@@ -1031,32 +1059,18 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
         w.unit = cur_unit++;
         return true;
       }
-      for (;;) {
-        while (wnode < n_hi && !part_item_active(g.split, g.child, wnode)) {
-          ++wnode;
-          wf = 0;
-        }
-        if (wnode >= n_hi) return false;
-        int gsz, nun;
-        item_len(wnode, gsz, nun);
-        const bool mine = (widx % ts.C) == ts.c;
-        ++widx;
-        cw.node = wnode;
-        cw.f0 = wf;
-        cw.g = min(gsz, g.p - wf);
-        cw.unit = 0;
-        wf += cw.g;
-        if (wf >= g.p) {
-          ++wnode;
-          wf = 0;
-        }
-        if (mine) {
-          cur_nun = cw.g > 1 ? 1 : nun;
-          cur_unit = 1;
-          w = cw;
-          return true;
-        }
-      }
+      if (jcur >= jend) return false;
+      const int2 it = g.imap[jcur];
+      jcur += ts.C;
+      const int a = g.nodes[it.x].a;
+      cw.node = it.x;
+      cw.f0 = it.y;
+      cw.g = min(part_group(a, g.p), g.p - it.y);
+      cw.unit = 0;
+      cur_nun = cw.g > 1 ? 1 : (a + TPUNIT - 1) / TPUNIT;
+      cur_unit = 1;
+      w = cw;
+      return true;
     };
     auto issue = [&](const PWork& w, int slot) {
       const LNode nd = g.nodes[w.node];
@@ -2299,6 +2313,12 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
     const int64_t cap_pieces = (int64_t)B * n / PIECE + cap_level + 1;
     DBuf<int32_t> pcnt(cap_level, s), poff(cap_level, s), pmap(cap_pieces, s), ptot(1, s);
     DBuf<double> csum(2 * cap_level, s);
+    // partition work items (at most p per node)
+    DBuf<int32_t> icnt(cap_level + 1, s), ioff(cap_level + 1, s);
+    DBuf<int2> imap(cap_level * p, s);
+    size_t items_tb = 0;
+    cub::DeviceScan::ExclusiveSum(nullptr, items_tb, icnt.p, ioff.p, (int)(cap_level + 1), s);
+    DBuf<char> items_tmp(std::max<size_t>(items_tb, 16), s);
     size_t piece_tb = 0;
     cub::DeviceScan::ExclusiveSum(nullptr, piece_tb, pcnt.p, poff.p, (int)cap_level, s);
     DBuf<char> piece_tmp(std::max<size_t>(piece_tb, 16), s);
@@ -2493,7 +2513,14 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
         if (lvl_timing) cudaEventRecord(lev[2], s);
         // ---- a9 partition: tree-affine CTAs own whole items; goes-right bitmap in shared memory
         {
-          TPartArgs ga{nc, split.p, child.p, p, Bc, Ec, sideb.p, nw, bm_smem ? 1 : 0, En, Es.p, tlo.p, thi.p};
+          KScope ks_("k_part_items", s, 0.0);
+          k_part_items_count<<<(unsigned)ceil_div(N + 1, 256), 256, 0, s>>>(N, p, nc, split.p, child.p, icnt.p);
+          size_t tb3 = items_tb;
+          BF_CUDA_CHECK(cub::DeviceScan::ExclusiveSum(items_tmp.p, tb3, icnt.p, ioff.p, N + 1, s));
+          k_part_items_map<<<(unsigned)ceil_div(N, 256), 256, 0, s>>>(N, p, nc, icnt.p, ioff.p, imap.p);
+        }
+        {
+          TPartArgs ga{nc, split.p, child.p, p, Bc, Ec, sideb.p, nw, bm_smem ? 1 : 0, En, Es.p, tlo.p, thi.p, ioff.p, imap.p};
           KScope ks_("k_partition_tree", s, 0.0);
           k_partition_tree<<<grid_tpart, TPNT, tpart_smem, s>>>(ga);
         }

@@ -53,6 +53,62 @@ __device__ __forceinline__ int64_t feistel(uint64_t seed, uint32_t t, uint32_t m
   return (int64_t)v;
 }
 
+// pi_tm for every OOB position of a batch, precomputed per (tree, predictor):
+// perm[(b * p + m) * n + a] = pi_tm(a), a < n_o.  The Feistel round function
+// F_r(R) only takes h-bit inputs (h = b/2), so for h <= 12 a CTA first fills
+// the 6 x 2^h round values of its (t, m) in shared memory (6 x 2^h Philox
+// calls) and every pi(a) is then 6 shared-memory lookups per cycle-walking
+// step; otherwise F is computed on the fly.  Same values as feistel().
+constexpr int PH_MAX = 12;
+__device__ __forceinline__ int feistel_h(int64_t n_o) {
+  int b = 64 - __clzll((unsigned long long)(n_o - 1));
+  if (n_o <= 1) b = 0;
+  if (b < 2) b = 2;
+  b += b & 1;
+  return b >> 1;
+}
+__global__ void __launch_bounds__(512) k_perm_fill(uint64_t seed, int32_t t0, int p, int64_t n, const int64_t* nout,
+                                                   int32_t* perm) {
+  extern __shared__ uint32_t ftab[];  // 6 x 2^h (h <= PH_MAX)
+  const int b = blockIdx.z, m = blockIdx.y;
+  const int64_t n_o = nout[b];
+  if (n_o <= 0) return;
+  const uint32_t t = (uint32_t)(t0 + b);
+  const int h = feistel_h(n_o);
+  const uint32_t mask = (uint32_t)((1ull << h) - 1ull);
+  const bool tab = h <= PH_MAX;
+  if (tab) {
+    const int S = 1 << h;
+    for (int k = threadIdx.x; k < 6 * S; k += blockDim.x) {
+      uint32_t x[4];
+      philox4x32_10((uint32_t)(k & (S - 1)), (uint32_t)(k >> h), 3u | ((uint32_t)m << 8), t, (uint32_t)seed,
+                    (uint32_t)(seed >> 32), x);
+      ftab[k] = x[0];
+    }
+    __syncthreads();
+  }
+  int32_t* out = perm + ((int64_t)b * p + m) * n;
+  const int64_t step = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t a = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; a < n_o; a += step) {
+    if (!tab) {
+      out[a] = (int32_t)feistel(seed, t, (uint32_t)m, n_o, a);
+      continue;
+    }
+    uint64_t v = (uint64_t)a;
+    do {
+      uint32_t L = (uint32_t)(v >> h), R = (uint32_t)(v & mask);
+#pragma unroll
+      for (int r = 0; r < 6; ++r) {
+        const uint32_t nR = L ^ (ftab[(r << h) + R] & mask);
+        L = R;
+        R = nR;
+      }
+      v = ((uint64_t)L << h) | R;
+    } while ((int64_t)v >= n_o);
+    out[a] = (int32_t)v;
+  }
+}
+
 __global__ void k_perm(uint64_t seed, int32_t t, int32_t m, int64_t n_o, int64_t* out) {
   const int64_t a = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (a < n_o) out[a] = feistel(seed, (uint32_t)t, (uint32_t)m, n_o, a);
@@ -147,65 +203,128 @@ struct ImpArgs {
   double* oob_sum;
   int32_t* oob_cnt;
   double* e_t;
+  const int32_t* perm;  // pi_tm(a) of the batch (k_perm_fill), stride n per (tree, predictor)
 };
 
-__global__ void __launch_bounds__(NT) k_importance(ImpArgs g) {
-  extern __shared__ double sacc[];  // p partial sums of (e_tm - e_t) for this CTA's tree
-  __shared__ double serr[NT / 32];
+constexpr int IPT = 128;  // OOB rows per CTA (one thread each; their predictors staged in shared memory)
+constexpr int ILP = 4;    // permuted walks interleaved per thread
+
+// One CTA = IPT consecutive OOB positions a of one tree.  The rows' predictors
+// are staged row-major in shared memory (coalesced column loads of the
+// ascending OOB rows), so every walk reads x from shared memory and only the
+// node array (L2-resident: the CTAs of one tree run together) and the
+// permuted value x_{O_t[pi(a)], m} come from global memory.  The first
+// occurrences of each predictor on the original path are collected ILP at a
+// time and their re-walks run interleaved (independent dependency chains).
+__global__ void __launch_bounds__(IPT) k_importance(ImpArgs g) {
+  extern __shared__ double ism[];  // sacc[p] | x tile IPT x (p|1)
+  double* sacc = ism;
+  const int stride = g.p | 1;
+  double* sx = ism + ((g.p + 1) & ~1);
+  __shared__ double serr[IPT / 32];
   const int b = blockIdx.y;
   const int32_t i = g.i0 + b;
   const uint32_t t = (uint32_t)(g.tree_begin + i);
-  for (int m = threadIdx.x; m < g.p; m += NT) sacc[m] = 0.0;
-  __syncthreads();
   const int64_t n_o = g.nout[b];
-  const int64_t a = blockIdx.x * (int64_t)NT + threadIdx.x;
+  const int64_t a0 = (int64_t)blockIdx.x * IPT;
+  if (a0 >= n_o) return;  // uniform per CTA
+  for (int m = threadIdx.x; m < g.p; m += IPT) sacc[m] = 0.0;
+  const uint32_t* Ob = g.O + (int64_t)b * g.n;
+  const int64_t a = a0 + threadIdx.x;
+  const bool act = a < n_o;
+  const uint32_t r = act ? Ob[a] : Ob[a0];
+  {  // stage the tile: 16 column loads in flight per thread
+    double* xs = sx + threadIdx.x * stride;
+    for (int f0 = 0; f0 < g.p; f0 += 16) {
+      double v[16];
+#pragma unroll
+      for (int u = 0; u < 16; ++u) v[u] = (f0 + u < g.p) ? __ldg(g.X + (int64_t)(f0 + u) * g.ldx + r) : 0.0;
+#pragma unroll
+      for (int u = 0; u < 16; ++u)
+        if (f0 + u < g.p) xs[f0 + u] = v[u];
+    }
+  }
+  __syncthreads();
   double err0 = 0.0;
-  if (a < n_o) {
-    const uint32_t* Ob = g.O + (int64_t)b * g.n;
-    const uint32_t r = Ob[a];
+  if (act) {
+    const double* x = sx + threadIdx.x * stride;
     const Node16* tn = g.nodes + g.off[i];
     const double yr = g.y[r];
     // original walk
     Node16 nd = ld_node(tn);
-    while (nd.feature >= 0) nd = ld_node(tn + (g.X[(int64_t)nd.feature * g.ldx + r] <= nd.v ? nd.left : nd.left + 1));
+    while (nd.feature >= 0) nd = ld_node(tn + (x[nd.feature] <= nd.v ? nd.left : nd.left + 1));
     const double f0 = nd.v;
     const double d0 = yr - f0;
     err0 = d0 * d0;
     atomicAdd(&g.oob_sum[r], f0);
     atomicAdd(&g.oob_cnt[r], 1);
-    // permuted walks: first occurrence of each predictor on the path
+    // permuted walks from the first occurrence of each predictor on the path
     uint64_t seen = 0;
-    int k = 0;
-    nd = ld_node(tn);
     int depth = 0;
-    while (nd.feature >= 0) {
-      const int m = nd.feature;
-      bool first = !((seen >> (m & 63)) & 1ull);
-      if (!first && g.p > 64) {  // bitmask collision possible: verify on the path prefix
-        first = true;
-        int kk = 0;
-        for (int d = 0; d < depth; ++d) {
-          const Node16 q = ld_node(tn + kk);
-          if (q.feature == m) { first = false; break; }
-          kk = g.X[(int64_t)q.feature * g.ldx + r] <= q.v ? q.left : q.left + 1;
+    nd = ld_node(tn);
+    for (;;) {
+      int cnt = 0;
+      int qm[ILP];
+      Node16 q[ILP];
+      while (nd.feature >= 0 && cnt < ILP) {
+        const int m = nd.feature;
+        bool first = !((seen >> (m & 63)) & 1ull);
+        if (!first && g.p > 64) {  // bitmask collision possible: verify on the path prefix
+          first = true;
+          int kk = 0;
+          for (int d = 0; d < depth; ++d) {
+            const Node16 pq = ld_node(tn + kk);
+            if (pq.feature == m) {
+              first = false;
+              break;
+            }
+            kk = x[pq.feature] <= pq.v ? pq.left : pq.left + 1;
+          }
+        }
+        seen |= 1ull << (m & 63);
+        if (first) {
+#pragma unroll
+          for (int u = 0; u < ILP; ++u)
+            if (u == cnt) {
+              qm[u] = m;
+              q[u] = nd;
+            }
+          ++cnt;
+        }
+        nd = ld_node(tn + (x[m] <= nd.v ? nd.left : nd.left + 1));
+        ++depth;
+      }
+      if (cnt == 0) break;
+      double xm[ILP];
+#pragma unroll
+      for (int u = 0; u < ILP; ++u) {
+        if (u < cnt) {
+          const int64_t pa = __ldg(g.perm + ((int64_t)b * g.p + qm[u]) * g.n + a);
+          xm[u] = __ldg(g.X + (int64_t)qm[u] * g.ldx + Ob[pa]);
+        } else {
+          q[u].feature = -1;
+          qm[u] = -1;
+          xm[u] = 0.0;
         }
       }
-      seen |= 1ull << (m & 63);
-      if (first) {
-        const int64_t pa = feistel(g.seed, t, (uint32_t)m, n_o, a);
-        const double xm = g.X[(int64_t)m * g.ldx + Ob[pa]];
-        Node16 q = nd;
-        while (q.feature >= 0) {
-          const double xv = q.feature == m ? xm : g.X[(int64_t)q.feature * g.ldx + r];
-          q = ld_node(tn + (xv <= q.v ? q.left : q.left + 1));
-        }
-        const double d1 = yr - q.v;
-        const double diff = d1 * d1 - err0;
-        if (diff != 0.0) atomicAdd(&sacc[m], diff);
+      bool any = true;
+      while (any) {
+        any = false;
+#pragma unroll
+        for (int u = 0; u < ILP; ++u)
+          if (q[u].feature >= 0) {
+            const double xv = q[u].feature == qm[u] ? xm[u] : x[q[u].feature];
+            q[u] = ld_node(tn + (xv <= q[u].v ? q[u].left : q[u].left + 1));
+            any = true;
+          }
       }
-      k = g.X[(int64_t)m * g.ldx + r] <= nd.v ? nd.left : nd.left + 1;
-      nd = ld_node(tn + k);
-      ++depth;
+#pragma unroll
+      for (int u = 0; u < ILP; ++u)
+        if (u < cnt) {
+          const double d1 = yr - q[u].v;
+          const double diff = d1 * d1 - err0;
+          if (diff != 0.0) atomicAdd(&sacc[qm[u]], diff);
+        }
     }
   }
   // e_t
@@ -214,10 +333,10 @@ __global__ void __launch_bounds__(NT) k_importance(ImpArgs g) {
   __syncthreads();
   if (threadIdx.x == 0) {
     double s = 0.0;
-    for (int j = 0; j < NT / 32; ++j) s += serr[j];
+    for (int j = 0; j < IPT / 32; ++j) s += serr[j];
     if (s != 0.0) atomicAdd(&g.e_t[i], s);
   }
-  for (int m = threadIdx.x; m < g.p; m += NT)
+  for (int m = threadIdx.x; m < g.p; m += IPT)
     if (sacc[m] != 0.0) atomicAdd(&g.d_slots[(int64_t)i * g.p + m], sacc[m]);
 }
 
@@ -327,12 +446,16 @@ void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, co
   }
   BF_CUDA_CHECK(cudaMemsetAsync(oob_sum, 0, sizeof(double) * n, s));
   BF_CUDA_CHECK(cudaMemsetAsync(oob_cnt, 0, sizeof(int32_t) * n, s));
-  const int B = std::max(1, std::min<int>(T, 64));
+  // trees per batch: the batch's pi tables (B x p x n int32) stay under 1 GiB
+  const int B = (int)std::max<int64_t>(1, std::min<int64_t>({(int64_t)T, 64, ((int64_t)1 << 28) / std::max<int64_t>(1, (int64_t)p * n)}));
   const int nchunk = (int)ceil_div(n, OCH);
   DBuf<int32_t> w((size_t)B * n, s), cnt((size_t)B * nchunk, s);
   DBuf<uint32_t> O((size_t)B * n, s);
-  const size_t smem = sizeof(double) * (size_t)p;
-  if (smem > 48 * 1024) BF_REQUIRE(smem <= (size_t)dyn_smem_limit(k_importance), BF_ENOTIMPL, "p too large");
+  DBuf<int32_t> perm((size_t)B * p * n, s);
+  const size_t smem = sizeof(double) * ((size_t)((p + 1) & ~1) + (size_t)IPT * (size_t)(p | 1));
+  static int ismax = 0;
+  if (!ismax) ismax = dyn_smem_limit(k_importance);
+  BF_REQUIRE(smem <= (size_t)ismax, BF_ENOTIMPL, "bf_oob_importance: p too large for the shared-memory row tile");
   for (int32_t i0 = 0; i0 < T; i0 += B) {
     const int Bc = std::min(B, T - i0);
     bootstrap_impl(f->info.seed, f->info.tree_begin + i0, Bc, n, f->info.sampsize, f->info.replace, w.p, s);
@@ -352,6 +475,13 @@ void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, co
       KScope ks_("k_npur", s, 0.0);
       k_npur<<<dim3(64, Bc), NT, 0, s>>>(f->d_nodes, f->d_drss, f->d_tree_off, i0, p, npur);
     }
+    {
+      static int pfs = 0;
+      if (!pfs) pfs = dyn_smem_limit(k_perm_fill);
+      KScope ks_("k_perm_fill", s, 0.0);
+      k_perm_fill<<<dim3((unsigned)std::max<int64_t>(1, std::min<int64_t>(8, ceil_div(n, 65536))), p, Bc), 512,
+                    sizeof(uint32_t) * 6 * (1 << PH_MAX), s>>>(f->info.seed, f->info.tree_begin + i0, p, n, nout_t + i0, perm.p);
+    }
     BF_CUDA_CHECK(cudaGetLastError());
     ImpArgs g;
     g.nodes = f->d_nodes;
@@ -370,10 +500,11 @@ void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, co
     g.oob_sum = oob_sum;
     g.oob_cnt = oob_cnt;
     g.e_t = e_t;
+    g.perm = perm.p;
     // OOB rows per tree <= n; grid sized for n (CTAs past n_o exit early)
     {
       KScope ks_("k_importance", s, 0.0);
-      k_importance<<<dim3((unsigned)ceil_div(n, NT), Bc), NT, smem, s>>>(g);
+      k_importance<<<dim3((unsigned)ceil_div(n, IPT), Bc), IPT, smem, s>>>(g);
     }
     BF_CUDA_CHECK(cudaGetLastError());
   }

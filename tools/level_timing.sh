@@ -1,5 +1,5 @@
 # per-level timing of the global phase for one C4 batch of 20 trees (second fit; first is warm-up)
-timeout 300 python -c "
+BF_LEVEL_TIMING=1 BF_FIT_TIMING=1 timeout 300 python -c "
 import sys; sys.path.insert(0,'.')
 import torch, paper_conf_ipps_madougouvln16_b200 as bf
 from paper_conf_ipps_madougouvln16_b200 import synthetic as S
