@@ -1018,6 +1018,10 @@ __global__ void k_part_items_map(int N, int p, const LNode* nodes, const int32_t
 // with a running left count.
 struct PWork {
   int node, f0, g, unit;  // node index, first feature, features in the unit, unit index inside the feature
+  int a, nun;             // the node's entries per feature; units of the item
+  int64_t base;
+  int kl, al, kr, ar;     // children: kind and entries per feature
+  int64_t bl, br;         // children: block offsets
 };
 
 __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
@@ -1030,6 +1034,7 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
   __shared__ int32_t tpre[TPNT];                // per-thread exclusive prefix of lefts in the unit
   __shared__ uint32_t tmask[TPNT];              // per-thread left mask
   __shared__ int s_off[2];
+  __shared__ PWork s_w[2];
   const int tid = threadIdx.x;
   const TreeSched ts = tree_sched(g.B);
   if (tid == 0) {
@@ -1051,48 +1056,84 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
     // an owned item yields all its units in order (so the running left count stays inside one CTA)
     int jcur = g.ioff[n_lo] + ts.c;
     const int jend = g.ioff[n_hi];
-    int cur_nun = 0, cur_unit = 0;  // units left of the owned item being emitted
+    // thread 0 walks the items; the map entry of the next item is loaded one item ahead and its node /
+    // children records (and the map entry after it) are prefetched into L1, so taking an item costs L1 hits
+    auto pf = [&](const void* ptr) { asm volatile("prefetch.global.L1 [%0];" ::"l"(ptr)); };
+    auto pf_item = [&](int2 it) {
+      pf(g.nodes + it.x);
+      pf(g.child + 2 * it.x);
+    };
+    int2 nxt = make_int2(-1, 0);
+    if (tid == 0 && jcur < jend) {
+      nxt = g.imap[jcur];
+      pf_item(nxt);
+      if (jcur + ts.C < jend) pf(g.imap + jcur + ts.C);
+    }
     PWork cw;
+    cw.nun = 0;
+    int cur_unit = 0;  // next unit of the owned item being emitted
     auto next_mine = [&](PWork& w) -> bool {
-      if (cur_unit < cur_nun) {
+      if (cur_unit < cw.nun) {
         w = cw;
         w.unit = cur_unit++;
         return true;
       }
       if (jcur >= jend) return false;
-      const int2 it = g.imap[jcur];
+      const int2 it = nxt;
       jcur += ts.C;
-      const int a = g.nodes[it.x].a;
+      if (jcur < jend) {
+        nxt = g.imap[jcur];
+        pf_item(nxt);
+        if (jcur + ts.C < jend) pf(g.imap + jcur + ts.C);
+      }
+      const LNode nd = g.nodes[it.x];
+      const Child c0 = g.child[2 * it.x], c1 = g.child[2 * it.x + 1];
       cw.node = it.x;
       cw.f0 = it.y;
-      cw.g = min(part_group(a, g.p), g.p - it.y);
+      cw.a = nd.a;
+      cw.base = nd.base;
+      cw.g = min(part_group(nd.a, g.p), g.p - it.y);
+      cw.nun = cw.g > 1 ? 1 : (nd.a + TPUNIT - 1) / TPUNIT;
       cw.unit = 0;
-      cur_nun = cw.g > 1 ? 1 : (a + TPUNIT - 1) / TPUNIT;
+      cw.kl = c0.kind;
+      cw.al = c0.a;
+      cw.bl = c0.base;
+      cw.kr = c1.kind;
+      cw.ar = c1.a;
+      cw.br = c1.base;
       cur_unit = 1;
       w = cw;
       return true;
     };
     auto issue = [&](const PWork& w, int slot) {
-      const LNode nd = g.nodes[w.node];
       const int u0 = w.unit * TPUNIT;
-      const int cnt = w.g > 1 ? w.g * nd.a : min(TPUNIT, nd.a - u0);
+      const int cnt = w.g > 1 ? w.g * w.a : min(TPUNIT, w.a - u0);
       s_off[slot] = stage_entries(bufs + (size_t)slot * (TPUNIT + 2),
-                                  g.Ecur + nd.base + (int64_t)w.f0 * nd.a + (w.g > 1 ? 0 : u0), cnt, &bar[slot]);
+                                  g.Ecur + w.base + (int64_t)w.f0 * w.a + (w.g > 1 ? 0 : u0), cnt, &bar[slot]);
     };
-    PWork w, wn;
-    bool have = next_mine(w);
-    if (!have) continue;
-    if (tid == 0) issue(w, cur);
+    // thread 0 runs the item pipeline and publishes each unit's work record in s_w[slot] (slot = its buffer)
+    if (tid == 0) {
+      PWork w0;
+      if (!next_mine(w0)) w0.node = -1;
+      s_w[cur] = w0;
+      if (w0.node >= 0) issue(w0, cur);
+    }
+    __syncthreads();
+    if (s_w[cur].node < 0) continue;
     int64_t carry_l = 0;
-    while (have) {
-      const bool havn = next_mine(wn);
-      __syncthreads();
-      if (tid == 0 && havn) issue(wn, cur ^ 1);
-      const LNode nd = g.nodes[w.node];
-      const int a = nd.a;
+    for (;;) {
+      __syncthreads();  // the other buffer and s_w slot are free
+      const PWork w = s_w[cur];
+      if (w.node < 0) break;
+      if (tid == 0) {
+        PWork wn;
+        if (!next_mine(wn)) wn.node = -1;
+        s_w[cur ^ 1] = wn;
+        if (wn.node >= 0) issue(wn, cur ^ 1);
+      }
+      const int a = w.a;
       const int u0 = w.unit * TPUNIT;
       const int cnt = w.g > 1 ? w.g * a : min(TPUNIT, a - u0);
-      const Child cl = g.child[2 * w.node], cr = g.child[2 * w.node + 1];
       mbar_wait(&bar[cur], phase[cur]);
       phase[cur] ^= 1u;
       const uint64_t* buf = bufs + (size_t)cur * (TPUNIT + 2) + s_off[cur];
@@ -1118,7 +1159,7 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
         }
       int32_t tot;
       const int32_t lbl = block_excl_scan(c, sm, tot);
-      const int al = cl.a, ar = cr.a;  // lefts / rights per feature segment
+      const int al = w.al, ar = w.ar;  // lefts / rights per feature segment
       if (w.g > 1) {
         tpre[tid] = lbl;
         tmask[tid] = lmask;
@@ -1149,22 +1190,23 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
         }
       }
       __syncthreads();
-      const bool keepL = cl.kind == KIND_LARGE || cl.kind == KIND_SMALL;
-      const bool keepR = cr.kind == KIND_LARGE || cr.kind == KIND_SMALL;
+      const bool keepL = w.kl == KIND_LARGE || w.kl == KIND_SMALL;
+      const bool keepR = w.kr == KIND_LARGE || w.kr == KIND_SMALL;
       const int64_t exl = w.g > 1 ? 0 : carry_l, exr = w.g > 1 ? 0 : (int64_t)u0 - carry_l;
       const int nl_out = w.g > 1 ? w.g * al : tot, nr_out = cnt - nl_out;
       if (keepL) {
-        uint64_t* dl = (cl.kind == KIND_LARGE ? g.Enext : g.Esmall) + cl.base + (int64_t)w.f0 * al + exl;
+        uint64_t* dl = (w.kl == KIND_LARGE ? g.Enext : g.Esmall) + w.bl + (int64_t)w.f0 * al + exl;
         for (int i = tid; i < nl_out; i += TPNT) dl[i] = outb[i];
       }
       if (keepR) {
-        uint64_t* dr = (cr.kind == KIND_LARGE ? g.Enext : g.Esmall) + cr.base + (int64_t)w.f0 * ar + exr;
+        uint64_t* dr = (w.kr == KIND_LARGE ? g.Enext : g.Esmall) + w.br + (int64_t)w.f0 * ar + exr;
         for (int i = tid; i < nr_out; i += TPNT) dr[i] = outb[nl_out + i];
       }
       carry_l += tot;
-      if (!havn || wn.node != w.node || wn.f0 != w.f0) carry_l = 0;
-      w = wn;
-      have = havn;
+      {
+        const PWork& wn = s_w[cur ^ 1];  // published before this unit's block scan barriers
+        if (wn.node != w.node || wn.f0 != w.f0) carry_l = 0;
+      }
       cur ^= 1;
     }
   }
