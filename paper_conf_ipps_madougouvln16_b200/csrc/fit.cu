@@ -1805,6 +1805,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       warp_draw_mtry(g.seed, t, nd.key, p, g.mtry, mind, feats, lane);
       const long long c1_ = g.stats ? clock64() : 0;
       const int64_t nk = nd.n, Sk = nd.S;
+      const double nkd = (double)nk, Skd = (double)Sk;
       uint32_t* stg = temp;  // the medium levels' partition buffer (>= TGRP * TINY entries)
       const unsigned lt = (1u << lane) - 1u;
       // lane-local best over all (feature, boundary) items: key g, tie = (feature << 16 | rank)
@@ -1835,75 +1836,119 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
           if (v1) stg[u * an + __popc(m0) + __popc(m1 & lt)] = ev[2 * u + 1];
         }
         __syncwarp();
-        // dense passes over the ng*an (slot, position) items: segmented scans by slot,
-        // TPU passes at a time with their loads and shuffles interleaved
+        // the ng*an (slot, position) items, K consecutive ones per lane: (A) lane-serial sums of the lane's
+        // trailing slot run; one segmented warp scan of those runs; (B) lane-serial prefixes and cheap rigorous
+        // bounds gL <= g <= gU at every boundary; M = warp max of the lower bounds (and of the best exact key
+        // so far); (C) only lanes holding an item with gU >= M redo their items and take the exact S4.3 key.
         const int total = ng * an;
-        int32_t cw = 0;
-        int64_t cs = 0;
-        for (int i0 = 0; i0 < total; i0 += 32 * TPU) {
-          uint32_t e[TPU], en[TPU];
-          int32_t w[TPU];
-          int64_t wv[TPU];
-          int jj[TPU];
-#pragma unroll
-          for (int k = 0; k < TPU; ++k) {
-            const int i = i0 + 32 * k + lane;
-            const bool act = i < total;
-            const int sl = act ? i / an : ng;
-            jj[k] = act ? i - sl * an : 0;
-            e[k] = act ? stg[i] : 0u;
-            en[k] = (act && jj[k] + 1 < an) ? stg[i + 1] : 0u;
+        const int K = (total + 31) >> 5;
+        const int i0 = min(lane * K, total), i1 = min(i0 + K, total);
+        const int slot0 = i0 / an, jj0 = i0 - slot0 * an;
+        int32_t rw = 0;
+        int64_t rsum = 0;
+        bool hs = false;
+        {
+          int jj = jj0;
+#pragma unroll 4
+          for (int i = i0; i < i1; ++i) {
+            if (jj == 0) {
+              rw = 0;
+              rsum = 0;
+              hs = true;
+            }
+            const uint32_t lr = stg[i] & 0xffffu;
+            rw += wl[lr];
+            rsum += wy[lr];
+            if (++jj == an) jj = 0;
           }
-#pragma unroll
-          for (int k = 0; k < TPU; ++k) {
-            const bool act = i0 + 32 * k + lane < total;
-            const uint32_t lr = e[k] & 0xffffu;
-            w[k] = act ? wl[lr] : 0;
-            wv[k] = act ? wy[lr] : 0;
-          }
-          // inclusive segmented scans (segments are slot runs; lane-o is in my slot iff o <= j)
+        }
+        // segmented inclusive scan over lanes: (v, f) (+) (v', f') = (f' ? v' : v + v', f | f')
+        {
+          bool f = hs;
 #pragma unroll
           for (int o = 1; o < 32; o <<= 1) {
-#pragma unroll
-            for (int k = 0; k < TPU; ++k) {
-              const int32_t uw = __shfl_up_sync(0xffffffffu, w[k], o);
-              const int64_t uv = __shfl_up_sync(0xffffffffu, wv[k], o);
-              if (lane >= o && o <= jj[k]) {
-                w[k] += uw;
-                wv[k] += uv;
+            const int32_t uw = __shfl_up_sync(0xffffffffu, rw, o);
+            const int64_t us = __shfl_up_sync(0xffffffffu, rsum, o);
+            const bool uf = __shfl_up_sync(0xffffffffu, f, o);
+            if (lane >= o) {
+              if (!f) {
+                rw += uw;
+                rsum += us;
               }
+              f = f || uf;
             }
           }
-#pragma unroll
-          for (int k = 0; k < TPU; ++k) {
-            if (i0 + 32 * k >= total) break;
-            // my slot started before this pass (j > lane): add the previous pass's carry
-            if (jj[k] > lane) {
-              w[k] += cw;
-              wv[k] += cs;
+        }
+        int32_t cw0 = __shfl_up_sync(0xffffffffu, rw, 1);
+        int64_t cs0 = __shfl_up_sync(0xffffffffu, rsum, 1);
+        if (lane == 0 || jj0 == 0) {
+          cw0 = 0;
+          cs0 = 0;
+        }
+        double mL = lg, mU = -1.0;
+        {
+          int jj = jj0;
+          int32_t cw = cw0;
+          int64_t cs = cs0;
+#pragma unroll 2
+          for (int i = i0; i < i1; ++i) {
+            if (jj == 0) {
+              cw = 0;
+              cs = 0;
             }
-            const int32_t lw = __shfl_sync(0xffffffffu, w[k], 31);
-            const int64_t lv = __shfl_sync(0xffffffffu, wv[k], 31);
-            const int lj = __shfl_sync(0xffffffffu, jj[k], 31);
-            const bool cont = lj + 1 < an;  // last item's slot continues into the next pass
-            cw = cont ? lw : 0;
-            cs = cont ? lv : 0;
+            const uint32_t e = stg[i], lr = e & 0xffffu;
+            cw += wl[lr];
+            cs += wy[lr];
+            if (jj + 1 < an && (stg[i + 1] >> 16) != (e >> 16)) {
+              double gL, gU;
+              key_bounds(nkd, Skd, nk, cw, cs, gL, gU);
+              mL = fmax(mL, gL);
+              mU = fmax(mU, gU);
+            }
+            if (++jj == an) jj = 0;
           }
-#pragma unroll
-          for (int k = 0; k < TPU; ++k) {
-            const int i = i0 + 32 * k + lane;
-            if (i < total && jj[k] + 1 < an && (en[k] >> 16) != (e[k] >> 16) &&
-                screen_may_win(nk, Sk, w[k], wv[k], lg)) {
-              const double gk = split_key(nk, Sk, w[k], wv[k]);
-              const uint32_t tie = ((uint32_t)feats[s0 + i / an] << 16) | (e[k] >> 16);
-              if (gk > lg || (gk == lg && tie < ltie)) {
-                lg = gk;
-                ltie = tie;
-                lnl = w[k];
-                lSl = wv[k];
-                lra = e[k] & 0xffffu;
-                lrb = en[k] & 0xffffu;
+        }
+        double M;
+        {
+          const uint64_t kb = gkey(mL);
+          const uint32_t hi = __reduce_max_sync(0xffffffffu, (uint32_t)(kb >> 32));
+          const uint32_t lo = __reduce_max_sync(0xffffffffu, ((uint32_t)(kb >> 32) == hi) ? (uint32_t)kb : 0u);
+          M = (hi | lo) ? __longlong_as_double((long long)((((uint64_t)hi << 32) | lo) - 1ull)) : -1.0;
+        }
+        if (mU >= M && mU >= 0.0) {
+          int jj = jj0, sl = slot0;
+          int32_t cw = cw0;
+          int64_t cs = cs0;
+          for (int i = i0; i < i1; ++i) {
+            if (jj == 0) {
+              cw = 0;
+              cs = 0;
+            }
+            const uint32_t e = stg[i], lr = e & 0xffffu;
+            cw += wl[lr];
+            cs += wy[lr];
+            if (jj + 1 < an) {
+              const uint32_t en = stg[i + 1];
+              if ((en >> 16) != (e >> 16)) {
+                double gL, gU;
+                key_bounds(nkd, Skd, nk, cw, cs, gL, gU);
+                if (gU >= M) {
+                  const double gk = split_key(nk, Sk, cw, cs);
+                  const uint32_t tie = ((uint32_t)feats[s0 + sl] << 16) | (e >> 16);
+                  if (gk > lg || (gk == lg && tie < ltie)) {
+                    lg = gk;
+                    ltie = tie;
+                    lnl = cw;
+                    lSl = cs;
+                    lra = lr;
+                    lrb = en & 0xffffu;
+                  }
+                }
               }
+            }
+            if (++jj == an) {
+              jj = 0;
+              ++sl;
             }
           }
         }

@@ -6,7 +6,10 @@ os.environ["BF_FIT_TIMING"] = "1"
 import torch
 import paper_conf_ipps_madougouvln16_b200 as bf
 from paper_conf_ipps_madougouvln16_b200 import synthetic as S
-for cfg, T, As in [("C1", 500, [0]), ("C2", 100, [0, 128]), ("C4", 16, [0, 256, 128])]:
+CFGS = [("C1", 500, [0]), ("C2", 100, [0, 128]), ("C4", 16, [0, 256, 128])]
+if len(sys.argv) > 1 and sys.argv[1] == "c4":
+    CFGS = [("C4", 16, [0])]
+for cfg, T, As in CFGS:
     X, y, c = S.dataset(cfg)
     Xd, yd = torch.from_numpy(X).cuda(), torch.from_numpy(y).cuda()
     for A in As:
