@@ -1278,6 +1278,7 @@ __global__ void __launch_bounds__(NT) k_dest_bits(DestArgs g, uint32_t* sideb, i
 // list partition is needed.  Tiny nodes go through a CTA-wide work queue so
 // every warp stays busy until the whole subtree is grown.
 constexpr int TINY = 64;
+constexpr int HBITS = 12, HSLOTS = 1 << HBITS;  // load-phase hash table (global row -> local id), a0 <= 1024
 constexpr int TGRP = 7;   // drawn predictors staged per group in the tiny path
 constexpr int TPU = 4;    // scan passes interleaved in the tiny path
 
@@ -1315,6 +1316,7 @@ struct WRec {  // best candidate found by one warp for its share of a node's fea
 __host__ __device__ inline size_t align16(size_t x) { return (x + 15) & ~size_t(15); }
 __host__ __device__ inline int max_medium(int A) { return A / (TINY + 1) + 2; }
 __host__ __device__ inline int sub_temp(int A) { return A > TGRP * TINY ? A : TGRP * TINY; }
+static_assert(HSLOTS * 6 <= SUB_NW * TGRP * TINY * 4, "the load-phase hash table must fit the scratch area");
 
 __host__ __device__ inline size_t subtree_smem(int A, int p) {
   size_t s = 0;
@@ -1343,7 +1345,6 @@ struct SubArgs {
   int p, mtry, nodesize, q, A;
   uint64_t seed;
   int32_t t0;
-  uint16_t* loc;
   Pool pool;
   unsigned long long* stats;  // optional phase counters (BF_SUBTREE_STATS=1), else NULL
 };
@@ -1431,7 +1432,6 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   const int a0 = root.a;
   const int b = root.b;
   const uint32_t t = (uint32_t)(g.t0 + b);
-  uint16_t* loc = g.loc + (int64_t)b * g.n;
   const uint64_t* src = g.Es + root.base;
   int16_t* mind = mind_all + wid * p;
   int16_t* feats = feats_all + wid * p;
@@ -1441,21 +1441,83 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   int n_med = 0, n_tiny = 0;
   long long busy = 0;
 
-  // ---- load 1: local rows = feature 0's order; payload; global row -> local id
+  // ---- load 1: local rows = feature 0's order; payload; global row -> local id in a shared-memory hash
+  // table (open addressing over HSLOTS slots, built in the scratch area that the later phases reuse)
+  uint32_t* hkey = temp_all;
+  uint16_t* hval = (uint16_t*)(temp_all + HSLOTS);
+  for (int k = tid; k < HSLOTS; k += SUB_NT) hkey[k] = 0xffffffffu;
+  __syncthreads();
   for (int j = tid; j < a0; j += SUB_NT) {
     const uint64_t ej = src[j];
     const uint32_t row = e_row(ej);
     const int32_t wv = e_w(ej);
+    const int64_t yqr = g.yq[row];
+    const double yr = g.y[row];
     grow[j] = row;
-    loc[row] = (uint16_t)j;
+    uint32_t h = (row * 0x9E3779B1u) >> (32 - HBITS);
+    while (atomicCAS(&hkey[h], 0xffffffffu, row) != 0xffffffffu) h = (h + 1) & (HSLOTS - 1);
+    hval[h] = (uint16_t)j;
     wl[j] = wv;
-    wy[j] = (int64_t)wv * g.yq[row];
-    wyd[j] = __dmul_rn((double)wv, g.y[row]);
+    wy[j] = (int64_t)wv * yqr;
+    wyd[j] = __dmul_rn((double)wv, yr);
   }
   for (int j = tid; j <= a0; j += SUB_NT) tq[j].n = 0;
   __syncthreads();
+  auto hfind = [&](uint32_t row) -> uint16_t {
+    uint32_t h = (row * 0x9E3779B1u) >> (32 - HBITS);
+    while (hkey[h] != row) h = (h + 1) & (HSLOTS - 1);
+    return hval[h];
+  };
   // ---- load 2: warp per feature; local rank = index of the first entry of the same value
-  {
+  if (a0 <= 32 * 16) {  // K <= 16 consecutive entries per lane, all loads in flight; one warp max-scan per feature
+    const int K = (a0 + 31) >> 5;
+    const int j0 = lane * K, j1 = min(j0 + K, a0);
+    for (int f = wid; f < p; f += SUB_NW) {
+      const uint64_t* sf = src + (int64_t)f * a0;
+      uint32_t rk[16];
+      uint16_t lr[16];
+#pragma unroll
+      for (int q = 0; q < 16; ++q) {
+        const int j = j0 + q;
+        const uint64_t e = (q < K && j < j1) ? sf[j] : ~0ull;
+        rk[q] = e_rank(e);
+      }
+#pragma unroll
+      for (int q = 0; q < 16; ++q) {
+        const int j = j0 + q;
+        lr[q] = (q < K && j < j1) ? hfind(e_row(sf[j])) : 0;
+      }
+      // lane-local breaks: gs = j where the value changes, -1 = continues from the previous lane
+      uint32_t lastrk = 0xffffffffu;
+      int gl = -1;
+#pragma unroll
+      for (int q = 0; q < 16; ++q)
+        if (q < K && j0 + q < j1) {
+          lastrk = rk[q];
+          if (q > 0 && rk[q] != rk[q - 1]) gl = j0 + q;
+        }
+      const uint32_t prv = __shfl_up_sync(0xffffffffu, lastrk, 1);
+      const bool brk0 = j0 < j1 && (lane == 0 || rk[0] != prv);  // my first entry starts a value
+      int glast = gl >= 0 ? gl : (brk0 ? j0 : -1);
+      int inc = glast;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int v = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= o) inc = max(inc, v);
+      }
+      int cur = __shfl_up_sync(0xffffffffu, inc, 1);  // the last break before my entries
+      if (lane == 0) cur = 0;
+      uint32_t* lf = list + (size_t)f * a0;
+#pragma unroll
+      for (int q = 0; q < 16; ++q) {
+        const int j = j0 + q;
+        if (q < K && j < j1) {
+          if (q == 0 ? brk0 : rk[q] != rk[q - 1]) cur = j;
+          lf[j] = ((uint32_t)cur << 16) | lr[q];
+        }
+      }
+    }
+  } else {
     constexpr int GRP = 8;  // chunks of 32 entries in flight per warp
     const int nch = (a0 + 31) >> 5;
     for (int f = wid; f < p; f += SUB_NW) {
@@ -1470,7 +1532,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
           const int j = (c0 + c) * 32 + lane;
           const uint64_t e = j < a0 ? sf[j] : ~0ull;
           rk[c] = j < a0 ? e_rank(e) : 0xffffffffu;
-          lr[c] = j < a0 ? loc[e_row(e)] : 0;
+          lr[c] = j < a0 ? hfind(e_row(e)) : 0;
         }
 #pragma unroll
         for (int c = 0; c < GRP; ++c) {
@@ -1536,7 +1598,9 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   tclk[1] = clock64();
 
   // ================= medium levels (a > TINY): level-synchronous inside the CTA
+  long long mclk[3] = {0, 0, 0};  // medium phase: scan+finalize, next level, partition (thread 0, stats only)
   while (s_ncur > 0) {
+    const long long mc0 = clock64();
     const int ncur = s_ncur;
     n_med += ncur;
     int G = 1;
@@ -1555,40 +1619,80 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         int64_t bSl = 0;
         uint32_t bra = 0, brb = 0, brk = 0xffffffffu;
         const int64_t nk = nd.n, Sk = nd.S;
+        const double nkd = (double)nk, Skd = (double)Sk;
         for (int s = sub; s < g.mtry; s += G) {
           const int f = feats[s];
           const uint32_t* seg = list + (size_t)f * a0 + nd.lo;
-          int32_t cc = 0;
-          int64_t cs = 0;
           double lg = -1.0;
           uint32_t lrk = 0xffffffffu, lra = 0, lrb = 0;
           int lpos = -1, lnl = 0;
           int64_t lSl = 0;
-          for (int j0 = 0; j0 < nd.a; j0 += 32) {
-            const int j = j0 + lane;
-            const uint32_t e = j < nd.a ? seg[j] : 0u;
-            const uint32_t lr = e & 0xffffu;
-            const int32_t w = j < nd.a ? wl[lr] : 0;
-            const int64_t ws = j < nd.a ? wy[lr] : 0;
-            const int32_t ic = warp_incl_scan(w, lane) + cc;
-            const int64_t is = warp_incl_scan(ws, lane) + cs;
-            if (j + 1 < nd.a) {
-              const uint32_t en = seg[j + 1];
-              if ((en >> 16) != (e >> 16) && screen_may_win(nk, Sk, ic, is, lg)) {
-                const double gk = split_key(nk, Sk, ic, is);
-                if (rec_better(gk, e >> 16, lg, lrk)) {
-                  lg = gk;
-                  lrk = e >> 16;
-                  lra = lr;
-                  lrb = en & 0xffffu;
-                  lpos = j;
-                  lnl = ic;
-                  lSl = is;
+          // K consecutive entries per lane: lane-serial sums, one warp scan, a bounds pass screened by the
+          // warp max of the lower bounds (and the warp's best so far), exact keys only where they may win
+          const int aN = nd.a, K = (aN + 31) >> 5;
+          const int i0 = min(lane * K, aN), i1 = min(i0 + K, aN);
+          int32_t rw = 0;
+          int64_t rsum = 0;
+#pragma unroll 4
+          for (int i = i0; i < i1; ++i) {
+            const uint32_t lr = seg[i] & 0xffffu;
+            rw += wl[lr];
+            rsum += wy[lr];
+          }
+          const int32_t cw0 = warp_incl_scan(rw, lane) - rw;
+          const int64_t cs0 = warp_incl_scan(rsum, lane) - rsum;
+          double mL = -1.0, mU = -1.0;
+          {
+            int32_t cw = cw0;
+            int64_t cs = cs0;
+#pragma unroll 2
+            for (int i = i0; i < i1; ++i) {
+              const uint32_t e = seg[i], lr = e & 0xffffu;
+              cw += wl[lr];
+              cs += wy[lr];
+              if (i + 1 < aN && (seg[i + 1] >> 16) != (e >> 16)) {
+                double gL, gU;
+                key_bounds(nkd, Skd, nk, cw, cs, gL, gU);
+                mL = fmax(mL, gL);
+                mU = fmax(mU, gU);
+              }
+            }
+          }
+          double M;
+          {
+            const uint64_t kb = gkey(mL);
+            const uint32_t hi = __reduce_max_sync(0xffffffffu, (uint32_t)(kb >> 32));
+            const uint32_t lo = __reduce_max_sync(0xffffffffu, ((uint32_t)(kb >> 32) == hi) ? (uint32_t)kb : 0u);
+            M = (hi | lo) ? __longlong_as_double((long long)((((uint64_t)hi << 32) | lo) - 1ull)) : -1.0;
+            M = fmax(M, bg);
+          }
+          if (mU >= M && mU >= 0.0) {
+            int32_t cw = cw0;
+            int64_t cs = cs0;
+            for (int i = i0; i < i1; ++i) {
+              const uint32_t e = seg[i], lr = e & 0xffffu;
+              cw += wl[lr];
+              cs += wy[lr];
+              if (i + 1 < aN) {
+                const uint32_t en = seg[i + 1];
+                if ((en >> 16) != (e >> 16)) {
+                  double gL, gU;
+                  key_bounds(nkd, Skd, nk, cw, cs, gL, gU);
+                  if (gU >= M) {
+                    const double gk = split_key(nk, Sk, cw, cs);
+                    if (rec_better(gk, e >> 16, lg, lrk)) {
+                      lg = gk;
+                      lrk = e >> 16;
+                      lra = lr;
+                      lrb = en & 0xffffu;
+                      lpos = i;
+                      lnl = cw;
+                      lSl = cs;
+                    }
+                  }
                 }
               }
             }
-            cc = __shfl_sync(0xffffffffu, ic, 31);
-            cs = __shfl_sync(0xffffffffu, is, 31);
           }
           const int srcl = max(warp_argmax_key(gkey(lg), lrk), 0);
           lg = __shfl_sync(0xffffffffu, lg, srcl);
@@ -1685,6 +1789,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       }
       __syncthreads();
     }
+    const long long mc1 = clock64();
     // ---- next medium level (block scan) and tiny roots (work queue; processed after the medium levels)
     {
       int kc = 0;
@@ -1729,6 +1834,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       }
       if (tid == 0) s_ncur = totc;
     }
+    const long long mc2 = clock64();
     // ---- in-place stable partition of every feature row of every split node with a non-leaf child
     for (int it = wid; it < ncur * p; it += SUB_NW) {
       const int i = it / p, f = it - i * p;
@@ -1736,23 +1842,42 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       if (!nd.split || (nd.kind[0] == KIND_LEAF && nd.kind[1] == KIND_LEAF)) continue;
       uint32_t* seg = list + (size_t)f * a0 + nd.lo;
       const int al = nd.al;
+      const int aN = nd.a;
       int carry = 0;
-      for (int j0 = 0; j0 < nd.a; j0 += 32) {
-        const int j = j0 + lane;
-        const bool valid = j < nd.a;
-        const uint32_t e = valid ? seg[j] : 0u;
-        const int sdv = valid ? side[e & 0xffffu] : 1;
-        const unsigned m = __ballot_sync(0xffffffffu, valid && sdv == 0);
-        const int lb = carry + __popc(m & ((1u << lane) - 1u));
-        if (valid) temp[sdv ? al + (j - lb) : lb] = e;
-        carry += __popc(m);
+      for (int j0 = 0; j0 < aN; j0 += 128) {  // 4 rows of 32 with their loads in flight together
+        uint32_t e[4];
+        int sdv[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) e[u] = j0 + 32 * u + lane < aN ? seg[j0 + 32 * u + lane] : 0u;
+#pragma unroll
+        for (int u = 0; u < 4; ++u) sdv[u] = j0 + 32 * u + lane < aN ? side[e[u] & 0xffffu] : 1;
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const int j = j0 + 32 * u + lane;
+          const bool valid = j < aN;
+          const unsigned m = __ballot_sync(0xffffffffu, valid && sdv[u] == 0);
+          const int lb = carry + __popc(m & ((1u << lane) - 1u));
+          if (valid) temp[sdv[u] ? al + (j - lb) : lb] = e[u];
+          carry += __popc(m);
+        }
       }
       __syncwarp();
-      for (int j = lane; j < nd.a; j += 32) seg[j] = temp[j];
+      for (int j0 = 0; j0 < aN; j0 += 128) {
+        uint32_t v[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) v[u] = j0 + 32 * u + lane < aN ? temp[j0 + 32 * u + lane] : 0u;
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+          if (j0 + 32 * u + lane < aN) seg[j0 + 32 * u + lane] = v[u];
+      }
       __syncwarp();
     }
     __syncthreads();
     {
+      const long long mc3 = clock64();
+      mclk[0] += mc1 - mc0;
+      mclk[1] += mc2 - mc1;
+      mclk[2] += mc3 - mc2;
       MNode* tl = curl;
       curl = nxtl;
       nxtl = tl;
@@ -2084,6 +2209,9 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       atomicAdd(&g.stats[1], (unsigned long long)(tclk[2] - tclk[1]));
       atomicAdd(&g.stats[2], (unsigned long long)(tclk[3] - tclk[2]));
       atomicAdd(&g.stats[3], (unsigned long long)(tclk[4] - tclk[3]));
+      atomicAdd(&g.stats[13], (unsigned long long)mclk[0]);
+      atomicAdd(&g.stats[14], (unsigned long long)mclk[1]);
+      atomicAdd(&g.stats[15], (unsigned long long)mclk[2]);
       atomicAdd(&g.stats[4], (unsigned long long)n_med);
       atomicAdd(&g.stats[5], 1ull);
       atomicAdd(&g.stats[6], (unsigned long long)a0);
@@ -2373,7 +2501,6 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
     DBuf<int32_t> wmax(1, s);
     BF_CUDA_CHECK(cudaMemsetAsync(wmax.p, 0, sizeof(int32_t), s));
     DBuf<uint8_t> side((size_t)B * n, s);
-    DBuf<uint16_t> loc((size_t)B * n, s);
     DBuf<int32_t> pf((size_t)B * cap_nodes, s), pl((size_t)B * cap_nodes, s), pc((size_t)B * cap_nodes, s),
         pnn(B, s);
     DBuf<double> pt((size_t)B * cap_nodes, s), pv((size_t)B * cap_nodes, s), pd((size_t)B * cap_nodes, s);
@@ -2661,7 +2788,6 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
           ga.A = A;
           ga.seed = prm.seed;
           ga.t0 = tb;
-          ga.loc = loc.p;
           ga.pool = pool;
           ga.stats = nullptr;
           static const bool want_stats = getenv("BF_SUBTREE_STATS") != nullptr;
@@ -2681,6 +2807,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
             BF_CUDA_CHECK(cudaStreamSynchronize(s));
             const double c = (double)h[5];
             fprintf(stderr, "[subtree tiny] draw=%.0f groups=%.0f per tiny node\n", h[11] / (double)(h[7] ? h[7] : 1), h[12] / (double)(h[7] ? h[7] : 1));
+            fprintf(stderr, "[subtree medium] per cta: scan+finalize=%.0f next=%.0f partition=%.0f cycles\n", h[13] / (double)(h[5] ? h[5] : 1), h[14] / (double)(h[5] ? h[5] : 1), h[15] / (double)(h[5] ? h[5] : 1));
             fprintf(stderr, "[subtree] A=%d ctas=%llu mean_a0=%.1f cyc/cta: load=%.0f medium=%.0f tiny=%.0f flush=%.0f | medium nodes/cta=%.1f tiny nodes/cta=%.1f nodes/cta=%.1f warp-cyc in tiny/cta=%.0f busy=%.0f (%.0f per tiny node)\n",
                     A, h[5], h[6] / c, h[0] / c, h[1] / c, h[2] / c, h[3] / c, h[4] / c, h[7] / c, h[9] / c, h[8] / c,
                     h[10] / c, h[10] / (double)(h[7] ? h[7] : 1));
