@@ -1603,136 +1603,135 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
     const long long mc0 = clock64();
     const int ncur = s_ncur;
     n_med += ncur;
-    int G = 1;
-    while (G * 2 * ncur <= SUB_NW) G *= 2;
-    const int ngroups = SUB_NW / G, group = wid / G, sub = wid - group * G;
-    const int rounds = (ncur + ngroups - 1) / ngroups;
-    for (int rd = 0; rd < rounds; ++rd) {
-      const int i = rd * ngroups + group;
-      const bool active = i < ncur;
-      MNode nd;
-      if (active) {
-        nd = curl[i];
-        warp_draw_mtry(g.seed, t, nd.key, p, g.mtry, mind, feats, lane);
-        double bg = -1.0;
-        int bf = 0x7fffffff, bpos = -1, bnl = 0;
-        int64_t bSl = 0;
-        uint32_t bra = 0, brb = 0, brk = 0xffffffffu;
+    // (node, drawn predictor) items over all warps; per-item winners in the scratch area; one warp per node
+    // reduces its items (lowest predictor on equal keys) and finalizes the split.  Nodes go in groups whose
+    // items fit the scratch area (and whose draws fit the per-warp feature slots).
+    WRec* irec = (WRec*)temp_all;
+    const int cap_items = (int)((size_t)SUB_NW * sub_temp(A) * 4 / sizeof(WRec));
+    const int NG = max(1, min(SUB_NW, cap_items / g.mtry));
+    for (int n0 = 0; n0 < ncur; n0 += NG) {
+      const int nn = min(NG, ncur - n0);
+      if (wid < nn) warp_draw_mtry(g.seed, t, curl[n0 + wid].key, p, g.mtry, mind_all + wid * p, feats_all + wid * p, lane);
+      __syncthreads();
+      const int nit = nn * g.mtry;
+      for (int it = wid; it < nit; it += SUB_NW) {
+        const int li = it / g.mtry;
+        const MNode nd = curl[n0 + li];
+        const int f = feats_all[li * p + (it - li * g.mtry)];
+        const uint32_t* seg = list + (size_t)f * a0 + nd.lo;
         const int64_t nk = nd.n, Sk = nd.S;
         const double nkd = (double)nk, Skd = (double)Sk;
-        for (int s = sub; s < g.mtry; s += G) {
-          const int f = feats[s];
-          const uint32_t* seg = list + (size_t)f * a0 + nd.lo;
           double lg = -1.0;
-          uint32_t lrk = 0xffffffffu, lra = 0, lrb = 0;
-          int lpos = -1, lnl = 0;
-          int64_t lSl = 0;
-          // K consecutive entries per lane: lane-serial sums, one warp scan, a bounds pass screened by the
-          // warp max of the lower bounds (and the warp's best so far), exact keys only where they may win
-          const int aN = nd.a, K = (aN + 31) >> 5;
-          const int i0 = min(lane * K, aN), i1 = min(i0 + K, aN);
-          int32_t rw = 0;
-          int64_t rsum = 0;
+        uint32_t lrk = 0xffffffffu, lra = 0, lrb = 0;
+        int lpos = -1, lnl = 0;
+        int64_t lSl = 0;
+        // K consecutive entries per lane: lane-serial sums, one warp scan, a bounds pass screened by the
+        // warp max of the lower bounds (and the warp's best so far), exact keys only where they may win
+        const int aN = nd.a, K = (aN + 31) >> 5;
+        const int i0 = min(lane * K, aN), i1 = min(i0 + K, aN);
+        int32_t rw = 0;
+        int64_t rsum = 0;
 #pragma unroll 4
-          for (int i = i0; i < i1; ++i) {
-            const uint32_t lr = seg[i] & 0xffffu;
-            rw += wl[lr];
-            rsum += wy[lr];
-          }
-          const int32_t cw0 = warp_incl_scan(rw, lane) - rw;
-          const int64_t cs0 = warp_incl_scan(rsum, lane) - rsum;
-          double mL = -1.0, mU = -1.0;
-          {
-            int32_t cw = cw0;
-            int64_t cs = cs0;
+        for (int i = i0; i < i1; ++i) {
+          const uint32_t lr = seg[i] & 0xffffu;
+          rw += wl[lr];
+          rsum += wy[lr];
+        }
+        const int32_t cw0 = warp_incl_scan(rw, lane) - rw;
+        const int64_t cs0 = warp_incl_scan(rsum, lane) - rsum;
+        double mL = -1.0, mU = -1.0;
+        {
+          int32_t cw = cw0;
+          int64_t cs = cs0;
 #pragma unroll 2
-            for (int i = i0; i < i1; ++i) {
-              const uint32_t e = seg[i], lr = e & 0xffffu;
-              cw += wl[lr];
-              cs += wy[lr];
-              if (i + 1 < aN && (seg[i + 1] >> 16) != (e >> 16)) {
-                double gL, gU;
-                key_bounds(nkd, Skd, nk, cw, cs, gL, gU);
-                mL = fmax(mL, gL);
-                mU = fmax(mU, gU);
-              }
+          for (int i = i0; i < i1; ++i) {
+            const uint32_t e = seg[i], lr = e & 0xffffu;
+            cw += wl[lr];
+            cs += wy[lr];
+            if (i + 1 < aN && (seg[i + 1] >> 16) != (e >> 16)) {
+              double gL, gU;
+              key_bounds(nkd, Skd, nk, cw, cs, gL, gU);
+              mL = fmax(mL, gL);
+              mU = fmax(mU, gU);
             }
           }
-          double M;
-          {
-            const uint64_t kb = gkey(mL);
-            const uint32_t hi = __reduce_max_sync(0xffffffffu, (uint32_t)(kb >> 32));
-            const uint32_t lo = __reduce_max_sync(0xffffffffu, ((uint32_t)(kb >> 32) == hi) ? (uint32_t)kb : 0u);
-            M = (hi | lo) ? __longlong_as_double((long long)((((uint64_t)hi << 32) | lo) - 1ull)) : -1.0;
-            M = fmax(M, bg);
-          }
-          if (mU >= M && mU >= 0.0) {
-            int32_t cw = cw0;
-            int64_t cs = cs0;
-            for (int i = i0; i < i1; ++i) {
-              const uint32_t e = seg[i], lr = e & 0xffffu;
-              cw += wl[lr];
-              cs += wy[lr];
-              if (i + 1 < aN) {
-                const uint32_t en = seg[i + 1];
-                if ((en >> 16) != (e >> 16)) {
-                  double gL, gU;
-                  key_bounds(nkd, Skd, nk, cw, cs, gL, gU);
-                  if (gU >= M) {
-                    const double gk = split_key(nk, Sk, cw, cs);
-                    if (rec_better(gk, e >> 16, lg, lrk)) {
-                      lg = gk;
-                      lrk = e >> 16;
-                      lra = lr;
-                      lrb = en & 0xffffu;
-                      lpos = i;
-                      lnl = cw;
-                      lSl = cs;
-                    }
+        }
+        double M;
+        {
+          const uint64_t kb = gkey(mL);
+          const uint32_t hi = __reduce_max_sync(0xffffffffu, (uint32_t)(kb >> 32));
+          const uint32_t lo = __reduce_max_sync(0xffffffffu, ((uint32_t)(kb >> 32) == hi) ? (uint32_t)kb : 0u);
+          M = (hi | lo) ? __longlong_as_double((long long)((((uint64_t)hi << 32) | lo) - 1ull)) : -1.0;
+        }
+        if (mU >= M && mU >= 0.0) {
+          int32_t cw = cw0;
+          int64_t cs = cs0;
+          for (int i = i0; i < i1; ++i) {
+            const uint32_t e = seg[i], lr = e & 0xffffu;
+            cw += wl[lr];
+            cs += wy[lr];
+            if (i + 1 < aN) {
+              const uint32_t en = seg[i + 1];
+              if ((en >> 16) != (e >> 16)) {
+                double gL, gU;
+                key_bounds(nkd, Skd, nk, cw, cs, gL, gU);
+                if (gU >= M) {
+                  const double gk = split_key(nk, Sk, cw, cs);
+                  if (rec_better(gk, e >> 16, lg, lrk)) {
+                    lg = gk;
+                    lrk = e >> 16;
+                    lra = lr;
+                    lrb = en & 0xffffu;
+                    lpos = i;
+                    lnl = cw;
+                    lSl = cs;
                   }
                 }
               }
             }
           }
-          const int srcl = max(warp_argmax_key(gkey(lg), lrk), 0);
-          lg = __shfl_sync(0xffffffffu, lg, srcl);
-          lrk = __shfl_sync(0xffffffffu, lrk, srcl);
-          const int wpos = __shfl_sync(0xffffffffu, lpos, srcl);
-          const int wnl = __shfl_sync(0xffffffffu, lnl, srcl);
-          const int64_t wSl = __shfl_sync(0xffffffffu, lSl, srcl);
-          const uint32_t wra = __shfl_sync(0xffffffffu, lra, srcl);
-          const uint32_t wrb = __shfl_sync(0xffffffffu, lrb, srcl);
-          if (lg >= 0.0 && (lg > bg || (lg == bg && f < bf))) {
-            bg = lg;
-            bf = f;
-            brk = lrk;
-            bpos = wpos;
-            bnl = wnl;
-            bSl = wSl;
-            bra = wra;
-            brb = wrb;
-          }
         }
+        const int srcl = max(warp_argmax_key(gkey(lg), lrk), 0);
+        lg = __shfl_sync(0xffffffffu, lg, srcl);
+        lrk = __shfl_sync(0xffffffffu, lrk, srcl);
+        const int wpos = __shfl_sync(0xffffffffu, lpos, srcl);
+        const int wnl = __shfl_sync(0xffffffffu, lnl, srcl);
+        const int64_t wSl = __shfl_sync(0xffffffffu, lSl, srcl);
+        const uint32_t wra = __shfl_sync(0xffffffffu, lra, srcl);
+        const uint32_t wrb = __shfl_sync(0xffffffffu, lrb, srcl);
         if (lane == 0) {
           WRec r;
-          r.g = bg;
-          r.f = bf;
-          r.lrank = brk;
-          r.pos = bpos;
-          r.nl = bnl;
-          r.Sl = bSl;
-          r.ra = bra;
-          r.rb = brb;
-          wrec[wid] = r;
+          r.g = lg >= 0.0 ? lg : -1.0;
+          r.f = f;
+          r.lrank = lrk;
+          r.pos = wpos;
+          r.nl = wnl;
+          r.Sl = wSl;
+          r.ra = wra;
+          r.rb = wrb;
+          irec[it] = r;
         }
       }
       __syncthreads();
-      if (active && sub == 0) {
-        WRec best = wrec[wid];
-        for (int k = 1; k < G; ++k) {
-          const WRec r = wrec[wid + k];
-          if (r.g >= 0.0 && (r.g > best.g || (r.g == best.g && r.f < best.f))) best = r;
+      if (wid < nn) {
+        const int i = n0 + wid;
+        MNode nd = curl[i];
+        // the node's best item: lane-local over its items, then the warp (key desc, predictor asc)
+        double lgb = -1.0;
+        int lfb = 0x7fffffff, lsb = -1;
+        for (int s2 = lane; s2 < g.mtry; s2 += 32) {
+          const WRec& r = irec[wid * g.mtry + s2];
+          if (r.g >= 0.0 && (r.g > lgb || (r.g == lgb && r.f < lfb))) {
+            lgb = r.g;
+            lfb = r.f;
+            lsb = s2;
+          }
         }
+        const int wln = warp_argmax_key(gkey(lgb), (uint32_t)lfb);
+        const int sb = __shfl_sync(0xffffffffu, lsb, wln >= 0 ? wln : 0);
+        WRec best;
+        best.g = -1.0;
+        if (wln >= 0) best = irec[wid * g.mtry + sb];
         if (best.g > 0.0) {
           int lid = 0;
           if (lane == 0) {
