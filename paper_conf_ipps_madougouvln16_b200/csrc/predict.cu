@@ -1,12 +1,11 @@
 // predict.cu -- batched forest prediction (P:95 step 3, S5).
 //
 // One thread per query row; a CTA stages its rows' predictors in shared
-// memory row-major (coalesced column loads), then every thread walks the
-// trees of one tree block with PILP walks in flight (16-byte node loads
-// through the read-only path) and sums the leaf values in fp64.  All CTAs
-// walk the same block, so its nodes stay L2-resident.
+// memory row-major (coalesced column loads), then every thread walks all the
+// forest's trees in tree order (16-byte node loads through the read-only
+// path) and sums the leaf values in fp64.  All CTAs advance through the trees
+// in the same order, so the trees being walked at any moment stay L2-resident.
 #include <algorithm>
-#include <cstdlib>
 
 #include "bf_internal.cuh"
 
@@ -14,7 +13,7 @@ namespace bf {
 namespace {
 
 constexpr int PT = 128;   // rows per CTA
-constexpr int PILP = 12;  // trees walked concurrently by one thread
+constexpr int PILP = 8;  // trees walked concurrently by one thread
 
 __device__ __forceinline__ Node16 load_node(const Node16* p) {
   const int4 v = __ldg(reinterpret_cast<const int4*>(p));
@@ -26,7 +25,8 @@ __device__ __forceinline__ Node16 load_node(const Node16* p) {
 }
 
 // Trees [t_begin, t_end) of one tree block for every row; partial sums are
-// accumulated into yhat_sum (first block writes).
+// accumulated into yhat_sum (first block writes), so leaves are still added in
+// tree order.  A block of a few trees stays L2-resident while all rows walk it.
 __global__ void __launch_bounds__(PT) k_predict_smem(const Node16* __restrict__ nodes, const int64_t* __restrict__ off,
                                                      int32_t t_begin, int32_t t_end, int first, int last,
                                                      const double* __restrict__ Xq, int64_t ldq,
@@ -55,47 +55,33 @@ __global__ void __launch_bounds__(PT) k_predict_smem(const Node16* __restrict__ 
   const int64_t rr = r0 + threadIdx.x;
   double acc = first ? 0.0 : yhat_sum[rr];
   unsigned long long nv = 0;
-  // PILP independent walks in flight per thread: a slot that reaches a leaf adds
-  // its value and takes the block's next tree at once, so the dependency chains
-  // stay full until the last trees (leaf values are added in completion order;
-  // the sum is order-free up to rounding, R22)
-  int32_t tnext = t_begin;
-  const Node16* tn[PILP];
-  Node16 nd[PILP];
-#pragma unroll
-  for (int u = 0; u < PILP; ++u) {
-    if (tnext < t_end) {
-      tn[u] = nodes + off[tnext++];
-      nd[u] = load_node(tn[u]);
-      ++nv;
-    } else {
-      tn[u] = nodes;
-      nd[u].feature = -2;  // empty slot
-      nd[u].v = 0.0;
-      nd[u].left = 0;
-    }
-  }
-  bool any = true;
-  while (any) {
-    any = false;
+  // ILP trees walked together (independent dependency chains; the last group
+  // of a block is masked); leaf values are added in tree order, as in S5
+  for (int32_t t = t_begin; t < t_end; t += PILP) {
+    const int na = t_end - t < PILP ? t_end - t : PILP;
+    const Node16* tn[PILP];
+    Node16 nd[PILP];
 #pragma unroll
     for (int u = 0; u < PILP; ++u) {
-      if (nd[u].feature >= 0) {
-        nd[u] = load_node(tn[u] + (x[nd[u].feature] <= nd[u].v ? nd[u].left : nd[u].left + 1));
-        ++nv;
-        any = true;
-      } else if (nd[u].feature == -1) {
-        acc += nd[u].v;
-        if (tnext < t_end) {
-          tn[u] = nodes + off[tnext++];
-          nd[u] = load_node(tn[u]);
+      tn[u] = nodes + off[t + (u < na ? u : 0)];
+      nd[u] = load_node(tn[u]);
+      if (u >= na) nd[u].feature = -1;
+    }
+    nv += na;
+    bool any = true;
+    while (any) {
+      any = false;
+#pragma unroll
+      for (int u = 0; u < PILP; ++u)
+        if (nd[u].feature >= 0) {
+          nd[u] = load_node(tn[u] + (x[nd[u].feature] <= nd[u].v ? nd[u].left : nd[u].left + 1));
           ++nv;
           any = true;
-        } else {
-          nd[u].feature = -2;
         }
-      }
     }
+#pragma unroll
+    for (int u = 0; u < PILP; ++u)
+      if (u < na) acc += nd[u].v;
   }
   if (visits) atomicAdd(visits, nv);
   yhat_sum[rr] = acc;
@@ -152,11 +138,12 @@ void predict_impl(const bf_forest* f, const double* Xq_in, int64_t ldq, int64_t 
       ytmp.alloc(m, s);
       ysum = ytmp.p;
     }
-    static const int64_t block_bytes = (getenv("BF_PREDICT_BLOCK_MB") ? atoll(getenv("BF_PREDICT_BLOCK_MB")) : 64ll) << 20;
+    const int64_t block_bytes = 64ll << 20;
     int32_t t0 = 0;
     while (t0 < nt || (nt == 0 && t0 == 0)) {
       int32_t t1 = t0 + 1;
       while (t1 < nt && (f->tree_off[t1 + 1] - f->tree_off[t0]) * (int64_t)sizeof(Node16) <= block_bytes) ++t1;
+      if (t1 < nt && t1 - t0 > PILP) t1 = t0 + (t1 - t0) / PILP * PILP;  // whole ILP groups
       if (nt == 0) t1 = 0;
       {
         KScope ks_("k_predict_smem", s, 0.0);
