@@ -145,6 +145,25 @@ int bf_forest_import(const bf_forest_view* v, void* stream, bf_forest** out);
 int bf_predict(const bf_forest* f, const double* Xq, int64_t ldq, int64_t m,
                double* yhat_sum, double* yhat, int32_t ntree_total, void* stream);
 
+/* Partial dependence of the response on predictor m ("the partial
+ * dependence plot, shows how the response changes as a predictor ...
+ * change(s)"; readings R23, R24).  X: the n x p rows to
+ * average over (column-major, ldx >= n; normally the training data), grid:
+ * G values v_g of predictor m (host or device).
+ *   pd_sum[g] = sum_i sum_{held t} f_t(x_i with x_im := v_g)   (may be NULL)
+ *   pd[g]     = pd_sum[g] / (n * ntree_total)                  (may be NULL;
+ *               ntree_total <= 0 -> number of held trees)
+ * Multi-GPU: ranks holding disjoint tree ranges all-reduce pd_sum.         */
+int bf_partial_dependence(const bf_forest* f, const double* X, int64_t ldx, int64_t n, int32_t p, int32_t m,
+                          const double* grid, int32_t G, double* pd_sum, double* pd, int32_t ntree_total,
+                          void* stream);
+/* Default partial-dependence grid of a predictor column x (n values; reading
+ * R23 = R randomForest partialPlot): G = min(n_pt, distinct values of x),
+ * v_g = min + g * ((max - min) / (G - 1)) for g < G - 1, v_{G-1} = max
+ * (G = 1: v_0 = min).  grid must hold n_pt values; *G (host) receives G.
+ * Synchronous.                                                             */
+int bf_pd_grid(const double* x, int64_t n, int32_t n_pt, double* grid, int32_t* G, void* stream);
+
 /* OOB prediction + permutation importance over the forest's trees (P:130,
  * P:157; S6-S8).  X, y must be the training data of bf_fit.               */
 int bf_oob_importance(const bf_forest* f, const double* X, int64_t ldx, const double* y,
@@ -164,6 +183,19 @@ int bf_importance_finalize(const double* d_slots, const double* npur_slots, cons
  * may be NULL), scores (n x k column-major, may be NULL).                  */
 int bf_pca(const double* X, int64_t ldx, int64_t n, int32_t p, int32_t scale, int32_t k,
            double* sdev, double* rotation, double* center, double* scores, void* stream);
+
+/* Varimax rotation of factor loadings ("the factor loadings of the
+ * variable with relation to the retained principal components"; reading R25
+ * = R stats::varimax).  L: p x k column-major (ldl >= p), e.g. rotation[:, :k]
+ * scaled by sdev[:k].  normalize != 0: rows scaled to unit length before and
+ * back after (a zero row -> BF_EINVAL).  Iterates T <- U V^T of
+ * B = x^T (Z^3 - Z diag(colsum(Z^2))/p), Z = x T, until the sum of singular
+ * values d grows by less than a factor (1 + eps) [R: eps = 1e-5], at most 1000
+ * times.  Outputs: loadings (p x k, ld = p), rotmat (k x k), *iters (host,
+ * may be NULL).  1 <= k <= 32; 2 p k + p doubles must fit shared memory.
+ * Synchronous.                                                             */
+int bf_varimax(const double* L, int64_t ldl, int32_t p, int32_t k, int32_t normalize, double eps, double* loadings,
+               double* rotmat, int32_t* iters, void* stream);
 
 /* ---- single-step entry points (parity tests) ---- */
 /* Philox4x32-10 on `count` counters (S1): ctr[4*i..], out[4*i..].          */

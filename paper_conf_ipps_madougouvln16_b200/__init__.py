@@ -77,6 +77,9 @@ def lib():
             "bf_oob_importance": ([vp, vp, i64, vp, i64, i32, C.POINTER(Accum), vp], C.c_int),
             "bf_importance_finalize": ([vp] * 5 + [i64, i32, i32] + [vp] * 6 + [vp], C.c_int),
             "bf_pca": ([vp, i64, i64, i32, i32, i32, vp, vp, vp, vp, vp], C.c_int),
+            "bf_partial_dependence": ([vp, vp, i64, i64, i32, i32, vp, i32, vp, vp, i32, vp], C.c_int),
+            "bf_pd_grid": ([vp, i64, i32, vp, C.POINTER(C.c_int32), vp], C.c_int),
+            "bf_varimax": ([vp, i64, i32, i32, i32, C.c_double, vp, vp, C.POINTER(C.c_int32), vp], C.c_int),
             "bf_philox": ([vp, C.c_uint32, C.c_uint32, vp, i64, vp], C.c_int),
             "bf_i128_to_double": ([vp, vp, vp, i64, vp], C.c_int),
             "bf_fixed_point": ([vp, i64, i64, vp, C.POINTER(C.c_int32), vp], C.c_int),
@@ -100,7 +103,7 @@ def exported_symbols():
                         "bf_forest_info_get", "bf_forest_export", "bf_forest_import", "bf_predict",
                         "bf_oob_importance", "bf_importance_finalize", "bf_pca", "bf_philox", "bf_i128_to_double",
                         "bf_fixed_point", "bf_bootstrap", "bf_perm", "bf_profile_enable", "bf_profile_read",
-                        "bf_launch_count")]
+                        "bf_launch_count", "bf_partial_dependence", "bf_pd_grid", "bf_varimax")]
 
 
 class KernelStat(C.Structure):
@@ -217,6 +220,20 @@ class Forest:
         _check(lib().bf_predict(self._h, _ptr(Xq), m, m, _ptr(ys), _ptr(yh), ntree_total, _stream()), "bf_predict")
         return ys, yh
 
+    def partial_dependence(self, X, m: int, grid=None, n_pt: int = 51, ntree_total: int = 0):
+        """Partial dependence of the response on predictor m (bf_partial_dependence).
+        X: (p, n) rows to average over.  grid: G values (default bf_pd_grid of X[m], n_pt points).
+        Returns (grid, pd_sum, pd) on X's side (device tensors or numpy)."""
+        p, n = X.shape
+        if grid is None:
+            grid = pd_grid(X[m], n_pt)
+        G = int(grid.shape[0])
+        ps = _empty_like_dev(X, (G,), np.float64)
+        pd = _empty_like_dev(X, (G,), np.float64)
+        _check(lib().bf_partial_dependence(self._h, _ptr(X), n, n, p, m, _ptr(grid), G, _ptr(ps), _ptr(pd),
+                                           ntree_total, _stream()), "bf_partial_dependence")
+        return grid, ps, pd
+
     def oob_importance(self, X, y, out: dict | None = None) -> dict:
         p, n = X.shape
         inf = self.info
@@ -276,6 +293,29 @@ def importance_finalize(d_slots, npur_slots, oob_sum, oob_cnt, y) -> dict:
     outs["oob_mse"] = sc[0]
     outs["rsq"] = sc[1]
     return outs
+
+
+def pd_grid(x, n_pt: int = 51):
+    """Default partial-dependence grid of one predictor column (bf_pd_grid, reading R23)."""
+    n = int(x.shape[0])
+    buf = _empty_like_dev(x, (n_pt,), np.float64)
+    G = C.c_int32()
+    xx = x if (isinstance(x, np.ndarray) and x.flags.c_contiguous) or (not isinstance(x, np.ndarray) and x.is_contiguous()) \
+        else (np.ascontiguousarray(x) if isinstance(x, np.ndarray) else x.contiguous())
+    _check(lib().bf_pd_grid(_ptr(xx), n, n_pt, _ptr(buf), C.byref(G), _stream()), "bf_pd_grid")
+    return buf[: G.value]
+
+
+def varimax(L, normalize: bool = True, eps: float = 1e-5) -> dict:
+    """Varimax rotation of p x k loadings (bf_varimax, reading R25).  L: (k, p) array/tensor = column-major
+    p x k.  Returns loadings (k, p), rotmat (k, k) (column-major k x k as (k, k) row blocks) and iterations."""
+    k, p = L.shape
+    lo = _empty_like_dev(L, (k, p), np.float64)
+    ro = _empty_like_dev(L, (k, k), np.float64)
+    it = C.c_int32()
+    _check(lib().bf_varimax(_ptr(L), p, p, k, int(normalize), float(eps), _ptr(lo), _ptr(ro), C.byref(it),
+                            _stream()), "bf_varimax")
+    return {"loadings": lo, "rotmat": ro, "iters": int(it.value)}
 
 
 def pca(X, scale: bool = True, k: int | None = None) -> dict:

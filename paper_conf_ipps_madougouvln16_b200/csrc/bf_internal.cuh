@@ -224,6 +224,10 @@ void bootstrap_impl(uint64_t seed, int32_t t0, int32_t ntrees, int64_t n, int64_
 // predict.cu
 void predict_impl(const bf_forest* f, const double* Xq, int64_t ldq, int64_t m, double* yhat_sum, double* yhat,
                   int32_t ntree_total, cudaStream_t s);
+void pd_grid_impl(const double* x, int64_t n, int32_t n_pt, double* grid, int32_t* G_host, cudaStream_t s);
+void partial_dependence_impl(const bf_forest* f, const double* X, int64_t ldx, int64_t n, int32_t m,
+                             const double* grid, int32_t G, double* pd_sum, double* pd, int32_t ntree_total,
+                             cudaStream_t s);
 // importance.cu
 void oob_importance_impl(const bf_forest* f, const double* X, int64_t ldx, const double* y, int64_t n, int32_t p,
                          const bf_oob_accum& acc, cudaStream_t s);
@@ -234,6 +238,8 @@ void perm_impl(uint64_t seed, int32_t t, int32_t m, int64_t n_o, int64_t* out, c
 // pca.cu
 void pca_impl(const double* X, int64_t ldx, int64_t n, int32_t p, int32_t scale, int32_t k, double* sdev,
               double* rotation, double* center, double* scores, cudaStream_t s);
+void varimax_impl(const double* L, int64_t ldl, int32_t p, int32_t k, int32_t normalize, double eps, double* loadings,
+                  double* rotmat, int32_t* iters_host, cudaStream_t s);
 // misc kernels (capi.cu)
 void philox_impl(const uint32_t* ctr, uint32_t k0, uint32_t k1, uint32_t* out, int64_t count, cudaStream_t s);
 void i128_impl(const int64_t* hi, const uint64_t* lo, double* out, int64_t count, cudaStream_t s);

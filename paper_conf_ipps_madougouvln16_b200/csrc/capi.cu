@@ -290,6 +290,25 @@ int bf_predict(const bf_forest* f, const double* Xq, int64_t ldq, int64_t m, dou
   BF_API_END
 }
 
+int bf_pd_grid(const double* x, int64_t n, int32_t n_pt, double* grid, int32_t* G, void* stream) {
+  BF_API_BEGIN
+  BF_REQUIRE(x && grid && G, BF_EINVAL, "bf_pd_grid: NULL");
+  BF_REQUIRE(n >= 1 && n < (int64_t(1) << 31) && n_pt >= 1, BF_EINVAL, "bf_pd_grid: need 1 <= n < 2^31, n_pt >= 1");
+  pd_grid_impl(x, n, n_pt, grid, G, (cudaStream_t)stream);
+  BF_API_END
+}
+
+int bf_partial_dependence(const bf_forest* f, const double* X, int64_t ldx, int64_t n, int32_t p, int32_t m,
+                          const double* grid, int32_t G, double* pd_sum, double* pd, int32_t ntree_total,
+                          void* stream) {
+  BF_API_BEGIN
+  BF_REQUIRE(f && X && grid, BF_EINVAL, "bf_partial_dependence: NULL");
+  BF_REQUIRE(p == f->info.p && n >= 0 && ldx >= n && m >= 0 && m < p && G >= 1, BF_EINVAL,
+             "bf_partial_dependence: need p == forest p, ldx >= n, 0 <= m < p, G >= 1");
+  partial_dependence_impl(f, X, ldx, n, m, grid, G, pd_sum, pd, ntree_total, (cudaStream_t)stream);
+  BF_API_END
+}
+
 int bf_oob_importance(const bf_forest* f, const double* X, int64_t ldx, const double* y, int64_t n, int32_t p,
                       const bf_oob_accum* acc, void* stream) {
   BF_API_BEGIN
@@ -333,6 +352,16 @@ int bf_pca(const double* X, int64_t ldx, int64_t n, int32_t p, int32_t scale, in
   BF_REQUIRE(n >= 2 && p >= 1 && ldx >= n && k >= 0 && k <= p, BF_EINVAL, "bf_pca: bad sizes");
   BF_REQUIRE(p <= 1024, BF_ENOTIMPL, "bf_pca: p > 1024");
   pca_impl(X, ldx, n, p, scale, k, sdev, rotation, center, scores, (cudaStream_t)stream);
+  BF_API_END
+}
+
+int bf_varimax(const double* L, int64_t ldl, int32_t p, int32_t k, int32_t normalize, double eps, double* loadings,
+               double* rotmat, int32_t* iters, void* stream) {
+  BF_API_BEGIN
+  BF_REQUIRE(L && loadings && rotmat, BF_EINVAL, "bf_varimax: NULL");
+  BF_REQUIRE(p >= 1 && k >= 1 && k <= 32 && ldl >= p && eps >= 0.0, BF_EINVAL,
+             "bf_varimax: need p >= 1, 1 <= k <= 32, ldl >= p, eps >= 0");
+  varimax_impl(L, ldl, p, k, normalize, eps, loadings, rotmat, iters, (cudaStream_t)stream);
   BF_API_END
 }
 

@@ -1938,6 +1938,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       int32_t lnl = 0;
       int64_t lSl = 0;
       for (int s0 = 0; s0 < g.mtry; s0 += TGRP) {
+        const long long gqs = g.stats ? clock64() : 0;
         const int ng = min(TGRP, g.mtry - s0);
         // stage: the node's entries of each drawn feature, in value order, packed [slot][0..an).
         // All loads of the group are issued before any store (ILP across features).
@@ -1960,6 +1961,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
           if (v1) stg[u * an + __popc(m0) + __popc(m1 & lt)] = ev[2 * u + 1];
         }
         __syncwarp();
+        const long long gq0 = g.stats ? clock64() : 0;
         // the ng*an (slot, position) items, K consecutive ones per lane: (A) lane-serial sums of the lane's
         // trailing slot run; one segmented warp scan of those runs; (B) lane-serial prefixes and cheap rigorous
         // bounds gL <= g <= gU at every boundary; M = warp max of the lower bounds (and of the best exact key
@@ -1986,6 +1988,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
             if (++jj == an) jj = 0;
           }
         }
+        const long long gq1 = g.stats ? clock64() : 0;
         // segmented inclusive scan over lanes: (v, f) (+) (v', f') = (f' ? v' : v + v', f | f')
         {
           bool f = hs;
@@ -2009,6 +2012,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
           cw0 = 0;
           cs0 = 0;
         }
+        const long long gq2 = g.stats ? clock64() : 0;
         double mL = lg, mU = -1.0;
         {
           int jj = jj0;
@@ -2032,6 +2036,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
             if (++jj == an) jj = 0;
           }
         }
+        const long long gq3 = g.stats ? clock64() : 0;
         double M;
         {
           const uint64_t kb = gkey(mL);
@@ -2039,6 +2044,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
           const uint32_t lo = __reduce_max_sync(0xffffffffu, ((uint32_t)(kb >> 32) == hi) ? (uint32_t)kb : 0u);
           M = (hi | lo) ? __longlong_as_double((long long)((((uint64_t)hi << 32) | lo) - 1ull)) : -1.0;
         }
+        const long long gq4 = g.stats ? clock64() : 0;
         if (mU >= M && mU >= 0.0) {
           int jj = jj0, sl = slot0;
           int32_t cw = cw0;
@@ -2075,6 +2081,15 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
               ++sl;
             }
           }
+        }
+        if (g.stats && lane == 0) {
+          const long long gq5 = clock64();
+          atomicAdd(&g.stats[21], (unsigned long long)(gq0 - gqs));
+          atomicAdd(&g.stats[16], (unsigned long long)(gq1 - gq0));
+          atomicAdd(&g.stats[17], (unsigned long long)(gq2 - gq1));
+          atomicAdd(&g.stats[18], (unsigned long long)(gq3 - gq2));
+          atomicAdd(&g.stats[19], (unsigned long long)(gq4 - gq3));
+          atomicAdd(&g.stats[20], (unsigned long long)(gq5 - gq4));
         }
         __syncwarp();
       }
@@ -2792,8 +2807,8 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
           static const bool want_stats = getenv("BF_SUBTREE_STATS") != nullptr;
           DBuf<unsigned long long> st;
           if (want_stats) {
-            st.alloc(16, s);
-            BF_CUDA_CHECK(cudaMemsetAsync(st.p, 0, 16 * 8, s));
+            st.alloc(24, s);
+            BF_CUDA_CHECK(cudaMemsetAsync(st.p, 0, 24 * 8, s));
             ga.stats = st.p;
           }
           {
@@ -2801,11 +2816,12 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
             k_subtree<<<(unsigned)ls.nsmall, SUB_NT, subtree_smem(A, p), s>>>(ga);
           }
           if (want_stats) {
-            unsigned long long h[16];
-            d2h(h, st.p, 16, s);
+            unsigned long long h[24];
+            d2h(h, st.p, 24, s);
             BF_CUDA_CHECK(cudaStreamSynchronize(s));
             const double c = (double)h[5];
             fprintf(stderr, "[subtree tiny] draw=%.0f groups=%.0f per tiny node\n", h[11] / (double)(h[7] ? h[7] : 1), h[12] / (double)(h[7] ? h[7] : 1));
+            fprintf(stderr, "[subtree tiny group] per tiny node: stage=%.0f passA=%.0f segscan=%.0f passB=%.0f wmax=%.0f passC=%.0f\n", h[21] / (double)(h[7] ? h[7] : 1), h[16] / (double)(h[7] ? h[7] : 1), h[17] / (double)(h[7] ? h[7] : 1), h[18] / (double)(h[7] ? h[7] : 1), h[19] / (double)(h[7] ? h[7] : 1), h[20] / (double)(h[7] ? h[7] : 1));
             fprintf(stderr, "[subtree medium] per cta: scan+finalize=%.0f next=%.0f partition=%.0f cycles\n", h[13] / (double)(h[5] ? h[5] : 1), h[14] / (double)(h[5] ? h[5] : 1), h[15] / (double)(h[5] ? h[5] : 1));
             fprintf(stderr, "[subtree] A=%d ctas=%llu mean_a0=%.1f cyc/cta: load=%.0f medium=%.0f tiny=%.0f flush=%.0f | medium nodes/cta=%.1f tiny nodes/cta=%.1f nodes/cta=%.1f warp-cyc in tiny/cta=%.0f busy=%.0f (%.0f per tiny node)\n",
                     A, h[5], h[6] / c, h[0] / c, h[1] / c, h[2] / c, h[3] / c, h[4] / c, h[7] / c, h[9] / c, h[8] / c,

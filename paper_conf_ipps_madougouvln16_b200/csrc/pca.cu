@@ -250,7 +250,163 @@ __global__ void k_scores(const double* X, int64_t ldx, int64_t n, int p, int k, 
   scores[(int64_t)j * n + r] = s;
 }
 
+// ------------------------------------------------------------------ varimax (reading R25)
+// One CTA: x and Z = x T resident in shared memory (column-major, ld = p).  Per
+// iteration: Z = x T; c_j = sum_i Z_ij^2; B = x^T (Z^3 - Z diag(c) / p); the
+// polar factor T = U V^T of B by one-sided Jacobi (warp 0: lane i holds row i
+// of the working columns, cyclic sweeps until every column pair is orthogonal
+// to 1e-15); d = sum of singular values; stop when d < d_past (1 + eps).
+constexpr int VK = 32;  // largest k
+__device__ __forceinline__ double warp_sum_d(double v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+__global__ void k_varimax(const double* L, int64_t ldl, int p, int k, int normalize, double eps, int max_iter,
+                          double* load_o, double* rot_o, int32_t* iters_o, int* bad) {
+  extern __shared__ double vsm[];
+  double* x = vsm;                  // p x k
+  double* Z = x + (size_t)p * k;    // p x k
+  double* sc = Z + (size_t)p * k;   // p
+  __shared__ double T[VK * VK], B[VK * VK], A[VK * VK], Vm[VK * VK], cs[VK], sv[VK];
+  __shared__ double s_d;
+  __shared__ int s_stop, s_it;
+  const int tid = threadIdx.x, nt = blockDim.x, lane = tid & 31, wid = tid >> 5;
+  for (int e = tid; e < p * k; e += nt) x[e] = L[(int64_t)(e / p) * ldl + (e % p)];
+  __syncthreads();
+  if (normalize) {
+    for (int i = tid; i < p; i += nt) {
+      double s2 = 0.0;
+      for (int j = 0; j < k; ++j) s2 += x[i + p * j] * x[i + p * j];
+      sc[i] = sqrt(s2);
+      if (!(sc[i] > 0.0)) atomicExch(bad, 1);
+    }
+    __syncthreads();
+    for (int e = tid; e < p * k; e += nt) x[e] = x[e] / sc[e % p];
+  }
+  for (int e = tid; e < k * k; e += nt) T[e] = (e % k == e / k) ? 1.0 : 0.0;
+  if (tid == 0) {
+    s_d = 0.0;
+    s_stop = 0;
+    s_it = 0;
+  }
+  __syncthreads();
+  for (int it = 1; it <= max_iter && k >= 2; ++it) {
+    for (int e = tid; e < p * k; e += nt) {  // Z = x T
+      const int i = e % p, j = e / p;
+      double z = 0.0;
+      for (int l = 0; l < k; ++l) z += x[i + p * l] * T[l + k * j];
+      Z[e] = z;
+    }
+    __syncthreads();
+    for (int j = wid; j < k; j += nt / 32) {  // c_j = sum_i Z_ij^2
+      double c = 0.0;
+      for (int i = lane; i < p; i += 32) c += Z[i + p * j] * Z[i + p * j];
+      c = warp_sum_d(c);
+      if (lane == 0) cs[j] = c / p;
+    }
+    __syncthreads();
+    for (int e = tid; e < k * k; e += nt) {  // B = x^T (Z^3 - Z c / p)
+      const int a = e % k, b = e / k;
+      double v = 0.0;
+      for (int i = 0; i < p; ++i) {
+        const double z = Z[i + p * b];
+        v += x[i + p * a] * (z * z * z - z * cs[b]);
+      }
+      B[e] = v;
+      A[e] = v;
+      Vm[e] = (a == b) ? 1.0 : 0.0;
+    }
+    __syncthreads();
+    if (wid == 0) {  // one-sided Jacobi on the columns of A = B; Vm accumulates the rotations
+      for (int sweep = 0; sweep < 60; ++sweep) {
+        bool rotated = false;
+        for (int a = 0; a < k - 1; ++a)
+          for (int b = a + 1; b < k; ++b) {
+            const double ua = lane < k ? A[lane + k * a] : 0.0, ub = lane < k ? A[lane + k * b] : 0.0;
+            const double alpha = warp_sum_d(ua * ua), beta = warp_sum_d(ub * ub), gamma = warp_sum_d(ua * ub);
+            if (fabs(gamma) > 1e-15 * sqrt(alpha * beta) && gamma != 0.0) {
+              rotated = true;
+              const double zeta = (beta - alpha) / (2.0 * gamma);
+              const double t = (zeta >= 0.0 ? 1.0 : -1.0) / (fabs(zeta) + sqrt(1.0 + zeta * zeta));
+              const double c = 1.0 / sqrt(1.0 + t * t), sn = c * t;
+              if (lane < k) {
+                A[lane + k * a] = c * ua - sn * ub;
+                A[lane + k * b] = sn * ua + c * ub;
+                const double va = Vm[lane + k * a], vb = Vm[lane + k * b];
+                Vm[lane + k * a] = c * va - sn * vb;
+                Vm[lane + k * b] = sn * va + c * vb;
+              }
+            }
+            __syncwarp();
+          }
+        if (!rotated) break;
+      }
+      for (int j = 0; j < k; ++j) {  // singular values = column norms; U = A / s
+        const double u = lane < k ? A[lane + k * j] : 0.0;
+        const double sj = sqrt(warp_sum_d(u * u));
+        if (lane == 0) sv[j] = sj;
+        if (lane < k) A[lane + k * j] = sj > 0.0 ? u / sj : 0.0;
+      }
+      __syncwarp();
+    }
+    __syncthreads();
+    for (int e = tid; e < k * k; e += nt) {  // T = U V^T
+      const int a = e % k, b = e / k;
+      double v = 0.0;
+      for (int l = 0; l < k; ++l) v += A[a + k * l] * Vm[b + k * l];
+      T[e] = v;
+    }
+    if (tid == 0) {
+      double d = 0.0;
+      for (int j = 0; j < k; ++j) d += sv[j];
+      const double dp = s_d;
+      s_d = d;
+      s_it = it;
+      if (d < dp * (1.0 + eps)) s_stop = 1;
+    }
+    __syncthreads();
+    if (s_stop) break;
+  }
+  for (int e = tid; e < p * k; e += nt) {  // loadings = x T (rows scaled back)
+    const int i = e % p, j = e / p;
+    double z = 0.0;
+    for (int l = 0; l < k; ++l) z += x[i + p * l] * T[l + k * j];
+    load_o[e] = normalize ? z * sc[i] : z;
+  }
+  for (int e = tid; e < k * k; e += nt) rot_o[e] = T[e];
+  if (tid == 0 && iters_o) *iters_o = s_it;
+}
+
 }  // namespace
+
+void varimax_impl(const double* L_in, int64_t ldl, int32_t p, int32_t k, int32_t normalize, double eps,
+                  double* load_o, double* rot_o, int32_t* iters_host, cudaStream_t s) {
+  InStage Ls(L_in, sizeof(double) * (size_t)(ldl * (k - 1) + p), s);
+  OutStage lo(load_o, sizeof(double) * (size_t)p * k, s), ro(rot_o, sizeof(double) * (size_t)k * k, s);
+  DBuf<int32_t> it(1, s);
+  DBuf<int> bad(1, s);
+  BF_CUDA_CHECK(cudaMemsetAsync(bad.p, 0, sizeof(int), s));
+  const size_t smem = sizeof(double) * (2 * (size_t)p * k + p);
+  static int vmax = 0;
+  if (!vmax) vmax = dyn_smem_limit(k_varimax);
+  BF_REQUIRE(smem <= (size_t)vmax, BF_ENOTIMPL, "bf_varimax: p x k too large for shared memory");
+  {
+    KScope ks_("k_varimax", s, 0.0);
+    k_varimax<<<1, 256, smem, s>>>((const double*)Ls.dptr, ldl, p, k, normalize, eps, 1000, (double*)lo.dptr,
+                                   (double*)ro.dptr, it.p, bad.p);
+  }
+  BF_CUDA_CHECK(cudaGetLastError());
+  int hbad = 0;
+  int32_t hit = 0;
+  BF_CUDA_CHECK(cudaMemcpyAsync(&hbad, bad.p, sizeof(int), cudaMemcpyDeviceToHost, s));
+  BF_CUDA_CHECK(cudaMemcpyAsync(&hit, it.p, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+  lo.finish(s);
+  ro.finish(s);
+  BF_CUDA_CHECK(cudaStreamSynchronize(s));
+  BF_REQUIRE(!hbad, BF_EINVAL, "bf_varimax: a row of zero loadings cannot be normalised");
+  if (iters_host) *iters_host = hit;
+}
 
 void pca_impl(const double* X_in, int64_t ldx, int64_t n, int32_t p, int32_t scale, int32_t k, double* sdev_o,
               double* rot_o, double* center_o, double* scores_o, cudaStream_t s) {

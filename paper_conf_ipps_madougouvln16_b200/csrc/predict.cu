@@ -7,6 +7,8 @@
 // in the same order, so the trees being walked at any moment stay L2-resident.
 #include <algorithm>
 
+#include <cub/cub.cuh>
+
 #include "bf_internal.cuh"
 
 namespace bf {
@@ -111,7 +113,187 @@ __global__ void __launch_bounds__(PT) k_predict_gmem(const Node16* __restrict__ 
   if (yhat) yhat[r] = acc * inv_t;
 }
 
+// ------------------------------------------------------------------ partial dependence
+// P:130 ("the partial dependence plot, shows how the response changes as a
+// predictor ... change(s)"); readings R23 (grid) and R24 (definition):
+//   pd_sum[g] = sum_i sum_t f_t(x_i with x_im := v_g).
+// CTA = (tile of PT training rows, grid point g): the tile is staged like the
+// predict tile, column m is overwritten with v_g, the rows walk the tree
+// block (8 walks in flight per thread), the CTA reduces its rows' sums and
+// adds one value to pd_sum[g] (fp64 atomics: order-free up to rounding, R22).
+__global__ void __launch_bounds__(PT) k_pdep(const Node16* __restrict__ nodes, const int64_t* __restrict__ off,
+                                             int32_t t_begin, int32_t t_end, const double* __restrict__ X, int64_t ldx,
+                                             int64_t n, int p, int mcol, const double* __restrict__ grid,
+                                             double* pd_sum) {
+  extern __shared__ double sx[];
+  __shared__ double sred[PT / 32];
+  const int stride = p | 1;
+  const int64_t r0 = (int64_t)blockIdx.x * PT;
+  const int rows = (int)(n - r0 < PT ? n - r0 : PT);
+  const double vg = grid[blockIdx.y];
+  {
+    const int r = threadIdx.x;
+    const bool ok = r < rows;
+    const double* src = X + r0 + (ok ? r : 0);
+    for (int f0 = 0; f0 < p; f0 += 16) {
+      double v[16];
+#pragma unroll
+      for (int u = 0; u < 16; ++u) v[u] = (f0 + u < p) ? __ldg(src + (int64_t)(f0 + u) * ldx) : 0.0;
+#pragma unroll
+      for (int u = 0; u < 16; ++u)
+        if (f0 + u < p && ok) sx[r * stride + f0 + u] = (f0 + u == mcol) ? vg : v[u];
+    }
+  }
+  __syncthreads();
+  double acc = 0.0;
+  if ((int)threadIdx.x < rows) {
+    const double* x = sx + threadIdx.x * stride;
+    for (int32_t t = t_begin; t < t_end; t += PILP) {
+      const int na = t_end - t < PILP ? t_end - t : PILP;
+      const Node16* tn[PILP];
+      Node16 nd[PILP];
+#pragma unroll
+      for (int u = 0; u < PILP; ++u) {
+        tn[u] = nodes + off[t + (u < na ? u : 0)];
+        nd[u] = load_node(tn[u]);
+        if (u >= na) nd[u].feature = -1;
+      }
+      bool any = true;
+      while (any) {
+        any = false;
+#pragma unroll
+        for (int u = 0; u < PILP; ++u)
+          if (nd[u].feature >= 0) {
+            nd[u] = load_node(tn[u] + (x[nd[u].feature] <= nd[u].v ? nd[u].left : nd[u].left + 1));
+            any = true;
+          }
+      }
+#pragma unroll
+      for (int u = 0; u < PILP; ++u)
+        if (u < na) acc += nd[u].v;
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) acc += __shfl_down_sync(0xffffffffu, acc, o);
+  if ((threadIdx.x & 31) == 0) sred[threadIdx.x >> 5] = acc;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double tot = 0.0;
+    for (int w = 0; w < PT / 32; ++w) tot += sred[w];
+    atomicAdd(&pd_sum[blockIdx.y], tot);
+  }
+}
+
+__global__ void k_pdep_scale(const double* pd_sum, int G, double denom, double* pd) {
+  const int g = blockIdx.x * blockDim.x + threadIdx.x;
+  if (g < G) pd[g] = __ddiv_rn(pd_sum[g], denom);
+}
+
+// R23 grid: G = min(n_pt, distinct values of x); v_g = lo + g * ((hi - lo) / (G - 1)), v_{G-1} = hi.
+__global__ void k_sort_key_of(const double* x, int64_t n, uint64_t* keys) {
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  uint64_t b = (uint64_t)__double_as_longlong(__dadd_rn(x[i], 0.0));  // -0 -> +0 (R18)
+  keys[i] = (b >> 63) ? ~b : (b | 0x8000000000000000ull);               // order-preserving
+}
+__global__ void k_count_distinct(const uint64_t* keys, int64_t n, unsigned long long* cnt) {
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  const bool d = i < n && (i == 0 || keys[i] != keys[i - 1]);
+  const unsigned b = __ballot_sync(0xffffffffu, d);
+  if ((threadIdx.x & 31) == 0 && b) atomicAdd(cnt, (unsigned long long)__popc(b));
+}
+__device__ __forceinline__ double key_to_double(uint64_t k) {
+  const uint64_t b = (k >> 63) ? (k & 0x7fffffffffffffffull) : ~k;
+  return __longlong_as_double((long long)b);
+}
+__global__ void k_pd_grid(const uint64_t* sorted, int64_t n, const unsigned long long* cnt, int n_pt, double* grid,
+                          int32_t* G_out) {
+  const double lo = key_to_double(sorted[0]), hi = key_to_double(sorted[n - 1]);
+  const int G = (int)min((unsigned long long)n_pt, *cnt);
+  const double by = G > 1 ? __ddiv_rn(__dsub_rn(hi, lo), (double)(G - 1)) : 0.0;
+  for (int g = threadIdx.x; g < G; g += blockDim.x)
+    grid[g] = (g == G - 1 && G > 1) ? hi : __dadd_rn(lo, __dmul_rn((double)g, by));
+  if (threadIdx.x == 0) *G_out = G;
+}
+
 }  // namespace
+
+void pd_grid_impl(const double* x_in, int64_t n, int32_t n_pt, double* grid_in, int32_t* G_host, cudaStream_t s) {
+  InStage xs(x_in, sizeof(double) * (size_t)n, s);
+  OutStage gs(grid_in, sizeof(double) * (size_t)n_pt, s);
+  DBuf<uint64_t> keys(n, s), sorted(n, s);
+  DBuf<unsigned long long> cnt(1, s);
+  DBuf<int32_t> Gd(1, s);
+  BF_CUDA_CHECK(cudaMemsetAsync(cnt.p, 0, 8, s));
+  {
+    KScope ks_("k_sort_key_of", s, 0.0);
+    k_sort_key_of<<<(unsigned)ceil_div(n, 256), 256, 0, s>>>((const double*)xs.dptr, n, keys.p);
+  }
+  size_t tb = 0;
+  cub::DeviceRadixSort::SortKeys(nullptr, tb, keys.p, sorted.p, (int)n, 0, 64, s);
+  DBuf<char> tmp(std::max<size_t>(tb, 16), s);
+  {
+    KScope ks_("cub_SortKeys", s, 0.0);
+    BF_CUDA_CHECK(cub::DeviceRadixSort::SortKeys(tmp.p, tb, keys.p, sorted.p, (int)n, 0, 64, s));
+  }
+  {
+    KScope ks_("k_count_distinct", s, 0.0);
+    k_count_distinct<<<(unsigned)ceil_div(n, 256), 256, 0, s>>>(sorted.p, n, cnt.p);
+  }
+  {
+    KScope ks_("k_pd_grid", s, 0.0);
+    k_pd_grid<<<1, 64, 0, s>>>(sorted.p, n, cnt.p, n_pt, (double*)gs.dptr, Gd.p);
+  }
+  BF_CUDA_CHECK(cudaGetLastError());
+  BF_CUDA_CHECK(cudaMemcpyAsync(G_host, Gd.p, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+  gs.finish(s);
+  BF_CUDA_CHECK(cudaStreamSynchronize(s));
+}
+
+void partial_dependence_impl(const bf_forest* f, const double* X_in, int64_t ldx, int64_t n, int32_t mcol,
+                             const double* grid_in, int32_t G, double* pd_sum_in, double* pd_in, int32_t ntree_total,
+                             cudaStream_t s) {
+  const int p = f->info.p;
+  const int32_t nt = f->info.tree_end - f->info.tree_begin;
+  InStage Xs(X_in, sizeof(double) * (size_t)(ldx * (p - 1) + n), s);
+  InStage gs(grid_in, sizeof(double) * (size_t)G, s);
+  OutStage ps(pd_sum_in, pd_sum_in ? sizeof(double) * G : 0, s), pp(pd_in, pd_in ? sizeof(double) * G : 0, s);
+  DBuf<double> tmp_sum;
+  double* psum = pd_sum_in ? (double*)ps.dptr : nullptr;
+  if (!psum) {
+    tmp_sum.alloc(G, s);
+    psum = tmp_sum.p;
+  }
+  BF_CUDA_CHECK(cudaMemsetAsync(psum, 0, sizeof(double) * G, s));
+  const size_t smem = sizeof(double) * (size_t)PT * (size_t)(p | 1);
+  static int smax = 0;
+  if (!smax) smax = dyn_smem_limit(k_pdep);
+  BF_REQUIRE(smem <= (size_t)smax, BF_ENOTIMPL, "bf_partial_dependence: p too large for the shared-memory row tile");
+  if (n > 0 && nt > 0) {
+    const int64_t block_bytes = 64ll << 20;  // tree blocks L2-resident while every (row tile, g) walks them
+    int32_t t0 = 0;
+    while (t0 < nt) {
+      int32_t t1 = t0 + 1;
+      while (t1 < nt && (f->tree_off[t1 + 1] - f->tree_off[t0]) * (int64_t)sizeof(Node16) <= block_bytes) ++t1;
+      if (t1 < nt && t1 - t0 > PILP) t1 = t0 + (t1 - t0) / PILP * PILP;
+      {
+        KScope ks_("k_pdep", s, 0.0);
+        k_pdep<<<dim3((unsigned)ceil_div(n, PT), (unsigned)G), PT, smem, s>>>(
+            f->d_nodes, f->d_tree_off, t0, t1, (const double*)Xs.dptr, ldx, n, p, mcol, (const double*)gs.dptr, psum);
+      }
+      t0 = t1;
+    }
+  }
+  if (pd_in) {
+    const double denom = (double)n * (double)(ntree_total > 0 ? ntree_total : std::max(nt, 1));
+    KScope ks_("k_pdep_scale", s, 0.0);
+    k_pdep_scale<<<(unsigned)ceil_div(G, 128), 128, 0, s>>>(psum, G, denom, (double*)pp.dptr);
+  }
+  BF_CUDA_CHECK(cudaGetLastError());
+  if (pd_sum_in) ps.finish(s);
+  if (pd_in) pp.finish(s);
+  if (ps.host || pp.host || Xs.tmp.p || gs.tmp.p) BF_CUDA_CHECK(cudaStreamSynchronize(s));
+}
 
 void predict_impl(const bf_forest* f, const double* Xq_in, int64_t ldq, int64_t m, double* ys_in, double* yh_in,
                   int32_t ntree_total, cudaStream_t s) {
