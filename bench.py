@@ -318,7 +318,9 @@ def run_ours(args):
                 "avg_launch_ms": d["ms"] / max(d["launches"], 1)}
     kernels = {k: {"ms_per_step": v["ms"] / args.steps, "launches_per_step": v["launches"] / args.steps,
                    "GBps": (v["bytes"] / (v["ms"] / 1e3) / 1e9) if v["ms"] > 0 and v["bytes"] > 0 else None}
-               for k, v in sorted(stats.items(), key=lambda kv: -kv[1]["ms"])}
+               for k, v in sorted(stats.items(), key=lambda kv: -kv[1]["ms"]) if v["launches"] > 0}
+    vis = stats.get("predict_node_visits", {}).get("bytes", 0.0)
+    fbk = stats.get("predict_fp64_fallbacks", {}).get("bytes", 0.0)
     cpu = None
     if not args.no_cpu_baseline and world == 1:
         cpu = cpu_baseline(args, S, cfg, T, X, y)
@@ -331,6 +333,8 @@ def run_ours(args):
                    "m_query": m, "pca_k": k_pca, "parallelism": f"tree-sharded x{world}",
                    "l2": "inputs larger than L2 (X 512 MB, lists GBs); no flush"},
         "predictions_per_s": (m / (phase[1] / 1e3)) if m and phase[1] > 0 else None,
+        "predict_node_visits_per_walk": (vis / args.steps / (m * (t1 - t0))) if m and vis else None,
+        "predict_fp64_fallbacks_per_visit": (fbk / vis) if vis else None,
         "phases_ms": {"fit": phase[0], "predict": phase[1], "importance": phase[2], "pca": phase[3]},
         "gpu_launches": int(launches),
         "roofline": roof,

@@ -208,6 +208,11 @@ struct bf_forest {
   int32_t* d_count = nullptr;
   double* d_value = nullptr;
   double* d_drss = nullptr;
+  // Compact 8-byte traversal copy of d_nodes (predict.cu, built on first use):
+  // 0 not built, 1 built, -1 not representable (p > 256, >= 2^31 nodes, or a child stored before its parent).
+  uint2* d_nodes8 = nullptr;
+  uint32_t* d_roots8 = nullptr;  // per tree: global root id | 1<<31 if the tree is a single leaf
+  int nodes8_state = 0;
   int device = 0;
 };
 
@@ -222,6 +227,7 @@ void fixed_point_impl(const double* y, int64_t n, int64_t sampsize, int64_t* yq,
 void bootstrap_impl(uint64_t seed, int32_t t0, int32_t ntrees, int64_t n, int64_t sampsize, int32_t replace,
                     int32_t* w, cudaStream_t s);
 // predict.cu
+const uint2* nodes8_get(bf_forest* f, cudaStream_t s);  // NULL if not representable
 void predict_impl(const bf_forest* f, const double* Xq, int64_t ldq, int64_t m, double* yhat_sum, double* yhat,
                   int32_t ntree_total, cudaStream_t s);
 void pd_grid_impl(const double* x, int64_t n, int32_t n_pt, double* grid, int32_t* G_host, cudaStream_t s);

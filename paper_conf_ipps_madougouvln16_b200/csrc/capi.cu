@@ -106,6 +106,11 @@ void forest_release(bf_forest* f) {
   dev_free(f->d_value, s);
   dev_free(f->d_drss, s);
   dev_free(f->d_tree_off, s);
+  if (f->d_nodes8) dev_free(f->d_nodes8, s);
+  if (f->d_roots8) dev_free(f->d_roots8, s);
+  f->d_nodes8 = nullptr;
+  f->d_roots8 = nullptr;
+  f->nodes8_state = 0;
   f->d_nodes = nullptr;
 }
 
@@ -284,7 +289,7 @@ int bf_forest_import(const bf_forest_view* v, void* stream, bf_forest** out) {
 int bf_predict(const bf_forest* f, const double* Xq, int64_t ldq, int64_t m, double* yhat_sum, double* yhat,
                int32_t ntree_total, void* stream) {
   BF_API_BEGIN
-  BF_REQUIRE(f && Xq, BF_EINVAL, "bf_predict: NULL");
+  BF_REQUIRE(f && (Xq || m == 0), BF_EINVAL, "bf_predict: NULL");
   BF_REQUIRE(m >= 0 && ldq >= m, BF_EINVAL, "bf_predict: need m >= 0, ldq >= m");
   predict_impl(f, Xq, ldq, m, yhat_sum, yhat, ntree_total, (cudaStream_t)stream);
   BF_API_END

@@ -6,6 +6,7 @@
 // path) and sums the leaf values in fp64.  All CTAs advance through the trees
 // in the same order, so the trees being walked at any moment stay L2-resident.
 #include <algorithm>
+#include <cstdlib>
 
 #include <cub/cub.cuh>
 
@@ -85,7 +86,152 @@ __global__ void __launch_bounds__(PT) k_predict_smem(const Node16* __restrict__ 
     for (int u = 0; u < PILP; ++u)
       if (u < na) acc += nd[u].v;
   }
-  if (visits) atomicAdd(visits, nv);
+  if (visits) {  // one atomic per warp
+    const unsigned act = __activemask();
+    const unsigned long long wv = __reduce_add_sync(act, (uint32_t)nv);
+    if ((threadIdx.x & 31) == __ffs(act) - 1) atomicAdd(visits, wv);
+  }
+  yhat_sum[rr] = acc;
+  if (last && yhat) yhat[rr] = acc * inv_t;
+}
+
+// ------------------------------------------------------------------ compact 8-byte traversal nodes
+// Node8 (built once per forest from Node16 by k_pack8):
+//   internal: word0 = float bits of RN_f32(thr); word1 = LL<<31 | RL<<30 | feature<<22 | rel
+//             (LL/RL: the left/right child is a leaf; rel = left child's id - this node's id >= 1, so the
+//             children of global node g are g + rel and g + rel + 1)
+//   leaf:     the 8 bytes are the fp64 leaf value (a walk lands on a leaf only through its parent's LL/RL
+//             bit, or at the root of a single-node tree, flagged in the tree's root word).
+// The comparison x <= thr of S5 is decided on floats where that is exact: rounding to float is monotone, so
+// RN_f32(x) < RN_f32(thr) implies x < thr and RN_f32(x) > RN_f32(thr) implies x > thr; only
+// RN_f32(x) == RN_f32(thr) (or NaN) falls back to the fp64 x (global X) and the fp64 thr (Node16).  The walk
+// therefore takes exactly the S5 path, with half the node bytes and half the shared-memory row tile.
+constexpr int N8_FEAT_BITS = 8, N8_REL_BITS = 22;
+constexpr uint32_t ROOT_LEAF = 0x80000000u;  // roots8[t] = global root id | ROOT_LEAF for single-node trees
+
+__global__ void k_pack8(const Node16* __restrict__ nodes, const int64_t* __restrict__ off, uint2* __restrict__ out,
+                        uint32_t* __restrict__ roots, int* __restrict__ bad) {
+  const int32_t t = blockIdx.y;
+  const int64_t lo = off[t], hi = off[t + 1];
+  if (blockIdx.x == 0 && threadIdx.x == 0) roots[t] = (uint32_t)lo | (hi - lo == 1 ? ROOT_LEAF : 0u);
+  for (int64_t k = lo + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < hi; k += (int64_t)gridDim.x * blockDim.x) {
+    const Node16 nd = nodes[k];
+    uint2 o;
+    if (nd.feature < 0) {
+      const unsigned long long b = (unsigned long long)__double_as_longlong(nd.v);
+      o.x = (uint32_t)b;
+      o.y = (uint32_t)(b >> 32);
+    } else {
+      const int64_t rel = (int64_t)nd.left - (k - lo);
+      if (rel < 1 || rel >= (1ll << N8_REL_BITS) || lo + nd.left + 1 >= hi) {
+        *bad = 1;  // children not after their parent: the forest keeps the Node16 path
+        o = make_uint2(0u, 0u);
+      } else {
+        const uint32_t ll = nodes[lo + nd.left].feature < 0, rl = nodes[lo + nd.left + 1].feature < 0;
+        o.x = __float_as_uint(__double2float_rn(nd.v));
+        o.y = (ll << 31) | (rl << 30) | ((uint32_t)nd.feature << N8_REL_BITS) | (uint32_t)rel;
+      }
+    }
+    out[k] = o;
+  }
+}
+
+__device__ __forceinline__ double leaf8(uint2 v) { return __hiloint2double((int)v.y, (int)v.x); }
+
+constexpr int PT8 = 128;  // rows per CTA
+constexpr int S8 = 8;     // walks in flight per thread (a finished slot restarts with the block's next tree;
+                          // measured: 12 or 16 slots lower occupancy and run slower)
+
+// Trees [t_begin, t_end) of one tree block for every row of the CTA's tile (a block is a few trees that stay
+// L2-resident while all CTAs walk it).  Each thread keeps S8 walks in flight, a slot being (global node id,
+// node word); a slot that reaches a leaf adds the value and restarts at the block's next tree (a fixed order
+// per row: deterministic sums).  PROF counts node loads and fp64 fallbacks (profile mode only).
+template <bool PROF>
+__global__ void __launch_bounds__(PT8, 6) k_predict8(const uint2* __restrict__ nodes8, const Node16* __restrict__ nodes16,
+                                                     const uint32_t* __restrict__ roots, int32_t t_begin, int32_t t_end,
+                                                     int first, int last, const double* __restrict__ Xq, int64_t ldq,
+                                                     int64_t m, int p, double* yhat_sum, double* yhat, double inv_t,
+                                                     unsigned long long* visits) {
+  extern __shared__ float sxf[];  // PT8 x (p|1), row-major
+  const int stride = p | 1;
+  const int64_t r0 = (int64_t)blockIdx.x * PT8;
+  const int rows = (int)(m - r0 < PT8 ? m - r0 : PT8);
+  {  // stage the tile as floats: 8 column loads in flight per thread
+    const int r = threadIdx.x;
+    const bool ok = r < rows;
+    const double* src = Xq + r0 + (ok ? r : 0);
+    for (int f0 = 0; f0 < p; f0 += 8) {
+      double v[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) v[u] = (f0 + u < p) ? __ldcs(src + (int64_t)(f0 + u) * ldq) : 0.0;
+#pragma unroll
+      for (int u = 0; u < 8; ++u)
+        if (f0 + u < p && ok) sxf[r * stride + f0 + u] = __double2float_rn(v[u]);
+    }
+  }
+  __syncthreads();
+  if ((int)threadIdx.x >= rows) return;
+  const float* xs = sxf + threadIdx.x * stride;
+  const int64_t rr = r0 + threadIdx.x;
+  const double* xg = Xq + rr;
+  double acc = first ? 0.0 : yhat_sum[rr];
+  uint32_t nv = 0, nfb = 0;
+  uint32_t gid[S8];  // global node id of the slot's current node; ~0u = idle
+  uint2 nd[S8];
+  int32_t tnext = t_begin;
+  // next non-trivial tree of the block into slot u (single-node trees add their value at once)
+  auto start = [&](int u) {
+    gid[u] = ~0u;
+    while (tnext < t_end) {
+      const uint32_t rw = __ldg(roots + tnext++);
+      const uint2 rn = __ldg(nodes8 + (rw & ~ROOT_LEAF));
+      if (PROF) ++nv;
+      if (rw & ROOT_LEAF) {
+        acc += leaf8(rn);
+        continue;
+      }
+      gid[u] = rw;
+      nd[u] = rn;
+      break;
+    }
+  };
+#pragma unroll
+  for (int u = 0; u < S8; ++u) start(u);
+  bool any = true;
+  while (any) {
+    any = false;
+#pragma unroll
+    for (int u = 0; u < S8; ++u) {
+      if (gid[u] == ~0u) continue;
+      any = true;
+      const uint2 w = nd[u];
+      const uint32_t f = (w.y >> N8_REL_BITS) & ((1u << N8_FEAT_BITS) - 1u);
+      const float xf = xs[f], tf = __uint_as_float(w.x);
+      uint32_t right = xf > tf;
+      if (xf == tf || xf != xf) {  // float tie (or NaN): decide in fp64 (S5)
+        right = !(__ldg(xg + (int64_t)f * ldq) <= __ldg(&nodes16[gid[u]].v));
+        if (PROF) ++nfb;
+      }
+      const uint32_t c = gid[u] + (w.y & ((1u << N8_REL_BITS) - 1u)) + right;
+      const uint2 ch = __ldg(nodes8 + c);
+      if (PROF) ++nv;
+      if ((w.y >> (31 - right)) & 1u) {
+        acc += leaf8(ch);
+        start(u);
+      } else {
+        gid[u] = c;
+        nd[u] = ch;
+      }
+    }
+  }
+  if (PROF) {  // one atomic per warp (per-thread atomics on one address would serialise in L2)
+    const unsigned act = __activemask();
+    const uint32_t wv = __reduce_add_sync(act, nv), wf = __reduce_add_sync(act, nfb);
+    if ((threadIdx.x & 31) == __ffs(act) - 1) {
+      atomicAdd(visits, (unsigned long long)wv);
+      atomicAdd(visits + 1, (unsigned long long)wf);
+    }
+  }
   yhat_sum[rr] = acc;
   if (last && yhat) yhat[rr] = acc * inv_t;
 }
@@ -108,7 +254,11 @@ __global__ void __launch_bounds__(PT) k_predict_gmem(const Node16* __restrict__ 
     }
     acc += nd.v;
   }
-  if (visits) atomicAdd(visits, nv);
+  if (visits) {  // one atomic per warp
+    const unsigned act = __activemask();
+    const unsigned long long wv = __reduce_add_sync(act, (uint32_t)nv);
+    if ((threadIdx.x & 31) == __ffs(act) - 1) atomicAdd(visits, wv);
+  }
   if (yhat_sum) yhat_sum[r] = acc;
   if (yhat) yhat[r] = acc * inv_t;
 }
@@ -295,6 +445,48 @@ void partial_dependence_impl(const bf_forest* f, const double* X_in, int64_t ldx
   if (ps.host || pp.host || Xs.tmp.p || gs.tmp.p) BF_CUDA_CHECK(cudaStreamSynchronize(s));
 }
 
+// Bytes of nodes per tree block (L2-resident while every row walks the block); BF_PREDICT_BLOCK_BYTES
+// overrides it (tests force many blocks on small forests).
+// Defaults measured on the C4 forest with a 10M-row batch (tools/predict_exp.py): 32 MB of Node8, 48 MB of
+// Node16 (larger blocks start to miss in L2, smaller ones re-stage the row tiles too often).
+static int64_t predict_block_bytes(int64_t dflt) {
+  const char* e = getenv("BF_PREDICT_BLOCK_BYTES");
+  const long long v = e ? atoll(e) : 0;
+  return v > 0 ? (int64_t)v : dflt;
+}
+
+const uint2* nodes8_get(bf_forest* f, cudaStream_t s) {
+  if (f->nodes8_state == 0) {
+    const int32_t nt = f->info.tree_end - f->info.tree_begin;
+    const bool ok = f->info.p <= (1 << N8_FEAT_BITS) && f->info.total_nodes > 0 && nt > 0 &&
+                    f->info.total_nodes < (int64_t(1) << 31);
+    f->nodes8_state = -1;
+    if (ok) {
+      f->d_nodes8 = (uint2*)dev_alloc(sizeof(uint2) * (size_t)f->info.total_nodes, s);
+      f->d_roots8 = (uint32_t*)dev_alloc(sizeof(uint32_t) * (size_t)nt, s);
+      DBuf<int> bad(1, s);
+      BF_CUDA_CHECK(cudaMemsetAsync(bad.p, 0, sizeof(int), s));
+      {
+        KScope ks_("k_pack8", s, 24.0 * (double)f->info.total_nodes);
+        k_pack8<<<dim3(64, (unsigned)nt), 256, 0, s>>>(f->d_nodes, f->d_tree_off, f->d_nodes8, f->d_roots8, bad.p);
+      }
+      BF_CUDA_CHECK(cudaGetLastError());
+      int hbad = 0;
+      BF_CUDA_CHECK(cudaMemcpyAsync(&hbad, bad.p, sizeof(int), cudaMemcpyDeviceToHost, s));
+      BF_CUDA_CHECK(cudaStreamSynchronize(s));
+      if (hbad) {
+        dev_free(f->d_nodes8, s);
+        dev_free(f->d_roots8, s);
+        f->d_nodes8 = nullptr;
+        f->d_roots8 = nullptr;
+      } else {
+        f->nodes8_state = 1;
+      }
+    }
+  }
+  return f->nodes8_state > 0 ? f->d_nodes8 : nullptr;
+}
+
 void predict_impl(const bf_forest* f, const double* Xq_in, int64_t ldq, int64_t m, double* ys_in, double* yh_in,
                   int32_t ntree_total, cudaStream_t s) {
   if (m == 0) return;
@@ -309,10 +501,35 @@ void predict_impl(const bf_forest* f, const double* Xq_in, int64_t ldq, int64_t 
   if (!smax) smax = dyn_smem_limit(k_predict_smem);
   DBuf<unsigned long long> vis;
   if (prof_enabled()) {
-    vis.alloc(1, s);
-    BF_CUDA_CHECK(cudaMemsetAsync(vis.p, 0, 8, s));
+    vis.alloc(2, s);
+    BF_CUDA_CHECK(cudaMemsetAsync(vis.p, 0, 16, s));
   }
-  if (smem <= (size_t)smax) {
+  const char* force16 = getenv("BF_PREDICT_NODE16");
+  const uint2* n8 = (force16 && force16[0] == '1') ? nullptr : nodes8_get(const_cast<bf_forest*>(f), s);
+  const size_t smem8 = sizeof(float) * (size_t)PT8 * (size_t)(p | 1);
+  static int smax8 = 0;
+  if (!smax8) smax8 = std::min(dyn_smem_limit(k_predict8<true>), dyn_smem_limit(k_predict8<false>));
+  if (n8 && smem8 <= (size_t)smax8) {
+    // tree blocks of <= 32 MB of Node8 (L2-resident while every row walks them)
+    double* ysum = ys_in ? (double*)ys.dptr : nullptr;
+    DBuf<double> ytmp;
+    if (!ysum) {
+      ytmp.alloc(m, s);
+      ysum = ytmp.p;
+    }
+    const int64_t block_bytes = predict_block_bytes(32ll << 20);
+    for (int32_t t0 = 0; t0 < nt;) {
+      int32_t t1 = t0 + 1;
+      while (t1 < nt && (f->tree_off[t1 + 1] - f->tree_off[t0]) * (int64_t)sizeof(uint2) <= block_bytes) ++t1;
+      {
+        KScope ks_("k_predict8", s, 0.0);
+        (vis.p ? k_predict8<true> : k_predict8<false>)<<<(unsigned)ceil_div(m, PT8), PT8, smem8, s>>>(
+            n8, f->d_nodes, f->d_roots8, t0, t1, t0 == 0, t1 >= nt, (const double*)Xs.dptr, ldq, m, p, ysum,
+            yh_in ? (double*)yh.dptr : nullptr, inv_t, vis.p);
+      }
+      t0 = t1;
+    }
+  } else if (smem <= (size_t)smax) {
     // tree blocks of <= 64 MB of nodes (L2-resident while every row walks them)
     double* ysum = ys_in ? (double*)ys.dptr : nullptr;
     DBuf<double> ytmp;
@@ -320,7 +537,7 @@ void predict_impl(const bf_forest* f, const double* Xq_in, int64_t ldq, int64_t 
       ytmp.alloc(m, s);
       ysum = ytmp.p;
     }
-    const int64_t block_bytes = 64ll << 20;
+    const int64_t block_bytes = predict_block_bytes(48ll << 20);
     int32_t t0 = 0;
     while (t0 < nt || (nt == 0 && t0 == 0)) {
       int32_t t1 = t0 + 1;
@@ -345,11 +562,16 @@ void predict_impl(const bf_forest* f, const double* Xq_in, int64_t ldq, int64_t 
   }
   BF_CUDA_CHECK(cudaGetLastError());
   if (vis.p) {  // profile mode: algorithmic bytes = node visits x 16 B + rows x (8p + 16) B
-    unsigned long long hv = 0;
-    BF_CUDA_CHECK(cudaMemcpyAsync(&hv, vis.p, 8, cudaMemcpyDeviceToHost, s));
+    unsigned long long hv2[2] = {0, 0};
+    BF_CUDA_CHECK(cudaMemcpyAsync(hv2, vis.p, 16, cudaMemcpyDeviceToHost, s));
     BF_CUDA_CHECK(cudaStreamSynchronize(s));
-    prof_add_bytes(smem <= (size_t)smax ? "k_predict_smem" : "k_predict_gmem",
-                   16.0 * (double)hv + (double)m * (8.0 * p + 16.0 * ((ys_in != nullptr) + (yh_in != nullptr))));
+    const unsigned long long hv = hv2[0];
+    prof_add_bytes("predict_node_visits", (double)hv);
+    prof_add_bytes("predict_fp64_fallbacks", (double)hv2[1]);
+    const bool used8 = n8 && smem8 <= (size_t)smax8;
+    prof_add_bytes(used8 ? "k_predict8" : smem <= (size_t)smax ? "k_predict_smem" : "k_predict_gmem",
+                   (used8 ? 8.0 : 16.0) * (double)hv +
+                       (double)m * (8.0 * p + 16.0 * ((ys_in != nullptr) + (yh_in != nullptr))));
   }
   if (ys_in) ys.finish(s);
   if (yh_in) yh.finish(s);
