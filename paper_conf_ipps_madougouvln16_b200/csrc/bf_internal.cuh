@@ -198,6 +198,14 @@ struct Node16 {  // packed node for traversal: 16 B, one sector-aligned load
 };
 static_assert(sizeof(Node16) == 16, "Node16 must be 16 bytes");
 
+// Compact traversal node (predict.cu k_pack8; layout documented there): internal = {float thr, LL<<31 |
+// RL<<30 | feature<<22 | rel}, leaf = the fp64 value; roots8[t] = root id | ROOT_LEAF for one-node trees.
+constexpr int N8_FEAT_BITS = 8, N8_REL_BITS = 22;
+constexpr uint32_t ROOT_LEAF = 0x80000000u;
+__device__ __forceinline__ double leaf8(uint2 v) { return __hiloint2double((int)v.y, (int)v.x); }
+__device__ __forceinline__ uint32_t n8_feature(uint2 w) { return (w.y >> N8_REL_BITS) & ((1u << N8_FEAT_BITS) - 1u); }
+__device__ __forceinline__ uint32_t n8_rel(uint2 w) { return w.y & ((1u << N8_REL_BITS) - 1u); }
+
 }  // namespace bf
 
 struct bf_forest {

@@ -11,6 +11,7 @@
 //     e_tm - e_t is exactly zero and is skipped; predictors never used by the
 //     tree get d_tm = 0 exactly (S7).
 #include <algorithm>
+#include <cstdlib>
 
 #include "bf_internal.cuh"
 
@@ -340,6 +341,198 @@ __global__ void __launch_bounds__(IPT) k_importance(ImpArgs g) {
     if (sacc[m] != 0.0) atomicAdd(&g.d_slots[(int64_t)i * g.p + m], sacc[m]);
 }
 
+// k_importance8: k_importance on the compact nodes (predict.cu k_pack8) with a float row tile: the same
+// walks, exact by the float-tie fallback of S5 (the fp64 x of the row from X, or the fp64 permuted value,
+// against the fp64 threshold of Node16).  Half the shared memory per row (twice the CTAs per SM) and half
+// the node bytes.
+struct Imp8Args {
+  ImpArgs a;
+  const uint2* nodes8;
+  const uint32_t* roots8;  // per local tree (forest numbering)
+};
+
+__global__ void __launch_bounds__(IPT) k_importance8(Imp8Args g8) {
+  const ImpArgs& g = g8.a;
+  extern __shared__ double ism[];  // sacc[p] | float x tile IPT x (p|1)
+  double* sacc = ism;
+  const int stride = g.p | 1;
+  float* sx = reinterpret_cast<float*>(ism + ((g.p + 1) & ~1));
+  __shared__ double serr[IPT / 32];
+  const int b = blockIdx.y;
+  const int32_t i = g.i0 + b;
+  const int64_t n_o = g.nout[b];
+  const int64_t a0 = (int64_t)blockIdx.x * IPT;
+  if (a0 >= n_o) return;  // uniform per CTA
+  for (int m = threadIdx.x; m < g.p; m += IPT) sacc[m] = 0.0;
+  const uint32_t* Ob = g.O + (int64_t)b * g.n;
+  const int64_t a = a0 + threadIdx.x;
+  const bool act = a < n_o;
+  const uint32_t r = act ? Ob[a] : Ob[a0];
+  {  // stage the tile as floats: 8 column loads in flight per thread
+    float* xs = sx + threadIdx.x * stride;
+    for (int f0 = 0; f0 < g.p; f0 += 8) {
+      double v[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) v[u] = (f0 + u < g.p) ? __ldg(g.X + (int64_t)(f0 + u) * g.ldx + r) : 0.0;
+#pragma unroll
+      for (int u = 0; u < 8; ++u)
+        if (f0 + u < g.p) xs[f0 + u] = __double2float_rn(v[u]);
+    }
+  }
+  __syncthreads();
+  double err0 = 0.0;
+  if (act) {
+    const float* xs = sx + threadIdx.x * stride;
+    const double* xg = g.X + r;
+    const uint2* n8 = g8.nodes8;
+    const Node16* n16 = g.nodes;
+    const uint32_t rw = __ldg(g8.roots8 + i);
+    const uint32_t root = rw & ~ROOT_LEAF;
+    const double yr = g.y[r];
+    // child of internal node (gid, w) for this row, feature pm (if tested) taking the value (xpf, xpd)
+    auto child = [&](uint32_t gid, uint2 w, int pm, float xpf, double xpd, bool& leaf) -> uint32_t {
+      const uint32_t f = n8_feature(w);
+      const bool pf = (int)f == pm;
+      const float xf = pf ? xpf : xs[f], tf = __uint_as_float(w.x);
+      uint32_t right = xf > tf;
+      if (xf == tf || xf != xf) {  // float tie: decide in fp64 (S5)
+        const double xd = pf ? xpd : __ldg(xg + (int64_t)f * g.ldx);
+        right = !(xd <= __ldg(&n16[gid].v));
+      }
+      leaf = (w.y >> (31 - right)) & 1u;
+      return gid + n8_rel(w) + right;
+    };
+    // original walk
+    double f0v;
+    if (rw & ROOT_LEAF) {
+      f0v = leaf8(__ldg(n8 + root));
+    } else {
+      uint32_t gid = root;
+      uint2 w = __ldg(n8 + gid);
+      for (;;) {
+        bool leaf;
+        const uint32_t c = child(gid, w, -1, 0.f, 0.0, leaf);
+        const uint2 ch = __ldg(n8 + c);
+        if (leaf) {
+          f0v = leaf8(ch);
+          break;
+        }
+        gid = c;
+        w = ch;
+      }
+    }
+    const double d0 = yr - f0v;
+    err0 = d0 * d0;
+    atomicAdd(&g.oob_sum[r], f0v);
+    atomicAdd(&g.oob_cnt[r], 1);
+    // permuted walks from the first occurrence of each predictor on the path
+    if (!(rw & ROOT_LEAF)) {
+      uint64_t seen = 0;
+      int depth = 0;
+      uint32_t gid = root;
+      uint2 w = __ldg(n8 + gid);
+      bool at_leaf = false;
+      for (;;) {
+        int cnt = 0;
+        int qm[ILP];
+        uint32_t qg[ILP];
+        uint2 qw[ILP];
+        while (!at_leaf && cnt < ILP) {
+          const int m = (int)n8_feature(w);
+          bool first = !((seen >> (m & 63)) & 1ull);
+          if (!first && g.p > 64) {  // bitmask collision possible: verify on the path prefix
+            first = true;
+            uint32_t kg = root;
+            for (int d = 0; d < depth; ++d) {
+              const uint2 pw = __ldg(n8 + kg);
+              if ((int)n8_feature(pw) == m) {
+                first = false;
+                break;
+              }
+              bool lf;
+              kg = child(kg, pw, -1, 0.f, 0.0, lf);
+            }
+          }
+          seen |= 1ull << (m & 63);
+          if (first) {
+#pragma unroll
+            for (int u = 0; u < ILP; ++u)
+              if (u == cnt) {
+                qm[u] = m;
+                qg[u] = gid;
+                qw[u] = w;
+              }
+            ++cnt;
+          }
+          bool leaf;
+          const uint32_t c = child(gid, w, -1, 0.f, 0.0, leaf);
+          if (leaf) {
+            at_leaf = true;
+          } else {
+            gid = c;
+            w = __ldg(n8 + c);
+          }
+          ++depth;
+        }
+        if (cnt == 0) break;
+        double xm[ILP];
+        float xmf[ILP];
+        bool live[ILP];
+#pragma unroll
+        for (int u = 0; u < ILP; ++u) {
+          live[u] = u < cnt;
+          xm[u] = 0.0;
+          if (live[u]) {
+            const int64_t pa = __ldg(g.perm + ((int64_t)b * g.p + qm[u]) * g.n + a);
+            xm[u] = __ldg(g.X + (int64_t)qm[u] * g.ldx + Ob[pa]);
+          } else {
+            qm[u] = -1;
+          }
+          xmf[u] = __double2float_rn(xm[u]);
+        }
+        double val[ILP];
+        bool any = true;
+        while (any) {
+          any = false;
+#pragma unroll
+          for (int u = 0; u < ILP; ++u)
+            if (live[u]) {
+              bool leaf;
+              const uint32_t c = child(qg[u], qw[u], qm[u], xmf[u], xm[u], leaf);
+              const uint2 ch = __ldg(n8 + c);
+              if (leaf) {
+                val[u] = leaf8(ch);
+                live[u] = false;
+              } else {
+                qg[u] = c;
+                qw[u] = ch;
+                any = true;
+              }
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < ILP; ++u)
+          if (u < cnt) {
+            const double d1 = yr - val[u];
+            const double diff = d1 * d1 - err0;
+            if (diff != 0.0) atomicAdd(&sacc[qm[u]], diff);
+          }
+      }
+    }
+  }
+  // e_t
+  for (int o = 16; o > 0; o >>= 1) err0 += __shfl_down_sync(0xffffffffu, err0, o);
+  if ((threadIdx.x & 31) == 0) serr[threadIdx.x >> 5] = err0;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double s = 0.0;
+    for (int j = 0; j < IPT / 32; ++j) s += serr[j];
+    if (s != 0.0) atomicAdd(&g.e_t[i], s);
+  }
+  for (int m = threadIdx.x; m < g.p; m += IPT)
+    if (sacc[m] != 0.0) atomicAdd(&g.d_slots[(int64_t)i * g.p + m], sacc[m]);
+}
+
 __global__ void k_divide(double* d_slots, const int64_t* nout_t, int32_t T, int p) {
   const int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (k >= (int64_t)T * p) return;
@@ -456,6 +649,11 @@ void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, co
   static int ismax = 0;
   if (!ismax) ismax = dyn_smem_limit(k_importance);
   BF_REQUIRE(smem <= (size_t)ismax, BF_ENOTIMPL, "bf_oob_importance: p too large for the shared-memory row tile");
+  const char* force16 = getenv("BF_PREDICT_NODE16");  // same switch as predict: keep the Node16 walks
+  const uint2* n8 = (force16 && force16[0] == '1') ? nullptr : nodes8_get(const_cast<bf_forest*>(f), s);
+  const size_t smem8 = sizeof(double) * (size_t)((p + 1) & ~1) + sizeof(float) * (size_t)IPT * (size_t)(p | 1);
+  static int ismax8 = 0;
+  if (!ismax8) ismax8 = dyn_smem_limit(k_importance8);
   for (int32_t i0 = 0; i0 < T; i0 += B) {
     const int Bc = std::min(B, T - i0);
     bootstrap_impl(f->info.seed, f->info.tree_begin + i0, Bc, n, f->info.sampsize, f->info.replace, w.p, s);
@@ -479,8 +677,13 @@ void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, co
       static int pfs = 0;
       if (!pfs) pfs = dyn_smem_limit(k_perm_fill);
       KScope ks_("k_perm_fill", s, 0.0);
+      // round tables sized for the largest possible n_o (<= n): 6 x 2^h words, h = feistel_h(n) <= PH_MAX
+      int hb = 64 - __builtin_clzll((unsigned long long)std::max<int64_t>(n - 1, 1));
+      hb = std::max(hb, 2);
+      hb += hb & 1;
+      const int hmax = std::min(hb / 2, PH_MAX);
       k_perm_fill<<<dim3((unsigned)std::max<int64_t>(1, std::min<int64_t>(8, ceil_div(n, 65536))), p, Bc), 512,
-                    sizeof(uint32_t) * 6 * (1 << PH_MAX), s>>>(f->info.seed, f->info.tree_begin + i0, p, n, nout_t + i0, perm.p);
+                    sizeof(uint32_t) * 6 * ((size_t)1 << hmax), s>>>(f->info.seed, f->info.tree_begin + i0, p, n, nout_t + i0, perm.p);
     }
     BF_CUDA_CHECK(cudaGetLastError());
     ImpArgs g;
@@ -502,7 +705,14 @@ void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, co
     g.e_t = e_t;
     g.perm = perm.p;
     // OOB rows per tree <= n; grid sized for n (CTAs past n_o exit early)
-    {
+    if (n8 && smem8 <= (size_t)ismax8) {
+      Imp8Args g8;
+      g8.a = g;
+      g8.nodes8 = n8;
+      g8.roots8 = f->d_roots8;
+      KScope ks_("k_importance8", s, 0.0);
+      k_importance8<<<dim3((unsigned)ceil_div(n, IPT), Bc), IPT, smem8, s>>>(g8);
+    } else {
       KScope ks_("k_importance", s, 0.0);
       k_importance<<<dim3((unsigned)ceil_div(n, IPT), Bc), IPT, smem, s>>>(g);
     }

@@ -106,8 +106,6 @@ __global__ void __launch_bounds__(PT) k_predict_smem(const Node16* __restrict__ 
 // RN_f32(x) < RN_f32(thr) implies x < thr and RN_f32(x) > RN_f32(thr) implies x > thr; only
 // RN_f32(x) == RN_f32(thr) (or NaN) falls back to the fp64 x (global X) and the fp64 thr (Node16).  The walk
 // therefore takes exactly the S5 path, with half the node bytes and half the shared-memory row tile.
-constexpr int N8_FEAT_BITS = 8, N8_REL_BITS = 22;
-constexpr uint32_t ROOT_LEAF = 0x80000000u;  // roots8[t] = global root id | ROOT_LEAF for single-node trees
 
 __global__ void k_pack8(const Node16* __restrict__ nodes, const int64_t* __restrict__ off, uint2* __restrict__ out,
                         uint32_t* __restrict__ roots, int* __restrict__ bad) {
@@ -136,7 +134,6 @@ __global__ void k_pack8(const Node16* __restrict__ nodes, const int64_t* __restr
   }
 }
 
-__device__ __forceinline__ double leaf8(uint2 v) { return __hiloint2double((int)v.y, (int)v.x); }
 
 constexpr int PT8 = 128;  // rows per CTA
 constexpr int S8 = 8;     // walks in flight per thread (a finished slot restarts with the block's next tree;

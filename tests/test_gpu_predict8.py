@@ -170,3 +170,29 @@ def test_predict8_tiny_row_counts(m):
     assert a.shape == (m,)
     if m:
         assert rel_close(a, of.predict_sum(np.ascontiguousarray(Q)), 1e-9)
+
+
+@pytest.mark.parametrize("node16", [False, True])
+def test_importance_float_ties_vs_oracle(node16):
+    """OOB importance walks (original and permuted) on the compact nodes take the fp64 decision on float
+    ties: slots, OOB sums and counts agree with the oracle (S6-S7 tolerances) on tie-heavy data."""
+    X, y = _float_tie_data(n=2000, seed=21)
+    T = 12
+    of = O.fit(X, y, ntree=T, seed=5, nthreads=4)
+    gf = bf.fit(dev(X), dev(y), ntree=T, seed=5)
+    env = {"BF_PREDICT_NODE16": "1"} if node16 else {}
+    old = {k: os.environ.get(k) for k in env}
+    try:
+        os.environ.update(env)
+        r = gf.oob_importance(dev(X), dev(y))
+    finally:
+        for k, v in old.items():
+            if v is None:
+                os.environ.pop(k, None)
+    ro = of.oob_importance(X, y)
+    assert np.array_equal(r["nout_t"].cpu().numpy(), ro["nout_t"])
+    assert np.array_equal(r["oob_cnt"].cpu().numpy(), ro["oob_cnt"])
+    assert rel_close(r["oob_sum"].cpu().numpy(), ro["oob_sum"], 1e-9)
+    assert rel_close(r["e_t"].cpu().numpy(), ro["e_t"], 1e-9)
+    ds = ro["d_slots"]
+    assert rel_close(r["d_slots"].cpu().numpy(), ds, 1e-6, atol_scale=1e-9)
