@@ -11,7 +11,7 @@ timeout 1800 ncu --metrics gpu__time_duration.sum --clock-control none --csv --l
 echo "launch list rc=$?"
 python tools/ncu_summary.py launches $O/launches.csv $O/launch_summary.txt | head -25
 # kernel, launches to skip (a representative launch of the second batch / a mid level)
-for spec in "k_subtree 1" "k_partition_tree 40" "k_split_scan_tree 40" "k_predict_smem 7" "k_importance 1" "k_dest_bits 40" "k_list_scatter 1"; do
+for spec in "k_subtree 1" "k_partition_tree 40" "k_split_scan_tree 40" "k_predict8 3" "k_importance8 1" "k_perm_fill 1" "k_list_scatter 1"; do
   set -- $spec
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:$1 -s $2 -c 1 -f -o $O/prof_$1 python $B > $O/ncu_$1.log 2>&1
   echo "$1 rc=$?"
