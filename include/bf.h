@@ -197,6 +197,32 @@ int bf_pca(const double* X, int64_t ldx, int64_t n, int32_t p, int32_t scale, in
 int bf_varimax(const double* L, int64_t ldl, int32_t p, int32_t k, int32_t normalize, double eps, double* loadings,
                double* rotmat, int32_t* iters, void* stream);
 
+/* Counter models ("(generalized) linear models
+ * are sufficient", "generalized linear models ... residual
+ * deviance"; reading R26 = R glm, default gaussian family, identity link):
+ * least squares of each of the r response columns of Y (n x r, column-major,
+ * ldy >= n; e.g. retained counters) on the shared design Z (n x k,
+ * column-major, ldz >= n; built by the caller from problem/platform
+ * characteristics, intercept column included by the caller).  Outputs: coef
+ * (k x r, ld k), deviance (r, residual sum of squares; may be NULL),
+ * null_deviance (r, sum of squares about the mean; may be NULL).  Solved by
+ * column-scaled CholeskyQR2 in fp64.  1 <= k <= 32, 1 <= r <= 64, n >= k;
+ * a rank-deficient design -> BF_EINVAL.  Synchronous.                      */
+int bf_glm_gaussian(const double* Z, int64_t ldz, int64_t n, int32_t k, const double* Y, int64_t ldy, int32_t r,
+                    double* coef, double* deviance, double* null_deviance, void* stream);
+/* The counter models on new rows ("generate values for the most
+ * influential variables from an unseen problem size"): out (n x r,
+ * column-major, ldo >= n) = Z (n x k, ldz >= n) coef (k x r, ld k).         */
+int bf_glm_predict(const double* Z, int64_t ldz, int64_t n, int32_t k, const double* coef, int32_t r, double* out,
+                   int64_t ldo, void* stream);
+/* Similarity of two importance rankings of the same p predictors (SURVEY 8(f)
+ * NEXT-4; "the same variable importance ranking", P:295 platform
+ * "similarity"; reading R27): out[0] = Spearman's rho (Pearson correlation of
+ * mid-ranks), out[1] = Kendall's tau-b (ties excluded pairwise); NaN when a
+ * vector is constant.  a, b, out: host or device.  2 p doubles must fit in
+ * shared memory (p <= 14000).                                              */
+int bf_rank_similarity(const double* a, const double* b, int32_t p, double* out, void* stream);
+
 /* ---- single-step entry points (parity tests) ---- */
 /* Philox4x32-10 on `count` counters (S1): ctr[4*i..], out[4*i..].          */
 int bf_philox(const uint32_t* ctr, uint32_t key0, uint32_t key1, uint32_t* out, int64_t count, void* stream);

@@ -80,6 +80,9 @@ def lib():
             "bf_partial_dependence": ([vp, vp, i64, i64, i32, i32, vp, i32, vp, vp, i32, vp], C.c_int),
             "bf_pd_grid": ([vp, i64, i32, vp, C.POINTER(C.c_int32), vp], C.c_int),
             "bf_varimax": ([vp, i64, i32, i32, i32, C.c_double, vp, vp, C.POINTER(C.c_int32), vp], C.c_int),
+            "bf_glm_gaussian": ([vp, i64, i64, i32, vp, i64, i32, vp, vp, vp, vp], C.c_int),
+            "bf_rank_similarity": ([vp, vp, i32, vp, vp], C.c_int),
+            "bf_glm_predict": ([vp, i64, i64, i32, vp, i32, vp, i64, vp], C.c_int),
             "bf_philox": ([vp, C.c_uint32, C.c_uint32, vp, i64, vp], C.c_int),
             "bf_i128_to_double": ([vp, vp, vp, i64, vp], C.c_int),
             "bf_fixed_point": ([vp, i64, i64, vp, C.POINTER(C.c_int32), vp], C.c_int),
@@ -103,7 +106,8 @@ def exported_symbols():
                         "bf_forest_info_get", "bf_forest_export", "bf_forest_import", "bf_predict",
                         "bf_oob_importance", "bf_importance_finalize", "bf_pca", "bf_philox", "bf_i128_to_double",
                         "bf_fixed_point", "bf_bootstrap", "bf_perm", "bf_profile_enable", "bf_profile_read",
-                        "bf_launch_count", "bf_partial_dependence", "bf_pd_grid", "bf_varimax")]
+                        "bf_launch_count", "bf_partial_dependence", "bf_pd_grid", "bf_varimax",
+                        "bf_glm_gaussian", "bf_glm_predict", "bf_rank_similarity")]
 
 
 class KernelStat(C.Structure):
@@ -316,6 +320,38 @@ def varimax(L, normalize: bool = True, eps: float = 1e-5) -> dict:
     _check(lib().bf_varimax(_ptr(L), p, p, k, int(normalize), float(eps), _ptr(lo), _ptr(ro), C.byref(it),
                             _stream()), "bf_varimax")
     return {"loadings": lo, "rotmat": ro, "iters": int(it.value)}
+
+
+def glm_gaussian(Z, Y) -> dict:
+    """Counter models (bf_glm_gaussian, reading R26): Z (k, n) design = column-major n x k, Y (r, n) responses.
+    Returns coef (r, k) (row j = coefficients of response j), deviance (r), null_deviance (r)."""
+    k, n = Z.shape
+    Y2 = Y.reshape(1, -1) if len(Y.shape) == 1 else Y
+    r = Y2.shape[0]
+    coef = _empty_like_dev(Z, (r, k), np.float64)
+    dev = _empty_like_dev(Z, (r,), np.float64)
+    nul = _empty_like_dev(Z, (r,), np.float64)
+    _check(lib().bf_glm_gaussian(_ptr(Z), n, n, k, _ptr(Y2), n, r, _ptr(coef), _ptr(dev), _ptr(nul), _stream()),
+           "bf_glm_gaussian")
+    return {"coef": coef, "deviance": dev, "null_deviance": nul}
+
+
+def glm_predict(Z, coef):
+    """Counter models on new rows (bf_glm_predict): Z (k, n) design, coef (r, k).  Returns (r, n)."""
+    k, n = Z.shape
+    r = coef.shape[0]
+    out = _empty_like_dev(Z, (r, n), np.float64)
+    _check(lib().bf_glm_predict(_ptr(Z), n, n, k, _ptr(coef), r, _ptr(out), n, _stream()), "bf_glm_predict")
+    return out
+
+
+def rank_similarity(a, b) -> tuple:
+    """(Spearman rho, Kendall tau-b) of two importance vectors (bf_rank_similarity, reading R27)."""
+    p = int(a.shape[0])
+    out = _empty_like_dev(a, (2,), np.float64)
+    _check(lib().bf_rank_similarity(_ptr(a), _ptr(b), p, _ptr(out), _stream()), "bf_rank_similarity")
+    o = out.cpu().numpy() if hasattr(out, "cpu") else out
+    return float(o[0]), float(o[1])
 
 
 def pca(X, scale: bool = True, k: int | None = None) -> dict:

@@ -14,7 +14,7 @@ ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 LIBDIR = os.path.join(HERE, "_lib")
 LIB = os.path.join(LIBDIR, "libbf.so")
-SOURCES = ["capi.cu", "fit.cu", "predict.cu", "importance.cu", "pca.cu"]
+SOURCES = ["capi.cu", "fit.cu", "predict.cu", "importance.cu", "pca.cu", "models.cu"]
 HEADERS = ["bf_internal.cuh"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 

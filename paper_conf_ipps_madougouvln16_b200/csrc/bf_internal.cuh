@@ -254,6 +254,12 @@ void pca_impl(const double* X, int64_t ldx, int64_t n, int32_t p, int32_t scale,
               double* rotation, double* center, double* scores, cudaStream_t s);
 void varimax_impl(const double* L, int64_t ldl, int32_t p, int32_t k, int32_t normalize, double eps, double* loadings,
                   double* rotmat, int32_t* iters_host, cudaStream_t s);
+// models.cu
+void glm_gaussian_impl(const double* Z, int64_t ldz, int64_t n, int32_t k, const double* Y, int64_t ldy, int32_t r,
+                       double* coef, double* deviance, double* null_deviance, cudaStream_t s);
+void glm_predict_impl(const double* Z, int64_t ldz, int64_t n, int32_t k, const double* coef, int32_t r, double* out,
+                      int64_t ldo, cudaStream_t s);
+void rank_similarity_impl(const double* a, const double* b, int32_t p, double* out, cudaStream_t s);
 // misc kernels (capi.cu)
 void philox_impl(const uint32_t* ctr, uint32_t k0, uint32_t k1, uint32_t* out, int64_t count, cudaStream_t s);
 void i128_impl(const int64_t* hi, const uint64_t* lo, double* out, int64_t count, cudaStream_t s);

@@ -370,6 +370,32 @@ int bf_varimax(const double* L, int64_t ldl, int32_t p, int32_t k, int32_t norma
   BF_API_END
 }
 
+int bf_glm_gaussian(const double* Z, int64_t ldz, int64_t n, int32_t k, const double* Y, int64_t ldy, int32_t r,
+                    double* coef, double* deviance, double* null_deviance, void* stream) {
+  BF_API_BEGIN
+  BF_REQUIRE(Z && Y && coef, BF_EINVAL, "bf_glm_gaussian: NULL");
+  BF_REQUIRE(ldz >= n && ldy >= n, BF_EINVAL, "bf_glm_gaussian: need ldz >= n, ldy >= n");
+  glm_gaussian_impl(Z, ldz, n, k, Y, ldy, r, coef, deviance, null_deviance, (cudaStream_t)stream);
+  BF_API_END
+}
+
+int bf_glm_predict(const double* Z, int64_t ldz, int64_t n, int32_t k, const double* coef, int32_t r, double* out,
+                   int64_t ldo, void* stream) {
+  BF_API_BEGIN
+  BF_REQUIRE(Z && coef && out, BF_EINVAL, "bf_glm_predict: NULL");
+  BF_REQUIRE(ldz >= n && ldo >= n, BF_EINVAL, "bf_glm_predict: need ldz >= n, ldo >= n");
+  glm_predict_impl(Z, ldz, n, k, coef, r, out, ldo, (cudaStream_t)stream);
+  BF_API_END
+}
+
+int bf_rank_similarity(const double* a, const double* b, int32_t p, double* out, void* stream) {
+  BF_API_BEGIN
+  BF_REQUIRE(a && b && out, BF_EINVAL, "bf_rank_similarity: NULL");
+  BF_REQUIRE(p >= 1, BF_EINVAL, "bf_rank_similarity: need p >= 1");
+  rank_similarity_impl(a, b, p, out, (cudaStream_t)stream);
+  BF_API_END
+}
+
 int bf_philox(const uint32_t* ctr, uint32_t key0, uint32_t key1, uint32_t* out, int64_t count, void* stream) {
   BF_API_BEGIN
   cudaStream_t s = (cudaStream_t)stream;
