@@ -72,6 +72,25 @@ def ncu_traffic(kernel: str):
     return None, None
 
 
+def ncu_issue(kernel: str):
+    """Issue-slot utilisation of `kernel` from the newest committed ncu summary: the bound of the latency /
+    issue-limited kernels (4 warp-instructions per SM per cycle is the sm_100 issue peak)."""
+    import glob
+    for d in sorted(glob.glob(os.path.join(ROOT, "profiles", "r[0-9]*")), reverse=True):
+        f = os.path.join(d, f"full_{kernel}.json")
+        if os.path.exists(f):
+            try:
+                m = json.load(open(f))["metrics"]
+                ipc = float(m["sm__inst_executed.avg.per_cycle_active"])
+                return {"bound": "issue", "achieved_ipc": ipc, "peak_ipc": 4.0, "frac": ipc / 4.0,
+                        "warps_active_pct": float(m["sm__warps_active.avg.pct_of_peak_sustained_active"]),
+                        "dram_pct_of_peak": float(m["gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed"]),
+                        "source": os.path.relpath(f, ROOT)}
+            except Exception:
+                pass
+    return None
+
+
 class Clocks:
     """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
 
@@ -315,7 +334,8 @@ def run_ours(args):
                 "frac": achieved / hbm, "traffic": traffic, "traffic_source": tsrc, "peak_source": hbm_src,
                 "algorithmic_bytes_per_launch": d["bytes"] / max(d["launches"], 1),
                 "share_of_step": d["ms"] / args.steps / ms,
-                "avg_launch_ms": d["ms"] / max(d["launches"], 1)}
+                "avg_launch_ms": d["ms"] / max(d["launches"], 1),
+                "issue": ncu_issue(dom)}
     kernels = {k: {"ms_per_step": v["ms"] / args.steps, "launches_per_step": v["launches"] / args.steps,
                    "GBps": (v["bytes"] / (v["ms"] / 1e3) / 1e9) if v["ms"] > 0 and v["bytes"] > 0 else None}
                for k, v in sorted(stats.items(), key=lambda kv: -kv[1]["ms"]) if v["launches"] > 0}
