@@ -991,7 +991,15 @@ __device__ __forceinline__ bool part_item_active(const Split* split, const Child
   return kl == KIND_LARGE || kl == KIND_SMALL || kr == KIND_LARGE || kr == KIND_SMALL;
 }
 
-__host__ __device__ __forceinline__ int part_group(int a, int p) { return a >= TPUNIT ? 1 : min(p, TPUNIT / a); }
+// Features per work item: an item is a contiguous range of the node's block (its feature segments are
+// contiguous, and every segment has exactly al lefts), so the item is stable-partitioned as ONE stream with a
+// running left count: lefts land at f0 * al + (lefts so far), rights at f0 * ar + (rights so far).  Items of
+// about PART_ITEM_UNITS units keep the units full (only an item's last unit is partial).
+constexpr int PART_ITEM_UNITS = 8;
+__host__ __device__ __forceinline__ int part_group(int a, int p) {
+  const int tgt = PART_ITEM_UNITS * TPUNIT;
+  return a >= tgt ? 1 : min(p, tgt / a);
+}
 
 // Work items of the partition (node, group of consecutive features), listed per level so that a
 // partition CTA finds its next item with one load instead of walking the tree's item sequence.
@@ -1011,13 +1019,13 @@ __global__ void k_part_items_map(int N, int p, const LNode* nodes, const int32_t
 }
 
 // a9 partition: one CTA owns whole work items of one tree; lefts first, stable.
-// A work item is (node, group of G consecutive features) with G = max(1,
-// TPUNIT / a): the node's feature segments are contiguous, so a group is ONE
-// bulk copy, and the left (right) outputs of consecutive features are
-// contiguous in the child's block.  Items with a > TPUNIT are walked in units
-// with a running left count.
+// A work item is (node, group of G consecutive features), G = part_group(a, p):
+// a contiguous range of the node's block, walked in full units of TPUNIT
+// entries (bulk copies that may straddle feature segments) with a running left
+// count; the left (right) outputs of consecutive features are contiguous in
+// the child's block, so the group partitions as one stream.
 struct PWork {
-  int node, f0, g, unit;  // node index, first feature, features in the unit, unit index inside the feature
+  int node, f0, g, unit;  // node index, first feature, features in the item, unit index inside the item
   int a, nun;             // the node's entries per feature; units of the item
   int64_t base;
   int kl, al, kr, ar;     // children: kind and entries per feature
@@ -1031,8 +1039,6 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
   uint32_t* bm = (uint32_t*)(outb + TPUNIT);    // nw words (if staged)
   __shared__ uint64_t bar[2];
   __shared__ int32_t sm[TPNT / 32];
-  __shared__ int32_t tpre[TPNT];                // per-thread exclusive prefix of lefts in the unit
-  __shared__ uint32_t tmask[TPNT];              // per-thread left mask
   __shared__ int s_off[2];
   __shared__ PWork s_w[2];
   const int tid = threadIdx.x;
@@ -1093,7 +1099,7 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
       cw.a = nd.a;
       cw.base = nd.base;
       cw.g = min(part_group(nd.a, g.p), g.p - it.y);
-      cw.nun = cw.g > 1 ? 1 : (nd.a + TPUNIT - 1) / TPUNIT;
+      cw.nun = (int)(((int64_t)cw.g * nd.a + TPUNIT - 1) / TPUNIT);
       cw.unit = 0;
       cw.kl = c0.kind;
       cw.al = c0.a;
@@ -1107,9 +1113,9 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
     };
     auto issue = [&](const PWork& w, int slot) {
       const int u0 = w.unit * TPUNIT;
-      const int cnt = w.g > 1 ? w.g * w.a : min(TPUNIT, w.a - u0);
-      s_off[slot] = stage_entries(bufs + (size_t)slot * (TPUNIT + 2),
-                                  g.Ecur + w.base + (int64_t)w.f0 * w.a + (w.g > 1 ? 0 : u0), cnt, &bar[slot]);
+      const int cnt = min(TPUNIT, w.g * w.a - u0);
+      s_off[slot] = stage_entries(bufs + (size_t)slot * (TPUNIT + 2), g.Ecur + w.base + (int64_t)w.f0 * w.a + u0, cnt,
+                                  &bar[slot]);
     };
     // thread 0 runs the item pipeline and publishes each unit's work record in s_w[slot] (slot = its buffer)
     if (tid == 0) {
@@ -1133,7 +1139,7 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
       }
       const int a = w.a;
       const int u0 = w.unit * TPUNIT;
-      const int cnt = w.g > 1 ? w.g * a : min(TPUNIT, a - u0);
+      const int cnt = min(TPUNIT, w.g * a - u0);
       mbar_wait(&bar[cur], phase[cur]);
       phase[cur] ^= 1u;
       const uint64_t* buf = bufs + (size_t)cur * (TPUNIT + 2) + s_off[cur];
@@ -1160,25 +1166,7 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
       int32_t tot;
       const int32_t lbl = block_excl_scan(c, sm, tot);
       const int al = w.al, ar = w.ar;  // lefts / rights per feature segment
-      if (w.g > 1) {
-        tpre[tid] = lbl;
-        tmask[tid] = lmask;
-        __syncthreads();
-        int pl = lbl;
-#pragma unroll
-        for (int q = 0; q < TPV; ++q) {
-          const int j = jl + q;
-          if (j < cnt) {
-            const int sgm = j / a, s0 = sgm * a;
-            const int t0 = s0 / TPV, o0 = s0 - t0 * TPV;
-            const int ps = tpre[t0] + __popc(tmask[t0] & ((1u << o0) - 1u));  // lefts before the segment start
-            const int lb = pl - ps;                                            // lefts before j in the segment
-            if ((lmask >> q) & 1u) outb[sgm * al + lb] = ev[q];
-            else outb[w.g * al + sgm * ar + (j - s0 - lb)] = ev[q];
-            pl += (lmask >> q) & 1u;
-          }
-        }
-      } else {
+      {
         int li = lbl, ri = tot + (jl - lbl);
 #pragma unroll
         for (int q = 0; q < TPV; ++q) {
@@ -1192,8 +1180,8 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
       __syncthreads();
       const bool keepL = w.kl == KIND_LARGE || w.kl == KIND_SMALL;
       const bool keepR = w.kr == KIND_LARGE || w.kr == KIND_SMALL;
-      const int64_t exl = w.g > 1 ? 0 : carry_l, exr = w.g > 1 ? 0 : (int64_t)u0 - carry_l;
-      const int nl_out = w.g > 1 ? w.g * al : tot, nr_out = cnt - nl_out;
+      const int64_t exl = carry_l, exr = (int64_t)u0 - carry_l;
+      const int nl_out = tot, nr_out = cnt - nl_out;
       if (keepL) {
         uint64_t* dl = (w.kl == KIND_LARGE ? g.Enext : g.Esmall) + w.bl + (int64_t)w.f0 * al + exl;
         for (int i = tid; i < nl_out; i += TPNT) dl[i] = outb[i];
