@@ -312,21 +312,53 @@ __global__ void k_roots(int B, int64_t ns, int nodesize, const int32_t* a_root, 
 // ------------------------------------------------------------------ a5 root lists (two-pass stable compaction)
 constexpr int LCH = 2048;  // entries per CTA chunk (256 threads x 8)
 
-__global__ void k_list_count(const uint64_t* srt, int64_t n, const int32_t* wts, const int32_t* kind, int nchunk,
-                             int32_t* cnt) {
-  const int c = blockIdx.x, f = blockIdx.y, b = blockIdx.z, p = gridDim.y;
-  if (kind[b] != KIND_LARGE && kind[b] != KIND_SMALL) return;
-  __shared__ int32_t sm[NT / 32];
-  const uint64_t* col = srt + (int64_t)f * n;
-  const int32_t* W = wts + (int64_t)b * n;
-  int32_t k = 0;
-  for (int u = threadIdx.x; u < LCH; u += NT) {
-    const int64_t i = (int64_t)c * LCH + u;
-    if (i < n) k += W[e_row(col[i])] > 0;
+// The batch's multiplicities row-major as uint16 (w <= 65535 is checked after k_payload): wp[row * Bp + b],
+// Bp = B rounded up to LTG, so one 16-byte load gives a row's weights for LTG trees.
+constexpr int LTG = 8;  // trees per list-init CTA
+__global__ void k_w_pack(const int32_t* w, int64_t n, int B, int Bp, uint16_t* wp) {
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  uint16_t v[LTG];
+  for (int b0 = 0; b0 < Bp; b0 += LTG) {
+#pragma unroll
+    for (int u = 0; u < LTG; ++u) v[u] = b0 + u < B ? (uint16_t)w[(int64_t)(b0 + u) * n + i] : (uint16_t)0;
+    uint4 q;
+    q.x = v[0] | ((uint32_t)v[1] << 16);
+    q.y = v[2] | ((uint32_t)v[3] << 16);
+    q.z = v[4] | ((uint32_t)v[5] << 16);
+    q.w = v[6] | ((uint32_t)v[7] << 16);
+    *reinterpret_cast<uint4*>(wp + i * Bp + b0) = q;
   }
-  int32_t tot;
-  block_excl_scan(k, sm, tot);
-  if (threadIdx.x == 0) cnt[((int64_t)b * p + f) * nchunk + c] = tot;
+}
+__device__ __forceinline__ uint32_t wp_get(const uint4& q, int u) {
+  const uint32_t w2 = u < 2 ? q.x : u < 4 ? q.y : u < 6 ? q.z : q.w;
+  return (u & 1) ? (w2 >> 16) : (w2 & 0xffffu);
+}
+
+// One CTA = one chunk of one presorted column for LTG trees of the batch (blockIdx.z = tree group): the
+// chunk is read once per group and each entry's weights for the group are ONE 16-byte gather.
+__global__ void k_list_count(const uint64_t* srt, int64_t n, const uint16_t* wp, int Bp, const int32_t* kind,
+                             int nchunk, int B, int32_t* cnt) {
+  const int c = blockIdx.x, f = blockIdx.y, b0 = blockIdx.z * LTG, p = gridDim.y;
+  __shared__ int32_t sm[NT / 32];
+  constexpr int V = LCH / NT;
+  const uint64_t* col = srt + (int64_t)f * n;
+  const int64_t i0 = (int64_t)c * LCH + (int64_t)threadIdx.x * V;
+  uint4 q[V];
+#pragma unroll
+  for (int u = 0; u < V; ++u)
+    q[u] = i0 + u < n ? *reinterpret_cast<const uint4*>(wp + (int64_t)e_row(col[i0 + u]) * Bp + b0)
+                      : make_uint4(0u, 0u, 0u, 0u);
+  for (int t = 0; t < LTG && b0 + t < B; ++t) {
+    const int b = b0 + t;
+    if (kind[b] != KIND_LARGE && kind[b] != KIND_SMALL) continue;  // uniform per CTA
+    int32_t k = 0;
+#pragma unroll
+    for (int u = 0; u < V; ++u) k += wp_get(q[u], t) > 0;
+    int32_t tot;
+    block_excl_scan(k, sm, tot);
+    if (threadIdx.x == 0) cnt[((int64_t)b * p + f) * nchunk + c] = tot;
+  }
 }
 
 __global__ void k_list_prefix(int32_t* cnt, int nseg, int nchunk) {
@@ -341,38 +373,38 @@ __global__ void k_list_prefix(int32_t* cnt, int nseg, int nchunk) {
   }
 }
 
-__global__ void k_list_scatter(const uint64_t* srt, int64_t n, const int32_t* wts, const int32_t* kind,
-                               const int64_t* base, const int32_t* a_root, int nchunk, const int32_t* cnt,
+__global__ void k_list_scatter(const uint64_t* srt, int64_t n, const uint16_t* wp, int Bp, const int32_t* kind,
+                               const int64_t* base, const int32_t* a_root, int nchunk, int B, const int32_t* cnt,
                                uint64_t* Elarge, uint64_t* Esmall) {
-  const int c = blockIdx.x, f = blockIdx.y, b = blockIdx.z, p = gridDim.y;
-  const int kd = kind[b];
-  if (kd != KIND_LARGE && kd != KIND_SMALL) return;
+  const int c = blockIdx.x, f = blockIdx.y, b0 = blockIdx.z * LTG, p = gridDim.y;
   __shared__ int32_t sm[NT / 32];
-  const uint64_t* col = srt + (int64_t)f * n;
-  const int32_t* W = wts + (int64_t)b * n;
   constexpr int V = LCH / NT;
-  uint64_t e[V];
-  bool keep[V];
-  int32_t k = 0;
+  const uint64_t* col = srt + (int64_t)f * n;
   const int64_t i0 = (int64_t)c * LCH + (int64_t)threadIdx.x * V;
+  uint64_t e[V];
+  uint4 q[V];
 #pragma unroll
-  for (int u = 0; u < V; ++u) {
-    const int64_t i = i0 + u;
-    keep[u] = false;
-    if (i < n) {
-      e[u] = col[i];
-      const int32_t wv = W[e_row(e[u])];
-      keep[u] = wv > 0;
-      e[u] |= (uint64_t)(uint32_t)wv;
-    }
-    k += keep[u];
-  }
-  int32_t tot;
-  int32_t pre = block_excl_scan(k, sm, tot) + cnt[((int64_t)b * p + f) * nchunk + c];
-  uint64_t* dst = (kd == KIND_LARGE ? Elarge : Esmall) + base[b] + (int64_t)f * a_root[b];
+  for (int u = 0; u < V; ++u) e[u] = i0 + u < n ? col[i0 + u] : ~0ull;
 #pragma unroll
   for (int u = 0; u < V; ++u)
-    if (keep[u]) dst[pre++] = e[u];
+    q[u] = e[u] != ~0ull ? *reinterpret_cast<const uint4*>(wp + (int64_t)e_row(e[u]) * Bp + b0)
+                         : make_uint4(0u, 0u, 0u, 0u);
+  for (int t = 0; t < LTG && b0 + t < B; ++t) {
+    const int b = b0 + t;
+    const int kd = kind[b];
+    if (kd != KIND_LARGE && kd != KIND_SMALL) continue;  // uniform per CTA
+    int32_t k = 0;
+#pragma unroll
+    for (int u = 0; u < V; ++u) k += wp_get(q[u], t) > 0;
+    int32_t tot;
+    int32_t pre = block_excl_scan(k, sm, tot) + cnt[((int64_t)b * p + f) * nchunk + c];
+    uint64_t* dst = (kd == KIND_LARGE ? Elarge : Esmall) + base[b] + (int64_t)f * a_root[b];
+#pragma unroll
+    for (int u = 0; u < V; ++u) {
+      const uint32_t wv = wp_get(q[u], t);
+      if (wv > 0) dst[pre++] = e[u] | (uint64_t)wv;
+    }
+  }
 }
 
 // ------------------------------------------------------------------ a6 mtry (global phase)
@@ -2638,10 +2670,16 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
       {
         const int nchunk = (int)ceil_div(n, LCH);
         DBuf<int32_t> cnt((size_t)Bc * p * nchunk, s);
-        dim3 grid((unsigned)nchunk, (unsigned)p, (unsigned)Bc);
+        const int Bp = (Bc + LTG - 1) / LTG * LTG;
+        DBuf<uint16_t> wpk((size_t)n * Bp, s);
+        {
+          KScope ks_("k_w_pack", s, (double)n * Bc * 4.0 + (double)n * Bp * 2.0);
+          k_w_pack<<<(unsigned)ceil_div(n, NT), NT, 0, s>>>(w.p, n, Bc, Bp, wpk.p);
+        }
+        dim3 grid((unsigned)nchunk, (unsigned)p, (unsigned)(Bp / LTG));
         {
           KScope ks_("k_list_count", s, 0.0);
-          k_list_count<<<grid, NT, 0, s>>>(srt.p, n, w.p, kind_d.p, nchunk, cnt.p);
+          k_list_count<<<grid, NT, 0, s>>>(srt.p, n, wpk.p, Bp, kind_d.p, nchunk, Bc, cnt.p);
         }
         {
           KScope ks_("k_list_prefix", s, 0.0);
@@ -2649,10 +2687,12 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
         }
         {
           KScope ks_("k_list_scatter", s, 0.0);
-          k_list_scatter<<<grid, NT, 0, s>>>(srt.p, n, w.p, kind_d.p, base_d.p, a_root.p, nchunk, cnt.p, E0.p, Es.p);
+          k_list_scatter<<<grid, NT, 0, s>>>(srt.p, n, wpk.p, Bp, kind_d.p, base_d.p, a_root.p, nchunk, Bc, cnt.p, E0.p,
+                                            Es.p);
         }
         BF_CUDA_CHECK(cudaGetLastError());
-        prof_add_bytes("k_list_scatter", (double)Bc * n * p * 8.0 + (double)(offL + offS) * 8.0);
+        // presort chunk read once per tree group + one 16 B weight gather per (entry, group) + written entries
+        prof_add_bytes("k_list_scatter", (double)(Bp / LTG) * n * p * 24.0 + (double)(offL + offS) * 8.0);
       }
       ptm.mark("boot+lists");
       LevelSummary ls{};
