@@ -68,8 +68,27 @@ __device__ __forceinline__ int feistel_h(int64_t n_o) {
   b += b & 1;
   return b >> 1;
 }
+// Round tables of the batch, computed once per (tree, predictor): gtab[(b * p + m) * tstride + r * 2^h + R] =
+// F_r(R) & mask (h = feistel_h(n_o) <= PH_MAX); every k_perm_fill CTA of (b, m) copies its table from L2.
+__global__ void k_ftab_fill(uint64_t seed, int32_t t0, int p, const int64_t* nout, int tstride, uint32_t* gtab) {
+  const int b = blockIdx.z, m = blockIdx.y;
+  const int64_t n_o = nout[b];
+  if (n_o <= 0) return;
+  const int h = feistel_h(n_o);
+  if (h > PH_MAX) return;
+  const int S = 1 << h;
+  const uint32_t mask = (uint32_t)S - 1u, t = (uint32_t)(t0 + b);
+  uint32_t* out = gtab + ((int64_t)b * p + m) * tstride;
+  for (int k = blockIdx.x * blockDim.x + threadIdx.x; k < 6 * S; k += gridDim.x * blockDim.x) {
+    uint32_t x[4];
+    philox4x32_10((uint32_t)(k & (S - 1)), (uint32_t)(k >> h), 3u | ((uint32_t)m << 8), t, (uint32_t)seed,
+                  (uint32_t)(seed >> 32), x);
+    out[k] = x[0] & mask;
+  }
+}
+
 __global__ void __launch_bounds__(512) k_perm_fill(uint64_t seed, int32_t t0, int p, int64_t n, const int64_t* nout,
-                                                   int32_t* perm) {
+                                                   const uint32_t* gtab, int tstride, int32_t* perm) {
   extern __shared__ uint32_t ftab[];  // 6 x 2^h (h <= PH_MAX)
   const int b = blockIdx.z, m = blockIdx.y;
   const int64_t n_o = nout[b];
@@ -78,14 +97,9 @@ __global__ void __launch_bounds__(512) k_perm_fill(uint64_t seed, int32_t t0, in
   const int h = feistel_h(n_o);
   const uint32_t mask = (uint32_t)((1ull << h) - 1ull);
   const bool tab = h <= PH_MAX;
-  if (tab) {
-    const int S = 1 << h;
-    for (int k = threadIdx.x; k < 6 * S; k += blockDim.x) {
-      uint32_t x[4];
-      philox4x32_10((uint32_t)(k & (S - 1)), (uint32_t)(k >> h), 3u | ((uint32_t)m << 8), t, (uint32_t)seed,
-                    (uint32_t)(seed >> 32), x);
-      ftab[k] = x[0];
-    }
+  if (tab) {  // F_r(R) & mask for every round r and h-bit input R (k_ftab_fill)
+    const uint32_t* src = gtab + ((int64_t)b * p + m) * tstride;
+    for (int k = threadIdx.x; k < (6 << h); k += blockDim.x) ftab[k] = src[k];
     __syncthreads();
   }
   int32_t* out = perm + ((int64_t)b * p + m) * n;
@@ -95,17 +109,25 @@ __global__ void __launch_bounds__(512) k_perm_fill(uint64_t seed, int32_t t0, in
       out[a] = (int32_t)feistel(seed, t, (uint32_t)m, n_o, a);
       continue;
     }
-    uint64_t v = (uint64_t)a;
+    // 2h <= 2 * PH_MAX bits: 32-bit arithmetic throughout (n_o < 2^31)
+    const uint32_t* f0 = ftab;
+    const uint32_t* f1 = f0 + (1u << h);
+    const uint32_t* f2 = f1 + (1u << h);
+    const uint32_t* f3 = f2 + (1u << h);
+    const uint32_t* f4 = f3 + (1u << h);
+    const uint32_t* f5 = f4 + (1u << h);
+    const uint32_t no = (uint32_t)n_o;
+    uint32_t v = (uint32_t)a;
     do {
-      uint32_t L = (uint32_t)(v >> h), R = (uint32_t)(v & mask);
-#pragma unroll
-      for (int r = 0; r < 6; ++r) {
-        const uint32_t nR = L ^ (ftab[(r << h) + R] & mask);
-        L = R;
-        R = nR;
-      }
-      v = ((uint64_t)L << h) | R;
-    } while ((int64_t)v >= n_o);
+      uint32_t L = v >> h, R = v & mask;
+      L ^= f0[R];
+      R ^= f1[L];
+      L ^= f2[R];
+      R ^= f3[L];
+      L ^= f4[R];
+      R ^= f5[L];
+      v = (L << h) | R;  // six rounds (L, R) <- (R, L ^ F_r(R)) end with the halves back in place
+    } while (v >= no);
     out[a] = (int32_t)v;
   }
 }
@@ -645,6 +667,10 @@ void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, co
   DBuf<int32_t> w((size_t)B * n, s), cnt((size_t)B * nchunk, s);
   DBuf<uint32_t> O((size_t)B * n, s);
   DBuf<int32_t> perm((size_t)B * p * n, s);
+  int hb_all = 64 - __builtin_clzll((unsigned long long)std::max<int64_t>(n - 1, 1));
+  hb_all = std::max(hb_all, 2);
+  hb_all += hb_all & 1;
+  DBuf<uint32_t> gtab((size_t)B * p * (6u << std::min(hb_all / 2, PH_MAX)), s);
   const size_t smem = sizeof(double) * ((size_t)((p + 1) & ~1) + (size_t)IPT * (size_t)(p | 1));
   static int ismax = 0;
   if (!ismax) ismax = dyn_smem_limit(k_importance);
@@ -676,14 +702,21 @@ void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, co
     {
       static int pfs = 0;
       if (!pfs) pfs = dyn_smem_limit(k_perm_fill);
-      KScope ks_("k_perm_fill", s, 0.0);
       // round tables sized for the largest possible n_o (<= n): 6 x 2^h words, h = feistel_h(n) <= PH_MAX
       int hb = 64 - __builtin_clzll((unsigned long long)std::max<int64_t>(n - 1, 1));
       hb = std::max(hb, 2);
       hb += hb & 1;
       const int hmax = std::min(hb / 2, PH_MAX);
+      const int tstride = 6 << hmax;
+      {
+        KScope ks2_("k_ftab_fill", s, 0.0);
+        k_ftab_fill<<<dim3((unsigned)ceil_div(tstride, 256), p, Bc), 256, 0, s>>>(f->info.seed, f->info.tree_begin + i0, p,
+                                                                              nout_t + i0, tstride, gtab.p);
+      }
+      KScope ks_("k_perm_fill", s, 0.0);
       k_perm_fill<<<dim3((unsigned)std::max<int64_t>(1, std::min<int64_t>(8, ceil_div(n, 65536))), p, Bc), 512,
-                    sizeof(uint32_t) * 6 * ((size_t)1 << hmax), s>>>(f->info.seed, f->info.tree_begin + i0, p, n, nout_t + i0, perm.p);
+                    sizeof(uint32_t) * 6 * ((size_t)1 << hmax), s>>>(f->info.seed, f->info.tree_begin + i0, p, n,
+                                                                     nout_t + i0, gtab.p, tstride, perm.p);
     }
     BF_CUDA_CHECK(cudaGetLastError());
     ImpArgs g;
