@@ -215,6 +215,26 @@ int bf_glm_gaussian(const double* Z, int64_t ldz, int64_t n, int32_t k, const do
  * column-major, ldo >= n) = Z (n x k, ldz >= n) coef (k x r, ld k).         */
 int bf_glm_predict(const double* Z, int64_t ldz, int64_t n, int32_t k, const double* coef, int32_t r, double* out,
                    int64_t ldo, void* stream);
+/* MARS counter models (eq. (4), P:173, P:256 R earth; reading R28:
+ * earth's additive defaults).  X: n x d column-major predictors (ldx >= n;
+ * problem / platform characteristics), y: n responses (one counter); host or
+ * device.  Forward pass: hinge pairs max(0, x_v - t), max(0, t - x_v) at the
+ * knots t = distinct values of x_v other than its min and max, the pair
+ * giving the smallest RSS added each step (ties within 1e-12 TSS -> lowest v,
+ * t) while the RSq gain >= thresh [0.001], RSq < 1 - thresh and terms + 2 <=
+ * nk [0 -> min(200, max(20, 2 d)) + 1]; backward pass: greedy removal of the
+ * term whose loss raises RSS least, subset with the smallest GCV =
+ * (RSS/n) / (1 - C/n)^2, C = terms + penalty (terms - 1) / 2 [penalty 2].
+ * Outputs (HOST): *nterms, term_var / term_knot / term_dir (0 = intercept,
+ * +1 = max(0, x - t), -1 = max(0, t - x)) and coef, each >= nk long; stats =
+ * {RSS, GCV, RSq}.  At most 31 terms.  Synchronous.                        */
+int bf_mars_fit(const double* X, int64_t ldx, int64_t n, int32_t d, const double* y, int32_t nk, double thresh,
+                double penalty, int32_t* nterms, int32_t* term_var, double* term_knot, int32_t* term_dir, double* coef,
+                double* stats, void* stream);
+/* A MARS model on new rows: out[i] = sum_j coef_j B_j(x_i).  Terms and coef
+ * host or device; X (m x d, ldx >= m) and out host or device.              */
+int bf_mars_predict(const double* X, int64_t ldx, int64_t m, int32_t d, int32_t nterms, const int32_t* term_var,
+                    const double* term_knot, const int32_t* term_dir, const double* coef, double* out, void* stream);
 /* Similarity of two importance rankings of the same p predictors (SURVEY 8(f)
  * NEXT-4; "the same variable importance ranking", P:295 platform
  * "similarity"; reading R27): out[0] = Spearman's rho (Pearson correlation of

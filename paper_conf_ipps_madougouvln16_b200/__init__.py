@@ -83,6 +83,9 @@ def lib():
             "bf_glm_gaussian": ([vp, i64, i64, i32, vp, i64, i32, vp, vp, vp, vp], C.c_int),
             "bf_rank_similarity": ([vp, vp, i32, vp, vp], C.c_int),
             "bf_glm_predict": ([vp, i64, i64, i32, vp, i32, vp, i64, vp], C.c_int),
+            "bf_mars_fit": ([vp, i64, i64, i32, vp, i32, C.c_double, C.c_double, C.POINTER(C.c_int32), vp, vp, vp, vp,
+                             vp, vp], C.c_int),
+            "bf_mars_predict": ([vp, i64, i64, i32, i32, vp, vp, vp, vp, vp, vp], C.c_int),
             "bf_philox": ([vp, C.c_uint32, C.c_uint32, vp, i64, vp], C.c_int),
             "bf_i128_to_double": ([vp, vp, vp, i64, vp], C.c_int),
             "bf_fixed_point": ([vp, i64, i64, vp, C.POINTER(C.c_int32), vp], C.c_int),
@@ -107,7 +110,8 @@ def exported_symbols():
                         "bf_oob_importance", "bf_importance_finalize", "bf_pca", "bf_philox", "bf_i128_to_double",
                         "bf_fixed_point", "bf_bootstrap", "bf_perm", "bf_profile_enable", "bf_profile_read",
                         "bf_launch_count", "bf_partial_dependence", "bf_pd_grid", "bf_varimax",
-                        "bf_glm_gaussian", "bf_glm_predict", "bf_rank_similarity")]
+                        "bf_glm_gaussian", "bf_glm_predict", "bf_rank_similarity", "bf_mars_fit",
+                        "bf_mars_predict")]
 
 
 class KernelStat(C.Structure):
@@ -342,6 +346,35 @@ def glm_predict(Z, coef):
     r = coef.shape[0]
     out = _empty_like_dev(Z, (r, n), np.float64)
     _check(lib().bf_glm_predict(_ptr(Z), n, n, k, _ptr(coef), r, _ptr(out), n, _stream()), "bf_glm_predict")
+    return out
+
+
+def mars_fit(X, y, nk: int = 0, thresh: float = 0.001, penalty: float = 2.0) -> dict:
+    """MARS model of one response on (d, n) predictors (bf_mars_fit, reading R28).  Returns terms
+    [(var, knot, dir)] (dir 0 = intercept), coef (numpy), rss, gcv, rsq."""
+    d, n = X.shape
+    cap = 32
+    nt = C.c_int32()
+    tv = np.zeros(cap, np.int32)
+    tk = np.zeros(cap, np.float64)
+    td = np.zeros(cap, np.int32)
+    cf = np.zeros(cap, np.float64)
+    st = np.zeros(3, np.float64)
+    _check(lib().bf_mars_fit(_ptr(X), n, n, d, _ptr(y), nk, float(thresh), float(penalty), C.byref(nt), _ptr(tv),
+                             _ptr(tk), _ptr(td), _ptr(cf), _ptr(st), _stream()), "bf_mars_fit")
+    k = nt.value
+    return {"terms": [(int(tv[j]), float(tk[j]), int(td[j])) for j in range(k)], "coef": cf[:k].copy(),
+            "rss": float(st[0]), "gcv": float(st[1]), "rsq": float(st[2]),
+            "_arrays": (tv[:k].copy(), tk[:k].copy(), td[:k].copy(), cf[:k].copy())}
+
+
+def mars_predict(model: dict, X):
+    """A bf_mars_fit model on new (d, m) rows (bf_mars_predict)."""
+    d, m = X.shape
+    tv, tk, td, cf = model["_arrays"]
+    out = _empty_like_dev(X, (m,), np.float64)
+    _check(lib().bf_mars_predict(_ptr(X), m, m, d, len(tv), _ptr(tv), _ptr(tk), _ptr(td), _ptr(cf), _ptr(out),
+                                 _stream()), "bf_mars_predict")
     return out
 
 

@@ -259,6 +259,11 @@ void glm_gaussian_impl(const double* Z, int64_t ldz, int64_t n, int32_t k, const
                        double* coef, double* deviance, double* null_deviance, cudaStream_t s);
 void glm_predict_impl(const double* Z, int64_t ldz, int64_t n, int32_t k, const double* coef, int32_t r, double* out,
                       int64_t ldo, cudaStream_t s);
+void mars_fit_impl(const double* X, int64_t ldx, int64_t n, int32_t d, const double* y, int32_t nk, double thresh,
+                   double penalty, int32_t* nterms, int32_t* tvar, double* tknot, int32_t* tdir, double* coef,
+                   double* stats, cudaStream_t s);
+void mars_predict_impl(const double* X, int64_t ldx, int64_t m, int32_t d, int32_t nt, const int32_t* tvar,
+                       const double* tknot, const int32_t* tdir, const double* coef, double* out, cudaStream_t s);
 void rank_similarity_impl(const double* a, const double* b, int32_t p, double* out, cudaStream_t s);
 // misc kernels (capi.cu)
 void philox_impl(const uint32_t* ctr, uint32_t k0, uint32_t k1, uint32_t* out, int64_t count, cudaStream_t s);

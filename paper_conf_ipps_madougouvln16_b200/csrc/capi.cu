@@ -388,6 +388,28 @@ int bf_glm_predict(const double* Z, int64_t ldz, int64_t n, int32_t k, const dou
   BF_API_END
 }
 
+int bf_mars_fit(const double* X, int64_t ldx, int64_t n, int32_t d, const double* y, int32_t nk, double thresh,
+                double penalty, int32_t* nterms, int32_t* term_var, double* term_knot, int32_t* term_dir, double* coef,
+                double* stats, void* stream) {
+  BF_API_BEGIN
+  BF_REQUIRE(X && y && nterms && term_var && term_knot && term_dir && coef && stats, BF_EINVAL, "bf_mars_fit: NULL");
+  BF_REQUIRE(ldx >= n && thresh >= 0.0 && penalty >= 0.0, BF_EINVAL, "bf_mars_fit: need ldx >= n, thresh, penalty >= 0");
+  mars_fit_impl(X, ldx, n, d, y, nk, thresh, penalty, nterms, term_var, term_knot, term_dir, coef, stats,
+                (cudaStream_t)stream);
+  BF_API_END
+}
+
+int bf_mars_predict(const double* X, int64_t ldx, int64_t m, int32_t d, int32_t nterms, const int32_t* term_var,
+                    const double* term_knot, const int32_t* term_dir, const double* coef, double* out, void* stream) {
+  BF_API_BEGIN
+  BF_REQUIRE(X && out && (nterms == 0 || (term_var && term_knot && term_dir && coef)), BF_EINVAL, "bf_mars_predict: NULL");
+  BF_REQUIRE(ldx >= m && nterms >= 0 && d >= 1, BF_EINVAL, "bf_mars_predict: need ldx >= m, d >= 1");
+  for (int j = 0; j < nterms; ++j)
+    BF_REQUIRE(term_var[j] >= 0 && term_var[j] < d, BF_EINVAL, "bf_mars_predict: term variable out of range");
+  mars_predict_impl(X, ldx, m, d, nterms, term_var, term_knot, term_dir, coef, out, (cudaStream_t)stream);
+  BF_API_END
+}
+
 int bf_rank_similarity(const double* a, const double* b, int32_t p, double* out, void* stream) {
   BF_API_BEGIN
   BF_REQUIRE(a && b && out, BF_EINVAL, "bf_rank_similarity: NULL");

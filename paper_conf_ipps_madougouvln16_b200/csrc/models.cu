@@ -17,6 +17,9 @@
 // exact integers in one CTA.
 #include <algorithm>
 #include <cmath>
+#include <vector>
+
+#include <cub/cub.cuh>
 
 #include "bf_internal.cuh"
 
@@ -333,7 +336,542 @@ __global__ void k_glm_predict(const double* __restrict__ Z, int64_t ldz, int64_t
   }
 }
 
+// ------------------------------------------------------------------ MARS (reading R28)
+// Forward pass: every candidate (v, t) is one CTA that sums, over the rows, the products of its two hinges
+// c1 = max(0, x_v - t), c2 = max(0, t - x_v) with the orthonormal basis Q (16 columns per pass), with
+// themselves and with the residual r (fixed-order block reductions).  The RSS of basis + pair is
+// RSS - b^T G^-1 b with G = [c_i.c_j - (Q^T c_i).(Q^T c_j)] (c1.c2 = 0: disjoint supports), b = [c_i.r];
+// a column whose projected norm is below 1e-10 of its norm lies in span(Q) and is left out (the oracle's
+// rank-deficient least squares).  The accepted pair is appended to B and, orthogonalised twice (CGS2), to Q.
+constexpr int MQC = 16;  // Q columns per candidate pass
+constexpr int MNT = 256;
+
+__device__ __forceinline__ double block_sum_d(double v, double* red) {
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xffffffffu, v, o);
+  __syncthreads();
+  if (lane == 0) red[wid] = v;
+  __syncthreads();
+  double t = 0.0;
+  for (int w = 0; w < MNT / 32; ++w) t += red[w];
+  return t;
+}
+
+// sums[c * SW + ...]: [0, 2M) = Q^T c1, Q^T c2 interleaved per column; 2M.. = c1.c1, c2.c2, c1.r, c2.r
+__global__ void __launch_bounds__(MNT) k_mars_cand(const double* __restrict__ X, int64_t ldx, int64_t n,
+                                                  const int32_t* __restrict__ cvar, const double* __restrict__ cknot,
+                                                  const double* __restrict__ Q, int M, const double* __restrict__ r,
+                                                  int SW, double* __restrict__ sums) {
+  __shared__ double red[MNT / 32];
+  const int c = blockIdx.x;
+  const int v = cvar[c];
+  const double t = cknot[c];
+  const double* x = X + (int64_t)v * ldx;
+  double* out = sums + (int64_t)c * SW;
+  for (int j0 = 0; j0 < M; j0 += MQC) {
+    double a1[MQC], a2[MQC];
+#pragma unroll
+    for (int u = 0; u < MQC; ++u) a1[u] = a2[u] = 0.0;
+    for (int64_t i = threadIdx.x; i < n; i += MNT) {
+      const double xi = x[i], h1 = fmax(xi - t, 0.0), h2 = fmax(t - xi, 0.0);
+#pragma unroll
+      for (int u = 0; u < MQC; ++u)
+        if (j0 + u < M) {
+          const double q = Q[(int64_t)(j0 + u) * n + i];
+          a1[u] += h1 * q;
+          a2[u] += h2 * q;
+        }
+    }
+    for (int u = 0; u < MQC && j0 + u < M; ++u) {
+      const double s1 = block_sum_d(a1[u], red), s2 = block_sum_d(a2[u], red);
+      if (threadIdx.x == 0) {
+        out[2 * (j0 + u)] = s1;
+        out[2 * (j0 + u) + 1] = s2;
+      }
+    }
+  }
+  double e11 = 0.0, e22 = 0.0, e1r = 0.0, e2r = 0.0;
+  for (int64_t i = threadIdx.x; i < n; i += MNT) {
+    const double xi = x[i], h1 = fmax(xi - t, 0.0), h2 = fmax(t - xi, 0.0), ri = r[i];
+    e11 += h1 * h1;
+    e22 += h2 * h2;
+    e1r += h1 * ri;
+    e2r += h2 * ri;
+  }
+  e11 = block_sum_d(e11, red);
+  e22 = block_sum_d(e22, red);
+  e1r = block_sum_d(e1r, red);
+  e2r = block_sum_d(e2r, red);
+  if (threadIdx.x == 0) {
+    out[2 * M] = e11;
+    out[2 * M + 1] = e22;
+    out[2 * M + 2] = e1r;
+    out[2 * M + 3] = e2r;
+  }
+}
+
+// RSS of basis + pair for every candidate; then (one CTA) the chosen candidate by R28's tie rule:
+// the lowest index among those within tol * TSS of the minimum (candidates are in (v, t) order).
+__global__ void k_mars_rss(const double* __restrict__ sums, int SW, int M, int K, double rss0,
+                           double* __restrict__ rss) {
+  const int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= K) return;
+  const double* s = sums + (int64_t)c * SW;
+  double g11 = s[2 * M], g22 = s[2 * M + 1], g12 = 0.0;
+  const double n11 = g11, n22 = g22;
+  for (int j = 0; j < M; ++j) {
+    g11 -= s[2 * j] * s[2 * j];
+    g22 -= s[2 * j + 1] * s[2 * j + 1];
+    g12 -= s[2 * j] * s[2 * j + 1];
+  }
+  const double b1 = s[2 * M + 2], b2 = s[2 * M + 3];
+  const bool ok1 = g11 > 1e-10 * n11 && n11 > 0.0, ok2 = g22 > 1e-10 * n22 && n22 > 0.0;
+  double drop = 0.0;
+  if (ok1 && ok2) {
+    const double det = g11 * g22 - g12 * g12;
+    drop = det > 1e-12 * g11 * g22 ? (g22 * b1 * b1 - 2.0 * g12 * b1 * b2 + g11 * b2 * b2) / det
+                                   : fmax(b1 * b1 / g11, b2 * b2 / g22);
+  } else if (ok1) {
+    drop = b1 * b1 / g11;
+  } else if (ok2) {
+    drop = b2 * b2 / g22;
+  }
+  rss[c] = fmax(rss0 - drop, 0.0);
+}
+
+__global__ void k_mars_pick(const double* __restrict__ rss, int K, double tolabs, int* __restrict__ pick,
+                            double* __restrict__ prss) {
+  __shared__ double sm[MNT];
+  __shared__ int si[MNT];
+  double m = 1e308;
+  for (int c = threadIdx.x; c < K; c += MNT) m = fmin(m, rss[c]);
+  sm[threadIdx.x] = m;
+  __syncthreads();
+  for (int s = MNT / 2; s > 0; s >>= 1) {
+    if (threadIdx.x < s) sm[threadIdx.x] = fmin(sm[threadIdx.x], sm[threadIdx.x + s]);
+    __syncthreads();
+  }
+  const double lim = sm[0] + tolabs;
+  __syncthreads();
+  int best = K;
+  for (int c = threadIdx.x; c < K; c += MNT)
+    if (rss[c] <= lim) {
+      best = c;
+      break;
+    }
+  si[threadIdx.x] = best;
+  __syncthreads();
+  for (int s = MNT / 2; s > 0; s >>= 1) {
+    if (threadIdx.x < s) si[threadIdx.x] = min(si[threadIdx.x], si[threadIdx.x + s]);
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    *pick = si[0] < K ? si[0] : -1;
+    *prss = si[0] < K ? rss[si[0]] : 0.0;
+  }
+}
+
+// Append column `col` (hinge of candidate c, direction dir; dir 0 = the intercept) to B, and to Q after two
+// Gram-Schmidt passes unless it lies in span(Q); then r -= q (q . r).  One CTA (n is the counter-model size).
+__global__ void __launch_bounds__(MNT) k_mars_append(const double* __restrict__ X, int64_t ldx, int64_t n, int v,
+                                                    double t, int dir, double* __restrict__ B, int mb,
+                                                    double* __restrict__ Q, int* __restrict__ Mq, double* __restrict__ r,
+                                                    double* __restrict__ w) {
+  __shared__ double red[MNT / 32];
+  __shared__ double dots[GMAXK];
+  const double* x = X + (int64_t)v * ldx;
+  const int M = *Mq;
+  double nn = 0.0;
+  for (int64_t i = threadIdx.x; i < n; i += MNT) {
+    const double h = dir == 0 ? 1.0 : dir > 0 ? fmax(x[i] - t, 0.0) : fmax(t - x[i], 0.0);
+    B[(int64_t)mb * n + i] = h;
+    w[i] = h;
+    nn += h * h;
+  }
+  nn = block_sum_d(nn, red);
+  for (int pass = 0; pass < 2; ++pass) {
+    for (int j = 0; j < M; ++j) {
+      double s = 0.0;
+      for (int64_t i = threadIdx.x; i < n; i += MNT) s += Q[(int64_t)j * n + i] * w[i];
+      s = block_sum_d(s, red);
+      if (threadIdx.x == 0) dots[j] = s;
+    }
+    __syncthreads();
+    for (int64_t i = threadIdx.x; i < n; i += MNT) {
+      double wi = w[i];
+      for (int j = 0; j < M; ++j) wi -= dots[j] * Q[(int64_t)j * n + i];
+      w[i] = wi;
+    }
+    __syncthreads();
+  }
+  double qq = 0.0;
+  for (int64_t i = threadIdx.x; i < n; i += MNT) qq += w[i] * w[i];
+  qq = block_sum_d(qq, red);
+  if (!(qq > 1e-20 * nn) || nn == 0.0) return;  // in span(Q): B keeps the column, Q does not grow
+  const double inv = 1.0 / sqrt(qq);
+  double qr = 0.0;
+  for (int64_t i = threadIdx.x; i < n; i += MNT) {
+    const double q = w[i] * inv;
+    Q[(int64_t)M * n + i] = q;
+    qr += q * r[i];
+  }
+  qr = block_sum_d(qr, red);
+  for (int64_t i = threadIdx.x; i < n; i += MNT) r[i] -= Q[(int64_t)M * n + i] * qr;
+  __syncthreads();
+  if (threadIdx.x == 0) *Mq = M + 1;
+}
+
+__global__ void k_mars_rss_direct(const double* __restrict__ r, int64_t n, double* __restrict__ out) {
+  __shared__ double red[MNT / 32];
+  double s = 0.0;
+  for (int64_t i = threadIdx.x; i < n; i += MNT) s += r[i] * r[i];
+  s = block_sum_d(s, red);
+  if (threadIdx.x == 0) *out = s;
+}
+
+// Backward pass (one CTA).  With the forward pass's orthonormal Q (Mq columns) and R = Q^T B, d = Q^T y,
+// RSS(S) = RSS_perp + min_c || d - R_S c ||^2 (B = Q R, y = Q d + r_perp), a least-squares problem of at most
+// 32 x 31 solved by Householder QR with column skipping (a column whose remaining norm is below 1e-12 of its
+// norm is dependent: the rank-deficient least squares of the oracle).  No normal equations: the RSS of
+// nearly dependent subsets (hinge pairs at close knots) stays accurate, so R28's tie rules decide the same
+// way as the oracle's lstsq.  Each step, thread j evaluates the removal of term j (its own local scratch).
+__device__ double qr_subset_rss(const double* Rm, const double* dv, int Mq, int M, unsigned mask, double* A, double* b,
+                                double* coef) {
+  int cols[GMAXK], k = 0;
+  for (int j = 0; j < M; ++j)
+    if ((mask >> j) & 1u) cols[k++] = j;
+  for (int c = 0; c < k; ++c)
+    for (int i = 0; i < Mq; ++i) A[c * GMAXK + i] = Rm[(int64_t)cols[c] * Mq + i];
+  for (int i = 0; i < Mq; ++i) b[i] = dv[i];
+  int r = 0;
+  int piv[GMAXK];
+  for (int c = 0; c < k; ++c) {
+    double cn = 0.0, nr = 0.0;
+    for (int i = 0; i < Mq; ++i) cn += A[c * GMAXK + i] * A[c * GMAXK + i];
+    for (int i = r; i < Mq; ++i) nr += A[c * GMAXK + i] * A[c * GMAXK + i];
+    piv[c] = -1;
+    if (r >= Mq || !(nr > 1e-24 * cn) || cn == 0.0) continue;  // dependent column
+    const double alpha = A[c * GMAXK + r] > 0.0 ? -sqrt(nr) : sqrt(nr);
+    const double v0 = A[c * GMAXK + r] - alpha;
+    const double vnorm2 = nr - A[c * GMAXK + r] * A[c * GMAXK + r] + v0 * v0;
+    // reflect columns c.. and b with v = (v0, A[r+1.., c])
+    for (int c2 = c; c2 < k; ++c2) {
+      double t = v0 * A[c2 * GMAXK + r];
+      for (int i = r + 1; i < Mq; ++i) t += A[c * GMAXK + i] * A[c2 * GMAXK + i];
+      if (c2 == c) continue;
+      t = 2.0 * t / vnorm2;
+      A[c2 * GMAXK + r] -= t * v0;
+      for (int i = r + 1; i < Mq; ++i) A[c2 * GMAXK + i] -= t * A[c * GMAXK + i];
+    }
+    {
+      double t = v0 * b[r];
+      for (int i = r + 1; i < Mq; ++i) t += A[c * GMAXK + i] * b[i];
+      t = 2.0 * t / vnorm2;
+      b[r] -= t * v0;
+      for (int i = r + 1; i < Mq; ++i) b[i] -= t * A[c * GMAXK + i];
+    }
+    A[c * GMAXK + r] = alpha;
+    piv[c] = r;
+    ++r;
+  }
+  double res = 0.0;
+  for (int i = r; i < Mq; ++i) res += b[i] * b[i];
+  if (coef) {  // back substitution over the kept columns (rows piv[c]); dependent columns get 0
+    for (int c = 0; c < k; ++c) coef[cols[c]] = 0.0;
+    for (int c = k - 1; c >= 0; --c) {
+      if (piv[c] < 0) continue;
+      const int rr = piv[c];
+      double t = b[rr];
+      for (int c2 = c + 1; c2 < k; ++c2)
+        if (piv[c2] >= 0) t -= A[c2 * GMAXK + rr] * coef[cols[c2]];
+      coef[cols[c]] = t / A[c * GMAXK + rr];
+    }
+  }
+  return res;
+}
+
+// qty: Q^T [B | y] as an Mq x (M + 1) column-major block (column M = Q^T y); rss_perp = || y - Q Q^T y ||^2.
+__global__ void k_mars_backward(const double* __restrict__ qty, int Mq, int M, double rss_perp, double tss, int64_t n,
+                                double penalty, double* __restrict__ scratch, unsigned* __restrict__ best_mask,
+                                double* __restrict__ coef) {
+  __shared__ double rj[GMAXK];
+  __shared__ unsigned sS, sbest;
+  __shared__ double sbg;
+  const int tid = threadIdx.x;
+  const double tol = 1e-12 * tss;
+  const double* Rm = qty;
+  const double* dv = qty + (int64_t)M * Mq;
+  auto gcv = [&](double rr, int m) {
+    const double C = m + penalty * (m - 1) / 2.0;
+    const double dd = 1.0 - C / (double)n;
+    return (rr / (double)n) / (dd * dd);
+  };
+  // per thread (global, L1-cached): GMAXK * GMAXK (A) + GMAXK (b)
+  double* myA = scratch + (size_t)tid * (GMAXK * GMAXK + GMAXK);
+  double* myb = myA + GMAXK * GMAXK;
+  if (tid == 0) {
+    sS = (M >= 32) ? 0xffffffffu : ((1u << M) - 1u);
+    sbest = sS;
+    sbg = gcv(rss_perp + qr_subset_rss(Rm, dv, Mq, M, sS, myA, myb, nullptr), M);
+  }
+  __syncthreads();
+  for (int m = M; m > 1; --m) {
+    const unsigned S = sS;
+    if (tid >= 1 && tid < M && ((S >> tid) & 1u)) rj[tid] = rss_perp + qr_subset_rss(Rm, dv, Mq, M, S & ~(1u << tid), myA, myb, nullptr);
+    __syncthreads();
+    if (tid == 0) {
+      double rmin = 1e308;
+      for (int j = 1; j < M; ++j)
+        if ((S >> j) & 1u) rmin = fmin(rmin, rj[j]);
+      int drop = -1;
+      for (int j = 1; j < M && drop < 0; ++j)
+        if (((S >> j) & 1u) && rj[j] <= rmin + tol) drop = j;
+      sS = S & ~(1u << drop);
+      const double g = gcv(rj[drop], m - 1);
+      if (g <= sbg + tol / (double)n) {
+        sbg = g;
+        sbest = sS;
+      }
+    }
+    __syncthreads();
+  }
+  if (tid == 0) {
+    double cf[GMAXK];
+    qr_subset_rss(Rm, dv, Mq, M, sbest, myA, myb, cf);
+    *best_mask = sbest;
+    for (int j = 0; j < M; ++j) coef[j] = ((sbest >> j) & 1u) ? cf[j] : 0.0;
+  }
+}
+
+// residual of the chosen model (for its RSS), and the model on new rows
+__global__ void k_mars_eval(const double* __restrict__ X, int64_t ldx, int64_t n, int nt, const int32_t* __restrict__ tv,
+                            const double* __restrict__ tk, const int32_t* __restrict__ td, const double* __restrict__ coef,
+                            const double* __restrict__ y, double* __restrict__ out) {
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  double f = 0.0;
+  for (int j = 0; j < nt; ++j) {
+    const int d = td[j];
+    const double h = d == 0 ? 1.0 : d > 0 ? fmax(X[(int64_t)tv[j] * ldx + i] - tk[j], 0.0)
+                                          : fmax(tk[j] - X[(int64_t)tv[j] * ldx + i], 0.0);
+    f += coef[j] * h;
+  }
+  out[i] = y ? y[i] - f : f;
+}
+
+__global__ void k_mars_canon(const double* __restrict__ x, int64_t n, double* __restrict__ out) {
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i < n) out[i] = __dadd_rn(x[i], 0.0);  // -0 -> +0 (R18)
+}
+__global__ void k_mars_sums(const double* __restrict__ y, int64_t n, double* __restrict__ out /* tss, yy */) {
+  __shared__ double red[MNT / 32];
+  double s = 0.0;
+  for (int64_t i = threadIdx.x; i < n; i += MNT) s += y[i];
+  s = block_sum_d(s, red);
+  const double mean = s / (double)n;
+  double t = 0.0, q = 0.0;
+  for (int64_t i = threadIdx.x; i < n; i += MNT) {
+    const double dv = y[i] - mean;
+    t += dv * dv;
+    q += y[i] * y[i];
+  }
+  t = block_sum_d(t, red);
+  q = block_sum_d(q, red);
+  if (threadIdx.x == 0) {
+    out[0] = t;
+    out[1] = q;
+  }
+}
+
 }  // namespace
+
+void mars_fit_impl(const double* X_in, int64_t ldx, int64_t n, int32_t d, const double* y_in, int32_t nk, double thresh,
+                   double penalty, int32_t* nterms, int32_t* tvar, double* tknot, int32_t* tdir, double* coef_out,
+                   double* stats, cudaStream_t s) {
+  if (nk <= 0) nk = std::min(200, std::max(20, 2 * d)) + 1;
+  BF_REQUIRE(d >= 1 && nk >= 1 && nk <= GMAXK - 1 && n >= 2, BF_EINVAL,
+             "bf_mars_fit: need d >= 1, n >= 2 and at most 31 terms (d <= 15 with the default nk)");
+  InStage Xs(X_in, sizeof(double) * (size_t)(ldx * (d - 1) + n), s), ys(y_in, sizeof(double) * (size_t)n, s);
+  const double* X = (const double*)Xs.dptr;
+  const double* y = (const double*)ys.dptr;
+  // candidate knots: the distinct values of every predictor other than its minimum and maximum
+  std::vector<int32_t> hv;
+  std::vector<double> hk;
+  {
+    DBuf<double> col(n, s), srt(n, s), uq(n, s);
+    DBuf<int> nu(1, s);
+    size_t tb1 = 0, tb2 = 0;
+    cub::DeviceRadixSort::SortKeys(nullptr, tb1, col.p, srt.p, (int)n, 0, 64, s);
+    cub::DeviceSelect::Unique(nullptr, tb2, srt.p, uq.p, nu.p, (int)n, s);
+    DBuf<char> tmp(std::max<size_t>(std::max(tb1, tb2), 16), s);
+    std::vector<double> hu;
+    for (int v = 0; v < d; ++v) {
+      k_mars_canon<<<(unsigned)ceil_div(n, 256), 256, 0, s>>>(X + (int64_t)v * ldx, n, col.p);
+      {
+        KScope ks_("cub_SortKeys", s, 0.0);
+        BF_CUDA_CHECK(cub::DeviceRadixSort::SortKeys(tmp.p, tb1, col.p, srt.p, (int)n, 0, 64, s));
+      }
+      {
+        KScope ks_("cub_Unique", s, 0.0);
+        BF_CUDA_CHECK(cub::DeviceSelect::Unique(tmp.p, tb2, srt.p, uq.p, nu.p, (int)n, s));
+      }
+      int hn = 0;
+      BF_CUDA_CHECK(cudaMemcpyAsync(&hn, nu.p, sizeof(int), cudaMemcpyDeviceToHost, s));
+      BF_CUDA_CHECK(cudaStreamSynchronize(s));
+      if (hn > 2) {
+        hu.resize(hn);
+        BF_CUDA_CHECK(cudaMemcpyAsync(hu.data(), uq.p, sizeof(double) * hn, cudaMemcpyDeviceToHost, s));
+        BF_CUDA_CHECK(cudaStreamSynchronize(s));
+        for (int k = 1; k + 1 < hn; ++k) {
+          hv.push_back(v);
+          hk.push_back(hu[k]);
+        }
+      }
+    }
+  }
+  const int K = (int)hv.size();
+  DBuf<int32_t> cvar(std::max(K, 1), s);
+  DBuf<double> cknot(std::max(K, 1), s);
+  if (K) {
+    BF_CUDA_CHECK(cudaMemcpyAsync(cvar.p, hv.data(), sizeof(int32_t) * K, cudaMemcpyHostToDevice, s));
+    BF_CUDA_CHECK(cudaMemcpyAsync(cknot.p, hk.data(), sizeof(double) * K, cudaMemcpyHostToDevice, s));
+  }
+  const int SW = 2 * nk + 4;
+  DBuf<double> B((size_t)n * (nk + 1), s), Q((size_t)n * nk, s), r(n, s), w(n, s), sums((size_t)std::max(K, 1) * SW, s),
+      crss(std::max(K, 1), s), sc(4, s), prss(1, s);
+  DBuf<int> Mq(1, s), pick(1, s);
+  const int* Mq_dev_ptr = Mq.p;
+  BF_CUDA_CHECK(cudaMemsetAsync(Mq.p, 0, sizeof(int), s));
+  BF_CUDA_CHECK(cudaMemcpyAsync(r.p, y, sizeof(double) * n, cudaMemcpyDeviceToDevice, s));
+  double hs[2];
+  {
+    KScope ks_("k_mars_sums", s, 0.0);
+    k_mars_sums<<<1, MNT, 0, s>>>(y, n, sc.p);
+  }
+  BF_CUDA_CHECK(cudaMemcpyAsync(hs, sc.p, sizeof(double) * 2, cudaMemcpyDeviceToHost, s));
+  auto append = [&](int v, double t, int dir, int mb) {
+    KScope ks_("k_mars_append", s, 0.0);
+    k_mars_append<<<1, MNT, 0, s>>>(X, ldx, n, v, t, dir, B.p, mb, Q.p, Mq.p, r.p, w.p);
+  };
+  auto rss_now = [&]() {
+    double h = 0.0;
+    k_mars_rss_direct<<<1, MNT, 0, s>>>(r.p, n, prss.p);
+    BF_CUDA_CHECK(cudaMemcpyAsync(&h, prss.p, sizeof(double), cudaMemcpyDeviceToHost, s));
+    BF_CUDA_CHECK(cudaStreamSynchronize(s));
+    return h;
+  };
+  append(0, 0.0, 0, 0);  // intercept
+  BF_CUDA_CHECK(cudaStreamSynchronize(s));
+  const double tss = hs[0];
+  double rss = rss_now();
+  std::vector<int32_t> fv{0};
+  std::vector<double> fk{0.0};
+  std::vector<int32_t> fd{0};
+  int M = 1;
+  while (M + 2 <= nk && tss > 0.0 && K > 0) {
+    int hq = 0;
+    BF_CUDA_CHECK(cudaMemcpyAsync(&hq, Mq.p, sizeof(int), cudaMemcpyDeviceToHost, s));
+    BF_CUDA_CHECK(cudaStreamSynchronize(s));
+    {
+      KScope ks_("k_mars_cand", s, 8.0 * (double)K * n * (hq + 2));
+      k_mars_cand<<<K, MNT, 0, s>>>(X, ldx, n, cvar.p, cknot.p, Q.p, hq, r.p, SW, sums.p);
+    }
+    {
+      KScope ks_("k_mars_rss", s, 0.0);
+      k_mars_rss<<<(unsigned)ceil_div(K, 128), 128, 0, s>>>(sums.p, SW, hq, K, rss, crss.p);
+    }
+    {
+      KScope ks_("k_mars_pick", s, 0.0);
+      k_mars_pick<<<1, MNT, 0, s>>>(crss.p, K, 1e-12 * tss, pick.p, prss.p);
+    }
+    BF_CUDA_CHECK(cudaGetLastError());
+    int hp = -1;
+    double hr = 0.0;
+    BF_CUDA_CHECK(cudaMemcpyAsync(&hp, pick.p, sizeof(int), cudaMemcpyDeviceToHost, s));
+    BF_CUDA_CHECK(cudaMemcpyAsync(&hr, prss.p, sizeof(double), cudaMemcpyDeviceToHost, s));
+    BF_CUDA_CHECK(cudaStreamSynchronize(s));
+    if (hp < 0 || (rss - hr) / tss < thresh) break;
+    append(hv[hp], hk[hp], 1, M);
+    append(hv[hp], hk[hp], -1, M + 1);
+    fv.insert(fv.end(), {hv[hp], hv[hp]});
+    fk.insert(fk.end(), {hk[hp], hk[hp]});
+    fd.insert(fd.end(), {1, -1});
+    M += 2;
+    rss = rss_now();
+    if (1.0 - rss / tss >= 1.0 - thresh) break;
+  }
+  // backward pass on R = Q^T B, d = Q^T y (k_glm_cross: Q^T [Q | B | y]; Q has Mq <= M columns)
+  int nq = 0;
+  BF_CUDA_CHECK(cudaMemcpyAsync(&nq, Mq_dev_ptr, sizeof(int), cudaMemcpyDeviceToHost, s));
+  BF_CUDA_CHECK(cudaStreamSynchronize(s));
+  BF_CUDA_CHECK(cudaMemcpyAsync(B.p + (size_t)M * n, y, sizeof(double) * n, cudaMemcpyDeviceToDevice, s));
+  const int nblk = (int)std::max<int64_t>(1, std::min<int64_t>(296, ceil_div(n, GROWS)));
+  const int ne = nq * (nq + M + 1);
+  DBuf<double> part((size_t)nblk * ne, s), cross(ne, s), cf(M, s), bscr((size_t)32 * (GMAXK * GMAXK + GMAXK), s);
+  DBuf<unsigned> bm(1, s);
+  {
+    KScope ks_("k_glm_cross", s, 8.0 * (double)n * (nq + M + 1));
+    k_glm_cross<<<nblk, GT, 0, s>>>(Q.p, n, n, nq, nullptr, B.p, n, M + 1, part.p);
+  }
+  k_reduce_partials<<<(unsigned)ceil_div(ne, 128), 128, 0, s>>>(part.p, nblk, ne, cross.p);
+  {
+    KScope ks_("k_mars_backward", s, 0.0);
+    k_mars_backward<<<1, 32, 0, s>>>(cross.p + (size_t)nq * nq, nq, M, rss, tss, n, penalty, bscr.p, bm.p, cf.p);
+  }
+  BF_CUDA_CHECK(cudaGetLastError());
+  unsigned hb = 0;
+  std::vector<double> hc(M);
+  BF_CUDA_CHECK(cudaMemcpyAsync(&hb, bm.p, sizeof(unsigned), cudaMemcpyDeviceToHost, s));
+  BF_CUDA_CHECK(cudaMemcpyAsync(hc.data(), cf.p, sizeof(double) * M, cudaMemcpyDeviceToHost, s));
+  BF_CUDA_CHECK(cudaStreamSynchronize(s));
+  int nt = 0;
+  for (int j = 0; j < M; ++j)
+    if ((hb >> j) & 1u) {
+      tvar[nt] = fv[j];
+      tknot[nt] = fk[j];
+      tdir[nt] = fd[j];
+      coef_out[nt] = hc[j];
+      ++nt;
+    }
+  *nterms = nt;
+  // RSS of the chosen model from its residual; GCV and RSq (R28)
+  DBuf<int32_t> dv(nt, s), dd(nt, s);
+  DBuf<double> dk(nt, s), dc(nt, s);
+  BF_CUDA_CHECK(cudaMemcpyAsync(dv.p, tvar, sizeof(int32_t) * nt, cudaMemcpyHostToDevice, s));
+  BF_CUDA_CHECK(cudaMemcpyAsync(dd.p, tdir, sizeof(int32_t) * nt, cudaMemcpyHostToDevice, s));
+  BF_CUDA_CHECK(cudaMemcpyAsync(dk.p, tknot, sizeof(double) * nt, cudaMemcpyHostToDevice, s));
+  BF_CUDA_CHECK(cudaMemcpyAsync(dc.p, coef_out, sizeof(double) * nt, cudaMemcpyHostToDevice, s));
+  {
+    KScope ks_("k_mars_eval", s, 8.0 * (double)n * (nt + 2));
+    k_mars_eval<<<(unsigned)ceil_div(n, 256), 256, 0, s>>>(X, ldx, n, nt, dv.p, dk.p, dd.p, dc.p, y, r.p);
+  }
+  const double rb = rss_now();
+  const double C = nt + penalty * (nt - 1) / 2.0, den = 1.0 - C / (double)n;
+  stats[0] = rb;
+  stats[1] = (rb / (double)n) / (den * den);
+  stats[2] = tss > 0.0 ? 1.0 - rb / tss : 1.0;
+}
+
+void mars_predict_impl(const double* X_in, int64_t ldx, int64_t m, int32_t d, int32_t nt, const int32_t* tvar,
+                       const double* tknot, const int32_t* tdir, const double* coef, double* out_in, cudaStream_t s) {
+  if (m == 0 || nt == 0) return;
+  InStage Xs(X_in, sizeof(double) * (size_t)(ldx * (d - 1) + m), s);
+  OutStage os(out_in, sizeof(double) * (size_t)m, s);
+  DBuf<int32_t> dv(nt, s), dd(nt, s);
+  DBuf<double> dk(nt, s), dc(nt, s);
+  BF_CUDA_CHECK(cudaMemcpyAsync(dv.p, tvar, sizeof(int32_t) * nt, cudaMemcpyDefault, s));
+  BF_CUDA_CHECK(cudaMemcpyAsync(dd.p, tdir, sizeof(int32_t) * nt, cudaMemcpyDefault, s));
+  BF_CUDA_CHECK(cudaMemcpyAsync(dk.p, tknot, sizeof(double) * nt, cudaMemcpyDefault, s));
+  BF_CUDA_CHECK(cudaMemcpyAsync(dc.p, coef, sizeof(double) * nt, cudaMemcpyDefault, s));
+  {
+    KScope ks_("k_mars_eval", s, 8.0 * (double)m * (nt + 1));
+    k_mars_eval<<<(unsigned)ceil_div(m, 256), 256, 0, s>>>((const double*)Xs.dptr, ldx, m, nt, dv.p, dk.p, dd.p, dc.p,
+                                                         nullptr, (double*)os.dptr);
+  }
+  BF_CUDA_CHECK(cudaGetLastError());
+  os.finish(s);
+  BF_CUDA_CHECK(cudaStreamSynchronize(s));
+}
 
 void glm_predict_impl(const double* Z_in, int64_t ldz, int64_t n, int32_t k, const double* coef_in, int32_t r,
                       double* out_in, int64_t ldo, cudaStream_t s) {

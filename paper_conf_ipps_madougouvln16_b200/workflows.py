@@ -2,14 +2,15 @@
 (SURVEY.md 8(f) NEXT-3 and NEXT-4).  Argument marshalling and selection only:
 every numerical step runs in libbf.so kernels (bf_fit, bf_predict,
 bf_oob_importance, bf_importance_finalize, bf_pca, bf_glm_gaussian,
-bf_glm_predict, bf_rank_similarity); the host picks rows and columns.
+bf_glm_predict, bf_mars_fit, bf_mars_predict, bf_rank_similarity); the host
+picks rows and columns.
 
 problem_scaling  -- P:173 ("we can use the models to generate values for the
     most influential variables from an unseen problem size for which the
     execution time will be predicted by the random forest"), P:222-224 (MM:
     80:20 split, keep the first 6-8 important variables, re-validate, model
     them as generalized linear models of the matrix size, predict unseen
-    sizes).
+    sizes), P:256 (NW: the same with MARS models, R earth).
 hardware_scaling -- P:258-274 (machine characteristics of Table 2 injected
     as predictors; train on some GPUs, predict another), P:260/P:295 (the
     importance rankings of the platforms compared: "similarity").
@@ -18,7 +19,7 @@ from __future__ import annotations
 
 import numpy as np
 
-from . import fit, glm_gaussian, glm_predict, importance_finalize, pca, rank_similarity
+from . import fit, glm_gaussian, glm_predict, importance_finalize, mars_fit, mars_predict, pca, rank_similarity
 
 
 def _torch():
@@ -42,10 +43,11 @@ def log_size_design(size) -> "object":
 
 
 def problem_scaling(X, y, size_row: int, train, test, top: int = 6, ntree: int = 500, seed: int = 0,
-                    design=log_size_design) -> dict:
+                    design=log_size_design, counter_model: str = "glm") -> dict:
     """X: (p, n) device tensor, y: (n,), size_row: the predictor holding the problem size, train/test: index
-    tensors.  Returns the retained predictors, the re-validated forest's OOB statistics, the GLM deviances,
-    the modelled counters of the test rows and the predicted test times (MSE, explained variance)."""
+    tensors.  Returns the retained predictors, the re-validated forest's OOB statistics, the counter models
+    (counter_model "glm": R26, P:224 for MM; "mars": R28, P:256 for NW), the modelled counters of the test
+    rows and the predicted test times (MSE, explained variance)."""
     torch = _torch()
     Xtr, ytr = X[:, train].contiguous(), y[train].contiguous()
     f_all = fit(Xtr, ytr, ntree=ntree, seed=seed)
@@ -57,13 +59,22 @@ def problem_scaling(X, y, size_row: int, train, test, top: int = 6, ntree: int =
     Xk = X[keep][:, train].contiguous()
     f_keep = fit(Xk, ytr, ntree=ntree, seed=seed + 1)           # re-validation on the retained set
     imp_k = inc_mse(f_keep, Xk, ytr)
-    # counters as GLMs of the problem size, predicted for the test sizes
-    Ztr = design(X[size_row, train].contiguous())
-    Zte = design(X[size_row, test].contiguous())
-    models = glm_gaussian(Ztr, X[keep_c][:, train].contiguous()) if keep_c else None
+    # counters as models of the problem size (GLM P:224 / MARS P:256), predicted for the test sizes
     Xh = torch.empty((len(keep), int(test.numel())), dtype=torch.float64, device=X.device)
-    if keep_c:
+    models = None
+    if keep_c and counter_model == "mars":
+        Str, Ste = X[size_row, train][None, :].contiguous(), X[size_row, test][None, :].contiguous()
+        models = {"mars": [mars_fit(Str, X[j, train].contiguous()) for j in keep_c]}
+        models["deviance"] = torch.tensor([m["rss"] for m in models["mars"]], dtype=torch.float64)
+        models["null_deviance"] = None
+        models["coef"] = None
+        mod = torch.stack([mars_predict(m, Ste) for m in models["mars"]])
+    elif keep_c:
+        Ztr = design(X[size_row, train].contiguous())
+        Zte = design(X[size_row, test].contiguous())
+        models = glm_gaussian(Ztr, X[keep_c][:, train].contiguous())
         mod = glm_predict(Zte, models["coef"])
+    if keep_c:
         for i, j in enumerate(keep):
             if j != size_row:
                 Xh[i] = mod[keep_c.index(j)]
@@ -76,7 +87,7 @@ def problem_scaling(X, y, size_row: int, train, test, top: int = 6, ntree: int =
     var = float(((yte - yte.mean()) ** 2).mean())
     f_keep.free()
     return {"keep": keep, "oob_mse": float(imp_k["oob_mse"]), "rsq": float(imp_k["rsq"]),
-            "deviance": None if models is None else models["deviance"],
+            "models": models, "deviance": None if models is None else models["deviance"],
             "null_deviance": None if models is None else models["null_deviance"],
             "coef": None if models is None else models["coef"], "X_model": Xh, "yhat": yh,
             "test_mse": mse, "test_explained": 1.0 - mse / var if var > 0 else float("nan")}

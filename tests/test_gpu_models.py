@@ -102,3 +102,42 @@ def test_rank_similarity_parity(p, ties):
     # identical and reversed rankings
     r1, t1 = bf.rank_similarity(dev(a), dev(a))
     assert math.isclose(r1, 1.0, rel_tol=1e-14) and math.isclose(t1, 1.0, rel_tol=1e-14)
+
+
+# ------------------------------------------------------------------ MARS (R28)
+from oracle import mars as Ms  # noqa: E402
+
+
+def _mars_cases():
+    rng = np.random.default_rng(11)
+    x = np.arange(0.0, 21.0)
+    yield "hinge", x[None, :], 3.0 + 2.0 * np.maximum(0.0, x - 5.0)
+    xs = rng.uniform(0, 10, 500)
+    yield "noisy_1d", xs[None, :], np.sin(xs) + 0.3 * xs + 0.05 * rng.normal(size=500)
+    X2 = rng.uniform(0, 10, (2, 400))
+    yield "additive_2d", X2, np.maximum(0, X2[0] - 3) + 2 * np.maximum(0, 7 - X2[1]) + 0.01 * rng.normal(size=400)
+    L = 64.0 * rng.integers(1, 129, 1500)                           # NW sequence lengths
+    yield "nw_counter", L[None, :], 1e-3 * L**1.5 + 40 * np.log(L) + rng.normal(0, 5, 1500)
+    X3 = np.stack([L, rng.integers(0, 3, 1500).astype(float), rng.uniform(0, 1, 1500)])
+    yield "nw_3pred", X3, 1e-3 * L**1.5 * (1 + 0.3 * X3[1]) + rng.normal(0, 5, 1500)
+
+
+@pytest.mark.parametrize("case", [c[0] for c in _mars_cases()])
+def test_mars_parity(case):
+    name, X, y = next(c for c in _mars_cases() if c[0] == case)
+    mo = Ms.mars_fit(X, y)
+    mg = bf.mars_fit(dev(X), dev(y))
+    to = [(0, 0.0, 0) if t is None else t for t in mo["terms"]]
+    assert mg["terms"] == to, (mg["terms"], to)
+    scale = np.abs(y).max()
+    fo, fg = Ms.mars_predict(mo, X), bf.mars_predict(mg, dev(X)).cpu().numpy()
+    assert np.all(np.abs(fg - fo) <= 1e-9 * scale)
+    tss = ((y - y.mean()) ** 2).sum()
+    assert abs(mg["rss"] - mo["rss"]) <= 1e-9 * mo["rss"] + 1e-12 * tss
+    assert abs(mg["rsq"] - mo["rsq"]) <= 1e-9
+    assert abs(mg["gcv"] - mo["gcv"]) <= 1e-9 * mo["gcv"] + 1e-12 * tss / X.shape[1]
+    # host-pointer path and new rows
+    mh = bf.mars_fit(X, y)
+    assert mh["terms"] == mg["terms"]
+    Xn = X + 0.37
+    assert np.allclose(bf.mars_predict(mg, Xn), Ms.mars_predict(mo, Xn), rtol=0, atol=1e-9 * scale)

@@ -83,3 +83,27 @@ def test_hardware_scaling_nw_matches_oracle_composition():
     rho, tau = r["similarity"][(0, 1)]
     assert math.isclose(rho, Sc.spearman(imps[0], imps[1]), rel_tol=1e-9, abs_tol=1e-12)
     assert math.isclose(tau, Sc.kendall_tau_b(imps[0], imps[1]), rel_tol=1e-9, abs_tol=1e-12)
+
+
+def test_problem_scaling_nw_with_mars_matches_oracle_composition():
+    from oracle import mars as Ms
+    Xc, L, M, y = S.gen_nw(6000)
+    g0 = M[2] == 15                                              # one GPU (GTX480 rows)
+    X = np.ascontiguousarray(np.concatenate([Xc[:, g0], L[None, g0]], axis=0))
+    yy = y[g0]
+    size_row = X.shape[0] - 1
+    unseen = np.unique(X[size_row])[3::7]
+    te_mask = np.isin(X[size_row], unseen)
+    tr, te = np.nonzero(~te_mask)[0], np.nonzero(te_mask)[0]
+    T, seed = 30, 9
+    r = W.problem_scaling(dev(X), dev(yy), size_row, dev(tr), dev(te), top=6, ntree=T, seed=seed,
+                          counter_model="mars")
+    _, imp = _oracle_inc_mse(X[:, tr], yy[tr], T, seed)
+    assert r["keep"] == list(np.argsort(-imp, kind="stable")[:6])
+    keep_c = [j for j in r["keep"] if j != size_row]
+    for j, mg in zip(keep_c, r["models"]["mars"]):
+        mo = Ms.mars_fit(X[size_row, tr][None, :], X[j, tr])
+        assert mg["terms"] == [(0, 0.0, 0) if t is None else t for t in mo["terms"]]
+    Xh = r["X_model"].cpu().numpy()
+    ofk = O.fit(np.ascontiguousarray(X[r["keep"]][:, tr]), yy[tr], ntree=T, seed=seed + 1, nthreads=8)
+    assert rel_close(r["yhat"].cpu().numpy(), ofk.predict_sum(Xh) / T, 1e-9)

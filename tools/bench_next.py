@@ -105,3 +105,17 @@ ms, st, r = timed(lambda: W.hardware_scaling(Xcd, torch.from_numpy(L).to(dev), t
 emit("NEXT-4 hardware-scaling workflow", workload="C3 (NW x 3 generations), 500 trees, train {0,1} test 2", ms=ms,
      k=r["k"], test_mse=r["test_mse"], test_explained=r["test_explained"],
      similarity={f"{k[0]}-{k[1]}": v for k, v in r["similarity"].items()}, dominant=dominant(st, 1))
+
+# NEXT-3 MARS counter models (R28): one NW counter vs sequence length, 16384 runs (C3 size)
+Lh = torch.from_numpy(L[None, :]).to(dev)
+jc = int(np.argmax([abs(np.corrcoef(np.log2(L), c)[0, 1]) for c in Xc]))  # the counter that tracks L most
+cnt = torch.from_numpy(Xc[jc]).to(dev)
+ms, st, mg = timed(lambda: bf.mars_fit(Lh, cnt), reps=1)
+from oracle import mars as Ms  # noqa: E402  (cpu_baseline leg: the oracle timed on the host, bounded sample)
+sub = np.arange(0, L.shape[0], 8)
+t0 = time.perf_counter()
+Ms.mars_fit(L[None, sub], Xc[jc][sub])
+cpu_s = time.perf_counter() - t0
+emit("NEXT-3 MARS counter model", workload=f"C3: counter {jc} vs L, n=16384 (128 distinct L)", ms=ms,
+     terms=len(mg["terms"]), rsq=mg["rsq"], dominant=dominant(st, 1),
+     cpu_oracle_s_on_1_in_8_rows=cpu_s, cpu_cores=1)
