@@ -757,7 +757,8 @@ struct TScanArgs {
 };
 
 constexpr int TSV = 9;              // entries per thread (odd: conflict-free 64-bit shared loads)
-constexpr int TUNIT = NT * TSV;     // 2304 entries per unit (18 KB bulk copy)
+constexpr int SNT = 128;            // threads of the split-scan CTA (4 CTAs per SM: independent unit pipelines)
+constexpr int TUNIT = SNT * TSV;    // 1152 entries per unit (9 KB bulk copy); measured: 64 threads / TSV 7 or 13 slower
 
 // The exact key off the unrolled scan loops (rarely reached: only where the upper bound passes the screen).
 __device__ __noinline__ double split_key_call(int64_t nk, int64_t Sk, int64_t nl, int64_t Sl) {
@@ -779,10 +780,10 @@ struct WBest {  // best exact candidate of one warp for the current unit
 // block max, and only boundaries with gU >= M get the exact S4.3 key.  Four
 // barriers per unit; each thread re-derives the block results from the
 // per-warp values, so there are no broadcast round trips.
-__global__ void __launch_bounds__(NT, 2) k_split_scan_tree(TScanArgs g) {
+__global__ void __launch_bounds__(SNT, 4) k_split_scan_tree(TScanArgs g) {
   extern __shared__ __align__(16) unsigned char dsm[];
   uint64_t* bufs = (uint64_t*)dsm;  // 2 x (TUNIT + 4)
-  constexpr int NW = NT / 32;
+  constexpr int NW = SNT / 32;
   __shared__ uint64_t bar[2];
   __shared__ int32_t smc[NW];
   __shared__ int64_t sms[NW];
@@ -2600,7 +2601,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
     const size_t tpart_smem = tpart_base + (bm_smem ? (size_t)nw * 4 : 0);
     BF_CUDA_CHECK(cudaFuncSetAttribute(k_split_scan_tree, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tscan_smem));
     int occ_ts = 0, occ_tp = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_ts, k_split_scan_tree, NT, tscan_smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_ts, k_split_scan_tree, SNT, tscan_smem);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_tp, k_partition_tree, TPNT, tpart_smem);
     const unsigned grid_tscan = (unsigned)std::max(1, occ_ts * nsm), grid_tpart = (unsigned)std::max(1, occ_tp * nsm);
     DBuf<uint64_t> E0, E1, Es;
@@ -2729,7 +2730,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
         {  // ---- a7 split search: tree-affine CTAs own whole (node, drawn feature) items
           TScanArgs ga{nc, feat.p, mtry, Bc, Ec, yq.p, tlo.p, thi.p, rec.p};
           KScope ks_("k_split_scan_tree", s, 0.0);
-          k_split_scan_tree<<<grid_tscan, NT, tscan_smem, s>>>(ga);
+          k_split_scan_tree<<<grid_tscan, SNT, tscan_smem, s>>>(ga);
         }
         if (lvl_timing) cudaEventRecord(lev[1], s);
         {
