@@ -1015,8 +1015,10 @@ struct TPartArgs {
 };
 
 constexpr int TPNT = 512;           // threads of the partition CTA (one CTA per SM: the bitmap fills shared memory)
+constexpr int TPG = 2;              // independent unit pipelines per CTA (thread groups sharing the bitmap)
+constexpr int TPGT = TPNT / TPG;    // threads per group
 constexpr int TPV = 7;
-constexpr int TPUNIT = TPNT * TPV;  // 3584 entries per unit
+constexpr int TPUNIT = TPGT * TPV;  // 1792 entries per unit
 
 __device__ __forceinline__ bool part_item_active(const Split* split, const Child* child, int node) {
   if (!split[node].split) return false;
@@ -1028,7 +1030,7 @@ __device__ __forceinline__ bool part_item_active(const Split* split, const Child
 // contiguous, and every segment has exactly al lefts), so the item is stable-partitioned as ONE stream with a
 // running left count: lefts land at f0 * al + (lefts so far), rights at f0 * ar + (rights so far).  Items of
 // about PART_ITEM_UNITS units keep the units full (only an item's last unit is partial).
-constexpr int PART_ITEM_UNITS = 8;
+constexpr int PART_ITEM_UNITS = 16;
 __host__ __device__ __forceinline__ int part_group(int a, int p) {
   const int tgt = PART_ITEM_UNITS * TPUNIT;
   return a >= tgt ? 1 : min(p, tgt / a);
@@ -1065,18 +1067,48 @@ struct PWork {
   int64_t bl, br;         // children: block offsets
 };
 
+// Group-local barrier (named barrier 1 + group over the group's TPGT threads) and exclusive scan.
+__device__ __forceinline__ void group_sync(int grp) {
+  asm volatile("bar.sync %0, %1;" ::"r"(1 + grp), "r"(TPGT) : "memory");
+}
+__device__ __forceinline__ int32_t group_excl_scan(int32_t v, int32_t* sm, int32_t& total, int grp, int lt) {
+  const int lane = lt & 31, wid = lt >> 5;
+  constexpr int nw = TPGT / 32;
+  int32_t inc = warp_incl_scan(v, lane);
+  if (lane == 31) sm[wid] = inc;
+  group_sync(grp);
+  if (wid == 0) {
+    int32_t x = lane < nw ? sm[lane] : 0;
+    x = warp_incl_scan(x, lane);
+    if (lane < nw) sm[lane] = x;
+  }
+  group_sync(grp);
+  const int32_t pre = wid ? sm[wid - 1] : 0;
+  total = sm[nw - 1];
+  group_sync(grp);
+  return pre + inc - v;
+}
+
+// The CTA's TPG thread groups share the tree's goes-right bitmap in shared memory and run independent unit
+// pipelines (own bulk-copy buffers, mbarriers and named barriers) over alternate items of the CTA's slice,
+// so one group's barrier and copy waits overlap the other group's work.
 __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
   extern __shared__ __align__(16) unsigned char dsm[];
-  uint64_t* bufs = (uint64_t*)dsm;              // 2 x (TPUNIT + 2)
+  const int tid = threadIdx.x, grp = tid / TPGT, lt = tid % TPGT;
+  uint64_t* gbase = (uint64_t*)dsm + (size_t)grp * (3 * TPUNIT + 4);
+  uint64_t* bufs = gbase;                       // 2 x (TPUNIT + 2)
   uint64_t* outb = bufs + 2 * (TPUNIT + 2);     // TPUNIT
-  uint32_t* bm = (uint32_t*)(outb + TPUNIT);    // nw words (if staged)
-  __shared__ uint64_t bar[2];
-  __shared__ int32_t sm[TPNT / 32];
-  __shared__ int s_off[2];
-  __shared__ PWork s_w[2];
-  const int tid = threadIdx.x;
+  uint32_t* bm = (uint32_t*)((uint64_t*)dsm + (size_t)TPG * (3 * TPUNIT + 4));  // nw words (if staged)
+  __shared__ uint64_t bars[TPG][2];
+  __shared__ int32_t sms[TPG][TPGT / 32];
+  __shared__ int s_offs[TPG][2];
+  __shared__ PWork s_ws[TPG][2];
+  uint64_t* bar = bars[grp];
+  int32_t* sm = sms[grp];
+  int* s_off = s_offs[grp];
+  PWork* s_w = s_ws[grp];
   const TreeSched ts = tree_sched(g.B);
-  if (tid == 0) {
+  if (lt == 0) {
     mbar_init(&bar[0]);
     mbar_init(&bar[1]);
   }
@@ -1087,26 +1119,29 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
     const int n_lo = g.tlo[b], n_hi = g.thi[b];
     if (n_lo >= n_hi) continue;
     const uint32_t* sideg = g.sideb + (int64_t)b * g.nw;
-    __syncthreads();
+    __syncthreads();  // both groups are done with the previous tree's bitmap
     if (g.bitmap_smem)
       for (int64_t w = tid; w < g.nw; w += TPNT) bm[w] = sideg[w];
+    __syncthreads();
     const uint32_t* sb = g.bitmap_smem ? bm : sideg;
-    // this CTA's work items of the tree: every C-th item of the tree's contiguous item range (k_part_items_*);
-    // an owned item yields all its units in order (so the running left count stays inside one CTA)
-    int jcur = g.ioff[n_lo] + ts.c;
+    // this group's work items of the tree: the CTA takes every C-th item of the tree's contiguous item range
+    // (k_part_items_*), its groups alternate; an owned item yields all its units in order (the running left
+    // count stays inside one group)
+    const int step = ts.C * TPG;
+    int jcur = g.ioff[n_lo] + ts.c + grp * ts.C;
     const int jend = g.ioff[n_hi];
-    // thread 0 walks the items; the map entry of the next item is loaded one item ahead and its node /
-    // children records (and the map entry after it) are prefetched into L1, so taking an item costs L1 hits
+    // the group's thread 0 walks the items; the map entry of the next item is loaded one item ahead and its
+    // node / children records (and the map entry after it) are prefetched into L1
     auto pf = [&](const void* ptr) { asm volatile("prefetch.global.L1 [%0];" ::"l"(ptr)); };
     auto pf_item = [&](int2 it) {
       pf(g.nodes + it.x);
       pf(g.child + 2 * it.x);
     };
     int2 nxt = make_int2(-1, 0);
-    if (tid == 0 && jcur < jend) {
+    if (lt == 0 && jcur < jend) {
       nxt = g.imap[jcur];
       pf_item(nxt);
-      if (jcur + ts.C < jend) pf(g.imap + jcur + ts.C);
+      if (jcur + step < jend) pf(g.imap + jcur + step);
     }
     PWork cw;
     cw.nun = 0;
@@ -1119,11 +1154,11 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
       }
       if (jcur >= jend) return false;
       const int2 it = nxt;
-      jcur += ts.C;
+      jcur += step;
       if (jcur < jend) {
         nxt = g.imap[jcur];
         pf_item(nxt);
-        if (jcur + ts.C < jend) pf(g.imap + jcur + ts.C);
+        if (jcur + step < jend) pf(g.imap + jcur + step);
       }
       const LNode nd = g.nodes[it.x];
       const Child c0 = g.child[2 * it.x], c1 = g.child[2 * it.x + 1];
@@ -1150,21 +1185,21 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
       s_off[slot] = stage_entries(bufs + (size_t)slot * (TPUNIT + 2), g.Ecur + w.base + (int64_t)w.f0 * w.a + u0, cnt,
                                   &bar[slot]);
     };
-    // thread 0 runs the item pipeline and publishes each unit's work record in s_w[slot] (slot = its buffer)
-    if (tid == 0) {
+    // the group's thread 0 runs the item pipeline and publishes each unit's record in s_w[slot]
+    if (lt == 0) {
       PWork w0;
       if (!next_mine(w0)) w0.node = -1;
       s_w[cur] = w0;
       if (w0.node >= 0) issue(w0, cur);
     }
-    __syncthreads();
+    group_sync(grp);
     if (s_w[cur].node < 0) continue;
     int64_t carry_l = 0;
     for (;;) {
-      __syncthreads();  // the other buffer and s_w slot are free
+      group_sync(grp);  // the other buffer and s_w slot are free
       const PWork w = s_w[cur];
       if (w.node < 0) break;
-      if (tid == 0) {
+      if (lt == 0) {
         PWork wn;
         if (!next_mine(wn)) wn.node = -1;
         s_w[cur ^ 1] = wn;
@@ -1176,7 +1211,7 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
       mbar_wait(&bar[cur], phase[cur]);
       phase[cur] ^= 1u;
       const uint64_t* buf = bufs + (size_t)cur * (TPUNIT + 2) + s_off[cur];
-      const int jl = tid * TPV;
+      const int jl = lt * TPV;
       uint64_t ev[TPV];
       uint32_t bw[TPV];
 #pragma unroll
@@ -1197,7 +1232,7 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
           ++c;
         }
       int32_t tot;
-      const int32_t lbl = block_excl_scan(c, sm, tot);
+      const int32_t lbl = group_excl_scan(c, sm, tot, grp, lt);
       const int al = w.al, ar = w.ar;  // lefts / rights per feature segment
       {
         int li = lbl, ri = tot + (jl - lbl);
@@ -1210,22 +1245,22 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
           }
         }
       }
-      __syncthreads();
+      group_sync(grp);
       const bool keepL = w.kl == KIND_LARGE || w.kl == KIND_SMALL;
       const bool keepR = w.kr == KIND_LARGE || w.kr == KIND_SMALL;
       const int64_t exl = carry_l, exr = (int64_t)u0 - carry_l;
       const int nl_out = tot, nr_out = cnt - nl_out;
       if (keepL) {
         uint64_t* dl = (w.kl == KIND_LARGE ? g.Enext : g.Esmall) + w.bl + (int64_t)w.f0 * al + exl;
-        for (int i = tid; i < nl_out; i += TPNT) dl[i] = outb[i];
+        for (int i = lt; i < nl_out; i += TPGT) dl[i] = outb[i];
       }
       if (keepR) {
         uint64_t* dr = (w.kr == KIND_LARGE ? g.Enext : g.Esmall) + w.br + (int64_t)w.f0 * ar + exr;
-        for (int i = tid; i < nr_out; i += TPNT) dr[i] = outb[nl_out + i];
+        for (int i = lt; i < nr_out; i += TPGT) dr[i] = outb[nl_out + i];
       }
       carry_l += tot;
       {
-        const PWork& wn = s_w[cur ^ 1];  // published before this unit's block scan barriers
+        const PWork& wn = s_w[cur ^ 1];  // published before this unit's scan barriers
         if (wn.node != w.node || wn.f0 != w.f0) carry_l = 0;
       }
       cur ^= 1;
@@ -2595,7 +2630,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
     DBuf<uint32_t> sideb((size_t)B * nw, s);
     DBuf<int32_t> tlo(B, s), thi(B, s);
     const size_t tscan_smem = sizeof(uint64_t) * 2 * (TUNIT + 4);
-    const size_t tpart_base = sizeof(uint64_t) * (3 * TPUNIT + 4);
+    const size_t tpart_base = sizeof(uint64_t) * (size_t)TPG * (3 * TPUNIT + 4);
     const int smem_optin = dyn_smem_limit(k_partition_tree);
     const bool bm_smem = getenv("BF_PART_L2") == nullptr && tpart_base + (size_t)nw * 4 <= (size_t)smem_optin;
     const size_t tpart_smem = tpart_base + (bm_smem ? (size_t)nw * 4 : 0);
