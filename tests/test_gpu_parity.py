@@ -265,3 +265,58 @@ def test_c4_full_size_sampled_trees():
     Q = S.gen_query(X, 2000)
     ys, _ = gf.predict(dev(Q))
     assert rel_close(ys.cpu().numpy(), of.predict_sum(Q), 1e-9)
+
+
+# ------------------------------------------------------------------ C4 in the bench.py launch configuration
+def test_c4_bench_configuration_sampled():
+    """The whole 1000-tree C4 forest fitted as bench.py fits it (batches of trees in flight), sampled trees
+    from the first, a middle and the last batch compared with the oracle bit for bit; predictions of the
+    10M-row query batch (generated on the device as bench.py does) checked on sampled rows against a host
+    walk of the exported forest; importance slots of the sampled trees against the oracle's."""
+    from concurrent.futures import ThreadPoolExecutor
+    from tests.helpers import compare_tree
+    X, y = S.gen_scaled()
+    p, n = X.shape
+    T, seed = 1000, S.FOREST_SEED + 4
+    Xd, yd = dev(X), dev(y)
+    gf = bf.fit(Xd, yd, ntree=T, seed=seed)
+    sample = (0, 517, 999)
+    with ThreadPoolExecutor(len(sample)) as ex:  # ctypes releases the GIL: one oracle tree per host thread
+        ofs = list(ex.map(lambda t: O.fit(X, y, ntree=T, seed=seed, tree_begin=t, tree_end=t + 1), sample))
+    e = gf.export()
+    for t, of in zip(sample, ofs):
+        lo, hi = e["tree_off"][t], e["tree_off"][t + 1]
+        compare_tree({k: e[k][lo:hi] for k in ("feature", "left", "thr_or_value", "count", "value", "drss")},
+                     of.tree(0), tag=f"tree {t}")
+    # 10M query rows drawn on the device exactly as bench.py draws them
+    m = 10_000_000
+    g = torch.Generator(device=DEV)
+    g.manual_seed(S.QUERY_SEED)
+    idx = torch.randint(0, n, (m,), device=DEV, generator=g)
+    Qd = Xd[:, idx]
+    jit = torch.rand((p, m), device=DEV, generator=g) < 0.5
+    Qd = torch.where(jit, Qd * (1.0 + 0.01 * torch.randn((p, m), device=DEV, generator=g, dtype=torch.float64)), Qd)
+    Qd = Qd.contiguous()
+    del idx, jit
+    ys, _ = gf.predict(Qd, ntree_total=T)
+    rows = np.random.default_rng(3).integers(0, m, 48)
+    Qs = Qd[:, torch.from_numpy(rows).to(DEV)].cpu().numpy()
+    got = ys[torch.from_numpy(rows).to(DEV)].cpu().numpy()
+    del Qd, ys
+    feat, left, thr, off = e["feature"], e["left"], e["thr_or_value"], e["tree_off"]
+    ref = np.zeros(len(rows))
+    for t in range(T):
+        base = off[t]
+        for r in range(len(rows)):
+            k = 0
+            while feat[base + k] >= 0:
+                k = left[base + k] + (0 if Qs[feat[base + k], r] <= thr[base + k] else 1)
+            ref[r] += thr[base + k]
+    assert rel_close(got, ref, 1e-9)
+    # importance slots of the sampled trees (S7) in the batched launch configuration
+    acc = gf.oob_importance(Xd, yd)
+    d = acc["d_slots"].cpu().numpy()
+    for t, of in zip(sample, ofs):
+        ro = of.oob_importance(X, y)
+        assert int(acc["nout_t"][t]) == int(ro["nout_t"][0])
+        assert rel_close(d[t], ro["d_slots"][0], 1e-6, atol_scale=1e-9)
