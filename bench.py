@@ -337,7 +337,8 @@ def run_ours(args):
                 "avg_launch_ms": d["ms"] / max(d["launches"], 1),
                 "issue": ncu_issue(dom)}
     kernels = {k: {"ms_per_step": v["ms"] / args.steps, "launches_per_step": v["launches"] / args.steps,
-                   "GBps": (v["bytes"] / (v["ms"] / 1e3) / 1e9) if v["ms"] > 0 and v["bytes"] > 0 else None}
+                   "GBps": (v["bytes"] / (v["ms"] / 1e3) / 1e9) if v["ms"] > 0 and v["bytes"] > 0 else None,
+                   "frac_hbm": (v["bytes"] / (v["ms"] / 1e3) / 1e9 / hbm) if v["ms"] > 0 and v["bytes"] > 0 else None}
                for k, v in sorted(stats.items(), key=lambda kv: -kv[1]["ms"]) if v["launches"] > 0}
     vis = stats.get("predict_node_visits", {}).get("bytes", 0.0)
     fbk = stats.get("predict_fp64_fallbacks", {}).get("bytes", 0.0)
