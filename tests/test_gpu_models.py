@@ -141,3 +141,35 @@ def test_mars_parity(case):
     assert mh["terms"] == mg["terms"]
     Xn = X + 0.37
     assert np.allclose(bf.mars_predict(mg, Xn), Ms.mars_predict(mo, Xn), rtol=0, atol=1e-9 * scale)
+
+
+def test_mars_edge_cases():
+    rng = np.random.default_rng(2)
+    # a constant predictor has no knots; the other carries the model
+    x = rng.uniform(0, 5, 300)
+    X = np.stack([np.full(300, 3.0), x])
+    y = np.abs(x - 2.0) + 0.01 * rng.normal(size=300)
+    mg, mo = bf.mars_fit(dev(X), dev(y)), Ms.mars_fit(X, y)
+    assert mg["terms"] == [(0, 0.0, 0) if t is None else t for t in mo["terms"]]
+    assert all(t[0] == 1 for t in mg["terms"][1:])
+    # constant response: intercept only
+    mc = bf.mars_fit(dev(X), dev(np.full(300, 7.5)))
+    assert mc["terms"] == [(0, 0.0, 0)] and abs(mc["coef"][0] - 7.5) < 1e-12 and mc["rss"] <= 1e-20
+    # two distinct values: no interior knot, intercept only
+    X2 = np.array([[0.0, 1.0, 0.0, 1.0, 1.0]])
+    m2 = bf.mars_fit(dev(X2), dev(np.array([1.0, 2.0, 1.0, 2.0, 2.0])))
+    assert m2["terms"] == [(0, 0.0, 0)]
+    # too many predictors for the default 31-term cap
+    with pytest.raises(bf.BFError) as ei:
+        bf.mars_fit(dev(rng.normal(size=(16, 50))), dev(rng.normal(size=50)))
+    assert ei.value.code == -1
+
+
+def test_glm_single_column_and_ragged_host():
+    rng = np.random.default_rng(4)
+    n = 1001
+    Z = np.ones((1, n))
+    Y = rng.normal(size=(3, n)) + np.array([[1.0], [2.0], [3.0]])
+    g = bf.glm_gaussian(Z, Y)                       # intercept-only model, host pointers
+    assert np.allclose(g["coef"][:, 0], Y.mean(axis=1), rtol=1e-13)
+    assert np.allclose(g["deviance"], g["null_deviance"], rtol=1e-12)
