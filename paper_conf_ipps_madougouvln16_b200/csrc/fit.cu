@@ -1972,6 +1972,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       __threadfence_block();
     }
     h = __shfl_sync(0xffffffffu, h, 0);
+    __syncwarp();  // orders every lane's reads of the entry after lane 0's acquire (flag + fence)
     if (h < 0) break;
     TNode nd = tq[h];
     bool have = true;
