@@ -199,14 +199,21 @@ __global__ void k_oob_scatter(const int32_t* w, int64_t n, int nchunk, const int
 }
 
 // IncNodePurity slots: sum of drss of splits on m, per local tree.
+// (per-CTA shared-memory histogram over the predictors, one global atomic per (CTA, predictor))
 __global__ void k_npur(const Node16* nodes, const double* drss, const int64_t* off, int32_t i0, int p, double* npur) {
+  extern __shared__ double hp[];  // p
   const int b = blockIdx.y;
   const int32_t i = i0 + b;
+  for (int f = threadIdx.x; f < p; f += NT) hp[f] = 0.0;
+  __syncthreads();
   const int64_t lo = off[i], hi = off[i + 1];
   for (int64_t k = lo + blockIdx.x * (int64_t)NT + threadIdx.x; k < hi; k += (int64_t)gridDim.x * NT) {
     const int f = nodes[k].feature;
-    if (f >= 0) atomicAdd(&npur[(int64_t)i * p + f], drss[k]);
+    if (f >= 0) atomicAdd(&hp[f], drss[k]);
   }
+  __syncthreads();
+  for (int f = threadIdx.x; f < p; f += NT)
+    if (hp[f] != 0.0) atomicAdd(&npur[(int64_t)i * p + f], hp[f]);
 }
 
 struct ImpArgs {
@@ -697,7 +704,7 @@ void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, co
     }
     {
       KScope ks_("k_npur", s, 0.0);
-      k_npur<<<dim3(64, Bc), NT, 0, s>>>(f->d_nodes, f->d_drss, f->d_tree_off, i0, p, npur);
+      k_npur<<<dim3(64, Bc), NT, sizeof(double) * (size_t)p, s>>>(f->d_nodes, f->d_drss, f->d_tree_off, i0, p, npur);
     }
     {
       static int pfs = 0;
