@@ -237,6 +237,7 @@ struct ImpArgs {
 };
 
 constexpr int IPT = 128;  // OOB rows per CTA (one thread each; their predictors staged in shared memory)
+constexpr int IPT_WIDE = 32;  // rows per CTA of the Node16 kernel when p is too large for a 128-row tile
 constexpr int ILP = 4;    // permuted walks interleaved per thread
 
 // One CTA = IPT consecutive OOB positions a of one tree.  The rows' predictors
@@ -246,19 +247,20 @@ constexpr int ILP = 4;    // permuted walks interleaved per thread
 // permuted value x_{O_t[pi(a)], m} come from global memory.  The first
 // occurrences of each predictor on the original path are collected ILP at a
 // time and their re-walks run interleaved (independent dependency chains).
-__global__ void __launch_bounds__(IPT) k_importance(ImpArgs g) {
-  extern __shared__ double ism[];  // sacc[p] | x tile IPT x (p|1)
+template <int TP>  // OOB rows per CTA: TP, or TP_WIDE when a 128-row fp64 tile exceeds shared memory (large p)
+__global__ void __launch_bounds__(TP) k_importance(ImpArgs g) {
+  extern __shared__ double ism[];  // sacc[p] | x tile TP x (p|1)
   double* sacc = ism;
   const int stride = g.p | 1;
   double* sx = ism + ((g.p + 1) & ~1);
-  __shared__ double serr[IPT / 32];
+  __shared__ double serr[TP / 32];
   const int b = blockIdx.y;
   const int32_t i = g.i0 + b;
   const uint32_t t = (uint32_t)(g.tree_begin + i);
   const int64_t n_o = g.nout[b];
-  const int64_t a0 = (int64_t)blockIdx.x * IPT;
+  const int64_t a0 = (int64_t)blockIdx.x * TP;
   if (a0 >= n_o) return;  // uniform per CTA
-  for (int m = threadIdx.x; m < g.p; m += IPT) sacc[m] = 0.0;
+  for (int m = threadIdx.x; m < g.p; m += TP) sacc[m] = 0.0;
   const uint32_t* Ob = g.O + (int64_t)b * g.n;
   const int64_t a = a0 + threadIdx.x;
   const bool act = a < n_o;
@@ -363,10 +365,10 @@ __global__ void __launch_bounds__(IPT) k_importance(ImpArgs g) {
   __syncthreads();
   if (threadIdx.x == 0) {
     double s = 0.0;
-    for (int j = 0; j < IPT / 32; ++j) s += serr[j];
+    for (int j = 0; j < TP / 32; ++j) s += serr[j];
     if (s != 0.0) atomicAdd(&g.e_t[i], s);
   }
-  for (int m = threadIdx.x; m < g.p; m += IPT)
+  for (int m = threadIdx.x; m < g.p; m += TP)
     if (sacc[m] != 0.0) atomicAdd(&g.d_slots[(int64_t)i * g.p + m], sacc[m]);
 }
 
@@ -678,9 +680,11 @@ void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, co
   hb_all = std::max(hb_all, 2);
   hb_all += hb_all & 1;
   DBuf<uint32_t> gtab((size_t)B * p * (6u << std::min(hb_all / 2, PH_MAX)), s);
-  const size_t smem = sizeof(double) * ((size_t)((p + 1) & ~1) + (size_t)IPT * (size_t)(p | 1));
+  size_t smem = sizeof(double) * ((size_t)((p + 1) & ~1) + (size_t)IPT * (size_t)(p | 1));
   static int ismax = 0;
-  if (!ismax) ismax = dyn_smem_limit(k_importance);
+  if (!ismax) ismax = std::min(dyn_smem_limit(k_importance<IPT>), dyn_smem_limit(k_importance<IPT_WIDE>));
+  const bool wide = smem > (size_t)ismax;
+  if (wide) smem = sizeof(double) * ((size_t)((p + 1) & ~1) + (size_t)IPT_WIDE * (size_t)(p | 1));
   BF_REQUIRE(smem <= (size_t)ismax, BF_ENOTIMPL, "bf_oob_importance: p too large for the shared-memory row tile");
   const char* force16 = getenv("BF_PREDICT_NODE16");  // same switch as predict: keep the Node16 walks
   const uint2* n8 = (force16 && force16[0] == '1') ? nullptr : nodes8_get(const_cast<bf_forest*>(f), s);
@@ -754,7 +758,10 @@ void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, co
       k_importance8<<<dim3((unsigned)ceil_div(n, IPT), Bc), IPT, smem8, s>>>(g8);
     } else {
       KScope ks_("k_importance", s, 0.0);
-      k_importance<<<dim3((unsigned)ceil_div(n, IPT), Bc), IPT, smem, s>>>(g);
+      if (wide)
+        k_importance<IPT_WIDE><<<dim3((unsigned)ceil_div(n, IPT_WIDE), Bc), IPT_WIDE, smem, s>>>(g);
+      else
+        k_importance<IPT><<<dim3((unsigned)ceil_div(n, IPT), Bc), IPT, smem, s>>>(g);
     }
     BF_CUDA_CHECK(cudaGetLastError());
   }

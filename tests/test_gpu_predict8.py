@@ -196,3 +196,21 @@ def test_importance_float_ties_vs_oracle(node16):
     assert rel_close(r["e_t"].cpu().numpy(), ro["e_t"], 1e-9)
     ds = ro["d_slots"]
     assert rel_close(r["d_slots"].cpu().numpy(), ds, 1e-6, atol_scale=1e-9)
+
+
+def test_wide_forest_uses_node16_path_and_matches_oracle():
+    """p = 300 > 256: the compact layout cannot hold the feature index, so predict and importance take the
+    Node16 kernels automatically; both still agree with the oracle."""
+    rng = np.random.default_rng(30)
+    n, p, T = 400, 300, 6
+    X = rng.normal(size=(p, n))
+    y = X[7] + 0.5 * X[280] ** 2 + 0.1 * rng.normal(size=n)
+    of = O.fit(X, y, ntree=T, seed=4, nthreads=4)
+    gf = bf.fit(dev(X), dev(y), ntree=T, seed=4)
+    Q = S.gen_query(X, 999)
+    ys, _ = _predict(gf, Q, T)
+    assert rel_close(ys, of.predict_sum(Q), 1e-9)
+    r = gf.oob_importance(dev(X), dev(y))
+    ro = of.oob_importance(X, y)
+    assert np.array_equal(r["oob_cnt"].cpu().numpy(), ro["oob_cnt"])
+    assert rel_close(r["d_slots"].cpu().numpy(), ro["d_slots"], 1e-6, atol_scale=1e-9)
