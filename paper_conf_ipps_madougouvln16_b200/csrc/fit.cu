@@ -1403,6 +1403,8 @@ struct SubArgs {
   int32_t t0;
   Pool pool;
   unsigned long long* stats;  // optional phase counters (BF_SUBTREE_STATS=1), else NULL
+  int tq_sleep_max;           // idle-warp back-off cap in ns (BF_TQ_SLEEP_MAX, default 2048)
+  int tq_bigger_first;        // continue with the child of more distinct rows (BF_TQ_BIGGER_FIRST, default 1)
 };
 
 // S4.2 mtry draw by one warp, in parallel.  Draw i picks position
@@ -1964,7 +1966,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
           break;
         } else {
           __nanosleep(ns);  // idle warp: back off so the busy warps keep the issue slots
-          ns = min(ns * 2, 2048);
+          ns = min(ns * 2, (unsigned)g.tq_sleep_max);
         }
       }
       if (h >= 0)
@@ -2231,8 +2233,10 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         cr.key = kr;
         // continue with one child in this warp, hand the sibling to the queue
         if (gl && gr) {
-          if (lane == 0) tq_push(tq, &s_alloc, &s_pending, cr);
-          nd = cl;
+          // the larger child keeps the warp (the longer remaining chain stays off the queue's hand-off latency)
+          const bool keep_r = g.tq_bigger_first && __popcll(mR) > __popcll(mL);
+          if (lane == 0) tq_push(tq, &s_alloc, &s_pending, keep_r ? cl : cr);
+          nd = keep_r ? cr : cl;
           have = true;
         } else if (gl) {
           nd = cl;
@@ -2869,6 +2873,10 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
           ga.t0 = tb;
           ga.pool = pool;
           ga.stats = nullptr;
+          static const int tq_sleep_max = getenv("BF_TQ_SLEEP_MAX") ? atoi(getenv("BF_TQ_SLEEP_MAX")) : 2048;
+          static const int tq_bigger_first = getenv("BF_TQ_BIGGER_FIRST") ? atoi(getenv("BF_TQ_BIGGER_FIRST")) : 1;
+          ga.tq_sleep_max = tq_sleep_max < 32 ? 32 : tq_sleep_max;
+          ga.tq_bigger_first = tq_bigger_first;
           static const bool want_stats = getenv("BF_SUBTREE_STATS") != nullptr;
           DBuf<unsigned long long> st;
           if (want_stats) {
