@@ -320,3 +320,32 @@ def test_c4_bench_configuration_sampled():
         ro = of.oob_importance(X, y)
         assert int(acc["nout_t"][t]) == int(ro["nout_t"][0])
         assert rel_close(d[t], ro["d_slots"][0], 1e-6, atol_scale=1e-9)
+
+
+_TQ_SCRIPT = r"""
+import sys
+sys.path.insert(0, sys.argv[1])
+import torch
+import paper_conf_ipps_madougouvln16_b200 as bf
+from paper_conf_ipps_madougouvln16_b200 import synthetic as S
+from oracle import oracle as O
+from tests.helpers import compare_forest
+X, y = S.small_random(2500, 12, seed=4242, kind="mixed")
+of = O.fit(X, y, ntree=8, nodesize=1, seed=99, nthreads=4)
+gf = bf.fit(torch.from_numpy(X).cuda(), torch.from_numpy(y).cuda(), ntree=8, nodesize=1, seed=99, small_node_max=0)
+assert compare_forest(gf, of) > 0
+print("ok")
+"""
+
+
+@pytest.mark.parametrize("env", [{"BF_TQ_BIGGER_FIRST": "0"}, {"BF_TQ_BIGGER_FIRST": "1", "BF_TQ_SLEEP_MAX": "32"}])
+def test_tiny_queue_schedule_does_not_change_the_forest(env):
+    """The subtree kernel's tiny-node queue order (which child keeps the warp, idle back-off) is scheduling only:
+    every node's split depends on its own rows and Philox key, so the forest stays bit-exact vs the oracle.
+    The switches are read once per process, hence the subprocess."""
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-c", _TQ_SCRIPT, root], env={**os.environ, **env}, cwd=root,
+                       capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0 and r.stdout.strip().endswith("ok"), r.stderr[-2000:]
