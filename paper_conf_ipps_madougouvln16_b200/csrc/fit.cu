@@ -1428,6 +1428,7 @@ __device__ __forceinline__ void warp_draw_mtry(uint64_t seed, uint32_t t, uint64
     const int i = i0 + lane;
     if (i < mtry) {
       int x = jbuf[i];
+#pragma unroll 4
       for (int k = i - 1; k >= 0; --k) {
         const int jk = jbuf[k], lk = p - 1 - k;
         x = (x == jk) ? lk : ((x == lk) ? jk : x);
