@@ -2078,7 +2078,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
           int jj = jj0;
           int32_t cw = cw0;
           int64_t cs = cs0;
-#pragma unroll 2
+#pragma unroll 1
           for (int i = i0; i < i1; ++i) {
             if (jj == 0) {
               cw = 0;
