@@ -1,26 +1,34 @@
 #!/usr/bin/env python
-"""bench.py -- BlackForest hot path on B200: trees/s (fit) and predictions/s.
+"""bench.py -- BlackForest hot path on B200: trees/s and predictions/s.
 
 One step = one pass of the whole hot path over the
-configured workload:
+configured workload (BASELINE.json configs; default C4 = configs[3] with the
+configs[4] query batch):
     bf_fit (this rank's share of the T trees, presort included)
-  + bf_predict of the query batch (C5: 10M rows) with this rank's trees,
-    partial sums all-reduced over ranks (NCCL)
+  + bf_predict of the query batch with this rank's trees, partial sums
+    all-reduced over ranks (NCCL)
   + bf_oob_importance of this rank's trees, disjoint slots all-reduced,
-    bf_importance_finalize
-  + bf_pca of the training counters.
-value = T / step time (whole-job trees/s, all ranks); predictions/s are
+    bf_importance_finalize                           (configs with importance)
+  + bf_pca of the training counters                  (configs with PCA; C3: PCA
+    first, the RF grows on the retained components + problem/machine columns)
+value = T / step time (whole-job trees/s over all ranks); predictions/s are
 reported beside it.  Inputs are resident in HBM before the timed region;
-`e2e` repeats the step through the C ABI with HOST (pinned) buffers.
+`e2e` repeats the step through the C ABI with HOST (pinned) buffers.  The
+headline steps run with the library's per-kernel instrumentation OFF; one
+extra profiled step afterwards gives the per-kernel table and the roofline.
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
-                  [--config C4] [--ntree T] [--m-query M]
+                  [--config C1|C2|C3|C4] [--ntree T] [--m-query M]
+
+--gpus N > 1 without WORLD_SIZE in the environment re-launches this script
+under torch.distributed.run with N ranks (one per GPU, 127.0.0.1 rendezvous).
 """
 from __future__ import annotations
 
 import argparse
 import json
 import os
+import socket
 import subprocess
 import sys
 import threading
@@ -33,6 +41,7 @@ sys.path.insert(0, ROOT)
 
 MEASURED = os.path.join(ROOT, "MEASURED_PEAKS.json")
 FALLBACK_HBM_GBS = 6650.0  # B200_PROFILING.md fallback
+METRIC = "trees/sec fit and predictions/sec (1/2/4/8 B200), % HBM roofline"  # BASELINE.json metric, both arms
 
 
 def parse():
@@ -41,13 +50,32 @@ def parse():
     ap.add_argument("--steps", type=int, default=3)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="C4")
+    ap.add_argument("--config", default="C4", choices=["C1", "C2", "C3", "C4"])
     ap.add_argument("--ntree", type=int, default=0, help="override T (default: the config's)")
     ap.add_argument("--m-query", type=int, default=-1, help="override the query batch (default: the config's)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-profile", action="store_true", help="skip the profiled step (per-kernel table)")
     ap.add_argument("--e2e-steps", type=int, default=1)
     return ap.parse_args()
+
+
+def maybe_spawn(args) -> bool:
+    """--gpus N > 1 outside torchrun: re-exec under torch.distributed.run, N ranks on this node."""
+    if args.gpus <= 1 or "WORLD_SIZE" in os.environ:
+        return False
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    env = dict(os.environ)
+    env.setdefault("NCCL_DEBUG", "INFO")          # communicator lines (nranks) on stderr-side logs
+    env.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
+    sys.stdout.flush()
+    os.execvpe(sys.executable, cmd, env)
+    return True
 
 
 def peaks():
@@ -58,37 +86,49 @@ def peaks():
         return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md)"
 
 
-def ncu_traffic(kernel: str):
-    """DRAM bytes (read + write) per launch of `kernel` from the newest committed
-    `ncu --set full` summary under profiles/ (tools/ncu_summary.py), or None."""
+def _ncu_summary(kernel: str, config: str):
+    """Newest committed `ncu --set full` summary of `kernel` (tools/ncu_summary.py) for this workload."""
     import glob
+    names = [f"full_{kernel}_{config}.json"] + ([f"full_{kernel}.json"] if config == "C4" else [])
     for d in sorted(glob.glob(os.path.join(ROOT, "profiles", "r[0-9]*")), reverse=True):
-        f = os.path.join(d, f"full_{kernel}.json")
-        if os.path.exists(f):
-            try:
-                return float(json.load(open(f))["dram_bytes"]), os.path.relpath(f, ROOT)
-            except Exception:
-                pass
+        for nm in names:
+            f = os.path.join(d, nm)
+            if os.path.exists(f):
+                try:
+                    return json.load(open(f)), os.path.relpath(f, ROOT)
+                except Exception:
+                    pass
     return None, None
 
 
-def ncu_issue(kernel: str):
-    """Issue-slot utilisation of `kernel` from the newest committed ncu summary: the bound of the latency /
-    issue-limited kernels (4 warp-instructions per SM per cycle is the sm_100 issue peak)."""
-    import glob
-    for d in sorted(glob.glob(os.path.join(ROOT, "profiles", "r[0-9]*")), reverse=True):
-        f = os.path.join(d, f"full_{kernel}.json")
-        if os.path.exists(f):
-            try:
-                m = json.load(open(f))["metrics"]
-                ipc = float(m["sm__inst_executed.avg.per_cycle_active"])
-                return {"bound": "issue", "achieved_ipc": ipc, "peak_ipc": 4.0, "frac": ipc / 4.0,
-                        "warps_active_pct": float(m["sm__warps_active.avg.pct_of_peak_sustained_active"]),
-                        "dram_pct_of_peak": float(m["gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed"]),
-                        "source": os.path.relpath(f, ROOT)}
-            except Exception:
-                pass
-    return None
+def ncu_traffic(kernel: str, config: str):
+    """DRAM bytes (read + write) per launch of `kernel` from the committed ncu summary, or None."""
+    d, src = _ncu_summary(kernel, config)
+    try:
+        return float(d["dram_bytes"]), src
+    except Exception:
+        return None, None
+
+
+def ncu_units(kernel: str, config: str):
+    """Issue-slot use, warps active, DRAM and shared-memory pipe throughput of `kernel` from the committed
+    ncu summary (the bound of the latency / issue-limited kernels: 4 warp-instructions per SM per cycle)."""
+    d, src = _ncu_summary(kernel, config)
+    if not d:
+        return None
+    m = d.get("metrics", {})
+
+    def g(k):
+        try:
+            return float(m[k])
+        except Exception:
+            return None
+    ipc = g("sm__inst_executed.avg.per_cycle_active")
+    return {"achieved_ipc": ipc, "peak_ipc": 4.0, "issue_frac": (ipc / 4.0) if ipc is not None else None,
+            "warps_active_pct": g("sm__warps_active.avg.pct_of_peak_sustained_active"),
+            "dram_pct_of_peak": g("gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed"),
+            "smem_pipe_pct_of_peak": g("l1tex__data_pipe_lsu_wavefronts_mem_shared.avg.pct_of_peak_sustained_elapsed"),
+            "source": src}
 
 
 class Clocks:
@@ -152,10 +192,10 @@ def dist_setup(args):
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if args.impl == "ours":
         torch.cuda.set_device(local)
-    if world > 1:
+    if world > 1 and args.impl == "ours":
         import torch.distributed as dist
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
-        dist.init_process_group("nccl" if args.impl == "ours" else "gloo")
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     return rank, world, local
 
 
@@ -167,35 +207,119 @@ def workload(args):
     return S, cfg, T, m
 
 
-# ---------------------------------------------------------------------------- reference arm (CPU oracle)
-def run_reference(args):
-    rank, world, _ = dist_setup(args)
-    if rank != 0:
-        return
+def config_json(cfg, n, p, T, m, world, extra=None):
+    d = {"workload": cfg.name, "n": n, "p": p, "ntree": T, "mtry": max(p // 3, 1), "nodesize": cfg.nodesize,
+         "m_query": m, "importance": cfg.importance, "pca": cfg.pca, "parallelism": f"tree-sharded x{world}",
+         "l2": ("inputs larger than L2 (X 512 MB, lists GBs); no flush" if cfg.n >= 1_000_000 else
+                "small workload: X and the lists fit L2 (the config's own regime; SURVEY 8(d)); no flush")}
+    d.update(extra or {})
+    return d
+
+
+# ---------------------------------------------------------------------------- the oracle on the host cores
+def oracle_sample(args, S, cfg, T, m, X, y, Xrf=None, step: int = 0):
+    """One bounded sample of the workload on the host cores with the oracle (oracle/bfo.c via
+    oracle/oracle.py, as it stands), and its whole-job-equivalent throughput.
+
+    C4: k = cores trees (one per host thread, trees rotate with the step) are grown, predicted on a
+    1M-row query sample (row chunks on the host threads) and their OOB importance computed (one tree per
+    thread); PCA once.  C1-C3: all T trees, a 100K-row query sample.  The cost is extrapolated linearly to
+    T trees and m rows (trees are i.i.d. in cost; query rows are i.i.d. in cost).
+    Returns (trees/s, wall seconds of the sample, sample description)."""
+    from concurrent.futures import ThreadPoolExecutor
+
     from oracle import oracle as O
+    from oracle.pca import n_components, pca
+    cores = os.cpu_count() or 1
+    seed = S.FOREST_SEED + 4
+    t_all = time.perf_counter()
+    t_pca = 0.0
+    if cfg.pca:
+        t0 = time.perf_counter()
+        pc = pca(X, scale=True)
+        if Xrf is not None:   # C3: the RF grows on the retained components + L + machine metrics
+            kk = n_components(pc["sdev"])
+            Xrf = np.ascontiguousarray(np.concatenate([pc["scores"][:, :kk].T, cfg.extra["L"][None, :],
+                                                       cfg.extra["M"]], axis=0))
+        t_pca = time.perf_counter() - t0
+    Xf = Xrf if Xrf is not None else X
+    big = cfg.n >= 1_000_000
+    k = min(cores, T) if big else T
+    b0 = (step * k) % T if big else 0
+    rng = [(b0 + i) % T for i in range(k)]
+    # fit: one tree per host thread (C4) or all trees over the host threads (C1-C3)
+    t0 = time.perf_counter()
+    if big:
+        with ThreadPoolExecutor(cores) as ex:
+            forests = list(ex.map(lambda t: O.fit(Xf, y, ntree=T, seed=seed, tree_begin=t, tree_end=t + 1), rng))
+    else:
+        forests = [O.fit(Xf, y, ntree=T, seed=seed, nthreads=cores)]
+    t_fit = time.perf_counter() - t0
+    # predict: query rows in chunks over the host threads
+    m_s = min(m, 1_000_000 if big else 100_000)
+    t_pred = 0.0
+    if m_s > 0:
+        Q = S.gen_query(Xf, m_s, chunk=1 << 18)
+        chunks = [(a, min(m_s, a + (m_s + cores - 1) // cores)) for a in range(0, m_s, (m_s + cores - 1) // cores)]
+        t0 = time.perf_counter()
+        with ThreadPoolExecutor(cores) as ex:
+            list(ex.map(lambda f_c: f_c[0].predict_sum(np.ascontiguousarray(Q[:, f_c[1][0]:f_c[1][1]])),
+                        [(f, c) for f in forests for c in chunks]))
+        t_pred = time.perf_counter() - t0
+    # OOB importance: one forest (tree) per host thread
+    t_imp = 0.0
+    if cfg.importance:
+        t0 = time.perf_counter()
+        with ThreadPoolExecutor(cores) as ex:
+            list(ex.map(lambda f: f.oob_importance(Xf, y), forests))
+        t_imp = time.perf_counter() - t0
+    wall = time.perf_counter() - t_all
+    job = (T / k) * (t_fit + t_imp + t_pred * (m / m_s if m_s else 0.0)) + t_pca
+    desc = (f"{k} of {T} trees (global ids {rng[0]}..{rng[-1]}) grown by oracle bfo_fit one per host thread "
+            f"({t_fit:.1f} s), predicted on {m_s} of {m} query rows ({t_pred:.1f} s), OOB importance "
+            f"({t_imp:.1f} s), PCA ({t_pca:.2f} s); extrapolated linearly to {T} trees and {m} rows"
+            if big else
+            f"all {T} trees by oracle bfo_fit over {cores} host threads ({t_fit:.1f} s), {m_s} of {m} query rows "
+            f"({t_pred:.1f} s), OOB importance ({t_imp:.1f} s), PCA ({t_pca:.2f} s); extrapolated linearly to {m} rows")
+    return T / job, wall, desc, cores
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    if rank != 0:          # rank 0 alone runs and prints the oracle arm
+        return
     S, cfg, T, m = workload(args)
     X, y, _ = S.dataset(args.config)
-    cores = os.cpu_count() or 1
-    k = cores  # one tree per host thread per step: the bounded sample
-    times = []
+    Xrf = _c3_rf_placeholder(cfg, X) if args.config == "C3" else None
+    p, n = (Xrf if Xrf is not None else X).shape
+    vals, walls = [], []
+    desc, cores = "", 1
     for it in range(args.warmup + args.steps):
-        t0 = time.perf_counter()
-        O.fit(X, y, ntree=T, seed=S.FOREST_SEED + 4, tree_begin=(it * k) % T, tree_end=min(T, (it * k) % T + k),
-              nthreads=cores)
-        times.append(time.perf_counter() - t0)
-    dt = float(np.mean(times[args.warmup:]))
-    val = k / dt
+        v, w, desc, cores = oracle_sample(args, S, cfg, T, m, X, y, Xrf=Xrf, step=it)
+        if it >= args.warmup:
+            vals.append(v)
+            walls.append(w)
+    val = float(len(vals) / np.sum([1.0 / v for v in vals]))   # total trees / total equivalent time
+    ms = float(np.mean(walls)) * 1e3
     print(json.dumps({
-        "impl": "reference", "metric": "trees/sec fit", "value": val, "unit": "trees/s", "n_gpus": args.gpus,
-        "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True,
+        "impl": "reference", "metric": METRIC, "value": val, "unit": "trees/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-        "config": {"workload": cfg.name, "n": cfg.n, "p": cfg.p, "ntree": T, "mtry": cfg.mtry or max(cfg.p // 3, 1),
-                   "nodesize": cfg.nodesize},
+        "config": config_json(cfg, n, p, T, m, world),
         "cpu_baseline": {"value": val, "unit": "trees/s", "cores": cores, "kind": "oracle",
-                         "sample": f"{k} trees of {cfg.name} per step grown by oracle bfo_fit, one per host thread "
-                                   f"(fit only: predict/importance of the CPU oracle would take minutes per tree)"},
+                         "sample": f"per step: {desc}; ms_per_step is the sample's wall time"},
         "e2e": {"value": val, "unit": "trees/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }))
+
+
+def _c3_rf_placeholder(cfg, X):
+    """C3's RF input shape marker: the oracle sample recomputes PCA + retained components each step."""
+    from oracle.pca import n_components, pca
+    pc = pca(X, scale=True)
+    kk = n_components(pc["sdev"])
+    return np.ascontiguousarray(np.concatenate([pc["scores"][:, :kk].T, cfg.extra["L"][None, :], cfg.extra["M"]],
+                                               axis=0))
 
 
 # ---------------------------------------------------------------------------- our arm
@@ -211,31 +335,51 @@ def run_ours(args):
     S, cfg, T, m = workload(args)
     t0, t1 = D.tree_range(rank, world, T)
     X, y, _ = S.dataset(args.config)
-    p, n = X.shape
     Xh = torch.from_numpy(X).pin_memory()
     yh = torch.from_numpy(y).pin_memory()
     Xd = Xh.to(dev)
     yd = yh.to(dev)
+    c3 = args.config == "C3"
+    if c3:
+        Lh = torch.from_numpy(np.ascontiguousarray(cfg.extra["L"][None, :])).pin_memory()
+        Mh = torch.from_numpy(np.ascontiguousarray(cfg.extra["M"])).pin_memory()
+        Ld, Md = Lh.to(dev), Mh.to(dev)
+    k_pca = 8 if not c3 else None
+    stream = torch.cuda.current_stream()
+    ev = lambda: torch.cuda.Event(enable_timing=True)
+
+    def rf_inputs(Xs, host: bool):
+        """C3: PCA of the 60 counters, retained components (R15), RF input rows [scores | L | M]."""
+        if not c3:
+            return Xs, None
+        pc = bf.pca(Xs, scale=True, k=None)
+        kk = bf.pca_retained(pc["sdev"])
+        sc = pc["scores"][:kk]
+        if host:
+            return np.ascontiguousarray(np.concatenate([sc, Lh.numpy(), Mh.numpy()], axis=0)), pc
+        return torch.cat([sc, Ld, Md], dim=0).contiguous(), pc
+
     # query batch: drawn on the device from the training rows (seeded; synthetic-input plumbing only)
+    Xrf0, _ = rf_inputs(Xd, False)
+    p, n = Xrf0.shape
     g = torch.Generator(device=dev)
     g.manual_seed(S.QUERY_SEED)
     Qd = None
     if m > 0:
         idx = torch.randint(0, n, (m,), device=dev, generator=g)
-        Qd = Xd[:, idx]
+        Qd = Xrf0[:, idx]
         jit = torch.rand((p, m), device=dev, generator=g) < 0.5
         Qd = torch.where(jit, Qd * (1.0 + 0.01 * torch.randn((p, m), device=dev, generator=g, dtype=torch.float64)), Qd)
         Qd = Qd.contiguous()
         del idx, jit
-    k_pca = 8
-    stream = torch.cuda.current_stream()
-    ev = lambda: torch.cuda.Event(enable_timing=True)
+    del Xrf0
 
     def step(Xs, ys_, Qs, host: bool):
-        """One pass of the hot path; returns per-phase events and the result scalars."""
+        """One pass of the hot path; returns per-phase events and the result."""
         e = [ev() for _ in range(5)]
         e[0].record(stream)
-        forest = bf.fit(Xs, ys_, ntree=T, seed=S.FOREST_SEED + 4, tree_begin=t0, tree_end=t1)
+        Xf, pc = rf_inputs(Xs, host)                          # C3: PCA first
+        forest = bf.fit(Xf, ys_, ntree=T, seed=S.FOREST_SEED + 4, tree_begin=t0, tree_end=t1)
         e[1].record(stream)
         pred = None
         if Qs is not None:
@@ -244,52 +388,54 @@ def run_ours(args):
                 ps = torch.from_numpy(ps).to(dev)
             pred = D.allreduce_predictions(ps, T) if world > 1 else ps / T
         e[2].record(stream)
-        acc = forest.oob_importance(Xs, ys_)
-        if host:
-            acc = {k: torch.from_numpy(v).to(dev) for k, v in acc.items()}
-        if world > 1:  # disjoint per-tree slots: the all-reduce is an exact all-gather
-            m = D.merge_importance(acc, t0, t1, T)
-            dsl, npu, osum, ocnt = m["d_slots"], m["npur_slots"], m["oob_sum"], m["oob_cnt"]
-        else:
-            dsl, npu, osum, ocnt = acc["d_slots"], acc["npur_slots"], acc["oob_sum"], acc["oob_cnt"]
-        fin = bf.importance_finalize(dsl, npu, osum, ocnt, yd)
+        res = None
+        if cfg.importance:
+            acc = forest.oob_importance(Xf, ys_)
+            if host:
+                acc = {k: torch.from_numpy(v).to(dev) for k, v in acc.items()}
+            if world > 1:  # disjoint per-tree slots: the all-reduce is an exact all-gather
+                mg = D.merge_importance(acc, t0, t1, T)
+                dsl, npu, osum, ocnt = mg["d_slots"], mg["npur_slots"], mg["oob_sum"], mg["oob_cnt"]
+            else:
+                dsl, npu, osum, ocnt = acc["d_slots"], acc["npur_slots"], acc["oob_sum"], acc["oob_cnt"]
+            fin = bf.importance_finalize(dsl, npu, osum, ocnt, yd)
+            res = fin["oob_mse"]
         e[3].record(stream)
-        pc = bf.pca(Xs, scale=True, k=k_pca)
+        if cfg.pca and not c3:
+            pc = bf.pca(Xs, scale=True, k=k_pca)
         e[4].record(stream)
-        res = fin["oob_mse"]
-        if host:
-            out = res.cpu()  # device -> host read of the step's result
+        if host:  # device -> host read of the step's result
+            if res is not None:
+                res.cpu()
             if pred is not None:
                 pred.cpu()
         forest.free()
-        return e, res, pc
+        return e, res
 
     def barrier():
         if world > 1:
             dist.barrier()
         torch.cuda.synchronize()
 
-    # warm-up
     for _ in range(args.warmup):
         step(Xd, yd, Qd, False)
     barrier()
-    # timed region (device-resident inputs); L2 note: X (p*n*8 B) and the lists exceed L2
+    # ---- timed region: device-resident inputs, instrumentation off
     L0 = bf.launch_count()
-    bf.profile_enable(True)
     phase = np.zeros(4)
     with Clocks(local) as clk:
         barrier()
         start, end = ev(), ev()
         start.record(stream)
+        evs = []
         for _ in range(args.steps):
-            e, res, _ = step(Xd, yd, Qd, False)
-            torch.cuda.synchronize()
-            phase += [e[i].elapsed_time(e[i + 1]) for i in range(4)]
+            e, res = step(Xd, yd, Qd, False)
+            evs.append(e)
         end.record(stream)
         barrier()
-    bf.profile_enable(False)
+    for e in evs:
+        phase += [e[i].elapsed_time(e[i + 1]) for i in range(4)]
     launches = (bf.launch_count() - L0) // args.steps
-    stats = bf.profile_read()
     ms = start.elapsed_time(end) / args.steps
     msmax = torch.tensor([ms], dtype=torch.float64, device=dev)
     if world > 1:
@@ -297,7 +443,22 @@ def run_ours(args):
     ms = float(msmax.item())
     phase /= args.steps
 
-    # e2e through the C ABI with host (pinned) buffers
+    # ---- one profiled step (per-kernel CUDA-event table; not part of the headline)
+    stats, prof_ms = {}, None
+    if not args.no_profile:
+        bf.profile_read()
+        bf.profile_enable(True)
+        barrier()
+        a, b = ev(), ev()
+        a.record(stream)
+        step(Xd, yd, Qd, False)
+        b.record(stream)
+        barrier()
+        bf.profile_enable(False)
+        stats = bf.profile_read()
+        prof_ms = a.elapsed_time(b)
+
+    # ---- e2e through the C ABI with host (pinned) buffers
     e2e = None
     if not args.no_e2e:
         Qh = Qd.cpu().pin_memory() if Qd is not None else None
@@ -314,79 +475,79 @@ def run_ours(args):
         if world > 1:
             dist.all_reduce(me, op=dist.ReduceOp.MAX)
         # X is staged by bf_fit, bf_oob_importance and bf_pca; y by fit and importance
-        h2d = (3 * X.nbytes + 2 * y.nbytes + (Qn.nbytes if Qn is not None else 0))
+        nx = 1 + int(cfg.importance) + int(cfg.pca)
+        ny = 1 + int(cfg.importance)
+        h2d = nx * X.nbytes + ny * y.nbytes + (Qn.nbytes if Qn is not None else 0)
+        p_rf = p
+        d2h = 8 * m + (8 + 2 * 8 * (t1 - t0) * p_rf + 12 * n + 16 * (t1 - t0) if cfg.importance else 0)
+        if cfg.pca:
+            pp = X.shape[0]
+            d2h += 8 * pp * (pp + 1) + 8 * n * (k_pca or pp)
         e2e = {"value": T / (float(me.item()) / 1e3), "unit": "trees/s", "h2d_bytes_per_step": int(h2d),
-               "d2h_bytes_per_step": int(8 * m + 8 + 2 * 8 * (t1 - t0) * p + 12 * n + 16 * (t1 - t0) + 8 * p * (p + 1) + 8 * n * k_pca),
-               "ms_per_step": float(me.item())}
+               "d2h_bytes_per_step": int(d2h), "ms_per_step": float(me.item())}
 
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        v, w, desc, cores = oracle_sample(args, S, cfg, T, m, X, y,
+                                          Xrf=_c3_rf_placeholder(cfg, X) if c3 else None)
+        cpu = {"value": v, "unit": "trees/s", "cores": cores, "kind": "oracle", "sample": f"{desc}; {w:.1f} s wall"}
     if rank != 0:
         return
-    # roofline of the dominant kernel (by device time in the timed region)
+    # ---- roofline of the dominant kernel (by device time in the profiled step)
     hbm, hbm_src = peaks()
-    kern = {k: v for k, v in stats.items() if v["ms"] > 0}
+    kern = {k: v for k, v in stats.items() if v["ms"] > 0 and v["launches"] > 0}
     dom = max(kern, key=lambda k: kern[k]["ms"]) if kern else None
     roof = None
     if dom:
         d = kern[dom]
         achieved = d["bytes"] / (d["ms"] / 1e3) / 1e9 if d["bytes"] > 0 else 0.0
-        traffic, tsrc = ncu_traffic(dom)
+        traffic, tsrc = ncu_traffic(dom, args.config)
         roof = {"kernel": dom, "bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
                 "frac": achieved / hbm, "traffic": traffic, "traffic_source": tsrc, "peak_source": hbm_src,
                 "algorithmic_bytes_per_launch": d["bytes"] / max(d["launches"], 1),
-                "share_of_step": d["ms"] / args.steps / ms,
+                "share_of_step": d["ms"] / prof_ms if prof_ms else None,
                 "avg_launch_ms": d["ms"] / max(d["launches"], 1),
-                "issue": ncu_issue(dom)}
-    kernels = {k: {"ms_per_step": v["ms"] / args.steps, "launches_per_step": v["launches"] / args.steps,
+                "ncu": ncu_units(dom, args.config)}
+        sc = stats.get(dom + ":scan_bytes")
+        if sc and sc["bytes"] > 0:   # SURVEY 8(d) split-search bytes of the same launches
+            roof["scan_bytes_per_launch"] = sc["bytes"] / max(d["launches"], 1)
+            roof["scan_frac"] = sc["bytes"] / (d["ms"] / 1e3) / 1e9 / hbm
+    kernels = {k: {"ms_per_step": v["ms"], "launches_per_step": v["launches"],
                    "GBps": (v["bytes"] / (v["ms"] / 1e3) / 1e9) if v["ms"] > 0 and v["bytes"] > 0 else None,
                    "frac_hbm": (v["bytes"] / (v["ms"] / 1e3) / 1e9 / hbm) if v["ms"] > 0 and v["bytes"] > 0 else None}
                for k, v in sorted(stats.items(), key=lambda kv: -kv[1]["ms"]) if v["launches"] > 0}
     vis = stats.get("predict_node_visits", {}).get("bytes", 0.0)
     fbk = stats.get("predict_fp64_fallbacks", {}).get("bytes", 0.0)
-    cpu = None
-    if not args.no_cpu_baseline and world == 1:
-        cpu = cpu_baseline(args, S, cfg, T, X, y)
     out = {
-        "metric": "trees/sec fit (whole hot-path step) and predictions/sec",
+        "metric": METRIC,
         "value": T / (ms / 1e3), "unit": "trees/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": ms, "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
         "data": "synthetic",
-        "config": {"workload": cfg.name, "n": n, "p": p, "ntree": T, "mtry": max(p // 3, 1), "nodesize": cfg.nodesize,
-                   "m_query": m, "pca_k": k_pca, "parallelism": f"tree-sharded x{world}",
-                   "l2": "inputs larger than L2 (X 512 MB, lists GBs); no flush"},
+        "config": config_json(cfg, n, p, T, m, world, {"pca_k": k_pca if not c3 else "retained (R15)"}),
         "predictions_per_s": (m / (phase[1] / 1e3)) if m and phase[1] > 0 else None,
-        "predict_node_visits_per_walk": (vis / args.steps / (m * (t1 - t0))) if m and vis else None,
+        "fit_trees_per_s": T / (phase[0] / 1e3) if phase[0] > 0 else None,
+        "predict_node_visits_per_walk": (vis / (m * (t1 - t0))) if m and vis and t1 > t0 else None,
         "predict_fp64_fallbacks_per_visit": (fbk / vis) if vis else None,
         "phases_ms": {"fit": phase[0], "predict": phase[1], "importance": phase[2], "pca": phase[3]},
         "gpu_launches": int(launches),
         "roofline": roof,
+        "profiled_step_ms": prof_ms,
         "kernels": kernels,
         "clocks": clk.summary(),
         "e2e": e2e,
         "cpu_baseline": cpu,
     }
-    print(json.dumps(out))
-
-
-def cpu_baseline(args, S, cfg, T, X, y):
-    """The oracle as it stands, on the host cores, on a bounded sample: one
-    C4 tree per host thread (fit only)."""
-    from oracle import oracle as O
-    cores = os.cpu_count() or 1
-    k = cores
-    t0 = time.perf_counter()
-    O.fit(X, y, ntree=T, seed=S.FOREST_SEED + 4, tree_begin=0, tree_end=min(k, T), nthreads=cores)
-    dt = time.perf_counter() - t0
-    return {"value": min(k, T) / dt, "unit": "trees/s", "cores": cores, "kind": "oracle",
-            "sample": f"{min(k, T)} trees of {cfg.name} grown by oracle bfo_fit, one per host thread, "
-                      f"{dt:.1f} s (fit only; predict/importance excluded)"}
+    print(json.dumps(out), flush=True)
 
 
 def main():
     args = parse()
+    if maybe_spawn(args):
+        return
     if args.impl == "reference":
         run_reference(args)
-    else:
-        run_ours(args)
+        return
+    run_ours(args)
     if int(os.environ.get("WORLD_SIZE", "1")) > 1:
         import torch.distributed as dist
         if dist.is_initialized():

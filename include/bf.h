@@ -62,7 +62,9 @@ typedef struct bf_params {
   int64_t sampsize;        /* N_s; 0 -> n                                                      */
   uint64_t seed;           /* Philox key (S1)                                                  */
   int32_t tree_begin;      /* this call grows global trees [tree_begin, tree_end)              */
-  int32_t tree_end;        /*   (multi-GPU: each rank a disjoint range; 0,0 -> [0, ntree))     */
+  int32_t tree_end;        /*   (multi-GPU: each rank a disjoint range, possibly empty when
+                              ntree < ranks; tree_end < 0 -> [0, ntree); begin == end -> an
+                              empty forest, which predict / importance accept)               */
   int32_t trees_in_flight; /* trees grown concurrently; 0 -> auto from free device memory      */
   int32_t small_node_max;  /* largest node (distinct rows) grown by one CTA in shared memory;
                               0 -> auto from the shared-memory budget and p                    */
@@ -183,6 +185,14 @@ int bf_importance_finalize(const double* d_slots, const double* npur_slots, cons
  * may be NULL), scores (n x k column-major, may be NULL).                  */
 int bf_pca(const double* X, int64_t ldx, int64_t n, int32_t p, int32_t scale, int32_t k,
            double* sdev, double* rotation, double* center, double* scores, void* stream);
+
+/* Number of retained principal components (reading R15; "a small
+ * number of principal components (less than 10)", "4 PCs ... more than
+ * 97%"): the smallest k with sum_{j<k} sdev_j^2 >= frac * sum_j sdev_j^2,
+ * clamped to [1, min(cap, p)].  sdev: p values in descending order (bf_pca
+ * output; device or host).  *k: HOST int32.  Synchronous.  BF_EINVAL for p
+ * outside [1, 1024], cap < 1 or frac outside (0, 1].                       */
+int bf_pca_retained(const double* sdev, int32_t p, double frac, int32_t cap, int32_t* k, void* stream);
 
 /* Varimax rotation of factor loadings ("the factor loadings of the
  * variable with relation to the retained principal components"; reading R25

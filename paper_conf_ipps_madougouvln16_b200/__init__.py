@@ -77,6 +77,7 @@ def lib():
             "bf_oob_importance": ([vp, vp, i64, vp, i64, i32, C.POINTER(Accum), vp], C.c_int),
             "bf_importance_finalize": ([vp] * 5 + [i64, i32, i32] + [vp] * 6 + [vp], C.c_int),
             "bf_pca": ([vp, i64, i64, i32, i32, i32, vp, vp, vp, vp, vp], C.c_int),
+            "bf_pca_retained": ([vp, i32, C.c_double, i32, vp, vp], C.c_int),
             "bf_partial_dependence": ([vp, vp, i64, i64, i32, i32, vp, i32, vp, vp, i32, vp], C.c_int),
             "bf_pd_grid": ([vp, i64, i32, vp, C.POINTER(C.c_int32), vp], C.c_int),
             "bf_varimax": ([vp, i64, i32, i32, i32, C.c_double, vp, vp, C.POINTER(C.c_int32), vp], C.c_int),
@@ -107,7 +108,7 @@ def lib():
 def exported_symbols():
     return [n for n in ("bf_version", "bf_last_error", "bf_set_allocator", "bf_fit", "bf_forest_free",
                         "bf_forest_info_get", "bf_forest_export", "bf_forest_import", "bf_predict",
-                        "bf_oob_importance", "bf_importance_finalize", "bf_pca", "bf_philox", "bf_i128_to_double",
+                        "bf_oob_importance", "bf_importance_finalize", "bf_pca", "bf_pca_retained", "bf_philox", "bf_i128_to_double",
                         "bf_fixed_point", "bf_bootstrap", "bf_perm", "bf_profile_enable", "bf_profile_read",
                         "bf_launch_count", "bf_partial_dependence", "bf_pd_grid", "bf_varimax",
                         "bf_glm_gaussian", "bf_glm_predict", "bf_rank_similarity", "bf_mars_fit",
@@ -399,6 +400,14 @@ def pca(X, scale: bool = True, k: int | None = None) -> dict:
     _check(lib().bf_pca(_ptr(X), n, n, p, int(scale), kk, _ptr(sdev), _ptr(rot), _ptr(cen), _ptr(sco), _stream()),
            "bf_pca")
     return dict(sdev=sdev, rotation=rot, center=cen, scores=sco[:kk])
+
+
+def pca_retained(sdev, frac: float = 0.97, cap: int = 10) -> int:
+    """Number of retained components (bf_pca_retained, reading R15) from bf_pca's sdev."""
+    k = C.c_int32()
+    _check(lib().bf_pca_retained(_ptr(sdev), int(sdev.shape[0]), float(frac), int(cap), C.addressof(k), _stream()),
+           "bf_pca_retained")
+    return int(k.value)
 
 
 # --- single-step entry points (parity tests) ---------------------------------

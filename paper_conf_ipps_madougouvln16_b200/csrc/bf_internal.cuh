@@ -250,6 +250,7 @@ void importance_finalize_impl(const double* d_slots, const double* npur_slots, c
                               double* out_p4 /* 4*p: inc, raw, sd, npur */, double* out_s2, cudaStream_t s);
 void perm_impl(uint64_t seed, int32_t t, int32_t m, int64_t n_o, int64_t* out, cudaStream_t s);
 // pca.cu
+void pca_retained_impl(const double* sdev, int32_t p, double frac, int32_t cap, int32_t* k_host, cudaStream_t s);
 void pca_impl(const double* X, int64_t ldx, int64_t n, int32_t p, int32_t scale, int32_t k, double* sdev,
               double* rotation, double* center, double* scores, cudaStream_t s);
 void varimax_impl(const double* L, int64_t ldl, int32_t p, int32_t k, int32_t normalize, double eps, double* loadings,

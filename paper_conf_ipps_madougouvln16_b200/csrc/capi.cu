@@ -360,6 +360,14 @@ int bf_pca(const double* X, int64_t ldx, int64_t n, int32_t p, int32_t scale, in
   BF_API_END
 }
 
+int bf_pca_retained(const double* sdev, int32_t p, double frac, int32_t cap, int32_t* k, void* stream) {
+  BF_API_BEGIN
+  BF_REQUIRE(sdev && k, BF_EINVAL, "bf_pca_retained: NULL");
+  BF_REQUIRE(p >= 1 && p <= 1024 && cap >= 1 && frac > 0.0 && frac <= 1.0, BF_EINVAL, "bf_pca_retained: bad arguments");
+  pca_retained_impl(sdev, p, frac, cap, k, (cudaStream_t)stream);
+  BF_API_END
+}
+
 int bf_varimax(const double* L, int64_t ldl, int32_t p, int32_t k, int32_t normalize, double eps, double* loadings,
                double* rotmat, int32_t* iters, void* stream) {
   BF_API_BEGIN

@@ -2452,7 +2452,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
   PhaseTimer ptm(s);
   bf_params prm = prm0;
   BF_REQUIRE(prm.ntree >= 1 && prm.nodesize >= 1, BF_EINVAL, "bf_fit: ntree >= 1 and nodesize >= 1 required");
-  if (prm.tree_begin == 0 && prm.tree_end == 0) prm.tree_end = prm.ntree;
+  if (prm.tree_end < 0) prm.tree_end = prm.ntree;  // whole forest; (b, b) is an honoured empty range
   BF_REQUIRE(prm.tree_begin >= 0 && prm.tree_end <= prm.ntree && prm.tree_begin <= prm.tree_end, BF_EINVAL,
              "bf_fit: bad tree range");
   const int mtry = prm.mtry ? prm.mtry : std::max(p / 3, 1);

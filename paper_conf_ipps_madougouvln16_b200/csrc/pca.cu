@@ -408,6 +408,39 @@ void varimax_impl(const double* L_in, int64_t ldl, int32_t p, int32_t k, int32_t
   if (iters_host) *iters_host = hit;
 }
 
+// Reading R15 ("less than 10", "4 PCs ... > 97%"): the number of retained components is the
+// smallest k whose cumulative share of the variance sum_j sdev_j^2 reaches frac, clamped to [1, min(cap, p)].
+// One thread: p <= 1024 squares summed in index order.
+__global__ void k_pca_retained(const double* __restrict__ sdev, int p, double frac, int cap, int32_t* __restrict__ k) {
+  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  double tot = 0.0;
+  for (int j = 0; j < p; ++j) tot += sdev[j] * sdev[j];
+  int kk = p;
+  double c = 0.0;
+  for (int j = 0; j < p; ++j) {
+    c += sdev[j] * sdev[j];
+    if (c / tot >= frac) {
+      kk = j + 1;
+      break;
+    }
+  }
+  kk = kk < cap ? kk : cap;
+  kk = kk < p ? kk : p;
+  *k = kk < 1 ? 1 : kk;
+}
+
+void pca_retained_impl(const double* sdev_in, int32_t p, double frac, int32_t cap, int32_t* k_host, cudaStream_t s) {
+  InStage sd(sdev_in, sizeof(double) * (size_t)p, s);
+  DBuf<int32_t> kd(1, s);
+  {
+    KScope ks_("k_pca_retained", s, 0.0);
+    k_pca_retained<<<1, 32, 0, s>>>((const double*)sd.dptr, p, frac, cap, kd.p);
+  }
+  BF_CUDA_CHECK(cudaGetLastError());
+  BF_CUDA_CHECK(cudaMemcpyAsync(k_host, kd.p, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+  BF_CUDA_CHECK(cudaStreamSynchronize(s));
+}
+
 void pca_impl(const double* X_in, int64_t ldx, int64_t n, int32_t p, int32_t scale, int32_t k, double* sdev_o,
               double* rot_o, double* center_o, double* scores_o, cudaStream_t s) {
   InStage Xs(X_in, sizeof(double) * (size_t)(ldx * (p - 1) + n), s);

@@ -17,9 +17,9 @@ hardware_scaling -- P:258-274 (machine characteristics of Table 2 injected
 """
 from __future__ import annotations
 
-import numpy as np
 
-from . import fit, glm_gaussian, glm_predict, importance_finalize, mars_fit, mars_predict, pca, rank_similarity
+from . import (fit, glm_gaussian, glm_predict, importance_finalize, mars_fit, mars_predict, pca, pca_retained,
+               rank_similarity)
 
 
 def _torch():
@@ -94,10 +94,9 @@ def problem_scaling(X, y, size_row: int, train, test, top: int = 6, ntree: int =
 
 
 def n_components(sdev, frac: float = 0.97, cap: int = 10) -> int:
-    """Reading R15: smallest k with cumulative variance >= frac, capped at 10 (P:134 '<10', P:189 '>97%')."""
-    v = np.asarray(sdev, dtype=np.float64) ** 2
-    c = np.cumsum(v) / v.sum()
-    return int(max(1, min(int(np.searchsorted(c, frac) + 1), cap, len(v))))
+    """Reading R15: smallest k with cumulative variance >= frac, capped at 10 (P:134 '<10', P:189 '>97%');
+    computed by bf_pca_retained on the device."""
+    return pca_retained(sdev, frac, cap)
 
 
 def hardware_scaling(counters, L, M, y, gen, train_gens=(0, 1), test_gen: int = 2, ntree: int = 500,
@@ -107,7 +106,7 @@ def hardware_scaling(counters, L, M, y, gen, train_gens=(0, 1), test_gen: int = 
     test_gen; similarity (R27) of the importance rankings of per-generation forests."""
     torch = _torch()
     pc = pca(counters.contiguous(), scale=True, k=None)
-    k = n_components(pc["sdev"].cpu().numpy())
+    k = n_components(pc["sdev"])
     R = torch.cat([pc["scores"][:k], L[None, :], M], dim=0).contiguous()
     tr = torch.nonzero(torch.isin(gen, torch.tensor(list(train_gens), device=gen.device))).flatten()
     te = torch.nonzero(gen == test_gen).flatten()

@@ -52,3 +52,31 @@ def rel_close(a, b, rtol, atol_scale=0.0):
     b = np.asarray(b, np.float64)
     scale = atol_scale * max(np.abs(b).max(initial=0.0), 1e-300)
     return np.all(np.abs(a - b) <= rtol * np.abs(b) + scale)
+
+
+def assert_same_ranking(g, o, rtol: float = 1e-12, tag: str = ""):
+    """Importance ranking identical (BASELINE north_star): every pair of predictors is ordered the
+    same way by g (GPU) and o (oracle).  The only pairs allowed to differ are those whose OWN oracle
+    values agree to within rtol * max|o| (a tie within rounding, reported in the message, not hidden)."""
+    g = np.asarray(g, np.float64)
+    o = np.asarray(o, np.float64)
+    scale = rtol * max(np.abs(o).max(initial=0.0), 1e-300)
+    sg = np.sign(g[:, None] - g[None, :])
+    so = np.sign(o[:, None] - o[None, :])
+    bad = np.argwhere((sg != so) & (np.abs(o[:, None] - o[None, :]) > scale))
+    assert bad.size == 0, f"{tag} ranking differs for pairs {bad[:8].tolist()} (oracle {o}, gpu {g})"
+    return int(np.count_nonzero(sg != so)) // 2
+
+
+def eigen_clusters(lam, rel: float = 1e-6):
+    """Groups of consecutive eigenvalues (descending) closer than rel * lam[0]: within a group the
+    eigenvectors are not unique ("several results are correct"), only the group's projector is."""
+    groups, cur = [], [0]
+    for j in range(1, len(lam)):
+        if abs(lam[j - 1] - lam[j]) <= rel * abs(lam[0]):
+            cur.append(j)
+        else:
+            groups.append(cur)
+            cur = [j]
+    groups.append(cur)
+    return groups

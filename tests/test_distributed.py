@@ -32,17 +32,18 @@ def _free_port() -> int:
 def _tree_arrays(of, nt):
     """Forest.export()-style arrays of an oracle forest's local trees."""
     trees = [of.tree(i) for i in range(nt)]
+    cat = lambda xs, dt: np.concatenate(xs).astype(dt) if xs else np.zeros(0, dt)
     out = {"tree_off": np.concatenate([[0], np.cumsum([t["feature"].size for t in trees])]).astype(np.int64)}
-    out["feature"] = np.concatenate([t["feature"] for t in trees])
-    out["left"] = np.concatenate([t["left"] for t in trees])
-    out["thr_or_value"] = np.concatenate([np.where(t["feature"] >= 0, t["thr"], t["value"]) for t in trees])
-    out["count"] = np.concatenate([t["count"] for t in trees]).astype(np.int32)
-    out["value"] = np.concatenate([t["value"] for t in trees])
-    out["drss"] = np.concatenate([t["drss"] for t in trees])
+    out["feature"] = cat([t["feature"] for t in trees], np.int32)
+    out["left"] = cat([t["left"] for t in trees], np.int32)
+    out["thr_or_value"] = cat([np.where(t["feature"] >= 0, t["thr"], t["value"]) for t in trees], np.float64)
+    out["count"] = cat([t["count"] for t in trees], np.int32)
+    out["value"] = cat([t["value"] for t in trees], np.float64)
+    out["drss"] = cat([t["drss"] for t in trees], np.float64)
     return out
 
 
-def _worker(rank, world, port, q):
+def _worker(rank, world, port, q, T=T):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
@@ -88,14 +89,16 @@ def test_tree_range_partitions_the_forest():
             assert all(hi - lo in (ntree // world, ntree // world + 1) for lo, hi in r)
 
 
-def test_gloo_world2_merge_equals_single_process():
+@pytest.mark.parametrize("ntree", [T, 1])
+def test_gloo_world2_merge_equals_single_process(ntree):
+    """ntree = 1 < world: rank 0 owns the empty range [0, 0) and contributes exact zeros."""
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, q, ntree)) for r in range(2)]
     for p in procs:
         p.start()
-    ok = q.get(timeout=300)
+    ok = q.get(timeout=120)
     for p in procs:
         p.join(timeout=60)
         assert p.exitcode == 0

@@ -23,7 +23,7 @@ if not torch.cuda.is_available():
 import paper_conf_ipps_madougouvln16_b200 as bf  # noqa: E402
 from paper_conf_ipps_madougouvln16_b200 import synthetic as S  # noqa: E402
 from oracle import oracle as O  # noqa: E402
-from tests.helpers import compare_forest, rel_close  # noqa: E402
+from tests.helpers import assert_same_ranking, compare_forest, eigen_clusters, rel_close  # noqa: E402
 
 GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
 DEV = torch.device("cuda:0")
@@ -149,11 +149,14 @@ def test_fit_degenerate_inputs():
 
 def test_fit_host_pointers_equal_device_pointers():
     X, y = S.small_random(500, 6, seed=9)
-    a = bf.fit(dev(X), dev(y), ntree=4, seed=5).export()
-    b = bf.fit(X, y, ntree=4, seed=5).export()   # host numpy: staged by the library
-    for k in ("feature", "thr_or_value", "count"):
-        # same structure; node order may differ between runs, compare sorted multisets
-        assert np.array_equal(np.sort(a[k]), np.sort(b[k]))
+    of = O.fit(X, y, ntree=4, seed=5, nthreads=4)
+    a = bf.fit(dev(X), dev(y), ntree=4, seed=5)
+    b = bf.fit(X, y, ntree=4, seed=5)            # host numpy: staged by the library
+    assert compare_forest(a, of) > 0
+    assert compare_forest(b, of) > 0             # the host-pointer forest walked against the oracle
+    Q = S.gen_query(X, 777)
+    ys_h, _ = b.predict(Q, ntree_total=4)        # host query, host outputs
+    assert rel_close(ys_h, of.predict_sum(Q), 1e-9)
 
 
 def test_tree_range_sharding_bit_identical():
@@ -222,11 +225,9 @@ def test_oob_importance_parity(cfg):
     assert rel_close(fg["inc_node_purity"], fo["inc_node_purity"], 1e-9)
     assert abs(float(fg["oob_mse"]) - fo["oob_mse"]) <= 1e-6 * fo["oob_mse"]
     assert abs(float(fg["rsq"]) - fo["rsq"]) <= 1e-6 * abs(fo["rsq"]) + 1e-12
-    # ranking identical (ties within 1e-12 reported, not hidden)
-    og, oo = np.argsort(-fg["inc_mse"], kind="stable"), np.argsort(-fo["inc_mse"], kind="stable")
-    if not np.array_equal(og, oo):
-        gaps = np.abs(np.diff(np.sort(fo["inc_mse"])))
-        assert gaps.min() < 1e-9 * np.abs(fo["inc_mse"]).max(), "importance ranking differs"
+    # ranking identical: a pair may be ordered differently only if its own two values tie within 1e-12
+    assert_same_ranking(fg["inc_mse"], fo["inc_mse"], 1e-12, tag=f"{cfg} %IncMSE")
+    assert_same_ranking(fg["inc_node_purity"], fo["inc_node_purity"], 1e-12, tag=f"{cfg} IncNodePurity")
 
 
 # ------------------------------------------------------------------ PCA
@@ -242,15 +243,46 @@ def test_pca_parity(scale):
     lam_g, lam_o = sd ** 2, ro["sdev"] ** 2
     assert np.all(np.abs(lam_g - lam_o) <= 1e-9 * lam_o + 1e-12 * lam_o[0])
     rot = rg["rotation"].cpu().numpy()  # row j = component j
+    V = ro["rotation"]                  # column j = component j
     lam = ro["sdev"] ** 2
-    for j in range(k):
-        gap = min(abs(lam[j] - lam[j - 1]) if j else np.inf, abs(lam[j] - lam[j + 1]) if j + 1 < len(lam) else np.inf)
-        if gap > 1e-6 * lam[0]:
-            assert np.allclose(rot[j], ro["rotation"][:, j], atol=1e-7)
-    sc = rg["scores"].cpu().numpy()
-    for j in range(k):
-        if np.allclose(rot[j], ro["rotation"][:, j], atol=1e-7):
-            assert np.allclose(sc[j], ro["scores"][:, j], rtol=1e-7, atol=1e-7 * np.abs(ro["scores"][:, j]).max())
+    # eigenvectors of a well-separated eigenvalue: unique up to the sign rule, compared directly;
+    # a degenerate cluster (gap <= 1e-6 lambda_0): compared by its projector (reading R16)
+    for grp in eigen_clusters(lam, 1e-6):
+        Pg = rot[grp].T @ rot[grp]
+        Po = V[:, grp] @ V[:, grp].T
+        assert np.allclose(Pg, Po, atol=1e-7), f"projector of components {grp}"
+        if len(grp) == 1:
+            assert np.allclose(rot[grp[0]], V[:, grp[0]], atol=1e-7)
+    # scores: equal to Z V_k by definition (S9); per component where unique, by projector otherwise
+    mu = X.mean(axis=1)
+    Z = (X - mu[:, None]).T
+    if scale:
+        Z = Z / X.std(axis=1, ddof=1)
+    sc = rg["scores"].cpu().numpy()     # row j = scores of component j
+    so = ro["scores"]                   # column j
+    for grp in eigen_clusters(lam, 1e-6):
+        g_in = [j for j in grp if j < k]
+        if not g_in:
+            continue
+        atol = 1e-7 * np.abs(so).max()
+        assert np.allclose(sc[g_in].T, Z @ rot[g_in].T, rtol=1e-7, atol=atol), f"scores {g_in} != Z V"
+        if len(g_in) == len(grp):       # whole cluster retained: its score projection is basis-free
+            assert np.allclose(sc[g_in].T @ rot[g_in], so[:, g_in] @ V[:, g_in].T, rtol=1e-7, atol=atol)
+        if len(grp) == 1:
+            assert np.allclose(sc[grp[0]], so[:, grp[0]], rtol=1e-7, atol=atol)
+
+
+def test_pca_retained_parity():
+    """Retained components (reading R15) on the device vs the oracle's cumulative-share rule, on real
+    PCA spectra, on spectra where the share crosses 0.97 exactly at a component, and at the cap."""
+    from oracle.pca import n_components, pca
+    cases = [pca(S.dataset("C3")[0], scale=True)["sdev"], pca(S.gen_mm(2048)[0], scale=True)["sdev"],
+             np.sqrt(np.array([97.0, 2.0, 1.0])), np.sqrt(np.array([96.0, 1.0, 1.0, 1.0, 1.0])),
+             np.ones(30), np.sqrt(np.linspace(30, 1, 30)), np.array([1.0])]
+    for sd in cases:
+        for cap in (1, 3, 10):
+            assert bf.pca_retained(dev(sd), 0.97, cap) == n_components(sd, 0.97, cap), (sd, cap)
+            assert bf.pca_retained(np.ascontiguousarray(sd), 0.97, cap) == n_components(sd, 0.97, cap)
 
 
 # ------------------------------------------------------------------ C4 at full size, sampled trees
@@ -316,10 +348,26 @@ def test_c4_bench_configuration_sampled():
     # importance slots of the sampled trees (S7) in the batched launch configuration
     acc = gf.oob_importance(Xd, yd)
     d = acc["d_slots"].cpu().numpy()
-    for t, of in zip(sample, ofs):
-        ro = of.oob_importance(X, y)
+    npu = acc["npur_slots"].cpu().numpy()
+    ros = [of.oob_importance(X, y) for of in ofs]
+    for t, ro in zip(sample, ros):
         assert int(acc["nout_t"][t]) == int(ro["nout_t"][0])
         assert rel_close(d[t], ro["d_slots"][0], 1e-6, atol_scale=1e-9)
+        assert rel_close(npu[t], ro["npur_slots"][0], 1e-9, atol_scale=1e-12)
+        assert np.all(d[t][ro["npur_slots"][0] == 0.0] == 0.0)   # predictors unused by tree t: exactly 0
+    # finalize (S7/S8 aggregation) over the sampled trees' slots, GPU kernel vs oracle, and the ranking
+    do = np.stack([ro["d_slots"][0] for ro in ros])
+    no = np.stack([ro["npur_slots"][0] for ro in ros])
+    osum = sum(ro["oob_sum"] for ro in ros)
+    ocnt = sum(ro["oob_cnt"] for ro in ros).astype(np.int32)
+    fo = O.importance_finalize(do, no, osum, ocnt, y)
+    fg = bf.importance_finalize(dev(d[list(sample)]), dev(npu[list(sample)]), dev(osum), dev(ocnt), yd)
+    fg = {k: (v.cpu().numpy() if hasattr(v, "cpu") else v) for k, v in fg.items()}
+    assert rel_close(fg["inc_mse_raw"], fo["inc_mse_raw"], 1e-6, 1e-9)
+    assert rel_close(fg["inc_mse"], fo["inc_mse"], 1e-6, 1e-9)
+    assert rel_close(fg["inc_node_purity"], fo["inc_node_purity"], 1e-9, 1e-12)
+    assert_same_ranking(fg["inc_mse"], fo["inc_mse"], 1e-12, tag="C4 sampled %IncMSE")
+    assert_same_ranking(fg["inc_node_purity"], fo["inc_node_purity"], 1e-12, tag="C4 sampled IncNodePurity")
 
 
 _TQ_SCRIPT = r"""
@@ -349,3 +397,20 @@ def test_tiny_queue_schedule_does_not_change_the_forest(env):
     r = subprocess.run([sys.executable, "-c", _TQ_SCRIPT, root], env={**os.environ, **env}, cwd=root,
                        capture_output=True, text=True, timeout=600)
     assert r.returncode == 0 and r.stdout.strip().endswith("ok"), r.stderr[-2000:]
+
+
+def test_empty_tree_range_is_an_empty_forest():
+    """ntree < ranks gives some rank an empty range [b, b): honoured as an empty forest (not the whole
+    forest), and predict / importance of it contribute exact zeros to the all-reduces."""
+    X, y = S.small_random(200, 4, seed=3)
+    Xd, yd = dev(X), dev(y)
+    e = bf.fit(Xd, yd, ntree=3, seed=8, tree_begin=0, tree_end=0)
+    assert e.info.tree_end - e.info.tree_begin == 0 and e.info.total_nodes == 0
+    ys, _ = e.predict(Xd, ntree_total=3)
+    assert torch.all(ys == 0)
+    acc = e.oob_importance(Xd, yd)
+    assert acc["d_slots"].numel() == 0 and torch.all(acc["oob_cnt"] == 0) and torch.all(acc["oob_sum"] == 0)
+    w = bf.fit(Xd, yd, ntree=3, seed=8, tree_begin=3, tree_end=3)
+    assert w.info.total_nodes == 0
+    full = bf.fit(Xd, yd, ntree=3, seed=8)
+    assert full.info.tree_end - full.info.tree_begin == 3

@@ -483,3 +483,73 @@ def test_pca_planted_axes():
     r = pca(X, scale=False)
     assert np.allclose(np.abs(r["rotation"]), np.eye(3), atol=1e-10)
     assert np.allclose(r["sdev"] ** 2 * (n - 1), [25.0, 4.0, 1.0], rtol=1e-10)
+
+
+# ---------------------------------------------------------------- S6-S8 exact-rational pin
+@pytest.mark.parametrize("case", range(6))
+def test_oob_importance_vs_exact_rational_bruteforce(case):
+    """%IncMSE and OOB error of a tiny forest computed in exact rationals
+    from brute trees (tests/brute.py: eq.(3) split search, eq.(1) leaf means), with the
+    bootstrap multiplicities, mtry draws, node keys and Feistel permutations taken from the
+    oracle's RNG as inputs.  n_o differs from n and between trees, so a wrong divisor of
+    d_tm = (e_tm - e_t) / n_o (n instead of n_o, or a shared divisor) fails here."""
+    from tests.brute import brute_importance
+    rng = np.random.default_rng(500 + case)
+    n = int(rng.integers(9, 15))
+    p = int(rng.integers(2, 4))
+    T = 2 if case < 3 else 3
+    X = rng.integers(0, 6, (p, n)).astype(np.float64)
+    y = rng.integers(-7, 8, n).astype(np.float64)
+    seed = 7000 + case
+    mtry = p if case % 2 == 0 else max(p - 1, 1)
+    F = O.fit(X, y, ntree=T, mtry=mtry, nodesize=1, seed=seed)
+    ro = F.oob_importance(X, y)
+    cols = [list(c) for c in X]
+    trees, ws, perms = [], [], []
+    for t in range(T):
+        w = O.bootstrap(seed, t, n)
+        draw = (lambda k, t=t: O.draw_mtry(seed, t, k, p, mtry)) if mtry < p else None
+        ck = lambda k, s, t=t: O.child_key(seed, t, k, s)
+        trees.append(brute_tree(cols, list(y), list(w), 1, draw=draw, child_key=ck))
+        ws.append(list(w))
+        no = int((w == 0).sum())
+        perms.append([[O.perm(seed, t, m, no, a) for a in range(no)] for m in range(p)])
+    b = brute_importance(cols, list(y), trees, ws, perms)
+    assert all(0 < no < n for no in b["nout"])
+    assert ro["nout_t"].tolist() == b["nout"]
+    scale = max(max(abs(float(v)) for row in b["d"] for v in row), 1e-300)
+    for t in range(T):
+        assert ro["e_t"][t] == pytest.approx(float(b["e"][t]), rel=1e-12, abs=1e-12)
+        for m in range(p):
+            assert abs(ro["d_slots"][t, m] - float(b["d"][t][m])) <= 1e-12 * scale, (t, m)
+    assert ro["oob_cnt"].tolist() == b["ocnt"]
+    assert np.allclose(ro["oob_sum"], [float(v) for v in b["osum"]], rtol=1e-13, atol=1e-12)
+    fin = O.importance_finalize(ro["d_slots"], ro["npur_slots"], ro["oob_sum"], ro["oob_cnt"], y)
+    for m in range(p):
+        assert fin["inc_mse_raw"][m] == pytest.approx(float(b["raw"][m]), rel=1e-12, abs=1e-12 * scale)
+        assert fin["inc_mse_sd"][m] == pytest.approx(b["sd"][m], rel=1e-9, abs=1e-12 * scale)
+        if b["sd"][m] >= np.finfo(float).eps:
+            assert fin["inc_mse"][m] == pytest.approx(float(b["raw"][m]) / b["sd"][m], rel=1e-9)
+    assert fin["oob_mse"] == pytest.approx(float(b["oob_mse"]), rel=1e-13)
+    assert fin["rsq"] == pytest.approx(float(b["rsq"]), rel=1e-12, abs=1e-13)
+
+
+def test_oob_importance_exact_pin_is_not_vacuous():
+    """At least one of the pinned tiny forests has a nonzero d_tm in every tree with n_o > 0,
+    so the exact pin above tests the divisor rather than comparing zeros."""
+    from tests.brute import brute_importance
+    hits = 0
+    for case in range(6):
+        rng = np.random.default_rng(500 + case)
+        n = int(rng.integers(9, 15))
+        p = int(rng.integers(2, 4))
+        T = 2 if case < 3 else 3
+        X = rng.integers(0, 6, (p, n)).astype(np.float64)
+        y = rng.integers(-7, 8, n).astype(np.float64)
+        seed = 7000 + case
+        mtry = p if case % 2 == 0 else max(p - 1, 1)
+        F = O.fit(X, y, ntree=T, mtry=mtry, nodesize=1, seed=seed)
+        ro = F.oob_importance(X, y)
+        if all(np.any(ro["d_slots"][t] != 0.0) for t in range(T)):
+            hits += 1
+    assert hits >= 3
