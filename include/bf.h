@@ -21,8 +21,9 @@
  *     cudaPointerGetAttributes and stages them through device memory on the
  *     given stream (host<->device copies are then part of the call).
  *   - The caller owns every input and output buffer; the library never frees
- *     them.  The library owns bf_forest and its device memory (allocated with
- *     cudaMallocAsync on the call's stream, or through bf_set_allocator).
+ *     them.  The library owns bf_forest and its device memory (allocated
+ *     through the bf_set_allocator hooks -- the Python binding installs the
+ *     torch caching allocator -- else cudaMallocAsync on the call's stream).
  *   - Return value: BF_OK (0) or a negative BF_E* code; no exception crosses
  *     the ABI; on error outputs are unspecified and no forest is returned.
  *     bf_last_error() returns a thread-local message for the last failure.
@@ -120,11 +121,25 @@ typedef struct bf_oob_accum {
 const char* bf_version(void);
 const char* bf_last_error(void);
 
-/* Optional allocator hook (e.g. the torch caching allocator).  NULL restores
- * cudaMallocAsync / cudaFreeAsync.                                          */
+/* Allocator hook for every device buffer the library owns (fit work space,
+ * forests, staging copies of host inputs).  alloc(bytes, stream, ctx) returns
+ * a block usable in `stream` order (NULL -> BF_ENOMEM); free(ptr, stream,
+ * ctx) returns it in the order of the stream it was allocated on.  A forest
+ * used on another stream is released only after cudaDeviceSynchronize.  The
+ * Python binding installs torch's CUDA caching allocator (libbf_torch_alloc.so:
+ * raw_alloc_with_stream / raw_delete), so the library and the caller's
+ * tensors share one pool.  NULL hooks restore cudaMallocAsync /
+ * cudaFreeAsync on the device's default memory pool.  Not thread-safe against
+ * calls in flight: set it before the first call.                           */
 typedef void* (*bf_alloc_fn)(size_t bytes, void* stream, void* ctx);
 typedef void (*bf_free_fn)(void* ptr, void* stream, void* ctx);
 int bf_set_allocator(bf_alloc_fn alloc, bf_free_fn free_, void* ctx);
+/* Free device memory the caller's allocator can still hand out (bytes; 0 =
+ * ask the driver with cudaMemGetInfo).  bf_fit sizes its trees in flight from
+ * half of it.  The Python binding passes the driver's free memory plus the
+ * torch caching allocator's cached-but-unused blocks before every fit.
+ * BF_EINVAL for a negative value.                                          */
+int bf_set_memory_budget(int64_t bytes);
 
 /* Grow global trees [tree_begin, tree_end) of a T-tree forest (P:95 steps 1-2;
  * S2-S4).  X: n x p column-major (ldx >= n), y: n.  Synchronous.  *out
@@ -254,6 +269,16 @@ int bf_mars_predict(const double* X, int64_t ldx, int64_t m, int32_t d, int32_t 
 int bf_rank_similarity(const double* a, const double* b, int32_t p, double* out, void* stream);
 
 /* ---- single-step entry points (parity tests) ---- */
+/* The hand-written device primitives under the presort (row a3)
+ * and the per-level offsets: an ascending, stable LSD radix sort of nseg
+ * independent segments of n 64-bit keys (keys[seg*n + i]) carrying optional
+ * 32-bit values (vals may be NULL), in place; an exclusive (inclusive != 0:
+ * inclusive) prefix sum of n uint32; the distinct values of n sorted keys
+ * (*count: device int32).  Device pointers only (BF_EINVAL otherwise).
+ * Synchronous.                                                             */
+int bf_sort_u64(uint64_t* keys, uint32_t* vals, int64_t n, int32_t nseg, void* stream);
+int bf_scan_u32(const uint32_t* in, uint32_t* out, int64_t n, int32_t inclusive, void* stream);
+int bf_unique_u64(const uint64_t* sorted, int64_t n, uint64_t* out, int32_t* count, void* stream);
 /* Philox4x32-10 on `count` counters (S1): ctr[4*i..], out[4*i..].          */
 int bf_philox(const uint32_t* ctr, uint32_t key0, uint32_t key1, uint32_t* out, int64_t count, void* stream);
 /* Correctly rounded int128 -> double of (hi[i], lo[i]) (the key of S4.3). */

@@ -92,7 +92,11 @@ def lib():
             "bf_fixed_point": ([vp, i64, i64, vp, C.POINTER(C.c_int32), vp], C.c_int),
             "bf_bootstrap": ([u64, i32, i32, i64, i64, i32, vp, vp], C.c_int),
             "bf_perm": ([u64, i32, i32, i64, vp, vp], C.c_int),
+            "bf_sort_u64": ([vp, vp, i64, i32, vp], C.c_int),
+            "bf_scan_u32": ([vp, vp, i64, i32, vp], C.c_int),
+            "bf_unique_u64": ([vp, i64, vp, vp, vp], C.c_int),
             "bf_set_allocator": ([vp, vp, vp], C.c_int),
+            "bf_set_memory_budget": ([i64], C.c_int),
             "bf_profile_enable": ([C.c_int], C.c_int),
             "bf_profile_read": ([vp, C.c_int, C.POINTER(C.c_int)], C.c_int),
             "bf_launch_count": ([], C.c_int64),
@@ -102,14 +106,53 @@ def lib():
             fn.argtypes = args
             fn.restype = res
         _LIB = L
+        _install_torch_allocator(L)
     return _LIB
 
 
+_TORCH_ALLOC = None
+
+
+def _install_torch_allocator(L):
+    """Route every device allocation of libbf.so through torch's CUDA caching allocator (bf_set_allocator with
+    the hooks of libbf_torch_alloc.so), so the library and the caller's tensors share one memory pool.
+    Skipped without a CUDA device (nothing is allocated then) or with BF_TORCH_ALLOCATOR=0 (the library's own
+    cudaMallocAsync pool)."""
+    global _TORCH_ALLOC
+    if os.environ.get("BF_TORCH_ALLOCATOR", "1") == "0":
+        return
+    torch = _torch()
+    if not torch.cuda.is_available():
+        return
+    path = _build.TORCH_ALLOC
+    if not os.path.exists(path) or os.path.getmtime(path) < os.path.getmtime(os.path.join(_build.CSRC, "torch_alloc.cpp")):
+        path = _build.build_torch_alloc()
+    A = C.CDLL(path)
+    fa = C.cast(A.bf_torch_alloc, C.c_void_p).value
+    ff = C.cast(A.bf_torch_free, C.c_void_p).value
+    _check(L.bf_set_allocator(fa, ff, None), "bf_set_allocator")
+    _TORCH_ALLOC = A
+
+
+def torch_allocator_active() -> bool:
+    return _TORCH_ALLOC is not None
+
+
+def _memory_budget_hint():
+    """Free device memory as torch sees it (driver-free + torch-cached-but-unused blocks): bf_fit sizes its trees
+    in flight from it when the torch allocator is installed."""
+    if _TORCH_ALLOC is None:
+        return
+    torch = _torch()
+    free, _ = torch.cuda.mem_get_info()
+    lib().bf_set_memory_budget(int(free + torch.cuda.memory_reserved() - torch.cuda.memory_allocated()))
+
+
 def exported_symbols():
-    return [n for n in ("bf_version", "bf_last_error", "bf_set_allocator", "bf_fit", "bf_forest_free",
+    return [n for n in ("bf_version", "bf_last_error", "bf_set_allocator", "bf_set_memory_budget", "bf_fit", "bf_forest_free",
                         "bf_forest_info_get", "bf_forest_export", "bf_forest_import", "bf_predict",
                         "bf_oob_importance", "bf_importance_finalize", "bf_pca", "bf_pca_retained", "bf_philox", "bf_i128_to_double",
-                        "bf_fixed_point", "bf_bootstrap", "bf_perm", "bf_profile_enable", "bf_profile_read",
+                        "bf_fixed_point", "bf_bootstrap", "bf_perm", "bf_sort_u64", "bf_scan_u32", "bf_unique_u64", "bf_profile_enable", "bf_profile_read",
                         "bf_launch_count", "bf_partial_dependence", "bf_pd_grid", "bf_varimax",
                         "bf_glm_gaussian", "bf_glm_predict", "bf_rank_similarity", "bf_mars_fit",
                         "bf_mars_predict")]
@@ -267,7 +310,9 @@ def fit(X, y, ntree: int = 500, mtry: int = 0, nodesize: int = 5, replace: int =
                  tree_begin=tree_begin, tree_end=ntree if tree_end is None else tree_end,
                  trees_in_flight=trees_in_flight, small_node_max=small_node_max)
     h = C.c_void_p()
-    _check(lib().bf_fit(_ptr(X), n, _ptr(y), n, p, C.byref(prm), _stream(), C.byref(h)), "bf_fit")
+    L = lib()
+    _memory_budget_hint()
+    _check(L.bf_fit(_ptr(X), n, _ptr(y), n, p, C.byref(prm), _stream(), C.byref(h)), "bf_fit")
     return Forest(h)
 
 
@@ -417,6 +462,30 @@ def philox(ctr: np.ndarray, key0: int, key1: int) -> np.ndarray:
     out = np.empty_like(ctr)
     _check(lib().bf_philox(ctr.ctypes.data, key0, key1, out.ctypes.data, ctr.shape[0], _stream()), "bf_philox")
     return out
+
+
+def sort_u64(keys, vals=None, nseg: int = 1):
+    """In-place stable radix sort of device tensors (int64 storage of uint64 keys; int32 storage of uint32
+    values) in nseg equal segments (bf_sort_u64)."""
+    n = keys.numel() // nseg
+    _check(lib().bf_sort_u64(_ptr(keys), _ptr(vals) if vals is not None else None, n, nseg, _stream()), "bf_sort_u64")
+
+
+def scan_u32(x, inclusive: bool = False):
+    """Prefix sum of a device int32 tensor holding uint32 values (bf_scan_u32)."""
+    out = _torch().empty_like(x)
+    _check(lib().bf_scan_u32(_ptr(x), _ptr(out), x.numel(), int(inclusive), _stream()), "bf_scan_u32")
+    return out
+
+
+def unique_u64(sorted_keys):
+    """Distinct values of sorted device keys (bf_unique_u64) -> (values, count)."""
+    torch = _torch()
+    out = torch.empty_like(sorted_keys)
+    cnt = torch.zeros(1, dtype=torch.int32, device=sorted_keys.device)
+    _check(lib().bf_unique_u64(_ptr(sorted_keys), sorted_keys.numel(), _ptr(out), _ptr(cnt), _stream()), "bf_unique_u64")
+    k = int(cnt.item())
+    return out[:k], k
 
 
 def i128_to_double(hi: np.ndarray, lo: np.ndarray) -> np.ndarray:

@@ -14,7 +14,8 @@ ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 LIBDIR = os.path.join(HERE, "_lib")
 LIB = os.path.join(LIBDIR, "libbf.so")
-SOURCES = ["capi.cu", "fit.cu", "predict.cu", "importance.cu", "pca.cu", "models.cu"]
+TORCH_ALLOC = os.path.join(LIBDIR, "libbf_torch_alloc.so")
+SOURCES = ["capi.cu", "fit.cu", "predict.cu", "importance.cu", "pca.cu", "models.cu", "prims.cu"]
 HEADERS = ["bf_internal.cuh"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
@@ -65,5 +66,25 @@ def build(force: bool = False, verbose: bool = False) -> str:
     return LIB
 
 
+def build_torch_alloc(force: bool = False) -> str:
+    """libbf_torch_alloc.so: the bf_set_allocator hooks over torch's CUDA caching allocator (csrc/torch_alloc.cpp),
+    compiled with g++ against the installed torch's c10 headers and libraries (rpath to torch/lib)."""
+    src = os.path.join(CSRC, "torch_alloc.cpp")
+    if not force and os.path.exists(TORCH_ALLOC) and os.path.getmtime(TORCH_ALLOC) >= os.path.getmtime(src):
+        return TORCH_ALLOC
+    import torch
+    tdir = os.path.dirname(torch.__file__)
+    inc = [os.path.join(tdir, "include"), "/usr/local/cuda/include"]
+    lib = os.path.join(tdir, "lib")
+    os.makedirs(LIBDIR, exist_ok=True)
+    tmp = TORCH_ALLOC + ".tmp"
+    cmd = ["g++", "-O2", "-std=c++17", "-fPIC", "-shared", "-D_GLIBCXX_USE_CXX11_ABI=%d" % int(torch._C._GLIBCXX_USE_CXX11_ABI),
+           *[f"-I{d}" for d in inc], src, "-o", tmp, f"-L{lib}", "-lc10_cuda", "-lc10", f"-Wl,-rpath,{lib}"]
+    subprocess.check_call(cmd)
+    os.replace(tmp, TORCH_ALLOC)
+    return TORCH_ALLOC
+
+
 if __name__ == "__main__":
     print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))
+    print(build_torch_alloc(force="--force" in sys.argv))

@@ -34,6 +34,7 @@ void set_error(const std::string& m);
 
 // ------------------------------------------------------------------ memory
 void* dev_alloc(size_t bytes, cudaStream_t s);
+int64_t memory_budget();  // bf_set_memory_budget (0: ask the driver)
 void dev_free(void* p, cudaStream_t s);
 
 template <class T>
@@ -222,11 +223,29 @@ struct bf_forest {
   uint32_t* d_roots8 = nullptr;  // per tree: global root id | 1<<31 if the tree is a single leaf
   int nodes8_state = 0;
   int device = 0;
+  cudaStream_t stream = nullptr;       // stream the forest's memory was allocated on (freed stream-ordered on it)
+  mutable bool foreign_stream = false;  // some call used the forest on another stream (free waits for the device)
+  void touch(cudaStream_t s) const {
+    if (s != stream) foreign_stream = true;
+  }
 };
 
 namespace bf {
 void forest_alloc(bf_forest* f, int64_t total_nodes, int32_t ntrees, cudaStream_t s);
 void forest_release(bf_forest* f);
+
+// prims.cu: hand-written scans, LSD radix sort, unique (no library kernels on the path)
+void scan_exclusive(const uint64_t* in, uint64_t* out, int64_t n, cudaStream_t s);
+void scan_exclusive(const int32_t* in, int32_t* out, int64_t n, cudaStream_t s);
+void scan_exclusive(const uint32_t* in, uint32_t* out, int64_t n, cudaStream_t s);
+void scan_inclusive(const uint32_t* in, uint32_t* out, int64_t n, cudaStream_t s);
+// Sorts nseg equal-length segments of n keys (k0[seg * n + i]) independently, ascending and stable, with
+// optional 32-bit values (v0/v1 NULL: keys only); k1 / v1 are scratch of the same size.  Returns the buffer
+// that holds the sorted keys (k0 or k1); *vals_out the one with the values.
+const uint64_t* radix_sort_u64(uint64_t* k0, uint64_t* k1, uint32_t* v0, uint32_t* v1, int64_t n, int nseg,
+                               cudaStream_t s, uint32_t** vals_out);
+// Distinct values of sorted keys, in order; *count_dev (device int32) = how many.
+void unique_u64(const uint64_t* sorted, int64_t n, uint64_t* out, int32_t* count_dev, cudaStream_t s);
 
 // fit.cu
 void fit_impl(const double* X, int64_t ldx, const double* y, int64_t n, int32_t p, const bf_params& prm,

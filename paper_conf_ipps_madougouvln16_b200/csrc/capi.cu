@@ -3,6 +3,7 @@
 // single-step parity entry points.
 #include <cstdio>
 #include <cstring>
+#include <atomic>
 #include <mutex>
 
 #include "bf_internal.cuh"
@@ -15,6 +16,8 @@ void set_error(const std::string& m) { g_last_error = m; }
 static bf_alloc_fn g_alloc = nullptr;
 static bf_free_fn g_free = nullptr;
 static void* g_ctx = nullptr;
+static std::atomic<int64_t> g_budget{0};
+int64_t memory_budget() { return g_budget.load(); }
 
 void* dev_alloc(size_t bytes, cudaStream_t s) {
   if (bytes == 0) return nullptr;
@@ -90,6 +93,7 @@ void OutStage::finish(cudaStream_t s) {
 }
 
 void forest_alloc(bf_forest* f, int64_t total, int32_t ntrees, cudaStream_t s) {
+  f->stream = s;
   f->info.total_nodes = total;
   size_t t = (size_t)(total > 0 ? total : 1);
   f->d_nodes = (Node16*)dev_alloc(t * sizeof(Node16), s);
@@ -100,7 +104,11 @@ void forest_alloc(bf_forest* f, int64_t total, int32_t ntrees, cudaStream_t s) {
 }
 
 void forest_release(bf_forest* f) {
-  cudaStream_t s = nullptr;
+  // Freed stream-ordered on the allocation stream.  If a call (predict, importance, ...) used the forest on
+  // another stream, its kernels may still read the arrays: wait for the device first, so neither
+  // cudaFreeAsync nor a caching allocator (torch) can hand the blocks out while they are in use.
+  if (f->foreign_stream) cudaDeviceSynchronize();
+  cudaStream_t s = f->stream;
   dev_free(f->d_nodes, s);
   dev_free(f->d_count, s);
   dev_free(f->d_value, s);
@@ -167,6 +175,12 @@ int bf_set_allocator(bf_alloc_fn alloc, bf_free_fn free_, void* ctx) {
   g_alloc = alloc;
   g_free = free_;
   g_ctx = ctx;
+  return BF_OK;
+}
+
+int bf_set_memory_budget(int64_t bytes) {
+  if (bytes < 0) return BF_EINVAL;
+  bf::g_budget.store(bytes);
   return BF_OK;
 }
 
@@ -291,6 +305,7 @@ int bf_predict(const bf_forest* f, const double* Xq, int64_t ldq, int64_t m, dou
   BF_API_BEGIN
   BF_REQUIRE(f && (Xq || m == 0), BF_EINVAL, "bf_predict: NULL");
   BF_REQUIRE(m >= 0 && ldq >= m, BF_EINVAL, "bf_predict: need m >= 0, ldq >= m");
+  f->touch((cudaStream_t)stream);
   predict_impl(f, Xq, ldq, m, yhat_sum, yhat, ntree_total, (cudaStream_t)stream);
   BF_API_END
 }
@@ -310,6 +325,7 @@ int bf_partial_dependence(const bf_forest* f, const double* X, int64_t ldx, int6
   BF_REQUIRE(f && X && grid, BF_EINVAL, "bf_partial_dependence: NULL");
   BF_REQUIRE(p == f->info.p && n >= 0 && ldx >= n && m >= 0 && m < p && G >= 1, BF_EINVAL,
              "bf_partial_dependence: need p == forest p, ldx >= n, 0 <= m < p, G >= 1");
+  f->touch((cudaStream_t)stream);
   partial_dependence_impl(f, X, ldx, n, m, grid, G, pd_sum, pd, ntree_total, (cudaStream_t)stream);
   BF_API_END
 }
@@ -320,6 +336,7 @@ int bf_oob_importance(const bf_forest* f, const double* X, int64_t ldx, const do
   BF_REQUIRE(f && X && y && acc, BF_EINVAL, "bf_oob_importance: NULL");
   BF_REQUIRE(n == f->info.n && p == f->info.p && ldx >= n, BF_EINVAL,
              "bf_oob_importance: X/y shape differs from the training data");
+  f->touch((cudaStream_t)stream);
   oob_importance_impl(f, X, ldx, y, n, p, *acc, (cudaStream_t)stream);
   BF_API_END
 }
@@ -433,6 +450,42 @@ int bf_philox(const uint32_t* ctr, uint32_t key0, uint32_t key1, uint32_t* out, 
   OutStage co(out, sizeof(uint32_t) * 4 * count, s);
   philox_impl((const uint32_t*)ci.dptr, key0, key1, (uint32_t*)co.dptr, count, s);
   co.finish(s);
+  BF_CUDA_CHECK(cudaStreamSynchronize(s));
+  BF_API_END
+}
+
+int bf_sort_u64(uint64_t* keys, uint32_t* vals, int64_t n, int32_t nseg, void* stream) {
+  BF_API_BEGIN
+  cudaStream_t s = (cudaStream_t)stream;
+  BF_REQUIRE(keys && n >= 0 && nseg >= 1, BF_EINVAL, "bf_sort_u64: bad arguments");
+  BF_REQUIRE(is_device_ptr(keys) && is_device_ptr(vals), BF_EINVAL, "bf_sort_u64: device pointers required");
+  const int64_t tot = n * nseg;
+  DBuf<uint64_t> k1(tot, s);
+  DBuf<uint32_t> v1(vals ? tot : 0, s);
+  uint32_t* vres = nullptr;
+  const uint64_t* kres = radix_sort_u64(keys, k1.p, vals, vals ? v1.p : nullptr, n, nseg, s, &vres);
+  if (kres != keys && tot) BF_CUDA_CHECK(cudaMemcpyAsync(keys, kres, sizeof(uint64_t) * tot, cudaMemcpyDeviceToDevice, s));
+  if (vals && vres != vals && tot) BF_CUDA_CHECK(cudaMemcpyAsync(vals, vres, sizeof(uint32_t) * tot, cudaMemcpyDeviceToDevice, s));
+  BF_CUDA_CHECK(cudaStreamSynchronize(s));
+  BF_API_END
+}
+
+int bf_scan_u32(const uint32_t* in, uint32_t* out, int64_t n, int32_t inclusive, void* stream) {
+  BF_API_BEGIN
+  cudaStream_t s = (cudaStream_t)stream;
+  BF_REQUIRE(in && out && n >= 0 && is_device_ptr(in) && is_device_ptr(out), BF_EINVAL, "bf_scan_u32: bad arguments");
+  if (inclusive) scan_inclusive(in, out, n, s);
+  else scan_exclusive(in, out, n, s);
+  BF_CUDA_CHECK(cudaStreamSynchronize(s));
+  BF_API_END
+}
+
+int bf_unique_u64(const uint64_t* sorted, int64_t n, uint64_t* out, int32_t* count, void* stream) {
+  BF_API_BEGIN
+  cudaStream_t s = (cudaStream_t)stream;
+  BF_REQUIRE(sorted && out && count && n >= 0 && is_device_ptr(sorted) && is_device_ptr(out) && is_device_ptr(count),
+             BF_EINVAL, "bf_unique_u64: bad arguments");
+  unique_u64(sorted, n, out, count, s);
   BF_CUDA_CHECK(cudaStreamSynchronize(s));
   BF_API_END
 }

@@ -28,7 +28,7 @@
 // All split arithmetic is exact (int64 sums, int128 D, correctly rounded
 // key) so the topology is bit-identical to the CPU oracle whatever the scan
 // order, tile size or number of GPUs.
-#include <cub/cub.cuh>
+#include <cuda/atomic>
 
 #include <algorithm>
 #include <cstdio>
@@ -198,25 +198,35 @@ __global__ void k_yq(const double* y, int64_t n, double c, int q, int zero, int6
 }
 
 // ------------------------------------------------------------------ a3 presort
-__global__ void k_sort_keys(const double* col, int64_t n, uint64_t* keys, uint32_t* vals) {
-  for (int64_t i = blockIdx.x * (int64_t)NT + threadIdx.x; i < n; i += (int64_t)gridDim.x * NT) {
-    const uint64_t b = (uint64_t)__double_as_longlong(canon(col[i]));
-    keys[i] = (b >> 63) ? ~b : (b | 0x8000000000000000ull);  // order-preserving
-    vals[i] = (uint32_t)i;
+// All p features at once (feature-major arrays of p * n): order-preserving 64-bit keys of the canonical
+// values (-0 -> +0), one segmented radix sort (prims.cu), dense ranks by a scan of the value-change flags.
+__global__ void k_sort_keys(const double* X, int64_t ldx, int64_t n, int p, uint64_t* keys, uint32_t* vals) {
+  const int64_t tot = n * p;
+  for (int64_t k = blockIdx.x * (int64_t)NT + threadIdx.x; k < tot; k += (int64_t)gridDim.x * NT) {
+    const int64_t f = k / n, i = k - f * n;
+    const uint64_t b = (uint64_t)__double_as_longlong(canon(X[f * ldx + i]));
+    keys[k] = (b >> 63) ? ~b : (b | 0x8000000000000000ull);  // order-preserving
+    vals[k] = (uint32_t)i;
   }
 }
 
-__global__ void k_rank_flags(const uint64_t* keys, int64_t n, uint32_t* flags) {
-  for (int64_t i = blockIdx.x * (int64_t)NT + threadIdx.x; i < n; i += (int64_t)gridDim.x * NT)
-    flags[i] = (i > 0 && keys[i] != keys[i - 1]) ? 1u : 0u;
+__global__ void k_rank_flags(const uint64_t* keys, int64_t n, int p, uint32_t* flags) {
+  const int64_t tot = n * p;
+  for (int64_t k = blockIdx.x * (int64_t)NT + threadIdx.x; k < tot; k += (int64_t)gridDim.x * NT) {
+    const int64_t i = k % n;
+    flags[k] = (i > 0 && keys[k] != keys[k - 1]) ? 1u : 0u;
+  }
 }
 
-__global__ void k_fill_sorted(const double* col, const uint32_t* rows, const uint32_t* rank, int64_t n,
-                              uint64_t* srt, double* uniq) {
-  for (int64_t i = blockIdx.x * (int64_t)NT + threadIdx.x; i < n; i += (int64_t)gridDim.x * NT) {
-    const uint32_t r = rows[i], k = rank[i];
-    srt[i] = ((uint64_t)k << 40) | ((uint64_t)r << 16);
-    if (i == 0 || rank[i - 1] != k) uniq[k] = canon(col[r]);
+// rank: inclusive scan of the flags over all features; feature f's dense ranks are rank - rank[f * n].
+__global__ void k_fill_sorted(const double* X, int64_t ldx, const uint32_t* rows, const uint32_t* rank, int64_t n,
+                              int p, uint64_t* srt, double* uniq) {
+  const int64_t tot = n * p;
+  for (int64_t k = blockIdx.x * (int64_t)NT + threadIdx.x; k < tot; k += (int64_t)gridDim.x * NT) {
+    const int64_t f = k / n, i = k - f * n;
+    const uint32_t r = rows[k], rk = rank[k] - rank[f * n];
+    srt[k] = ((uint64_t)rk << 40) | ((uint64_t)r << 16);
+    if (i == 0 || rank[k - 1] != rank[k]) uniq[f * n + rk] = canon(X[f * ldx + r]);
   }
 }
 
@@ -1384,6 +1394,7 @@ __host__ __device__ inline size_t subtree_smem(int A, int p) {
   s += align16((size_t)2 * A * sizeof(SRec));         // node records
   s += align16((size_t)2 * max_medium(A) * sizeof(MNode));
   s += align16((size_t)(A + 1) * sizeof(TNode));      // tiny work queue
+  s += align16((size_t)(A + 1) * 4);                  // its ready flags
   s += align16((size_t)SUB_NW * p * 2) * 2;           // Fisher-Yates scratch, drawn features
   s += align16((size_t)SUB_NW * sizeof(WRec));
   s += 64;
@@ -1403,6 +1414,7 @@ struct SubArgs {
   int32_t t0;
   Pool pool;
   unsigned long long* stats;  // optional phase counters (BF_SUBTREE_STATS=1), else NULL
+  unsigned long long* visits; // optional (profile mode): split-search entry visits (mtry x distinct rows per node)
   int tq_sleep_max;           // idle-warp back-off cap in ns (BF_TQ_SLEEP_MAX, default 2048)
   int tq_bigger_first;        // continue with the child of more distinct rows (BF_TQ_BIGGER_FIRST, default 1)
 };
@@ -1439,15 +1451,51 @@ __device__ __forceinline__ void warp_draw_mtry(uint64_t seed, uint32_t t, uint64
   __syncwarp();
 }
 
-__device__ __forceinline__ void tq_push(TNode* q, int* alloc, int* pending, const TNode& nd) {
+// Tiny-node work queue (shared memory).  Every access to a queue entry, its ready flag and the queue
+// counters is an atomic (cuda::atomic_ref, block scope): the producer writes the entry's fields with relaxed
+// stores and publishes it with a release store of ready[idx]; the consumer's lane 0 spins on an acquire load
+// of the flag, reads the fields and broadcasts them to its warp.  So the hand-off is ordered by the memory
+// model (no volatile + fence idiom) and carries no plain shared-memory accesses for racecheck to flag.
+template <class T>
+using blk_ref = cuda::atomic_ref<T, cuda::thread_scope_block>;
+
+__device__ __forceinline__ void tq_push(TNode* q, int32_t* ready, int* alloc, int* pending, const TNode& c) {
   atomicAdd(pending, 1);
   const int idx = atomicAdd(alloc, 1);
-  TNode c = nd;
-  const int32_t n = c.n;
-  c.n = 0;
-  q[idx] = c;
-  __threadfence_block();
-  *(volatile int32_t*)&q[idx].n = n;
+  TNode& e = q[idx];
+  blk_ref<int32_t>(e.rlo).store(c.rlo, cuda::memory_order_relaxed);
+  blk_ref<int32_t>(e.ra).store(c.ra, cuda::memory_order_relaxed);
+  blk_ref<unsigned long long>(*(unsigned long long*)&e.mask).store(c.mask, cuda::memory_order_relaxed);
+  blk_ref<int32_t>(e.id).store(c.id, cuda::memory_order_relaxed);
+  blk_ref<int32_t>(e.n).store(c.n, cuda::memory_order_relaxed);
+  blk_ref<long long>(*(long long*)&e.S).store(c.S, cuda::memory_order_relaxed);
+  blk_ref<unsigned long long>(*(unsigned long long*)&e.key).store(c.key, cuda::memory_order_relaxed);
+  blk_ref<int32_t>(ready[idx]).store(1, cuda::memory_order_release);
+}
+
+__device__ __forceinline__ TNode tq_read(TNode* q, int idx) {  // after an acquire of ready[idx] (or a barrier)
+  TNode& e = q[idx];
+  TNode c;
+  c.rlo = blk_ref<int32_t>(e.rlo).load(cuda::memory_order_relaxed);
+  c.ra = blk_ref<int32_t>(e.ra).load(cuda::memory_order_relaxed);
+  c.mask = blk_ref<unsigned long long>(*(unsigned long long*)&e.mask).load(cuda::memory_order_relaxed);
+  c.id = blk_ref<int32_t>(e.id).load(cuda::memory_order_relaxed);
+  c.n = blk_ref<int32_t>(e.n).load(cuda::memory_order_relaxed);
+  c.S = blk_ref<long long>(*(long long*)&e.S).load(cuda::memory_order_relaxed);
+  c.key = blk_ref<unsigned long long>(*(unsigned long long*)&e.key).load(cuda::memory_order_relaxed);
+  return c;
+}
+
+__device__ __forceinline__ TNode tq_bcast(const TNode& c) {  // lane 0's entry to the whole warp
+  TNode r;
+  r.rlo = __shfl_sync(0xffffffffu, c.rlo, 0);
+  r.ra = __shfl_sync(0xffffffffu, c.ra, 0);
+  r.mask = __shfl_sync(0xffffffffu, c.mask, 0);
+  r.id = __shfl_sync(0xffffffffu, c.id, 0);
+  r.n = __shfl_sync(0xffffffffu, c.n, 0);
+  r.S = __shfl_sync(0xffffffffu, c.S, 0);
+  r.key = __shfl_sync(0xffffffffu, c.key, 0);
+  return r;
 }
 
 __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
@@ -1477,6 +1525,8 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   ptr += align16((size_t)2 * MM * sizeof(MNode));
   TNode* tq = (TNode*)ptr;
   ptr += align16((size_t)(A + 1) * sizeof(TNode));
+  int32_t* tq_ready = (int32_t*)ptr;
+  ptr += align16((size_t)(A + 1) * 4);
   int16_t* mind_all = (int16_t*)ptr;
   ptr += align16((size_t)SUB_NW * p * 2);
   int16_t* feats_all = (int16_t*)ptr;
@@ -1499,6 +1549,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   tclk[0] = clock64();
   int n_med = 0, n_tiny = 0;
   long long busy = 0;
+  unsigned long long nvis = 0;  // entry visits of this warp's split searches (profile mode)
 
   // ---- load 1: local rows = feature 0's order; payload; global row -> local id in a shared-memory hash
   // table (open addressing over HSLOTS slots, built in the scratch area that the later phases reuse)
@@ -1520,78 +1571,37 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
     wy[j] = (int64_t)wv * yqr;
     wyd[j] = __dmul_rn((double)wv, yr);
   }
-  for (int j = tid; j <= a0; j += SUB_NT) tq[j].n = 0;
+  for (int j = tid; j <= a0; j += SUB_NT) blk_ref<int32_t>(tq_ready[j]).store(0, cuda::memory_order_relaxed);
   __syncthreads();
   auto hfind = [&](uint32_t row) -> uint16_t {
     uint32_t h = (row * 0x9E3779B1u) >> (32 - HBITS);
     while (hkey[h] != row) h = (h + 1) & (HSLOTS - 1);
     return hval[h];
   };
-  // ---- load 2: warp per feature; local rank = index of the first entry of the same value
-  if (a0 <= 32 * 16) {  // K <= 16 consecutive entries per lane, all loads in flight; one warp max-scan per feature
-    const int K = (a0 + 31) >> 5;
-    const int j0 = lane * K, j1 = min(j0 + K, a0);
-    for (int f = wid; f < p; f += SUB_NW) {
-      const uint64_t* sf = src + (int64_t)f * a0;
-      uint32_t rk[16];
-      uint16_t lr[16];
-#pragma unroll
-      for (int q = 0; q < 16; ++q) {
-        const int j = j0 + q;
-        const uint64_t e = (q < K && j < j1) ? sf[j] : ~0ull;
-        rk[q] = e_rank(e);
-      }
-#pragma unroll
-      for (int q = 0; q < 16; ++q) {
-        const int j = j0 + q;
-        lr[q] = (q < K && j < j1) ? hfind(e_row(sf[j])) : 0;
-      }
-      // lane-local breaks: gs = j where the value changes, -1 = continues from the previous lane
-      uint32_t lastrk = 0xffffffffu;
-      int gl = -1;
-#pragma unroll
-      for (int q = 0; q < 16; ++q)
-        if (q < K && j0 + q < j1) {
-          lastrk = rk[q];
-          if (q > 0 && rk[q] != rk[q - 1]) gl = j0 + q;
-        }
-      const uint32_t prv = __shfl_up_sync(0xffffffffu, lastrk, 1);
-      const bool brk0 = j0 < j1 && (lane == 0 || rk[0] != prv);  // my first entry starts a value
-      int glast = gl >= 0 ? gl : (brk0 ? j0 : -1);
-      int inc = glast;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const int v = __shfl_up_sync(0xffffffffu, inc, o);
-        if (lane >= o) inc = max(inc, v);
-      }
-      int cur = __shfl_up_sync(0xffffffffu, inc, 1);  // the last break before my entries
-      if (lane == 0) cur = 0;
-      uint32_t* lf = list + (size_t)f * a0;
-#pragma unroll
-      for (int q = 0; q < 16; ++q) {
-        const int j = j0 + q;
-        if (q < K && j < j1) {
-          if (q == 0 ? brk0 : rk[q] != rk[q - 1]) cur = j;
-          lf[j] = ((uint32_t)cur << 16) | lr[q];
-        }
-      }
-    }
-  } else {
-    constexpr int GRP = 8;  // chunks of 32 entries in flight per warp
+  // ---- load 2: warp per feature; local rank = index of the first entry of the same value.  Coalesced: chunk c
+  // of 32 entries is read by lane l at entry 32c + l, each entry once (rank and row from the same 8-byte load),
+  // up to 16 chunks (a0 <= 512) in flight per warp; the value breaks are max-scanned per chunk with a carry.
+  {
+    constexpr int GRP = 16;
     const int nch = (a0 + 31) >> 5;
     for (int f = wid; f < p; f += SUB_NW) {
       const uint64_t* sf = src + (int64_t)f * a0;
       int carry_gs = 0;
       uint32_t prev_last = 0xffffffffu;
       for (int c0 = 0; c0 < nch; c0 += GRP) {
+        uint64_t ev[GRP];
+#pragma unroll
+        for (int c = 0; c < GRP; ++c) {
+          const int j = (c0 + c) * 32 + lane;
+          ev[c] = (c0 + c < nch && j < a0) ? sf[j] : ~0ull;
+        }
         uint32_t rk[GRP];
         uint16_t lr[GRP];
 #pragma unroll
         for (int c = 0; c < GRP; ++c) {
           const int j = (c0 + c) * 32 + lane;
-          const uint64_t e = j < a0 ? sf[j] : ~0ull;
-          rk[c] = j < a0 ? e_rank(e) : 0xffffffffu;
-          lr[c] = j < a0 ? hfind(e_row(e)) : 0;
+          rk[c] = j < a0 ? e_rank(ev[c]) : 0xffffffffu;
+          lr[c] = (c0 + c < nch && j < a0) ? hfind(e_row(ev[c])) : 0;
         }
 #pragma unroll
         for (int c = 0; c < GRP; ++c) {
@@ -1651,7 +1661,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
     c.n = root.n;
     c.S = root.S;
     c.key = root.key;
-    tq_push(tq, &s_alloc, &s_pending, c);
+    tq_push(tq, tq_ready, &s_alloc, &s_pending, c);
   }
   __syncthreads();
   tclk[1] = clock64();
@@ -1687,6 +1697,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         // K consecutive entries per lane: lane-serial sums, one warp scan, a bounds pass screened by the
         // warp max of the lower bounds (and the warp's best so far), exact keys only where they may win
         const int aN = nd.a, K = (aN + 31) >> 5;
+        nvis += (unsigned)aN;
         const int i0 = min(lane * K, aN), i1 = min(i0 + K, aN);
         int32_t rw = 0;
         int64_t rsum = 0;
@@ -1886,7 +1897,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
             c.n = nn;
             c.S = S;
             c.key = key;
-            tq_push(tq, &s_alloc, &s_pending, c);
+            tq_push(tq, tq_ready, &s_alloc, &s_pending, c);
           }
         }
       }
@@ -1945,39 +1956,40 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   // ================= tiny nodes: row index inside each tiny root, then the work queue
   tclk[2] = clock64();
   {
-    const int nroots = s_alloc;
+    const int nroots = blk_ref<int>(s_alloc).load(cuda::memory_order_relaxed);
     for (int qi = wid; qi < nroots; qi += SUB_NW) {
-      const TNode& r = tq[qi];
+      const TNode r = tq_read(tq, qi);  // pushed before the barrier above
       for (int k = lane; k < r.ra; k += 32) rmap[list[r.rlo + k] & 0xffffu] = (uint8_t)k;
     }
   }
   __syncthreads();
   for (;;) {
     int h = -1;
+    TNode nd;
     if (lane == 0) {
       unsigned ns = 32;
       for (;;) {
-        const int hd = *(volatile int*)&s_head;
-        if (hd < *(volatile int*)&s_alloc) {
+        const int hd = blk_ref<int>(s_head).load(cuda::memory_order_relaxed);
+        if (hd < blk_ref<int>(s_alloc).load(cuda::memory_order_relaxed)) {
           if (atomicCAS(&s_head, hd, hd + 1) == hd) {
             h = hd;
             break;
           }
-        } else if (*(volatile int*)&s_pending == 0) {
+        } else if (blk_ref<int>(s_pending).load(cuda::memory_order_relaxed) == 0) {
           break;
         } else {
           __nanosleep(ns);  // idle warp: back off so the busy warps keep the issue slots
           ns = min(ns * 2, (unsigned)g.tq_sleep_max);
         }
       }
-      if (h >= 0)
-        while (*(volatile int32_t*)&tq[h].n == 0) __nanosleep(32);
-      __threadfence_block();
+      if (h >= 0) {
+        while (blk_ref<int32_t>(tq_ready[h]).load(cuda::memory_order_acquire) == 0) __nanosleep(32);
+        nd = tq_read(tq, h);
+      }
     }
     h = __shfl_sync(0xffffffffu, h, 0);
-    __syncwarp();  // orders every lane's reads of the entry after lane 0's acquire (flag + fence)
     if (h < 0) break;
-    TNode nd = tq[h];
+    nd = tq_bcast(nd);
     bool have = true;
     const long long tb0 = clock64();
     while (have) {
@@ -1985,6 +1997,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       ++n_tiny;
       const int rlo = nd.rlo, ra = nd.ra;
       const int an = __popcll(nd.mask);  // distinct rows of the node
+      nvis += (unsigned long long)an * (unsigned)g.mtry;
       const long long c0_ = g.stats ? clock64() : 0;
       warp_draw_mtry(g.seed, t, nd.key, p, g.mtry, mind, feats, lane);
       const long long c1_ = g.stats ? clock64() : 0;
@@ -1997,28 +2010,52 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       uint32_t ltie = 0xffffffffu, lra = 0, lrb = 0;
       int32_t lnl = 0;
       int64_t lSl = 0;
-      for (int s0 = 0; s0 < g.mtry; s0 += TGRP) {
+      // Features go in groups as large as the staging area holds (ng * an <= sub_temp(A) entries): every drawn
+      // feature in ONE group when the node has few distinct rows, so the scan / bound / max passes and their
+      // fixed costs run once per node instead of once per TGRP features.
+      const int gcap = max(1, sub_temp(g.A) / max(an, 1));
+      for (int s0 = 0; s0 < g.mtry;) {
         const long long gqs = g.stats ? clock64() : 0;
-        const int ng = min(TGRP, g.mtry - s0);
-        // stage: the node's entries of each drawn feature, in value order, packed [slot][0..an).
-        // All loads of the group are issued before any store (ILP across features).
-        uint32_t ev[2 * TGRP];
-        uint8_t ri[2 * TGRP];
+        const int ng = min(gcap, g.mtry - s0);
+        // stage: the node's entries of each drawn feature, in value order, packed [slot][0..an), TGRP features
+        // at a time with all their loads issued before any store (ILP across features); the second half-warp row
+        // only when the tiny root has more than 32 rows (warp-uniform).
+        for (int u0 = 0; u0 < ng; u0 += TGRP) {
+          const int nu = min(TGRP, ng - u0);
+          uint32_t ev[2 * TGRP];
+          uint8_t ri[2 * TGRP];
+          if (ra > 32) {
 #pragma unroll
-        for (int u = 0; u < TGRP; ++u) {
-          const uint32_t* seg = list + (size_t)feats[s0 + (u < ng ? u : 0)] * a0 + rlo;
-          ev[2 * u] = (u < ng && lane < ra) ? seg[lane] : 0u;
-          ev[2 * u + 1] = (u < ng && lane + 32 < ra) ? seg[lane + 32] : 0u;
-        }
+            for (int u = 0; u < TGRP; ++u) {
+              const uint32_t* seg = list + (size_t)feats[s0 + u0 + (u < nu ? u : 0)] * a0 + rlo;
+              ev[2 * u] = (u < nu) ? seg[lane] : 0u;
+              ev[2 * u + 1] = (u < nu && lane + 32 < ra) ? seg[lane + 32] : 0u;
+            }
 #pragma unroll
-        for (int k = 0; k < 2 * TGRP; ++k) ri[k] = rmap[ev[k] & 0xffffu];
+            for (int k = 0; k < 2 * TGRP; ++k) ri[k] = rmap[ev[k] & 0xffffu];
 #pragma unroll
-        for (int u = 0; u < TGRP; ++u) {
-          const bool v0 = u < ng && lane < ra && ((nd.mask >> ri[2 * u]) & 1ull);
-          const bool v1 = u < ng && lane + 32 < ra && ((nd.mask >> ri[2 * u + 1]) & 1ull);
-          const unsigned m0 = __ballot_sync(0xffffffffu, v0), m1 = __ballot_sync(0xffffffffu, v1);
-          if (v0) stg[u * an + __popc(m0 & lt)] = ev[2 * u];
-          if (v1) stg[u * an + __popc(m0) + __popc(m1 & lt)] = ev[2 * u + 1];
+            for (int u = 0; u < TGRP; ++u) {
+              const bool v0 = u < nu && ((nd.mask >> ri[2 * u]) & 1ull);
+              const bool v1 = u < nu && lane + 32 < ra && ((nd.mask >> ri[2 * u + 1]) & 1ull);
+              const unsigned m0 = __ballot_sync(0xffffffffu, v0), m1 = __ballot_sync(0xffffffffu, v1);
+              if (v0) stg[(u0 + u) * an + __popc(m0 & lt)] = ev[2 * u];
+              if (v1) stg[(u0 + u) * an + __popc(m0) + __popc(m1 & lt)] = ev[2 * u + 1];
+            }
+          } else {
+#pragma unroll
+            for (int u = 0; u < TGRP; ++u) {
+              const uint32_t* seg = list + (size_t)feats[s0 + u0 + (u < nu ? u : 0)] * a0 + rlo;
+              ev[u] = (u < nu && lane < ra) ? seg[lane] : 0u;
+            }
+#pragma unroll
+            for (int k = 0; k < TGRP; ++k) ri[k] = rmap[ev[k] & 0xffffu];
+#pragma unroll
+            for (int u = 0; u < TGRP; ++u) {
+              const bool v0 = u < nu && lane < ra && ((nd.mask >> ri[u]) & 1ull);
+              const unsigned m0 = __ballot_sync(0xffffffffu, v0);
+              if (v0) stg[(u0 + u) * an + __popc(m0 & lt)] = ev[u];
+            }
+          }
         }
         __syncwarp();
         const long long gq0 = g.stats ? clock64() : 0;
@@ -2152,6 +2189,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
           atomicAdd(&g.stats[20], (unsigned long long)(gq5 - gq4));
         }
         __syncwarp();
+        s0 += ng;
       }
       const long long c2_ = g.stats ? clock64() : 0;
       if (g.stats && lane == 0) { atomicAdd(&g.stats[11], (unsigned long long)(c1_ - c0_)); atomicAdd(&g.stats[12], (unsigned long long)(c2_ - c1_)); }
@@ -2236,7 +2274,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         if (gl && gr) {
           // the larger child keeps the warp (the longer remaining chain stays off the queue's hand-off latency)
           const bool keep_r = g.tq_bigger_first && __popcll(mR) > __popcll(mL);
-          if (lane == 0) tq_push(tq, &s_alloc, &s_pending, keep_r ? cl : cr);
+          if (lane == 0) tq_push(tq, tq_ready, &s_alloc, &s_pending, keep_r ? cl : cr);
           nd = keep_r ? cr : cl;
           have = true;
         } else if (gl) {
@@ -2278,6 +2316,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       g.pool.value[gid] = r.value;
     }
   }
+  if (g.visits && lane == 0 && nvis) atomicAdd(g.visits, nvis);
   if (g.stats) {
     tclk[4] = clock64();
     if (tid == 0) {
@@ -2488,42 +2527,33 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
   int32_t q = 0;
   fixed_point_impl(y, n, ns, yq.p, &q, s);
 
-  // ---- a3 presort
+  // ---- a3 presort (hand-written segmented radix sort of all p features, prims.cu)
   DBuf<uint64_t> srt((size_t)p * n, s);
   DBuf<double> uniq((size_t)p * n, s);
   {
-    DBuf<uint64_t> k0(n, s), k1(n, s);
-    DBuf<uint32_t> v0(n, s), v1(n, s), fl(n, s), rk(n, s);
-    size_t tb1 = 0, tb2 = 0;
-    cub::DeviceRadixSort::SortPairs(nullptr, tb1, k0.p, k1.p, v0.p, v1.p, (int)n, 0, 64, s);
-    cub::DeviceScan::InclusiveSum(nullptr, tb2, fl.p, rk.p, (int)n, s);
-    DBuf<char> tmp(std::max(tb1, tb2), s);
-    for (int f = 0; f < p; ++f) {
-      const double* col = X + (int64_t)f * ldx;
-      {
-        KScope ks_("k_sort_keys", s, 0.0);
-        k_sort_keys<<<grid_for(n), NT, 0, s>>>(col, n, k0.p, v0.p);
-      }
-      size_t t1 = tb1;
-      {
-        KScope ks_("cub_SortPairs", s, 0.0);
-        BF_CUDA_CHECK(cub::DeviceRadixSort::SortPairs(tmp.p, t1, k0.p, k1.p, v0.p, v1.p, (int)n, 0, 64, s));
-      }
-      {
-        KScope ks_("k_rank_flags", s, 0.0);
-        k_rank_flags<<<grid_for(n), NT, 0, s>>>(k1.p, n, fl.p);
-      }
-      size_t t2 = tb2;
-      {
-        KScope ks_("cub_InclusiveSum", s, 0.0);
-        BF_CUDA_CHECK(cub::DeviceScan::InclusiveSum(tmp.p, t2, fl.p, rk.p, (int)n, s));
-      }
-      {
-        KScope ks_("k_fill_sorted", s, 0.0);
-        k_fill_sorted<<<grid_for(n), NT, 0, s>>>(col, v1.p, rk.p, n, srt.p + (int64_t)f * n, uniq.p + (int64_t)f * n);
-      }
-      BF_CUDA_CHECK(cudaGetLastError());
+    const int64_t tot = (int64_t)p * n;
+    DBuf<uint64_t> k0(tot, s), k1(tot, s);
+    DBuf<uint32_t> v0(tot, s), v1(tot, s);
+    {
+      KScope ks_("k_sort_keys", s, (double)tot * 20.0);
+      k_sort_keys<<<grid_for(tot), NT, 0, s>>>(X, ldx, n, p, k0.p, v0.p);
     }
+    BF_CUDA_CHECK(cudaGetLastError());
+    uint32_t* rows = nullptr;
+    const uint64_t* ks = radix_sort_u64(k0.p, k1.p, v0.p, v1.p, n, p, s, &rows);
+    uint32_t* fl = rows == v0.p ? v1.p : v0.p;  // the value buffer not holding the sorted rows
+    uint64_t* rk64 = const_cast<uint64_t*>(ks == k0.p ? k1.p : k0.p);
+    uint32_t* rk = reinterpret_cast<uint32_t*>(rk64);  // scratch: the key buffer not holding the sorted keys
+    {
+      KScope ks_("k_rank_flags", s, 0.0);
+      k_rank_flags<<<grid_for(tot), NT, 0, s>>>(ks, n, p, fl);
+    }
+    scan_inclusive(fl, rk, tot, s);
+    {
+      KScope ks_("k_fill_sorted", s, 0.0);
+      k_fill_sorted<<<grid_for(tot), NT, 0, s>>>(X, ldx, rows, rk, n, p, srt.p, uniq.p);
+    }
+    BF_CUDA_CHECK(cudaGetLastError());
   }
 
   ptm.mark("presort");
@@ -2542,6 +2572,9 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
   if (B <= 0) {
     size_t fr = 0, tot = 0;
     BF_CUDA_CHECK(cudaMemGetInfo(&fr, &tot));
+    // free memory as the allocator in use sees it: the driver's, or the caller's hint (bf_set_memory_budget:
+    // the torch caching allocator's cached-but-unused blocks count as free)
+    if (memory_budget() > 0) fr = (size_t)memory_budget();
     const size_t budget = fr / 2;
     B = (int)std::max<size_t>(1, std::min<size_t>(budget / std::max<size_t>(per_tree, 1), 256));
   }
@@ -2594,9 +2627,6 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
     DBuf<Split> split(cap_level, s);
     DBuf<Child> child(2 * cap_level, s);
     DBuf<uint64_t> packL(2 * cap_level, s), packS(2 * cap_level, s), scanL(2 * cap_level, s), scanS(2 * cap_level, s);
-    size_t scan_tb = 0;
-    cub::DeviceScan::ExclusiveSum(nullptr, scan_tb, packL.p, scanL.p, (int)(2 * cap_level), s);
-    DBuf<char> scan_tmp(std::max<size_t>(scan_tb, 16), s);
     DBuf<LevelSummary> dsum(1, s);
     PinnedSummary hs;
     // piece decomposition of the winning segments (k_dest_bits), sized for the largest level of a batch
@@ -2606,23 +2636,13 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
     // partition work items (at most p per node)
     DBuf<int32_t> icnt(cap_level + 1, s), ioff(cap_level + 1, s);
     DBuf<int2> imap(cap_level * p, s);
-    size_t items_tb = 0;
-    cub::DeviceScan::ExclusiveSum(nullptr, items_tb, icnt.p, ioff.p, (int)(cap_level + 1), s);
-    DBuf<char> items_tmp(std::max<size_t>(items_tb, 16), s);
-    size_t piece_tb = 0;
-    cub::DeviceScan::ExclusiveSum(nullptr, piece_tb, pcnt.p, poff.p, (int)cap_level, s);
-    DBuf<char> piece_tmp(std::max<size_t>(piece_tb, 16), s);
     auto piece_setup = [&](int mode, int nitems, int div, const LNode* nodes, const Split* sp, const Child* ch,
                            int32_t* cnt, int32_t* off, int32_t* map, int32_t* tot, cudaStream_t st) {
       {
         KScope ks_("k_piece_count", st, 0.0);
         k_piece_count<<<(unsigned)ceil_div(nitems, 256), 256, 0, st>>>(mode, nitems, div, nodes, sp, ch, cnt);
       }
-      {
-        KScope ks_("cub_ExclusiveSum", st, 0.0);
-        size_t tb2 = piece_tb;
-        BF_CUDA_CHECK(cub::DeviceScan::ExclusiveSum(piece_tmp.p, tb2, cnt, off, nitems, st));
-      }
+      scan_exclusive(cnt, off, nitems, st);
       {
         KScope ks_("k_piece_map", st, 0.0);
         k_piece_map<<<(unsigned)ceil_div(nitems, 256), 256, 0, st>>>(nitems, cnt, off, map, tot);
@@ -2781,16 +2801,8 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
         }
         BF_CUDA_CHECK(cudaGetLastError());
         const int N2 = 2 * N;
-        size_t t1 = scan_tb;
-        {
-          KScope ks_("cub_ExclusiveSum", s, 0.0);
-          BF_CUDA_CHECK(cub::DeviceScan::ExclusiveSum(scan_tmp.p, t1, packL.p, scanL.p, N2, s));
-        }
-        t1 = scan_tb;
-        {
-          KScope ks_("cub_ExclusiveSum", s, 0.0);
-          BF_CUDA_CHECK(cub::DeviceScan::ExclusiveSum(scan_tmp.p, t1, packS.p, scanS.p, N2, s));
-        }
+        scan_exclusive(packL.p, scanL.p, N2, s);
+        scan_exclusive(packS.p, scanS.p, N2, s);
         {
           KScope ks_("k_child_place", s, 0.0);
           k_child_place<<<(unsigned)ceil_div(N2, 128), 128, 0, s>>>(N2, p, nc, child.p, scanL.p, scanS.p, nx, sq.p,
@@ -2813,8 +2825,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
         {
           KScope ks_("k_part_items", s, 0.0);
           k_part_items_count<<<(unsigned)ceil_div(N + 1, 256), 256, 0, s>>>(N, p, nc, split.p, child.p, icnt.p);
-          size_t tb3 = items_tb;
-          BF_CUDA_CHECK(cub::DeviceScan::ExclusiveSum(items_tmp.p, tb3, icnt.p, ioff.p, N + 1, s));
+          scan_exclusive(icnt.p, ioff.p, N + 1, s);
           k_part_items_map<<<(unsigned)ceil_div(N, 256), 256, 0, s>>>(N, p, nc, icnt.p, ioff.p, imap.p);
         }
         {
@@ -2874,6 +2885,13 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
           ga.t0 = tb;
           ga.pool = pool;
           ga.stats = nullptr;
+          ga.visits = nullptr;
+          DBuf<unsigned long long> vis;
+          if (prof_enabled()) {
+            vis.alloc(1, s);
+            BF_CUDA_CHECK(cudaMemsetAsync(vis.p, 0, 8, s));
+            ga.visits = vis.p;
+          }
           static const int tq_sleep_max = getenv("BF_TQ_SLEEP_MAX") ? atoi(getenv("BF_TQ_SLEEP_MAX")) : 2048;
           static const int tq_bigger_first = getenv("BF_TQ_BIGGER_FIRST") ? atoi(getenv("BF_TQ_BIGGER_FIRST")) : 1;
           ga.tq_sleep_max = tq_sleep_max < 32 ? 32 : tq_sleep_max;
@@ -2888,6 +2906,12 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
           {
             KScope ks_("k_subtree", s, 0.0);
             k_subtree<<<(unsigned)ls.nsmall, SUB_NT, subtree_smem(A, p), s>>>(ga);
+          }
+          if (ga.visits) {  // SURVEY 8(d) split-search bytes of the subtree nodes: 20 B per entry visit
+            unsigned long long hv = 0;
+            d2h(&hv, vis.p, 1, s);
+            BF_CUDA_CHECK(cudaStreamSynchronize(s));
+            prof_add_bytes("k_subtree:scan_bytes", (double)hv * 20.0);
           }
           if (want_stats) {
             unsigned long long h[24];

@@ -19,7 +19,6 @@
 #include <cmath>
 #include <vector>
 
-#include <cub/cub.cuh>
 
 #include "bf_internal.cuh"
 
@@ -659,9 +658,18 @@ __global__ void k_mars_eval(const double* __restrict__ X, int64_t ldx, int64_t n
   out[i] = y ? y[i] - f : f;
 }
 
-__global__ void k_mars_canon(const double* __restrict__ x, int64_t n, double* __restrict__ out) {
+// order-preserving 64-bit key of the canonical value (-0 -> +0, R18) for the hand-written radix sort, and back
+__global__ void k_mars_key(const double* __restrict__ x, int64_t n, uint64_t* __restrict__ out) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-  if (i < n) out[i] = __dadd_rn(x[i], 0.0);  // -0 -> +0 (R18)
+  if (i >= n) return;
+  const uint64_t b = (uint64_t)__double_as_longlong(__dadd_rn(x[i], 0.0));
+  out[i] = (b >> 63) ? ~b : (b | 0x8000000000000000ull);
+}
+__global__ void k_mars_unkey(const uint64_t* __restrict__ k, int64_t n, double* __restrict__ out) {
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const uint64_t v = k[i];
+  out[i] = __longlong_as_double((long long)((v >> 63) ? (v & 0x7fffffffffffffffull) : ~v));
 }
 __global__ void k_mars_sums(const double* __restrict__ y, int64_t n, double* __restrict__ out /* tss, yy */) {
   __shared__ double red[MNT / 32];
@@ -698,23 +706,16 @@ void mars_fit_impl(const double* X_in, int64_t ldx, int64_t n, int32_t d, const 
   std::vector<int32_t> hv;
   std::vector<double> hk;
   {
-    DBuf<double> col(n, s), srt(n, s), uq(n, s);
-    DBuf<int> nu(1, s);
-    size_t tb1 = 0, tb2 = 0;
-    cub::DeviceRadixSort::SortKeys(nullptr, tb1, col.p, srt.p, (int)n, 0, 64, s);
-    cub::DeviceSelect::Unique(nullptr, tb2, srt.p, uq.p, nu.p, (int)n, s);
-    DBuf<char> tmp(std::max<size_t>(std::max(tb1, tb2), 16), s);
+    DBuf<uint64_t> k0(n, s), k1(n, s), uk(n, s);
+    DBuf<double> uq(n, s);
+    DBuf<int32_t> nu(1, s);
     std::vector<double> hu;
     for (int v = 0; v < d; ++v) {
-      k_mars_canon<<<(unsigned)ceil_div(n, 256), 256, 0, s>>>(X + (int64_t)v * ldx, n, col.p);
-      {
-        KScope ks_("cub_SortKeys", s, 0.0);
-        BF_CUDA_CHECK(cub::DeviceRadixSort::SortKeys(tmp.p, tb1, col.p, srt.p, (int)n, 0, 64, s));
-      }
-      {
-        KScope ks_("cub_Unique", s, 0.0);
-        BF_CUDA_CHECK(cub::DeviceSelect::Unique(tmp.p, tb2, srt.p, uq.p, nu.p, (int)n, s));
-      }
+      k_mars_key<<<(unsigned)ceil_div(n, 256), 256, 0, s>>>(X + (int64_t)v * ldx, n, k0.p);
+      const uint64_t* srt = radix_sort_u64(k0.p, k1.p, nullptr, nullptr, n, 1, s, nullptr);
+      unique_u64(srt, n, uk.p, nu.p, s);
+      k_mars_unkey<<<(unsigned)ceil_div(n, 256), 256, 0, s>>>(uk.p, n, uq.p);
+      BF_CUDA_CHECK(cudaGetLastError());
       int hn = 0;
       BF_CUDA_CHECK(cudaMemcpyAsync(&hn, nu.p, sizeof(int), cudaMemcpyDeviceToHost, s));
       BF_CUDA_CHECK(cudaStreamSynchronize(s));

@@ -8,8 +8,6 @@
 #include <algorithm>
 #include <cstdlib>
 
-#include <cub/cub.cuh>
-
 #include "bf_internal.cuh"
 
 namespace bf {
@@ -376,20 +374,14 @@ void pd_grid_impl(const double* x_in, int64_t n, int32_t n_pt, double* grid_in, 
     KScope ks_("k_sort_key_of", s, 0.0);
     k_sort_key_of<<<(unsigned)ceil_div(n, 256), 256, 0, s>>>((const double*)xs.dptr, n, keys.p);
   }
-  size_t tb = 0;
-  cub::DeviceRadixSort::SortKeys(nullptr, tb, keys.p, sorted.p, (int)n, 0, 64, s);
-  DBuf<char> tmp(std::max<size_t>(tb, 16), s);
-  {
-    KScope ks_("cub_SortKeys", s, 0.0);
-    BF_CUDA_CHECK(cub::DeviceRadixSort::SortKeys(tmp.p, tb, keys.p, sorted.p, (int)n, 0, 64, s));
-  }
+  const uint64_t* srt = radix_sort_u64(keys.p, sorted.p, nullptr, nullptr, n, 1, s, nullptr);
   {
     KScope ks_("k_count_distinct", s, 0.0);
-    k_count_distinct<<<(unsigned)ceil_div(n, 256), 256, 0, s>>>(sorted.p, n, cnt.p);
+    k_count_distinct<<<(unsigned)ceil_div(n, 256), 256, 0, s>>>(srt, n, cnt.p);
   }
   {
     KScope ks_("k_pd_grid", s, 0.0);
-    k_pd_grid<<<1, 64, 0, s>>>(sorted.p, n, cnt.p, n_pt, (double*)gs.dptr, Gd.p);
+    k_pd_grid<<<1, 64, 0, s>>>(srt, n, cnt.p, n_pt, (double*)gs.dptr, Gd.p);
   }
   BF_CUDA_CHECK(cudaGetLastError());
   BF_CUDA_CHECK(cudaMemcpyAsync(G_host, Gd.p, sizeof(int32_t), cudaMemcpyDeviceToHost, s));

@@ -67,3 +67,14 @@ def test_product_does_not_import_oracle():
             if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
                 txt = open(os.path.join(dirpath, f)).read()
                 assert not bad.search(txt), f
+
+
+def test_torch_allocator_hooks_build_and_export():
+    """libbf_torch_alloc.so (the bf_set_allocator hooks over torch's CUDA caching allocator) builds against the
+    installed torch and exports the two hook functions the binding passes to bf_set_allocator."""
+    from paper_conf_ipps_madougouvln16_b200 import build
+    path = build.build_torch_alloc()
+    out = subprocess.check_output(["nm", "-D", "--defined-only", path]).decode()
+    assert re.search(r" T bf_torch_alloc$", out, flags=re.M) and re.search(r" T bf_torch_free$", out, flags=re.M)
+    import ctypes as C
+    C.CDLL(path)  # resolves libc10_cuda / libc10 through its rpath

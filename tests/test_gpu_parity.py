@@ -414,3 +414,27 @@ def test_empty_tree_range_is_an_empty_forest():
     assert w.info.total_nodes == 0
     full = bf.fit(Xd, yd, ntree=3, seed=8)
     assert full.info.tree_end - full.info.tree_begin == 3
+
+
+def test_library_memory_comes_from_the_torch_caching_allocator():
+    """bf_set_allocator is installed with torch's caching allocator by the binding: a forest's device arrays are
+    torch allocations (memory_allocated grows while it lives and drops when it is freed), and the fit's work
+    space is returned to torch's pool (reserved, not allocated) after bf_fit."""
+    assert bf.torch_allocator_active()
+    X, y = S.small_random(3000, 8, seed=21)
+    Xd, yd = dev(X), dev(y)
+    torch.cuda.synchronize()
+    a0 = torch.cuda.memory_allocated()
+    f = bf.fit(Xd, yd, ntree=8, seed=3)
+    torch.cuda.synchronize()
+    a1 = torch.cuda.memory_allocated()
+    nodes = f.info.total_nodes
+    assert a1 - a0 >= nodes * 16          # at least the 16-byte node array
+    ys, _ = f.predict(Xd, ntree_total=8)  # the lazily built compact copy also comes from torch
+    side = torch.cuda.Stream()
+    with torch.cuda.stream(side):         # a call on another stream: free waits for the device
+        ys2, _ = f.predict(Xd, ntree_total=8)
+    f.free()
+    torch.cuda.synchronize()
+    assert torch.cuda.memory_allocated() - a0 <= 2 * ys.numel() * 8 * 2 + 4096
+    assert torch.equal(ys, ys2)
