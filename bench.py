@@ -57,6 +57,7 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-profile", action="store_true", help="skip the profiled step (per-kernel table)")
     ap.add_argument("--e2e-steps", type=int, default=1)
+    ap.add_argument("--trees-in-flight", type=int, default=0, help="bf_params.trees_in_flight (0: library's choice)")
     return ap.parse_args()
 
 
@@ -379,7 +380,8 @@ def run_ours(args):
         e = [ev() for _ in range(5)]
         e[0].record(stream)
         Xf, pc = rf_inputs(Xs, host)                          # C3: PCA first
-        forest = bf.fit(Xf, ys_, ntree=T, seed=S.FOREST_SEED + 4, tree_begin=t0, tree_end=t1)
+        forest = bf.fit(Xf, ys_, ntree=T, seed=S.FOREST_SEED + 4, tree_begin=t0, tree_end=t1,
+                        trees_in_flight=args.trees_in_flight)
         e[1].record(stream)
         pred = None
         if Qs is not None:

@@ -1366,9 +1366,10 @@ struct TNode {  // tiny node: mask over the rows of its tiny root [rlo, rlo+ra)
   int32_t rlo, ra;
   uint64_t mask;
   int32_t id;
-  int32_t n;           // written last: n > 0 marks the entry as ready
+  int32_t n;
   int64_t S;
   uint64_t key;
+  double value;  // node value (S4.7): the warp that grows the node writes its whole record
 };
 struct WRec {  // best candidate found by one warp for its share of a node's features
   double g;
@@ -1452,37 +1453,51 @@ __device__ __forceinline__ void warp_draw_mtry(uint64_t seed, uint32_t t, uint64
 }
 
 // Tiny-node work queue (shared memory).  Every access to a queue entry, its ready flag and the queue
-// counters is an atomic (cuda::atomic_ref, block scope): the producer writes the entry's fields with relaxed
-// stores and publishes it with a release store of ready[idx]; the consumer's lane 0 spins on an acquire load
-// of the flag, reads the fields and broadcasts them to its warp.  So the hand-off is ordered by the memory
-// model (no volatile + fence idiom) and carries no plain shared-memory accesses for racecheck to flag.
+// counters is an atomic read-modify-write through cuda::atomic_ref (block scope): the producer writes the
+// entry's fields with relaxed exchanges and publishes it with a release exchange of ready[idx]; the consumer's
+// lane 0 spins on an acquire fetch_or(0) of the flag, reads the fields with relaxed fetch_or(0) and broadcasts
+// them to its warp.  The hand-off is ordered by the memory model (release/acquire on the flag), and since
+// every cross-warp access is an atomic RMW, compute-sanitizer's racecheck (which models barriers and atomics,
+// not ld/st.acquire/release) has no plain shared-memory access to report.
 template <class T>
 using blk_ref = cuda::atomic_ref<T, cuda::thread_scope_block>;
+using u64 = unsigned long long;
+
+template <class T>
+__device__ __forceinline__ void a_put(T& x, T v) {
+  blk_ref<T>(x).exchange(v, cuda::memory_order_relaxed);
+}
+template <class T>
+__device__ __forceinline__ T a_get(T& x) {
+  return blk_ref<T>(x).fetch_or(T(0), cuda::memory_order_relaxed);
+}
 
 __device__ __forceinline__ void tq_push(TNode* q, int32_t* ready, int* alloc, int* pending, const TNode& c) {
   atomicAdd(pending, 1);
   const int idx = atomicAdd(alloc, 1);
   TNode& e = q[idx];
-  blk_ref<int32_t>(e.rlo).store(c.rlo, cuda::memory_order_relaxed);
-  blk_ref<int32_t>(e.ra).store(c.ra, cuda::memory_order_relaxed);
-  blk_ref<unsigned long long>(*(unsigned long long*)&e.mask).store(c.mask, cuda::memory_order_relaxed);
-  blk_ref<int32_t>(e.id).store(c.id, cuda::memory_order_relaxed);
-  blk_ref<int32_t>(e.n).store(c.n, cuda::memory_order_relaxed);
-  blk_ref<long long>(*(long long*)&e.S).store(c.S, cuda::memory_order_relaxed);
-  blk_ref<unsigned long long>(*(unsigned long long*)&e.key).store(c.key, cuda::memory_order_relaxed);
-  blk_ref<int32_t>(ready[idx]).store(1, cuda::memory_order_release);
+  a_put<int32_t>(e.rlo, c.rlo);
+  a_put<int32_t>(e.ra, c.ra);
+  a_put<u64>(*(u64*)&e.mask, (u64)c.mask);
+  a_put<int32_t>(e.id, c.id);
+  a_put<int32_t>(e.n, c.n);
+  a_put<u64>(*(u64*)&e.S, (u64)c.S);
+  a_put<u64>(*(u64*)&e.key, (u64)c.key);
+  a_put<u64>(*(u64*)&e.value, (u64)__double_as_longlong(c.value));
+  blk_ref<int32_t>(ready[idx]).exchange(1, cuda::memory_order_release);
 }
 
 __device__ __forceinline__ TNode tq_read(TNode* q, int idx) {  // after an acquire of ready[idx] (or a barrier)
   TNode& e = q[idx];
   TNode c;
-  c.rlo = blk_ref<int32_t>(e.rlo).load(cuda::memory_order_relaxed);
-  c.ra = blk_ref<int32_t>(e.ra).load(cuda::memory_order_relaxed);
-  c.mask = blk_ref<unsigned long long>(*(unsigned long long*)&e.mask).load(cuda::memory_order_relaxed);
-  c.id = blk_ref<int32_t>(e.id).load(cuda::memory_order_relaxed);
-  c.n = blk_ref<int32_t>(e.n).load(cuda::memory_order_relaxed);
-  c.S = blk_ref<long long>(*(long long*)&e.S).load(cuda::memory_order_relaxed);
-  c.key = blk_ref<unsigned long long>(*(unsigned long long*)&e.key).load(cuda::memory_order_relaxed);
+  c.rlo = a_get<int32_t>(e.rlo);
+  c.ra = a_get<int32_t>(e.ra);
+  c.mask = (uint64_t)a_get<u64>(*(u64*)&e.mask);
+  c.id = a_get<int32_t>(e.id);
+  c.n = a_get<int32_t>(e.n);
+  c.S = (int64_t)a_get<u64>(*(u64*)&e.S);
+  c.key = (uint64_t)a_get<u64>(*(u64*)&e.key);
+  c.value = __longlong_as_double((long long)a_get<u64>(*(u64*)&e.value));
   return c;
 }
 
@@ -1495,6 +1510,7 @@ __device__ __forceinline__ TNode tq_bcast(const TNode& c) {  // lane 0's entry t
   r.n = __shfl_sync(0xffffffffu, c.n, 0);
   r.S = __shfl_sync(0xffffffffu, c.S, 0);
   r.key = __shfl_sync(0xffffffffu, c.key, 0);
+  r.value = __shfl_sync(0xffffffffu, c.value, 0);
   return r;
 }
 
@@ -1571,7 +1587,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
     wy[j] = (int64_t)wv * yqr;
     wyd[j] = __dmul_rn((double)wv, yr);
   }
-  for (int j = tid; j <= a0; j += SUB_NT) blk_ref<int32_t>(tq_ready[j]).store(0, cuda::memory_order_relaxed);
+  for (int j = tid; j <= a0; j += SUB_NT) tq_ready[j] = 0;  // barrier-ordered before any queue use
   __syncthreads();
   auto hfind = [&](uint32_t row) -> uint16_t {
     uint32_t h = (row * 0x9E3779B1u) >> (32 - HBITS);
@@ -1661,6 +1677,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
     c.n = root.n;
     c.S = root.S;
     c.key = root.key;
+    c.value = 0.0;  // the root's value is the pool's (written before the subtree phase)
     tq_push(tq, tq_ready, &s_alloc, &s_pending, c);
   }
   __syncthreads();
@@ -1897,6 +1914,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
             c.n = nn;
             c.S = S;
             c.key = key;
+            c.value = recs[nd.lid + sdv].value;  // written by the node's warp before the last barrier
             tq_push(tq, tq_ready, &s_alloc, &s_pending, c);
           }
         }
@@ -1956,7 +1974,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   // ================= tiny nodes: row index inside each tiny root, then the work queue
   tclk[2] = clock64();
   {
-    const int nroots = blk_ref<int>(s_alloc).load(cuda::memory_order_relaxed);
+    const int nroots = a_get<int>(s_alloc);
     for (int qi = wid; qi < nroots; qi += SUB_NW) {
       const TNode r = tq_read(tq, qi);  // pushed before the barrier above
       for (int k = lane; k < r.ra; k += 32) rmap[list[r.rlo + k] & 0xffffu] = (uint8_t)k;
@@ -1969,13 +1987,13 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
     if (lane == 0) {
       unsigned ns = 32;
       for (;;) {
-        const int hd = blk_ref<int>(s_head).load(cuda::memory_order_relaxed);
-        if (hd < blk_ref<int>(s_alloc).load(cuda::memory_order_relaxed)) {
+        const int hd = a_get<int>(s_head);
+        if (hd < a_get<int>(s_alloc)) {
           if (atomicCAS(&s_head, hd, hd + 1) == hd) {
             h = hd;
             break;
           }
-        } else if (blk_ref<int>(s_pending).load(cuda::memory_order_relaxed) == 0) {
+        } else if (a_get<int>(s_pending) == 0) {
           break;
         } else {
           __nanosleep(ns);  // idle warp: back off so the busy warps keep the issue slots
@@ -1983,7 +2001,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         }
       }
       if (h >= 0) {
-        while (blk_ref<int32_t>(tq_ready[h]).load(cuda::memory_order_acquire) == 0) __nanosleep(32);
+        while (blk_ref<int32_t>(tq_ready[h]).fetch_or(0, cuda::memory_order_acquire) == 0) __nanosleep(32);
         nd = tq_read(tq, h);
       }
     }
@@ -2228,36 +2246,48 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
           vl += __shfl_down_sync(0xffffffffu, vl, o);
           vr += __shfl_down_sync(0xffffffffu, vr, o);
         }
+        const int nr = nd.n - bnl;
+        const bool gl = bnl > g.nodesize && __popcll(mL) >= 2;
+        const bool gr = nr > g.nodesize && __popcll(mR) >= 2;
+        const double val_l = __ddiv_rn(vl, (double)bnl), val_r = __ddiv_rn(vr, (double)nr);
+        // Records: a node's whole record is written by the warp that grows it (this one for nd); a child that
+        // stays a leaf gets its record here, a child that is grown further (here or by the warp that takes it
+        // from the queue) writes its own -- so no record is written by two warps without a barrier between.
         int lid = 0;
         if (lane == 0) {
           lid = atomicAdd(&s_nloc, 2);
-          SRec& r = recs[nd.id];
+          SRec r;
           r.feature = bf;
           r.left = lid;
+          r.count = nd.n;
           r.ra = (uint16_t)bra;
           r.rb = (uint16_t)brb;
+          r.value = nd.value;
           r.drss = ldexp(__ddiv_rn(bg, (double)nd.n), -2 * g.q);
-          const int nr = nd.n - bnl;
+          recs[nd.id] = r;
           SRec c;
           c.feature = -1;
           c.left = -1;
           c.ra = c.rb = 0;
           c.drss = 0.0;
-          c.count = bnl;
-          c.value = __ddiv_rn(vl, (double)bnl);
-          recs[lid] = c;
-          c.count = nr;
-          c.value = __ddiv_rn(vr, (double)nr);
-          recs[lid + 1] = c;
+          if (!gl) {
+            c.count = bnl;
+            c.value = val_l;
+            recs[lid] = c;
+          }
+          if (!gr) {
+            c.count = nr;
+            c.value = val_r;
+            recs[lid + 1] = c;
+          }
         }
         lid = __shfl_sync(0xffffffffu, lid, 0);
         // child keys on lanes 0 and 1
         const uint64_t ck = child_key(g.seed, t, nd.key, lane & 1);
         const uint64_t kl = __shfl_sync(0xffffffffu, ck, 0), kr = __shfl_sync(0xffffffffu, ck, 1);
-        const int nr = nd.n - bnl;
-        const bool gl = bnl > g.nodesize && __popcll(mL) >= 2;
-        const bool gr = nr > g.nodesize && __popcll(mR) >= 2;
         TNode cl, cr;
+        cl.value = val_l;
+        cr.value = val_r;
         cl.rlo = cr.rlo = nd.rlo;
         cl.ra = cr.ra = nd.ra;
         cl.mask = mL;
@@ -2284,6 +2314,15 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
           nd = cr;
           have = true;
         }
+      } else if (lane == 0) {  // no positive-gain split (S4.5): the node is a leaf; its record is written here
+        SRec r;
+        r.feature = -1;
+        r.left = -1;
+        r.count = nd.n;
+        r.ra = r.rb = 0;
+        r.value = nd.value;
+        r.drss = 0.0;
+        recs[nd.id] = r;
       }
 
     }
@@ -2577,6 +2616,16 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
     if (memory_budget() > 0) fr = (size_t)memory_budget();
     const size_t budget = fr / 2;
     B = (int)std::max<size_t>(1, std::min<size_t>(budget / std::max<size_t>(per_tree, 1), 256));
+    // Large trees: the split-scan and partition CTAs are bound to trees (148 / B CTAs per tree), so a level
+    // lasts as long as the tree with the fewest CTAs per unit of work.  Keep that count even: B = SMs / 4
+    // (4 partition CTAs per tree) when memory allows, else at most SMs / 7 (ragged 7-8 CTAs per tree).
+    if (n >= 65536) {
+      int nsm_ = 0, dv_ = 0;
+      cudaGetDevice(&dv_);
+      cudaDeviceGetAttribute(&nsm_, cudaDevAttrMultiProcessorCount, dv_);
+      nsm_ = std::max(nsm_, 8);
+      B = B >= nsm_ / 4 ? nsm_ / 4 : std::min(B, nsm_ / 7);
+    }
   }
   B = std::max(1, std::min(B, std::max(T_loc, 1)));
 

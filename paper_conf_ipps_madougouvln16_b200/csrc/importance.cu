@@ -380,6 +380,7 @@ struct Imp8Args {
   ImpArgs a;
   const uint2* nodes8;
   const uint32_t* roots8;  // per local tree (forest numbering)
+  unsigned long long* prof;  // profile mode: [0] node loads, [1] permuted re-walks (algorithmic bytes), else NULL
 };
 
 __global__ void __launch_bounds__(IPT) k_importance8(Imp8Args g8) {
@@ -420,6 +421,7 @@ __global__ void __launch_bounds__(IPT) k_importance8(Imp8Args g8) {
     const uint32_t rw = __ldg(g8.roots8 + i);
     const uint32_t root = rw & ~ROOT_LEAF;
     const double yr = g.y[r];
+    uint32_t nld = 1, nrw = 0;  // node loads, re-walks (profile counters)
     // child of internal node (gid, w) for this row, feature pm (if tested) taking the value (xpf, xpd)
     auto child = [&](uint32_t gid, uint2 w, int pm, float xpf, double xpd, bool& leaf) -> uint32_t {
       const uint32_t f = n8_feature(w);
@@ -444,6 +446,7 @@ __global__ void __launch_bounds__(IPT) k_importance8(Imp8Args g8) {
         bool leaf;
         const uint32_t c = child(gid, w, -1, 0.f, 0.0, leaf);
         const uint2 ch = __ldg(n8 + c);
+        ++nld;
         if (leaf) {
           f0v = leaf8(ch);
           break;
@@ -502,10 +505,12 @@ __global__ void __launch_bounds__(IPT) k_importance8(Imp8Args g8) {
           } else {
             gid = c;
             w = __ldg(n8 + c);
+            ++nld;
           }
           ++depth;
         }
         if (cnt == 0) break;
+        nrw += cnt;
         double xm[ILP];
         float xmf[ILP];
         bool live[ILP];
@@ -531,6 +536,7 @@ __global__ void __launch_bounds__(IPT) k_importance8(Imp8Args g8) {
               bool leaf;
               const uint32_t c = child(qg[u], qw[u], qm[u], xmf[u], xm[u], leaf);
               const uint2 ch = __ldg(n8 + c);
+              ++nld;
               if (leaf) {
                 val[u] = leaf8(ch);
                 live[u] = false;
@@ -548,6 +554,14 @@ __global__ void __launch_bounds__(IPT) k_importance8(Imp8Args g8) {
             const double diff = d1 * d1 - err0;
             if (diff != 0.0) atomicAdd(&sacc[qm[u]], diff);
           }
+      }
+    }
+    if (g8.prof) {  // one atomic pair per warp
+      const unsigned act_m = __activemask();
+      const uint32_t wl = __reduce_add_sync(act_m, nld), wr = __reduce_add_sync(act_m, nrw);
+      if ((threadIdx.x & 31) == __ffs(act_m) - 1) {
+        atomicAdd(&g8.prof[0], (unsigned long long)wl);
+        atomicAdd(&g8.prof[1], (unsigned long long)wr);
       }
     }
   }
@@ -691,6 +705,11 @@ void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, co
   const size_t smem8 = sizeof(double) * (size_t)((p + 1) & ~1) + sizeof(float) * (size_t)IPT * (size_t)(p | 1);
   static int ismax8 = 0;
   if (!ismax8) ismax8 = dyn_smem_limit(k_importance8);
+  DBuf<unsigned long long> prof;
+  if (prof_enabled()) {
+    prof.alloc(2, s);
+    BF_CUDA_CHECK(cudaMemsetAsync(prof.p, 0, 16, s));
+  }
   for (int32_t i0 = 0; i0 < T; i0 += B) {
     const int Bc = std::min(B, T - i0);
     bootstrap_impl(f->info.seed, f->info.tree_begin + i0, Bc, n, f->info.sampsize, f->info.replace, w.p, s);
@@ -754,6 +773,7 @@ void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, co
       g8.a = g;
       g8.nodes8 = n8;
       g8.roots8 = f->d_roots8;
+      g8.prof = prof.p;
       KScope ks_("k_importance8", s, 0.0);
       k_importance8<<<dim3((unsigned)ceil_div(n, IPT), Bc), IPT, smem8, s>>>(g8);
     } else {
@@ -764,6 +784,20 @@ void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, co
         k_importance<IPT><<<dim3((unsigned)ceil_div(n, IPT), Bc), IPT, smem, s>>>(g);
     }
     BF_CUDA_CHECK(cudaGetLastError());
+  }
+  if (prof.p && T > 0) {  // algorithmic bytes of k_importance8
+    unsigned long long hp[2] = {0, 0};
+    std::vector<int64_t> hno(T);
+    BF_CUDA_CHECK(cudaMemcpyAsync(hp, prof.p, 16, cudaMemcpyDeviceToHost, s));
+    BF_CUDA_CHECK(cudaMemcpyAsync(hno.data(), nout_t, sizeof(int64_t) * T, cudaMemcpyDeviceToHost, s));
+    BF_CUDA_CHECK(cudaStreamSynchronize(s));
+    double units = 0.0;
+    for (int64_t v : hno) units += (double)v;
+    // per (tree, OOB row): row gather 8p + y 8 + O index 4 + oob sum/count 12; per re-walk: pi 4 + x 8;
+    // per node load 8 (compact nodes)
+    prof_add_bytes("k_importance8", units * (8.0 * p + 24.0) + (double)hp[1] * 12.0 + (double)hp[0] * 8.0);
+    prof_add_bytes("importance_node_loads", (double)hp[0]);
+    prof_add_bytes("importance_rewalks", (double)hp[1]);
   }
   if (T > 0) {
     {
