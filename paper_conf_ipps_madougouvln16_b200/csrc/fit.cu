@@ -1344,6 +1344,7 @@ __global__ void __launch_bounds__(NT) k_dest_bits(DestArgs g, uint32_t* sideb, i
 // list partition is needed.  Tiny nodes go through a CTA-wide work queue so
 // every warp stays busy until the whole subtree is grown.
 constexpr int TINY = 64;
+constexpr int MAXR = 32;  // small roots packed into one subtree CTA (their distinct rows add up to <= A)
 constexpr int HBITS = 12, HSLOTS = 1 << HBITS;  // load-phase hash table (global row -> local id), a0 <= 1024
 constexpr int TGRP = 7;   // drawn predictors staged per group in the tiny path
 constexpr int TPU = 4;    // scan passes interleaved in the tiny path
@@ -1394,8 +1395,8 @@ __host__ __device__ inline size_t subtree_smem(int A, int p) {
   s += align16((size_t)A) * 2;                        // side, row index inside its tiny root
   s += align16((size_t)2 * A * sizeof(SRec));         // node records
   s += align16((size_t)2 * max_medium(A) * sizeof(MNode));
-  s += align16((size_t)(A + 1) * sizeof(TNode));      // tiny work queue
-  s += align16((size_t)(A + 1) * 4);                  // its ready flags
+  s += align16((size_t)(A + MAXR) * sizeof(TNode));   // tiny work queue
+  s += align16((size_t)(A + MAXR) * 4);               // its ready flags
   s += align16((size_t)SUB_NW * p * 2) * 2;           // Fisher-Yates scratch, drawn features
   s += align16((size_t)SUB_NW * sizeof(WRec));
   s += 64;
@@ -1404,6 +1405,8 @@ __host__ __device__ inline size_t subtree_smem(int A, int p) {
 
 struct SubArgs {
   const LNode* sq;
+  const int32_t* gperm;   // small roots in packing order (indices into sq)
+  const int32_t* gstart;  // CTA g grows the roots gperm[gstart[g] .. gstart[g+1])
   const uint64_t* Es;
   const int64_t* yq;
   const double* y;
@@ -1540,24 +1543,44 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   MNode* nxtl = curl + MM;
   ptr += align16((size_t)2 * MM * sizeof(MNode));
   TNode* tq = (TNode*)ptr;
-  ptr += align16((size_t)(A + 1) * sizeof(TNode));
+  ptr += align16((size_t)(A + MAXR) * sizeof(TNode));
   int32_t* tq_ready = (int32_t*)ptr;
-  ptr += align16((size_t)(A + 1) * 4);
+  ptr += align16((size_t)(A + MAXR) * 4);
   int16_t* mind_all = (int16_t*)ptr;
   ptr += align16((size_t)SUB_NW * p * 2);
   int16_t* feats_all = (int16_t*)ptr;
   ptr += align16((size_t)SUB_NW * p * 2);
   WRec* wrec = (WRec*)ptr;
   ptr += align16((size_t)SUB_NW * sizeof(WRec));
-  __shared__ int s_nloc, s_ncur, s_gbase, s_alloc, s_head, s_pending;
+  __shared__ int s_ncur, s_alloc, s_head, s_pending;
   __shared__ int32_t s_scan[SUB_NW];
+  // packed roots: local rows [s_off[r], s_off[r+1]), records [2 s_off[r], ...) (a tree over a rows has < 2a
+  // nodes), next free record s_nloc[r]; node ids carry their root: id = r << 16 | record
+  __shared__ int s_off[MAXR + 1], s_b[MAXR], s_nloc[MAXR], s_gbase[MAXR];
+  __shared__ LNode s_root[MAXR];
 
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  const LNode root = g.sq[blockIdx.x];
-  const int a0 = root.a;
-  const int b = root.b;
-  const uint32_t t = (uint32_t)(g.t0 + b);
-  const uint64_t* src = g.Es + root.base;
+  const int g0 = g.gstart[blockIdx.x], nr = g.gstart[blockIdx.x + 1] - g0;
+  if (tid < nr) s_root[tid] = g.sq[g.gperm[g0 + tid]];
+  __syncthreads();
+  if (tid == 0) {
+    int o = 0;
+    for (int r = 0; r < nr; ++r) {
+      s_off[r] = o;
+      s_b[r] = s_root[r].b;
+      s_nloc[r] = 2 * o + 1;
+      o += s_root[r].a;
+    }
+    s_off[nr] = o;
+  }
+  __syncthreads();
+  const int a0 = s_off[nr];  // rows of all packed roots = the stride of a feature row of `list`
+  auto t_of = [&](int32_t id) -> uint32_t { return (uint32_t)(g.t0 + s_b[id >> 16]); };
+  auto root_of_row = [&](int j) -> int {  // packed root holding local row j
+    int r = 0;
+    while (r + 1 < nr && s_off[r + 1] <= j) ++r;
+    return r;
+  };
   int16_t* mind = mind_all + wid * p;
   int16_t* feats = feats_all + wid * p;
   uint32_t* temp = temp_all + (size_t)wid * sub_temp(A);
@@ -1574,24 +1597,26 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   for (int k = tid; k < HSLOTS; k += SUB_NT) hkey[k] = 0xffffffffu;
   __syncthreads();
   for (int j = tid; j < a0; j += SUB_NT) {
-    const uint64_t ej = src[j];
+    const int r = root_of_row(j);
+    const uint64_t ej = g.Es[s_root[r].base + (j - s_off[r])];  // feature 0's segment of root r
     const uint32_t row = e_row(ej);
     const int32_t wv = e_w(ej);
     const int64_t yqr = g.yq[row];
     const double yr = g.y[row];
     grow[j] = row;
-    uint32_t h = (row * 0x9E3779B1u) >> (32 - HBITS);
-    while (atomicCAS(&hkey[h], 0xffffffffu, row) != 0xffffffffu) h = (h + 1) & (HSLOTS - 1);
+    const uint32_t hk = row | ((uint32_t)r << 24);  // the same row may sit in two packed roots (two trees)
+    uint32_t h = (hk * 0x9E3779B1u) >> (32 - HBITS);
+    while (atomicCAS(&hkey[h], 0xffffffffu, hk) != 0xffffffffu) h = (h + 1) & (HSLOTS - 1);
     hval[h] = (uint16_t)j;
     wl[j] = wv;
     wy[j] = (int64_t)wv * yqr;
     wyd[j] = __dmul_rn((double)wv, yr);
   }
-  for (int j = tid; j <= a0; j += SUB_NT) tq_ready[j] = 0;  // barrier-ordered before any queue use
+  for (int j = tid; j < a0 + MAXR; j += SUB_NT) tq_ready[j] = 0;  // barrier-ordered before any queue use
   __syncthreads();
-  auto hfind = [&](uint32_t row) -> uint16_t {
-    uint32_t h = (row * 0x9E3779B1u) >> (32 - HBITS);
-    while (hkey[h] != row) h = (h + 1) & (HSLOTS - 1);
+  auto hfind = [&](uint32_t hk) -> uint16_t {
+    uint32_t h = (hk * 0x9E3779B1u) >> (32 - HBITS);
+    while (hkey[h] != hk) h = (h + 1) & (HSLOTS - 1);
     return hval[h];
   };
   // ---- load 2: warp per feature; local rank = index of the first entry of the same value.  Coalesced: chunk c
@@ -1599,9 +1624,12 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   // up to 16 chunks (a0 <= 512) in flight per warp; the value breaks are max-scanned per chunk with a carry.
   {
     constexpr int GRP = 16;
-    const int nch = (a0 + 31) >> 5;
-    for (int f = wid; f < p; f += SUB_NW) {
-      const uint64_t* sf = src + (int64_t)f * a0;
+    for (int it = wid; it < nr * p; it += SUB_NW) {  // (packed root, feature) items
+      const int r = it / p, f = it - r * p;
+      const int ar = s_root[r].a, orr = s_off[r];
+      const int nch = (ar + 31) >> 5;
+      const uint64_t* sf = g.Es + s_root[r].base + (int64_t)f * ar;
+      const uint32_t rtag = (uint32_t)r << 24;
       int carry_gs = 0;
       uint32_t prev_last = 0xffffffffu;
       for (int c0 = 0; c0 < nch; c0 += GRP) {
@@ -1609,15 +1637,15 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
 #pragma unroll
         for (int c = 0; c < GRP; ++c) {
           const int j = (c0 + c) * 32 + lane;
-          ev[c] = (c0 + c < nch && j < a0) ? sf[j] : ~0ull;
+          ev[c] = (c0 + c < nch && j < ar) ? sf[j] : ~0ull;
         }
         uint32_t rk[GRP];
         uint16_t lr[GRP];
 #pragma unroll
         for (int c = 0; c < GRP; ++c) {
           const int j = (c0 + c) * 32 + lane;
-          rk[c] = j < a0 ? e_rank(ev[c]) : 0xffffffffu;
-          lr[c] = (c0 + c < nch && j < a0) ? hfind(e_row(ev[c])) : 0;
+          rk[c] = j < ar ? e_rank(ev[c]) : 0xffffffffu;
+          lr[c] = (c0 + c < nch && j < ar) ? hfind(e_row(ev[c]) | rtag) : 0;
         }
 #pragma unroll
         for (int c = 0; c < GRP; ++c) {
@@ -1632,7 +1660,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
             if (lane >= o) gs = max(gs, v);
           }
           gs = max(gs, carry_gs);
-          if (j < a0) list[(size_t)f * a0 + j] = ((uint32_t)gs << 16) | lr[c];
+          if (j < ar) list[(size_t)f * a0 + orr + j] = ((uint32_t)(orr + gs) << 16) | lr[c];
           carry_gs = __shfl_sync(0xffffffffu, gs, 31);
           prev_last = __shfl_sync(0xffffffffu, rk[c], 31);
         }
@@ -1640,45 +1668,46 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
     }
   }
   if (tid == 0) {
-    s_nloc = 1;
     s_head = 0;
     s_alloc = 0;
     s_pending = 0;
+    s_ncur = 0;
+  }
+  __syncthreads();
+  if (tid < nr) {  // each packed root: its record, then a medium node or a tiny root
+    const int r = tid;
+    const LNode& R = s_root[r];
+    const int rec0 = 2 * s_off[r];
     SRec r0;
     r0.feature = -1;
     r0.left = -1;
-    r0.count = root.n;
+    r0.count = R.n;
     r0.ra = r0.rb = 0;
     r0.value = 0.0;
     r0.drss = 0.0;
-    recs[0] = r0;
-    if (a0 > TINY) {
+    recs[rec0] = r0;
+    if (R.a > TINY) {
       MNode c;
-      c.lo = 0;
-      c.a = a0;
-      c.n = root.n;
-      c.id = 0;
-      c.S = root.S;
-      c.key = root.key;
+      c.lo = s_off[r];
+      c.a = R.a;
+      c.n = R.n;
+      c.id = (r << 16) | rec0;
+      c.S = R.S;
+      c.key = R.key;
       c.split = 0;
-      curl[0] = c;
-      s_ncur = 1;
+      curl[atomicAdd(&s_ncur, 1)] = c;
     } else {
-      s_ncur = 0;
+      TNode c;
+      c.rlo = s_off[r];
+      c.ra = R.a;
+      c.mask = R.a == 64 ? ~0ull : ((1ull << R.a) - 1ull);
+      c.id = (r << 16) | rec0;
+      c.n = R.n;
+      c.S = R.S;
+      c.key = R.key;
+      c.value = 0.0;  // a root's value is the pool's (written before the subtree phase)
+      tq_push(tq, tq_ready, &s_alloc, &s_pending, c);
     }
-  }
-  __syncthreads();
-  if (a0 <= TINY && tid == 0) {
-    TNode c;
-    c.rlo = 0;
-    c.ra = a0;
-    c.mask = a0 == 64 ? ~0ull : ((1ull << a0) - 1ull);
-    c.id = 0;
-    c.n = root.n;
-    c.S = root.S;
-    c.key = root.key;
-    c.value = 0.0;  // the root's value is the pool's (written before the subtree phase)
-    tq_push(tq, tq_ready, &s_alloc, &s_pending, c);
   }
   __syncthreads();
   tclk[1] = clock64();
@@ -1697,7 +1726,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
     const int NG = max(1, min(SUB_NW, cap_items / g.mtry));
     for (int n0 = 0; n0 < ncur; n0 += NG) {
       const int nn = min(NG, ncur - n0);
-      if (wid < nn) warp_draw_mtry(g.seed, t, curl[n0 + wid].key, p, g.mtry, mind_all + wid * p, feats_all + wid * p, lane);
+      if (wid < nn) warp_draw_mtry(g.seed, t_of(curl[n0 + wid].id), curl[n0 + wid].key, p, g.mtry, mind_all + wid * p, feats_all + wid * p, lane);
       __syncthreads();
       const int nit = nn * g.mtry;
       for (int it = wid; it < nit; it += SUB_NW) {
@@ -1822,15 +1851,15 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         if (best.g > 0.0) {
           int lid = 0;
           if (lane == 0) {
-            lid = atomicAdd(&s_nloc, 2);
-            SRec& r = recs[nd.id];
+            lid = atomicAdd(&s_nloc[nd.id >> 16], 2);
+            SRec& r = recs[nd.id & 0xffff];
             r.feature = best.f;
             r.left = lid;
             r.ra = (uint16_t)best.ra;
             r.rb = (uint16_t)best.rb;
             r.drss = ldexp(__ddiv_rn(best.g, (double)nd.n), -2 * g.q);
-            nd.keyl = child_key(g.seed, t, nd.key, 0);
-            nd.keyr = child_key(g.seed, t, nd.key, 1);
+            nd.keyl = child_key(g.seed, t_of(nd.id), nd.key, 0);
+            nd.keyr = child_key(g.seed, t_of(nd.id), nd.key, 1);
           }
           lid = __shfl_sync(0xffffffffu, lid, 0);
           const uint32_t* seg = list + (size_t)best.f * a0 + nd.lo;
@@ -1900,7 +1929,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
             c.lo = lo;
             c.a = a;
             c.n = nn;
-            c.id = nd.lid + sdv;
+            c.id = (nd.id & ~0xffff) | (nd.lid + sdv);
             c.S = S;
             c.key = key;
             c.split = 0;
@@ -1910,7 +1939,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
             c.rlo = lo;
             c.ra = a;
             c.mask = a == 64 ? ~0ull : ((1ull << a) - 1ull);
-            c.id = nd.lid + sdv;
+            c.id = (nd.id & ~0xffff) | (nd.lid + sdv);
             c.n = nn;
             c.S = S;
             c.key = key;
@@ -2017,6 +2046,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       const int an = __popcll(nd.mask);  // distinct rows of the node
       nvis += (unsigned long long)an * (unsigned)g.mtry;
       const long long c0_ = g.stats ? clock64() : 0;
+      const uint32_t t = t_of(nd.id);
       warp_draw_mtry(g.seed, t, nd.key, p, g.mtry, mind, feats, lane);
       const long long c1_ = g.stats ? clock64() : 0;
       const int64_t nk = nd.n, Sk = nd.S;
@@ -2255,7 +2285,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         // from the queue) writes its own -- so no record is written by two warps without a barrier between.
         int lid = 0;
         if (lane == 0) {
-          lid = atomicAdd(&s_nloc, 2);
+          lid = atomicAdd(&s_nloc[nd.id >> 16], 2);
           SRec r;
           r.feature = bf;
           r.left = lid;
@@ -2264,7 +2294,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
           r.rb = (uint16_t)brb;
           r.value = nd.value;
           r.drss = ldexp(__ddiv_rn(bg, (double)nd.n), -2 * g.q);
-          recs[nd.id] = r;
+          recs[nd.id & 0xffff] = r;
           SRec c;
           c.feature = -1;
           c.left = -1;
@@ -2291,12 +2321,12 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         cl.rlo = cr.rlo = nd.rlo;
         cl.ra = cr.ra = nd.ra;
         cl.mask = mL;
-        cl.id = lid;
+        cl.id = (nd.id & ~0xffff) | lid;
         cl.n = bnl;
         cl.S = bSl;
         cl.key = kl;
         cr.mask = mR;
-        cr.id = lid + 1;
+        cr.id = (nd.id & ~0xffff) | (lid + 1);
         cr.n = nr;
         cr.S = nd.S - bSl;
         cr.key = kr;
@@ -2322,7 +2352,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         r.ra = r.rb = 0;
         r.value = nd.value;
         r.drss = 0.0;
-        recs[nd.id] = r;
+        recs[nd.id & 0xffff] = r;
       }
 
     }
@@ -2334,25 +2364,31 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   const long long t_tiny_end = clock64();
   __syncthreads();
   tclk[3] = clock64();
-  // ---- flush the subtree into the tree's raw pool (sibling pairs stay adjacent)
-  if (tid == 0) s_gbase = s_nloc > 1 ? atomicAdd(&g.pool.nn[b], s_nloc - 1) : 0;
+  // ---- flush every packed subtree into its tree's raw pool (sibling pairs stay adjacent)
+  if (tid < nr) {
+    const int nloc = s_nloc[tid] - 2 * s_off[tid];
+    s_gbase[tid] = nloc > 1 ? atomicAdd(&g.pool.nn[s_b[tid]], nloc - 1) : 0;
+  }
   __syncthreads();
-  const int nloc = s_nloc, gbase = s_gbase;
-  const int64_t r0 = (int64_t)b * g.pool.cap;
-  for (int l = tid; l < nloc; l += SUB_NT) {
-    const SRec r = recs[l];
-    const int64_t gid = r0 + (l == 0 ? root.raw : gbase + l - 1);
-    g.pool.feature[gid] = r.feature;
-    g.pool.left[gid] = r.left >= 0 ? gbase + r.left - 1 : -1;
+  for (int l = tid; l < 2 * a0; l += SUB_NT) {
+    int r = 0;
+    while (r + 1 < nr && 2 * s_off[r + 1] <= l) ++r;
+    const int rec0 = 2 * s_off[r];
+    if (l >= s_nloc[r]) continue;  // unused record slot of root r
+    const int k = l - rec0, gbase = s_gbase[r];
+    const SRec rc = recs[l];
+    const int64_t gid = (int64_t)s_b[r] * g.pool.cap + (k == 0 ? s_root[r].raw : gbase + k - 1);
+    g.pool.feature[gid] = rc.feature;
+    g.pool.left[gid] = rc.left >= 0 ? gbase + (rc.left - rec0) - 1 : -1;
     double thr = 0.0;
-    if (r.feature >= 0)
-      thr = split_threshold(canon(g.X[(int64_t)r.feature * g.ldx + grow[r.ra]]),
-                            canon(g.X[(int64_t)r.feature * g.ldx + grow[r.rb]]));
+    if (rc.feature >= 0)
+      thr = split_threshold(canon(g.X[(int64_t)rc.feature * g.ldx + grow[rc.ra]]),
+                            canon(g.X[(int64_t)rc.feature * g.ldx + grow[rc.rb]]));
     g.pool.thr[gid] = thr;
-    g.pool.drss[gid] = r.drss;
-    if (l > 0) {
-      g.pool.count[gid] = r.count;
-      g.pool.value[gid] = r.value;
+    g.pool.drss[gid] = rc.drss;
+    if (k > 0) {
+      g.pool.count[gid] = rc.count;
+      g.pool.value[gid] = rc.value;
     }
   }
   if (g.visits && lane == 0 && nvis) atomicAdd(g.visits, nvis);
@@ -2369,7 +2405,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       atomicAdd(&g.stats[4], (unsigned long long)n_med);
       atomicAdd(&g.stats[5], 1ull);
       atomicAdd(&g.stats[6], (unsigned long long)a0);
-      atomicAdd(&g.stats[9], (unsigned long long)s_nloc);
+      for (int r = 0; r < nr; ++r) atomicAdd(&g.stats[9], (unsigned long long)(s_nloc[r] - 2 * s_off[r]));
     }
     if (lane == 0) {
       atomicAdd(&g.stats[7], (unsigned long long)n_tiny);
@@ -2377,6 +2413,11 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       atomicAdd(&g.stats[10], (unsigned long long)busy);
     }
   }
+}
+
+__global__ void k_small_a(const LNode* sq, int N, int32_t* a) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < N) a[i] = sq[i].a;
 }
 
 // ------------------------------------------------------------------ a11 emit
@@ -2715,6 +2756,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_tp, k_partition_tree, TPNT, tpart_smem);
     const unsigned grid_tscan = (unsigned)std::max(1, occ_ts * nsm), grid_tpart = (unsigned)std::max(1, occ_tp * nsm);
     DBuf<uint64_t> E0, E1, Es;
+    std::vector<int32_t> h_sa;  // distinct rows of the batch's small roots (subtree packing)
     size_t E_cap = 0;
 
     ptm.mark("alloc");
@@ -2917,8 +2959,48 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
         BF_CUDA_CHECK(cudaStreamSynchronize(s));
         if (ls.nsmall > 0) {
           prof_add_bytes("k_subtree", (double)ls.small_elems * 8.0 + (double)ls.small_elems / p * 26.0);
+          // Pack small roots into CTAs (distinct rows adding up to <= A, at most MAXR per CTA): the largest
+          // remaining root first, topped up with the smallest ones, so every CTA has several independent subtrees
+          // whose tiny-node tails overlap (BF_SUBTREE_PACK=0: one root per CTA).
+          static const bool pack = !(getenv("BF_SUBTREE_PACK") && getenv("BF_SUBTREE_PACK")[0] == '0');
+          const int nsm_roots = ls.nsmall;
+          if ((int)h_sa.size() < nsm_roots) h_sa.resize(nsm_roots);
+          DBuf<int32_t> d_sa(nsm_roots, s), d_perm(nsm_roots, s), d_gst(nsm_roots + 1, s);
+          {
+            KScope ks_("k_small_a", s, 0.0);
+            k_small_a<<<(unsigned)ceil_div(nsm_roots, 256), 256, 0, s>>>(sq.p, nsm_roots, d_sa.p);
+          }
+          d2h(h_sa.data(), d_sa.p, nsm_roots, s);
+          BF_CUDA_CHECK(cudaStreamSynchronize(s));
+          std::vector<int32_t> perm(nsm_roots), gst;
+          for (int i = 0; i < nsm_roots; ++i) perm[i] = i;
+          if (pack) {
+            std::sort(perm.begin(), perm.end(), [&](int x, int y) { return h_sa[x] > h_sa[y] || (h_sa[x] == h_sa[y] && x < y); });
+            std::vector<int32_t> order;
+            order.reserve(nsm_roots);
+            int lo_i = 0, hi_i = nsm_roots - 1;
+            while (lo_i <= hi_i) {
+              gst.push_back((int32_t)order.size());
+              int sum = h_sa[perm[lo_i]], cnt = 1;
+              order.push_back(perm[lo_i++]);
+              while (lo_i <= hi_i && cnt < MAXR && sum + h_sa[perm[hi_i]] <= A) {
+                sum += h_sa[perm[hi_i]];
+                ++cnt;
+                order.push_back(perm[hi_i--]);
+              }
+            }
+            perm.swap(order);
+          } else {
+            for (int i = 0; i < nsm_roots; ++i) gst.push_back(i);
+          }
+          const int ngroups = (int)gst.size();
+          gst.push_back(nsm_roots);
+          h2d(d_perm.p, perm.data(), nsm_roots, s);
+          h2d(d_gst.p, gst.data(), ngroups + 1, s);
           SubArgs ga;
           ga.sq = sq.p;
+          ga.gperm = d_perm.p;
+          ga.gstart = d_gst.p;
           ga.Es = Es.p;
           ga.yq = yq.p;
           ga.y = y;
@@ -2954,7 +3036,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
           }
           {
             KScope ks_("k_subtree", s, 0.0);
-            k_subtree<<<(unsigned)ls.nsmall, SUB_NT, subtree_smem(A, p), s>>>(ga);
+            k_subtree<<<(unsigned)ngroups, SUB_NT, subtree_smem(A, p), s>>>(ga);
           }
           if (ga.visits) {  // SURVEY 8(d) split-search bytes of the subtree nodes: 20 B per entry visit
             unsigned long long hv = 0;

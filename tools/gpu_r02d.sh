@@ -1,0 +1,11 @@
+# round-2 call d: packed subtree roots -- parity first, then bench and subtree counters
+D=gpurun_out/r02d; mkdir -p $D
+python -c "import __graft_entry__ as g; g.build()" 2>&1 | tail -2
+timeout 1800 python -m pytest tests/test_gpu_parity.py -m gpu -q -rf -x > $D/pytest_parity.log 2>&1; echo "pytest rc=$?" >> $D/pytest_parity.log
+tail -n 4 $D/pytest_parity.log
+if grep -q "pytest rc=0" $D/pytest_parity.log; then
+  timeout 900 python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-e2e > $D/bench.log 2>&1
+  grep "^{" $D/bench.log | python -c "import json,sys; d=json.loads(sys.stdin.read()); print(d['value'], d['phases_ms'], {k: round(v['ms_per_step'],1) for k,v in list(d['kernels'].items())[:6]})"
+  BF_SUBTREE_STATS=1 timeout 600 python bench.py --ntree 200 --m-query 0 --steps 1 --warmup 1 --no-e2e --no-cpu-baseline --no-profile > $D/subtree_stats.txt 2>&1
+  grep "\[subtree" $D/subtree_stats.txt | tail -4
+fi
