@@ -231,6 +231,114 @@ __global__ void __launch_bounds__(PT8, 6) k_predict8(const uint2* __restrict__ n
   if (last && yhat) yhat[rr] = acc * inv_t;
 }
 
+// k_predict8 with the tree block's root words and root nodes staged in shared memory (a slot restarts from
+// shared memory, not with two dependent global loads) and the float-tie fp64 fallback out of line (no
+// predicated global loads on the common path).  Used for blocks of <= RT8 trees (BF_PREDICT_V=1 restores
+// k_predict8).
+constexpr int RT8 = 64;
+__device__ __noinline__ uint32_t tie_right_fp64(const double* xg, int64_t ldq, uint32_t f, const Node16* n16,
+                                                uint32_t gid) {
+  return !(__ldg(xg + (int64_t)f * ldq) <= __ldg(&n16[gid].v));
+}
+
+template <bool PROF>
+__global__ void __launch_bounds__(PT8, 6) k_predict8s(const uint2* __restrict__ nodes8, const Node16* __restrict__ nodes16,
+                                                      const uint32_t* __restrict__ roots, int32_t t_begin, int32_t t_end,
+                                                      int first, int last, const double* __restrict__ Xq, int64_t ldq,
+                                                      int64_t m, int p, double* yhat_sum, double* yhat, double inv_t,
+                                                      unsigned long long* visits) {
+  extern __shared__ float sxf[];  // PT8 x (p|1), row-major
+  __shared__ uint32_t s_rw[RT8];
+  __shared__ uint2 s_rn[RT8];
+  const int stride = p | 1;
+  const int64_t r0 = (int64_t)blockIdx.x * PT8;
+  const int rows = (int)(m - r0 < PT8 ? m - r0 : PT8);
+  const int nt = t_end - t_begin;
+  if ((int)threadIdx.x < nt) {
+    const uint32_t rw = __ldg(roots + t_begin + threadIdx.x);
+    s_rw[threadIdx.x] = rw;
+    s_rn[threadIdx.x] = __ldg(nodes8 + (rw & ~ROOT_LEAF));
+  }
+  {  // stage the tile as floats: 8 column loads in flight per thread
+    const int r = threadIdx.x;
+    const bool ok = r < rows;
+    const double* src = Xq + r0 + (ok ? r : 0);
+    for (int f0 = 0; f0 < p; f0 += 8) {
+      double v[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) v[u] = (f0 + u < p) ? __ldcs(src + (int64_t)(f0 + u) * ldq) : 0.0;
+#pragma unroll
+      for (int u = 0; u < 8; ++u)
+        if (f0 + u < p && ok) sxf[r * stride + f0 + u] = __double2float_rn(v[u]);
+    }
+  }
+  __syncthreads();
+  if ((int)threadIdx.x >= rows) return;
+  const float* xs = sxf + threadIdx.x * stride;
+  const int64_t rr = r0 + threadIdx.x;
+  const double* xg = Xq + rr;
+  double acc = first ? 0.0 : yhat_sum[rr];
+  uint32_t nv = 0, nfb = 0;
+  uint32_t gid[S8];
+  uint2 nd[S8];
+  int tnext = 0;
+  int nact = 0;
+  auto start = [&](int u) {
+    gid[u] = ~0u;
+    while (tnext < nt) {
+      const uint32_t rw = s_rw[tnext];
+      const uint2 rn = s_rn[tnext];
+      ++tnext;
+      if (PROF) ++nv;
+      if (rw & ROOT_LEAF) {
+        acc += leaf8(rn);
+        continue;
+      }
+      gid[u] = rw;
+      nd[u] = rn;
+      ++nact;
+      break;
+    }
+  };
+#pragma unroll
+  for (int u = 0; u < S8; ++u) start(u);
+  while (nact > 0) {
+#pragma unroll
+    for (int u = 0; u < S8; ++u) {
+      if (gid[u] == ~0u) continue;
+      const uint2 w = nd[u];
+      const uint32_t f = (w.y >> N8_REL_BITS) & ((1u << N8_FEAT_BITS) - 1u);
+      const float xf = xs[f], tf = __uint_as_float(w.x);
+      uint32_t right = xf > tf;
+      if (__builtin_expect(xf == tf || xf != xf, 0)) {  // float tie (or NaN): decide in fp64 (S5)
+        right = tie_right_fp64(xg, ldq, f, nodes16, gid[u]);
+        if (PROF) ++nfb;
+      }
+      const uint32_t c = gid[u] + (w.y & ((1u << N8_REL_BITS) - 1u)) + right;
+      const uint2 ch = __ldg(nodes8 + c);
+      if (PROF) ++nv;
+      if ((w.y >> (31 - right)) & 1u) {
+        acc += leaf8(ch);
+        --nact;
+        start(u);
+      } else {
+        gid[u] = c;
+        nd[u] = ch;
+      }
+    }
+  }
+  if (PROF) {
+    const unsigned act = __activemask();
+    const uint32_t wv = __reduce_add_sync(act, nv), wf = __reduce_add_sync(act, nfb);
+    if ((threadIdx.x & 31) == __ffs(act) - 1) {
+      atomicAdd(visits, (unsigned long long)wv);
+      atomicAdd(visits + 1, (unsigned long long)wf);
+    }
+  }
+  yhat_sum[rr] = acc;
+  if (last && yhat) yhat[rr] = acc * inv_t;
+}
+
 __global__ void __launch_bounds__(PT) k_predict_gmem(const Node16* __restrict__ nodes, const int64_t* __restrict__ off,
                                                      int32_t ntrees, const double* __restrict__ Xq, int64_t ldq,
                                                      int64_t m, double* yhat_sum, double* yhat, double inv_t,
@@ -497,7 +605,10 @@ void predict_impl(const bf_forest* f, const double* Xq_in, int64_t ldq, int64_t 
   const uint2* n8 = (force16 && force16[0] == '1') ? nullptr : nodes8_get(const_cast<bf_forest*>(f), s);
   const size_t smem8 = sizeof(float) * (size_t)PT8 * (size_t)(p | 1);
   static int smax8 = 0;
-  if (!smax8) smax8 = std::min(dyn_smem_limit(k_predict8<true>), dyn_smem_limit(k_predict8<false>));
+  if (!smax8)
+    smax8 = std::min(std::min(dyn_smem_limit(k_predict8<true>), dyn_smem_limit(k_predict8<false>)),
+                     std::min(dyn_smem_limit(k_predict8s<true>), dyn_smem_limit(k_predict8s<false>)));
+  static const int pv = getenv("BF_PREDICT_V") ? atoi(getenv("BF_PREDICT_V")) : 2;
   if (n8 && smem8 <= (size_t)smax8) {
     // tree blocks of <= 32 MB of Node8 (L2-resident while every row walks them)
     double* ysum = ys_in ? (double*)ys.dptr : nullptr;
@@ -510,7 +621,12 @@ void predict_impl(const bf_forest* f, const double* Xq_in, int64_t ldq, int64_t 
     for (int32_t t0 = 0; t0 < nt;) {
       int32_t t1 = t0 + 1;
       while (t1 < nt && (f->tree_off[t1 + 1] - f->tree_off[t0]) * (int64_t)sizeof(uint2) <= block_bytes) ++t1;
-      {
+      if (t1 - t0 <= RT8 && pv != 1) {
+        KScope ks_("k_predict8", s, 0.0);
+        (vis.p ? k_predict8s<true> : k_predict8s<false>)<<<(unsigned)ceil_div(m, PT8), PT8, smem8, s>>>(
+            n8, f->d_nodes, f->d_roots8, t0, t1, t0 == 0, t1 >= nt, (const double*)Xs.dptr, ldq, m, p, ysum,
+            yh_in ? (double*)yh.dptr : nullptr, inv_t, vis.p);
+      } else {
         KScope ks_("k_predict8", s, 0.0);
         (vis.p ? k_predict8<true> : k_predict8<false>)<<<(unsigned)ceil_div(m, PT8), PT8, smem8, s>>>(
             n8, f->d_nodes, f->d_roots8, t0, t1, t0 == 0, t1 >= nt, (const double*)Xs.dptr, ldq, m, p, ysum,

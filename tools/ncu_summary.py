@@ -25,7 +25,10 @@ KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "smsp__issue_active.avg.pct_of_peak_sustained_active", "lts__t_sector_hit_rate.pct",
         "l1tex__data_bank_conflicts_pipe_lsu_mem_shared.sum", "launch__registers_per_thread", "launch__grid_size",
         "launch__block_size", "launch__shared_mem_per_block_dynamic", "launch__occupancy_limit_registers",
-        "launch__occupancy_limit_shared_mem", "launch__occupancy_limit_warps"]
+        "launch__occupancy_limit_shared_mem", "launch__occupancy_limit_warps",
+        "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum",
+        "l1tex__data_pipe_lsu_wavefronts_mem_shared.avg.pct_of_peak_sustained_elapsed",
+        "lts__t_bytes.sum"]
 
 
 def _num(v: str, unit: str) -> float:
