@@ -1007,266 +1007,6 @@ __global__ void __launch_bounds__(SNT, 4) k_split_scan_tree(TScanArgs g) {
   }
 }
 
-// a7 split search, warp-specialised (default; BF_SCAN_WS=0 selects k_split_scan_tree above).  Same items,
-// units, arithmetic and per-unit reduction as k_split_scan_tree, but the y_q gathers leave the scan's critical
-// path: 4 producer warps stage every unit -- the entries by one TMA bulk copy into a ring of WS_NS stages, then
-// w * y_q[row] of each entry gathered (9 loads in flight per thread) into the stage's int64 buffer -- while the
-// 4 consumer warps scan the previous stage from shared memory only.  Hand-offs: per stage a TMA mbarrier
-// (complete_tx), a "full" mbarrier (one arrive per producer warp) and an "empty" mbarrier (one arrive per
-// consumer warp once its registers hold the unit).  Consumer barriers are named (bar 1, 128 threads).
-constexpr int WS_NS = 3;
-constexpr int WS_CT = 128, WS_PT = 128, WS_NT = WS_CT + WS_PT;
-
-__device__ __forceinline__ void mbar_init_n(uint64_t* bar, int n) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(n) : "memory");
-}
-__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
-  asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
-}
-__device__ __forceinline__ void mbar_wait_acq(uint64_t* bar, uint32_t phase) {
-  asm volatile(
-      "{\n .reg .pred p;\n WAITA_%=:\n mbarrier.try_wait.parity.acquire.cta.shared::cta.b64 p, [%0], %1;\n @!p bra WAITA_%=;\n}\n" ::"r"(
-          smem_u32(bar)),
-      "r"(phase)
-      : "memory");
-}
-__device__ __forceinline__ void cons_sync() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
-
-__global__ void __launch_bounds__(WS_NT, 2) k_split_scan_ws(TScanArgs g) {
-  extern __shared__ __align__(16) unsigned char dsm[];
-  uint64_t* ent = (uint64_t*)dsm;                              // WS_NS x (TUNIT + 4) entries
-  int64_t* wyb = (int64_t*)(ent + (size_t)WS_NS * (TUNIT + 4));  // WS_NS x TUNIT
-  constexpr int NW = WS_CT / 32;
-  __shared__ uint64_t bar_tma[WS_NS], bar_full[WS_NS], bar_empty[WS_NS];
-  __shared__ int32_t smc[NW];
-  __shared__ int64_t sms[NW];
-  __shared__ double smL[NW];
-  __shared__ WBest swb[NW];
-  const int tid = threadIdx.x, lane = tid & 31;
-  const TreeSched ts = tree_sched(g.B);
-  if (tid == 0) {
-    for (int k = 0; k < WS_NS; ++k) {
-      mbar_init_n(&bar_tma[k], 1);
-      mbar_init_n(&bar_full[k], WS_PT / 32);
-      mbar_init_n(&bar_empty[k], WS_CT / 32);
-    }
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  __syncthreads();
-  if (tid >= WS_CT) {
-    // ================= producers
-    const int pt = tid - WS_CT;
-    uint32_t k = 0;
-    for (int b = ts.b0; b < g.B; b += ts.bstep) {
-      const int i_hi = g.thi[b] * g.mtry;
-      for (int item = g.tlo[b] * g.mtry + ts.c; item < i_hi; item += ts.C) {
-        const LNode nd = g.nodes[item / g.mtry];
-        const int f = g.feat[item];
-        const int nun = (nd.a + TUNIT - 1) / TUNIT;
-        for (int unit = 0; unit < nun; ++unit, ++k) {
-          const int st = (int)(k % WS_NS);
-          const uint32_t ph = (k / WS_NS) & 1u;
-          mbar_wait_acq(&bar_empty[st], ph ^ 1u);  // the consumers have taken the stage's previous unit
-          const int u0 = unit * TUNIT;
-          const int cload = min(TUNIT + 1, nd.a - u0), cnt = min(TUNIT, nd.a - u0);
-          const uint64_t* src = g.E + nd.base + (int64_t)f * nd.a + u0;
-          uint64_t* eb = ent + (size_t)st * (TUNIT + 4);
-          if (pt == 0) stage_entries(eb, src, cload, &bar_tma[st]);
-          const int off = (int)(((uintptr_t)src & 15) >> 3);
-          mbar_wait(&bar_tma[st], ph);
-          const uint64_t* buf = eb + off;
-          int64_t* wb = wyb + (size_t)st * TUNIT;
-          const int jl = pt * TSV;
-          int64_t yv[TSV];
-          int32_t wq[TSV];
-#pragma unroll
-          for (int q = 0; q < TSV; ++q) {
-            const bool in = jl + q < cnt;
-            const uint64_t e = in ? buf[jl + q] : 0ull;
-            wq[q] = in ? e_w(e) : 0;
-            yv[q] = ldg_s64_nc(g.yq + (in ? e_row(e) : 0u));
-          }
-#pragma unroll
-          for (int q = 0; q < TSV; ++q)
-            if (jl + q < cnt) wb[jl + q] = yv[q] * wq[q];
-          __syncwarp();
-          if (lane == 0) mbar_arrive(&bar_full[st]);
-        }
-      }
-    }
-    return;
-  }
-  // ================= consumers
-  const int wid = tid >> 5;
-  uint32_t k = 0;
-  for (int b = ts.b0; b < g.B; b += ts.bstep) {
-    const int i_hi = g.thi[b] * g.mtry;
-    for (int item = g.tlo[b] * g.mtry + ts.c; item < i_hi; item += ts.C) {
-      const LNode nd = g.nodes[item / g.mtry];
-      const int f = g.feat[item];
-      const int a = nd.a, nun = (a + TUNIT - 1) / TUNIT;
-      const int64_t nk = nd.n, Sk = nd.S;
-      const double nkd = (double)nk, Skd = (double)Sk;
-      int32_t carry_n = 0;
-      int64_t carry_S = 0;
-      WBest ib;
-      ib.g = -1.0;
-      ib.rank = 0xffffffffu;
-      ib.rb = 0;
-      ib.pos = -1;
-      ib.nl = 0;
-      ib.Sl = 0;
-      for (int unit = 0; unit < nun; ++unit, ++k) {
-        const int st = (int)(k % WS_NS);
-        const uint32_t ph = (k / WS_NS) & 1u;
-        const int u0 = unit * TUNIT, cnt = min(TUNIT, a - u0);
-        const uint64_t* src = g.E + nd.base + (int64_t)f * a + u0;
-        const int off = (int)(((uintptr_t)src & 15) >> 3);
-        mbar_wait_acq(&bar_full[st], ph);
-        const uint64_t* buf = ent + (size_t)st * (TUNIT + 4) + off;
-        const int64_t* wb = wyb + (size_t)st * TUNIT;
-        const int jl = tid * TSV;
-        uint32_t rk[TSV + 1];
-        int32_t wq[TSV];
-        int64_t wy[TSV];
-#pragma unroll
-        for (int q = 0; q < TSV; ++q) {
-          const bool in = jl + q < cnt;
-          const uint64_t e = buf[min(jl + q, cnt)];  // buf[cnt]: the next unit's first entry (if any)
-          rk[q] = e_rank(e);
-          wq[q] = in ? e_w(e) : 0;
-          wy[q] = in ? wb[jl + q] : 0;
-        }
-        rk[TSV] = e_rank(buf[min(jl + TSV, cnt)]);
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&bar_empty[st]);  // the stage's data is in registers: producers may refill it
-        int32_t tc = 0;
-        int64_t tsum = 0;
-#pragma unroll
-        for (int q = 0; q < TSV; ++q) {
-          tc += wq[q];
-          tsum += wy[q];
-        }
-        int32_t ic = tc;
-        int64_t is = tsum;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-          const int32_t uc = __shfl_up_sync(0xffffffffu, ic, o);
-          const int64_t us = __shfl_up_sync(0xffffffffu, is, o);
-          if (lane >= o) {
-            ic += uc;
-            is += us;
-          }
-        }
-        if (lane == 31) {
-          smc[wid] = ic;
-          sms[wid] = is;
-        }
-        cons_sync();
-        int32_t prc0 = carry_n + ic - tc, totc = 0;
-        int64_t prs0 = carry_S + is - tsum, tots = 0;
-#pragma unroll
-        for (int kk = 0; kk < NW; ++kk) {
-          const int32_t c = smc[kk];
-          const int64_t v = sms[kk];
-          if (kk < wid) {
-            prc0 += c;
-            prs0 += v;
-          }
-          totc += c;
-          tots += v;
-        }
-        float gUf[TSV];
-        double mL = ib.g;
-        {
-          int32_t prc = prc0;
-          int64_t prs = prs0;
-#pragma unroll
-          for (int q = 0; q < TSV; ++q) {
-            gUf[q] = -1.0f;
-            const int j = jl + q;
-            if (j < cnt) {
-              prc += wq[q];
-              prs += wy[q];
-              if (u0 + j + 1 < a && rk[q] != rk[q + 1]) {
-                double gL, gU;
-                key_bounds(nkd, Skd, nk, prc, prs, gL, gU);
-                mL = fmax(mL, gL);
-                gUf[q] = __double2float_ru(gU);
-              }
-            }
-          }
-        }
-        {
-          const uint64_t kb = gkey(mL);
-          const uint32_t hi = __reduce_max_sync(0xffffffffu, (uint32_t)(kb >> 32));
-          const uint32_t lo = __reduce_max_sync(0xffffffffu, ((uint32_t)(kb >> 32) == hi) ? (uint32_t)kb : 0u);
-          if (lane == 0) smL[wid] = (hi | lo) ? __longlong_as_double((long long)((((uint64_t)hi << 32) | lo) - 1ull)) : -1.0;
-        }
-        cons_sync();
-        double M = -1.0;
-#pragma unroll
-        for (int kk = 0; kk < NW; ++kk) M = fmax(M, smL[kk]);
-        WBest tb;
-        tb.g = -1.0;
-        tb.rank = 0xffffffffu;
-        tb.rb = 0;
-        tb.pos = -1;
-        tb.nl = 0;
-        tb.Sl = 0;
-        {
-          int32_t prc = prc0;
-          int64_t prs = prs0;
-#pragma unroll
-          for (int q = 0; q < TSV; ++q) {
-            const int j = jl + q;
-            if (j < cnt) {
-              prc += wq[q];
-              prs += wy[q];
-              if ((double)gUf[q] >= M && gUf[q] >= 0.0f) {
-                const double gk = split_key_call(nk, Sk, prc, prs);
-                const uint32_t ra = rk[q];
-                if (rec_better(gk, ra, tb.g, tb.rank)) {
-                  tb.g = gk;
-                  tb.rank = ra;
-                  tb.rb = rk[q + 1];
-                  tb.pos = u0 + j;
-                  tb.nl = prc;
-                  tb.Sl = prs;
-                }
-              }
-            }
-          }
-        }
-        {
-          const int wl = warp_argmax_key(gkey(tb.g), tb.rank);
-          if (wl >= 0 && lane == wl) swb[wid] = tb;
-          if (wl < 0 && lane == 0) swb[wid].g = -1.0;
-        }
-        cons_sync();
-#pragma unroll
-        for (int kk = 0; kk < NW; ++kk) {
-          const double kg = swb[kk].g;
-          if (kg >= 0.0 && (kg > ib.g || (kg == ib.g && swb[kk].rank < ib.rank))) ib = swb[kk];
-        }
-        carry_n += totc;
-        carry_S += tots;
-        cons_sync();  // smc / sms / smL / swb are rewritten by the next unit
-      }
-      if (tid == 0) {
-        Rec R;
-        R.g = ib.g;
-        R.rank_a = ib.rank;
-        R.rank_b = ib.rb;
-        R.pos = ib.pos;
-        R.nl = ib.nl;
-        R.Sl = ib.Sl;
-        g.rec[item] = R;
-      }
-    }
-  }
-}
-
 struct TPartArgs {
   const LNode* nodes;
   const Split* split;
@@ -3015,12 +2755,6 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_ts, k_split_scan_tree, SNT, tscan_smem);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_tp, k_partition_tree, TPNT, tpart_smem);
     const unsigned grid_tscan = (unsigned)std::max(1, occ_ts * nsm), grid_tpart = (unsigned)std::max(1, occ_tp * nsm);
-    static const bool scan_ws = !(getenv("BF_SCAN_WS") && getenv("BF_SCAN_WS")[0] == '0');
-    const size_t ws_smem = sizeof(uint64_t) * (size_t)WS_NS * (TUNIT + 4) + sizeof(int64_t) * (size_t)WS_NS * TUNIT;
-    BF_CUDA_CHECK(cudaFuncSetAttribute(k_split_scan_ws, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ws_smem));
-    int occ_ws = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_ws, k_split_scan_ws, WS_NT, ws_smem);
-    const unsigned grid_ws = (unsigned)std::max(1, occ_ws * nsm);
     DBuf<uint64_t> E0, E1, Es;
     std::vector<int32_t> h_sa;  // distinct rows of the batch's small roots (subtree packing)
     size_t E_cap = 0;
@@ -3147,13 +2881,8 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
         }
         {  // ---- a7 split search: tree-affine CTAs own whole (node, drawn feature) items
           TScanArgs ga{nc, feat.p, mtry, Bc, Ec, yq.p, tlo.p, thi.p, rec.p};
-          if (scan_ws) {
-            KScope ks_("k_split_scan_ws", s, 0.0);
-            k_split_scan_ws<<<grid_ws, WS_NT, ws_smem, s>>>(ga);
-          } else {
-            KScope ks_("k_split_scan_tree", s, 0.0);
-            k_split_scan_tree<<<grid_tscan, SNT, tscan_smem, s>>>(ga);
-          }
+          KScope ks_("k_split_scan_tree", s, 0.0);
+          k_split_scan_tree<<<grid_tscan, SNT, tscan_smem, s>>>(ga);
         }
         if (lvl_timing) cudaEventRecord(lev[1], s);
         {
@@ -3204,7 +2933,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
         BF_CUDA_CHECK(cudaStreamSynchronize(s));
         {  // algorithmic bytes
           const double sa = (double)hs.h->split_a;
-          prof_add_bytes(scan_ws ? "k_split_scan_ws" : "k_split_scan_tree", (double)cur_a * mtry * 16.0);
+          prof_add_bytes("k_split_scan_tree", (double)cur_a * mtry * 16.0);
           prof_add_bytes("k_dest_bits", sa * 17.0);
           prof_add_bytes("k_partition_tree", sa * p * 17.0);
         }
@@ -3246,7 +2975,19 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
           std::vector<int32_t> perm(nsm_roots), gst;
           for (int i = 0; i < nsm_roots; ++i) perm[i] = i;
           if (pack) {
-            std::sort(perm.begin(), perm.end(), [&](int x, int y) { return h_sa[x] > h_sa[y] || (h_sa[x] == h_sa[y] && x < y); });
+            // descending by distinct rows, ties by index: a counting sort over a in [0, A] (O(roots + A) on
+            // the host; a comparison sort of ~80K roots per batch cost ~7 ms)
+            {
+              std::vector<int32_t> cnt_a((size_t)A + 2, 0);
+              for (int i = 0; i < nsm_roots; ++i) ++cnt_a[(size_t)(A - std::min(h_sa[i], A))];
+              int run = 0;
+              for (size_t v = 0; v < cnt_a.size(); ++v) {
+                const int c = cnt_a[v];
+                cnt_a[v] = run;
+                run += c;
+              }
+              for (int i = 0; i < nsm_roots; ++i) perm[cnt_a[(size_t)(A - std::min(h_sa[i], A))]++] = i;
+            }
             std::vector<int32_t> order;
             order.reserve(nsm_roots);
             int lo_i = 0, hi_i = nsm_roots - 1;
