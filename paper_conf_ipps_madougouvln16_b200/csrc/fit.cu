@@ -1755,7 +1755,10 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         }
         const int32_t cw0 = warp_incl_scan(rw, lane) - rw;
         const int64_t cs0 = warp_incl_scan(rsum, lane) - rsum;
-        double mL = -1.0, mU = -1.0;
+        double mL = -1.0, mU = -1.0, u2 = -1.0;  // as in the tiny path: largest / second largest upper bound
+        int bi = -1;
+        int32_t bcw = 0;
+        int64_t bcs = 0;
         {
           int32_t cw = cw0;
           int64_t cs = cs0;
@@ -1768,7 +1771,15 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
               double gL, gU;
               key_bounds(nkd, Skd, nk, cw, cs, gL, gU);
               mL = fmax(mL, gL);
-              mU = fmax(mU, gU);
+              if (gU > mU) {
+                u2 = mU;
+                mU = gU;
+                bi = i;
+                bcw = cw;
+                bcs = cs;
+              } else {
+                u2 = fmax(u2, gU);
+              }
             }
           }
         }
@@ -1779,7 +1790,19 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
           const uint32_t lo = __reduce_max_sync(0xffffffffu, ((uint32_t)(kb >> 32) == hi) ? (uint32_t)kb : 0u);
           M = (hi | lo) ? __longlong_as_double((long long)((((uint64_t)hi << 32) | lo) - 1ull)) : -1.0;
         }
-        if (mU >= M && mU >= 0.0) {
+        if (mU >= M && mU >= 0.0 && u2 < M) {  // a single candidate item on this lane
+          const uint32_t e = seg[bi], en = seg[bi + 1];
+          const double gk = split_key(nk, Sk, bcw, bcs);
+          if (rec_better(gk, e >> 16, lg, lrk)) {
+            lg = gk;
+            lrk = e >> 16;
+            lra = e & 0xffffu;
+            lrb = en & 0xffffu;
+            lpos = bi;
+            lnl = bcw;
+            lSl = bcs;
+          }
+        } else if (mU >= M && mU >= 0.0) {
           int32_t cw = cw0;
           int64_t cs = cs0;
           for (int i = i0; i < i1; ++i) {
@@ -2000,14 +2023,42 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
     }
   }
 
-  // ================= tiny nodes: row index inside each tiny root, then the work queue
+  // ================= tiny nodes
+  // Renumber the local rows by their position in feature 0's list row: a tiny root's rows then carry the ids
+  // [rlo, rlo + ra) in that order, so a row's index inside its tiny root is (id - rlo) -- no lookup table on
+  // the tiny path.  The payload arrays and every list entry's row field are permuted accordingly (the records
+  // written so far too); ranks are unchanged.
   tclk[2] = clock64();
   {
-    const int nroots = a_get<int>(s_alloc);
-    for (int qi = wid; qi < nroots; qi += SUB_NW) {
-      const TNode r = tq_read(tq, qi);  // pushed before the barrier above
-      for (int k = lane; k < r.ra; k += 32) rmap[list[r.rlo + k] & 0xffffu] = (uint8_t)k;
+    uint16_t* pos = (uint16_t*)temp_all;                  // old id -> new id
+    int64_t* scr = (int64_t*)(temp_all + ((a0 + 7) & ~7));  // one payload array at a time
+    for (int j = tid; j < a0; j += SUB_NT) pos[list[j] & 0xffffu] = (uint16_t)j;
+    __syncthreads();
+    for (int j = tid; j < a0; j += SUB_NT) scr[pos[j]] = wy[j];
+    __syncthreads();
+    for (int j = tid; j < a0; j += SUB_NT) wy[j] = scr[j];
+    __syncthreads();
+    for (int j = tid; j < a0; j += SUB_NT) scr[pos[j]] = __double_as_longlong(wyd[j]);
+    __syncthreads();
+    for (int j = tid; j < a0; j += SUB_NT) wyd[j] = __longlong_as_double(scr[j]);
+    __syncthreads();
+    for (int j = tid; j < a0; j += SUB_NT) scr[pos[j]] = ((int64_t)wl[j] << 32) | grow[j];
+    __syncthreads();
+    for (int j = tid; j < a0; j += SUB_NT) {
+      const int64_t v = scr[j];
+      wl[j] = (int32_t)(v >> 32);
+      grow[j] = (uint32_t)v;
     }
+    for (int k = tid; k < p * a0; k += SUB_NT) {
+      const uint32_t e = list[k];
+      list[k] = (e & 0xffff0000u) | pos[e & 0xffffu];
+    }
+    for (int r = 0; r < nr; ++r)
+      for (int l = 2 * s_off[r] + tid; l < s_nloc[r]; l += SUB_NT)
+        if (recs[l].feature >= 0) {
+          recs[l].ra = pos[recs[l].ra];
+          recs[l].rb = pos[recs[l].rb];
+        }
   }
   __syncthreads();
   for (;;) {
@@ -2080,7 +2131,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
               ev[2 * u + 1] = (u < nu && lane + 32 < ra) ? seg[lane + 32] : 0u;
             }
 #pragma unroll
-            for (int k = 0; k < 2 * TGRP; ++k) ri[k] = rmap[ev[k] & 0xffffu];
+            for (int k = 0; k < 2 * TGRP; ++k) ri[k] = (uint8_t)((ev[k] & 0xffffu) - (uint32_t)rlo);
 #pragma unroll
             for (int u = 0; u < TGRP; ++u) {
               const bool v0 = u < nu && ((nd.mask >> ri[2 * u]) & 1ull);
@@ -2096,7 +2147,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
               ev[u] = (u < nu && lane < ra) ? seg[lane] : 0u;
             }
 #pragma unroll
-            for (int k = 0; k < TGRP; ++k) ri[k] = rmap[ev[k] & 0xffffu];
+            for (int k = 0; k < TGRP; ++k) ri[k] = (uint8_t)((ev[k] & 0xffffu) - (uint32_t)rlo);
 #pragma unroll
             for (int u = 0; u < TGRP; ++u) {
               const bool v0 = u < nu && lane < ra && ((nd.mask >> ri[u]) & 1ull);
@@ -2158,7 +2209,12 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
           cs0 = 0;
         }
         const long long gq2 = g.stats ? clock64() : 0;
-        double mL = lg, mU = -1.0;
+        // the lane's largest upper bound mU with its item (bi, prefix bcw / bcs) and the second largest u2: when
+        // u2 < M only item bi can reach the exact-key pass, which then evaluates it directly
+        double mL = lg, mU = -1.0, u2 = -1.0;
+        int bi = -1;
+        int32_t bcw = 0;
+        int64_t bcs = 0;
         {
           int jj = jj0;
           int32_t cw = cw0;
@@ -2176,7 +2232,15 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
               double gL, gU;
               key_bounds(nkd, Skd, nk, cw, cs, gL, gU);
               mL = fmax(mL, gL);
-              mU = fmax(mU, gU);
+              if (gU > mU) {
+                u2 = mU;
+                mU = gU;
+                bi = i;
+                bcw = cw;
+                bcs = cs;
+              } else {
+                u2 = fmax(u2, gU);
+              }
             }
             if (++jj == an) jj = 0;
           }
@@ -2190,7 +2254,19 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
           M = (hi | lo) ? __longlong_as_double((long long)((((uint64_t)hi << 32) | lo) - 1ull)) : -1.0;
         }
         const long long gq4 = g.stats ? clock64() : 0;
-        if (mU >= M && mU >= 0.0) {
+        if (mU >= M && mU >= 0.0 && u2 < M) {  // a single candidate item on this lane
+          const uint32_t e = stg[bi], en = stg[bi + 1];
+          const double gk = split_key(nk, Sk, bcw, bcs);
+          const uint32_t tie = ((uint32_t)feats[s0 + bi / an] << 16) | (e >> 16);
+          if (gk > lg || (gk == lg && tie < ltie)) {
+            lg = gk;
+            ltie = tie;
+            lnl = bcw;
+            lSl = bcs;
+            lra = e & 0xffffu;
+            lrb = en & 0xffffu;
+          }
+        } else if (mU >= M && mU >= 0.0) {
           int jj = jj0, sl = slot0;
           int32_t cw = cw0;
           int64_t cs = cs0;
@@ -2261,7 +2337,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
           const int k = lane + 32 * hh;
           const uint32_t e = k < ra ? seg[k] : 0u;
           const uint32_t lrow = e & 0xffffu;
-          const int ri = k < ra ? rmap[lrow] : 0;
+          const int ri = k < ra ? (int)lrow - rlo : 0;
           const bool valid = k < ra && ((nd.mask >> ri) & 1ull);
           const bool left = valid && (e >> 16) <= brk;
           const uint32_t lo = __reduce_or_sync(0xffffffffu, (left && ri < 32) ? (1u << ri) : 0u);
