@@ -2023,42 +2023,14 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
     }
   }
 
-  // ================= tiny nodes
-  // Renumber the local rows by their position in feature 0's list row: a tiny root's rows then carry the ids
-  // [rlo, rlo + ra) in that order, so a row's index inside its tiny root is (id - rlo) -- no lookup table on
-  // the tiny path.  The payload arrays and every list entry's row field are permuted accordingly (the records
-  // written so far too); ranks are unchanged.
+  // ================= tiny nodes: row index inside each tiny root, then the work queue
   tclk[2] = clock64();
   {
-    uint16_t* pos = (uint16_t*)temp_all;                  // old id -> new id
-    int64_t* scr = (int64_t*)(temp_all + ((a0 + 7) & ~7));  // one payload array at a time
-    for (int j = tid; j < a0; j += SUB_NT) pos[list[j] & 0xffffu] = (uint16_t)j;
-    __syncthreads();
-    for (int j = tid; j < a0; j += SUB_NT) scr[pos[j]] = wy[j];
-    __syncthreads();
-    for (int j = tid; j < a0; j += SUB_NT) wy[j] = scr[j];
-    __syncthreads();
-    for (int j = tid; j < a0; j += SUB_NT) scr[pos[j]] = __double_as_longlong(wyd[j]);
-    __syncthreads();
-    for (int j = tid; j < a0; j += SUB_NT) wyd[j] = __longlong_as_double(scr[j]);
-    __syncthreads();
-    for (int j = tid; j < a0; j += SUB_NT) scr[pos[j]] = ((int64_t)wl[j] << 32) | grow[j];
-    __syncthreads();
-    for (int j = tid; j < a0; j += SUB_NT) {
-      const int64_t v = scr[j];
-      wl[j] = (int32_t)(v >> 32);
-      grow[j] = (uint32_t)v;
+    const int nroots = a_get<int>(s_alloc);
+    for (int qi = wid; qi < nroots; qi += SUB_NW) {
+      const TNode r = tq_read(tq, qi);  // pushed before the barrier above
+      for (int k = lane; k < r.ra; k += 32) rmap[list[r.rlo + k] & 0xffffu] = (uint8_t)k;
     }
-    for (int k = tid; k < p * a0; k += SUB_NT) {
-      const uint32_t e = list[k];
-      list[k] = (e & 0xffff0000u) | pos[e & 0xffffu];
-    }
-    for (int r = 0; r < nr; ++r)
-      for (int l = 2 * s_off[r] + tid; l < s_nloc[r]; l += SUB_NT)
-        if (recs[l].feature >= 0) {
-          recs[l].ra = pos[recs[l].ra];
-          recs[l].rb = pos[recs[l].rb];
-        }
   }
   __syncthreads();
   for (;;) {
@@ -2131,7 +2103,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
               ev[2 * u + 1] = (u < nu && lane + 32 < ra) ? seg[lane + 32] : 0u;
             }
 #pragma unroll
-            for (int k = 0; k < 2 * TGRP; ++k) ri[k] = (uint8_t)((ev[k] & 0xffffu) - (uint32_t)rlo);
+            for (int k = 0; k < 2 * TGRP; ++k) ri[k] = rmap[ev[k] & 0xffffu];
 #pragma unroll
             for (int u = 0; u < TGRP; ++u) {
               const bool v0 = u < nu && ((nd.mask >> ri[2 * u]) & 1ull);
@@ -2147,7 +2119,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
               ev[u] = (u < nu && lane < ra) ? seg[lane] : 0u;
             }
 #pragma unroll
-            for (int k = 0; k < TGRP; ++k) ri[k] = (uint8_t)((ev[k] & 0xffffu) - (uint32_t)rlo);
+            for (int k = 0; k < TGRP; ++k) ri[k] = rmap[ev[k] & 0xffffu];
 #pragma unroll
             for (int u = 0; u < TGRP; ++u) {
               const bool v0 = u < nu && lane < ra && ((nd.mask >> ri[u]) & 1ull);
@@ -2337,7 +2309,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
           const int k = lane + 32 * hh;
           const uint32_t e = k < ra ? seg[k] : 0u;
           const uint32_t lrow = e & 0xffffu;
-          const int ri = k < ra ? (int)lrow - rlo : 0;
+          const int ri = k < ra ? rmap[lrow] : 0;
           const bool valid = k < ra && ((nd.mask >> ri) & 1ull);
           const bool left = valid && (e >> 16) <= brk;
           const uint32_t lo = __reduce_or_sync(0xffffffffu, (left && ri < 32) ? (1u << ri) : 0u);
