@@ -383,7 +383,7 @@ struct Imp8Args {
   unsigned long long* prof;  // profile mode: [0] node loads, [1] permuted re-walks (algorithmic bytes), else NULL
 };
 
-__global__ void __launch_bounds__(IPT, 6) k_importance8(Imp8Args g8) {
+__global__ void __launch_bounds__(IPT) k_importance8(Imp8Args g8) {
   const ImpArgs& g = g8.a;
   extern __shared__ double ism[];  // sacc[p] | float x tile IPT x (p|1)
   double* sacc = ism;
