@@ -435,8 +435,10 @@ def run_ours(args):
             evs.append(e)
         end.record(stream)
         barrier()
+    step_ms = []
     for e in evs:
         phase += [e[i].elapsed_time(e[i + 1]) for i in range(4)]
+        step_ms.append(e[0].elapsed_time(e[4]))
     launches = (bf.launch_count() - L0) // args.steps
     ms = start.elapsed_time(end) / args.steps
     msmax = torch.tensor([ms], dtype=torch.float64, device=dev)
@@ -540,6 +542,7 @@ def run_ours(args):
         "predict_node_visits_per_walk": (vis / (m * (t1 - t0))) if m and vis and t1 > t0 else None,
         "predict_fp64_fallbacks_per_visit": (fbk / vis) if vis else None,
         "phases_ms": {"fit": phase[0], "predict": phase[1], "importance": phase[2], "pca": phase[3]},
+        "step_ms": step_ms,
         "gpu_launches": int(launches),
         "roofline": roof,
         "profiled_step_ms": prof_ms,

@@ -965,29 +965,41 @@ __global__ void __launch_bounds__(SNT, 4) k_split_scan_tree(TScanArgs g) {
           }
         }
       }
-      // S3: per-warp winners; every thread merges them (unit order == position order)
+      // the warp's winner of the unit merges into the warp's running best (no block barrier per unit: every
+      // warp's best is an exact candidate key, so the block max of the lower bounds above still screens
+      // correctly); the warps' bests are merged once per item
       {
         const int wl = warp_argmax_key(gkey(tb.g), tb.rank);
-        if (wl >= 0 && lane == wl) swb[wid] = tb;
-        if (wl < 0 && lane == 0) swb[wid].g = -1.0;
-      }
-      __syncthreads();
-#pragma unroll
-      for (int k = 0; k < NW; ++k) {
-        const double kg = swb[k].g;
-        if (kg >= 0.0 && (kg > ib.g || (kg == ib.g && swb[k].rank < ib.rank))) ib = swb[k];
+        if (wl >= 0) {
+          WBest wb;
+          wb.g = __shfl_sync(0xffffffffu, tb.g, wl);
+          wb.rank = __shfl_sync(0xffffffffu, tb.rank, wl);
+          wb.rb = __shfl_sync(0xffffffffu, tb.rb, wl);
+          wb.pos = __shfl_sync(0xffffffffu, tb.pos, wl);
+          wb.nl = __shfl_sync(0xffffffffu, tb.nl, wl);
+          wb.Sl = __shfl_sync(0xffffffffu, tb.Sl, wl);
+          if (wb.g > ib.g || (wb.g == ib.g && wb.rank < ib.rank)) ib = wb;
+        }
       }
       carry_n += totc;
       carry_S += tots;
-      if (unit + 1 >= nun) {  // item done
+      if (unit + 1 >= nun) {  // item done: merge the warps' bests (position order == rank order)
+        if (lane == 0) swb[wid] = ib;
+        __syncthreads();
         if (tid == 0) {
+          WBest bb = swb[0];
+#pragma unroll
+          for (int k = 1; k < NW; ++k) {
+            const WBest& o = swb[k];
+            if (o.g >= 0.0 && (o.g > bb.g || (o.g == bb.g && o.rank < bb.rank))) bb = o;
+          }
           Rec R;
-          R.g = ib.g;
-          R.rank_a = ib.rank;
-          R.rank_b = ib.rb;
-          R.pos = ib.pos;
-          R.nl = ib.nl;
-          R.Sl = ib.Sl;
+          R.g = bb.g;
+          R.rank_a = bb.rank;
+          R.rank_b = bb.rb;
+          R.pos = bb.pos;
+          R.nl = bb.nl;
+          R.Sl = bb.Sl;
           g.rec[item] = R;
         }
         carry_n = 0;
@@ -1095,7 +1107,7 @@ __device__ __forceinline__ int32_t group_excl_scan(int32_t v, int32_t* sm, int32
   group_sync(grp);
   const int32_t pre = wid ? sm[wid - 1] : 0;
   total = sm[nw - 1];
-  group_sync(grp);
+  // no trailing barrier: the caller's next write of sm (the next unit's scan) follows its own group barriers
   return pre + inc - v;
 }
 
