@@ -2863,11 +2863,12 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
       size_t need = 0;
       for (int b = 0; b < Bc; ++b) need += (size_t)p * ha[b];
       need = std::max<size_t>(need, 1);
-      if (need > E_cap) {
-        E0.alloc(need + 16, s);
-        E1.alloc(need + 16, s);
-        Es.alloc(need + 16, s);
-        E_cap = need;
+      if (need > E_cap) {  // 3% headroom: later batches (sum of in-bag rows varies by ~0.1%) reuse the buffers
+        const size_t cap = need + need / 32 + 16;
+        E0.alloc(cap, s);
+        E1.alloc(cap, s);
+        Es.alloc(cap, s);
+        E_cap = cap - 16;
       }
       h2d(kind_d.p, hk.data(), Bc, s);
       h2d(lidx_d.p, hl.data(), Bc, s);

@@ -88,11 +88,14 @@ __global__ void k_ftab_fill(uint64_t seed, int32_t t0, int p, const int64_t* nou
 }
 
 __global__ void __launch_bounds__(512) k_perm_fill(uint64_t seed, int32_t t0, int p, int64_t n, const int64_t* nout,
-                                                   const uint32_t* gtab, int tstride, int32_t* perm) {
+                                                   const uint32_t* gtab, int tstride, int32_t* perm,
+                                                   const uint8_t* used) {
   extern __shared__ uint32_t ftab[];  // 6 x 2^h (h <= PH_MAX)
   const int b = blockIdx.z, m = blockIdx.y;
   const int64_t n_o = nout[b];
   if (n_o <= 0) return;
+  // a predictor no split of the tree uses is never re-walked (S7: its d_tm is 0): no permutation needed
+  if (!used[(int64_t)b * p + m]) return;
   const uint32_t t = (uint32_t)(t0 + b);
   const int h = feistel_h(n_o);
   const uint32_t mask = (uint32_t)((1ull << h) - 1ull);
@@ -104,31 +107,38 @@ __global__ void __launch_bounds__(512) k_perm_fill(uint64_t seed, int32_t t0, in
   }
   int32_t* out = perm + ((int64_t)b * p + m) * n;
   const int64_t step = (int64_t)gridDim.x * blockDim.x;
-  for (int64_t a = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; a < n_o; a += step) {
-    if (!tab) {
+  if (!tab) {
+    for (int64_t a = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; a < n_o; a += step)
       out[a] = (int32_t)feistel(seed, t, (uint32_t)m, n_o, a);
-      continue;
+    return;
+  }
+  // 2h <= 2 * PH_MAX bits: 32-bit arithmetic throughout (n_o < 2^31).  Cycle walking needs ~2.9 Feistel
+  // passes per value on average (the domain 2^2h is up to ~3x n_o) but the slowest lane of a warp needs ~9:
+  // each lane therefore walks its own sequence of positions one pass at a time and moves on to its next
+  // position as soon as the current one lands in [0, n_o), so no lane waits for the warp's slowest walk.
+  const uint32_t* f0 = ftab;
+  const uint32_t* f1 = f0 + (1u << h);
+  const uint32_t* f2 = f1 + (1u << h);
+  const uint32_t* f3 = f2 + (1u << h);
+  const uint32_t* f4 = f3 + (1u << h);
+  const uint32_t* f5 = f4 + (1u << h);
+  const uint32_t no = (uint32_t)n_o;
+  int64_t a = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  uint32_t v = (uint32_t)a;
+  while (a < n_o) {
+    uint32_t L = v >> h, R = v & mask;
+    L ^= f0[R];
+    R ^= f1[L];
+    L ^= f2[R];
+    R ^= f3[L];
+    L ^= f4[R];
+    R ^= f5[L];
+    v = (L << h) | R;  // six rounds (L, R) <- (R, L ^ F_r(R)) end with the halves back in place
+    if (v < no) {
+      out[a] = (int32_t)v;
+      a += step;
+      v = (uint32_t)a;
     }
-    // 2h <= 2 * PH_MAX bits: 32-bit arithmetic throughout (n_o < 2^31)
-    const uint32_t* f0 = ftab;
-    const uint32_t* f1 = f0 + (1u << h);
-    const uint32_t* f2 = f1 + (1u << h);
-    const uint32_t* f3 = f2 + (1u << h);
-    const uint32_t* f4 = f3 + (1u << h);
-    const uint32_t* f5 = f4 + (1u << h);
-    const uint32_t no = (uint32_t)n_o;
-    uint32_t v = (uint32_t)a;
-    do {
-      uint32_t L = v >> h, R = v & mask;
-      L ^= f0[R];
-      R ^= f1[L];
-      L ^= f2[R];
-      R ^= f3[L];
-      L ^= f4[R];
-      R ^= f5[L];
-      v = (L << h) | R;  // six rounds (L, R) <- (R, L ^ F_r(R)) end with the halves back in place
-    } while (v >= no);
-    out[a] = (int32_t)v;
   }
 }
 
@@ -200,20 +210,32 @@ __global__ void k_oob_scatter(const int32_t* w, int64_t n, int nchunk, const int
 
 // IncNodePurity slots: sum of drss of splits on m, per local tree.
 // (per-CTA shared-memory histogram over the predictors, one global atomic per (CTA, predictor))
-__global__ void k_npur(const Node16* nodes, const double* drss, const int64_t* off, int32_t i0, int p, double* npur) {
-  extern __shared__ double hp[];  // p
+// IncNodePurity slots of the batch's trees and the predictors each tree splits on (used[b * p + m] = 1;
+// zero-initialised by the caller).
+__global__ void k_npur(const Node16* nodes, const double* drss, const int64_t* off, int32_t i0, int p, double* npur,
+                       uint8_t* used) {
+  extern __shared__ double hp[];  // p doubles, then p flags
+  int* hu = reinterpret_cast<int*>(hp + p);
   const int b = blockIdx.y;
   const int32_t i = i0 + b;
-  for (int f = threadIdx.x; f < p; f += NT) hp[f] = 0.0;
+  for (int f = threadIdx.x; f < p; f += NT) {
+    hp[f] = 0.0;
+    hu[f] = 0;
+  }
   __syncthreads();
   const int64_t lo = off[i], hi = off[i + 1];
   for (int64_t k = lo + blockIdx.x * (int64_t)NT + threadIdx.x; k < hi; k += (int64_t)gridDim.x * NT) {
     const int f = nodes[k].feature;
-    if (f >= 0) atomicAdd(&hp[f], drss[k]);
+    if (f >= 0) {
+      atomicAdd(&hp[f], drss[k]);
+      atomicExch(&hu[f], 1);
+    }
   }
   __syncthreads();
-  for (int f = threadIdx.x; f < p; f += NT)
+  for (int f = threadIdx.x; f < p; f += NT) {
     if (hp[f] != 0.0) atomicAdd(&npur[(int64_t)i * p + f], hp[f]);
+    if (hu[f]) used[(int64_t)b * p + f] = 1;
+  }
 }
 
 struct ImpArgs {
@@ -690,6 +712,7 @@ void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, co
   DBuf<int32_t> w((size_t)B * n, s), cnt((size_t)B * nchunk, s);
   DBuf<uint32_t> O((size_t)B * n, s);
   DBuf<int32_t> perm((size_t)B * p * n, s);
+  DBuf<uint8_t> used((size_t)B * p, s);
   int hb_all = 64 - __builtin_clzll((unsigned long long)std::max<int64_t>(n - 1, 1));
   hb_all = std::max(hb_all, 2);
   hb_all += hb_all & 1;
@@ -727,7 +750,9 @@ void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, co
     }
     {
       KScope ks_("k_npur", s, 0.0);
-      k_npur<<<dim3(64, Bc), NT, sizeof(double) * (size_t)p, s>>>(f->d_nodes, f->d_drss, f->d_tree_off, i0, p, npur);
+      BF_CUDA_CHECK(cudaMemsetAsync(used.p, 0, (size_t)Bc * p, s));
+      k_npur<<<dim3(64, Bc), NT, (sizeof(double) + sizeof(int)) * (size_t)p, s>>>(f->d_nodes, f->d_drss, f->d_tree_off,
+                                                                                 i0, p, npur, used.p);
     }
     {
       static int pfs = 0;
@@ -746,7 +771,7 @@ void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, co
       KScope ks_("k_perm_fill", s, 0.0);
       k_perm_fill<<<dim3((unsigned)std::max<int64_t>(1, std::min<int64_t>(8, ceil_div(n, 65536))), p, Bc), 512,
                     sizeof(uint32_t) * 6 * ((size_t)1 << hmax), s>>>(f->info.seed, f->info.tree_begin + i0, p, n,
-                                                                     nout_t + i0, gtab.p, tstride, perm.p);
+                                                                     nout_t + i0, gtab.p, tstride, perm.p, used.p);
     }
     BF_CUDA_CHECK(cudaGetLastError());
     ImpArgs g;
