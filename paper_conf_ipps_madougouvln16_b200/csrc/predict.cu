@@ -241,7 +241,7 @@ __device__ __noinline__ uint32_t tie_right_fp64(const double* xg, int64_t ldq, u
   return !(__ldg(xg + (int64_t)f * ldq) <= __ldg(&n16[gid].v));
 }
 
-template <bool PROF>
+template <bool PROF, int NS>
 __global__ void __launch_bounds__(PT8, 6) k_predict8s(const uint2* __restrict__ nodes8, const Node16* __restrict__ nodes16,
                                                       const uint32_t* __restrict__ roots, int32_t t_begin, int32_t t_end,
                                                       int first, int last, const double* __restrict__ Xq, int64_t ldq,
@@ -279,8 +279,8 @@ __global__ void __launch_bounds__(PT8, 6) k_predict8s(const uint2* __restrict__ 
   const double* xg = Xq + rr;
   double acc = first ? 0.0 : yhat_sum[rr];
   uint32_t nv = 0, nfb = 0;
-  uint32_t gid[S8];
-  uint2 nd[S8];
+  uint32_t gid[NS];
+  uint2 nd[NS];
   int tnext = 0;
   int nact = 0;
   auto start = [&](int u) {
@@ -301,10 +301,10 @@ __global__ void __launch_bounds__(PT8, 6) k_predict8s(const uint2* __restrict__ 
     }
   };
 #pragma unroll
-  for (int u = 0; u < S8; ++u) start(u);
+  for (int u = 0; u < NS; ++u) start(u);
   while (nact > 0) {
 #pragma unroll
-    for (int u = 0; u < S8; ++u) {
+    for (int u = 0; u < NS; ++u) {
       if (gid[u] == ~0u) continue;
       const uint2 w = nd[u];
       const uint32_t f = (w.y >> N8_REL_BITS) & ((1u << N8_FEAT_BITS) - 1u);
@@ -605,9 +605,13 @@ void predict_impl(const bf_forest* f, const double* Xq_in, int64_t ldq, int64_t 
   const uint2* n8 = (force16 && force16[0] == '1') ? nullptr : nodes8_get(const_cast<bf_forest*>(f), s);
   const size_t smem8 = sizeof(float) * (size_t)PT8 * (size_t)(p | 1);
   static int smax8 = 0;
-  if (!smax8)
-    smax8 = std::min(std::min(dyn_smem_limit(k_predict8<true>), dyn_smem_limit(k_predict8<false>)),
-                     std::min(dyn_smem_limit(k_predict8s<true>), dyn_smem_limit(k_predict8s<false>)));
+  if (!smax8) {
+    smax8 = std::min(dyn_smem_limit(k_predict8<true>), dyn_smem_limit(k_predict8<false>));
+    smax8 = std::min(smax8, std::min(dyn_smem_limit(k_predict8s<true, 6>), dyn_smem_limit(k_predict8s<false, 6>)));
+    smax8 = std::min(smax8, std::min(dyn_smem_limit(k_predict8s<true, 8>), dyn_smem_limit(k_predict8s<false, 8>)));
+    smax8 = std::min(smax8, std::min(dyn_smem_limit(k_predict8s<true, 12>), dyn_smem_limit(k_predict8s<false, 12>)));
+  }
+  static const int slots = getenv("BF_PREDICT_SLOTS") ? atoi(getenv("BF_PREDICT_SLOTS")) : 8;
   static const int pv = getenv("BF_PREDICT_V") ? atoi(getenv("BF_PREDICT_V")) : 2;
   if (n8 && smem8 <= (size_t)smax8) {
     // tree blocks of <= 32 MB of Node8 (L2-resident while every row walks them)
@@ -623,7 +627,9 @@ void predict_impl(const bf_forest* f, const double* Xq_in, int64_t ldq, int64_t 
       while (t1 < nt && (f->tree_off[t1 + 1] - f->tree_off[t0]) * (int64_t)sizeof(uint2) <= block_bytes) ++t1;
       if (t1 - t0 <= RT8 && pv != 1) {
         KScope ks_("k_predict8", s, 0.0);
-        (vis.p ? k_predict8s<true> : k_predict8s<false>)<<<(unsigned)ceil_div(m, PT8), PT8, smem8, s>>>(
+        auto kern = vis.p ? (slots == 6 ? k_predict8s<true, 6> : slots == 12 ? k_predict8s<true, 12> : k_predict8s<true, 8>)
+                          : (slots == 6 ? k_predict8s<false, 6> : slots == 12 ? k_predict8s<false, 12> : k_predict8s<false, 8>);
+        kern<<<(unsigned)ceil_div(m, PT8), PT8, smem8, s>>>(
             n8, f->d_nodes, f->d_roots8, t0, t1, t0 == 0, t1 >= nt, (const double*)Xs.dptr, ldq, m, p, ysum,
             yh_in ? (double*)yh.dptr : nullptr, inv_t, vis.p);
       } else {
