@@ -735,6 +735,35 @@ __global__ void k_tree_ranges(int N, const LNode* nodes, int32_t* lo, int32_t* h
   if (k == N - 1 || nodes[k + 1].b != b) hi[b] = k + 1;
 }
 
+// The level's trees that have nodes (thi > tlo), in tree order; one CTA of >= B threads.
+__global__ void k_active_trees(int B, const int32_t* tlo, const int32_t* thi, int32_t* active, int32_t* nactive) {
+  __shared__ int32_t cnt;
+  if (threadIdx.x == 0) cnt = 0;
+  __syncthreads();
+  for (int b0 = 0; b0 < B; b0 += blockDim.x) {
+    const int b = b0 + threadIdx.x;
+    const bool on = b < B && thi[b] > tlo[b];
+    const unsigned m = __ballot_sync(0xffffffffu, on);
+    __shared__ int32_t wbase[32];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    if (lane == 0) wbase[wid] = __popc(m);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      int run = cnt;
+      for (int w = 0; w < (int)(blockDim.x >> 5); ++w) {
+        const int c = wbase[w];
+        wbase[w] = run;
+        run += c;
+      }
+      cnt = run;
+    }
+    __syncthreads();
+    if (on) active[wbase[wid] + __popc(m & ((1u << lane) - 1u))] = b;
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) *nactive = cnt;
+}
+
 struct TreeSched {  // CTA -> (tree, slot, slots per tree)
   int b0, bstep, c, C;
 };
@@ -764,6 +793,8 @@ struct TScanArgs {
   const int32_t* tlo;  // per tree: first node of the level (or 0) / one past the last
   const int32_t* thi;
   Rec* rec;
+  const int32_t* active;   // the level's trees that have nodes, and how many (k_active_trees)
+  const int32_t* nactive;
 };
 
 constexpr int TSV = 9;              // entries per thread (odd: conflict-free 64-bit shared loads)
@@ -801,7 +832,9 @@ __global__ void __launch_bounds__(SNT, 4) k_split_scan_tree(TScanArgs g) {
   __shared__ WBest swb[NW];
   __shared__ int s_off[2];
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  const TreeSched ts = tree_sched(g.B);
+  // CTAs are spread over the level's ACTIVE trees (deep levels often have nodes in a few trees only)
+  const int NA = *g.nactive;
+  const TreeSched ts = tree_sched(NA);
   if (tid == 0) {
     mbar_init(&bar[0]);
     mbar_init(&bar[1]);
@@ -809,7 +842,8 @@ __global__ void __launch_bounds__(SNT, 4) k_split_scan_tree(TScanArgs g) {
   __syncthreads();
   uint32_t phase[2] = {0u, 0u};
   int cur = 0;
-  for (int b = ts.b0; b < g.B; b += ts.bstep) {
+  for (int ai = ts.b0; ai < NA; ai += ts.bstep) {
+    const int b = g.active[ai];
     const int i_lo = g.tlo[b] * g.mtry, i_hi = g.thi[b] * g.mtry;
     int item = i_lo + ts.c, unit = 0;
     auto issue = [&](int it, int un, int slot) {
@@ -1034,6 +1068,8 @@ struct TPartArgs {
   const int32_t* thi;
   const int32_t* ioff;  // per node: first work item (N + 1 entries; items of a tree are contiguous)
   const int2* imap;     // per work item: (node, first feature)
+  const int32_t* active;   // the level's trees that have nodes, and how many (k_active_trees)
+  const int32_t* nactive;
 };
 
 constexpr int TPNT = 512;           // threads of the partition CTA (one CTA per SM: the bitmap fills shared memory)
@@ -1129,7 +1165,8 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
   int32_t* sm = sms[grp];
   int* s_off = s_offs[grp];
   PWork* s_w = s_ws[grp];
-  const TreeSched ts = tree_sched(g.B);
+  const int NA = *g.nactive;  // CTAs spread over the level's active trees
+  const TreeSched ts = tree_sched(NA);
   if (lt == 0) {
     mbar_init(&bar[0]);
     mbar_init(&bar[1]);
@@ -1137,7 +1174,8 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
   __syncthreads();
   uint32_t phase[2] = {0u, 0u};
   int cur = 0;
-  for (int b = ts.b0; b < g.B; b += ts.bstep) {
+  for (int ai = ts.b0; ai < NA; ai += ts.bstep) {
+    const int b = g.active[ai];
     const int n_lo = g.tlo[b], n_hi = g.thi[b];
     if (n_lo >= n_hi) continue;
     const uint32_t* sideg = g.sideb + (int64_t)b * g.nw;
@@ -2804,7 +2842,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
     // tree-affine kernels
     const int64_t nw = (n + 31) / 32;
     DBuf<uint32_t> sideb((size_t)B * nw, s);
-    DBuf<int32_t> tlo(B, s), thi(B, s);
+    DBuf<int32_t> tlo(B, s), thi(B, s), act(B, s), nact(1, s);
     const size_t tscan_smem = sizeof(uint64_t) * 2 * (TUNIT + 4);
     const size_t tpart_base = sizeof(uint64_t) * (size_t)TPG * (3 * TPUNIT + 4);
     const int smem_optin = dyn_smem_limit(k_partition_tree);
@@ -2937,11 +2975,12 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
         BF_CUDA_CHECK(cudaMemsetAsync(tlo.p, 0, sizeof(int32_t) * Bc, s));
         BF_CUDA_CHECK(cudaMemsetAsync(thi.p, 0, sizeof(int32_t) * Bc, s));
         {
-          KScope ks_("k_tree_ranges", s, 0.0);
+          KScope ks_("k_tree_ranges", s, 0.0, 2);
           k_tree_ranges<<<(unsigned)ceil_div(N, 256), 256, 0, s>>>(N, nc, tlo.p, thi.p);
+          k_active_trees<<<1, 256, 0, s>>>(Bc, tlo.p, thi.p, act.p, nact.p);
         }
         {  // ---- a7 split search: tree-affine CTAs own whole (node, drawn feature) items
-          TScanArgs ga{nc, feat.p, mtry, Bc, Ec, yq.p, tlo.p, thi.p, rec.p};
+          TScanArgs ga{nc, feat.p, mtry, Bc, Ec, yq.p, tlo.p, thi.p, rec.p, act.p, nact.p};
           KScope ks_("k_split_scan_tree", s, 0.0);
           k_split_scan_tree<<<grid_tscan, SNT, tscan_smem, s>>>(ga);
         }
@@ -2981,7 +3020,8 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
           k_part_items_map<<<(unsigned)ceil_div(N, 256), 256, 0, s>>>(N, p, nc, icnt.p, ioff.p, imap.p);
         }
         {
-          TPartArgs ga{nc, split.p, child.p, p, Bc, Ec, sideb.p, nw, bm_smem ? 1 : 0, En, Es.p, tlo.p, thi.p, ioff.p, imap.p};
+          TPartArgs ga{nc, split.p, child.p, p, Bc, Ec, sideb.p, nw, bm_smem ? 1 : 0, En, Es.p, tlo.p, thi.p, ioff.p, imap.p,
+                       act.p, nact.p};
           KScope ks_("k_partition_tree", s, 0.0);
           k_partition_tree<<<grid_tpart, TPNT, tpart_smem, s>>>(ga);
         }

@@ -611,7 +611,7 @@ void predict_impl(const bf_forest* f, const double* Xq_in, int64_t ldq, int64_t 
     smax8 = std::min(smax8, std::min(dyn_smem_limit(k_predict8s<true, 8>), dyn_smem_limit(k_predict8s<false, 8>)));
     smax8 = std::min(smax8, std::min(dyn_smem_limit(k_predict8s<true, 12>), dyn_smem_limit(k_predict8s<false, 12>)));
   }
-  static const int slots = getenv("BF_PREDICT_SLOTS") ? atoi(getenv("BF_PREDICT_SLOTS")) : 8;
+  static const int slots = getenv("BF_PREDICT_SLOTS") ? atoi(getenv("BF_PREDICT_SLOTS")) : 6;  // measured: 6 < 8 < 12 (profiles/r02o)
   static const int pv = getenv("BF_PREDICT_V") ? atoi(getenv("BF_PREDICT_V")) : 2;
   if (n8 && smem8 <= (size_t)smax8) {
     // tree blocks of <= 32 MB of Node8 (L2-resident while every row walks them)
