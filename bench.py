@@ -218,19 +218,26 @@ def config_json(cfg, n, p, T, m, world, extra=None):
 
 
 # ---------------------------------------------------------------------------- the oracle on the host cores
+_ORACLE_PREV = []  # C4: the previous sample's oracle forests (their importance runs beside the next fits)
+
+
 def oracle_sample(args, S, cfg, T, m, X, y, Xrf=None, step: int = 0):
     """One bounded sample of the workload on the host cores with the oracle (oracle/bfo.c via
     oracle/oracle.py, as it stands), and its whole-job-equivalent throughput.
 
-    C4: k = cores trees (one per host thread, trees rotate with the step) are grown, predicted on a
-    1M-row query sample (row chunks on the host threads) and their OOB importance computed (one tree per
-    thread); PCA once.  C1-C3: all T trees, a 100K-row query sample.  The cost is extrapolated linearly to
-    T trees and m rows (trees are i.i.d. in cost; query rows are i.i.d. in cost).
-    Returns (trees/s, wall seconds of the sample, sample description)."""
+    C4: 3/4 of the host threads each grow one tree (the trees rotate with the step) while the other 1/4 each
+    compute the OOB importance of one tree of the previous sample (of this sample's first trees if there is no
+    previous one), one tree per thread; then a 1M-row query sample is predicted with this sample's trees (row
+    chunks on all threads) and PCA runs once.  Per-tree fit and importance times are per thread, so the job
+    of T trees and m rows on `cores` threads takes T (t_fit + t_imp) / cores + the predict time scaled to T
+    trees and m rows (trees and query rows are i.i.d. in cost) + PCA; the step's wall time stays about one
+    tree's fit.  C1-C3: all T trees (fit over all threads), a 100K-row query sample, importance, PCA.
+    Returns (trees/s, wall seconds of the sample, sample description, threads)."""
     from concurrent.futures import ThreadPoolExecutor
 
     from oracle import oracle as O
     from oracle.pca import n_components, pca
+    global _ORACLE_PREV
     cores = os.cpu_count() or 1
     seed = S.FOREST_SEED + 4
     t_all = time.perf_counter()
@@ -245,19 +252,39 @@ def oracle_sample(args, S, cfg, T, m, X, y, Xrf=None, step: int = 0):
         t_pca = time.perf_counter() - t0
     Xf = Xrf if Xrf is not None else X
     big = cfg.n >= 1_000_000
-    k = min(cores, T) if big else T
-    b0 = (step * k) % T if big else 0
-    rng = [(b0 + i) % T for i in range(k)]
-    # fit: one tree per host thread (C4) or all trees over the host threads (C1-C3)
-    t0 = time.perf_counter()
-    if big:
-        with ThreadPoolExecutor(cores) as ex:
-            forests = list(ex.map(lambda t: O.fit(Xf, y, ntree=T, seed=seed, tree_begin=t, tree_end=t + 1), rng))
-    else:
-        forests = [O.fit(Xf, y, ntree=T, seed=seed, nthreads=cores)]
-    t_fit = time.perf_counter() - t0
-    # predict: query rows in chunks over the host threads
     m_s = min(m, 1_000_000 if big else 100_000)
+
+    def timed(fn, *a):
+        t0 = time.perf_counter()
+        r = fn(*a)
+        return r, time.perf_counter() - t0
+
+    if big:
+        ki = max(1, cores // 4) if cfg.importance else 0
+        kf = max(1, min(cores - ki, T))
+        b0 = (step * kf) % T
+        ids = [(b0 + i) % T for i in range(kf)]
+        prev = _ORACLE_PREV[:ki]
+        with ThreadPoolExecutor(cores) as ex:
+            ff = [ex.submit(timed, lambda t: O.fit(Xf, y, ntree=T, seed=seed, tree_begin=t, tree_end=t + 1), t)
+                  for t in ids]
+            fi = [ex.submit(timed, lambda f: f.oob_importance(Xf, y), f) for f in prev]
+            fits = [x.result() for x in ff]
+            imps = [x.result()[1] for x in fi]
+        forests = [f for f, _ in fits]
+        t_fit_tree = float(np.mean([d for _, d in fits]))
+        if ki and not imps:  # no previous sample: this sample's first trees
+            with ThreadPoolExecutor(cores) as ex:
+                imps = [d for _, d in ex.map(lambda f: timed(lambda g: g.oob_importance(Xf, y), f), forests[:ki])]
+        t_imp_tree = float(np.mean(imps)) if imps else 0.0
+        _ORACLE_PREV = forests
+        k = kf
+    else:
+        t0 = time.perf_counter()
+        forests = [O.fit(Xf, y, ntree=T, seed=seed, nthreads=cores)]
+        t_fit = time.perf_counter() - t0
+        k = T
+    # predict: query rows in chunks over the host threads
     t_pred = 0.0
     if m_s > 0:
         Q = S.gen_query(Xf, m_s, chunk=1 << 18)
@@ -267,21 +294,24 @@ def oracle_sample(args, S, cfg, T, m, X, y, Xrf=None, step: int = 0):
             list(ex.map(lambda f_c: f_c[0].predict_sum(np.ascontiguousarray(Q[:, f_c[1][0]:f_c[1][1]])),
                         [(f, c) for f in forests for c in chunks]))
         t_pred = time.perf_counter() - t0
-    # OOB importance: one forest (tree) per host thread
-    t_imp = 0.0
-    if cfg.importance:
-        t0 = time.perf_counter()
-        with ThreadPoolExecutor(cores) as ex:
-            list(ex.map(lambda f: f.oob_importance(Xf, y), forests))
-        t_imp = time.perf_counter() - t0
+    if big:
+        job = T * (t_fit_tree + t_imp_tree) / cores + t_pred * (m / m_s) * (T / k) + t_pca
+        desc = (f"{k} of {T} trees (global ids {ids[0]}..{ids[-1]}) grown by oracle bfo_fit one per host thread "
+                f"({t_fit_tree:.1f} s per tree) beside the OOB importance of {len(imps)} trees of the previous "
+                f"sample ({t_imp_tree:.1f} s per tree), predicted on {m_s} of {m} query rows ({t_pred:.1f} s), PCA "
+                f"({t_pca:.2f} s); job = T (fit + importance per tree) / threads + predict scaled to {T} trees and "
+                f"{m} rows + PCA")
+    else:
+        t_imp = 0.0
+        if cfg.importance:
+            t0 = time.perf_counter()
+            forests[0].oob_importance(Xf, y)
+            t_imp = time.perf_counter() - t0
+        job = t_fit + t_imp + t_pred * (m / m_s if m_s else 0.0) + t_pca
+        desc = (f"all {T} trees by oracle bfo_fit over {cores} host threads ({t_fit:.1f} s), {m_s} of {m} query "
+                f"rows ({t_pred:.1f} s), OOB importance ({t_imp:.1f} s), PCA ({t_pca:.2f} s); extrapolated "
+                f"linearly to {m} rows")
     wall = time.perf_counter() - t_all
-    job = (T / k) * (t_fit + t_imp + t_pred * (m / m_s if m_s else 0.0)) + t_pca
-    desc = (f"{k} of {T} trees (global ids {rng[0]}..{rng[-1]}) grown by oracle bfo_fit one per host thread "
-            f"({t_fit:.1f} s), predicted on {m_s} of {m} query rows ({t_pred:.1f} s), OOB importance "
-            f"({t_imp:.1f} s), PCA ({t_pca:.2f} s); extrapolated linearly to {T} trees and {m} rows"
-            if big else
-            f"all {T} trees by oracle bfo_fit over {cores} host threads ({t_fit:.1f} s), {m_s} of {m} query rows "
-            f"({t_pred:.1f} s), OOB importance ({t_imp:.1f} s), PCA ({t_pca:.2f} s); extrapolated linearly to {m} rows")
     return T / job, wall, desc, cores
 
 

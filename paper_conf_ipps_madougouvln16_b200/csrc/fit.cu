@@ -383,41 +383,56 @@ __global__ void k_list_prefix(int32_t* cnt, int nseg, int nchunk) {
   }
 }
 
+// Warp w of the CTA owns the chunk's entries [w * 256, (w + 1) * 256), read in rounds of 32 (entry
+// w * 256 + 32 u + lane): per round the in-bag entries of one tree are consecutive in the output, so every store
+// instruction writes one contiguous run; one block barrier per tree for the warps' in-bag counts.
 __global__ void k_list_scatter(const uint64_t* srt, int64_t n, const uint16_t* wp, int Bp, const int32_t* kind,
                                const int64_t* base, const int32_t* a_root, int nchunk, int B, const int32_t* cnt,
                                uint64_t* Elarge, uint64_t* Esmall) {
   const int c = blockIdx.x, f = blockIdx.y, b0 = blockIdx.z * LTG, p = gridDim.y;
-  __shared__ int32_t sm[NT / 32];
-  constexpr int V = LCH / NT;
+  constexpr int V = LCH / NT, NW = NT / 32;
+  __shared__ int32_t sm[2][NW];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const uint64_t* col = srt + (int64_t)f * n;
-  const int64_t i0 = (int64_t)c * LCH + (int64_t)threadIdx.x * V;
+  const int64_t i0 = (int64_t)c * LCH + (int64_t)wid * (V * 32) + lane;
   uint64_t e[V];
   uint4 q[V];
 #pragma unroll
-  for (int u = 0; u < V; ++u) e[u] = i0 + u < n ? col[i0 + u] : ~0ull;
+  for (int u = 0; u < V; ++u) e[u] = i0 + 32 * u < n ? col[i0 + 32 * u] : ~0ull;
 #pragma unroll
   for (int u = 0; u < V; ++u)
     q[u] = e[u] != ~0ull ? *reinterpret_cast<const uint4*>(wp + (int64_t)e_row(e[u]) * Bp + b0)
                          : make_uint4(0u, 0u, 0u, 0u);
+  const uint32_t ltm = (1u << lane) - 1u;
+  int par = 0;
   for (int t = 0; t < LTG && b0 + t < B; ++t) {
     const int b = b0 + t;
     const int kd = kind[b];
     if (kd != KIND_LARGE && kd != KIND_SMALL) continue;  // uniform per CTA
-    int32_t k = 0;
-#pragma unroll
-    for (int u = 0; u < V; ++u) k += wp_get(q[u], t) > 0;
-    int32_t tot;
-    int32_t pre = block_excl_scan(k, sm, tot) + cnt[((int64_t)b * p + f) * nchunk + c];
-    uint64_t* dst = (kd == KIND_LARGE ? Elarge : Esmall) + base[b] + (int64_t)f * a_root[b];
+    uint32_t m[V];
+    int32_t wc = 0;
 #pragma unroll
     for (int u = 0; u < V; ++u) {
-      const uint32_t wv = wp_get(q[u], t);
-      if (wv > 0) dst[pre++] = e[u] | (uint64_t)wv;
+      m[u] = __ballot_sync(0xffffffffu, wp_get(q[u], t) > 0);
+      wc += __popc(m[u]);
+    }
+    if (lane == 0) sm[par][wid] = wc;
+    __syncthreads();  // sm[par] is next written two trees later, after another barrier
+    int32_t pre = cnt[((int64_t)b * p + f) * nchunk + c];
+#pragma unroll
+    for (int k = 0; k < NW; ++k)
+      if (k < wid) pre += sm[par][k];
+    par ^= 1;
+    uint64_t* dst = (kd == KIND_LARGE ? Elarge : Esmall) + base[b] + (int64_t)f * a_root[b] + pre;
+    int run = 0;
+#pragma unroll
+    for (int u = 0; u < V; ++u) {
+      if ((m[u] >> lane) & 1u) dst[run + __popc(m[u] & ltm)] = e[u] | (uint64_t)wp_get(q[u], t);
+      run += __popc(m[u]);
     }
   }
 }
 
-// ------------------------------------------------------------------ a6 mtry (global phase)
 __global__ void k_mtry(const LNode* nodes, int N, int p, int mtry, uint64_t seed, int32_t t0, int32_t* feat,
                        int16_t* scratch) {
   const int k = blockIdx.x * blockDim.x + threadIdx.x;
@@ -1125,38 +1140,19 @@ struct PWork {
   int64_t bl, br;         // children: block offsets
 };
 
-// Group-local barrier (named barrier 1 + group over the group's TPGT threads) and exclusive scan.
+// Group-local barrier (named barrier 1 + group over the group's TPGT threads).
 __device__ __forceinline__ void group_sync(int grp) {
   asm volatile("bar.sync %0, %1;" ::"r"(1 + grp), "r"(TPGT) : "memory");
 }
-__device__ __forceinline__ int32_t group_excl_scan(int32_t v, int32_t* sm, int32_t& total, int grp, int lt) {
-  const int lane = lt & 31, wid = lt >> 5;
-  constexpr int nw = TPGT / 32;
-  int32_t inc = warp_incl_scan(v, lane);
-  if (lane == 31) sm[wid] = inc;
-  group_sync(grp);
-  if (wid == 0) {
-    int32_t x = lane < nw ? sm[lane] : 0;
-    x = warp_incl_scan(x, lane);
-    if (lane < nw) sm[lane] = x;
-  }
-  group_sync(grp);
-  const int32_t pre = wid ? sm[wid - 1] : 0;
-  total = sm[nw - 1];
-  // no trailing barrier: the caller's next write of sm (the next unit's scan) follows its own group barriers
-  return pre + inc - v;
-}
-
 // The CTA's TPG thread groups share the tree's goes-right bitmap in shared memory and run independent unit
 // pipelines (own bulk-copy buffers, mbarriers and named barriers) over alternate items of the CTA's slice,
 // so one group's barrier and copy waits overlap the other group's work.
 __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
   extern __shared__ __align__(16) unsigned char dsm[];
   const int tid = threadIdx.x, grp = tid / TPGT, lt = tid % TPGT;
-  uint64_t* gbase = (uint64_t*)dsm + (size_t)grp * (3 * TPUNIT + 4);
+  uint64_t* gbase = (uint64_t*)dsm + (size_t)grp * (2 * TPUNIT + 4);
   uint64_t* bufs = gbase;                       // 2 x (TPUNIT + 2)
-  uint64_t* outb = bufs + 2 * (TPUNIT + 2);     // TPUNIT
-  uint32_t* bm = (uint32_t*)((uint64_t*)dsm + (size_t)TPG * (3 * TPUNIT + 4));  // nw words (if staged)
+  uint32_t* bm = (uint32_t*)((uint64_t*)dsm + (size_t)TPG * (2 * TPUNIT + 4));  // nw words (if staged)
   __shared__ uint64_t bars[TPG][2];
   __shared__ int32_t sms[TPG][TPGT / 32];
   __shared__ int s_offs[TPG][2];
@@ -1271,11 +1267,16 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
       mbar_wait(&bar[cur], phase[cur]);
       phase[cur] ^= 1u;
       const uint64_t* buf = bufs + (size_t)cur * (TPUNIT + 2) + s_off[cur];
-      const int jl = lt * TPV;
+      // Warp wg of the group owns the unit's entries [wg * 32 TPV, (wg + 1) * 32 TPV), read striped (entry
+      // wg * 32 TPV + 32 q + lane): per round q the lanes' lefts (rights) are consecutive in the output, so each
+      // store instruction writes one contiguous run straight to the child block in global memory -- no shared
+      // staging buffer, one group barrier per unit for the warps' left counts.
+      const int lane = lt & 31, wg = lt >> 5;
+      const int wb0 = wg * (TPV * 32);
       uint64_t ev[TPV];
       uint32_t bw[TPV];
 #pragma unroll
-      for (int q = 0; q < TPV; ++q) ev[q] = buf[min(jl + q, cnt - 1)];
+      for (int q = 0; q < TPV; ++q) ev[q] = buf[min(wb0 + 32 * q + lane, cnt - 1)];
       if (g.bitmap_smem) {
 #pragma unroll
         for (int q = 0; q < TPV; ++q) bw[q] = sb[e_row(ev[q]) >> 5];
@@ -1283,40 +1284,44 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
 #pragma unroll
         for (int q = 0; q < TPV; ++q) bw[q] = ldg_u32_nc(sb + (e_row(ev[q]) >> 5));
       }
-      uint32_t lmask = 0;
-      int32_t c = 0;
+      uint32_t lmk[TPV];
+      int32_t wl_cnt = 0;
 #pragma unroll
-      for (int q = 0; q < TPV; ++q)
-        if (jl + q < cnt && !((bw[q] >> (e_row(ev[q]) & 31)) & 1u)) {
-          lmask |= 1u << q;
-          ++c;
-        }
-      int32_t tot;
-      const int32_t lbl = group_excl_scan(c, sm, tot, grp, lt);
-      const int al = w.al, ar = w.ar;  // lefts / rights per feature segment
-      {
-        int li = lbl, ri = tot + (jl - lbl);
-#pragma unroll
-        for (int q = 0; q < TPV; ++q) {
-          const int j = jl + q;
-          if (j < cnt) {
-            if ((lmask >> q) & 1u) outb[li++] = ev[q];
-            else outb[ri++] = ev[q];
-          }
-        }
+      for (int q = 0; q < TPV; ++q) {
+        const bool left = wb0 + 32 * q + lane < cnt && !((bw[q] >> (e_row(ev[q]) & 31)) & 1u);
+        lmk[q] = __ballot_sync(0xffffffffu, left);
+        wl_cnt += __popc(lmk[q]);
       }
+      if (lane == 0) sm[wg] = wl_cnt;
       group_sync(grp);
+      int32_t preL = 0, tot = 0;
+#pragma unroll
+      for (int k = 0; k < TPGT / 32; ++k) {
+        const int32_t v = sm[k];
+        if (k < wg) preL += v;
+        tot += v;
+      }
+      const int al = w.al, ar = w.ar;  // lefts / rights per feature segment
       const bool keepL = w.kl == KIND_LARGE || w.kl == KIND_SMALL;
       const bool keepR = w.kr == KIND_LARGE || w.kr == KIND_SMALL;
       const int64_t exl = carry_l, exr = (int64_t)u0 - carry_l;
-      const int nl_out = tot, nr_out = cnt - nl_out;
-      if (keepL) {
-        uint64_t* dl = (w.kl == KIND_LARGE ? g.Enext : g.Esmall) + w.bl + (int64_t)w.f0 * al + exl;
-        for (int i = lt; i < nl_out; i += TPGT) dl[i] = outb[i];
-      }
-      if (keepR) {
-        uint64_t* dr = (w.kr == KIND_LARGE ? g.Enext : g.Esmall) + w.br + (int64_t)w.f0 * ar + exr;
-        for (int i = lt; i < nr_out; i += TPGT) dr[i] = outb[nl_out + i];
+      uint64_t* dl = (w.kl == KIND_LARGE ? g.Enext : g.Esmall) + w.bl + (int64_t)w.f0 * al + exl + preL;
+      uint64_t* dr = (w.kr == KIND_LARGE ? g.Enext : g.Esmall) + w.br + (int64_t)w.f0 * ar + exr +
+                     (min(wb0, cnt) - preL);
+      const uint32_t ltm = (1u << lane) - 1u;
+      int runL = 0, runR = 0;
+#pragma unroll
+      for (int q = 0; q < TPV; ++q) {
+        const int j = wb0 + 32 * q + lane;
+        const uint32_t vm = __ballot_sync(0xffffffffu, j < cnt);
+        const uint32_t rm = vm & ~lmk[q];
+        if ((lmk[q] >> lane) & 1u) {
+          if (keepL) dl[runL + __popc(lmk[q] & ltm)] = ev[q];
+        } else if ((rm >> lane) & 1u) {
+          if (keepR) dr[runR + __popc(rm & ltm)] = ev[q];
+        }
+        runL += __popc(lmk[q]);
+        runR += __popc(rm);
       }
       carry_l += tot;
       {
@@ -2844,7 +2849,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
     DBuf<uint32_t> sideb((size_t)B * nw, s);
     DBuf<int32_t> tlo(B, s), thi(B, s), act(B, s), nact(1, s);
     const size_t tscan_smem = sizeof(uint64_t) * 2 * (TUNIT + 4);
-    const size_t tpart_base = sizeof(uint64_t) * (size_t)TPG * (3 * TPUNIT + 4);
+    const size_t tpart_base = sizeof(uint64_t) * (size_t)TPG * (2 * TPUNIT + 4);
     const int smem_optin = dyn_smem_limit(k_partition_tree);
     const bool bm_smem = getenv("BF_PART_L2") == nullptr && tpart_base + (size_t)nw * 4 <= (size_t)smem_optin;
     const size_t tpart_smem = tpart_base + (bm_smem ? (size_t)nw * 4 : 0);
