@@ -1092,6 +1092,7 @@ constexpr int TPG = 2;              // independent unit pipelines per CTA (threa
 constexpr int TPGT = TPNT / TPG;    // threads per group
 constexpr int TPV = 7;
 constexpr int TPUNIT = TPGT * TPV;  // 1792 entries per unit
+constexpr int TPNS = 3;             // bulk-copy buffers per group (units in flight: TPNS - 1 ahead)
 
 __device__ __forceinline__ bool part_item_active(const Split* split, const Child* child, int node) {
   if (!split[node].split) return false;
@@ -1150,25 +1151,23 @@ __device__ __forceinline__ void group_sync(int grp) {
 __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
   extern __shared__ __align__(16) unsigned char dsm[];
   const int tid = threadIdx.x, grp = tid / TPGT, lt = tid % TPGT;
-  uint64_t* gbase = (uint64_t*)dsm + (size_t)grp * (2 * TPUNIT + 4);
-  uint64_t* bufs = gbase;                       // 2 x (TPUNIT + 2)
-  uint32_t* bm = (uint32_t*)((uint64_t*)dsm + (size_t)TPG * (2 * TPUNIT + 4));  // nw words (if staged)
-  __shared__ uint64_t bars[TPG][2];
+  uint64_t* gbase = (uint64_t*)dsm + (size_t)grp * (TPNS * (TPUNIT + 2));
+  uint64_t* bufs = gbase;                       // TPNS x (TPUNIT + 2): bulk-copy ring, TPNS - 1 units ahead
+  uint32_t* bm = (uint32_t*)((uint64_t*)dsm + (size_t)TPG * (TPNS * (TPUNIT + 2)));  // nw words (if staged)
+  __shared__ uint64_t bars[TPG][TPNS];
   __shared__ int32_t sms[TPG][TPGT / 32];
-  __shared__ int s_offs[TPG][2];
-  __shared__ PWork s_ws[TPG][2];
+  __shared__ int s_offs[TPG][TPNS];
+  __shared__ PWork s_ws[TPG][TPNS];
   uint64_t* bar = bars[grp];
   int32_t* sm = sms[grp];
   int* s_off = s_offs[grp];
   PWork* s_w = s_ws[grp];
   const int NA = *g.nactive;  // CTAs spread over the level's active trees
   const TreeSched ts = tree_sched(NA);
-  if (lt == 0) {
-    mbar_init(&bar[0]);
-    mbar_init(&bar[1]);
-  }
+  if (lt == 0)
+    for (int k = 0; k < TPNS; ++k) mbar_init(&bar[k]);
   __syncthreads();
-  uint32_t phase[2] = {0u, 0u};
+  uint32_t phase[TPNS] = {};
   int cur = 0;
   for (int ai = ts.b0; ai < NA; ai += ts.bstep) {
     const int b = g.active[ai];
@@ -1241,25 +1240,34 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
       s_off[slot] = stage_entries(bufs + (size_t)slot * (TPUNIT + 2), g.Ecur + w.base + (int64_t)w.f0 * w.a + u0, cnt,
                                   &bar[slot]);
     };
-    // the group's thread 0 runs the item pipeline and publishes each unit's record in s_w[slot]
+    // the group's thread 0 runs the item pipeline TPNS - 1 units ahead and publishes each unit's record in s_w
     if (lt == 0) {
-      PWork w0;
-      if (!next_mine(w0)) w0.node = -1;
-      s_w[cur] = w0;
-      if (w0.node >= 0) issue(w0, cur);
+      bool more = true;
+      for (int k = 0; k + 1 < TPNS; ++k) {
+        PWork w0;
+        if (!more || !next_mine(w0)) {
+          w0.node = -1;
+          more = false;
+        }
+        const int sl = (cur + k) % TPNS;
+        s_w[sl] = w0;
+        if (w0.node >= 0) issue(w0, sl);
+      }
     }
     group_sync(grp);
     if (s_w[cur].node < 0) continue;
     int64_t carry_l = 0;
     for (;;) {
-      group_sync(grp);  // the other buffer and s_w slot are free
+      group_sync(grp);  // the buffer and s_w slot of unit k - 1 are free
       const PWork w = s_w[cur];
       if (w.node < 0) break;
+      const int nxt = (cur + 1) % TPNS;
       if (lt == 0) {
+        const int sl = (cur + TPNS - 1) % TPNS;  // unit k + TPNS - 1
         PWork wn;
-        if (!next_mine(wn)) wn.node = -1;
-        s_w[cur ^ 1] = wn;
-        if (wn.node >= 0) issue(wn, cur ^ 1);
+        if (s_w[(cur + TPNS - 2) % TPNS].node < 0 || !next_mine(wn)) wn.node = -1;
+        s_w[sl] = wn;
+        if (wn.node >= 0) issue(wn, sl);
       }
       const int a = w.a;
       const int u0 = w.unit * TPUNIT;
@@ -1325,10 +1333,10 @@ __global__ void __launch_bounds__(TPNT) k_partition_tree(TPartArgs g) {
       }
       carry_l += tot;
       {
-        const PWork& wn = s_w[cur ^ 1];  // published before this unit's scan barriers
+        const PWork& wn = s_w[nxt];  // published a unit ago
         if (wn.node != w.node || wn.f0 != w.f0) carry_l = 0;
       }
-      cur ^= 1;
+      cur = nxt;
     }
   }
 }
@@ -2849,7 +2857,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
     DBuf<uint32_t> sideb((size_t)B * nw, s);
     DBuf<int32_t> tlo(B, s), thi(B, s), act(B, s), nact(1, s);
     const size_t tscan_smem = sizeof(uint64_t) * 2 * (TUNIT + 4);
-    const size_t tpart_base = sizeof(uint64_t) * (size_t)TPG * (2 * TPUNIT + 4);
+    const size_t tpart_base = sizeof(uint64_t) * (size_t)TPG * (TPNS * (TPUNIT + 2));
     const int smem_optin = dyn_smem_limit(k_partition_tree);
     const bool bm_smem = getenv("BF_PART_L2") == nullptr && tpart_base + (size_t)nw * 4 <= (size_t)smem_optin;
     const size_t tpart_smem = tpart_base + (bm_smem ? (size_t)nw * 4 : 0);
