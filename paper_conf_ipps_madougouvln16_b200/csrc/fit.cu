@@ -1092,7 +1092,7 @@ constexpr int TPG = 2;              // independent unit pipelines per CTA (threa
 constexpr int TPGT = TPNT / TPG;    // threads per group
 constexpr int TPV = 7;
 constexpr int TPUNIT = TPGT * TPV;  // 1792 entries per unit
-constexpr int TPNS = 3;             // bulk-copy buffers per group (units in flight: TPNS - 1 ahead)
+constexpr int TPNS = 2;             // bulk-copy buffers per group (units in flight: TPNS - 1 ahead; 3 measured slower)
 
 __device__ __forceinline__ bool part_item_active(const Split* split, const Child* child, int node) {
   if (!split[node].split) return false;
