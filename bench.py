@@ -571,6 +571,8 @@ def run_ours(args):
         "fit_trees_per_s": T / (phase[0] / 1e3) if phase[0] > 0 else None,
         "predict_node_visits_per_walk": (vis / (m * (t1 - t0))) if m and vis and t1 > t0 else None,
         "predict_fp64_fallbacks_per_visit": (fbk / vis) if vis else None,
+        "importance_node_loads": stats.get("importance_node_loads", {}).get("bytes"),
+        "importance_rewalks": stats.get("importance_rewalks", {}).get("bytes"),
         "phases_ms": {"fit": phase[0], "predict": phase[1], "importance": phase[2], "pca": phase[3]},
         "step_ms": step_ms,
         "gpu_launches": int(launches),

@@ -268,6 +268,18 @@ int bf_mars_predict(const double* X, int64_t ldx, int64_t m, int32_t d, int32_t 
  * shared memory (p <= 14000).                                              */
 int bf_rank_similarity(const double* a, const double* b, int32_t p, double* out, void* stream);
 
+/* Default counter-model design of one problem characteristic (reading R26;
+ * P:222 sizes 2^5..2^11, P:254 lengths 64..8192): u = (log2 s - mean) / sd
+ * over the n sizes (sample sd, n - 1); Z row r at Z[r * ldz + i] (the k x n
+ * design layout of bf_glm_gaussian) = [1, u, u^2, u^3].  size > 0; n >= 2.
+ * Device or host pointers.                                                 */
+int bf_log_size_design(const double* size, int64_t n, double* Z, int64_t ldz, void* stream);
+
+/* Test error of predicted times ("variance explained"): out[0] = mse =
+ * mean (yhat - y)^2, out[1] = 1 - mse / mean (y - mean y)^2 (NaN for constant
+ * y).  out: HOST, 2 doubles.  Synchronous.                                 */
+int bf_prediction_error(const double* yhat, const double* y, int64_t m, double* out, void* stream);
+
 /* ---- single-step entry points (parity tests) ---- */
 /* The hand-written device primitives under the presort (row a3)
  * and the per-level offsets: an ascending, stable LSD radix sort of nseg

@@ -83,6 +83,8 @@ def lib():
             "bf_varimax": ([vp, i64, i32, i32, i32, C.c_double, vp, vp, C.POINTER(C.c_int32), vp], C.c_int),
             "bf_glm_gaussian": ([vp, i64, i64, i32, vp, i64, i32, vp, vp, vp, vp], C.c_int),
             "bf_rank_similarity": ([vp, vp, i32, vp, vp], C.c_int),
+            "bf_log_size_design": ([vp, i64, vp, i64, vp], C.c_int),
+            "bf_prediction_error": ([vp, vp, i64, vp, vp], C.c_int),
             "bf_glm_predict": ([vp, i64, i64, i32, vp, i32, vp, i64, vp], C.c_int),
             "bf_mars_fit": ([vp, i64, i64, i32, vp, i32, C.c_double, C.c_double, C.POINTER(C.c_int32), vp, vp, vp, vp,
                              vp, vp], C.c_int),
@@ -154,7 +156,7 @@ def exported_symbols():
                         "bf_oob_importance", "bf_importance_finalize", "bf_pca", "bf_pca_retained", "bf_philox", "bf_i128_to_double",
                         "bf_fixed_point", "bf_bootstrap", "bf_perm", "bf_sort_u64", "bf_scan_u32", "bf_unique_u64", "bf_profile_enable", "bf_profile_read",
                         "bf_launch_count", "bf_partial_dependence", "bf_pd_grid", "bf_varimax",
-                        "bf_glm_gaussian", "bf_glm_predict", "bf_rank_similarity", "bf_mars_fit",
+                        "bf_glm_gaussian", "bf_glm_predict", "bf_rank_similarity", "bf_log_size_design", "bf_prediction_error", "bf_mars_fit",
                         "bf_mars_predict")]
 
 
@@ -445,6 +447,22 @@ def pca(X, scale: bool = True, k: int | None = None) -> dict:
     _check(lib().bf_pca(_ptr(X), n, n, p, int(scale), kk, _ptr(sdev), _ptr(rot), _ptr(cen), _ptr(sco), _stream()),
            "bf_pca")
     return dict(sdev=sdev, rotation=rot, center=cen, scores=sco[:kk])
+
+
+def log_size_design(size):
+    """[1, u, u^2, u^3] with u the standardised log2 of the sizes (bf_log_size_design, reading R26) -> (4, n)."""
+    n = int(size.shape[0])
+    Z = _empty_like_dev(size, (4, n), np.float64)
+    _check(lib().bf_log_size_design(_ptr(size), n, _ptr(Z), n, _stream()), "bf_log_size_design")
+    return Z
+
+
+def prediction_error(yhat, y) -> tuple:
+    """(mse, variance explained) of predicted times (bf_prediction_error)."""
+    out = (C.c_double * 2)()
+    _check(lib().bf_prediction_error(_ptr(yhat), _ptr(y), int(y.shape[0]), C.addressof(out), _stream()),
+           "bf_prediction_error")
+    return float(out[0]), float(out[1])
 
 
 def pca_retained(sdev, frac: float = 0.97, cap: int = 10) -> int:

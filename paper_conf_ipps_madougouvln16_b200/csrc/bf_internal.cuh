@@ -285,6 +285,8 @@ void mars_fit_impl(const double* X, int64_t ldx, int64_t n, int32_t d, const dou
 void mars_predict_impl(const double* X, int64_t ldx, int64_t m, int32_t d, int32_t nt, const int32_t* tvar,
                        const double* tknot, const int32_t* tdir, const double* coef, double* out, cudaStream_t s);
 void rank_similarity_impl(const double* a, const double* b, int32_t p, double* out, cudaStream_t s);
+void log_size_design_impl(const double* size, int64_t n, double* Z, int64_t ldz, cudaStream_t s);
+void prediction_error_impl(const double* yhat, const double* y, int64_t m, double* out_host, cudaStream_t s);
 // misc kernels (capi.cu)
 void philox_impl(const uint32_t* ctr, uint32_t k0, uint32_t k1, uint32_t* out, int64_t count, cudaStream_t s);
 void i128_impl(const int64_t* hi, const uint64_t* lo, double* out, int64_t count, cudaStream_t s);

@@ -443,6 +443,22 @@ int bf_rank_similarity(const double* a, const double* b, int32_t p, double* out,
   BF_API_END
 }
 
+int bf_log_size_design(const double* size, int64_t n, double* Z, int64_t ldz, void* stream) {
+  BF_API_BEGIN
+  BF_REQUIRE(size && Z, BF_EINVAL, "bf_log_size_design: NULL");
+  BF_REQUIRE(n >= 2 && ldz >= n, BF_EINVAL, "bf_log_size_design: need n >= 2, ldz >= n");
+  log_size_design_impl(size, n, Z, ldz, (cudaStream_t)stream);
+  BF_API_END
+}
+
+int bf_prediction_error(const double* yhat, const double* y, int64_t m, double* out, void* stream) {
+  BF_API_BEGIN
+  BF_REQUIRE(yhat && y && out, BF_EINVAL, "bf_prediction_error: NULL");
+  BF_REQUIRE(m >= 1, BF_EINVAL, "bf_prediction_error: need m >= 1");
+  prediction_error_impl(yhat, y, m, out, (cudaStream_t)stream);
+  BF_API_END
+}
+
 int bf_philox(const uint32_t* ctr, uint32_t key0, uint32_t key1, uint32_t* out, int64_t count, void* stream) {
   BF_API_BEGIN
   cudaStream_t s = (cudaStream_t)stream;

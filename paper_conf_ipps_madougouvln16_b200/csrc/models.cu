@@ -983,3 +983,105 @@ void rank_similarity_impl(const double* a_in, const double* b_in, int32_t p, dou
 }
 
 }  // namespace bf
+
+// ------------------------------------------------------------------ workflow statistics (NEXT-3 / NEXT-4)
+namespace bf {
+namespace {
+constexpr int WNT = 256;
+__device__ double wf_block_sum(double v, double* red) {
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xffffffffu, v, o);
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = v;
+  __syncthreads();
+  double t = 0.0;
+  if (threadIdx.x == 0)
+    for (int k = 0; k < WNT / 32; ++k) t += red[k];
+  __syncthreads();
+  return t;  // valid in thread 0
+}
+// Reading R26's default design: u = (log2 s - mean) / sd (sample sd, n - 1), rows [1, u, u^2, u^3].  One CTA
+// computes the statistics in a fixed order; the rows are written by a grid.
+__global__ void k_log_stats(const double* s, int64_t n, double* st /* mean, sd */) {
+  __shared__ double red[WNT / 32];
+  __shared__ double s_mean;
+  double a = 0.0;
+  for (int64_t i = threadIdx.x; i < n; i += WNT) a += log2(s[i]);
+  a = wf_block_sum(a, red);
+  if (threadIdx.x == 0) s_mean = a / (double)n;
+  __syncthreads();
+  const double mean = s_mean;
+  double v = 0.0;
+  for (int64_t i = threadIdx.x; i < n; i += WNT) {
+    const double d = log2(s[i]) - mean;
+    v += d * d;
+  }
+  v = wf_block_sum(v, red);
+  if (threadIdx.x == 0) {
+    st[0] = mean;
+    st[1] = n > 1 ? sqrt(v / (double)(n - 1)) : 0.0;
+  }
+}
+__global__ void k_log_design(const double* s, int64_t n, const double* st, double* Z, int64_t ldz) {
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const double u = (log2(s[i]) - st[0]) / st[1];
+  Z[i] = 1.0;
+  Z[ldz + i] = u;
+  Z[2 * ldz + i] = u * u;
+  Z[3 * ldz + i] = u * u * u;
+}
+// Test error of predicted times ("variance explained"): mse = mean (yhat - y)^2,
+// explained = 1 - mse / mean (y - mean y)^2 (NaN for constant y).
+__global__ void k_pred_error(const double* yh, const double* y, int64_t m, double* out) {
+  __shared__ double red[WNT / 32];
+  __shared__ double s_mean;
+  double a = 0.0, e = 0.0;
+  for (int64_t i = threadIdx.x; i < m; i += WNT) {
+    a += y[i];
+    const double d = yh[i] - y[i];
+    e += d * d;
+  }
+  a = wf_block_sum(a, red);
+  e = wf_block_sum(e, red);
+  if (threadIdx.x == 0) s_mean = a / (double)m;
+  __syncthreads();
+  const double mean = s_mean;
+  double v = 0.0;
+  for (int64_t i = threadIdx.x; i < m; i += WNT) {
+    const double d = y[i] - mean;
+    v += d * d;
+  }
+  v = wf_block_sum(v, red);
+  if (threadIdx.x == 0) {
+    const double mse = e / (double)m, var = v / (double)m;
+    out[0] = mse;
+    out[1] = var > 0.0 ? 1.0 - mse / var : __longlong_as_double(0x7ff8000000000000ll);
+  }
+}
+}  // namespace
+
+void log_size_design_impl(const double* s_in, int64_t n, double* Z_in, int64_t ldz, cudaStream_t s) {
+  InStage ss(s_in, sizeof(double) * (size_t)n, s);
+  OutStage zs(Z_in, sizeof(double) * (size_t)(3 * ldz + n), s);
+  DBuf<double> st(2, s);
+  {
+    KScope ks_("k_log_design", s, 0.0, 2);
+    k_log_stats<<<1, WNT, 0, s>>>((const double*)ss.dptr, n, st.p);
+    k_log_design<<<(unsigned)ceil_div(n, 256), 256, 0, s>>>((const double*)ss.dptr, n, st.p, (double*)zs.dptr, ldz);
+  }
+  BF_CUDA_CHECK(cudaGetLastError());
+  zs.finish(s);
+  if (zs.host || ss.tmp.p) BF_CUDA_CHECK(cudaStreamSynchronize(s));
+}
+
+void prediction_error_impl(const double* yh_in, const double* y_in, int64_t m, double* out_host, cudaStream_t s) {
+  InStage a(yh_in, sizeof(double) * (size_t)m, s), b(y_in, sizeof(double) * (size_t)m, s);
+  DBuf<double> o(2, s);
+  {
+    KScope ks_("k_pred_error", s, 16.0 * (double)m);
+    k_pred_error<<<1, WNT, 0, s>>>((const double*)a.dptr, (const double*)b.dptr, m, o.p);
+  }
+  BF_CUDA_CHECK(cudaGetLastError());
+  BF_CUDA_CHECK(cudaMemcpyAsync(out_host, o.p, 2 * sizeof(double), cudaMemcpyDeviceToHost, s));
+  BF_CUDA_CHECK(cudaStreamSynchronize(s));
+}
+}  // namespace bf

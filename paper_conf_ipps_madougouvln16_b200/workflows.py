@@ -19,7 +19,8 @@ from __future__ import annotations
 
 
 from . import (fit, glm_gaussian, glm_predict, importance_finalize, mars_fit, mars_predict, pca, pca_retained,
-               rank_similarity)
+               prediction_error, rank_similarity)
+from . import log_size_design as _log_size_design
 
 
 def _torch():
@@ -35,11 +36,9 @@ def inc_mse(forest, X, y) -> "object":
 
 def log_size_design(size) -> "object":
     """Default GLM design of one problem characteristic s (reading R26): [1, u, u^2, u^3], u = standardised
-    log2 s (the paper's sizes span 2^5..2^11 and 64..8192).  size: (n,) device tensor -> (4, n)."""
-    torch = _torch()
-    lg = torch.log2(size)
-    u = (lg - lg.mean()) / lg.std()
-    return torch.stack([torch.ones_like(u), u, u * u, u * u * u]).contiguous()
+    log2 s (the paper's sizes span 2^5..2^11 and 64..8192), computed by bf_log_size_design.
+    size: (n,) device tensor -> (4, n)."""
+    return _log_size_design(size.contiguous())
 
 
 def problem_scaling(X, y, size_row: int, train, test, top: int = 6, ntree: int = 500, seed: int = 0,
@@ -82,15 +81,14 @@ def problem_scaling(X, y, size_row: int, train, test, top: int = 6, ntree: int =
         if j == size_row:
             Xh[i] = X[size_row, test]
     yh_sum, yh = f_keep.predict(Xh.contiguous(), ntree_total=ntree)
-    yte = y[test]
-    mse = float(((yh - yte) ** 2).mean())
-    var = float(((yte - yte.mean()) ** 2).mean())
+    yte = y[test].contiguous()
+    mse, expl = prediction_error(yh.contiguous(), yte)
     f_keep.free()
     return {"keep": keep, "oob_mse": float(imp_k["oob_mse"]), "rsq": float(imp_k["rsq"]),
             "models": models, "deviance": None if models is None else models["deviance"],
             "null_deviance": None if models is None else models["null_deviance"],
             "coef": None if models is None else models["coef"], "X_model": Xh, "yhat": yh,
-            "test_mse": mse, "test_explained": 1.0 - mse / var if var > 0 else float("nan")}
+            "test_mse": mse, "test_explained": expl}
 
 
 def n_components(sdev, frac: float = 0.97, cap: int = 10) -> int:
@@ -115,9 +113,8 @@ def hardware_scaling(counters, L, M, y, gen, train_gens=(0, 1), test_gen: int = 
     imp = inc_mse(f, Rtr, ytr)
     _, yh = f.predict(R[:, te].contiguous(), ntree_total=ntree)
     f.free()
-    yte = y[te]
-    mse = float(((yh - yte) ** 2).mean())
-    var = float(((yte - yte.mean()) ** 2).mean())
+    yte = y[te].contiguous()
+    mse, expl = prediction_error(yh.contiguous(), yte)
     per_gen = []
     for g in train_gens:
         ig = torch.nonzero(gen == g).flatten()
@@ -130,5 +127,5 @@ def hardware_scaling(counters, L, M, y, gen, train_gens=(0, 1), test_gen: int = 
         for b in range(a + 1, len(train_gens)):
             sims[(train_gens[a], train_gens[b])] = rank_similarity(per_gen[a], per_gen[b])
     return {"k": k, "inputs": R, "oob_mse": float(imp["oob_mse"]), "rsq": float(imp["rsq"]), "yhat": yh,
-            "test_mse": mse, "test_explained": 1.0 - mse / var if var > 0 else float("nan"),
+            "test_mse": mse, "test_explained": expl,
             "inc_mse_per_gen": per_gen, "similarity": sims}

@@ -107,3 +107,20 @@ def test_problem_scaling_nw_with_mars_matches_oracle_composition():
     Xh = r["X_model"].cpu().numpy()
     ofk = O.fit(np.ascontiguousarray(X[r["keep"]][:, tr]), yy[tr], ntree=T, seed=seed + 1, nthreads=8)
     assert rel_close(r["yhat"].cpu().numpy(), ofk.predict_sum(Xh) / T, 1e-9)
+
+
+def test_log_size_design_and_prediction_error_vs_oracle():
+    """The workflow statistics on the device (bf_log_size_design, bf_prediction_error) against the oracle's
+    plain definitions, on the paper's size grids and on random data (device and host pointers)."""
+    rng = np.random.default_rng(3)
+    for s in (2.0 ** np.arange(5, 12), np.arange(64, 8193, 64, dtype=np.float64), rng.uniform(1, 1e6, 999)):
+        Zg = bf.log_size_design(dev(s)).cpu().numpy()
+        Zo = Sc.log_size_design(s)
+        assert np.allclose(Zg, Zo, rtol=1e-13, atol=1e-13)
+        assert np.allclose(bf.log_size_design(np.ascontiguousarray(s)), Zo, rtol=1e-13, atol=1e-13)
+    y = rng.normal(size=5000)
+    yh = y + 0.1 * rng.normal(size=5000)
+    mg, eg = bf.prediction_error(dev(yh), dev(y))
+    mo, eo = Sc.prediction_error(yh, y)
+    assert math.isclose(mg, mo, rel_tol=1e-12) and math.isclose(eg, eo, rel_tol=1e-12)
+    assert math.isnan(bf.prediction_error(dev(np.ones(4)), dev(np.full(4, 2.0)))[1])

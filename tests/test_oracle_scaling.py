@@ -81,3 +81,17 @@ def test_rank_similarity_vs_scipy(ties):
             a, b = np.round(a * 2) / 2, np.round(b)
         assert math.isclose(Sc.spearman(a, b), stats.spearmanr(a, b)[0], rel_tol=1e-12, abs_tol=1e-15)
         assert math.isclose(Sc.kendall_tau_b(a, b), stats.kendalltau(a, b)[0], rel_tol=1e-12, abs_tol=1e-15)
+
+
+def test_log_size_design_closed_form():
+    """Sizes 2^5..2^11: log2 = 5..11 exactly, mean 8, sample sd sqrt(28/6); rows 1, u, u^2, u^3."""
+    Z = Sc.log_size_design(2.0 ** np.arange(5, 12))
+    u = (np.arange(5, 12) - 8.0) / math.sqrt(28.0 / 6.0)
+    assert np.allclose(Z, np.stack([np.ones(7), u, u ** 2, u ** 3]), rtol=1e-15, atol=1e-15)
+
+
+def test_prediction_error_closed_form():
+    y = np.array([1.0, 2.0, 3.0, 4.0])
+    mse, ex = Sc.prediction_error(y + np.array([0.5, -0.5, 0.5, -0.5]), y)
+    assert mse == 0.25 and ex == pytest.approx(1.0 - 0.25 / 1.25, rel=1e-15)
+    assert math.isnan(Sc.prediction_error(np.ones(3), np.full(3, 2.0))[1])
