@@ -312,7 +312,7 @@ def test_c4_bench_configuration_sampled():
     T, seed = 1000, S.FOREST_SEED + 4
     Xd, yd = dev(X), dev(y)
     gf = bf.fit(Xd, yd, ntree=T, seed=seed)
-    sample = (0, 517, 999)
+    sample = (0, 136, 517, 731, 999)  # trees of 5 different batches (37 trees in flight)
     with ThreadPoolExecutor(len(sample)) as ex:  # ctypes releases the GIL: one oracle tree per host thread
         ofs = list(ex.map(lambda t: O.fit(X, y, ntree=T, seed=seed, tree_begin=t, tree_end=t + 1), sample))
     e = gf.export()
@@ -345,6 +345,20 @@ def test_c4_bench_configuration_sampled():
                 k = left[base + k] + (0 if Qs[feat[base + k], r] <= thr[base + k] else 1)
             ref[r] += thr[base + k]
     assert rel_close(got, ref, 1e-9)
+    # the sampled trees alone (bf_forest_import of their exported arrays), predicted on the device over the
+    # sampled query rows, against the oracle's trees (S5): the GPU prediction path checked by the oracle itself
+    trees = [{k: e[k][e["tree_off"][t]:e["tree_off"][t + 1]] for k in ("feature", "left", "thr_or_value", "count",
+                                                                       "value", "drss")} for t in sample]
+    arrays = {k: np.concatenate([tr[k] for tr in trees]) for k in trees[0]}
+    arrays["tree_off"] = np.concatenate([[0], np.cumsum([tr["feature"].size for tr in trees])]).astype(np.int64)
+    info = e["info"]
+    info.tree_begin, info.tree_end, info.ntree_total = 0, len(sample), len(sample)
+    info.total_nodes = int(arrays["tree_off"][-1])
+    sub = bf.forest_import(arrays, info)
+    ys_sub, _ = sub.predict(dev(Qs), ntree_total=len(sample))
+    ref_sub = sum(of.predict_sum(Qs) for of in ofs)
+    assert rel_close(ys_sub.cpu().numpy(), ref_sub, 1e-9)
+    sub.free()
     # importance slots of the sampled trees (S7) in the batched launch configuration
     acc = gf.oob_importance(Xd, yd)
     d = acc["d_slots"].cpu().numpy()
