@@ -734,6 +734,33 @@ __device__ __forceinline__ void key_bounds(double nkd, double Skd, int64_t nk, i
   gL = lo * lo * r * (1.0 - 9.5367431640625e-07);
 }
 
+// The same screen in fp32 on t = sqrt(g) = |D| / sqrt(n_l n_r) (monotone in the key, < 2^84 so no overflow):
+// tL <= t <= tU rigorously.  a = RN32(n_k RN32(S_l)), b = RN32(n_l RN32(S_k)) each lie within 2^-23 (1 + 2^-23)
+// of n_k S_l, n_l S_k, and RN32|a - b| within 2^-24 more, so |D| is within E = (|a| + |b|) 2^-21 of
+// RN32|a - b|; the directed roundings and the (1 +- 2^-20) factors absorb rsqrtf's error (< 2^-22) and make
+// tU >= t (1 + 2^-21), tL <= t (1 - 2^-21): a candidate screened out (tU < M) has a key below every key
+// that reaches M by a relative 2^-19, so it can neither beat nor tie it.
+__device__ __forceinline__ void key_bounds_t(float nkf, float Skf, int64_t nk, int32_t nl, int64_t Sl, float& tL,
+                                             float& tU) {
+  const float a = nkf * __ll2float_rn(Sl), b = __int2float_rn(nl) * Skf;
+  const float d = fabsf(a - b);
+  const float E = (fabsf(a) + fabsf(b)) * 4.76837158203125e-07f;  // 2^-21
+  const float hi = __fadd_ru(d, E), lo = fmaxf(__fsub_rd(d, E), 0.0f);
+  const float nlf = __int2float_rn(nl), nrf = __ll2float_rn(nk - nl);  // exact: < 2^24
+  tU = __fmul_ru(__fmul_ru(hi, rsqrtf(__fmul_rd(nlf, nrf))), 1.00000095367431640625f);  // (1 + 2^-20)
+  tL = __fmul_rd(__fmul_rd(lo, rsqrtf(__fmul_ru(nlf, nrf))), 0.99999904632568359375f);  // (1 - 2^-20)
+}
+// A lower bound of t for an exact key g (the running best): sqrt(g) (1 - 2^-20), rounded down; -1 for none.
+__device__ __forceinline__ float key_t_lower(double g) {
+  return g >= 0.0 ? __fmul_rd(__fsqrt_rd(__double2float_rd(g)), 0.99999904632568359375f) : -1.0f;
+}
+// Warp max of non-negative floats (-1 = none) through their bit patterns.
+__device__ __forceinline__ float warp_max_t(float v) {
+  const uint32_t k = v >= 0.0f ? __float_as_uint(v) + 1u : 0u;
+  const uint32_t m = __reduce_max_sync(0xffffffffu, k);
+  return m ? __uint_as_float(m - 1u) : -1.0f;
+}
+
 // ------------------------------------------------------------------ tree-affine item kernels (global phase v6)
 // Nodes of a level are ordered by tree, so each tree's items (node, feature)
 // form a contiguous range.  A CTA is bound to one tree and owns whole items
@@ -843,7 +870,7 @@ __global__ void __launch_bounds__(SNT, 4) k_split_scan_tree(TScanArgs g) {
   __shared__ uint64_t bar[2];
   __shared__ int32_t smc[NW];
   __shared__ int64_t sms[NW];
-  __shared__ double smL[NW];
+  __shared__ float smL[NW];
   __shared__ WBest swb[NW];
   __shared__ int s_off[2];
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
@@ -893,7 +920,7 @@ __global__ void __launch_bounds__(SNT, 4) k_split_scan_tree(TScanArgs g) {
       if (tid == 0 && nitem < i_hi) issue(nitem, nunit, cur ^ 1);
       const int a = nd.a, u0 = unit * TUNIT, cnt = min(TUNIT, a - u0);
       const int64_t nk = nd.n, Sk = nd.S;
-      const double nkd = (double)nk, Skd = (double)Sk;
+      const float nkf = __ll2float_rn(nk), Skf = __ll2float_rn(Sk);  // nk < 2^24: exact
       mbar_wait(&bar[cur], phase[cur]);
       phase[cur] ^= 1u;
       const uint64_t* buf = bufs + (size_t)cur * (TUNIT + 4) + s_off[cur];
@@ -949,9 +976,9 @@ __global__ void __launch_bounds__(SNT, 4) k_split_scan_tree(TScanArgs g) {
         totc += c;
         tots += v;
       }
-      // bounds of every boundary; the thread's best lower bound
+      // bounds of every boundary (fp32, t = sqrt(key) space); the thread's best lower bound
       float gUf[TSV];
-      double mL = ib.g;
+      float mL = key_t_lower(ib.g);
       {
         int32_t prc = prc0;
         int64_t prs = prs0;
@@ -963,25 +990,23 @@ __global__ void __launch_bounds__(SNT, 4) k_split_scan_tree(TScanArgs g) {
             prc += wq[q];
             prs += wy[q];
             if (u0 + j + 1 < a && rk[q] != rk[q + 1]) {
-              double gL, gU;
-              key_bounds(nkd, Skd, nk, prc, prs, gL, gU);
-              mL = fmax(mL, gL);
-              gUf[q] = __double2float_ru(gU);
+              float tL, tU;
+              key_bounds_t(nkf, Skf, nk, prc, prs, tL, tU);
+              mL = fmaxf(mL, tL);
+              gUf[q] = tU;
             }
           }
         }
       }
       // S2: block max of the lower bounds -> M
       {
-        const uint64_t kb = gkey(mL);
-        const uint32_t hi = __reduce_max_sync(0xffffffffu, (uint32_t)(kb >> 32));
-        const uint32_t lo = __reduce_max_sync(0xffffffffu, ((uint32_t)(kb >> 32) == hi) ? (uint32_t)kb : 0u);
-        if (lane == 0) smL[wid] = (hi | lo) ? __longlong_as_double((long long)((((uint64_t)hi << 32) | lo) - 1ull)) : -1.0;
+        const float wm = warp_max_t(mL);
+        if (lane == 0) smL[wid] = wm;
       }
       __syncthreads();
-      double M = -1.0;
+      float M = -1.0f;
 #pragma unroll
-      for (int k = 0; k < NW; ++k) M = fmax(M, smL[k]);
+      for (int k = 0; k < NW; ++k) M = fmaxf(M, smL[k]);
       // exact keys where the upper bound reaches M
       WBest tb;
       tb.g = -1.0;
@@ -999,7 +1024,7 @@ __global__ void __launch_bounds__(SNT, 4) k_split_scan_tree(TScanArgs g) {
           if (j < cnt) {
             prc += wq[q];
             prs += wy[q];
-            if ((double)gUf[q] >= M && gUf[q] >= 0.0f) {
+            if (gUf[q] >= M && gUf[q] >= 0.0f) {
               const double gk = split_key_call(nk, Sk, prc, prs);
               const uint32_t ra = rk[q];
               if (rec_better(gk, ra, tb.g, tb.rank)) {
@@ -1798,7 +1823,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         const int f = feats_all[li * p + (it - li * g.mtry)];
         const uint32_t* seg = list + (size_t)f * a0 + nd.lo;
         const int64_t nk = nd.n, Sk = nd.S;
-        const double nkd = (double)nk, Skd = (double)Sk;
+        const float nkf = __ll2float_rn(nk), Skf = __ll2float_rn(Sk);
           double lg = -1.0;
         uint32_t lrk = 0xffffffffu, lra = 0, lrb = 0;
         int lpos = -1, lnl = 0;
@@ -1818,7 +1843,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         }
         const int32_t cw0 = warp_incl_scan(rw, lane) - rw;
         const int64_t cs0 = warp_incl_scan(rsum, lane) - rsum;
-        double mL = -1.0, mU = -1.0, u2 = -1.0;  // as in the tiny path: largest / second largest upper bound
+        float mL = -1.0f, mU = -1.0f, u2 = -1.0f;  // fp32 t-space screen; largest / second largest upper bound
         int bi = -1;
         int32_t bcw = 0;
         int64_t bcs = 0;
@@ -1831,9 +1856,9 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
             cw += wl[lr];
             cs += wy[lr];
             if (i + 1 < aN && (seg[i + 1] >> 16) != (e >> 16)) {
-              double gL, gU;
-              key_bounds(nkd, Skd, nk, cw, cs, gL, gU);
-              mL = fmax(mL, gL);
+              float gL, gU;
+              key_bounds_t(nkf, Skf, nk, cw, cs, gL, gU);
+              mL = fmaxf(mL, gL);
               if (gU > mU) {
                 u2 = mU;
                 mU = gU;
@@ -1841,19 +1866,13 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
                 bcw = cw;
                 bcs = cs;
               } else {
-                u2 = fmax(u2, gU);
+                u2 = fmaxf(u2, gU);
               }
             }
           }
         }
-        double M;
-        {
-          const uint64_t kb = gkey(mL);
-          const uint32_t hi = __reduce_max_sync(0xffffffffu, (uint32_t)(kb >> 32));
-          const uint32_t lo = __reduce_max_sync(0xffffffffu, ((uint32_t)(kb >> 32) == hi) ? (uint32_t)kb : 0u);
-          M = (hi | lo) ? __longlong_as_double((long long)((((uint64_t)hi << 32) | lo) - 1ull)) : -1.0;
-        }
-        if (mU >= M && mU >= 0.0 && u2 < M) {  // a single candidate item on this lane
+        const float M = warp_max_t(mL);
+        if (mU >= M && mU >= 0.0f && u2 < M) {  // a single candidate item on this lane
           const uint32_t e = seg[bi], en = seg[bi + 1];
           const double gk = split_key(nk, Sk, bcw, bcs);
           if (rec_better(gk, e >> 16, lg, lrk)) {
@@ -1865,7 +1884,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
             lnl = bcw;
             lSl = bcs;
           }
-        } else if (mU >= M && mU >= 0.0) {
+        } else if (mU >= M && mU >= 0.0f) {
           int32_t cw = cw0;
           int64_t cs = cs0;
           for (int i = i0; i < i1; ++i) {
@@ -1875,8 +1894,8 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
             if (i + 1 < aN) {
               const uint32_t en = seg[i + 1];
               if ((en >> 16) != (e >> 16)) {
-                double gL, gU;
-                key_bounds(nkd, Skd, nk, cw, cs, gL, gU);
+                float gL, gU;
+                key_bounds_t(nkf, Skf, nk, cw, cs, gL, gU);
                 if (gU >= M) {
                   const double gk = split_key(nk, Sk, cw, cs);
                   if (rec_better(gk, e >> 16, lg, lrk)) {
@@ -2136,7 +2155,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       warp_draw_mtry(g.seed, t, nd.key, p, g.mtry, mind, feats, lane);
       const long long c1_ = g.stats ? clock64() : 0;
       const int64_t nk = nd.n, Sk = nd.S;
-      const double nkd = (double)nk, Skd = (double)Sk;
+      const float nkf = __ll2float_rn(nk), Skf = __ll2float_rn(Sk);
       uint32_t* stg = temp;  // the medium levels' partition buffer (>= TGRP * TINY entries)
       const unsigned lt = (1u << lane) - 1u;
       // lane-local best over all (feature, boundary) items: key g, tie = (feature << 16 | rank)
@@ -2246,7 +2265,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         const long long gq2 = g.stats ? clock64() : 0;
         // the lane's largest upper bound mU with its item (bi, prefix bcw / bcs) and the second largest u2: when
         // u2 < M only item bi can reach the exact-key pass, which then evaluates it directly
-        double mL = lg, mU = -1.0, u2 = -1.0;
+        float mL = key_t_lower(lg), mU = -1.0f, u2 = -1.0f;  // fp32 t-space screen
         int bi = -1;
         int32_t bcw = 0;
         int64_t bcs = 0;
@@ -2264,9 +2283,9 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
             cw += wl[lr];
             cs += wy[lr];
             if (jj + 1 < an && (stg[i + 1] >> 16) != (e >> 16)) {
-              double gL, gU;
-              key_bounds(nkd, Skd, nk, cw, cs, gL, gU);
-              mL = fmax(mL, gL);
+              float gL, gU;
+              key_bounds_t(nkf, Skf, nk, cw, cs, gL, gU);
+              mL = fmaxf(mL, gL);
               if (gU > mU) {
                 u2 = mU;
                 mU = gU;
@@ -2274,22 +2293,16 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
                 bcw = cw;
                 bcs = cs;
               } else {
-                u2 = fmax(u2, gU);
+                u2 = fmaxf(u2, gU);
               }
             }
             if (++jj == an) jj = 0;
           }
         }
         const long long gq3 = g.stats ? clock64() : 0;
-        double M;
-        {
-          const uint64_t kb = gkey(mL);
-          const uint32_t hi = __reduce_max_sync(0xffffffffu, (uint32_t)(kb >> 32));
-          const uint32_t lo = __reduce_max_sync(0xffffffffu, ((uint32_t)(kb >> 32) == hi) ? (uint32_t)kb : 0u);
-          M = (hi | lo) ? __longlong_as_double((long long)((((uint64_t)hi << 32) | lo) - 1ull)) : -1.0;
-        }
+        const float M = warp_max_t(mL);
         const long long gq4 = g.stats ? clock64() : 0;
-        if (mU >= M && mU >= 0.0 && u2 < M) {  // a single candidate item on this lane
+        if (mU >= M && mU >= 0.0f && u2 < M) {  // a single candidate item on this lane
           const uint32_t e = stg[bi], en = stg[bi + 1];
           const double gk = split_key(nk, Sk, bcw, bcs);
           const uint32_t tie = ((uint32_t)feats[s0 + bi / an] << 16) | (e >> 16);
@@ -2301,7 +2314,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
             lra = e & 0xffffu;
             lrb = en & 0xffffu;
           }
-        } else if (mU >= M && mU >= 0.0) {
+        } else if (mU >= M && mU >= 0.0f) {
           int jj = jj0, sl = slot0;
           int32_t cw = cw0;
           int64_t cs = cs0;
@@ -2316,8 +2329,8 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
             if (jj + 1 < an) {
               const uint32_t en = stg[i + 1];
               if ((en >> 16) != (e >> 16)) {
-                double gL, gU;
-                key_bounds(nkd, Skd, nk, cw, cs, gL, gU);
+                float gL, gU;
+                key_bounds_t(nkf, Skf, nk, cw, cs, gL, gU);
                 if (gU >= M) {
                   const double gk = split_key(nk, Sk, cw, cs);
                   const uint32_t tie = ((uint32_t)feats[s0 + sl] << 16) | (e >> 16);
