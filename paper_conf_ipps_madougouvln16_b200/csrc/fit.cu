@@ -1390,8 +1390,7 @@ __global__ void __launch_bounds__(NT) k_dest_bits(DestArgs g, uint32_t* sideb, i
     if (j < nd.a) {
       const uint32_t row = e_row(ev[u]);
       const int s = j > sp.pos;
-      if (s) atomicOr(&sb[row >> 5], 1u << (row & 31));
-      else atomicAnd(&sb[row >> 5], ~(1u << (row & 31)));
+      if (s) atomicOr(&sb[row >> 5], 1u << (row & 31));  // the level's bitmap starts cleared
       const double v = __dmul_rn((double)e_w(ev[u]), yv[u]);
       if (s) accr += v;
       else accl += v;
@@ -3028,6 +3027,8 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
         // ---- a9/a10 goes-right flags and child values over pieces of the winning segments
         piece_setup(1, N, 1, nc, split.p, child.p, pcnt.p, poff.p, pmap.p, ptot.p, s);
         BF_CUDA_CHECK(cudaMemsetAsync(csum.p, 0, sizeof(double) * 2 * (size_t)N, s));
+        // goes-right bitmap cleared per level (n/8 bytes per tree), so only right-going rows need an atomic
+        BF_CUDA_CHECK(cudaMemsetAsync(sideb.p, 0, sizeof(uint32_t) * (size_t)Bc * nw, s));
         {
           DestArgs ga{nc, split.p, Ec, y, n, side.p, poff.p, pmap.p, ptot.p, csum.p};
           KScope ks_("k_dest_bits", s, 0.0);
