@@ -16,6 +16,7 @@ for spec in "k_subtree 0" "k_partition_tree 4" "k_split_scan_tree 4" "k_predict8
   timeout 900 ncu --set full $X --clock-control none --import-source on -k regex:$1 -s $2 -c 1 -f -o $O/prof_$1 python $B > $O/ncu_$1.log 2>&1
   echo "$1 rc=$?"
   python tools/ncu_summary.py full $O/prof_$1.ncu-rep $O/full_$1 > /dev/null 2>&1
+  ncu -i $O/prof_$1.ncu-rep --page details --print-details all > $O/details_$1.txt 2>&1
   head -3 $O/full_$1.txt
 done
 ls $O/*.ncu-rep | grep -v k_subtree | xargs rm -f
