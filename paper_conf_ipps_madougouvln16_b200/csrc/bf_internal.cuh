@@ -222,6 +222,12 @@ struct bf_forest {
   uint2* d_nodes8 = nullptr;
   uint32_t* d_roots8 = nullptr;  // per tree: global root id | 1<<31 if the tree is a single leaf
   int nodes8_state = 0;
+  // Two-level 32-byte groups (predict.cu g32_get, built on first use; same states as nodes8_state): a group holds
+  // an internal node at even depth and its two children, so one 256-bit load decides two levels of a walk.
+  ulonglong4* d_g32 = nullptr;
+  uint32_t* d_g32_root = nullptr;  // per tree: global slot of the root | ROOT_LEAF if the tree is a single leaf
+  std::vector<int64_t> g32_off;    // host: first slot of each tree, ntrees + 1
+  int g32_state = 0;
   int device = 0;
   cudaStream_t stream = nullptr;       // stream the forest's memory was allocated on (freed stream-ordered on it)
   mutable bool foreign_stream = false;  // some call used the forest on another stream (free waits for the device)
@@ -255,6 +261,7 @@ void bootstrap_impl(uint64_t seed, int32_t t0, int32_t ntrees, int64_t n, int64_
                     int32_t* w, cudaStream_t s);
 // predict.cu
 const uint2* nodes8_get(bf_forest* f, cudaStream_t s);  // NULL if not representable
+const ulonglong4* g32_get(bf_forest* f, cudaStream_t s);  // NULL if not representable
 void predict_impl(const bf_forest* f, const double* Xq, int64_t ldq, int64_t m, double* yhat_sum, double* yhat,
                   int32_t ntree_total, cudaStream_t s);
 void pd_grid_impl(const double* x, int64_t n, int32_t n_pt, double* grid, int32_t* G_host, cudaStream_t s);
@@ -262,6 +269,8 @@ void partial_dependence_impl(const bf_forest* f, const double* X, int64_t ldx, i
                              const double* grid, int32_t G, double* pd_sum, double* pd, int32_t ntree_total,
                              cudaStream_t s);
 // importance.cu
+// row-major RN_f32 copy of a column-major fp64 matrix (stride xfs floats, a multiple of 4, zero padded)
+void xf_rows_impl(const double* X, int64_t ldx, int64_t n, int p, float* Xf, int xfs, cudaStream_t s);
 void oob_importance_impl(const bf_forest* f, const double* X, int64_t ldx, const double* y, int64_t n, int32_t p,
                          const bf_oob_accum& acc, cudaStream_t s);
 void importance_finalize_impl(const double* d_slots, const double* npur_slots, const double* oob_sum,

@@ -119,6 +119,11 @@ void forest_release(bf_forest* f) {
   f->d_nodes8 = nullptr;
   f->d_roots8 = nullptr;
   f->nodes8_state = 0;
+  if (f->d_g32) dev_free(f->d_g32, s);
+  if (f->d_g32_root) dev_free(f->d_g32_root, s);
+  f->d_g32 = nullptr;
+  f->d_g32_root = nullptr;
+  f->g32_state = 0;
   f->d_nodes = nullptr;
 }
 

@@ -1450,15 +1450,62 @@ struct MNode {  // medium node (a > TINY) of a subtree level
   uint64_t keyl, keyr;
   int32_t kind[2];
 };
-struct TNode {  // tiny node: mask over the rows of its tiny root [rlo, rlo+ra)
+template <int NWD>
+struct TNodeT {  // tiny node: mask (NWD 64-bit words) over the rows of its tiny root [rlo, rlo+ra)
   int32_t rlo, ra;
-  uint64_t mask;
+  uint64_t mask[NWD];
   int32_t id;
   int32_t n;
   int64_t S;
   uint64_t key;
   double value;  // node value (S4.7): the warp that grows the node writes its whole record
 };
+
+// Row masks of tiny nodes (bit i = the row at feature-0 position i of the tiny root), 1 or 2 words; no dynamic
+// indexing of the word array (it stays in registers).
+template <int NWD>
+__device__ __forceinline__ int m_popc(const uint64_t (&m)[NWD]) {
+  int c = __popcll(m[0]);
+  if constexpr (NWD == 2) c += __popcll(m[1]);
+  return c;
+}
+template <int NWD>
+__device__ __forceinline__ bool m_test(const uint64_t (&m)[NWD], int i) {
+  if constexpr (NWD == 1) return (m[0] >> i) & 1ull;
+  else return ((i < 64 ? m[0] : m[1]) >> (i & 63)) & 1ull;
+}
+template <int NWD>
+__device__ __forceinline__ void m_set(uint64_t (&m)[NWD], int i) {
+  if constexpr (NWD == 1) m[0] |= 1ull << i;
+  else {
+    const uint64_t b = 1ull << (i & 63);
+    m[0] |= i < 64 ? b : 0ull;
+    m[1] |= i < 64 ? 0ull : b;
+  }
+}
+template <int NWD>
+__device__ __forceinline__ void m_full(uint64_t (&m)[NWD], int a) {  // bits [0, a)
+  m[0] = a >= 64 ? ~0ull : ((1ull << a) - 1ull);
+  if constexpr (NWD == 2) m[1] = a >= 128 ? ~0ull : (a <= 64 ? 0ull : ((1ull << (a - 64)) - 1ull));
+}
+// index of the lowest set bit, which is cleared (0 for an empty mask)
+template <int NWD>
+__device__ __forceinline__ int m_pop(uint64_t (&m)[NWD]) {
+  if constexpr (NWD == 1) {
+    const int b = __ffsll((long long)m[0]) - 1;
+    m[0] &= m[0] - 1;
+    return b < 0 ? 0 : b;
+  } else {
+    const bool lo = m[0] != 0;
+    const uint64_t v = lo ? m[0] : m[1];
+    const int b = __ffsll((long long)v) - 1;
+    const uint64_t v2 = v & (v - 1);
+    m[0] = lo ? v2 : m[0];
+    m[1] = lo ? m[1] : v2;
+    return b < 0 ? 0 : b + (lo ? 0 : 64);
+  }
+}
+
 struct WRec {  // best candidate found by one warp for its share of a node's features
   double g;
   int32_t f;
@@ -1471,18 +1518,25 @@ struct WRec {  // best candidate found by one warp for its share of a node's fea
 __host__ __device__ inline size_t align16(size_t x) { return (x + 15) & ~size_t(15); }
 __host__ __device__ inline int max_medium(int A) { return A / (TINY + 1) + 2; }
 __host__ __device__ inline int sub_temp(int A) { return A > TGRP * TINY ? A : TGRP * TINY; }
+// The per-warp scratch area (medium partition temp / tiny staging of the TV = 0 path); in the tiny phase of the
+// TV = 1 path it holds the position table ppos (p x A bytes), so it is sized for both.
+__host__ __device__ inline size_t sub_temp_bytes(int A, int p) {
+  const size_t a = (size_t)SUB_NW * sub_temp(A) * 4, b = (size_t)p * A;
+  return a > b ? a : b;
+}
 static_assert(HSLOTS * 6 <= SUB_NW * TGRP * TINY * 4, "the load-phase hash table must fit the scratch area");
 
-__host__ __device__ inline size_t subtree_smem(int A, int p) {
+__host__ __device__ inline size_t subtree_smem(int A, int p, int tt = 64) {
   size_t s = 0;
   s += align16((size_t)p * A * 4);                    // list
-  s += align16((size_t)SUB_NW * sub_temp(A) * 4);     // per-warp partition temp / tiny staging
+  s += align16(sub_temp_bytes(A, p));                 // per-warp partition temp / tiny staging / ppos
   s += align16((size_t)A * 8) * 2;                    // wy, w*y
   s += align16((size_t)A * 4) * 2;                    // w, global row
   s += align16((size_t)A) * 2;                        // side, row index inside its tiny root
   s += align16((size_t)2 * A * sizeof(SRec));         // node records
+  s += align16((size_t)2 * A * 2);                    // per record: tiny root of a deferred value (or 0xffff)
   s += align16((size_t)2 * max_medium(A) * sizeof(MNode));
-  s += align16((size_t)(A + MAXR) * sizeof(TNode));   // tiny work queue
+  s += align16((size_t)(A + MAXR) * (tt > 64 ? sizeof(TNodeT<2>) : sizeof(TNodeT<1>)));   // tiny work queue
   s += align16((size_t)(A + MAXR) * 4);               // its ready flags
   s += align16((size_t)SUB_NW * p * 2) * 2;           // Fisher-Yates scratch, drawn features
   s += align16((size_t)SUB_NW * sizeof(WRec));
@@ -1518,6 +1572,23 @@ struct SubArgs {
 // from the j values of the earlier draws (kept in shared memory).
 __device__ __forceinline__ void warp_draw_mtry(uint64_t seed, uint32_t t, uint64_t key, int p, int mtry, int16_t* jbuf,
                                                int16_t* feats, int lane) {
+  if (mtry <= 32) {  // one draw per lane; the earlier draws' j come by shuffle (no shared-memory round trips)
+    int j = 0;
+    if (lane < mtry) {
+      uint64_t u0, u1;
+      philox_u64x2(seed, (uint32_t)key, (uint32_t)(key >> 32), t, 0x20000000u | (uint32_t)(lane >> 1), u0, u1);
+      j = (int)mulhi64((lane & 1) ? u1 : u0, (uint64_t)(p - lane));
+    }
+    int x = j;
+#pragma unroll 4
+    for (int k = mtry - 2; k >= 0; --k) {  // lane i applies k = i-1 .. 0 (warp-uniform loop)
+      const int jk = __shfl_sync(0xffffffffu, j, k), lk = p - 1 - k;
+      if (k < lane) x = (x == jk) ? lk : ((x == lk) ? jk : x);
+    }
+    if (lane < mtry) feats[lane] = (int16_t)x;
+    __syncwarp();
+    return;
+  }
   for (int i0 = 0; i0 < mtry; i0 += 32) {
     const int i = i0 + lane;
     if (i < mtry) {
@@ -1562,13 +1633,16 @@ __device__ __forceinline__ T a_get(T& x) {
   return blk_ref<T>(x).fetch_or(T(0), cuda::memory_order_relaxed);
 }
 
-__device__ __forceinline__ void tq_push(TNode* q, int32_t* ready, int* alloc, int* pending, const TNode& c) {
+template <int NWD>
+__device__ __forceinline__ void tq_push(TNodeT<NWD>* q, int32_t* ready, int* alloc, int* pending,
+                                        const TNodeT<NWD>& c) {
   atomicAdd(pending, 1);
   const int idx = atomicAdd(alloc, 1);
-  TNode& e = q[idx];
+  TNodeT<NWD>& e = q[idx];
   a_put<int32_t>(e.rlo, c.rlo);
   a_put<int32_t>(e.ra, c.ra);
-  a_put<u64>(*(u64*)&e.mask, (u64)c.mask);
+#pragma unroll
+  for (int w = 0; w < NWD; ++w) a_put<u64>(*(u64*)&e.mask[w], (u64)c.mask[w]);
   a_put<int32_t>(e.id, c.id);
   a_put<int32_t>(e.n, c.n);
   a_put<u64>(*(u64*)&e.S, (u64)c.S);
@@ -1577,12 +1651,14 @@ __device__ __forceinline__ void tq_push(TNode* q, int32_t* ready, int* alloc, in
   blk_ref<int32_t>(ready[idx]).exchange(1, cuda::memory_order_release);
 }
 
-__device__ __forceinline__ TNode tq_read(TNode* q, int idx) {  // after an acquire of ready[idx] (or a barrier)
-  TNode& e = q[idx];
-  TNode c;
+template <int NWD>
+__device__ __forceinline__ TNodeT<NWD> tq_read(TNodeT<NWD>* q, int idx) {  // after an acquire of ready[idx] (or a barrier)
+  TNodeT<NWD>& e = q[idx];
+  TNodeT<NWD> c;
   c.rlo = a_get<int32_t>(e.rlo);
   c.ra = a_get<int32_t>(e.ra);
-  c.mask = (uint64_t)a_get<u64>(*(u64*)&e.mask);
+#pragma unroll
+  for (int w = 0; w < NWD; ++w) c.mask[w] = (uint64_t)a_get<u64>(*(u64*)&e.mask[w]);
   c.id = a_get<int32_t>(e.id);
   c.n = a_get<int32_t>(e.n);
   c.S = (int64_t)a_get<u64>(*(u64*)&e.S);
@@ -1591,11 +1667,13 @@ __device__ __forceinline__ TNode tq_read(TNode* q, int idx) {  // after an acqui
   return c;
 }
 
-__device__ __forceinline__ TNode tq_bcast(const TNode& c) {  // lane 0's entry to the whole warp
-  TNode r;
+template <int NWD>
+__device__ __forceinline__ TNodeT<NWD> tq_bcast(const TNodeT<NWD>& c) {  // lane 0's entry to the whole warp
+  TNodeT<NWD> r;
   r.rlo = __shfl_sync(0xffffffffu, c.rlo, 0);
   r.ra = __shfl_sync(0xffffffffu, c.ra, 0);
-  r.mask = __shfl_sync(0xffffffffu, c.mask, 0);
+#pragma unroll
+  for (int w = 0; w < NWD; ++w) r.mask[w] = __shfl_sync(0xffffffffu, c.mask[w], 0);
   r.id = __shfl_sync(0xffffffffu, c.id, 0);
   r.n = __shfl_sync(0xffffffffu, c.n, 0);
   r.S = __shfl_sync(0xffffffffu, c.S, 0);
@@ -1604,14 +1682,19 @@ __device__ __forceinline__ TNode tq_bcast(const TNode& c) {  // lane 0's entry t
   return r;
 }
 
+// TV: tiny-node search (0 staged warp items, 1 lane per drawn feature); TT: largest tiny root (64 or 128 rows)
+template <int TV, int TT>
 __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
+  static_assert(TT == 64 || (TT == 128 && TV == 1), "tiny roots of 128 rows need the lane-per-feature search");
+  constexpr int NWD = TT / 64;
+  using TN = TNodeT<NWD>;
   extern __shared__ __align__(16) unsigned char smem[];
   const int A = g.A, p = g.p, MM = max_medium(A);
   unsigned char* ptr = smem;
   uint32_t* list = (uint32_t*)ptr;
   ptr += align16((size_t)p * A * 4);
   uint32_t* temp_all = (uint32_t*)ptr;
-  ptr += align16((size_t)SUB_NW * sub_temp(A) * 4);
+  ptr += align16(sub_temp_bytes(A, p));
   int64_t* wy = (int64_t*)ptr;
   ptr += align16((size_t)A * 8);
   double* wyd = (double*)ptr;
@@ -1626,11 +1709,16 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   ptr += align16((size_t)A);
   SRec* recs = (SRec*)ptr;
   ptr += align16((size_t)2 * A * sizeof(SRec));
+  // DEFER (lane-per-feature search, 64-row tiny roots): the value of a tiny-phase record is computed at the flush
+  // from its row mask (held in the record's value field) over its tiny root's rows, off the critical path
+  constexpr bool DEFER = TV == 1 && NWD == 1;
+  uint16_t* rdef = (uint16_t*)ptr;
+  ptr += align16((size_t)2 * A * 2);
   MNode* curl = (MNode*)ptr;
   MNode* nxtl = curl + MM;
   ptr += align16((size_t)2 * MM * sizeof(MNode));
-  TNode* tq = (TNode*)ptr;
-  ptr += align16((size_t)(A + MAXR) * sizeof(TNode));
+  TN* tq = (TN*)ptr;
+  ptr += align16((size_t)(A + MAXR) * sizeof(TN));
   int32_t* tq_ready = (int32_t*)ptr;
   ptr += align16((size_t)(A + MAXR) * 4);
   int16_t* mind_all = (int16_t*)ptr;
@@ -1700,6 +1788,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
     wyd[j] = __dmul_rn((double)wv, yr);
   }
   for (int j = tid; j < a0 + MAXR; j += SUB_NT) tq_ready[j] = 0;  // barrier-ordered before any queue use
+  for (int j = tid; j < 2 * a0; j += SUB_NT) rdef[j] = 0xffffu;
   __syncthreads();
   auto hfind = [&](uint32_t hk) -> uint16_t {
     uint32_t h = (hk * 0x9E3779B1u) >> (32 - HBITS);
@@ -1773,7 +1862,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
     r0.value = 0.0;
     r0.drss = 0.0;
     recs[rec0] = r0;
-    if (R.a > TINY) {
+    if (R.a > TT) {
       MNode c;
       c.lo = s_off[r];
       c.a = R.a;
@@ -1784,10 +1873,10 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       c.split = 0;
       curl[atomicAdd(&s_ncur, 1)] = c;
     } else {
-      TNode c;
+      TN c;
       c.rlo = s_off[r];
       c.ra = R.a;
-      c.mask = R.a == 64 ? ~0ull : ((1ull << R.a) - 1ull);
+      m_full(c.mask, R.a);
       c.id = (r << 16) | rec0;
       c.n = R.n;
       c.S = R.S;
@@ -1998,8 +2087,8 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
             nd.al = al;
             nd.nl = best.nl;
             nd.Sl = best.Sl;
-            nd.kind[0] = (best.nl <= g.nodesize || al < 2) ? KIND_LEAF : (al <= TINY ? KIND_SMALL : KIND_LARGE);
-            nd.kind[1] = (nr <= g.nodesize || ar < 2) ? KIND_LEAF : (ar <= TINY ? KIND_SMALL : KIND_LARGE);
+            nd.kind[0] = (best.nl <= g.nodesize || al < 2) ? KIND_LEAF : (al <= TT ? KIND_SMALL : KIND_LARGE);
+            nd.kind[1] = (nr <= g.nodesize || ar < 2) ? KIND_LEAF : (ar <= TT ? KIND_SMALL : KIND_LARGE);
             curl[i] = nd;
           }
         } else if (lane == 0) {
@@ -2039,10 +2128,10 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
             c.split = 0;
             nxtl[idx++] = c;
           } else {
-            TNode c;
+            TN c;
             c.rlo = lo;
             c.ra = a;
-            c.mask = a == 64 ? ~0ull : ((1ull << a) - 1ull);
+            m_full(c.mask, a);
             c.id = (nd.id & ~0xffff) | (nd.lid + sdv);
             c.n = nn;
             c.S = S;
@@ -2109,14 +2198,29 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   {
     const int nroots = a_get<int>(s_alloc);
     for (int qi = wid; qi < nroots; qi += SUB_NW) {
-      const TNode r = tq_read(tq, qi);  // pushed before the barrier above
+      const TN r = tq_read(tq, qi);  // pushed before the barrier above
       for (int k = lane; k < r.ra; k += 32) rmap[list[r.rlo + k] & 0xffffu] = (uint8_t)k;
     }
   }
   __syncthreads();
+  // TV = 1: ppos[f * a0 + rlo + i] = position, in feature f's segment of its tiny root, of the row at feature-0
+  // position i (the scratch area is free once the medium levels are done), so a node's rows in feature f's order
+  // are the set bits of one 64-bit mask built from the node's mask (no staging, no pass over non-member rows)
+  uint8_t* ppos = (uint8_t*)temp_all;
+  if constexpr (TV == 1) {
+    const int nroots = a_get<int>(s_alloc);
+    for (int it = wid; it < nroots * p; it += SUB_NW) {
+      const int qi = it / p, f = it - qi * p;
+      const int rlo = a_get<int32_t>(tq[qi].rlo), ra = a_get<int32_t>(tq[qi].ra);
+      const uint32_t* seg = list + (size_t)f * a0 + rlo;
+      uint8_t* pp = ppos + (size_t)f * a0 + rlo;
+      for (int k = lane; k < ra; k += 32) pp[rmap[seg[k] & 0xffffu]] = (uint8_t)k;
+    }
+    __syncthreads();
+  }
   for (;;) {
     int h = -1;
-    TNode nd;
+    TN nd;
     if (lane == 0) {
       unsigned ns = 32;
       for (;;) {
@@ -2147,11 +2251,12 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       have = false;
       ++n_tiny;
       const int rlo = nd.rlo, ra = nd.ra;
-      const int an = __popcll(nd.mask);  // distinct rows of the node
+      const int an = m_popc(nd.mask);  // distinct rows of the node
       nvis += (unsigned long long)an * (unsigned)g.mtry;
       const long long c0_ = g.stats ? clock64() : 0;
       const uint32_t t = t_of(nd.id);
       warp_draw_mtry(g.seed, t, nd.key, p, g.mtry, mind, feats, lane);
+      const uint64_t ck = child_key(g.seed, t, nd.key, lane & 1);  // independent of the split: off the tail
       const long long c1_ = g.stats ? clock64() : 0;
       const int64_t nk = nd.n, Sk = nd.S;
       const float nkf = __ll2float_rn(nk), Skf = __ll2float_rn(Sk);
@@ -2162,6 +2267,103 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       uint32_t ltie = 0xffffffffu, lra = 0, lrb = 0;
       int32_t lnl = 0;
       int64_t lSl = 0;
+      if constexpr (TV == 1) {
+        // Lane s scans drawn feature feats[s] (s = lane, lane + 32, ...) serially over the node's own rows: the
+        // node's rows in that feature's value order are the set bits of Mf (positions in the tiny root's
+        // segment), so the loop runs an times with no staging, no segmented warp scan and no idle positions.
+        // Per boundary the fp32 bounds tL <= t <= tU (key_bounds_t); M = warp max of the lower bounds; a lane
+        // whose second-largest upper bound is below M evaluates its one candidate directly, any other lane with
+        // an upper bound >= M re-walks its features taking the exact S4.3 key where tU >= M.
+        auto feat_mask = [&](int f, uint64_t (&Mf)[NWD]) {
+          const uint8_t* pp = ppos + (size_t)f * a0 + rlo;
+          uint64_t m[NWD];
+#pragma unroll
+          for (int w = 0; w < NWD; ++w) {
+            m[w] = nd.mask[w];
+            Mf[w] = 0ull;
+          }
+#pragma unroll 4
+          for (int c = 0; c < an; ++c) m_set(Mf, (int)pp[m_pop(m)]);
+        };
+        float mLt = -1.0f, mU = -1.0f, u2 = -1.0f;
+        int bs = -1;
+        uint32_t be = 0, ben = 0;
+        int32_t bcw = 0;
+        int64_t bcs = 0;
+        for (int s = lane; s < g.mtry; s += 32) {
+          const uint32_t* seg = list + (size_t)feats[s] * a0 + rlo;
+          uint64_t Mf[NWD];
+          feat_mask(feats[s], Mf);
+          uint32_t pe = seg[m_pop(Mf)];
+          int32_t cw = wl[pe & 0xffffu];
+          int64_t cs = wy[pe & 0xffffu];
+#pragma unroll 2
+          for (int c = 1; c < an; ++c) {
+            const uint32_t e = seg[m_pop(Mf)];
+            if ((e >> 16) != (pe >> 16)) {
+              float tL, tU;
+              key_bounds_t(nkf, Skf, nk, cw, cs, tL, tU);
+              mLt = fmaxf(mLt, tL);
+              if (tU > mU) {
+                u2 = mU;
+                mU = tU;
+                bs = s;
+                be = pe;
+                ben = e;
+                bcw = cw;
+                bcs = cs;
+              } else {
+                u2 = fmaxf(u2, tU);
+              }
+            }
+            cw += wl[e & 0xffffu];
+            cs += wy[e & 0xffffu];
+            pe = e;
+          }
+        }
+        const float M = warp_max_t(mLt);
+        if (mU >= M && mU >= 0.0f && u2 < M) {  // a single candidate on this lane
+          lg = split_key(nk, Sk, bcw, bcs);
+          ltie = ((uint32_t)feats[bs] << 16) | (be >> 16);
+          lnl = bcw;
+          lSl = bcs;
+          lra = be & 0xffffu;
+          lrb = ben & 0xffffu;
+        } else if (mU >= M && mU >= 0.0f) {
+          for (int s = lane; s < g.mtry; s += 32) {
+            const uint32_t* seg = list + (size_t)feats[s] * a0 + rlo;
+            uint64_t Mf[NWD];
+            feat_mask(feats[s], Mf);
+            uint32_t pe = seg[m_pop(Mf)];
+            int32_t cw = wl[pe & 0xffffu];
+            int64_t cs = wy[pe & 0xffffu];
+            for (int c = 1; c < an; ++c) {
+              const uint32_t e = seg[m_pop(Mf)];
+              if ((e >> 16) != (pe >> 16)) {
+                float tL, tU;
+                key_bounds_t(nkf, Skf, nk, cw, cs, tL, tU);
+                if (tU >= M) {
+                  const double gk = split_key(nk, Sk, cw, cs);
+                  const uint32_t tie = ((uint32_t)feats[s] << 16) | (pe >> 16);
+                  if (gk > lg || (gk == lg && tie < ltie)) {
+                    lg = gk;
+                    ltie = tie;
+                    lnl = cw;
+                    lSl = cs;
+                    lra = pe & 0xffffu;
+                    lrb = e & 0xffffu;
+                  }
+                }
+              }
+              cw += wl[e & 0xffffu];
+              cs += wy[e & 0xffffu];
+              pe = e;
+            }
+          }
+        }
+        (void)stg;
+        (void)lt;
+      } else {
       // Features go in groups as large as the staging area holds (ng * an <= sub_temp(A) entries): every drawn
       // feature in ONE group when the node has few distinct rows, so the scan / bound / max passes and their
       // fixed costs run once per node instead of once per TGRP features.
@@ -2187,8 +2389,8 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
             for (int k = 0; k < 2 * TGRP; ++k) ri[k] = rmap[ev[k] & 0xffffu];
 #pragma unroll
             for (int u = 0; u < TGRP; ++u) {
-              const bool v0 = u < nu && ((nd.mask >> ri[2 * u]) & 1ull);
-              const bool v1 = u < nu && lane + 32 < ra && ((nd.mask >> ri[2 * u + 1]) & 1ull);
+              const bool v0 = u < nu && ((nd.mask[0] >> ri[2 * u]) & 1ull);
+              const bool v1 = u < nu && lane + 32 < ra && ((nd.mask[0] >> ri[2 * u + 1]) & 1ull);
               const unsigned m0 = __ballot_sync(0xffffffffu, v0), m1 = __ballot_sync(0xffffffffu, v1);
               if (v0) stg[(u0 + u) * an + __popc(m0 & lt)] = ev[2 * u];
               if (v1) stg[(u0 + u) * an + __popc(m0) + __popc(m1 & lt)] = ev[2 * u + 1];
@@ -2203,7 +2405,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
             for (int k = 0; k < TGRP; ++k) ri[k] = rmap[ev[k] & 0xffffu];
 #pragma unroll
             for (int u = 0; u < TGRP; ++u) {
-              const bool v0 = u < nu && lane < ra && ((nd.mask >> ri[u]) & 1ull);
+              const bool v0 = u < nu && lane < ra && ((nd.mask[0] >> ri[u]) & 1ull);
               const unsigned m0 = __ballot_sync(0xffffffffu, v0);
               if (v0) stg[(u0 + u) * an + __popc(m0 & lt)] = ev[u];
             }
@@ -2362,6 +2564,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         __syncwarp();
         s0 += ng;
       }
+      }  // TV == 0
       const long long c2_ = g.stats ? clock64() : 0;
       if (g.stats && lane == 0) { atomicAdd(&g.stats[11], (unsigned long long)(c1_ - c0_)); atomicAdd(&g.stats[12], (unsigned long long)(c2_ - c1_)); }
       const int wlane = warp_argmax_key(gkey(lg), ltie);
@@ -2377,32 +2580,44 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         const uint32_t brb = __shfl_sync(0xffffffffu, lrb, wlane);
         // child masks from the winning feature's order: left = rank <= brk
         const uint32_t* seg = list + (size_t)bf * a0 + rlo;
-        uint64_t mL = 0;
+        uint32_t lw[2 * NWD];  // this lane's left rows, by 32-bit word of the mask
+#pragma unroll
+        for (int w = 0; w < 2 * NWD; ++w) lw[w] = 0u;
         double vl = 0.0, vr = 0.0;
   #pragma unroll
-        for (int hh = 0; hh < 2; ++hh) {
+        for (int hh = 0; hh < TT / 32; ++hh) {
           const int k = lane + 32 * hh;
+          if (TT > 64 && 32 * hh >= ra) break;  // warp-uniform
           const uint32_t e = k < ra ? seg[k] : 0u;
           const uint32_t lrow = e & 0xffffu;
           const int ri = k < ra ? rmap[lrow] : 0;
-          const bool valid = k < ra && ((nd.mask >> ri) & 1ull);
+          const bool valid = k < ra && m_test(nd.mask, ri);
           const bool left = valid && (e >> 16) <= brk;
-          const uint32_t lo = __reduce_or_sync(0xffffffffu, (left && ri < 32) ? (1u << ri) : 0u);
-          const uint32_t hi = __reduce_or_sync(0xffffffffu, (left && ri >= 32) ? (1u << (ri - 32)) : 0u);
-          mL |= ((uint64_t)hi << 32) | lo;
-          if (left) vl += wyd[lrow];
-          else if (valid) vr += wyd[lrow];
+#pragma unroll
+          for (int w = 0; w < 2 * NWD; ++w) lw[w] |= (left && (ri >> 5) == w) ? 1u << (ri & 31) : 0u;
+          if (!DEFER) {
+            if (left) vl += wyd[lrow];
+            else if (valid) vr += wyd[lrow];
+          }
         }
-        const uint64_t mR = nd.mask & ~mL;
+        uint64_t mL[NWD], mR[NWD];
+#pragma unroll
+        for (int w = 0; w < NWD; ++w) {
+          mL[w] = ((uint64_t)__reduce_or_sync(0xffffffffu, lw[2 * w + 1]) << 32) | __reduce_or_sync(0xffffffffu, lw[2 * w]);
+          mR[w] = nd.mask[w] & ~mL[w];
+        }
+        if (!DEFER) {
   #pragma unroll
-        for (int o = 16; o > 0; o >>= 1) {
-          vl += __shfl_down_sync(0xffffffffu, vl, o);
-          vr += __shfl_down_sync(0xffffffffu, vr, o);
+          for (int o = 16; o > 0; o >>= 1) {
+            vl += __shfl_down_sync(0xffffffffu, vl, o);
+            vr += __shfl_down_sync(0xffffffffu, vr, o);
+          }
         }
         const int nr = nd.n - bnl;
-        const bool gl = bnl > g.nodesize && __popcll(mL) >= 2;
-        const bool gr = nr > g.nodesize && __popcll(mR) >= 2;
-        const double val_l = __ddiv_rn(vl, (double)bnl), val_r = __ddiv_rn(vr, (double)nr);
+        const bool gl = bnl > g.nodesize && m_popc(mL) >= 2;
+        const bool gr = nr > g.nodesize && m_popc(mR) >= 2;
+        const double val_l = DEFER ? __longlong_as_double((long long)mL[0]) : __ddiv_rn(vl, (double)bnl);
+        const double val_r = DEFER ? __longlong_as_double((long long)mR[0]) : __ddiv_rn(vr, (double)nr);
         // Records: a node's whole record is written by the warp that grows it (this one for nd); a child that
         // stays a leaf gets its record here, a child that is grown further (here or by the warp that takes it
         // from the queue) writes its own -- so no record is written by two warps without a barrier between.
@@ -2415,9 +2630,10 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
           r.count = nd.n;
           r.ra = (uint16_t)bra;
           r.rb = (uint16_t)brb;
-          r.value = nd.value;
+          r.value = DEFER ? __longlong_as_double((long long)nd.mask[0]) : nd.value;
           r.drss = ldexp(__ddiv_rn(bg, (double)nd.n), -2 * g.q);
           recs[nd.id & 0xffff] = r;
+          if (DEFER) rdef[nd.id & 0xffff] = (uint16_t)rlo;
           SRec c;
           c.feature = -1;
           c.left = -1;
@@ -2427,28 +2643,32 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
             c.count = bnl;
             c.value = val_l;
             recs[lid] = c;
+            if (DEFER) rdef[lid] = (uint16_t)rlo;
           }
           if (!gr) {
             c.count = nr;
             c.value = val_r;
             recs[lid + 1] = c;
+            if (DEFER) rdef[lid + 1] = (uint16_t)rlo;
           }
         }
         lid = __shfl_sync(0xffffffffu, lid, 0);
-        // child keys on lanes 0 and 1
-        const uint64_t ck = child_key(g.seed, t, nd.key, lane & 1);
+        // child keys on lanes 0 and 1 (computed before the search)
         const uint64_t kl = __shfl_sync(0xffffffffu, ck, 0), kr = __shfl_sync(0xffffffffu, ck, 1);
-        TNode cl, cr;
+        TN cl, cr;
         cl.value = val_l;
         cr.value = val_r;
         cl.rlo = cr.rlo = nd.rlo;
         cl.ra = cr.ra = nd.ra;
-        cl.mask = mL;
+#pragma unroll
+        for (int w = 0; w < NWD; ++w) {
+          cl.mask[w] = mL[w];
+          cr.mask[w] = mR[w];
+        }
         cl.id = (nd.id & ~0xffff) | lid;
         cl.n = bnl;
         cl.S = bSl;
         cl.key = kl;
-        cr.mask = mR;
         cr.id = (nd.id & ~0xffff) | (lid + 1);
         cr.n = nr;
         cr.S = nd.S - bSl;
@@ -2456,7 +2676,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         // continue with one child in this warp, hand the sibling to the queue
         if (gl && gr) {
           // the larger child keeps the warp (the longer remaining chain stays off the queue's hand-off latency)
-          const bool keep_r = g.tq_bigger_first && __popcll(mR) > __popcll(mL);
+          const bool keep_r = g.tq_bigger_first && m_popc(mR) > m_popc(mL);
           if (lane == 0) tq_push(tq, tq_ready, &s_alloc, &s_pending, keep_r ? cl : cr);
           nd = keep_r ? cr : cl;
           have = true;
@@ -2473,9 +2693,10 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         r.left = -1;
         r.count = nd.n;
         r.ra = r.rb = 0;
-        r.value = nd.value;
+        r.value = DEFER ? __longlong_as_double((long long)nd.mask[0]) : nd.value;
         r.drss = 0.0;
         recs[nd.id & 0xffff] = r;
+        if (DEFER) rdef[nd.id & 0xffff] = (uint16_t)rlo;
       }
 
     }
@@ -2511,7 +2732,18 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
     g.pool.drss[gid] = rc.drss;
     if (k > 0) {
       g.pool.count[gid] = rc.count;
-      g.pool.value[gid] = rc.value;
+      double v = rc.value;
+      if (DEFER && rdef[l] != 0xffffu) {  // S4.7 node value from the record's row mask over its tiny root
+        const int rl = rdef[l];
+        uint64_t mk = (uint64_t)__double_as_longlong(rc.value);
+        double sw = 0.0;
+        while (mk) {
+          sw += wyd[list[rl + __ffsll((long long)mk) - 1] & 0xffffu];
+          mk &= mk - 1;
+        }
+        v = __ddiv_rn(sw, (double)rc.count);
+      }
+      g.pool.value[gid] = v;
     }
   }
   if (g.visits && lane == 0 && nvis) atomicAdd(g.visits, nvis);
@@ -2761,10 +2993,17 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
 
   ptm.mark("presort");
   // ---- sizing: subtree capacity A and trees in flight B
-  const int smax = dyn_smem_limit(k_subtree);
+  const int smax = std::min(std::min(dyn_smem_limit(k_subtree<0, 64>), dyn_smem_limit(k_subtree<1, 64>)),
+                            dyn_smem_limit(k_subtree<1, 128>));
   int A = 2;
-  while (A < 1024 && subtree_smem(A + 1, p) <= (size_t)smax) ++A;  // load 2 holds <= 32 chunks of 32
-  BF_REQUIRE(subtree_smem(2, p) <= (size_t)smax, BF_ENOTIMPL, "bf_fit: p too large for the shared-memory subtree kernel");
+  // tiny-node search: 1 = lane per drawn feature over the node's own rows (default), 0 = staged (slot, position)
+  // items scanned by the whole warp (BF_TINY_V=0); largest tiny root 64 rows (default) or 128 (BF_TINY_MAX=128,
+  // lane-per-feature search only; measured slower: the longer tiny chains outweigh the shorter medium phase)
+  static const int tiny_v = getenv("BF_TINY_V") ? atoi(getenv("BF_TINY_V")) : 1;
+  static const int tiny_max = (tiny_v != 0 && getenv("BF_TINY_MAX") && atoi(getenv("BF_TINY_MAX")) == 128) ? 128 : 64;
+  while (A < 1024 && subtree_smem(A + 1, p, tiny_max) <= (size_t)smax) ++A;  // load 2 holds <= 32 chunks of 32
+  BF_REQUIRE(subtree_smem(2, p, tiny_max) <= (size_t)smax, BF_ENOTIMPL,
+             "bf_fit: p too large for the shared-memory subtree kernel");
   if (prm.small_node_max > 0) A = std::max(2, std::min(A, prm.small_node_max));
 
   const int32_t T_loc = prm.tree_end - prm.tree_begin;
@@ -3176,7 +3415,12 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
           }
           {
             KScope ks_("k_subtree", s, 0.0);
-            k_subtree<<<(unsigned)ngroups, SUB_NT, subtree_smem(A, p), s>>>(ga);
+            if (tiny_v == 0)
+              k_subtree<0, 64><<<(unsigned)ngroups, SUB_NT, subtree_smem(A, p, 64), s>>>(ga);
+            else if (tiny_max == 64)
+              k_subtree<1, 64><<<(unsigned)ngroups, SUB_NT, subtree_smem(A, p, 64), s>>>(ga);
+            else
+              k_subtree<1, 128><<<(unsigned)ngroups, SUB_NT, subtree_smem(A, p, 128), s>>>(ga);
           }
           if (ga.visits) {  // SURVEY 8(d) split-search bytes of the subtree nodes: 20 B per entry visit
             unsigned long long hv = 0;

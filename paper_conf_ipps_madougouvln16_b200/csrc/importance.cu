@@ -394,12 +394,33 @@ __global__ void __launch_bounds__(TP) k_importance(ImpArgs g) {
     if (sacc[m] != 0.0) atomicAdd(&g.d_slots[(int64_t)i * g.p + m], sacc[m]);
 }
 
+// Row-major RN_f32 copy of the column-major X (stride xfs floats, a multiple of 4): 32 x 32 tiles through shared
+// memory, coalesced on both sides.
+__global__ void k_xf_rows(const double* __restrict__ X, int64_t ldx, int64_t n, int p, float* __restrict__ Xf, int xfs) {
+  __shared__ float t[32][33];
+  const int64_t r0 = (int64_t)blockIdx.x * 32;
+  const int f0 = blockIdx.y * 32;
+  for (int j = threadIdx.y; j < 32; j += blockDim.y) {  // j: feature in the tile, threadIdx.x: row
+    const int64_t r = r0 + threadIdx.x;
+    const int f = f0 + j;
+    t[j][threadIdx.x] = (r < n && f < p) ? __double2float_rn(X[(int64_t)f * ldx + r]) : 0.0f;
+  }
+  __syncthreads();
+  for (int j = threadIdx.y; j < 32; j += blockDim.y) {  // j: row in the tile, threadIdx.x: feature
+    const int64_t r = r0 + j;
+    const int f = f0 + threadIdx.x;
+    if (r < n && f < xfs) Xf[r * xfs + f] = f < p ? t[threadIdx.x][j] : 0.0f;
+  }
+}
+
 // k_importance8: k_importance on the compact nodes (predict.cu k_pack8) with a float row tile: the same
 // walks, exact by the float-tie fallback of S5 (the fp64 x of the row from X, or the fp64 permuted value,
 // against the fp64 threshold of Node16).  Half the shared memory per row (twice the CTAs per SM) and half
 // the node bytes.
 struct Imp8Args {
   ImpArgs a;
+  const float* Xf;  // row-major RN_f32 copy of X, stride xfs (k_xf_rows): a row's tile is 4 p contiguous bytes
+  int xfs;
   const uint2* nodes8;
   const uint32_t* roots8;  // per local tree (forest numbering)
   unsigned long long* prof;  // profile mode: [0] node loads, [1] permuted re-walks (algorithmic bytes), else NULL
@@ -422,15 +443,22 @@ __global__ void __launch_bounds__(IPT) k_importance8(Imp8Args g8) {
   const int64_t a = a0 + threadIdx.x;
   const bool act = a < n_o;
   const uint32_t r = act ? Ob[a] : Ob[a0];
-  {  // stage the tile as floats: 8 column loads in flight per thread
+  {  // stage the tile from the row-major float copy: the row's 4 p bytes as 16-byte loads, 8 in flight
     float* xs = sx + threadIdx.x * stride;
-    for (int f0 = 0; f0 < g.p; f0 += 8) {
-      double v[8];
+    const float4* src = reinterpret_cast<const float4*>(g8.Xf + (int64_t)r * g8.xfs);
+    const int nq = (g.p + 3) >> 2;
+    for (int q0 = 0; q0 < nq; q0 += 8) {
+      float4 v[8];
 #pragma unroll
-      for (int u = 0; u < 8; ++u) v[u] = (f0 + u < g.p) ? __ldg(g.X + (int64_t)(f0 + u) * g.ldx + r) : 0.0;
+      for (int u = 0; u < 8; ++u) v[u] = (q0 + u < nq) ? __ldg(src + q0 + u) : make_float4(0.f, 0.f, 0.f, 0.f);
 #pragma unroll
-      for (int u = 0; u < 8; ++u)
-        if (f0 + u < g.p) xs[f0 + u] = __double2float_rn(v[u]);
+      for (int u = 0; u < 8; ++u) {
+        const int f = 4 * (q0 + u);
+        if (f < g.p) xs[f] = v[u].x;
+        if (f + 1 < g.p) xs[f + 1] = v[u].y;
+        if (f + 2 < g.p) xs[f + 2] = v[u].z;
+        if (f + 3 < g.p) xs[f + 3] = v[u].w;
+      }
     }
   }
   __syncthreads();
@@ -683,6 +711,13 @@ void perm_impl(uint64_t seed, int32_t t, int32_t m, int64_t n_o, int64_t* out, c
   BF_CUDA_CHECK(cudaGetLastError());
 }
 
+void xf_rows_impl(const double* X, int64_t ldx, int64_t n, int p, float* Xf, int xfs, cudaStream_t s) {
+  if (n <= 0) return;
+  KScope ks_("k_xf_rows", s, (double)n * p * 8.0 + (double)n * xfs * 4.0);
+  k_xf_rows<<<dim3((unsigned)ceil_div(n, 32), (unsigned)ceil_div(xfs, 32)), dim3(32, 8), 0, s>>>(X, ldx, n, p, Xf, xfs);
+  BF_CUDA_CHECK(cudaGetLastError());
+}
+
 void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, const double* y_in, int64_t n, int32_t p,
                          const bf_oob_accum& acc, cudaStream_t s) {
   const int32_t T = f->info.tree_end - f->info.tree_begin;
@@ -733,6 +768,8 @@ void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, co
     prof.alloc(2, s);
     BF_CUDA_CHECK(cudaMemsetAsync(prof.p, 0, 16, s));
   }
+  DBuf<float> Xf;
+  const int xfs = (p + 3) & ~3;
   for (int32_t i0 = 0; i0 < T; i0 += B) {
     const int Bc = std::min(B, T - i0);
     bootstrap_impl(f->info.seed, f->info.tree_begin + i0, Bc, n, f->info.sampsize, f->info.replace, w.p, s);
@@ -794,8 +831,14 @@ void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, co
     g.perm = perm.p;
     // OOB rows per tree <= n; grid sized for n (CTAs past n_o exit early)
     if (n8 && smem8 <= (size_t)ismax8) {
+      if (!Xf.p) {  // once per call: the row-major float copy the CTAs stage their OOB rows from
+        Xf.alloc((size_t)n * xfs, s);
+        xf_rows_impl(X, ldx, n, p, Xf.p, xfs, s);
+      }
       Imp8Args g8;
       g8.a = g;
+      g8.Xf = Xf.p;
+      g8.xfs = xfs;
       g8.nodes8 = n8;
       g8.roots8 = f->d_roots8;
       g8.prof = prof.p;
@@ -818,9 +861,9 @@ void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, co
     BF_CUDA_CHECK(cudaStreamSynchronize(s));
     double units = 0.0;
     for (int64_t v : hno) units += (double)v;
-    // per (tree, OOB row): row gather 8p + y 8 + O index 4 + oob sum/count 12; per re-walk: pi 4 + x 8;
+    // per (tree, OOB row): float row gather 4p + y 8 + O index 4 + oob sum/count 12; per re-walk: pi 4 + x 8;
     // per node load 8 (compact nodes)
-    prof_add_bytes("k_importance8", units * (8.0 * p + 24.0) + (double)hp[1] * 12.0 + (double)hp[0] * 8.0);
+    prof_add_bytes("k_importance8", units * (4.0 * p + 24.0) + (double)hp[1] * 12.0 + (double)hp[0] * 8.0);
     prof_add_bytes("importance_node_loads", (double)hp[0]);
     prof_add_bytes("importance_rewalks", (double)hp[1]);
   }

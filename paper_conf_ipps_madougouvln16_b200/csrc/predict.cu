@@ -339,6 +339,293 @@ __global__ void __launch_bounds__(PT8, 6) k_predict8s(const uint2* __restrict__ 
   if (last && yhat) yhat[rr] = acc * inv_t;
 }
 
+
+// ------------------------------------------------------------------ two-level 32-byte groups (G32)
+// Every node at even depth owns a slot of 32 bytes.  For an internal node k (children L, R = L + 1):
+//   q0 = {float RN_f32(thr_k), feature_k | LL<<8 | RL<<9 | GL<<10 (4 bits: grandchild slot is a leaf)}
+//   q1 = L: leaf -> its fp64 value; internal -> {float RN_f32(thr_L), feature_L | rel<<8}  (rel = id(L) - id(k))
+//   q2 = R: likewise, rel the same (id(R) = id(k) + rel + 1)
+//   q3 = {first grandchild slot (global), id(k) (global Node16 index, for the fp64 tie fallback)}
+// The grandchildren (children of L if L is internal, then children of R if R is internal) occupy consecutive
+// slots from q3.lo; a grandchild that is a leaf holds its fp64 value in q0.  One 256-bit load per group decides
+// two levels of a walk (S5: x <= thr goes left), with the same float-then-fp64 comparison as Node8.
+// Slots: depth parity by pointer jumping over parent links, then per group the number of grandchild slots,
+// one exclusive scan (the root of every tree takes one extra slot first), and the slots written top-down.
+constexpr uint32_t G32_LEAF = 0x80000000u;  // walk state: the slot being loaded is a leaf
+
+__global__ void k_g32_parent(const Node16* __restrict__ nodes, const int64_t* __restrict__ off, int32_t* anc,
+                             uint8_t* bit) {
+  const int32_t t = blockIdx.y;
+  const int64_t lo = off[t], hi = off[t + 1];
+  for (int64_t k = lo + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < hi; k += (int64_t)gridDim.x * blockDim.x) {
+    if (k == lo) {
+      anc[k] = -1;
+      bit[k] = 0;
+    }
+    const Node16 nd = nodes[k];
+    if (nd.feature >= 0) {
+      const int64_t c = lo + nd.left;
+      anc[c] = (int32_t)k;
+      anc[c + 1] = (int32_t)k;
+      bit[c] = 1;
+      bit[c + 1] = 1;
+    }
+  }
+}
+
+// one pointer-jumping round: bit = parity of the distance to anc; anc moves twice as far up
+__global__ void k_g32_jump(const int32_t* __restrict__ anc, const uint8_t* __restrict__ bit, int32_t* anc2,
+                           uint8_t* bit2, int64_t total, int* more) {
+  const int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (k >= total) return;
+  const int32_t a = anc[k];
+  if (a < 0) {
+    anc2[k] = -1;
+    bit2[k] = bit[k];
+    return;
+  }
+  const int32_t aa = anc[a];
+  anc2[k] = aa;
+  bit2[k] = bit[k] ^ bit[a];
+  if (aa >= 0) *more = 1;
+}
+
+// grandchild slots of every group (even-depth internal node), plus the root's own slot
+__global__ void k_g32_count(const Node16* __restrict__ nodes, const int64_t* __restrict__ off,
+                            const uint8_t* __restrict__ bit, uint32_t* cnt) {
+  const int32_t t = blockIdx.y;
+  const int64_t lo = off[t], hi = off[t + 1];
+  for (int64_t k = lo + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < hi; k += (int64_t)gridDim.x * blockDim.x) {
+    uint32_t c = k == lo;
+    const Node16 nd = nodes[k];
+    if (bit[k] == 0 && nd.feature >= 0) {
+      const int64_t l = lo + nd.left;
+      c += 2u * (nodes[l].feature >= 0) + 2u * (nodes[l + 1].feature >= 0);
+    }
+    cnt[k] = c;
+  }
+}
+
+__global__ void k_g32_slots(const Node16* __restrict__ nodes, const int64_t* __restrict__ off,
+                            const uint8_t* __restrict__ bit, const uint32_t* __restrict__ ex, uint32_t* slot,
+                            int64_t* tree_slot) {
+  const int32_t t = blockIdx.y;
+  const int64_t lo = off[t], hi = off[t + 1];
+  for (int64_t k = lo + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < hi; k += (int64_t)gridDim.x * blockDim.x) {
+    if (k == lo) {
+      slot[k] = ex[k];
+      tree_slot[t] = ex[k];
+    }
+    const Node16 nd = nodes[k];
+    if (bit[k] != 0 || nd.feature < 0) continue;
+    uint32_t b = ex[k] + (k == lo);
+    const int64_t l = lo + nd.left;
+#pragma unroll
+    for (int c = 0; c < 2; ++c) {
+      const Node16 ch = nodes[l + c];
+      if (ch.feature >= 0) {
+        slot[lo + ch.left] = b++;
+        slot[lo + ch.left + 1] = b++;
+      }
+    }
+  }
+}
+
+__device__ __forceinline__ unsigned long long g32_child(const Node16& ch, uint32_t rel, int* bad) {
+  if (ch.feature < 0) return (unsigned long long)__double_as_longlong(ch.v);
+  return (unsigned long long)__float_as_uint(__double2float_rn(ch.v)) |
+         ((unsigned long long)((uint32_t)ch.feature | (rel << 8)) << 32);
+}
+
+__global__ void k_g32_emit(const Node16* __restrict__ nodes, const int64_t* __restrict__ off,
+                           const uint8_t* __restrict__ bit, const uint32_t* __restrict__ ex,
+                           const uint32_t* __restrict__ slot, ulonglong4* __restrict__ g32, uint32_t* __restrict__ roots,
+                           int* bad) {
+  const int32_t t = blockIdx.y;
+  const int64_t lo = off[t], hi = off[t + 1];
+  if (blockIdx.x == 0 && threadIdx.x == 0) roots[t] = slot[lo] | (nodes[lo].feature < 0 ? ROOT_LEAF : 0u);
+  for (int64_t k = lo + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < hi; k += (int64_t)gridDim.x * blockDim.x) {
+    if (bit[k] != 0) continue;
+    const Node16 nd = nodes[k];
+    ulonglong4 G = make_ulonglong4(0ull, 0ull, 0ull, 0ull);
+    if (nd.feature < 0) {
+      G.x = (unsigned long long)__double_as_longlong(nd.v);
+    } else {
+      const int64_t l = lo + nd.left;
+      const int64_t rel = l - k;
+      if (rel < 1 || rel >= (1ll << 24) || nd.feature >= 256) {
+        *bad = 1;
+        continue;
+      }
+      const Node16 L = nodes[l], R = nodes[l + 1];
+      uint32_t gl = 0, gi = 0;
+      if (L.feature >= 0) {
+        gl |= (uint32_t)(nodes[lo + L.left].feature < 0) << gi;
+        gl |= (uint32_t)(nodes[lo + L.left + 1].feature < 0) << (gi + 1);
+        gi += 2;
+        if (L.feature >= 256) *bad = 1;
+      }
+      if (R.feature >= 0) {
+        gl |= (uint32_t)(nodes[lo + R.left].feature < 0) << gi;
+        gl |= (uint32_t)(nodes[lo + R.left + 1].feature < 0) << (gi + 1);
+        if (R.feature >= 256) *bad = 1;
+      }
+      const uint32_t w0 = (uint32_t)nd.feature | ((uint32_t)(L.feature < 0) << 8) | ((uint32_t)(R.feature < 0) << 9) |
+                          (gl << 10);
+      G.x = (unsigned long long)__float_as_uint(__double2float_rn(nd.v)) | ((unsigned long long)w0 << 32);
+      G.y = g32_child(L, (uint32_t)rel, bad);
+      G.z = g32_child(R, (uint32_t)rel, bad);
+      G.w = (unsigned long long)(ex[k] + (k == lo)) | ((unsigned long long)(uint32_t)k << 32);
+    }
+    g32[slot[k]] = G;
+  }
+}
+
+__device__ __forceinline__ ulonglong4 ldg256(const ulonglong4* p) {
+  ulonglong4 v;
+  asm volatile("ld.global.nc.v4.u64 {%0,%1,%2,%3}, [%4];" : "=l"(v.x), "=l"(v.y), "=l"(v.z), "=l"(v.w) : "l"(p));
+  return v;
+}
+
+// k_predict8s on G32 groups: a slot (walk in flight) holds the 32 bytes of its current group; per step it
+// decides the group's node and the chosen child, then loads the grandchild's slot (a leaf slot ends the walk
+// one load later).  Trees [t_begin, t_end) of one block, rows staged as floats exactly as in k_predict8s.
+template <bool PROF, int NS>
+__global__ void __launch_bounds__(PT8) k_predict32(const ulonglong4* __restrict__ g32, const Node16* __restrict__ nodes16,
+                                                   const uint32_t* __restrict__ roots, int32_t t_begin, int32_t t_end,
+                                                   int first, int last, const double* __restrict__ Xq, int64_t ldq,
+                                                   const float* __restrict__ Xqf, int xfs,
+                                                   int64_t m, int p, double* yhat_sum, double* yhat, double inv_t,
+                                                   unsigned long long* visits) {
+  extern __shared__ float sxf[];  // PT8 x (p|1), row-major
+  __shared__ uint32_t s_rw[RT8];
+  __shared__ ulonglong4 s_rn[RT8];
+  const int stride = p | 1;
+  const int64_t r0 = (int64_t)blockIdx.x * PT8;
+  const int rows = (int)(m - r0 < PT8 ? m - r0 : PT8);
+  const int nt = t_end - t_begin;
+  if ((int)threadIdx.x < nt) {
+    const uint32_t rw = __ldg(roots + t_begin + threadIdx.x);
+    s_rw[threadIdx.x] = rw;
+    s_rn[threadIdx.x] = ldg256(g32 + (rw & ~ROOT_LEAF));
+  }
+  if (Xqf) {  // stage the tile from the row-major float copy: the row's 4 p bytes as 16-byte loads, 8 in flight
+    const int r = threadIdx.x;
+    if (r < rows) {
+      const float4* src = reinterpret_cast<const float4*>(Xqf + (r0 + r) * (int64_t)xfs);
+      float* xs = sxf + r * stride;
+      const int nq = (p + 3) >> 2;
+      for (int q0 = 0; q0 < nq; q0 += 8) {
+        float4 v[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) v[u] = (q0 + u < nq) ? __ldcs(src + q0 + u) : make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+        for (int u = 0; u < 8; ++u) {
+          const int f = 4 * (q0 + u);
+          if (f < p) xs[f] = v[u].x;
+          if (f + 1 < p) xs[f + 1] = v[u].y;
+          if (f + 2 < p) xs[f + 2] = v[u].z;
+          if (f + 3 < p) xs[f + 3] = v[u].w;
+        }
+      }
+    }
+  } else {  // stage the tile as floats: 8 column loads in flight per thread
+    const int r = threadIdx.x;
+    const bool ok = r < rows;
+    const double* src = Xq + r0 + (ok ? r : 0);
+    for (int f0 = 0; f0 < p; f0 += 8) {
+      double v[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) v[u] = (f0 + u < p) ? __ldcs(src + (int64_t)(f0 + u) * ldq) : 0.0;
+#pragma unroll
+      for (int u = 0; u < 8; ++u)
+        if (f0 + u < p && ok) sxf[r * stride + f0 + u] = __double2float_rn(v[u]);
+    }
+  }
+  __syncthreads();
+  if ((int)threadIdx.x >= rows) return;
+  const float* xs = sxf + threadIdx.x * stride;
+  const int64_t rr = r0 + threadIdx.x;
+  const double* xg = Xq + rr;
+  double acc = first ? 0.0 : yhat_sum[rr];
+  uint32_t nv = 0, nfb = 0;
+  uint32_t gs[NS];
+  ulonglong4 nd[NS];
+  int tnext = 0;
+  int nact = 0;
+  auto start = [&](int u) {
+    gs[u] = ~0u;
+    while (tnext < nt) {
+      const uint32_t rw = s_rw[tnext];
+      const ulonglong4 rn = s_rn[tnext];
+      ++tnext;
+      if (PROF) ++nv;
+      if (rw & ROOT_LEAF) {
+        acc += __longlong_as_double((long long)rn.x);
+        continue;
+      }
+      gs[u] = rw;
+      nd[u] = rn;
+      ++nact;
+      break;
+    }
+  };
+#pragma unroll
+  for (int u = 0; u < NS; ++u) start(u);
+  while (nact > 0) {
+#pragma unroll
+    for (int u = 0; u < NS; ++u) {
+      if (gs[u] == ~0u) continue;
+      const ulonglong4 G = nd[u];
+      if (gs[u] & G32_LEAF) {
+        acc += __longlong_as_double((long long)G.x);
+        --nact;
+        start(u);
+        continue;
+      }
+      const uint32_t w0 = (uint32_t)(G.x >> 32);
+      const uint32_t f0 = w0 & 0xffu;
+      const float xf0 = xs[f0], tf0 = __uint_as_float((uint32_t)G.x);
+      uint32_t right = xf0 > tf0;
+      if (__builtin_expect(xf0 == tf0 || xf0 != xf0, 0)) {  // float tie (or NaN): decide in fp64 (S5)
+        right = tie_right_fp64(xg, ldq, f0, nodes16, (uint32_t)(G.w >> 32));
+        if (PROF) ++nfb;
+      }
+      const unsigned long long c = right ? G.z : G.y;
+      if ((w0 >> (8 + right)) & 1u) {  // the chosen child is a leaf: c is its value
+        acc += __longlong_as_double((long long)c);
+        --nact;
+        start(u);
+        continue;
+      }
+      const uint32_t cw = (uint32_t)(c >> 32);
+      const uint32_t f1 = cw & 0xffu;
+      const float xf1 = xs[f1], tf1 = __uint_as_float((uint32_t)c);
+      uint32_t r1 = xf1 > tf1;
+      if (__builtin_expect(xf1 == tf1 || xf1 != xf1, 0)) {
+        r1 = tie_right_fp64(xg, ldq, f1, nodes16, (uint32_t)(G.w >> 32) + (cw >> 8) + right);
+        if (PROF) ++nfb;
+      }
+      const uint32_t ci = 2u * (right & ~(w0 >> 8) & 1u) + r1;  // going right past an internal L: skip its 2
+      uint32_t ns = (uint32_t)G.w + ci;
+      nd[u] = ldg256(g32 + ns);
+      if (PROF) ++nv;
+      if ((w0 >> (10 + ci)) & 1u) ns |= G32_LEAF;
+      gs[u] = ns;
+    }
+  }
+  if (PROF) {
+    const unsigned act = __activemask();
+    const uint32_t wv = __reduce_add_sync(act, nv), wf = __reduce_add_sync(act, nfb);
+    if ((threadIdx.x & 31) == __ffs(act) - 1) {
+      atomicAdd(visits, (unsigned long long)wv);
+      atomicAdd(visits + 1, (unsigned long long)wf);
+    }
+  }
+  yhat_sum[rr] = acc;
+  if (last && yhat) yhat[rr] = acc * inv_t;
+}
+
 __global__ void __launch_bounds__(PT) k_predict_gmem(const Node16* __restrict__ nodes, const int64_t* __restrict__ off,
                                                      int32_t ntrees, const double* __restrict__ Xq, int64_t ldq,
                                                      int64_t m, double* yhat_sum, double* yhat, double inv_t,
@@ -584,6 +871,84 @@ const uint2* nodes8_get(bf_forest* f, cudaStream_t s) {
   return f->nodes8_state > 0 ? f->d_nodes8 : nullptr;
 }
 
+
+const ulonglong4* g32_get(bf_forest* f, cudaStream_t s) {
+  if (f->g32_state == 0) {
+    const int32_t nt = f->info.tree_end - f->info.tree_begin;
+    const int64_t total = f->info.total_nodes;
+    f->g32_state = -1;
+    if (f->info.p <= 256 && total > 0 && nt > 0 && total < (int64_t(1) << 31)) {
+      DBuf<int32_t> anc0(total, s), anc1(total, s);
+      DBuf<uint8_t> bit0(total, s), bit1(total, s);
+      DBuf<int> flag(2, s);
+      const dim3 tg(64, (unsigned)nt);
+      {
+        KScope ks_("k_g32_build", s, 0.0);
+        k_g32_parent<<<tg, 256, 0, s>>>(f->d_nodes, f->d_tree_off, anc0.p, bit0.p);
+      }
+      BF_CUDA_CHECK(cudaGetLastError());
+      int32_t* a = anc0.p;
+      int32_t* a2 = anc1.p;
+      uint8_t* b = bit0.p;
+      uint8_t* b2 = bit1.p;
+      for (int it = 0; it < 40; ++it) {  // depth < 2^40: ends when every node's ancestor link is the root's
+        int more = 0;
+        BF_CUDA_CHECK(cudaMemsetAsync(flag.p, 0, sizeof(int), s));
+        {
+          KScope ks_("k_g32_build", s, 0.0);
+          k_g32_jump<<<(unsigned)ceil_div(total, 256), 256, 0, s>>>(a, b, a2, b2, total, flag.p);
+        }
+        BF_CUDA_CHECK(cudaMemcpyAsync(&more, flag.p, sizeof(int), cudaMemcpyDeviceToHost, s));
+        BF_CUDA_CHECK(cudaStreamSynchronize(s));
+        std::swap(a, a2);
+        std::swap(b, b2);
+        if (!more) break;
+      }
+      uint32_t* cnt = reinterpret_cast<uint32_t*>(a2);  // the other ancestor buffer is free now
+      uint32_t* ex = reinterpret_cast<uint32_t*>(a);
+      DBuf<int64_t> tslot((size_t)nt + 1, s);
+      {
+        KScope ks_("k_g32_build", s, 0.0);
+        k_g32_count<<<tg, 256, 0, s>>>(f->d_nodes, f->d_tree_off, b, cnt);
+      }
+      DBuf<uint32_t> exb(total, s);
+      scan_exclusive(cnt, exb.p, total, s);
+      uint32_t last_ex = 0, last_cnt = 0;
+      BF_CUDA_CHECK(cudaMemcpyAsync(&last_ex, exb.p + total - 1, 4, cudaMemcpyDeviceToHost, s));
+      BF_CUDA_CHECK(cudaMemcpyAsync(&last_cnt, cnt + total - 1, 4, cudaMemcpyDeviceToHost, s));
+      BF_CUDA_CHECK(cudaStreamSynchronize(s));
+      const int64_t nslots = (int64_t)last_ex + last_cnt;
+      {
+        KScope ks_("k_g32_build", s, 0.0);
+        k_g32_slots<<<tg, 256, 0, s>>>(f->d_nodes, f->d_tree_off, b, exb.p, ex, tslot.p);
+      }
+      f->d_g32 = (ulonglong4*)dev_alloc(sizeof(ulonglong4) * (size_t)nslots, s);
+      f->d_g32_root = (uint32_t*)dev_alloc(sizeof(uint32_t) * (size_t)nt, s);
+      BF_CUDA_CHECK(cudaMemsetAsync(flag.p + 1, 0, sizeof(int), s));
+      {
+        KScope ks_("k_g32_build", s, 0.0);
+        k_g32_emit<<<tg, 256, 0, s>>>(f->d_nodes, f->d_tree_off, b, exb.p, ex, f->d_g32, f->d_g32_root, flag.p + 1);
+      }
+      BF_CUDA_CHECK(cudaGetLastError());
+      f->g32_off.assign((size_t)nt + 1, 0);
+      int hbad = 0;
+      BF_CUDA_CHECK(cudaMemcpyAsync(f->g32_off.data(), tslot.p, sizeof(int64_t) * nt, cudaMemcpyDeviceToHost, s));
+      BF_CUDA_CHECK(cudaMemcpyAsync(&hbad, flag.p + 1, sizeof(int), cudaMemcpyDeviceToHost, s));
+      BF_CUDA_CHECK(cudaStreamSynchronize(s));
+      f->g32_off[nt] = nslots;
+      if (hbad || nslots >= (int64_t(1) << 31)) {
+        dev_free(f->d_g32, s);
+        dev_free(f->d_g32_root, s);
+        f->d_g32 = nullptr;
+        f->d_g32_root = nullptr;
+      } else {
+        f->g32_state = 1;
+      }
+    }
+  }
+  return f->g32_state > 0 ? f->d_g32 : nullptr;
+}
+
 void predict_impl(const bf_forest* f, const double* Xq_in, int64_t ldq, int64_t m, double* ys_in, double* yh_in,
                   int32_t ntree_total, cudaStream_t s) {
   if (m == 0) return;
@@ -612,8 +977,45 @@ void predict_impl(const bf_forest* f, const double* Xq_in, int64_t ldq, int64_t 
     smax8 = std::min(smax8, std::min(dyn_smem_limit(k_predict8s<true, 12>), dyn_smem_limit(k_predict8s<false, 12>)));
   }
   static const int slots = getenv("BF_PREDICT_SLOTS") ? atoi(getenv("BF_PREDICT_SLOTS")) : 6;  // measured: 6 < 8 < 12 (profiles/r02o)
-  static const int pv = getenv("BF_PREDICT_V") ? atoi(getenv("BF_PREDICT_V")) : 2;
-  if (n8 && smem8 <= (size_t)smax8) {
+  // walk kernel: 3 = G32 groups, 2 = Node8 with the block's roots in shared memory, 1 = Node8 (read per call,
+  // so tests can compare the paths on one forest)
+  const int pv = getenv("BF_PREDICT_V") ? atoi(getenv("BF_PREDICT_V")) : 3;
+  static int smax32 = 0;
+  if (!smax32)
+    smax32 = std::min(std::min(dyn_smem_limit(k_predict32<true, 4>), dyn_smem_limit(k_predict32<false, 4>)),
+                      std::min(dyn_smem_limit(k_predict32<true, 6>), dyn_smem_limit(k_predict32<false, 6>)));
+  const ulonglong4* g32 = (pv == 3 && !(force16 && force16[0] == '1')) ? g32_get(const_cast<bf_forest*>(f), s) : nullptr;
+  if (g32 && smem8 <= (size_t)smax32) {
+    // G32 groups: tree blocks of <= 48 MB of slots (one 256-bit load per two levels)
+    double* ysum = ys_in ? (double*)ys.dptr : nullptr;
+    DBuf<double> ytmp;
+    if (!ysum) {
+      ytmp.alloc(m, s);
+      ysum = ytmp.p;
+    }
+    static const int slots32 = getenv("BF_PREDICT32_SLOTS") ? atoi(getenv("BF_PREDICT32_SLOTS")) : 4;
+    const int64_t block_bytes = predict_block_bytes(48ll << 20);
+    // with more than one tree block the row tiles are staged once per block: from a row-major float copy of
+    // the query batch (half the bytes of the fp64 columns, contiguous per row), built once per call
+    static const int use_xf = getenv("BF_PREDICT_XF") ? atoi(getenv("BF_PREDICT_XF")) : 0;  // measured: no gain (189 vs 188 ms per 200 C4 trees)
+    const int xfs = (p + 3) & ~3;
+    DBuf<float> Xqf;
+    if (use_xf && f->g32_off[nt] * (int64_t)sizeof(ulonglong4) > block_bytes) {
+      Xqf.alloc((size_t)m * xfs, s);
+      xf_rows_impl((const double*)Xs.dptr, ldq, m, p, Xqf.p, xfs, s);
+    }
+    for (int32_t t0 = 0; t0 < nt;) {
+      int32_t t1 = t0 + 1;
+      while (t1 < nt && t1 - t0 < RT8 && (f->g32_off[t1 + 1] - f->g32_off[t0]) * (int64_t)sizeof(ulonglong4) <= block_bytes) ++t1;
+      KScope ks_("k_predict32", s, 0.0);
+      auto kern = vis.p ? (slots32 == 6 ? k_predict32<true, 6> : k_predict32<true, 4>)
+                        : (slots32 == 6 ? k_predict32<false, 6> : k_predict32<false, 4>);
+      kern<<<(unsigned)ceil_div(m, PT8), PT8, smem8, s>>>(g32, f->d_nodes, f->d_g32_root, t0, t1, t0 == 0, t1 >= nt,
+                                                         (const double*)Xs.dptr, ldq, Xqf.p, xfs, m, p, ysum,
+                                                         yh_in ? (double*)yh.dptr : nullptr, inv_t, vis.p);
+      t0 = t1;
+    }
+  } else if (n8 && smem8 <= (size_t)smax8) {
     // tree blocks of <= 32 MB of Node8 (L2-resident while every row walks them)
     double* ysum = ys_in ? (double*)ys.dptr : nullptr;
     DBuf<double> ytmp;
@@ -679,9 +1081,10 @@ void predict_impl(const bf_forest* f, const double* Xq_in, int64_t ldq, int64_t 
     const unsigned long long hv = hv2[0];
     prof_add_bytes("predict_node_visits", (double)hv);
     prof_add_bytes("predict_fp64_fallbacks", (double)hv2[1]);
-    const bool used8 = n8 && smem8 <= (size_t)smax8;
-    prof_add_bytes(used8 ? "k_predict8" : smem <= (size_t)smax ? "k_predict_smem" : "k_predict_gmem",
-                   (used8 ? 8.0 : 16.0) * (double)hv +
+    const bool used32 = g32 && smem8 <= (size_t)smax32;
+    const bool used8 = !used32 && n8 && smem8 <= (size_t)smax8;
+    prof_add_bytes(used32 ? "k_predict32" : used8 ? "k_predict8" : smem <= (size_t)smax ? "k_predict_smem" : "k_predict_gmem",
+                   (used32 ? 32.0 : used8 ? 8.0 : 16.0) * (double)hv +
                        (double)m * (8.0 * p + 16.0 * ((ys_in != nullptr) + (yh_in != nullptr))));
   }
   if (ys_in) ys.finish(s);

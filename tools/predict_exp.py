@@ -30,12 +30,15 @@ print("trees", T, "nodes", f.info.total_nodes, flush=True)
 ref = None
 CASES = [("node16_blk48", {"BF_PREDICT_NODE16": "1"})]
 CASES += [(f"node8_blk{b}", {"BF_PREDICT_BLOCK_BYTES": str(b << 20)}) for b in (16, 24, 32, 48, 64)]
-if os.environ.get("PEXP_CASES"):
+if os.environ.get("PEXP_CASES") == "env":  # one case: the caller's environment (BF_PREDICT_V, block bytes, ...)
+    CASES = [("env", None)]
+elif os.environ.get("PEXP_CASES"):
     CASES = [c for c in CASES if c[0] in os.environ["PEXP_CASES"].split(",")]
 for name, env in CASES:
-    for k in ("BF_PREDICT_NODE16", "BF_PREDICT_BLOCK_BYTES"):
-        os.environ.pop(k, None)
-    os.environ.update(env)
+    if env is not None:
+        for k in ("BF_PREDICT_NODE16", "BF_PREDICT_BLOCK_BYTES"):
+            os.environ.pop(k, None)
+        os.environ.update(env)
     ys, _ = f.predict(Qd, ntree_total=T)
     torch.cuda.synchronize()
     a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
