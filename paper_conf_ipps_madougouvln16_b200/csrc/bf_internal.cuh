@@ -206,6 +206,13 @@ constexpr uint32_t ROOT_LEAF = 0x80000000u;
 __device__ __forceinline__ double leaf8(uint2 v) { return __hiloint2double((int)v.y, (int)v.x); }
 __device__ __forceinline__ uint32_t n8_feature(uint2 w) { return (w.y >> N8_REL_BITS) & ((1u << N8_FEAT_BITS) - 1u); }
 __device__ __forceinline__ uint32_t n8_rel(uint2 w) { return w.y & ((1u << N8_REL_BITS) - 1u); }
+// Two-level 32-byte groups (predict.cu g32_get; layout documented there): one 256-bit read-only load per group.
+constexpr uint32_t G32_LEAF = 0x80000000u;  // walk state: the slot being loaded is a leaf
+__device__ __forceinline__ ulonglong4 ldg256(const ulonglong4* p) {
+  ulonglong4 v;
+  asm volatile("ld.global.nc.v4.u64 {%0,%1,%2,%3}, [%4];" : "=l"(v.x), "=l"(v.y), "=l"(v.z), "=l"(v.w) : "l"(p));
+  return v;
+}
 
 }  // namespace bf
 

@@ -1890,10 +1890,13 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
 
   // ================= medium levels (a > TINY): level-synchronous inside the CTA
   long long mclk[3] = {0, 0, 0};  // medium phase: scan+finalize, next level, partition (thread 0, stats only)
+  long long mfin = 0;             // of which finalize (warp per node after the item barrier)
+  int n_mlev = 0;                 // medium levels
   while (s_ncur > 0) {
     const long long mc0 = clock64();
     const int ncur = s_ncur;
     n_med += ncur;
+    ++n_mlev;
     // (node, drawn predictor) items over all warps; per-item winners in the scratch area; one warp per node
     // reduces its items (lowest predictor on equal keys) and finalizes the split.  Nodes go in groups whose
     // items fit the scratch area (and whose draws fit the per-warp feature slots).
@@ -2022,6 +2025,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         }
       }
       __syncthreads();
+      const long long mf0 = clock64();
       if (wid < nn) {
         const int i = n0 + wid;
         MNode nd = curl[i];
@@ -2096,6 +2100,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         }
       }
       __syncthreads();
+      mfin += clock64() - mf0;
     }
     const long long mc1 = clock64();
     // ---- next medium level (block scan) and tiny roots (work queue; processed after the medium levels)
@@ -2736,8 +2741,10 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       if (DEFER && rdef[l] != 0xffffu) {  // S4.7 node value from the record's row mask over its tiny root
         const int rl = rdef[l];
         uint64_t mk = (uint64_t)__double_as_longlong(rc.value);
+        const int nb = __popcll(mk);
         double sw = 0.0;
-        while (mk) {
+#pragma unroll 4
+        for (int c = 0; c < nb; ++c) {  // countable: the row loads of several members are in flight together
           sw += wyd[list[rl + __ffsll((long long)mk) - 1] & 0xffffu];
           mk &= mk - 1;
         }
@@ -2757,6 +2764,8 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       atomicAdd(&g.stats[13], (unsigned long long)mclk[0]);
       atomicAdd(&g.stats[14], (unsigned long long)mclk[1]);
       atomicAdd(&g.stats[15], (unsigned long long)mclk[2]);
+      atomicAdd(&g.stats[22], (unsigned long long)n_mlev);
+      atomicAdd(&g.stats[23], (unsigned long long)mfin);
       atomicAdd(&g.stats[4], (unsigned long long)n_med);
       atomicAdd(&g.stats[5], 1ull);
       atomicAdd(&g.stats[6], (unsigned long long)a0);
@@ -3435,7 +3444,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
             const double c = (double)h[5];
             fprintf(stderr, "[subtree tiny] draw=%.0f groups=%.0f per tiny node\n", h[11] / (double)(h[7] ? h[7] : 1), h[12] / (double)(h[7] ? h[7] : 1));
             fprintf(stderr, "[subtree tiny group] per tiny node: stage=%.0f passA=%.0f segscan=%.0f passB=%.0f wmax=%.0f passC=%.0f\n", h[21] / (double)(h[7] ? h[7] : 1), h[16] / (double)(h[7] ? h[7] : 1), h[17] / (double)(h[7] ? h[7] : 1), h[18] / (double)(h[7] ? h[7] : 1), h[19] / (double)(h[7] ? h[7] : 1), h[20] / (double)(h[7] ? h[7] : 1));
-            fprintf(stderr, "[subtree medium] per cta: scan+finalize=%.0f next=%.0f partition=%.0f cycles\n", h[13] / (double)(h[5] ? h[5] : 1), h[14] / (double)(h[5] ? h[5] : 1), h[15] / (double)(h[5] ? h[5] : 1));
+            fprintf(stderr, "[subtree medium] per cta: scan+finalize=%.0f (finalize %.0f) next=%.0f partition=%.0f cycles, %.2f levels\n", h[13] / (double)(h[5] ? h[5] : 1), h[23] / (double)(h[5] ? h[5] : 1), h[14] / (double)(h[5] ? h[5] : 1), h[15] / (double)(h[5] ? h[5] : 1), h[22] / (double)(h[5] ? h[5] : 1));
             fprintf(stderr, "[subtree] A=%d ctas=%llu mean_a0=%.1f cyc/cta: load=%.0f medium=%.0f tiny=%.0f flush=%.0f | medium nodes/cta=%.1f tiny nodes/cta=%.1f nodes/cta=%.1f warp-cyc in tiny/cta=%.0f busy=%.0f (%.0f per tiny node)\n",
                     A, h[5], h[6] / c, h[0] / c, h[1] / c, h[2] / c, h[3] / c, h[4] / c, h[7] / c, h[9] / c, h[8] / c,
                     h[10] / c, h[10] / (double)(h[7] ? h[7] : 1));

@@ -628,6 +628,238 @@ __global__ void __launch_bounds__(IPT) k_importance8(Imp8Args g8) {
     if (sacc[m] != 0.0) atomicAdd(&g.d_slots[(int64_t)i * g.p + m], sacc[m]);
 }
 
+
+// k_importance32: k_importance8's walks on the two-level 32-byte groups (predict.cu g32_get): one 256-bit load
+// decides two levels.  A permuted re-walk starts at the first node of the path that tests its predictor m: a
+// group's node k (even depth), or the group's chosen child c (odd depth; then k does not test m, so the walk
+// keeps the original decision at k).  Decisions are exactly S5's (float, then fp64 on a float tie: the row's
+// fp64 x from X, or the fp64 permuted value, against Node16's threshold by id).  p <= 64 (one bit per predictor
+// in the first-occurrence mask; wider forests take k_importance8).
+struct Imp32Args {
+  ImpArgs a;
+  const float* Xf;
+  int xfs;
+  const ulonglong4* g32;
+  const uint32_t* roots32;   // per local tree: root slot | ROOT_LEAF
+  unsigned long long* prof;  // profile mode: [0] group loads, [1] permuted re-walks, else NULL
+};
+
+template <int IL>
+__global__ void __launch_bounds__(IPT) k_importance32(Imp32Args g3) {
+  const ImpArgs& g = g3.a;
+  extern __shared__ double ism[];  // sacc[p] | float x tile IPT x (p|1)
+  double* sacc = ism;
+  const int stride = g.p | 1;
+  float* sx = reinterpret_cast<float*>(ism + ((g.p + 1) & ~1));
+  __shared__ double serr[IPT / 32];
+  const int b = blockIdx.y;
+  const int32_t i = g.i0 + b;
+  const int64_t n_o = g.nout[b];
+  const int64_t a0 = (int64_t)blockIdx.x * IPT;
+  if (a0 >= n_o) return;  // uniform per CTA
+  for (int m = threadIdx.x; m < g.p; m += IPT) sacc[m] = 0.0;
+  const uint32_t* Ob = g.O + (int64_t)b * g.n;
+  const int64_t a = a0 + threadIdx.x;
+  const bool act = a < n_o;
+  const uint32_t r = act ? Ob[a] : Ob[a0];
+  {  // stage the tile from the row-major float copy: the row's 4 p bytes as 16-byte loads, 8 in flight
+    float* xs = sx + threadIdx.x * stride;
+    const float4* src = reinterpret_cast<const float4*>(g3.Xf + (int64_t)r * g3.xfs);
+    const int nq = (g.p + 3) >> 2;
+    for (int q0 = 0; q0 < nq; q0 += 8) {
+      float4 v[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) v[u] = (q0 + u < nq) ? __ldg(src + q0 + u) : make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const int f = 4 * (q0 + u);
+        if (f < g.p) xs[f] = v[u].x;
+        if (f + 1 < g.p) xs[f + 1] = v[u].y;
+        if (f + 2 < g.p) xs[f + 2] = v[u].z;
+        if (f + 3 < g.p) xs[f + 3] = v[u].w;
+      }
+    }
+  }
+  __syncthreads();
+  double err0 = 0.0;
+  if (act) {
+    const float* xs = sx + threadIdx.x * stride;
+    const double* xg = g.X + r;
+    const ulonglong4* G32 = g3.g32;
+    const Node16* n16 = g.nodes;
+    const uint32_t rw = __ldg(g3.roots32 + i);
+    const uint32_t root = rw & ~ROOT_LEAF;
+    const double yr = g.y[r];
+    uint32_t nld = 1, nrw = 0;
+    // S5 decision (1 = right) at a node of feature f, float threshold tf, Node16 id; predictor pm takes (xpf, xpd)
+    auto decide = [&](uint32_t f, float tf, uint32_t id, int pm, float xpf, double xpd) -> uint32_t {
+      const bool pf = (int)f == pm;
+      const float xf = pf ? xpf : xs[f];
+      uint32_t right = xf > tf;
+      if (xf == tf || xf != xf) {  // float tie: decide in fp64 (S5)
+        const double xd = pf ? xpd : __ldg(xg + (int64_t)f * g.ldx);
+        right = !(xd <= __ldg(&n16[id].v));
+      }
+      return right;
+    };
+    auto dec_k = [&](const ulonglong4& G, int pm, float xpf, double xpd) -> uint32_t {
+      return decide((uint32_t)(G.x >> 32) & 0xffu, __uint_as_float((uint32_t)G.x), (uint32_t)(G.w >> 32), pm, xpf, xpd);
+    };
+    auto dec_c = [&](const ulonglong4& G, uint32_t r0, int pm, float xpf, double xpd) -> uint32_t {
+      const unsigned long long c = r0 ? G.z : G.y;
+      const uint32_t cw = (uint32_t)(c >> 32);
+      return decide(cw & 0xffu, __uint_as_float((uint32_t)c), (uint32_t)(G.w >> 32) + (cw >> 8) + r0, pm, xpf, xpd);
+    };
+    // the grandchild slot after decisions r0, r1 (G32_LEAF set if it holds a leaf value)
+    auto next_slot = [&](const ulonglong4& G, uint32_t r0, uint32_t r1) -> uint32_t {
+      const uint32_t w0 = (uint32_t)(G.x >> 32);
+      const uint32_t ci = 2u * (r0 & ~(w0 >> 8) & 1u) + r1;
+      return ((uint32_t)G.w + ci) | (((w0 >> (10 + ci)) & 1u) ? G32_LEAF : 0u);
+    };
+    auto child_leaf = [&](const ulonglong4& G, uint32_t r0) -> bool { return ((uint32_t)(G.x >> 32) >> (8 + r0)) & 1u; };
+    // original walk
+    double f0v;
+    if (rw & ROOT_LEAF) {
+      f0v = __longlong_as_double((long long)ldg256(G32 + root).x);
+    } else {
+      ulonglong4 G = ldg256(G32 + root);
+      for (;;) {
+        const uint32_t r0 = dec_k(G, -1, 0.f, 0.0);
+        if (child_leaf(G, r0)) {
+          f0v = __longlong_as_double((long long)(r0 ? G.z : G.y));
+          break;
+        }
+        const uint32_t ns = next_slot(G, r0, dec_c(G, r0, -1, 0.f, 0.0));
+        const ulonglong4 Gn = ldg256(G32 + (ns & ~G32_LEAF));
+        ++nld;
+        if (ns & G32_LEAF) {
+          f0v = __longlong_as_double((long long)Gn.x);
+          break;
+        }
+        G = Gn;
+      }
+    }
+    const double d0 = yr - f0v;
+    err0 = d0 * d0;
+    atomicAdd(&g.oob_sum[r], f0v);
+    atomicAdd(&g.oob_cnt[r], 1);
+    // permuted walks from the first occurrence of each predictor on the path, IL at a time
+    if (!(rw & ROOT_LEAF)) {
+      uint64_t seen = 0;
+      ulonglong4 G = ldg256(G32 + root);
+      uint32_t sub = 0, r0c = 0;  // cursor: at the group's node k (sub 0) or at its chosen child r0c (sub 1)
+      bool at_leaf = false;
+      for (;;) {
+        int cnt = 0;
+        int qm[IL];
+        ulonglong4 qG[IL];
+        uint32_t qs[IL];  // 0: start at the group's node k; 1 | r0 << 1: start at its child r0
+#pragma unroll
+        for (int u = 0; u < IL; ++u) qs[u] = 0;
+        while (!at_leaf && cnt < IL) {
+          const uint32_t m = sub == 0 ? ((uint32_t)(G.x >> 32) & 0xffu) : ((uint32_t)((r0c ? G.z : G.y) >> 32) & 0xffu);
+          if (!((seen >> m) & 1ull)) {
+            seen |= 1ull << m;
+#pragma unroll
+            for (int u = 0; u < IL; ++u)
+              if (u == cnt) {
+                qm[u] = (int)m;
+                qG[u] = G;
+                qs[u] = sub ? (1u | (r0c << 1)) : 0u;
+              }
+            ++cnt;
+          }
+          if (sub == 0) {
+            r0c = dec_k(G, -1, 0.f, 0.0);
+            if (child_leaf(G, r0c)) at_leaf = true;
+            else sub = 1;
+          } else {
+            const uint32_t ns = next_slot(G, r0c, dec_c(G, r0c, -1, 0.f, 0.0));
+            if (ns & G32_LEAF) {
+              at_leaf = true;
+            } else {
+              G = ldg256(G32 + ns);
+              ++nld;
+              sub = 0;
+            }
+          }
+        }
+        if (cnt == 0) break;
+        nrw += cnt;
+        double xm[IL];
+        float xmf[IL];
+        bool live[IL], lpend[IL];
+#pragma unroll
+        for (int u = 0; u < IL; ++u) {
+          live[u] = u < cnt;
+          lpend[u] = false;
+          xm[u] = 0.0;
+          if (live[u]) {
+            const int64_t pa = __ldg(g.perm + ((int64_t)b * g.p + qm[u]) * g.n + a);
+            xm[u] = __ldg(g.X + (int64_t)qm[u] * g.ldx + Ob[pa]);
+          } else {
+            qm[u] = -1;
+          }
+          xmf[u] = __double2float_rn(xm[u]);
+        }
+        double val[IL];
+        bool any = true;
+        while (any) {
+          any = false;
+#pragma unroll
+          for (int u = 0; u < IL; ++u)
+            if (live[u]) {
+              const ulonglong4 Gu = qG[u];
+              if (lpend[u]) {  // the slot just loaded is a leaf
+                val[u] = __longlong_as_double((long long)Gu.x);
+                live[u] = false;
+                continue;
+              }
+              const uint32_t r0 = (qs[u] & 1u) ? (qs[u] >> 1) : dec_k(Gu, qm[u], xmf[u], xm[u]);
+              if (child_leaf(Gu, r0)) {
+                val[u] = __longlong_as_double((long long)(r0 ? Gu.z : Gu.y));
+                live[u] = false;
+                continue;
+              }
+              const uint32_t ns = next_slot(Gu, r0, dec_c(Gu, r0, qm[u], xmf[u], xm[u]));
+              qG[u] = ldg256(G32 + (ns & ~G32_LEAF));
+              ++nld;
+              qs[u] = 0;
+              lpend[u] = (ns & G32_LEAF) != 0;
+              any = true;
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < IL; ++u)
+          if (u < cnt) {
+            const double d1 = yr - val[u];
+            const double diff = d1 * d1 - err0;
+            if (diff != 0.0) atomicAdd(&sacc[qm[u]], diff);
+          }
+      }
+    }
+    if (g3.prof) {  // one atomic pair per warp
+      const unsigned act_m = __activemask();
+      const uint32_t wl = __reduce_add_sync(act_m, nld), wr = __reduce_add_sync(act_m, nrw);
+      if ((threadIdx.x & 31) == __ffs(act_m) - 1) {
+        atomicAdd(&g3.prof[0], (unsigned long long)wl);
+        atomicAdd(&g3.prof[1], (unsigned long long)wr);
+      }
+    }
+  }
+  // e_t
+  for (int o = 16; o > 0; o >>= 1) err0 += __shfl_down_sync(0xffffffffu, err0, o);
+  if ((threadIdx.x & 31) == 0) serr[threadIdx.x >> 5] = err0;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double s = 0.0;
+    for (int j = 0; j < IPT / 32; ++j) s += serr[j];
+    if (s != 0.0) atomicAdd(&g.e_t[i], s);
+  }
+  for (int m = threadIdx.x; m < g.p; m += IPT)
+    if (sacc[m] != 0.0) atomicAdd(&g.d_slots[(int64_t)i * g.p + m], sacc[m]);
+}
+
 __global__ void k_divide(double* d_slots, const int64_t* nout_t, int32_t T, int p) {
   const int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (k >= (int64_t)T * p) return;
@@ -759,10 +991,21 @@ void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, co
   if (wide) smem = sizeof(double) * ((size_t)((p + 1) & ~1) + (size_t)IPT_WIDE * (size_t)(p | 1));
   BF_REQUIRE(smem <= (size_t)ismax, BF_ENOTIMPL, "bf_oob_importance: p too large for the shared-memory row tile");
   const char* force16 = getenv("BF_PREDICT_NODE16");  // same switch as predict: keep the Node16 walks
-  const uint2* n8 = (force16 && force16[0] == '1') ? nullptr : nodes8_get(const_cast<bf_forest*>(f), s);
   const size_t smem8 = sizeof(double) * (size_t)((p + 1) & ~1) + sizeof(float) * (size_t)IPT * (size_t)(p | 1);
   static int ismax8 = 0;
   if (!ismax8) ismax8 = dyn_smem_limit(k_importance8);
+  // walks on the two-level groups when the forest has them and p <= 64 (BF_PREDICT_V=2 keeps the Node8 walks)
+  static int ismax32 = 0;
+  if (!ismax32)
+    ismax32 = std::min(std::min(dyn_smem_limit(k_importance32<2>), dyn_smem_limit(k_importance32<3>)),
+                       dyn_smem_limit(k_importance32<4>));
+  // permuted walks interleaved per thread (measured per 200 C4 trees: 3 -> 119 ms, 4 -> 142 ms)
+  static const int il32 = getenv("BF_IMP32_ILP") ? atoi(getenv("BF_IMP32_ILP")) : 3;
+  const char* pvs = getenv("BF_PREDICT_V");
+  const bool want32 = p <= 64 && !(force16 && force16[0] == '1') && !(pvs && atoi(pvs) != 3);
+  const ulonglong4* g32 = want32 ? g32_get(const_cast<bf_forest*>(f), s) : nullptr;
+  const uint2* n8 = (force16 && force16[0] == '1') || (g32 && smem8 <= (size_t)ismax32)
+                        ? nullptr : nodes8_get(const_cast<bf_forest*>(f), s);
   DBuf<unsigned long long> prof;
   if (prof_enabled()) {
     prof.alloc(2, s);
@@ -830,7 +1073,26 @@ void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, co
     g.e_t = e_t;
     g.perm = perm.p;
     // OOB rows per tree <= n; grid sized for n (CTAs past n_o exit early)
-    if (n8 && smem8 <= (size_t)ismax8) {
+    if (g32 && smem8 <= (size_t)ismax32) {
+      if (!Xf.p) {  // once per call: the row-major float copy the CTAs stage their OOB rows from
+        Xf.alloc((size_t)n * xfs, s);
+        xf_rows_impl(X, ldx, n, p, Xf.p, xfs, s);
+      }
+      Imp32Args g3;
+      g3.a = g;
+      g3.Xf = Xf.p;
+      g3.xfs = xfs;
+      g3.g32 = g32;
+      g3.roots32 = f->d_g32_root;
+      g3.prof = prof.p;
+      KScope ks_("k_importance32", s, 0.0);
+      if (il32 == 2)
+        k_importance32<2><<<dim3((unsigned)ceil_div(n, IPT), Bc), IPT, smem8, s>>>(g3);
+      else if (il32 == 4)
+        k_importance32<4><<<dim3((unsigned)ceil_div(n, IPT), Bc), IPT, smem8, s>>>(g3);
+      else
+        k_importance32<3><<<dim3((unsigned)ceil_div(n, IPT), Bc), IPT, smem8, s>>>(g3);
+    } else if (n8 && smem8 <= (size_t)ismax8) {
       if (!Xf.p) {  // once per call: the row-major float copy the CTAs stage their OOB rows from
         Xf.alloc((size_t)n * xfs, s);
         xf_rows_impl(X, ldx, n, p, Xf.p, xfs, s);
@@ -863,7 +1125,9 @@ void oob_importance_impl(const bf_forest* f, const double* X_in, int64_t ldx, co
     for (int64_t v : hno) units += (double)v;
     // per (tree, OOB row): float row gather 4p + y 8 + O index 4 + oob sum/count 12; per re-walk: pi 4 + x 8;
     // per node load 8 (compact nodes)
-    prof_add_bytes("k_importance8", units * (4.0 * p + 24.0) + (double)hp[1] * 12.0 + (double)hp[0] * 8.0);
+    const bool used32 = g32 && smem8 <= (size_t)ismax32;
+    prof_add_bytes(used32 ? "k_importance32" : "k_importance8",
+                   units * (4.0 * p + 24.0) + (double)hp[1] * 12.0 + (double)hp[0] * (used32 ? 32.0 : 8.0));
     prof_add_bytes("importance_node_loads", (double)hp[0]);
     prof_add_bytes("importance_rewalks", (double)hp[1]);
   }

@@ -351,7 +351,6 @@ __global__ void __launch_bounds__(PT8, 6) k_predict8s(const uint2* __restrict__ 
 // two levels of a walk (S5: x <= thr goes left), with the same float-then-fp64 comparison as Node8.
 // Slots: depth parity by pointer jumping over parent links, then per group the number of grandchild slots,
 // one exclusive scan (the root of every tree takes one extra slot first), and the slots written top-down.
-constexpr uint32_t G32_LEAF = 0x80000000u;  // walk state: the slot being loaded is a leaf
 
 __global__ void k_g32_parent(const Node16* __restrict__ nodes, const int64_t* __restrict__ off, int32_t* anc,
                              uint8_t* bit) {
@@ -481,11 +480,6 @@ __global__ void k_g32_emit(const Node16* __restrict__ nodes, const int64_t* __re
   }
 }
 
-__device__ __forceinline__ ulonglong4 ldg256(const ulonglong4* p) {
-  ulonglong4 v;
-  asm volatile("ld.global.nc.v4.u64 {%0,%1,%2,%3}, [%4];" : "=l"(v.x), "=l"(v.y), "=l"(v.z), "=l"(v.w) : "l"(p));
-  return v;
-}
 
 // k_predict8s on G32 groups: a slot (walk in flight) holds the 32 bytes of its current group; per step it
 // decides the group's node and the chosen child, then loads the grandchild's slot (a leaf slot ends the walk

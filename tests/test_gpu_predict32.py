@@ -1,4 +1,4 @@
-"""GPU parity of the two-level 32-byte group walk (k_predict32, predict.cu; BF_PREDICT_V=3).
+"""GPU parity of the two-level 32-byte group walks (k_predict32, predict.cu; k_importance32, importance.cu).
 
 A G32 group holds an internal node at even depth and its two children; one 256-bit load decides two levels
 and the grandchild slot is loaded next.  The walk must take exactly the S5 path (P:95 step 3):
@@ -138,3 +138,33 @@ def test_predict32_configs_vs_oracle(cfg):
     Q = S.gen_query(X, 4099)
     a, _ = _predict(gf, Q, T, G32)
     assert rel_close(a, of.predict_sum(Q), 1e-9)
+
+
+@pytest.mark.parametrize("env", [{}, {"BF_PREDICT_V": "2"}])
+@pytest.mark.parametrize("mtry,ns", [(0, 5), (6, 1)])
+def test_importance32_float_ties_vs_oracle(env, mtry, ns):
+    """OOB importance on the G32 groups (default for p <= 64; BF_PREDICT_V=2: the Node8 walks): a permuted walk
+    starts at a group's node or at its chosen child, the fp64 tie decisions use the permuted fp64 value; the
+    slots, OOB sums and counts agree with the oracle (S6-S7 tolerances) on tie-heavy data."""
+    import os
+    X, y = _float_tie_data(n=2000, seed=21 + ns)
+    T = 12
+    of = O.fit(X, y, ntree=T, mtry=mtry, nodesize=ns, seed=5, nthreads=4)
+    gf = bf.fit(dev(X), dev(y), ntree=T, mtry=mtry, nodesize=ns, seed=5)
+    old = {k: os.environ.get(k) for k in env}
+    try:
+        os.environ.update(env)
+        r = gf.oob_importance(dev(X), dev(y))
+    finally:
+        for k, v in old.items():
+            if v is None:
+                os.environ.pop(k, None)
+            else:
+                os.environ[k] = v
+    ro = of.oob_importance(X, y)
+    assert np.array_equal(r["nout_t"].cpu().numpy(), ro["nout_t"])
+    assert np.array_equal(r["oob_cnt"].cpu().numpy(), ro["oob_cnt"])
+    assert rel_close(r["oob_sum"].cpu().numpy(), ro["oob_sum"], 1e-9)
+    assert rel_close(r["e_t"].cpu().numpy(), ro["e_t"], 1e-9)
+    assert rel_close(r["d_slots"].cpu().numpy(), ro["d_slots"], 1e-6, atol_scale=1e-9)
+    assert np.all(r["d_slots"].cpu().numpy()[ro["d_slots"] == 0.0] == 0.0)
