@@ -11,7 +11,7 @@ B="bench.py --ntree 74 --m-query 10000000 --steps 1 --warmup 0 --no-e2e --no-cpu
 timeout 1800 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches.csv python $B > $O/launch_run.log 2>&1
 echo "launch list rc=$?"
 python tools/ncu_summary.py launches $O/launches.csv $O/launch_summary.txt | head -16
-for spec in "k_subtree 0" "k_partition_tree 4" "k_split_scan_tree 4" "k_predict8 3" "k_importance8 1"; do
+for spec in "k_subtree 0" "k_partition_tree 4" "k_split_scan_tree 4" "k_predict32 3" "k_importance32 1"; do
   set -- $spec
   timeout 900 ncu --set full $X --clock-control none --import-source on -k regex:$1 -s $2 -c 1 -f -o $O/prof_$1 python $B > $O/ncu_$1.log 2>&1
   echo "$1 rc=$?"
