@@ -839,9 +839,9 @@ struct TScanArgs {
   const int32_t* nactive;
 };
 
-constexpr int TSV = 9;              // entries per thread (odd: conflict-free 64-bit shared loads)
 constexpr int SNT = 128;            // threads of the split-scan CTA (4 CTAs per SM: independent unit pipelines)
-constexpr int TUNIT = SNT * TSV;    // 1152 entries per unit (9 KB bulk copy); measured: 64 threads / TSV 7 or 13 slower
+// entries per thread: 9 (odd: conflict-free 64-bit shared loads; 1152-entry units, 9 KB bulk copies); measured:
+// 64 threads / 7 or 13 entries slower
 
 // The exact key off the unrolled scan loops (rarely reached: only where the upper bound passes the screen).
 __device__ __noinline__ double split_key_call(int64_t nk, int64_t Sk, int64_t nl, int64_t Sl) {
@@ -863,7 +863,10 @@ struct WBest {  // best exact candidate of one warp for the current unit
 // block max, and only boundaries with gU >= M get the exact S4.3 key.  Four
 // barriers per unit; each thread re-derives the block results from the
 // per-warp values, so there are no broadcast round trips.
-__global__ void __launch_bounds__(SNT, 4) k_split_scan_tree(TScanArgs g) {
+// TSV entries per thread (unit = SNT * TSV entries), MINB CTAs per SM for the register budget (BF_SCAN_TSV: 9 default)
+template <int TSV, int MINB>
+__global__ void __launch_bounds__(SNT, MINB) k_split_scan_tree(TScanArgs g) {
+  constexpr int TUNIT = SNT * TSV;
   extern __shared__ __align__(16) unsigned char dsm[];
   uint64_t* bufs = (uint64_t*)dsm;  // 2 x (TUNIT + 4)
   constexpr int NW = SNT / 32;
@@ -3116,14 +3119,16 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
     const int64_t nw = (n + 31) / 32;
     DBuf<uint32_t> sideb((size_t)B * nw, s);
     DBuf<int32_t> tlo(B, s), thi(B, s), act(B, s), nact(1, s);
-    const size_t tscan_smem = sizeof(uint64_t) * 2 * (TUNIT + 4);
+    static const int scan_tsv = getenv("BF_SCAN_TSV") ? atoi(getenv("BF_SCAN_TSV")) : 9;
+    auto scan_kern = scan_tsv == 5 ? k_split_scan_tree<5, 6> : scan_tsv == 7 ? k_split_scan_tree<7, 5> : k_split_scan_tree<9, 4>;
+    const size_t tscan_smem = sizeof(uint64_t) * 2 * ((size_t)SNT * (scan_tsv == 5 ? 5 : scan_tsv == 7 ? 7 : 9) + 4);
     const size_t tpart_base = sizeof(uint64_t) * (size_t)TPG * (TPNS * (TPUNIT + 2));
     const int smem_optin = dyn_smem_limit(k_partition_tree);
     const bool bm_smem = getenv("BF_PART_L2") == nullptr && tpart_base + (size_t)nw * 4 <= (size_t)smem_optin;
     const size_t tpart_smem = tpart_base + (bm_smem ? (size_t)nw * 4 : 0);
-    BF_CUDA_CHECK(cudaFuncSetAttribute(k_split_scan_tree, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tscan_smem));
+    BF_CUDA_CHECK(cudaFuncSetAttribute(scan_kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tscan_smem));
     int occ_ts = 0, occ_tp = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_ts, k_split_scan_tree, SNT, tscan_smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_ts, scan_kern, SNT, tscan_smem);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_tp, k_partition_tree, TPNT, tpart_smem);
     const unsigned grid_tscan = (unsigned)std::max(1, occ_ts * nsm), grid_tpart = (unsigned)std::max(1, occ_tp * nsm);
     DBuf<uint64_t> E0, E1, Es;
@@ -3255,7 +3260,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
         {  // ---- a7 split search: tree-affine CTAs own whole (node, drawn feature) items
           TScanArgs ga{nc, feat.p, mtry, Bc, Ec, yq.p, tlo.p, thi.p, rec.p, act.p, nact.p};
           KScope ks_("k_split_scan_tree", s, 0.0);
-          k_split_scan_tree<<<grid_tscan, SNT, tscan_smem, s>>>(ga);
+          scan_kern<<<grid_tscan, SNT, tscan_smem, s>>>(ga);
         }
         if (lvl_timing) cudaEventRecord(lev[1], s);
         {
