@@ -1565,6 +1565,7 @@ struct SubArgs {
   unsigned long long* visits; // optional (profile mode): split-search entry visits (mtry x distinct rows per node)
   int tq_sleep_max;           // idle-warp back-off cap in ns (BF_TQ_SLEEP_MAX, default 2048)
   int tq_bigger_first;        // continue with the child of more distinct rows (BF_TQ_BIGGER_FIRST, default 1)
+  int tq_lpt;                 // tiny roots queued before the tiny phase taken largest first (BF_TQ_LPT, default 1)
 };
 
 // S4.2 mtry draw by one warp, in parallel.  Draw i picks position
@@ -2226,6 +2227,30 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
     }
     __syncthreads();
   }
+  // The tiny roots queued before this phase are taken largest first (longest-processing-time order: the longest
+  // chains start first, so the tail of the phase is shorter).  rorder[h] = queue entry of the h-th pop, in the
+  // `side` bytes (free after the medium levels); up to 64 roots (else queue order).
+  int16_t* rorder = reinterpret_cast<int16_t*>(side);
+  __shared__ int s_nr0;
+  if (wid == 0) {
+    const int nr0 = a_get<int>(s_alloc);
+    const bool lpt = g.tq_lpt && nr0 <= 64 && 2 * nr0 <= A;
+    if (lpt) {
+      const int i0 = lane, i1 = lane + 32;
+      const int k0 = i0 < nr0 ? a_get<int32_t>(tq[i0].ra) : -1, k1 = i1 < nr0 ? a_get<int32_t>(tq[i1].ra) : -1;
+      int r0 = 0, r1 = 0;
+      for (int j = 0; j < nr0; ++j) {
+        const int kj = __shfl_sync(0xffffffffu, j < 32 ? k0 : k1, j & 31);
+        r0 += (kj > k0) || (kj == k0 && j < i0);
+        r1 += (kj > k1) || (kj == k1 && j < i1);
+      }
+      if (i0 < nr0) rorder[r0] = (int16_t)i0;
+      if (i1 < nr0) rorder[r1] = (int16_t)i1;
+    }
+    if (lane == 0) s_nr0 = lpt ? nr0 : 0;
+  }
+  __syncthreads();
+  const int nr0 = s_nr0;
   for (;;) {
     int h = -1;
     TN nd;
@@ -2246,6 +2271,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         }
       }
       if (h >= 0) {
+        if (h < nr0) h = rorder[h];  // a root queued before the phase: largest first
         while (blk_ref<int32_t>(tq_ready[h]).fetch_or(0, cuda::memory_order_acquire) == 0) __nanosleep(32);
         nd = tq_read(tq, h);
       }
@@ -3420,6 +3446,8 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
           static const int tq_bigger_first = getenv("BF_TQ_BIGGER_FIRST") ? atoi(getenv("BF_TQ_BIGGER_FIRST")) : 1;
           ga.tq_sleep_max = tq_sleep_max < 32 ? 32 : tq_sleep_max;
           ga.tq_bigger_first = tq_bigger_first;
+          static const int tq_lpt = getenv("BF_TQ_LPT") ? atoi(getenv("BF_TQ_LPT")) : 1;
+          ga.tq_lpt = tq_lpt;
           static const bool want_stats = getenv("BF_SUBTREE_STATS") != nullptr;
           DBuf<unsigned long long> st;
           if (want_stats) {
