@@ -1563,7 +1563,7 @@ struct SubArgs {
   Pool pool;
   unsigned long long* stats;  // optional phase counters (BF_SUBTREE_STATS=1), else NULL
   unsigned long long* visits; // optional (profile mode): split-search entry visits (mtry x distinct rows per node)
-  int tq_sleep_max;           // idle-warp back-off cap in ns (BF_TQ_SLEEP_MAX, default 2048)
+  int tq_sleep_max;           // idle-warp back-off cap in ns (BF_TQ_SLEEP_MAX, default 512)
   int tq_bigger_first;        // continue with the child of more distinct rows (BF_TQ_BIGGER_FIRST, default 1)
   int tq_lpt;                 // tiny roots queued before the tiny phase taken largest first (BF_TQ_LPT, default 1)
 };
@@ -1686,10 +1686,21 @@ __device__ __forceinline__ TNodeT<NWD> tq_bcast(const TNodeT<NWD>& c) {  // lane
   return r;
 }
 
-// TV: tiny-node search (0 staged warp items, 1 lane per drawn feature); TT: largest tiny root (64 or 128 rows)
-template <int TV, int TT>
+// TV: tiny-node search (0 staged warp items, 1 lane per drawn feature with a position table, 2 lane per drawn
+// feature with ballot masks); TT: largest tiny root (64 or 128 rows); HW: helper warps that grow tiny nodes
+// while the other SUB_NW - HW warps run the medium levels (named barrier 1), 0 = phases in sequence
+template <int TV, int TT, int HW>
 __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   static_assert(TT == 64 || (TT == 128 && TV == 1), "tiny roots of 128 rows need the lane-per-feature search");
+  static_assert(HW == 0 || TV == 2, "helper warps need the ballot masks (no position table during the medium levels)");
+  constexpr int NMW = SUB_NW - HW;  // warps of the medium levels
+  auto mbar = [&]() {
+    if constexpr (HW == 0) __syncthreads();
+    else asm volatile("bar.sync 1, %0;" ::"r"(NMW * 32) : "memory");
+  };
+  constexpr bool LPF = TV >= 1;  // lane-per-feature tiny search (1: masks from the position table, 2: by ballots,
+                                 // 3: position table built per tiny root by the warp that takes the root)
+  constexpr int ROOTF = 1 << 30;  // TV 3: queue entry of a tiny root whose rmap / ppos are not built yet (in ra)
   constexpr int NWD = TT / 64;
   using TN = TNodeT<NWD>;
   extern __shared__ __align__(16) unsigned char smem[];
@@ -1715,7 +1726,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   ptr += align16((size_t)2 * A * sizeof(SRec));
   // DEFER (lane-per-feature search, 64-row tiny roots): the value of a tiny-phase record is computed at the flush
   // from its row mask (held in the record's value field) over its tiny root's rows, off the critical path
-  constexpr bool DEFER = TV == 1 && NWD == 1;
+  constexpr bool DEFER = LPF && NWD == 1;
   uint16_t* rdef = (uint16_t*)ptr;
   ptr += align16((size_t)2 * A * 2);
   MNode* curl = (MNode*)ptr;
@@ -1881,14 +1892,19 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       c.rlo = s_off[r];
       c.ra = R.a;
       m_full(c.mask, R.a);
+      if constexpr (TV == 3) c.ra |= ROOTF;
       c.id = (r << 16) | rec0;
       c.n = R.n;
       c.S = R.S;
       c.key = R.key;
       c.value = 0.0;  // a root's value is the pool's (written before the subtree phase)
+      if constexpr (HW > 0)  // row index inside the tiny root, before it is published
+        for (int k = 0; k < R.a; ++k) rmap[list[s_off[r] + k] & 0xffffu] = (uint8_t)k;
       tq_push(tq, tq_ready, &s_alloc, &s_pending, c);
     }
   }
+  __shared__ int s_mdone, s_nidx[16];
+  if (tid == 0) s_mdone = 0;
   __syncthreads();
   tclk[1] = clock64();
 
@@ -1896,6 +1912,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   long long mclk[3] = {0, 0, 0};  // medium phase: scan+finalize, next level, partition (thread 0, stats only)
   long long mfin = 0;             // of which finalize (warp per node after the item barrier)
   int n_mlev = 0;                 // medium levels
+  if (HW == 0 || wid < NMW) {
   while (s_ncur > 0) {
     const long long mc0 = clock64();
     const int ncur = s_ncur;
@@ -1904,15 +1921,15 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
     // (node, drawn predictor) items over all warps; per-item winners in the scratch area; one warp per node
     // reduces its items (lowest predictor on equal keys) and finalizes the split.  Nodes go in groups whose
     // items fit the scratch area (and whose draws fit the per-warp feature slots).
-    WRec* irec = (WRec*)temp_all;
-    const int cap_items = (int)((size_t)SUB_NW * sub_temp(A) * 4 / sizeof(WRec));
-    const int NG = max(1, min(SUB_NW, cap_items / g.mtry));
+    WRec* irec = (WRec*)temp_all;  // the medium warps' scratch (helper warps keep theirs)
+    const int cap_items = (int)((size_t)NMW * sub_temp(A) * 4 / sizeof(WRec));
+    const int NG = max(1, min(NMW, cap_items / g.mtry));
     for (int n0 = 0; n0 < ncur; n0 += NG) {
       const int nn = min(NG, ncur - n0);
       if (wid < nn) warp_draw_mtry(g.seed, t_of(curl[n0 + wid].id), curl[n0 + wid].key, p, g.mtry, mind_all + wid * p, feats_all + wid * p, lane);
-      __syncthreads();
+      mbar();
       const int nit = nn * g.mtry;
-      for (int it = wid; it < nit; it += SUB_NW) {
+      for (int it = wid; it < nit; it += NMW) {
         const int li = it / g.mtry;
         const MNode nd = curl[n0 + li];
         const int f = feats_all[li * p + (it - li * g.mtry)];
@@ -2028,7 +2045,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
           irec[it] = r;
         }
       }
-      __syncthreads();
+      mbar();
       const long long mf0 = clock64();
       if (wid < nn) {
         const int i = n0 + wid;
@@ -2103,11 +2120,12 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
           curl[i].split = 0;
         }
       }
-      __syncthreads();
+      mbar();
       mfin += clock64() - mf0;
     }
     const long long mc1 = clock64();
-    // ---- next medium level (block scan) and tiny roots (work queue; processed after the medium levels)
+    // ---- next medium level (block scan) and tiny roots (work queue; processed after the medium levels, or by
+    // the helper warps once the level's partition is done)
     {
       int kc = 0;
       MNode nd;
@@ -2115,8 +2133,25 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         nd = curl[tid];
         if (nd.split) kc = (nd.kind[0] == KIND_LARGE) + (nd.kind[1] == KIND_LARGE);
       }
-      int totc;
-      int idx = block_excl_scan(kc, s_scan, totc);
+      int totc, idx;
+      if constexpr (HW == 0) {
+        idx = block_excl_scan(kc, s_scan, totc);
+      } else {  // ncur <= max_medium(A) nodes: one thread's running sum
+        if (tid < ncur) s_nidx[tid] = kc;
+        mbar();
+        if (tid == 0) {
+          int run = 0;
+          for (int i = 0; i < ncur; ++i) {
+            const int v = s_nidx[i];
+            s_nidx[i] = run;
+            run += v;
+          }
+          s_ncur = run;
+        }
+        mbar();
+        idx = tid < ncur ? s_nidx[tid] : 0;
+        totc = 0;
+      }
       if (tid < ncur && nd.split) {
         for (int sdv = 0; sdv < 2; ++sdv) {
           const int kd = nd.kind[sdv];
@@ -2141,20 +2176,21 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
             c.rlo = lo;
             c.ra = a;
             m_full(c.mask, a);
+            if constexpr (TV == 3) c.ra |= ROOTF;
             c.id = (nd.id & ~0xffff) | (nd.lid + sdv);
             c.n = nn;
             c.S = S;
             c.key = key;
             c.value = recs[nd.lid + sdv].value;  // written by the node's warp before the last barrier
-            tq_push(tq, tq_ready, &s_alloc, &s_pending, c);
+            if constexpr (HW == 0) tq_push(tq, tq_ready, &s_alloc, &s_pending, c);
           }
         }
       }
-      if (tid == 0) s_ncur = totc;
+      if (HW == 0 && tid == 0) s_ncur = totc;
     }
     const long long mc2 = clock64();
     // ---- in-place stable partition of every feature row of every split node with a non-leaf child
-    for (int it = wid; it < ncur * p; it += SUB_NW) {
+    for (int it = wid; it < ncur * p; it += NMW) {
       const int i = it / p, f = it - i * p;
       const MNode& nd = curl[i];
       if (!nd.split || (nd.kind[0] == KIND_LEAF && nd.kind[1] == KIND_LEAF)) continue;
@@ -2190,7 +2226,28 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       }
       __syncwarp();
     }
-    __syncthreads();
+    mbar();
+    if constexpr (HW > 0) {  // the level's tiny children: lists final now; row index, then publish (warp per node)
+      for (int i = wid; i < ncur; i += NMW) {
+        const MNode nd = curl[i];
+        if (!nd.split) continue;
+        for (int sdv = 0; sdv < 2; ++sdv) {
+          if (nd.kind[sdv] != KIND_SMALL) continue;
+          TN c;
+          c.rlo = sdv ? nd.lo + nd.al : nd.lo;
+          c.ra = sdv ? nd.a - nd.al : nd.al;
+          m_full(c.mask, c.ra);
+          c.id = (nd.id & ~0xffff) | (nd.lid + sdv);
+          c.n = sdv ? nd.n - nd.nl : nd.nl;
+          c.S = sdv ? nd.S - nd.Sl : nd.Sl;
+          c.key = sdv ? nd.keyr : nd.keyl;
+          c.value = recs[nd.lid + sdv].value;
+          for (int k = lane; k < c.ra; k += 32) rmap[list[c.rlo + k] & 0xffffu] = (uint8_t)k;
+          __syncwarp();
+          if (lane == 0) tq_push(tq, tq_ready, &s_alloc, &s_pending, c);
+        }
+      }
+    }
     {
       const long long mc3 = clock64();
       mclk[0] += mc1 - mc0;
@@ -2201,22 +2258,27 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       nxtl = tl;
     }
   }
+  if constexpr (HW > 0) {
+    mbar();  // every medium warp has published its tiny roots
+    if (tid == 0) blk_ref<int>(s_mdone).exchange(1, cuda::memory_order_release);
+  }
+  }  // medium warps
 
   // ================= tiny nodes: row index inside each tiny root, then the work queue
   tclk[2] = clock64();
-  {
+  if constexpr (HW == 0 && TV != 3) {
     const int nroots = a_get<int>(s_alloc);
     for (int qi = wid; qi < nroots; qi += SUB_NW) {
       const TN r = tq_read(tq, qi);  // pushed before the barrier above
       for (int k = lane; k < r.ra; k += 32) rmap[list[r.rlo + k] & 0xffffu] = (uint8_t)k;
     }
+    __syncthreads();
   }
-  __syncthreads();
   // TV = 1: ppos[f * a0 + rlo + i] = position, in feature f's segment of its tiny root, of the row at feature-0
   // position i (the scratch area is free once the medium levels are done), so a node's rows in feature f's order
   // are the set bits of one 64-bit mask built from the node's mask (no staging, no pass over non-member rows)
   uint8_t* ppos = (uint8_t*)temp_all;
-  if constexpr (TV == 1) {
+  if constexpr (TV == 1) {  // (TV 2 builds its masks by ballots instead)
     const int nroots = a_get<int>(s_alloc);
     for (int it = wid; it < nroots * p; it += SUB_NW) {
       const int qi = it / p, f = it - qi * p;
@@ -2232,7 +2294,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
   // `side` bytes (free after the medium levels); up to 64 roots (else queue order).
   int16_t* rorder = reinterpret_cast<int16_t*>(side);
   __shared__ int s_nr0;
-  if (wid == 0) {
+  if (HW == 0 && wid == 0) {
     const int nr0 = a_get<int>(s_alloc);
     const bool lpt = g.tq_lpt && nr0 <= 64 && 2 * nr0 <= A;
     if (lpt) {
@@ -2249,8 +2311,8 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
     }
     if (lane == 0) s_nr0 = lpt ? nr0 : 0;
   }
-  __syncthreads();
-  const int nr0 = s_nr0;
+  if constexpr (HW == 0) __syncthreads();
+  const int nr0 = HW == 0 ? s_nr0 : 0;
   for (;;) {
     int h = -1;
     TN nd;
@@ -2263,7 +2325,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
             h = hd;
             break;
           }
-        } else if (a_get<int>(s_pending) == 0) {
+        } else if (a_get<int>(s_pending) == 0 && (HW == 0 || a_get<int>(s_mdone) != 0)) {
           break;
         } else {
           __nanosleep(ns);  // idle warp: back off so the busy warps keep the issue slots
@@ -2284,6 +2346,30 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
     while (have) {
       have = false;
       ++n_tiny;
+      if constexpr (TV == 3) {
+        if (nd.ra & ROOTF) {  // first node of a tiny root: its row index and position table, by this warp
+          nd.ra &= ~ROOTF;
+          const int rl = nd.rlo, rr = nd.ra;
+          for (int k = lane; k < rr; k += 32) rmap[list[rl + k] & 0xffffu] = (uint8_t)k;
+          __syncwarp();
+          for (int f0 = 0; f0 < p; f0 += 8) {  // 8 features' loads in flight
+            uint32_t ev[16];
+#pragma unroll
+            for (int u = 0; u < 8; ++u) {
+              const uint32_t* sg = list + (size_t)min(f0 + u, p - 1) * a0 + rl;
+              ev[2 * u] = lane < rr ? sg[lane] : 0u;
+              ev[2 * u + 1] = lane + 32 < rr ? sg[lane + 32] : 0u;
+            }
+#pragma unroll
+            for (int u = 0; u < 8; ++u) {
+              uint8_t* pp = ppos + (size_t)min(f0 + u, p - 1) * a0 + rl;
+              if (f0 + u < p && lane < rr) pp[rmap[ev[2 * u] & 0xffffu]] = (uint8_t)lane;
+              if (f0 + u < p && lane + 32 < rr) pp[rmap[ev[2 * u + 1] & 0xffffu]] = (uint8_t)(lane + 32);
+            }
+          }
+          __syncwarp();
+        }
+      }
       const int rlo = nd.rlo, ra = nd.ra;
       const int an = m_popc(nd.mask);  // distinct rows of the node
       nvis += (unsigned long long)an * (unsigned)g.mtry;
@@ -2301,23 +2387,50 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
       uint32_t ltie = 0xffffffffu, lra = 0, lrb = 0;
       int32_t lnl = 0;
       int64_t lSl = 0;
-      if constexpr (TV == 1) {
+      if constexpr (LPF) {
         // Lane s scans drawn feature feats[s] (s = lane, lane + 32, ...) serially over the node's own rows: the
         // node's rows in that feature's value order are the set bits of Mf (positions in the tiny root's
         // segment), so the loop runs an times with no staging, no segmented warp scan and no idle positions.
         // Per boundary the fp32 bounds tL <= t <= tU (key_bounds_t); M = warp max of the lower bounds; a lane
         // whose second-largest upper bound is below M evaluates its one candidate directly, any other lane with
         // an upper bound >= M re-walks its features taking the exact S4.3 key where tU >= M.
-        auto feat_mask = [&](int f, uint64_t (&Mf)[NWD]) {
-          const uint8_t* pp = ppos + (size_t)f * a0 + rlo;
-          uint64_t m[NWD];
+        // TV 2: every drawn feature's member mask by ballots over the root's segment (lane k tests the row at
+        // position k), kept in the warp's scratch (no position table)
+        uint64_t* mkw = reinterpret_cast<uint64_t*>(temp + (((uintptr_t)temp >> 2) & 1));  // 8-byte aligned
+        if constexpr (TV == 2) {
+          static_assert(NWD == 1, "ballot masks cover tiny roots of <= 64 rows");
+          for (int u0 = 0; u0 < g.mtry; u0 += 7) {
+            uint32_t ev[14];
 #pragma unroll
-          for (int w = 0; w < NWD; ++w) {
-            m[w] = nd.mask[w];
-            Mf[w] = 0ull;
+            for (int u = 0; u < 7; ++u) {
+              const uint32_t* sg = list + (size_t)feats[min(u0 + u, g.mtry - 1)] * a0 + rlo;
+              ev[2 * u] = lane < ra ? sg[lane] : 0u;
+              ev[2 * u + 1] = lane + 32 < ra ? sg[lane + 32] : 0u;
+            }
+#pragma unroll
+            for (int u = 0; u < 7; ++u) {
+              const int ri0 = rmap[ev[2 * u] & 0xffffu], ri1 = rmap[ev[2 * u + 1] & 0xffffu];
+              const uint32_t b0 = __ballot_sync(0xffffffffu, lane < ra && ((nd.mask[0] >> ri0) & 1ull));
+              const uint32_t b1 = __ballot_sync(0xffffffffu, lane + 32 < ra && ((nd.mask[0] >> ri1) & 1ull));
+              if (lane == 0 && u0 + u < g.mtry) mkw[u0 + u] = ((uint64_t)b1 << 32) | b0;
+            }
           }
+          __syncwarp();
+        }
+        auto feat_mask_s = [&](int s, uint64_t (&Mf)[NWD]) {
+          if constexpr (TV == 2) {
+            Mf[0] = mkw[s];
+          } else {
+            const uint8_t* pp = ppos + (size_t)feats[s] * a0 + rlo;
+            uint64_t m[NWD];
+#pragma unroll
+            for (int w = 0; w < NWD; ++w) {
+              m[w] = nd.mask[w];
+              Mf[w] = 0ull;
+            }
 #pragma unroll 4
-          for (int c = 0; c < an; ++c) m_set(Mf, (int)pp[m_pop(m)]);
+            for (int c = 0; c < an; ++c) m_set(Mf, (int)pp[m_pop(m)]);
+          }
         };
         float mLt = -1.0f, mU = -1.0f, u2 = -1.0f;
         int bs = -1;
@@ -2327,7 +2440,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
         for (int s = lane; s < g.mtry; s += 32) {
           const uint32_t* seg = list + (size_t)feats[s] * a0 + rlo;
           uint64_t Mf[NWD];
-          feat_mask(feats[s], Mf);
+          feat_mask_s(s, Mf);
           uint32_t pe = seg[m_pop(Mf)];
           int32_t cw = wl[pe & 0xffffu];
           int64_t cs = wy[pe & 0xffffu];
@@ -2367,7 +2480,7 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
           for (int s = lane; s < g.mtry; s += 32) {
             const uint32_t* seg = list + (size_t)feats[s] * a0 + rlo;
             uint64_t Mf[NWD];
-            feat_mask(feats[s], Mf);
+            feat_mask_s(s, Mf);
             uint32_t pe = seg[m_pop(Mf)];
             int32_t cw = wl[pe & 0xffffu];
             int64_t cs = wy[pe & 0xffffu];
@@ -3031,14 +3144,16 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
 
   ptm.mark("presort");
   // ---- sizing: subtree capacity A and trees in flight B
-  const int smax = std::min(std::min(dyn_smem_limit(k_subtree<0, 64>), dyn_smem_limit(k_subtree<1, 64>)),
-                            dyn_smem_limit(k_subtree<1, 128>));
+  const int smax = std::min(std::min(std::min(dyn_smem_limit(k_subtree<0, 64, 0>), dyn_smem_limit(k_subtree<1, 64, 0>)),
+                                     std::min(dyn_smem_limit(k_subtree<1, 128, 0>), dyn_smem_limit(k_subtree<3, 64, 0>))),
+                            std::min(std::min(dyn_smem_limit(k_subtree<2, 64, 0>), dyn_smem_limit(k_subtree<2, 64, 4>)),
+                                     dyn_smem_limit(k_subtree<2, 64, 2>)));
   int A = 2;
   // tiny-node search: 1 = lane per drawn feature over the node's own rows (default), 0 = staged (slot, position)
   // items scanned by the whole warp (BF_TINY_V=0); largest tiny root 64 rows (default) or 128 (BF_TINY_MAX=128,
   // lane-per-feature search only; measured slower: the longer tiny chains outweigh the shorter medium phase)
-  static const int tiny_v = getenv("BF_TINY_V") ? atoi(getenv("BF_TINY_V")) : 1;
-  static const int tiny_max = (tiny_v != 0 && getenv("BF_TINY_MAX") && atoi(getenv("BF_TINY_MAX")) == 128) ? 128 : 64;
+  static const int tiny_v = getenv("BF_TINY_V") ? atoi(getenv("BF_TINY_V")) : 2;
+  static const int tiny_max = (tiny_v == 1 && getenv("BF_TINY_MAX") && atoi(getenv("BF_TINY_MAX")) == 128) ? 128 : 64;
   while (A < 1024 && subtree_smem(A + 1, p, tiny_max) <= (size_t)smax) ++A;  // load 2 holds <= 32 chunks of 32
   BF_REQUIRE(subtree_smem(2, p, tiny_max) <= (size_t)smax, BF_ENOTIMPL,
              "bf_fit: p too large for the shared-memory subtree kernel");
@@ -3442,7 +3557,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
             BF_CUDA_CHECK(cudaMemsetAsync(vis.p, 0, 8, s));
             ga.visits = vis.p;
           }
-          static const int tq_sleep_max = getenv("BF_TQ_SLEEP_MAX") ? atoi(getenv("BF_TQ_SLEEP_MAX")) : 2048;
+          static const int tq_sleep_max = getenv("BF_TQ_SLEEP_MAX") ? atoi(getenv("BF_TQ_SLEEP_MAX")) : 512;
           static const int tq_bigger_first = getenv("BF_TQ_BIGGER_FIRST") ? atoi(getenv("BF_TQ_BIGGER_FIRST")) : 1;
           ga.tq_sleep_max = tq_sleep_max < 32 ? 32 : tq_sleep_max;
           ga.tq_bigger_first = tq_bigger_first;
@@ -3457,12 +3572,22 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
           }
           {
             KScope ks_("k_subtree", s, 0.0);
+            // helper warps (BF_SUBTREE_HW=4: 4 warps grow tiny nodes during the medium levels; ballot masks)
+            static const int sub_hw = getenv("BF_SUBTREE_HW") ? atoi(getenv("BF_SUBTREE_HW")) : 0;
             if (tiny_v == 0)
-              k_subtree<0, 64><<<(unsigned)ngroups, SUB_NT, subtree_smem(A, p, 64), s>>>(ga);
+              k_subtree<0, 64, 0><<<(unsigned)ngroups, SUB_NT, subtree_smem(A, p, 64), s>>>(ga);
+            else if (sub_hw == 4 && tiny_max == 64)
+              k_subtree<2, 64, 4><<<(unsigned)ngroups, SUB_NT, subtree_smem(A, p, 64), s>>>(ga);
+            else if (sub_hw == 2 && tiny_max == 64)
+              k_subtree<2, 64, 2><<<(unsigned)ngroups, SUB_NT, subtree_smem(A, p, 64), s>>>(ga);
+            else if (tiny_v == 2)
+              k_subtree<2, 64, 0><<<(unsigned)ngroups, SUB_NT, subtree_smem(A, p, 64), s>>>(ga);
+            else if (tiny_v == 3)
+              k_subtree<3, 64, 0><<<(unsigned)ngroups, SUB_NT, subtree_smem(A, p, 64), s>>>(ga);
             else if (tiny_max == 64)
-              k_subtree<1, 64><<<(unsigned)ngroups, SUB_NT, subtree_smem(A, p, 64), s>>>(ga);
+              k_subtree<1, 64, 0><<<(unsigned)ngroups, SUB_NT, subtree_smem(A, p, 64), s>>>(ga);
             else
-              k_subtree<1, 128><<<(unsigned)ngroups, SUB_NT, subtree_smem(A, p, 128), s>>>(ga);
+              k_subtree<1, 128, 0><<<(unsigned)ngroups, SUB_NT, subtree_smem(A, p, 128), s>>>(ga);
           }
           if (ga.visits) {  // SURVEY 8(d) split-search bytes of the subtree nodes: 20 B per entry visit
             unsigned long long hv = 0;
