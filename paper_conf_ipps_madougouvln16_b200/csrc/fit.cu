@@ -3149,10 +3149,12 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
                             std::min(std::min(dyn_smem_limit(k_subtree<2, 64, 0>), dyn_smem_limit(k_subtree<2, 64, 4>)),
                                      dyn_smem_limit(k_subtree<2, 64, 2>)));
   int A = 2;
-  // tiny-node search: 1 = lane per drawn feature over the node's own rows (default), 0 = staged (slot, position)
-  // items scanned by the whole warp (BF_TINY_V=0); largest tiny root 64 rows (default) or 128 (BF_TINY_MAX=128,
-  // lane-per-feature search only; measured slower: the longer tiny chains outweigh the shorter medium phase)
-  static const int tiny_v = getenv("BF_TINY_V") ? atoi(getenv("BF_TINY_V")) : 2;
+  // tiny-node search (BF_TINY_V): 3 = lane per drawn feature, member masks from a position table built per tiny
+  // root by the warp that takes the root (default); 2 = masks by ballots; 1 = position table built for all tiny
+  // roots at the phase start; 0 = staged (slot, position) items scanned by the whole warp.  Measured per 200 C4
+  // trees: 452 / 484 / 526 / 600 ms.  Largest tiny root 64 rows (default) or 128 (BF_TINY_MAX=128 with TV 1;
+  // slower: the longer tiny chains outweigh the shorter medium phase)
+  static const int tiny_v = getenv("BF_TINY_V") ? atoi(getenv("BF_TINY_V")) : 3;
   static const int tiny_max = (tiny_v == 1 && getenv("BF_TINY_MAX") && atoi(getenv("BF_TINY_MAX")) == 128) ? 128 : 64;
   while (A < 1024 && subtree_smem(A + 1, p, tiny_max) <= (size_t)smax) ++A;  // load 2 holds <= 32 chunks of 32
   BF_REQUIRE(subtree_smem(2, p, tiny_max) <= (size_t)smax, BF_ENOTIMPL,

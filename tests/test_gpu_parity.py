@@ -402,16 +402,17 @@ print("ok")
 
 @pytest.mark.parametrize("env", [{"BF_TQ_BIGGER_FIRST": "0"}, {"BF_TQ_BIGGER_FIRST": "1", "BF_TQ_SLEEP_MAX": "32"},
                                  {"BF_SUBTREE_PACK": "0"}, {"BF_TINY_V": "0"}, {"BF_TINY_V": "1", "BF_TINY_MAX": "128"},
-                                 {"BF_TQ_LPT": "0"}, {"BF_TINY_V": "1"}, {"BF_TINY_V": "3"},
+                                 {"BF_TQ_LPT": "0"}, {"BF_TINY_V": "1"}, {"BF_TINY_V": "2"},
                                  {"BF_SUBTREE_HW": "4"}, {"BF_SUBTREE_HW": "2"}])
 def test_tiny_queue_schedule_does_not_change_the_forest(env):
     """The subtree kernel's tiny-node queue order (which child keeps the warp, idle back-off) and the packing of
     several small roots (of different trees) into one CTA are scheduling only:
     every node's split depends on its own rows and Philox key, so the forest stays bit-exact vs the oracle.
     So are the tiny-node search variants (BF_TINY_V=0: staged warp items over tiny roots of <= 64 rows;
-    BF_TINY_V=1: lane per drawn feature with a position table, also over tiny roots of up to 128 rows;
-    the default BF_TINY_V=2: lane per drawn feature with ballot-built member masks) and the helper warps that
-    grow tiny nodes while the others run the medium levels (BF_SUBTREE_HW=2 / 4).
+    BF_TINY_V=1: lane per drawn feature with a position table built for all tiny roots at the phase start, also
+    over tiny roots of up to 128 rows; BF_TINY_V=2: ballot-built member masks; the default BF_TINY_V=3: the
+    position table built per tiny root by the warp that takes it) and the helper warps that grow tiny nodes while
+    the others run the medium levels (BF_SUBTREE_HW=2 / 4, with the ballot masks).
     The switches are read once per process, hence the subprocess."""
     import subprocess
     import sys
