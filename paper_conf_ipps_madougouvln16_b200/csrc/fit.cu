@@ -1691,7 +1691,7 @@ __device__ __forceinline__ TNodeT<NWD> tq_bcast(const TNodeT<NWD>& c) {  // lane
 // while the other SUB_NW - HW warps run the medium levels (named barrier 1), 0 = phases in sequence
 template <int TV, int TT, int HW>
 __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
-  static_assert(TT == 64 || (TT == 128 && TV == 1), "tiny roots of 128 rows need the lane-per-feature search");
+  static_assert(TT == 64 || (TT == 128 && (TV == 1 || TV == 3)), "tiny roots of 128 rows need the position table");
   static_assert(HW == 0 || TV == 2, "helper warps need the ballot masks (no position table during the medium levels)");
   constexpr int NMW = SUB_NW - HW;  // warps of the medium levels
   auto mbar = [&]() {
@@ -2352,19 +2352,22 @@ __global__ void __launch_bounds__(SUB_NT) k_subtree(SubArgs g) {
           const int rl = nd.rlo, rr = nd.ra;
           for (int k = lane; k < rr; k += 32) rmap[list[rl + k] & 0xffffu] = (uint8_t)k;
           __syncwarp();
-          for (int f0 = 0; f0 < p; f0 += 8) {  // 8 features' loads in flight
-            uint32_t ev[16];
+          constexpr int FU = 16 / (TT / 32);  // features per round: 16 loads in flight per lane
+          for (int f0 = 0; f0 < p; f0 += FU) {
+            uint32_t ev[FU * (TT / 32)];
 #pragma unroll
-            for (int u = 0; u < 8; ++u) {
+            for (int u = 0; u < FU; ++u) {
               const uint32_t* sg = list + (size_t)min(f0 + u, p - 1) * a0 + rl;
-              ev[2 * u] = lane < rr ? sg[lane] : 0u;
-              ev[2 * u + 1] = lane + 32 < rr ? sg[lane + 32] : 0u;
+#pragma unroll
+              for (int hh = 0; hh < TT / 32; ++hh) ev[u * (TT / 32) + hh] = lane + 32 * hh < rr ? sg[lane + 32 * hh] : 0u;
             }
 #pragma unroll
-            for (int u = 0; u < 8; ++u) {
+            for (int u = 0; u < FU; ++u) {
               uint8_t* pp = ppos + (size_t)min(f0 + u, p - 1) * a0 + rl;
-              if (f0 + u < p && lane < rr) pp[rmap[ev[2 * u] & 0xffffu]] = (uint8_t)lane;
-              if (f0 + u < p && lane + 32 < rr) pp[rmap[ev[2 * u + 1] & 0xffffu]] = (uint8_t)(lane + 32);
+#pragma unroll
+              for (int hh = 0; hh < TT / 32; ++hh)
+                if (f0 + u < p && lane + 32 * hh < rr)
+                  pp[rmap[ev[u * (TT / 32) + hh] & 0xffffu]] = (uint8_t)(lane + 32 * hh);
             }
           }
           __syncwarp();
@@ -3145,7 +3148,8 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
   ptm.mark("presort");
   // ---- sizing: subtree capacity A and trees in flight B
   const int smax = std::min(std::min(std::min(dyn_smem_limit(k_subtree<0, 64, 0>), dyn_smem_limit(k_subtree<1, 64, 0>)),
-                                     std::min(dyn_smem_limit(k_subtree<1, 128, 0>), dyn_smem_limit(k_subtree<3, 64, 0>))),
+                                     std::min(std::min(dyn_smem_limit(k_subtree<1, 128, 0>), dyn_smem_limit(k_subtree<3, 64, 0>)),
+                                              dyn_smem_limit(k_subtree<3, 128, 0>))),
                             std::min(std::min(dyn_smem_limit(k_subtree<2, 64, 0>), dyn_smem_limit(k_subtree<2, 64, 4>)),
                                      dyn_smem_limit(k_subtree<2, 64, 2>)));
   int A = 2;
@@ -3155,7 +3159,8 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
   // trees: 452 / 484 / 526 / 600 ms.  Largest tiny root 64 rows (default) or 128 (BF_TINY_MAX=128 with TV 1;
   // slower: the longer tiny chains outweigh the shorter medium phase)
   static const int tiny_v = getenv("BF_TINY_V") ? atoi(getenv("BF_TINY_V")) : 3;
-  static const int tiny_max = (tiny_v == 1 && getenv("BF_TINY_MAX") && atoi(getenv("BF_TINY_MAX")) == 128) ? 128 : 64;
+  static const int tiny_max =
+      ((tiny_v == 1 || tiny_v == 3) && getenv("BF_TINY_MAX") && atoi(getenv("BF_TINY_MAX")) == 128) ? 128 : 64;
   while (A < 1024 && subtree_smem(A + 1, p, tiny_max) <= (size_t)smax) ++A;  // load 2 holds <= 32 chunks of 32
   BF_REQUIRE(subtree_smem(2, p, tiny_max) <= (size_t)smax, BF_ENOTIMPL,
              "bf_fit: p too large for the shared-memory subtree kernel");
@@ -3584,6 +3589,8 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
               k_subtree<2, 64, 2><<<(unsigned)ngroups, SUB_NT, subtree_smem(A, p, 64), s>>>(ga);
             else if (tiny_v == 2)
               k_subtree<2, 64, 0><<<(unsigned)ngroups, SUB_NT, subtree_smem(A, p, 64), s>>>(ga);
+            else if (tiny_v == 3 && tiny_max == 128)
+              k_subtree<3, 128, 0><<<(unsigned)ngroups, SUB_NT, subtree_smem(A, p, 128), s>>>(ga);
             else if (tiny_v == 3)
               k_subtree<3, 64, 0><<<(unsigned)ngroups, SUB_NT, subtree_smem(A, p, 64), s>>>(ga);
             else if (tiny_max == 64)

@@ -402,7 +402,7 @@ print("ok")
 
 @pytest.mark.parametrize("env", [{"BF_TQ_BIGGER_FIRST": "0"}, {"BF_TQ_BIGGER_FIRST": "1", "BF_TQ_SLEEP_MAX": "32"},
                                  {"BF_SUBTREE_PACK": "0"}, {"BF_TINY_V": "0"}, {"BF_TINY_V": "1", "BF_TINY_MAX": "128"},
-                                 {"BF_TQ_LPT": "0"}, {"BF_TINY_V": "1"}, {"BF_TINY_V": "2"},
+                                 {"BF_TQ_LPT": "0"}, {"BF_TINY_V": "1"}, {"BF_TINY_V": "2"}, {"BF_TINY_MAX": "128"},
                                  {"BF_SUBTREE_HW": "4"}, {"BF_SUBTREE_HW": "2"}])
 def test_tiny_queue_schedule_does_not_change_the_forest(env):
     """The subtree kernel's tiny-node queue order (which child keeps the warp, idle back-off) and the packing of
