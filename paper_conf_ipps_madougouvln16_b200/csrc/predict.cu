@@ -976,8 +976,9 @@ void predict_impl(const bf_forest* f, const double* Xq_in, int64_t ldq, int64_t 
   const int pv = getenv("BF_PREDICT_V") ? atoi(getenv("BF_PREDICT_V")) : 3;
   static int smax32 = 0;
   if (!smax32)
-    smax32 = std::min(std::min(dyn_smem_limit(k_predict32<true, 4>), dyn_smem_limit(k_predict32<false, 4>)),
-                      std::min(dyn_smem_limit(k_predict32<true, 6>), dyn_smem_limit(k_predict32<false, 6>)));
+    smax32 = std::min(std::min(std::min(dyn_smem_limit(k_predict32<true, 4>), dyn_smem_limit(k_predict32<false, 4>)),
+                               std::min(dyn_smem_limit(k_predict32<true, 6>), dyn_smem_limit(k_predict32<false, 6>))),
+                      std::min(dyn_smem_limit(k_predict32<true, 5>), dyn_smem_limit(k_predict32<false, 5>)));
   const ulonglong4* g32 = (pv == 3 && !(force16 && force16[0] == '1')) ? g32_get(const_cast<bf_forest*>(f), s) : nullptr;
   if (g32 && smem8 <= (size_t)smax32) {
     // G32 groups: tree blocks of <= 48 MB of slots (one 256-bit load per two levels)
@@ -1002,8 +1003,8 @@ void predict_impl(const bf_forest* f, const double* Xq_in, int64_t ldq, int64_t 
       int32_t t1 = t0 + 1;
       while (t1 < nt && t1 - t0 < RT8 && (f->g32_off[t1 + 1] - f->g32_off[t0]) * (int64_t)sizeof(ulonglong4) <= block_bytes) ++t1;
       KScope ks_("k_predict32", s, 0.0);
-      auto kern = vis.p ? (slots32 == 6 ? k_predict32<true, 6> : k_predict32<true, 4>)
-                        : (slots32 == 6 ? k_predict32<false, 6> : k_predict32<false, 4>);
+      auto kern = vis.p ? (slots32 == 6 ? k_predict32<true, 6> : slots32 == 5 ? k_predict32<true, 5> : k_predict32<true, 4>)
+                        : (slots32 == 6 ? k_predict32<false, 6> : slots32 == 5 ? k_predict32<false, 5> : k_predict32<false, 4>);
       kern<<<(unsigned)ceil_div(m, PT8), PT8, smem8, s>>>(g32, f->d_nodes, f->d_g32_root, t0, t1, t0 == 0, t1 >= nt,
                                                          (const double*)Xs.dptr, ldq, Xqf.p, xfs, m, p, ysum,
                                                          yh_in ? (double*)yh.dptr : nullptr, inv_t, vis.p);
