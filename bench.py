@@ -26,6 +26,7 @@ under torch.distributed.run with N ranks (one per GPU, 127.0.0.1 rendezvous).
 from __future__ import annotations
 
 import argparse
+import re
 import json
 import os
 import socket
@@ -91,7 +92,11 @@ def _ncu_summary(kernel: str, config: str):
     """Newest committed `ncu --set full` summary of `kernel` (tools/ncu_summary.py) for this workload."""
     import glob
     names = [f"full_{kernel}_{config}.json"] + ([f"full_{kernel}.json"] if config == "C4" else [])
-    for d in sorted(glob.glob(os.path.join(ROOT, "profiles", "r[0-9]*")), reverse=True):
+    def order(d):  # r02 < r02a < r02z < r02aa: round, then the suffix by length and letters
+        m = re.match(r"r(\d+)([a-z]*)$", os.path.basename(d))
+        return (int(m.group(1)), len(m.group(2)), m.group(2)) if m else (-1, 0, "")
+
+    for d in sorted(glob.glob(os.path.join(ROOT, "profiles", "r[0-9]*")), key=order, reverse=True):
         for nm in names:
             f = os.path.join(d, nm)
             if os.path.exists(f):
