@@ -30,3 +30,22 @@ def test_gpus_flag_spawns_ranks_reference_arm():
     assert d["impl"] == "reference" and d["n_gpus"] == 2
     assert d["metric"] == json.load(open(os.path.join(ROOT, "BASELINE.json")))["metric"]
     assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["cpu_baseline"]["kind"] == "oracle"
+
+
+def test_ncu_summary_picks_the_newest_profile_round():
+    """The roofline's `traffic` comes from the newest committed ncu summary: profile directories are ordered by
+    round, then suffix length, then suffix (r02z < r02aa), not by name."""
+    import importlib.util
+    import re
+    spec = importlib.util.spec_from_file_location("bench_mod", os.path.join(ROOT, "bench.py"))
+    mod = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(mod)
+    d, src = mod._ncu_summary("k_subtree", "C4")
+    assert d is not None and src is not None
+    have = [x for x in os.listdir(os.path.join(ROOT, "profiles"))
+            if os.path.exists(os.path.join(ROOT, "profiles", x, "full_k_subtree.json"))]
+
+    def key(x):
+        m = re.match(r"r(\d+)([a-z]*)$", x)
+        return (int(m.group(1)), len(m.group(2)), m.group(2))
+    assert src.split(os.sep)[1] == max(have, key=key)
