@@ -30,6 +30,8 @@
 // order, tile size or number of GPUs.
 #include <cuda/atomic>
 
+#include <mutex>
+
 #include <algorithm>
 #include <cstdio>
 #include <ctime>
@@ -2965,6 +2967,22 @@ void d2h(T* h, const T* d, size_t cnt, cudaStream_t s) {
   BF_CUDA_CHECK(cudaMemcpyAsync(h, d, cnt * sizeof(T), cudaMemcpyDeviceToHost, s));
 }
 
+// The node-list work space (E0, E1, Es: the three largest buffers of a fit, GBs each) is kept across bf_fit calls
+// and reused when large enough, so consecutive fits of one shape make no allocator calls for it (with torch's
+// caching allocator a fragmented cache otherwise sometimes releases and re-allocates them: +0.6 s on a C4 step).
+// One fit at a time owns it (a concurrent fit on another thread allocates its own); it is never freed at exit.
+// BF_LIST_WORKSPACE=0 allocates per fit.
+struct ListWorkspace {
+  std::mutex mu;
+  uint64_t* buf[3] = {nullptr, nullptr, nullptr};
+  size_t cap = 0;  // entries per buffer
+  int device = -1;
+};
+ListWorkspace& list_ws() {
+  static ListWorkspace* w = new ListWorkspace();
+  return *w;
+}
+
 struct PinnedSummary {
   LevelSummary* h = nullptr;
   PinnedSummary() { BF_CUDA_CHECK(cudaMallocHost(&h, sizeof(LevelSummary) * 2)); }
@@ -3178,6 +3196,11 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
     // free memory as the allocator in use sees it: the driver's, or the caller's hint (bf_set_memory_budget:
     // the torch caching allocator's cached-but-unused blocks count as free)
     if (memory_budget() > 0) fr = (size_t)memory_budget();
+    {  // a held list work space is this fit's memory too
+      int dv_ = 0;
+      cudaGetDevice(&dv_);
+      if (list_ws().device == dv_) fr += list_ws().cap * 3 * sizeof(uint64_t);
+    }
     const size_t budget = fr / 2;
     B = (int)std::max<size_t>(1, std::min<size_t>(budget / std::max<size_t>(per_tree, 1), 256));
     // Large trees: the split-scan and partition CTAs are bound to trees (148 / B CTAs per tree), so a level
@@ -3281,7 +3304,11 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_ts, scan_kern, SNT, tscan_smem);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_tp, k_partition_tree, TPNT, tpart_smem);
     const unsigned grid_tscan = (unsigned)std::max(1, occ_ts * nsm), grid_tpart = (unsigned)std::max(1, occ_tp * nsm);
-    DBuf<uint64_t> E0, E1, Es;
+    DBuf<uint64_t> E0, E1, Es;  // per-fit list buffers (when the shared work space is not used)
+    uint64_t *pE0 = nullptr, *pE1 = nullptr, *pEs = nullptr;
+    static const bool ws_on = !(getenv("BF_LIST_WORKSPACE") && getenv("BF_LIST_WORKSPACE")[0] == '0');
+    std::unique_lock<std::mutex> wsl(list_ws().mu, std::defer_lock);
+    const bool use_ws = ws_on && wsl.try_lock() && (list_ws().device < 0 || list_ws().device == dev_id);
     std::vector<int32_t> h_sa;  // distinct rows of the batch's small roots (subtree packing)
     size_t E_cap = 0;
 
@@ -3331,10 +3358,31 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
       need = std::max<size_t>(need, 1);
       if (need > E_cap) {  // 3% headroom: later batches (sum of in-bag rows varies by ~0.1%) reuse the buffers
         const size_t cap = need + need / 32 + 16;
-        E0.alloc(cap, s);
-        E1.alloc(cap, s);
-        Es.alloc(cap, s);
-        E_cap = cap - 16;
+        if (use_ws) {
+          ListWorkspace& w = list_ws();
+          if (w.cap < cap) {
+            for (auto& b : w.buf) {
+              dev_free(b, s);
+              b = nullptr;
+            }
+            w.cap = 0;
+            for (auto& b : w.buf) b = (uint64_t*)dev_alloc(cap * sizeof(uint64_t), s);
+            w.cap = cap;
+            w.device = dev_id;
+          }
+          pE0 = w.buf[0];
+          pE1 = w.buf[1];
+          pEs = w.buf[2];
+          E_cap = w.cap - 16;
+        } else {
+          E0.alloc(cap, s);
+          E1.alloc(cap, s);
+          Es.alloc(cap, s);
+          pE0 = E0.p;
+          pE1 = E1.p;
+          pEs = Es.p;
+          E_cap = cap - 16;
+        }
       }
       h2d(kind_d.p, hk.data(), Bc, s);
       h2d(lidx_d.p, hl.data(), Bc, s);
@@ -3367,8 +3415,8 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
         }
         {
           KScope ks_("k_list_scatter", s, 0.0);
-          k_list_scatter<<<grid, NT, 0, s>>>(srt.p, n, wpk.p, Bp, kind_d.p, base_d.p, a_root.p, nchunk, Bc, cnt.p, E0.p,
-                                            Es.p);
+          k_list_scatter<<<grid, NT, 0, s>>>(srt.p, n, wpk.p, Bp, kind_d.p, base_d.p, a_root.p, nchunk, Bc, cnt.p, pE0,
+                                            pEs);
         }
         BF_CUDA_CHECK(cudaGetLastError());
         // presort chunk read once per tree group + one 32 B weight gather per (entry, group) + written entries
@@ -3384,8 +3432,8 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
       // ---- global phase
       int N = nL;
       int64_t cur_elems = offL;  // sum of p*a over the level's nodes
-      uint64_t* Ec = E0.p;
-      uint64_t* En = E1.p;
+      uint64_t* Ec = pE0;
+      uint64_t* En = pE1;
       LNode* nc = ncur.p;
       LNode* nx = nnext.p;
       while (N > 0) {
@@ -3450,7 +3498,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
           k_part_items_map<<<(unsigned)ceil_div(N, 256), 256, 0, s>>>(N, p, nc, icnt.p, ioff.p, imap.p);
         }
         {
-          TPartArgs ga{nc, split.p, child.p, p, Bc, Ec, sideb.p, nw, bm_smem ? 1 : 0, En, Es.p, tlo.p, thi.p, ioff.p, imap.p,
+          TPartArgs ga{nc, split.p, child.p, p, Bc, Ec, sideb.p, nw, bm_smem ? 1 : 0, En, pEs, tlo.p, thi.p, ioff.p, imap.p,
                        act.p, nact.p};
           KScope ks_("k_partition_tree", s, 0.0);
           k_partition_tree<<<grid_tpart, TPNT, tpart_smem, s>>>(ga);
@@ -3544,7 +3592,7 @@ void fit_impl(const double* X_in, int64_t ldx, const double* y_in, int64_t n, in
           ga.sq = sq.p;
           ga.gperm = d_perm.p;
           ga.gstart = d_gst.p;
-          ga.Es = Es.p;
+          ga.Es = pEs;
           ga.yq = yq.p;
           ga.y = y;
           ga.X = X;
