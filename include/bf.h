@@ -140,6 +140,11 @@ int bf_set_allocator(bf_alloc_fn alloc, bf_free_fn free_, void* ctx);
  * torch caching allocator's cached-but-unused blocks before every fit.
  * BF_EINVAL for a negative value.                                          */
 int bf_set_memory_budget(int64_t bytes);
+/* Release the node-list work space bf_fit keeps across calls (the three list
+ * buffers of the largest fit so far, reused by the next fits of that size;
+ * BF_LIST_WORKSPACE=0 makes bf_fit allocate them per call instead).  Waits for
+ * the device first.  BF_OK, or BF_EINVAL while a fit is using it.           */
+int bf_release_workspace(void);
 
 /* Grow global trees [tree_begin, tree_end) of a T-tree forest (P:95 steps 1-2;
  * S2-S4).  X: n x p column-major (ldx >= n), y: n.  Synchronous.  *out

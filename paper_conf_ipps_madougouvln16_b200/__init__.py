@@ -99,6 +99,7 @@ def lib():
             "bf_unique_u64": ([vp, i64, vp, vp, vp], C.c_int),
             "bf_set_allocator": ([vp, vp, vp], C.c_int),
             "bf_set_memory_budget": ([i64], C.c_int),
+            "bf_release_workspace": ([], C.c_int),
             "bf_profile_enable": ([C.c_int], C.c_int),
             "bf_profile_read": ([vp, C.c_int, C.POINTER(C.c_int)], C.c_int),
             "bf_launch_count": ([], C.c_int64),
@@ -137,6 +138,7 @@ def _install_torch_allocator(L):
 
 
 def torch_allocator_active() -> bool:
+    lib()  # the hooks are installed when the library is loaded
     return _TORCH_ALLOC is not None
 
 
@@ -151,7 +153,7 @@ def _memory_budget_hint():
 
 
 def exported_symbols():
-    return [n for n in ("bf_version", "bf_last_error", "bf_set_allocator", "bf_set_memory_budget", "bf_fit", "bf_forest_free",
+    return [n for n in ("bf_version", "bf_last_error", "bf_set_allocator", "bf_set_memory_budget", "bf_release_workspace", "bf_fit", "bf_forest_free",
                         "bf_forest_info_get", "bf_forest_export", "bf_forest_import", "bf_predict",
                         "bf_oob_importance", "bf_importance_finalize", "bf_pca", "bf_pca_retained", "bf_philox", "bf_i128_to_double",
                         "bf_fixed_point", "bf_bootstrap", "bf_perm", "bf_sort_u64", "bf_scan_u32", "bf_unique_u64", "bf_profile_enable", "bf_profile_read",
@@ -176,6 +178,11 @@ def profile_read() -> dict:
     lib().bf_profile_read(buf, len(buf), C.byref(cnt))
     return {buf[i].name.decode(): dict(ms=buf[i].ms, launches=int(buf[i].launches), bytes=buf[i].bytes)
             for i in range(min(cnt.value, len(buf)))}
+
+
+def release_workspace() -> None:
+    """Release the node-list work space bf_fit keeps across calls (bf_release_workspace)."""
+    _check(lib().bf_release_workspace(), "bf_release_workspace")
 
 
 def launch_count() -> int:

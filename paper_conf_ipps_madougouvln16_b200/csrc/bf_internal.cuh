@@ -261,6 +261,7 @@ const uint64_t* radix_sort_u64(uint64_t* k0, uint64_t* k1, uint32_t* v0, uint32_
 void unique_u64(const uint64_t* sorted, int64_t n, uint64_t* out, int32_t* count_dev, cudaStream_t s);
 
 // fit.cu
+bool release_list_workspace();  // false while a fit holds it
 void fit_impl(const double* X, int64_t ldx, const double* y, int64_t n, int32_t p, const bf_params& prm,
               cudaStream_t s, bf_forest** out);
 void fixed_point_impl(const double* y, int64_t n, int64_t sampsize, int64_t* yq, int32_t* q, cudaStream_t s);

@@ -189,6 +189,12 @@ int bf_set_memory_budget(int64_t bytes) {
   return BF_OK;
 }
 
+int bf_release_workspace(void) {
+  BF_API_BEGIN
+  BF_REQUIRE(bf::release_list_workspace(), BF_EINVAL, "bf_release_workspace: a fit is using the work space");
+  BF_API_END
+}
+
 int bf_fit(const double* X, int64_t ldx, const double* y, int64_t n, int32_t p, const bf_params* prm, void* stream,
            bf_forest** out) {
   BF_API_BEGIN

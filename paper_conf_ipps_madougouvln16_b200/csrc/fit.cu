@@ -2983,6 +2983,26 @@ ListWorkspace& list_ws() {
   return *w;
 }
 
+}  // namespace
+
+bool release_list_workspace() {
+  ListWorkspace& w = list_ws();
+  std::unique_lock<std::mutex> lk(w.mu, std::try_to_lock);
+  if (!lk.owns_lock()) return false;
+  if (w.cap) {
+    cudaDeviceSynchronize();
+    for (auto& b : w.buf) {
+      dev_free(b, nullptr);
+      b = nullptr;
+    }
+    w.cap = 0;
+    w.device = -1;
+  }
+  return true;
+}
+
+namespace {
+
 struct PinnedSummary {
   LevelSummary* h = nullptr;
   PinnedSummary() { BF_CUDA_CHECK(cudaMallocHost(&h, sizeof(LevelSummary) * 2)); }
